@@ -1,0 +1,183 @@
+"""Pins of the oracle's CG and FEM operator (c8)
+against the analytic manufactured solution, a discrete eigenvector, a dense
+direct solve, analytic element-stiffness entries, rigid-body modes, the
+patch test and the strain-energy closed form."""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+from test_oracle_maps_stencil import dense_laplacian
+
+
+# ---- CG on A = -L ------------------------------------
+@pytest.mark.parametrize("n,max_it", [(16, 60), (24, 90)])
+def test_cg_manufactured_solution_converges_to_analytic(n, max_it):
+    b = synth.poisson_poly_rhs((n, n, n))
+    ustar = synth.poisson_poly_solution(n)
+    # u* is exactly the discrete solution: A u* = b (operator exact on quadratics)
+    assert np.max(np.abs(-oracle.laplace7(ustar) - b)) < 16 * 2.3e-16 * np.max(np.abs(ustar))
+    x, res, hist = oracle.cg(b, max_iter=max_it, rtol=1e-12)
+    assert res.converged == 1
+    assert res.iters < 3.2 * n
+    assert np.max(np.abs(x - ustar)) < 5e-14
+
+
+def test_cg_single_eigenvector_one_iteration():
+    n = 12
+    s = np.sin(np.pi * np.arange(1, n + 1) / (n + 1))
+    u = s[:, None, None] * s[None, :, None] * s[None, None, :]
+    lam = 3 * (2 - 2 * np.cos(np.pi / (n + 1)))
+    x, res, _ = oracle.cg(lam * u, max_iter=5, rtol=1e-13)
+    assert res.iters == 1
+    assert np.max(np.abs(x - u)) < 1e-14
+
+
+def test_cg_dense_direct_solve_8cubed():
+    shape = (8, 8, 8)
+    A = -dense_laplacian(shape)
+    b = synth.uniform(shape, seed=2)
+    xd = np.linalg.solve(A, b.ravel())
+    x, res, hist = oracle.cg(b, max_iter=60, rtol=0.0)
+    assert np.max(np.abs(x.ravel() - xd)) < 1e-13
+    # recursive residual tracks the true residual
+    rtrue = b.ravel() - A @ x.ravel()
+    assert abs(np.dot(rtrue, rtrue) - hist[-1]) < 1e-20 + 1e-6 * hist[-1]
+
+
+def test_cg_residual_history_monotone_in_energy_norm():
+    shape = (10, 9, 8)
+    A = -dense_laplacian(shape)
+    b = synth.uniform(shape[::-1], seed=3)
+    xd = np.linalg.solve(A, b.ravel())
+    errs = []
+    for k in range(1, 16, 2):
+        x, res, _ = oracle.cg(b, max_iter=k)
+        e = x.ravel() - xd
+        errs.append(e @ A @ e)
+    assert errs[-1] > 1e-24
+    assert all(a > b for a, b in zip(errs, errs[1:]))
+
+
+def test_cg_zero_rhs_is_zero_iterations():
+    x, res, _ = oracle.cg(np.zeros((4, 4, 4)), max_iter=5, rtol=1e-8)
+    assert res.iters == 0 and res.converged == 2 and np.all(x == 0)
+
+
+def test_sparse_cg_full_mask_reproduces_dense_bitwise():
+    b = synth.uniform((6, 7, 8), seed=4)
+    m = np.ones(b.shape, dtype=np.uint8)
+    x1, r1, h1 = oracle.cg(b, max_iter=20)
+    x2, r2, h2 = oracle.cg(b, max_iter=20, op=oracle.OP_SPARSE7, mask=m)
+    assert np.array_equal(x1, x2) and np.array_equal(h1, h2)
+
+
+def test_sparse_cg_vs_direct_on_sphere():
+    n = 8
+    m = synth.sphere_mask(n, 0.45)
+    act = m.ravel().astype(bool)
+    A = -dense_laplacian((n, n, n))[np.ix_(act, act)]
+    b = np.where(m, synth.uniform((n, n, n), seed=5), 0.0)
+    x, res, _ = oracle.cg(b, max_iter=80, op=oracle.OP_SPARSE7, mask=m, rtol=1e-14)
+    xd = np.linalg.solve(A, b.ravel()[act])
+    assert np.max(np.abs(x.ravel()[act] - xd)) < 1e-12
+    assert np.all(x.ravel()[~act] == 0.0)
+
+
+# ---- FEM -------------------------
+E, NU = 1.0, 0.3
+LAM = E * NU / ((1 + NU) * (1 - 2 * NU))
+MU = E / (2 * (1 + NU))
+
+
+def test_ke_analytic_entries():
+    ke = oracle.fem_ke(E, NU)
+    # K[0,0] = (lam + 4 mu) * int (dN0/dx)^2 = (lam + 4 mu)/9  (= 0.235043)
+    assert abs(ke[0, 0] - (LAM + 4 * MU) / 9) < 1e-15
+    assert abs(ke[0, 0] - 0.2350427350427350) < 1e-15
+    # K[0,1] (node 0 x-dof, node 0 y-dof) = (lam + mu) * int dN0/dx dN0/dy = (lam+mu)/12
+    assert abs(ke[0, 1] - (LAM + MU) / 12) < 1e-15
+    # node 0 x-dof vs node 1 (the +x neighbour) x-dof: (lam+2mu) int dN0x dN1x + mu (int dN0y dN1y + dN0z dN1z)
+    #   int dN0x dN1x = -1/9 ; int dN0y dN1y = int (1-x)x (1-z)^2 = 1/6 * 1/3 ... = 1/18 each
+    assert abs(ke[0, 3] - (-(LAM + 2 * MU) / 9 + MU * (1 / 18 + 1 / 18))) < 1e-15
+
+
+def test_ke_symmetric_with_six_rigid_modes():
+    ke = oracle.fem_ke(E, NU)
+    assert np.max(np.abs(ke - ke.T)) < 1e-16
+    ev = np.linalg.eigvalsh(ke)
+    assert np.all(np.abs(ev[:6]) < 1e-14) and ev[6] > 1e-2
+    # explicit rigid modes: 3 translations + 3 rotations about the centre
+    pts = np.array([[a & 1, (a >> 1) & 1, (a >> 2) & 1] for a in range(8)], dtype=float) - 0.5
+    modes = []
+    for d in range(3):
+        m = np.zeros((8, 3)); m[:, d] = 1; modes.append(m.ravel())
+    for axis in np.eye(3):
+        modes.append(np.cross(axis, pts).ravel())
+    for m in modes:
+        assert np.max(np.abs(ke @ m)) < 1e-15
+
+
+def test_ke_uniform_strain_energy_closed_form():
+    """u = G x on one element: u^T K_e u = eps^T D eps (unit volume)."""
+    ke = oracle.fem_ke(E, NU)
+    rng = np.random.default_rng(1)
+    G = rng.standard_normal((3, 3))
+    pts = np.array([[a & 1, (a >> 1) & 1, (a >> 2) & 1] for a in range(8)], dtype=float)
+    u = (pts @ G.T).ravel()
+    eps = np.array([G[0, 0], G[1, 1], G[2, 2], G[0, 1] + G[1, 0], G[1, 2] + G[2, 1], G[2, 0] + G[0, 2]])
+    D = np.zeros((6, 6)); D[:3, :3] = LAM; D[np.arange(3), np.arange(3)] += 2 * MU
+    D[np.arange(3, 6), np.arange(3, 6)] = MU
+    assert abs(u @ ke @ u - eps @ D @ eps) < 1e-13
+
+
+def test_fem_patch_test_and_rigid_motion_on_grid():
+    n = 5
+    Z, Y, X = np.meshgrid(np.arange(n), np.arange(n), np.arange(n), indexing="ij")
+    G = np.array([[0.3, -0.2, 0.1], [0.05, 0.4, -0.3], [0.2, 0.1, -0.1]])
+    u = np.stack([G[i, 0] * X + G[i, 1] * Y + G[i, 2] * Z for i in range(3)]).astype(float)
+    y = oracle.fem_apply(u, E, NU, dirichlet_z0=False)
+    inner = (slice(None), slice(1, -1), slice(1, -1), slice(1, -1))
+    assert np.max(np.abs(y[inner])) < 1e-14         # linear field: no interior force
+    assert np.max(np.abs(y.reshape(3, -1).sum(1))) < 1e-13  # equilibrium
+    # rigid rotation about z: u = (-y, x, 0) -> K u = 0 everywhere
+    rot = np.stack([-Y, X, 0 * X]).astype(float)
+    assert np.max(np.abs(oracle.fem_apply(rot, E, NU, dirichlet_z0=False))) < 1e-13
+
+
+def test_fem_brute_force_assembled_matrix():
+    """Dense K assembled here from K_e (independent loop) vs matrix-free apply."""
+    n = 4
+    ke = oracle.fem_ke(E, NU)
+    N = n ** 3
+    K = np.zeros((3 * N, 3 * N))
+    for ez in range(n - 1):
+        for ey in range(n - 1):
+            for ex in range(n - 1):
+                dofs = []
+                for a in range(8):
+                    i, j, k = ex + (a & 1), ey + ((a >> 1) & 1), ez + ((a >> 2) & 1)
+                    node = i + n * (j + n * k)
+                    dofs += [d * N + node for d in range(3)]
+                K[np.ix_(dofs, dofs)] += ke
+    fixed = np.zeros(3 * N, dtype=bool)
+    for d in range(3):
+        fixed[d * N: d * N + n * n] = True  # z = 0 plane
+    Kd = K.copy()
+    Kd[fixed, :] = 0; Kd[:, fixed] = 0; Kd[fixed, fixed] = 1
+    u = synth.uniform((n, n, n), card=3, seed=9)
+    y = oracle.fem_apply(u, E, NU, dirichlet_z0=True)
+    assert np.max(np.abs(y.ravel() - Kd @ u.ravel())) < 1e-14
+    # 27-point structure: an interior node couples to exactly 27 nodes
+    mid = 1 + n * (1 + n * 1)
+    cols = np.nonzero(np.abs(K[mid]) > 1e-15)[0] % N
+    assert len(set(cols.tolist())) == 27
+    # RHS: total load = p * area of the top face
+    b = oracle.fem_rhs((n, n, n), 1.0)
+    assert abs(b[2].sum() - (n - 1) ** 2) < 1e-14 and np.all(b[:2] == 0)
+    # FEM CG solves K u = b
+    x, res, _ = oracle.cg(b, max_iter=400, rtol=1e-13, op=oracle.OP_FEM27)
+    assert res.converged == 1
+    assert np.max(np.abs(Kd @ x.ravel() - b.ravel())) < 1e-11
+    assert np.allclose(x.ravel(), np.linalg.solve(Kd, b.ravel()), atol=1e-10)
