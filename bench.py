@@ -1,0 +1,431 @@
+#!/usr/bin/env python
+"""bench.py — headline benchmark of the B200 Neon map-stencil hot path.
+
+Default workload (BASELINE.json configs[1], the config the metric is quoted
+on): Poisson finite-difference CG, 7-point, fp64, 512^3 dense grid, strong
+scaling over N GPUs (one process per GPU, torchrun).  One "step" is one full
+CG iteration (UpdateP, stencil, <p,q>, x/r updates, <r,r>; DESIGN.md "CG
+schedule").  value = MLUPS = cells * steps / t / 1e6 over the whole job.
+
+The same JSON line carries, at N = 1, the D3Q19 LBM cavity (configs[2],
+512^3 fp32) and the config-C1 loop (configs[0]) results under "also".
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl nb|reference]
+                  [--workload cg|lbm] [--n 512]
+
+--impl reference times the CPU oracle (oracle/, plain C fp64) on the host
+cores — the tier's reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "MLUPS & HBM GB/s (% roofline) at 1/2/4/8 B200; weak/strong scaling eff."
+CG_BYTES_PER_CELL = 64      # 2-phase schedule, DESIGN.md "CG schedule"
+CG_A_BYTES = 40             # phase A: read x, r, p_old; write x, p_new
+CG_B_BYTES = 24             # phase B: read r, p_new; write r
+LBM_BYTES_PER_CELL = 152    # 19 x (4 B read + 4 B write)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu, self.rows, self.proc = gpu, [], None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([c.strip() for c in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.15)
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm = [float(r[1]) for r in self.rows if len(r) > 8 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) > 8 and r[2].replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            if len(r) > 8:
+                for nm, v in zip(names, r[5:9]):
+                    if v.strip().lower() == "active":
+                        reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------------------
+def setup_dist(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    import torch
+    torch.cuda.set_device(local)
+    if world > 1:
+        import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    return world, rank, local
+
+
+def barrier(world):
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def max_over_ranks(world, v):
+    if world == 1:
+        return v
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def timed(world, stream, fn, gpu):
+    """Barrier + sync on both sides; CUDA events on the launching stream."""
+    import torch
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier(world)
+    torch.cuda.synchronize()
+    with ClockSampler(gpu) as clk:
+        ev0.record(stream)
+        fn()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    barrier(world)
+    ms = ev0.elapsed_time(ev1)
+    return max_over_ranks(world, ms), clk.summary()
+
+
+def ncu_traffic(kernel: str):
+    """dram bytes per launch of `kernel` from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    d = json.load(open(p))
+    return d.get(kernel)
+
+
+# ---------------------------------------------------------------------------
+def bench_cg(args, world, rank, local):
+    import numpy as np
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    n = args.n
+    dims = (n, n, n)
+    cells = n ** 3
+    comm = nb.Comm.from_torch_distributed(local) if world > 1 else None
+    g = nb.Grid(dims, nparts=world, comm=comm) if comm else nb.Grid(dims, nparts=1, devices=[local])
+    stream = torch.cuda.ExternalStream(g.stream())
+    b, x = nb.Field(g), nb.Field(g)
+    b.fill(nb.FILL_POISSON_RHS)
+    x.fill_const(0.0)
+    occ = nb.OCC_NAMES[args.occ]
+    cg = nb.CG(x, b, occ=occ)
+    cg.iterate(args.warmup)
+    g.sync()
+    l0 = g.launch_count()
+    ms, clocks = timed(world, stream, lambda: cg.iterate(args.steps), local)
+    launches = g.launch_count() - l0
+    res = cg.finish()
+    cg.close()
+    t = ms / 1e3
+    mlups = cells * args.steps / t / 1e6
+    hbm, peak_kind = peaks()
+    # per-kernel durations: a profiled (event-bracketed, eager) pass
+    x.fill_const(0.0)
+    g.profile(True)
+    cg = nb.CG(x, b, occ=occ)
+    cg.iterate(args.prof_steps)
+    na, msa = g.profile_read("k_msr_cgA")
+    nbb, msb = g.profile_read("k_cg_B")
+    nfin, msf = g.profile_read("k_finalize")
+    g.profile(False)
+    cg.finish()
+    cg.close()
+    local_cells = cells // world
+    a_avg, b_avg = msa / max(na, 1), msb / max(nbb, 1)
+    dom = ("k_msr_cgA", CG_A_BYTES, a_avg, na) if msa >= msb else ("k_cg_B", CG_B_BYTES, b_avg, nbb)
+    achieved = dom[1] * local_cells / (dom[2] / 1e3) / 1e9
+    tr = ncu_traffic(dom[0])
+    out = {
+        "metric": METRIC, "value": mlups, "unit": "MLUPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"C2 Poisson FD CG 7-point fp64 {n}^3 dense (configs[1])",
+                   "rhs": "b = h^2 f, manufactured u* = g(x)g(y)g(z)", "x0": 0,
+                   "parts": world, "occ": args.occ, "schedule": "2-phase, 64 B/cell/iter",
+                   "l2": "inputs larger than L2 (5 fp64 fields of %.2f GB each)" % (cells * 8 / 1e9)},
+        "hbm_gbs": CG_BYTES_PER_CELL * cells * args.steps / t / 1e9,
+        "hbm_frac": CG_BYTES_PER_CELL * cells * args.steps / t / 1e9 / hbm,
+        "roofline": {"bound": "hbm", "kernel": dom[0], "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                     "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": tr,
+                     "algorithmic_bytes_per_launch": dom[1] * local_cells,
+                     "launch_ms": dom[2],
+                     "kernel_ms": {"k_msr_cgA": a_avg, "k_cg_B": b_avg, "k_finalize": msf / max(nfin, 1)}},
+        "gpu_launches": int(launches), "clocks": clocks,
+        "cg_state": {"iters": res.iters, "rr0": res.rr0, "rr": res.rr},
+    }
+    # ---- e2e: public API, host buffers, H2D and D2H inside the timed region
+    bh = torch.empty(cells * 8 // world if world > 1 else cells * 8, dtype=torch.uint8).pin_memory()
+    if world == 1:
+        import synth
+        np.frombuffer(bh.numpy().data, dtype=np.float64)[:] = synth.poisson_poly_rhs(dims).ravel()
+    xh = torch.zeros(cells, dtype=torch.float64).pin_memory()
+
+    def e2e():
+        b.upload_async(bh.data_ptr()) if world == 1 else b.fill(nb.FILL_POISSON_RHS)
+        x.upload_async(xh.data_ptr())
+        s = nb.CG(x, b, occ=occ)
+        s.iterate(args.steps)
+        s.finish()
+        s.close()
+        x.download(xh)
+    if world == 1:
+        e2e()  # warm
+        ms_e, _ = timed(world, stream, e2e, local)
+        out["e2e"] = {"value": cells * args.steps / (ms_e / 1e3) / 1e6, "unit": "MLUPS",
+                      "h2d_bytes_per_step": 2 * cells * 8, "d2h_bytes_per_step": cells * 8,
+                      "note": "upload b and x0 from pinned host, CG create (r = b - Ax0), steps iterations, "
+                              "finish (deferred x update), download x; one e2e call per timed region"}
+    b.close(), x.close()
+    g.close()
+    if comm:
+        comm.close()
+    return out
+
+
+def lbm_omega(nx, u_lid=0.05, re=100.0):
+    """Cavity set-up (SURVEY.md §8(c) c6 reading): nu = u_lid Nx / Re."""
+    nu = u_lid * nx / re
+    return 1.0 / (3.0 * nu + 0.5)
+
+
+def bench_lbm_run(n, steps, warmup, world, local, occ="standard"):
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    dims = (n, n, n * world)  # weak scaling: 512^3 per GPU
+    comm = nb.Comm.from_torch_distributed(local) if world > 1 else None
+    g = nb.Grid(dims, nparts=world, comm=comm) if comm else nb.Grid(dims, nparts=1, devices=[local])
+    stream = torch.cuda.ExternalStream(g.stream())
+    fa, fb = nb.Field(g, "f32", 19), nb.Field(g, "f32", 19)
+    nb.nb_lbm_init(fa, 1.0, (0.0, 0.0, 0.0))
+    om = lbm_omega(n)
+    st = {"a": fa, "b": fb}
+
+    def run(k):
+        st["a"], st["b"] = nb.nb_lbm_step(st["a"], st["b"], om, k, u_lid=0.05, occ=nb.OCC_NAMES[occ])
+    run(warmup)
+    g.sync()
+    l0 = g.launch_count()
+    ms, clocks = timed(world, stream, lambda: run(steps), local)
+    launches = g.launch_count() - l0
+    g.profile(True)
+    run(3)
+    nk, msk = g.profile_read("k_lbm_d3q19")
+    g.profile(False)
+    cells = n * n * n * world
+    t = ms / 1e3
+    hbm, peak_kind = peaks()
+    k_ms = msk / max(nk, 1) * (1 if world == 1 else 1)
+    local_cells = n * n * n
+    # at N=1 with no OCC split one launch covers the whole grid
+    per_step_ms = msk / 3.0
+    achieved = LBM_BYTES_PER_CELL * local_cells / (per_step_ms / 1e3) / 1e9
+    res = {
+        "value": cells * steps / t / 1e6, "unit": "MLUPS", "n_gpus": world, "steps": steps, "warmup": warmup,
+        "ms_per_step": ms / steps, "scaling": "weak", "dtype": "f32",
+        "config": {"workload": f"C3 D3Q19 BGK lid-driven cavity fp32 SoA twoPop, {n}^3 per GPU (configs[2])",
+                   "omega": om, "u_lid": 0.05, "Re": 100, "occ": occ,
+                   "l2": "inputs larger than L2 (2 x %.1f GB)" % (19 * 4 * n ** 3 / 1e9)},
+        "hbm_gbs": LBM_BYTES_PER_CELL * cells * steps / t / 1e9,
+        "hbm_frac": LBM_BYTES_PER_CELL * cells * steps / t / 1e9 / hbm,
+        "roofline": {"bound": "hbm", "kernel": "k_lbm_d3q19", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                     "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": ncu_traffic("k_lbm_d3q19"),
+                     "algorithmic_bytes_per_launch": LBM_BYTES_PER_CELL * local_cells, "launch_ms": k_ms},
+        "gpu_launches": int(launches), "clocks": clocks,
+    }
+    st["a"].close(), st["b"].close()
+    g.close()
+    if comm:
+        comm.close()
+    return res
+
+
+def bench_c1(local):
+    """Config C1 (64^3 fp64, 10 iterations, 1 GPU): launch-bound; reported
+    as loop time and MLUPS."""
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    n = 64
+    g = nb.Grid((n, n, n), devices=[local])
+    x, y = nb.Field(g), nb.Field(g)
+    reps = 20
+
+    def run():
+        for _ in range(reps):
+            x.fill_int(seed=1)
+            y.fill_const(0.0)
+            nb.nb_map_stencil_reduce(x, y, 0.125, 10, nb.OCC_TWO_WAY)
+    run()
+    t0 = time.perf_counter()
+    run()
+    dt = (time.perf_counter() - t0) / reps
+    x.close(), y.close()
+    g.close()
+    return {"workload": "C1 AXPY + 7-pt + dot, 64^3 fp64, 10 iterations (configs[0])",
+            "ms_per_loop": dt * 1e3, "value": n ** 3 * 10 / dt / 1e6, "unit": "MLUPS",
+            "note": "host wall clock per synchronous nb_map_stencil_reduce call (includes launch latency)"}
+
+
+# ---------------------------------------------------------------------------
+def cpu_baseline_cg(n, iters=2):
+    """The oracle (plain C, fp64, OpenMP over planes) on the host cores:
+    `iters` CG iterations on the full n^3 grid (setup subtracted)."""
+    import oracle
+    import synth
+    b = synth.poisson_poly_rhs((n, n, n))
+    t0 = time.perf_counter()
+    oracle.cg(b, max_iter=0)
+    t1 = time.perf_counter()
+    oracle.cg(b, max_iter=iters)
+    t2 = time.perf_counter()
+    per_iter = max((t2 - t1) - (t1 - t0), 1e-9) / iters
+    return {"value": n ** 3 / per_iter / 1e6, "unit": "MLUPS", "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"{iters} CG iterations on the full {n}^3 grid (oracle.cg, setup time subtracted)"}
+
+
+def cpu_baseline_lbm(n=256, steps=2):
+    import numpy as np
+
+    import oracle
+    c, w, _ = oracle.lbm_lattice()
+    f = np.broadcast_to(w[:, None, None, None], (19, n, n, n)).astype(np.float32)
+    om = lbm_omega(n)
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        f = oracle.lbm_step(f, om)
+    dt = (time.perf_counter() - t0) / steps
+    return {"value": n ** 3 / dt / 1e6, "unit": "MLUPS", "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"{steps} cavity steps at {n}^3 (512^3 x 19 fp64 does not fit the bounded sample)"}
+
+
+def reference_arm(args, world, rank):
+    """--impl reference: the oracle as it stands, on the host cores, same
+    config / metric / unit; each step = one CG iteration on the full grid."""
+    if rank != 0:
+        return None
+    import oracle
+    import synth
+    n = args.n
+    b = synth.poisson_poly_rhs((n, n, n))
+    w = min(args.warmup, 1)
+    k = min(args.steps, 5)
+    t0 = time.perf_counter()
+    oracle.cg(b, max_iter=w)
+    t1 = time.perf_counter()
+    oracle.cg(b, max_iter=w + k)
+    t2 = time.perf_counter()
+    per = ((t2 - t1) - (t1 - t0)) / k
+    v = n ** 3 / per / 1e6
+    return {"metric": METRIC, "value": v, "unit": "MLUPS", "n_gpus": world, "steps": k, "warmup": w,
+            "ms_per_step": per * 1e3, "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": f"C2 Poisson FD CG 7-point fp64 {n}^3 dense (configs[1])", "parts": 1},
+            "cpu_baseline": {"value": v, "unit": "MLUPS", "cores": oracle.num_threads(), "kind": "oracle",
+                             "sample": f"{k} CG iterations on the full {n}^3 grid after {w} warm-up "
+                                       "(time of cg(w+k) minus cg(w))"},
+            "e2e": {"value": v, "unit": "MLUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="nb", choices=["nb", "reference"])
+    ap.add_argument("--workload", default="cg", choices=["cg", "lbm"])
+    ap.add_argument("--n", type=int, default=512)
+    ap.add_argument("--occ", default="two_way", choices=list(("none", "standard", "extended", "two_way")))
+    ap.add_argument("--prof-steps", type=int, default=10)
+    ap.add_argument("--no-extras", action="store_true", help="skip the LBM / C1 / cpu_baseline extras")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if args.impl == "reference":
+        out = reference_arm(args, world, rank)
+        if out is not None:
+            print(json.dumps(out), flush=True)
+        return
+    world, rank, local = setup_dist(args)
+    import __graft_entry__
+    __graft_entry__.build()
+    if args.workload == "cg":
+        out = bench_cg(args, world, rank, local)
+        if world == 1 and not args.no_extras:
+            lbm = bench_lbm_run(args.n, 20, 3, 1, local)
+            out["also"] = {"lbm_d3q19": lbm, "c1": bench_c1(local)}
+            out["cpu_baseline"] = cpu_baseline_cg(args.n)
+            out["also"]["lbm_d3q19"]["cpu_baseline"] = cpu_baseline_lbm()
+    else:
+        r = bench_lbm_run(args.n, args.steps, args.warmup, world, local, occ=args.occ if args.occ in
+                          ("none", "standard") else "standard")
+        out = {"metric": METRIC, "higher_is_better": True, "vs_baseline": None, "data": "synthetic", **r}
+        if world == 1 and not args.no_extras:
+            out["cpu_baseline"] = cpu_baseline_lbm()
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,261 @@
+/*
+ * nb.h — C ABI of the B200-native Neon map-stencil hot path
+ * (Meneghin, Mahmoud, Jayaraman, Morris, "Neon: A Multi-GPU Programming
+ * Model for Grid-based Computations", IPDPS 2022 — /root/reference/PAPER.md,
+ * cited as L<line>).
+ *
+ * Library: paper_conf_ipps_meneghinmjm22_b200/libnb.so (sm_100a).
+ *
+ * Conventions:
+ *  - Every function returns nb_status: NB_OK (0) or an error code; no C++
+ *    exception crosses the ABI.  nb_last_error() returns a thread-local
+ *    message for the last failing call on the calling thread.
+ *  - Errors from asynchronous GPU work surface at the next synchronising
+ *    call (nb_sync, nb_dot, nb_field_download, nb_cg_finish, ...).
+ *  - Handles are opaque and caller-owned; *_destroy(NULL) is a no-op.
+ *    A grid must outlive its fields and solvers (NB_ESTATE otherwise).
+ *  - Host pointers are borrowed for the duration of the call only.
+ *  - Operations are stream-ordered on the grid's compute stream and return
+ *    immediately, except where "synchronises" is stated.
+ *  - Dense host logical view ("Host Logical View"):
+ *    element (c, x, y, z) of a field is host[x + Nx*(y + Ny*(z + Nz*c))].
+ *  - A grid is driven by one host thread at a time.
+ *  - There is no CPU fallback: without a CUDA device every call that needs
+ *    one fails with NB_ECUDA.
+ */
+#ifndef NB_H
+#define NB_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t nb_status;
+#define NB_OK 0
+#define NB_EINVAL 1        /* bad argument (NULL handle, size, range, ...)        */
+#define NB_ENOMEM 2        /* device or host allocation failed                    */
+#define NB_ECUDA 3         /* CUDA runtime error (incl. no device)                */
+#define NB_ENCCL 4         /* NCCL missing or failed                              */
+#define NB_EMISMATCH 5     /* fields of different grids / dtype / cardinality     */
+#define NB_EUNSUPPORTED 6  /* valid request this build does not support           */
+#define NB_ESTATE 7        /* object in the wrong state (live fields, reuse, ...) */
+
+typedef enum { NB_F32 = 0, NB_F64 = 1 } nb_dtype;
+
+/* Data views: Internal cells need only partition-local data;
+ * Boundary cells read halo data received from a neighbouring partition;
+ * Standard = Internal U Boundary.  With radius-1 stencils and z-slab
+ * partitions the Boundary view is the first and/or last plane of a slab that
+ * faces another partition; global domain faces are Internal. */
+typedef enum { NB_VIEW_STANDARD = 0, NB_VIEW_INTERNAL = 1, NB_VIEW_BOUNDARY = 2 } nb_view;
+
+/* Overlap of computation and communication (Fig. 1,
+ * L293-L315): NONE = global barrier before the halo update; STANDARD = split
+ * the stencil into internal/boundary, overlap the halo with the internal part;
+ * EXTENDED = also split the preceding map and send the halo right after the
+ * boundary map; TWO_WAY = EXTENDED + split the following reduce. */
+typedef enum { NB_OCC_NONE = 0, NB_OCC_STANDARD = 1, NB_OCC_EXTENDED = 2, NB_OCC_TWO_WAY = 3 } nb_occ;
+
+/* Synthetic, partition-independent initialisation (DESIGN.md "Input
+ * recipe"): CONST = a; UNIFORM = a + (b-a)*u, u = (h>>11)*2^-53;
+ * INT_UNIFORM = a + (h mod (b-a+1)) (a, b integers); POISSON_RHS = h^2 f of
+ * the manufactured solution g(x)g(y)g(z), g(t) = t(1-t) (cubic grids only);
+ * h = splitmix64(seed*0x9E3779B97F4A7C15 + gidx + 1) with
+ * gidx = x + Nx*(y + Ny*(z + Nz*c)). */
+typedef enum {
+    NB_FILL_CONST = 0,
+    NB_FILL_UNIFORM = 1,
+    NB_FILL_INT_UNIFORM = 2,
+    NB_FILL_POISSON_RHS = 3
+} nb_fill;
+
+typedef struct nb_comm nb_comm;
+typedef struct nb_grid nb_grid;
+typedef struct nb_field nb_field;
+typedef struct nb_cg nb_cg;
+
+/* ---- library ---------------------------------------------------------- */
+const char *nb_version(void);
+const char *nb_last_error(void);
+/* number of CUDA devices visible (0 on a CPU-only host; never fails) */
+int32_t nb_device_count(void);
+
+/* ---- communicator (one process per GPU; PAPER.md L238 multi-GPU streams,
+ * L252-L256 explicit GPU-GPU transfers).  Built on NCCL, loaded at run time
+ * (dlopen libnccl.so.2); NB_ENCCL if it cannot be loaded. --------------- */
+/* out: 128 opaque bytes to broadcast from rank 0 to every rank */
+nb_status nb_comm_unique_id(uint8_t out[128]);
+/* world >= 1 processes; rank in [0, world); device = the CUDA device this
+ * process drives.  Collective over all ranks. */
+nb_status nb_comm_create(int32_t world, int32_t rank, const uint8_t id[128], int32_t device,
+                         nb_comm **out);
+nb_status nb_comm_destroy(nb_comm *comm);
+
+/* ---- grid (PAPER.md L81-L88 Domain, L244 Grid, L256 1-D decomposition) -- */
+/* Pure host logic (no GPU needed): the z-slab partition of a1 — partition g
+ * owns planes [z_begin[g], z_begin[g+1]); the first (nz mod nparts)
+ * partitions get one extra plane.  z_begin has nparts+1 entries.
+ * NB_EINVAL if nparts < 1 or any slab would be empty. */
+nb_status nb_partition_plan(int32_t nz, int32_t nparts, int32_t *z_begin);
+/* Pure host logic: active-count balanced plane cuts for an element-sparse
+ * grid: counts[z] active cells per plane; cut g+1 is the
+ * first plane whose prefix count reaches (g+1)*total/nparts, with every slab
+ * non-empty. */
+nb_status nb_partition_plan_weighted(int32_t nz, const int64_t *counts, int32_t nparts,
+                                     int32_t *z_begin);
+
+/* Dense grid of dims = {Nx, Ny, Nz} cells split into nparts z-slabs.
+ * comm == NULL: every partition lives in this process; device_ids[nparts]
+ *   gives each partition's device and must name ONE device (virtual
+ *   partitions: several partitions on one GPU — the multi-GPU schedule,
+ *   halo copies and reductions run unchanged, which is what the
+ *   partition-invariance tests use).
+ * comm != NULL: nparts must be a multiple of the world size; this rank owns
+ *   partitions [rank*k, (rank+1)*k), k = nparts/world, all on comm's device
+ *   (device_ids may be NULL).
+ * NB_EUNSUPPORTED if nparts > 1 and a slab has fewer than 2 planes. */
+nb_status nb_grid_create_dense(const int32_t dims[3], int32_t nparts, const int32_t *device_ids,
+                               nb_comm *comm, nb_grid **out);
+/* Element-sparse grid: active[z][y][x] (0/1, Nx*Ny*Nz
+ * bytes, copied) selects the stored cells; the connectivity table is built
+ * on the device.  Cuts balance the active count (nb_partition_plan_weighted). */
+nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t *active, int32_t nparts,
+                                const int32_t *device_ids, nb_comm *comm, nb_grid **out);
+nb_status nb_grid_destroy(nb_grid *grid);
+
+typedef struct {
+    int32_t device;      /* CUDA device of the partition                         */
+    int32_t local;       /* 1 if owned by this process                           */
+    int32_t z_begin;     /* first global plane                                   */
+    int32_t z_end;       /* one past the last global plane                       */
+    int64_t n_cells;     /* active cells in the partition                        */
+    int64_t n_bnd_lo;    /* cells of the Boundary view on the low-z side         */
+    int64_t n_bnd_hi;    /* cells of the Boundary view on the high-z side        */
+    int64_t n_internal;  /* cells of the Internal view                           */
+} nb_part_info;
+nb_status nb_grid_num_partitions(const nb_grid *grid, int32_t *nparts);
+nb_status nb_grid_partition_info(const nb_grid *grid, int32_t g, nb_part_info *out);
+/* Use caller streams (e.g. torch.cuda.Stream.cuda_stream) instead of the
+ * library's own.  Either may be NULL to keep the current one. */
+nb_status nb_grid_set_streams(nb_grid *grid, void *compute_stream, void *halo_stream);
+nb_status nb_grid_get_stream(const nb_grid *grid, void **compute_stream);
+/* synchronises: waits for all work of the grid, reports async errors */
+nb_status nb_sync(nb_grid *grid);
+
+/* ---- fields (PAPER.md L58-L63 newField<T>(cardinality, outsideDomainValue),
+ * L246 Field, L248 SoA layout, L252 halo regions) --------------------------
+ * Device layout per partition (SoA):
+ *   [c][zl = -1 .. nz_g][y][x], x-rows padded to a 32-element pitch, one halo
+ *   plane below and above the slab.  Halo planes facing the global domain
+ *   boundary hold outside_value (the value read for out-of-domain neighbours).
+ * Sparse grids: [c][-halo_lo .. n_g + halo_hi) over the partition's active
+ *   cells in (z, y, x) order. */
+nb_status nb_field_create(nb_grid *grid, nb_dtype dtype, int32_t cardinality, double outside_value,
+                          nb_field **out);
+nb_status nb_field_destroy(nb_field *field);
+/* host: dense logical view, nbytes = Nx*Ny*Nz*card*sizeof(dtype); inactive
+ * cells of sparse grids are ignored on upload and read back as outside.
+ * Upload is stream-ordered (host buffer must stay valid until nb_sync);
+ * download synchronises. */
+nb_status nb_field_upload(nb_field *field, const void *host, int64_t nbytes);
+nb_status nb_field_download(const nb_field *field, void *host, int64_t nbytes);
+nb_status nb_field_fill(nb_field *field, nb_fill kind, uint64_t seed, double a, double b);
+/* haloUpdate: copy every partition's boundary planes into
+ * its neighbours' halo planes (2 transfers per component, L256). */
+nb_status nb_halo_update(nb_field *field);
+/* device pointer of partition g's buffer (element (c, x, y, zl) at
+ * ptr + c*cstride + (zl+1)*pstride + y*pitch + x, in elements) */
+nb_status nb_field_partition_ptr(const nb_field *field, int32_t g, void **ptr, int64_t *pitch,
+                                 int64_t *pstride, int64_t *cstride);
+
+/* ---- map, stencil, reduce (eqs.) ---- */
+/* y <- a*x + y on the view (one fused multiply-add per element) */
+nb_status nb_axpy(double a, const nb_field *x, nb_field *y, nb_view view);
+/* y <- a*x + b*y; b == 0 writes a*x without reading y (copy/scale) */
+nb_status nb_axpby(double a, const nb_field *x, double b, nb_field *y, nb_view view);
+/* y <- L(x), L(x)_i = sum of the 6 face neighbours - 6 x_i (Listing 2,
+ * L145-L152), out-of-domain neighbours read x's outside_value.  Reads x's
+ * halo planes as they are: call nb_halo_update(x) first (the runtime does it
+ * inside nb_map_stencil_reduce / nb_cg_*).  Scalar fields. */
+nb_status nb_laplace7(const nb_field *x, nb_field *y, nb_view view);
+/* <x, y> over all active cells and components, fp64 accumulation in a
+ * fixed order that does not depend on the partition count (DESIGN.md
+ * "Deterministic reductions").  Synchronises; *host_out receives the value. */
+nb_status nb_dot(const nb_field *x, const nb_field *y, double *host_out);
+
+/* Config C1 (Fig. 4a): for k < iters: x <- x + a*y;
+ * y <- L(x); dots[k] = <x, y>.  Halo on x (L280).  dots_out: host [iters].
+ * Synchronises. */
+nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, int32_t iters, nb_occ occ,
+                                double *dots_out);
+
+/* ---- conjugate gradient (Listing 3, UpdateP first L460) ------- */
+typedef enum { NB_OP_LAPLACE7 = 0, NB_OP_FEM27 = 1 } nb_operator;
+typedef struct {
+    int32_t max_iter;     /* iteration cap                                        */
+    double rtol;          /* stop when <r,r> <= rtol^2 <r0,r0> (0: fixed count)    */
+    nb_occ occ;           /* OCC schedule                                         */
+    int32_t check_every;  /* host convergence polling period (iterations)         */
+    nb_operator op;       /* A = -L (7-point Poisson) or FEM stiffness K          */
+    double fem_E, fem_nu; /* FEM material (op == NB_OP_FEM27)                     */
+} nb_cg_params;
+typedef struct {
+    int32_t iters;        /* iterations performed                                 */
+    int32_t converged;    /* 0 running/cap, 1 rtol reached, 2 rr == 0, 3 breakdown */
+    double rr0;           /* <r0, r0>                                             */
+    double rr;            /* final <r, r>                                         */
+} nb_cg_result;
+/* Set up r = b - A x, <r,r> on the device (stream-ordered, no sync). */
+nb_status nb_cg_create(nb_field *x, const nb_field *b, const nb_cg_params *params, nb_cg **out);
+/* Enqueue `iters` CG iterations (graph-launched; converged state turns
+ * later iterations into no-ops).  No sync. */
+nb_status nb_cg_iterate(nb_cg *cg, int32_t iters);
+/* Apply the deferred x update and read the scalars back.  Synchronises. */
+nb_status nb_cg_finish(nb_cg *cg, nb_cg_result *result);
+nb_status nb_cg_destroy(nb_cg *cg);
+/* create + iterate (polling every check_every) + finish + destroy */
+nb_status nb_cg_solve(nb_field *x, const nb_field *b, const nb_cg_params *params,
+                      nb_cg_result *result);
+
+/* ---- D3Q19 BGK lattice Boltzmann, twoPop ----------- */
+typedef enum { NB_LBM_CAVITY = 0, NB_LBM_PERIODIC = 1 } nb_lbm_bc;
+typedef struct {
+    double omega;   /* BGK relaxation rate                                     */
+    double u_lid;   /* lid velocity (+x) on the face y = Ny (cavity)           */
+    double rho_w;   /* wall density in the moving-wall bounce-back term         */
+    nb_lbm_bc bc;   /* CAVITY (bounce-back walls + lid) or PERIODIC             */
+} nb_lbm_params;
+/* f <- equilibrium(rho0, u0); f: fp32 field of cardinality 19 */
+nb_status nb_lbm_init(nb_field *f, double rho0, const double u0[3]);
+/* nsteps fused pull collide-and-stream steps; *fin and *fout are swapped
+ * after every step (twoPop, L451), so on return *fin holds the latest state.
+ * Halo: 5 populations per side (c_z = +1 up, c_z = -1 down). */
+nb_status nb_lbm_step(nb_field **fin, nb_field **fout, const nb_lbm_params *params,
+                      int32_t nsteps, nb_occ occ);
+/* rho (card 1) and u (card 3) fp32 fields from f */
+nb_status nb_lbm_macroscopic(const nb_field *f, nb_field *rho, nb_field *u);
+
+/* ---- FEM: Q1 hex linear elasticity, 27-point ------- */
+/* y = K u (card 3 fp64), Dirichlet u = 0 on the z = 0 plane (identity
+ * rows/cols).  Reads u's halo planes: call nb_halo_update(u) first. */
+nb_status nb_fem27_apply(const nb_field *u, nb_field *y, double E, double nu);
+/* b = consistent nodal load of pressure p on the top (z = Nz-1) face */
+nb_status nb_fem27_rhs(nb_field *b, double pressure);
+
+/* ---- measurement ------------------------------------------------------ */
+/* When enabled, every kernel launch is bracketed by CUDA events on the
+ * launching stream (graph launch is bypassed).  nb_profile_read
+ * synchronises and returns launch count and summed device time of the
+ * kernels whose name contains `name`. */
+nb_status nb_profile_enable(nb_grid *grid, int32_t enable);
+nb_status nb_profile_read(nb_grid *grid, const char *name, int64_t *launches, double *total_ms);
+/* Number of this library's kernels launched on the grid since creation
+ * (graph launches count their kernel nodes). */
+nb_status nb_launch_count(const nb_grid *grid, int64_t *count);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NB_H */

@@ -1,0 +1,436 @@
+"""B200-native Neon map-stencil hot path — thin Python binding over libnb.so.
+
+Argument marshalling only: every step of the path runs in the CUDA kernels
+of ``libnb.so`` (sm_100a), declared in ``include/nb.h``.  The functions keep
+the C names (``nb_axpy``, ``nb_laplace7``, ``nb_cg_solve`` ...); ``Grid`` and
+``Field`` own the opaque handles.  There is no CPU fallback: importing works
+on any host, but every call that needs a GPU raises ``NbError`` (status
+NB_ECUDA) without one, and a missing ``libnb.so`` raises ``ImportError`` on
+first use.
+
+Paper: Meneghin et al., "Neon: A Multi-GPU Programming Model for Grid-based
+Computations", IPDPS 2022.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+__all__ = [
+    "NbError", "Grid", "Field", "CG", "Comm", "lib", "LIB_PATH",
+    "NB_F32", "NB_F64", "VIEW_STANDARD", "VIEW_INTERNAL", "VIEW_BOUNDARY",
+    "OCC_NONE", "OCC_STANDARD", "OCC_EXTENDED", "OCC_TWO_WAY",
+]
+
+LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libnb.so")
+
+NB_OK, NB_EINVAL, NB_ENOMEM, NB_ECUDA, NB_ENCCL, NB_EMISMATCH, NB_EUNSUPPORTED, NB_ESTATE = range(8)
+NB_F32, NB_F64 = 0, 1
+VIEW_STANDARD, VIEW_INTERNAL, VIEW_BOUNDARY = 0, 1, 2
+OCC_NONE, OCC_STANDARD, OCC_EXTENDED, OCC_TWO_WAY = 0, 1, 2, 3
+FILL_CONST, FILL_UNIFORM, FILL_INT_UNIFORM, FILL_POISSON_RHS = 0, 1, 2, 3
+OP_LAPLACE7, OP_FEM27 = 0, 1
+LBM_CAVITY, LBM_PERIODIC = 0, 1
+OCC_NAMES = {"none": OCC_NONE, "standard": OCC_STANDARD, "extended": OCC_EXTENDED, "two_way": OCC_TWO_WAY}
+
+
+class NbError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"[nb status {status}] {msg}")
+        self.status = status
+
+
+class PartInfo(C.Structure):
+    _fields_ = [("device", C.c_int32), ("local", C.c_int32), ("z_begin", C.c_int32), ("z_end", C.c_int32),
+                ("n_cells", C.c_int64), ("n_bnd_lo", C.c_int64), ("n_bnd_hi", C.c_int64),
+                ("n_internal", C.c_int64)]
+
+
+class CgParams(C.Structure):
+    _fields_ = [("max_iter", C.c_int32), ("rtol", C.c_double), ("occ", C.c_int32),
+                ("check_every", C.c_int32), ("op", C.c_int32), ("fem_E", C.c_double), ("fem_nu", C.c_double)]
+
+
+class CgResult(C.Structure):
+    _fields_ = [("iters", C.c_int32), ("converged", C.c_int32), ("rr0", C.c_double), ("rr", C.c_double)]
+
+
+class LbmParams(C.Structure):
+    _fields_ = [("omega", C.c_double), ("u_lid", C.c_double), ("rho_w", C.c_double), ("bc", C.c_int32)]
+
+
+# exported symbols and their ctypes signatures (the whole of include/nb.h)
+P, I32, I64, D, U64 = C.c_void_p, C.c_int32, C.c_int64, C.c_double, C.c_uint64
+PP = C.POINTER(C.c_void_p)
+SIGNATURES = {
+    "nb_version": ([], C.c_char_p),
+    "nb_last_error": ([], C.c_char_p),
+    "nb_device_count": ([], I32),
+    "nb_comm_unique_id": ([P], I32),
+    "nb_comm_create": ([I32, I32, P, I32, PP], I32),
+    "nb_comm_destroy": ([P], I32),
+    "nb_partition_plan": ([I32, I32, P], I32),
+    "nb_partition_plan_weighted": ([I32, P, I32, P], I32),
+    "nb_grid_create_dense": ([P, I32, P, P, PP], I32),
+    "nb_grid_create_sparse": ([P, P, I32, P, P, PP], I32),
+    "nb_grid_destroy": ([P], I32),
+    "nb_grid_num_partitions": ([P, P], I32),
+    "nb_grid_partition_info": ([P, I32, P], I32),
+    "nb_grid_set_streams": ([P, P, P], I32),
+    "nb_grid_get_stream": ([P, PP], I32),
+    "nb_sync": ([P], I32),
+    "nb_field_create": ([P, I32, I32, D, PP], I32),
+    "nb_field_destroy": ([P], I32),
+    "nb_field_upload": ([P, P, I64], I32),
+    "nb_field_download": ([P, P, I64], I32),
+    "nb_field_fill": ([P, I32, U64, D, D], I32),
+    "nb_halo_update": ([P], I32),
+    "nb_field_partition_ptr": ([P, I32, PP, P, P, P], I32),
+    "nb_axpy": ([D, P, P, I32], I32),
+    "nb_axpby": ([D, P, D, P, I32], I32),
+    "nb_laplace7": ([P, P, I32], I32),
+    "nb_dot": ([P, P, P], I32),
+    "nb_map_stencil_reduce": ([P, P, D, I32, I32, P], I32),
+    "nb_cg_create": ([P, P, P, PP], I32),
+    "nb_cg_iterate": ([P, I32], I32),
+    "nb_cg_finish": ([P, P], I32),
+    "nb_cg_destroy": ([P], I32),
+    "nb_cg_solve": ([P, P, P, P], I32),
+    "nb_lbm_init": ([P, D, P], I32),
+    "nb_lbm_step": ([PP, PP, P, I32, I32], I32),
+    "nb_lbm_macroscopic": ([P, P, P], I32),
+    "nb_fem27_apply": ([P, P, D, D], I32),
+    "nb_fem27_rhs": ([P, D], I32),
+    "nb_profile_enable": ([P, I32], I32),
+    "nb_profile_read": ([P, C.c_char_p, P, P], I32),
+    "nb_launch_count": ([P, P], I32),
+}
+
+_lib = None
+
+
+def lib():
+    """Load libnb.so (loudly: ImportError if it was not built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
+                              "(python -m paper_conf_ipps_meneghinmjm22_b200.build)")
+        L = C.CDLL(LIB_PATH, mode=C.RTLD_GLOBAL)
+        for name, (args, res) in SIGNATURES.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = res
+        _lib = L
+    return _lib
+
+
+def _check(status: int) -> None:
+    if status != NB_OK:
+        raise NbError(status, lib().nb_last_error().decode(errors="replace"))
+
+
+def _h(obj):
+    return obj.handle if hasattr(obj, "handle") else obj
+
+
+_DT = {NB_F32: np.float32, NB_F64: np.float64, "f32": NB_F32, "f64": NB_F64,
+       np.float32: NB_F32, np.float64: NB_F64}
+
+
+def _dtype_code(dt) -> int:
+    if isinstance(dt, int):
+        return dt
+    if isinstance(dt, str):
+        return _DT[dt]
+    return _DT[np.dtype(dt).type]
+
+
+def nb_version() -> str:
+    return lib().nb_version().decode()
+
+
+def nb_device_count() -> int:
+    return int(lib().nb_device_count())
+
+
+def nb_partition_plan(nz: int, nparts: int) -> list:
+    zb = (C.c_int32 * (nparts + 1))()
+    _check(lib().nb_partition_plan(nz, nparts, zb))
+    return list(zb)
+
+
+def nb_partition_plan_weighted(counts, nparts: int) -> list:
+    c = np.ascontiguousarray(counts, dtype=np.int64)
+    zb = (C.c_int32 * (nparts + 1))()
+    _check(lib().nb_partition_plan_weighted(len(c), c.ctypes.data_as(P), nparts, zb))
+    return list(zb)
+
+
+# ---------------------------------------------------------------------------
+class Comm:
+    """One process per GPU: an NCCL communicator created inside libnb.  The
+    128-byte unique id is broadcast with torch.distributed (plumbing)."""
+
+    def __init__(self, world: int, rank: int, device: int, uid: bytes):
+        self.handle = P()
+        buf = (C.c_uint8 * 128).from_buffer_copy(uid)
+        _check(lib().nb_comm_create(world, rank, buf, device, C.byref(self.handle)))
+        self.world, self.rank, self.device = world, rank, device
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = (C.c_uint8 * 128)()
+        _check(lib().nb_comm_unique_id(buf))
+        return bytes(buf)
+
+    @classmethod
+    def from_torch_distributed(cls, device: int):
+        import torch
+        import torch.distributed as dist
+        world, rank = dist.get_world_size(), dist.get_rank()
+        uid = [cls.unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        return cls(world, rank, device, uid[0])
+
+    def close(self):
+        if self.handle:
+            _check(lib().nb_comm_destroy(self.handle))
+            self.handle = P()
+
+
+class Grid:
+    """Dense or element-sparse grid split into z-slabs."""
+
+    def __init__(self, dims, nparts: int = 1, devices=None, comm: Comm | None = None, active=None):
+        self.dims = tuple(int(d) for d in dims)
+        self.nparts = int(nparts)
+        d = (C.c_int32 * 3)(*self.dims)
+        if comm is None:
+            devs = [0] * self.nparts if devices is None else list(devices)
+            dv = (C.c_int32 * self.nparts)(*devs)
+        else:
+            k = self.nparts // comm.world
+            dv = (C.c_int32 * max(k, 1))(*([comm.device] * max(k, 1)))
+        self.handle = P()
+        self.comm = comm
+        self.sparse = active is not None
+        if active is None:
+            _check(lib().nb_grid_create_dense(d, self.nparts, dv, _h(comm) if comm else None,
+                                              C.byref(self.handle)))
+        else:
+            a = np.ascontiguousarray(active, dtype=np.uint8)
+            assert a.shape == self.dims[::-1], "active mask is [z][y][x]"
+            self._active = a
+            _check(lib().nb_grid_create_sparse(d, a.ctypes.data_as(P), self.nparts, dv,
+                                               _h(comm) if comm else None, C.byref(self.handle)))
+
+    @property
+    def ncells(self) -> int:
+        return self.dims[0] * self.dims[1] * self.dims[2]
+
+    def partition_info(self, g: int) -> dict:
+        pi = PartInfo()
+        _check(lib().nb_grid_partition_info(self.handle, g, C.byref(pi)))
+        return {k: getattr(pi, k) for k, _ in PartInfo._fields_}
+
+    def set_streams(self, compute=None, halo=None):
+        _check(lib().nb_grid_set_streams(self.handle, compute, halo))
+
+    def stream(self) -> int:
+        s = P()
+        _check(lib().nb_grid_get_stream(self.handle, C.byref(s)))
+        return s.value or 0
+
+    def sync(self):
+        _check(lib().nb_sync(self.handle))
+
+    def launch_count(self) -> int:
+        n = C.c_int64()
+        _check(lib().nb_launch_count(self.handle, C.byref(n)))
+        return n.value
+
+    def profile(self, enable: bool = True):
+        _check(lib().nb_profile_enable(self.handle, int(enable)))
+
+    def profile_read(self, name: str):
+        n, ms = C.c_int64(), C.c_double()
+        _check(lib().nb_profile_read(self.handle, name.encode(), C.byref(n), C.byref(ms)))
+        return n.value, ms.value
+
+    def close(self):
+        if self.handle:
+            _check(lib().nb_grid_destroy(self.handle))
+            self.handle = P()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+class Field:
+    """Field of `card` components (PAPER.md L58-L63 newField<T>(cardinality,
+    outsideDomainValue)); SoA layout with z halo planes."""
+
+    def __init__(self, grid: Grid, dtype="f64", card: int = 1, outside: float = 0.0):
+        self.grid = grid
+        self.dt = _dtype_code(dtype)
+        self.np_dtype = _DT[self.dt]
+        self.card = int(card)
+        self.outside = float(outside)
+        self.handle = P()
+        _check(lib().nb_field_create(grid.handle, self.dt, self.card, self.outside, C.byref(self.handle)))
+
+    @property
+    def shape(self):
+        nx, ny, nz = self.grid.dims
+        return (nz, ny, nx) if self.card == 1 else (self.card, nz, ny, nx)
+
+    @property
+    def nbytes(self) -> int:
+        return int(np.prod(self.shape)) * np.dtype(self.np_dtype).itemsize
+
+    def upload(self, host) -> None:
+        """host: numpy array (dense logical view) or a pinned CPU torch tensor."""
+        if hasattr(host, "data_ptr"):  # torch tensor (pinned for the e2e path)
+            assert host.numel() * host.element_size() == self.nbytes
+            _check(lib().nb_field_upload(self.handle, P(host.data_ptr()), self.nbytes))
+            self.grid.sync()
+            return
+        a = np.ascontiguousarray(host, dtype=self.np_dtype)
+        assert a.size * a.itemsize == self.nbytes, (a.shape, self.shape)
+        _check(lib().nb_field_upload(self.handle, a.ctypes.data_as(P), a.nbytes))
+        self.grid.sync()  # the host buffer is borrowed until the copy completes
+
+    def upload_async(self, ptr: int) -> None:
+        _check(lib().nb_field_upload(self.handle, P(ptr), self.nbytes))
+
+    def download(self, out=None):
+        if out is not None and hasattr(out, "data_ptr"):
+            _check(lib().nb_field_download(self.handle, P(out.data_ptr()), self.nbytes))
+            return out
+        a = np.empty(self.shape, dtype=self.np_dtype) if out is None else out
+        _check(lib().nb_field_download(self.handle, a.ctypes.data_as(P), self.nbytes))
+        return a
+
+    def fill(self, kind: int, seed: int = 0, a: float = 0.0, b: float = 0.0):
+        _check(lib().nb_field_fill(self.handle, kind, seed, a, b))
+
+    def fill_uniform(self, seed=1, lo=-1.0, hi=1.0):
+        self.fill(FILL_UNIFORM, seed, lo, hi)
+
+    def fill_int(self, seed=1, lo=-8, hi=8):
+        self.fill(FILL_INT_UNIFORM, seed, lo, hi)
+
+    def fill_const(self, v):
+        self.fill(FILL_CONST, 0, v, 0.0)
+
+    def halo_update(self):
+        _check(lib().nb_halo_update(self.handle))
+
+    def partition_ptr(self, g: int):
+        p, pitch, ps, cs = P(), C.c_int64(), C.c_int64(), C.c_int64()
+        _check(lib().nb_field_partition_ptr(self.handle, g, C.byref(p), C.byref(pitch), C.byref(ps),
+                                            C.byref(cs)))
+        return p.value, pitch.value, ps.value, cs.value
+
+    def close(self):
+        if self.handle:
+            _check(lib().nb_field_destroy(self.handle))
+            self.handle = P()
+
+
+# ---- ops (same names as the C ABI) -----------------------------------------
+def nb_axpy(a: float, x: Field, y: Field, view: int = VIEW_STANDARD):
+    _check(lib().nb_axpy(a, _h(x), _h(y), view))
+
+
+def nb_axpby(a: float, x: Field, b: float, y: Field, view: int = VIEW_STANDARD):
+    _check(lib().nb_axpby(a, _h(x), b, _h(y), view))
+
+
+def nb_laplace7(x: Field, y: Field, view: int = VIEW_STANDARD):
+    _check(lib().nb_laplace7(_h(x), _h(y), view))
+
+
+def nb_halo_update(f: Field):
+    _check(lib().nb_halo_update(_h(f)))
+
+
+def nb_dot(x: Field, y: Field) -> float:
+    out = C.c_double()
+    _check(lib().nb_dot(_h(x), _h(y), C.byref(out)))
+    return out.value
+
+
+def nb_map_stencil_reduce(x: Field, y: Field, a: float = 0.125, iters: int = 10, occ: int = OCC_TWO_WAY):
+    dots = np.zeros(max(iters, 1), dtype=np.float64)
+    _check(lib().nb_map_stencil_reduce(_h(x), _h(y), a, iters, occ, dots.ctypes.data_as(P)))
+    return dots[:iters]
+
+
+def _cg_params(max_iter, rtol, occ, check_every, op, E, nu):
+    return CgParams(int(max_iter), float(rtol), int(occ), int(check_every), int(op), float(E), float(nu))
+
+
+class CG:
+    """Matrix-free CG (Listing 3, UpdateP first L460) driven on the device."""
+
+    def __init__(self, x: Field, b: Field, max_iter=100, rtol=0.0, occ=OCC_TWO_WAY, check_every=16,
+                 op=OP_LAPLACE7, E=1.0, nu=0.3):
+        self.prm = _cg_params(max_iter, rtol, occ, check_every, op, E, nu)
+        self.handle = P()
+        _check(lib().nb_cg_create(_h(x), _h(b), C.byref(self.prm), C.byref(self.handle)))
+
+    def iterate(self, n: int):
+        _check(lib().nb_cg_iterate(self.handle, int(n)))
+
+    def finish(self) -> CgResult:
+        r = CgResult()
+        _check(lib().nb_cg_finish(self.handle, C.byref(r)))
+        return r
+
+    def close(self):
+        if self.handle:
+            _check(lib().nb_cg_destroy(self.handle))
+            self.handle = P()
+
+
+def nb_cg_solve(x: Field, b: Field, max_iter=100, rtol=0.0, occ=OCC_TWO_WAY, check_every=16,
+                op=OP_LAPLACE7, E=1.0, nu=0.3) -> CgResult:
+    prm = _cg_params(max_iter, rtol, occ, check_every, op, E, nu)
+    r = CgResult()
+    _check(lib().nb_cg_solve(_h(x), _h(b), C.byref(prm), C.byref(r)))
+    return r
+
+
+def nb_lbm_init(f: Field, rho0: float = 1.0, u0=(0.0, 0.0, 0.0)):
+    u = (C.c_double * 3)(*u0)
+    _check(lib().nb_lbm_init(_h(f), rho0, u))
+
+
+def nb_lbm_step(fin: Field, fout: Field, omega: float, nsteps: int = 1, u_lid: float = 0.05,
+                rho_w: float = 1.0, bc: int = LBM_CAVITY, occ: int = OCC_STANDARD):
+    """Returns (fin, fout) after the swaps: fin holds the latest state."""
+    prm = LbmParams(omega, u_lid, rho_w, bc)
+    a, b = P(fin.handle.value), P(fout.handle.value)
+    _check(lib().nb_lbm_step(C.byref(a), C.byref(b), C.byref(prm), int(nsteps), int(occ)))
+    if a.value == fin.handle.value:
+        return fin, fout
+    return fout, fin
+
+
+def nb_lbm_macroscopic(f: Field, rho: Field, u: Field):
+    _check(lib().nb_lbm_macroscopic(_h(f), _h(rho), _h(u)))
+
+
+def nb_fem27_apply(u: Field, y: Field, E: float = 1.0, nu: float = 0.3):
+    _check(lib().nb_fem27_apply(_h(u), _h(y), E, nu))
+
+
+def nb_fem27_rhs(b: Field, pressure: float = 1.0):
+    _check(lib().nb_fem27_rhs(_h(b), pressure))

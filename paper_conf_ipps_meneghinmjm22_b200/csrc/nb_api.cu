@@ -1,0 +1,1059 @@
+// nb_api.cu — grid, field, halo, map and reduce entry points of libnb.
+//
+// Paper: Neon (Meneghin et al., IPDPS 2022), /root/reference/PAPER.md.
+//   Grid / Field / views / haloUpdate: §IV-C
+//   MapOp / ReduceOp:                  §III-b L96-L131 (eqs.)
+//   Host logical view:                 L219-L221
+// Design: DESIGN.md ("Data layout", "Deterministic reductions", "Halo").
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstring>
+#include <mutex>
+
+#include "nb_device.cuh"
+#include "nb_internal.cuh"
+
+// ===========================================================================
+// errors, version
+// ===========================================================================
+static thread_local char g_err[1024] = "";
+
+void nb_set_error(const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+}
+
+extern "C" const char *nb_version(void) { return "nb 0.1.0 (sm_100a)"; }
+extern "C" const char *nb_last_error(void) { return g_err; }
+
+extern "C" int32_t nb_device_count(void) {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    return n;
+}
+
+nb_status nb_launch_check(const char *what) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "launch of %s failed: %s", what, cudaGetErrorString(e));
+    return NB_OK;
+}
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int d) {
+        cudaGetDevice(&prev);
+        if (prev != d) cudaSetDevice(d);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+// ===========================================================================
+// NCCL, loaded at run time (no link-time dependency; one process per GPU)
+// ===========================================================================
+namespace {
+typedef int nccl_res_t;
+struct NcclApi {
+    void *h = nullptr;
+    nccl_res_t (*GetUniqueId)(void *id) = nullptr;
+    nccl_res_t (*CommInitRank)(void **comm, int nranks, /*ncclUniqueId by value*/ ...) = nullptr;
+    nccl_res_t (*CommDestroy)(void *comm) = nullptr;
+    nccl_res_t (*Send)(const void *, size_t, int, int, void *, cudaStream_t) = nullptr;
+    nccl_res_t (*Recv)(void *, size_t, int, int, void *, cudaStream_t) = nullptr;
+    nccl_res_t (*AllReduce)(const void *, void *, size_t, int, int, void *, cudaStream_t) = nullptr;
+    nccl_res_t (*GroupStart)() = nullptr;
+    nccl_res_t (*GroupEnd)() = nullptr;
+    const char *(*GetErrorString)(nccl_res_t) = nullptr;
+};
+struct NcclUid {
+    char internal[128];
+};
+typedef nccl_res_t (*InitRankFn)(void **, int, NcclUid, int);
+NcclApi g_nccl;
+InitRankFn g_nccl_init = nullptr;
+std::mutex g_nccl_mu;
+constexpr int NCCL_UINT8 = 1, NCCL_FLOAT64 = 8, NCCL_SUM = 0;
+
+nb_status nccl_load() {
+    std::lock_guard<std::mutex> lk(g_nccl_mu);
+    if (g_nccl.h) return NB_OK;
+    const char *names[] = {"libnccl.so.2", "libnccl.so"};
+    void *h = nullptr;
+    for (const char *n : names)
+        if ((h = dlopen(n, RTLD_NOW | RTLD_GLOBAL))) break;
+    if (!h) {
+        // the torch-bundled NCCL of the venv
+        const char *env = getenv("NB_NCCL_LIB");
+        if (env) h = dlopen(env, RTLD_NOW | RTLD_GLOBAL);
+    }
+    if (!h) NB_FAIL(NB_ENCCL, "cannot dlopen libnccl.so.2 (set NB_NCCL_LIB)");
+#define LOAD(field, sym)                                                         \
+    *(void **)(&g_nccl.field) = dlsym(h, sym);                                   \
+    if (!g_nccl.field) NB_FAIL(NB_ENCCL, "libnccl is missing symbol %s", sym);
+    LOAD(GetUniqueId, "ncclGetUniqueId");
+    LOAD(CommDestroy, "ncclCommDestroy");
+    LOAD(Send, "ncclSend");
+    LOAD(Recv, "ncclRecv");
+    LOAD(AllReduce, "ncclAllReduce");
+    LOAD(GroupStart, "ncclGroupStart");
+    LOAD(GroupEnd, "ncclGroupEnd");
+    LOAD(GetErrorString, "ncclGetErrorString");
+#undef LOAD
+    *(void **)(&g_nccl_init) = dlsym(h, "ncclCommInitRank");
+    if (!g_nccl_init) NB_FAIL(NB_ENCCL, "libnccl is missing ncclCommInitRank");
+    g_nccl.h = h;
+    return NB_OK;
+}
+
+#define NB_NCCL(call)                                                                   \
+    do {                                                                                \
+        nccl_res_t _r = (call);                                                         \
+        if (_r != 0)                                                                    \
+            NB_FAIL(NB_ENCCL, "%s failed: %s", #call,                                   \
+                    g_nccl.GetErrorString ? g_nccl.GetErrorString(_r) : "?");           \
+    } while (0)
+}  // namespace
+
+extern "C" nb_status nb_comm_unique_id(uint8_t out[128]) {
+    if (!out) NB_FAIL(NB_EINVAL, "nb_comm_unique_id: out is NULL");
+    NB_TRY(nccl_load());
+    NcclUid id;
+    NB_NCCL(g_nccl.GetUniqueId(&id));
+    memcpy(out, id.internal, 128);
+    return NB_OK;
+}
+
+extern "C" nb_status nb_comm_create(int32_t world, int32_t rank, const uint8_t id[128],
+                                    int32_t device, nb_comm **out) {
+    if (!out || !id || world < 1 || rank < 0 || rank >= world)
+        NB_FAIL(NB_EINVAL, "nb_comm_create: bad arguments (world %d rank %d)", world, rank);
+    *out = nullptr;
+    if (device < 0 || device >= nb_device_count())
+        NB_FAIL(NB_ECUDA, "nb_comm_create: device %d not available", device);
+    nb_comm *c = new nb_comm();
+    c->world = world;
+    c->rank = rank;
+    c->device = device;
+    if (world > 1) {
+        nb_status s = nccl_load();
+        if (s != NB_OK) {
+            delete c;
+            return s;
+        }
+        DeviceGuard dg(device);
+        NcclUid uid;
+        memcpy(uid.internal, id, 128);
+        nccl_res_t r = g_nccl_init(&c->nccl, world, uid, rank);
+        if (r != 0) {
+            delete c;
+            NB_FAIL(NB_ENCCL, "ncclCommInitRank failed: %s", g_nccl.GetErrorString(r));
+        }
+    }
+    *out = c;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_comm_destroy(nb_comm *comm) {
+    if (!comm) return NB_OK;
+    if (comm->nccl) g_nccl.CommDestroy(comm->nccl);
+    delete comm;
+    return NB_OK;
+}
+
+nb_status nb_nccl_allreduce_sum(nb_grid *g, const double *send, double *recv, size_t n,
+                                cudaStream_t s) {
+    NB_NCCL(g_nccl.AllReduce(send, recv, n, NCCL_FLOAT64, NCCL_SUM, g->comm->nccl, s));
+    return NB_OK;
+}
+nb_status nb_nccl_group(nb_grid *g, bool start) {
+    (void)g;
+    if (start)
+        NB_NCCL(g_nccl.GroupStart());
+    else
+        NB_NCCL(g_nccl.GroupEnd());
+    return NB_OK;
+}
+nb_status nb_nccl_send(nb_grid *g, const void *buf, size_t bytes, int peer, cudaStream_t s) {
+    NB_NCCL(g_nccl.Send(buf, bytes, NCCL_UINT8, peer, g->comm->nccl, s));
+    return NB_OK;
+}
+nb_status nb_nccl_recv(nb_grid *g, void *buf, size_t bytes, int peer, cudaStream_t s) {
+    NB_NCCL(g_nccl.Recv(buf, bytes, NCCL_UINT8, peer, g->comm->nccl, s));
+    return NB_OK;
+}
+
+int nb_part_owner(const nb_grid *g, int part) {
+    if (!g->comm || g->comm->world <= 1) return 0;
+    return part / (g->nparts / g->comm->world);
+}
+
+// ===========================================================================
+// partition plans (a1) — pure host logic
+// ===========================================================================
+extern "C" nb_status nb_partition_plan(int32_t nz, int32_t nparts, int32_t *z_begin) {
+    if (!z_begin || nparts < 1 || nz < 1) NB_FAIL(NB_EINVAL, "nb_partition_plan: bad arguments");
+    if (nparts > nz) NB_FAIL(NB_EINVAL, "nb_partition_plan: %d partitions for %d planes", nparts, nz);
+    int base = nz / nparts, rem = nz % nparts, z = 0;
+    for (int g = 0; g < nparts; ++g) {
+        z_begin[g] = z;
+        z += base + (g < rem ? 1 : 0);
+    }
+    z_begin[nparts] = nz;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_partition_plan_weighted(int32_t nz, const int64_t *counts, int32_t nparts,
+                                                int32_t *z_begin) {
+    if (!z_begin || !counts || nparts < 1 || nz < 1 || nparts > nz)
+        NB_FAIL(NB_EINVAL, "nb_partition_plan_weighted: bad arguments");
+    int64_t total = 0;
+    for (int z = 0; z < nz; ++z) {
+        if (counts[z] < 0) NB_FAIL(NB_EINVAL, "nb_partition_plan_weighted: negative count");
+        total += counts[z];
+    }
+    z_begin[0] = 0;
+    int64_t pref = 0;
+    int z = 0;
+    for (int g = 1; g < nparts; ++g) {
+        // target prefix for the end of partition g-1; __int128 avoids overflow
+        __int128 target = (__int128)total * g;
+        int zmin = z_begin[g - 1] + 1;          // non-empty slab
+        int zmax = nz - (nparts - g);           // leave >= 1 plane per remaining part
+        while (z < zmin) pref += counts[z++];
+        while (z < zmax && (__int128)pref * nparts < target) pref += counts[z++];
+        // step back one plane if that lands closer to the target
+        if (z > zmin) {
+            __int128 over = (__int128)pref * nparts - target;
+            __int128 under = target - (__int128)(pref - counts[z - 1]) * nparts;
+            if (over > 0 && under < over) pref -= counts[--z];
+        }
+        z_begin[g] = z;
+    }
+    z_begin[nparts] = nz;
+    return NB_OK;
+}
+
+// ===========================================================================
+// grid
+// ===========================================================================
+static nb_status grid_alloc_common(nb_grid *g) {
+    DeviceGuard dg(g->device);
+    NB_CUDA(cudaStreamCreateWithFlags(&g->cs, cudaStreamNonBlocking));
+    NB_CUDA(cudaStreamCreateWithFlags(&g->hs, cudaStreamNonBlocking));
+    g->own_cs = g->own_hs = true;
+    g->tiles_x = (g->nx + DOT_TX - 1) / DOT_TX;
+    g->tiles_y = (g->ny + DOT_TY - 1) / DOT_TY;
+    g->T = g->tiles_x * g->tiles_y;
+    size_t planes = (size_t)g->max_card * g->nz;
+    NB_CUDA(cudaMalloc(&g->tp, sizeof(double) * planes * g->T));
+    NB_CUDA(cudaMalloc(&g->psum, sizeof(double) * planes));
+    NB_CUDA(cudaMalloc(&g->psum_send, sizeof(double) * planes));
+    NB_CUDA(cudaMalloc(&g->dots, sizeof(double) * NB_DOT_SLOTS));
+    NB_CUDA(cudaMalloc(&g->counter, sizeof(unsigned int) * 16));
+    NB_CUDA(cudaMemset(g->tp, 0, sizeof(double) * planes * g->T));
+    NB_CUDA(cudaMemset(g->psum, 0, sizeof(double) * planes));
+    NB_CUDA(cudaMemset(g->psum_send, 0, sizeof(double) * planes));
+    NB_CUDA(cudaMemset(g->dots, 0, sizeof(double) * NB_DOT_SLOTS));
+    NB_CUDA(cudaMemset(g->counter, 0, sizeof(unsigned int) * 16));
+    return NB_OK;
+}
+
+nb_status nb_grid_setup_parts(nb_grid *g, const int32_t *zb, int32_t nparts,
+                              const int32_t *device_ids, nb_comm *comm) {
+    g->nparts = nparts;
+    g->comm = comm;
+    int world = comm ? comm->world : 1, rank = comm ? comm->rank : 0;
+    if (nparts % world != 0)
+        NB_FAIL(NB_EINVAL, "nparts (%d) must be a multiple of the world size (%d)", nparts, world);
+    int k = nparts / world;
+    g->first_local = rank * k;
+    g->nlocal = k;
+    g->parts.resize(nparts);
+    for (int p = 0; p < nparts; ++p) {
+        NbPart &q = g->parts[p];
+        q.z0 = zb[p];
+        q.z1 = zb[p + 1];
+        q.lo = p > 0 ? p - 1 : -1;
+        q.hi = p < nparts - 1 ? p + 1 : -1;
+        q.local = (p >= g->first_local && p < g->first_local + k);
+    }
+    if (comm) {
+        g->device = comm->device;
+    } else {
+        if (!device_ids) NB_FAIL(NB_EINVAL, "device_ids is NULL");
+        g->device = device_ids[0];
+        for (int p = 0; p < nparts; ++p)
+            if (device_ids[p] != g->device)
+                NB_FAIL(NB_EUNSUPPORTED,
+                        "single-process grids keep all partitions on one device (got %d and %d); "
+                        "use one process per GPU with an nb_comm",
+                        g->device, device_ids[p]);
+    }
+    for (int p = 0; p < nparts; ++p) g->parts[p].device = g->device;
+    if (g->device < 0 || g->device >= nb_device_count())
+        NB_FAIL(NB_ECUDA, "CUDA device %d not available (no CPU fallback)", g->device);
+    return NB_OK;
+}
+
+extern "C" nb_status nb_grid_create_dense(const int32_t dims[3], int32_t nparts,
+                                          const int32_t *device_ids, nb_comm *comm,
+                                          nb_grid **out) {
+    if (!out || !dims) NB_FAIL(NB_EINVAL, "nb_grid_create_dense: NULL argument");
+    *out = nullptr;
+    if (dims[0] < 1 || dims[1] < 1 || dims[2] < 1 || dims[0] > 65535 || dims[1] > 65535)
+        NB_FAIL(NB_EINVAL, "nb_grid_create_dense: bad dims %d x %d x %d", dims[0], dims[1], dims[2]);
+    std::vector<int32_t> zb(nparts > 0 ? nparts + 1 : 1);
+    NB_TRY(nb_partition_plan(dims[2], nparts, zb.data()));
+    if (nparts > 1)
+        for (int p = 0; p < nparts; ++p)
+            if (zb[p + 1] - zb[p] < 2)
+                NB_FAIL(NB_EUNSUPPORTED, "slab %d has %d plane(s); need >= 2 (radius 1)", p,
+                        zb[p + 1] - zb[p]);
+    nb_grid *g = new nb_grid();
+    g->nx = dims[0];
+    g->ny = dims[1];
+    g->nz = dims[2];
+    nb_status s = nb_grid_setup_parts(g, zb.data(), nparts, device_ids, comm);
+    if (s == NB_OK) s = grid_alloc_common(g);
+    if (s != NB_OK) {
+        nb_grid_destroy(g);
+        return s;
+    }
+    for (auto &p : g->parts) {
+        int64_t plane = (int64_t)g->nx * g->ny;
+        p.n_act = plane * p.nz();
+        p.n_lo_bnd = p.lo >= 0 ? plane : 0;
+        p.n_hi_bnd = p.hi >= 0 ? plane : 0;
+    }
+    *out = g;
+    return NB_OK;
+}
+
+void nb_sparse_free(nb_grid *g);  // nb_sparse.cu
+
+extern "C" nb_status nb_grid_destroy(nb_grid *g) {
+    if (!g) return NB_OK;
+    if (g->nfields > 0 || g->nsolvers > 0)
+        NB_FAIL(NB_ESTATE, "nb_grid_destroy: %d field(s) and %d solver(s) still alive", g->nfields,
+                g->nsolvers);
+    DeviceGuard dg(g->device);
+    if (g->cs) cudaStreamSynchronize(g->cs);
+    if (g->hs) cudaStreamSynchronize(g->hs);
+    for (auto &r : g->prof) {
+        cudaEventDestroy(r.a);
+        cudaEventDestroy(r.b);
+    }
+    nb_sparse_free(g);
+    cudaFree(g->tp);
+    cudaFree(g->psum);
+    cudaFree(g->psum_send);
+    cudaFree(g->dots);
+    cudaFree(g->counter);
+    if (g->own_cs && g->cs) cudaStreamDestroy(g->cs);
+    if (g->own_hs && g->hs) cudaStreamDestroy(g->hs);
+    delete g;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_grid_num_partitions(const nb_grid *g, int32_t *n) {
+    if (!g || !n) NB_FAIL(NB_EINVAL, "NULL argument");
+    *n = g->nparts;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_grid_partition_info(const nb_grid *g, int32_t p, nb_part_info *o) {
+    if (!g || !o || p < 0 || p >= g->nparts) NB_FAIL(NB_EINVAL, "nb_grid_partition_info: bad arguments");
+    const NbPart &q = g->parts[p];
+    o->device = q.device;
+    o->local = q.local;
+    o->z_begin = q.z0;
+    o->z_end = q.z1;
+    o->n_cells = q.n_act;
+    o->n_bnd_lo = q.n_lo_bnd;
+    o->n_bnd_hi = q.n_hi_bnd;
+    o->n_internal = q.n_act - q.n_lo_bnd - (q.nz() > 1 ? q.n_hi_bnd : 0);
+    return NB_OK;
+}
+
+extern "C" nb_status nb_grid_set_streams(nb_grid *g, void *cs, void *hs) {
+    if (!g) NB_FAIL(NB_EINVAL, "NULL grid");
+    DeviceGuard dg(g->device);
+    if (cs) {
+        if (g->own_cs) {
+            cudaStreamSynchronize(g->cs);
+            cudaStreamDestroy(g->cs);
+        }
+        g->cs = (cudaStream_t)cs;
+        g->own_cs = false;
+    }
+    if (hs) {
+        if (g->own_hs) {
+            cudaStreamSynchronize(g->hs);
+            cudaStreamDestroy(g->hs);
+        }
+        g->hs = (cudaStream_t)hs;
+        g->own_hs = false;
+    }
+    return NB_OK;
+}
+
+extern "C" nb_status nb_grid_get_stream(const nb_grid *g, void **cs) {
+    if (!g || !cs) NB_FAIL(NB_EINVAL, "NULL argument");
+    *cs = (void *)g->cs;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_sync(nb_grid *g) {
+    if (!g) NB_FAIL(NB_EINVAL, "NULL grid");
+    DeviceGuard dg(g->device);
+    NB_CUDA(cudaStreamSynchronize(g->hs));
+    NB_CUDA(cudaStreamSynchronize(g->cs));
+    NB_CUDA(cudaGetLastError());
+    return NB_OK;
+}
+
+// ===========================================================================
+// fields (dense)
+// ===========================================================================
+nb_status nb_sparse_field_alloc(nb_field *f);            // nb_sparse.cu
+nb_status nb_sparse_upload(nb_field *f, const void *host);
+nb_status nb_sparse_download(const nb_field *f, void *host);
+nb_status nb_sparse_fill(nb_field *f, nb_fill kind, uint64_t seed, double a, double b);
+
+template <typename T>
+__global__ void k_fill_const(T *p, int64_t n, T v) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = v;
+}
+
+static nb_status fill_const_raw(nb_grid *g, void *p, int64_t n, nb_dtype dt, double v,
+                                cudaStream_t s) {
+    if (n <= 0) return NB_OK;
+    int blocks = (int)std::min<int64_t>((n + 255) / 256, 148 * 16);
+    LaunchScope ls(g, s, "k_fill_const");
+    if (dt == NB_F64)
+        k_fill_const<double><<<blocks, 256, 0, s>>>((double *)p, n, v);
+    else
+        k_fill_const<float><<<blocks, 256, 0, s>>>((float *)p, n, (float)v);
+    return nb_launch_check("k_fill_const");
+}
+
+extern "C" nb_status nb_field_create(nb_grid *g, nb_dtype dt, int32_t card, double outside,
+                                     nb_field **out) {
+    if (!g || !out) NB_FAIL(NB_EINVAL, "nb_field_create: NULL argument");
+    *out = nullptr;
+    if (dt != NB_F32 && dt != NB_F64) NB_FAIL(NB_EINVAL, "nb_field_create: bad dtype %d", (int)dt);
+    if (card < 1 || card > 64) NB_FAIL(NB_EINVAL, "nb_field_create: cardinality %d", card);
+    DeviceGuard dg(g->device);
+    nb_field *f = new nb_field();
+    f->g = g;
+    f->dt = dt;
+    f->card = card;
+    f->outside = outside;
+    f->esz = dt == NB_F64 ? 8 : 4;
+    f->base.assign(g->nparts, nullptr);
+    f->bytes.assign(g->nparts, 0);
+    nb_status s = NB_OK;
+    if (g->sparse) {
+        s = nb_sparse_field_alloc(f);
+    } else {
+        f->pitch = ((int64_t)g->nx + 31) / 32 * 32;
+        f->ps = f->pitch * g->ny;
+        for (int p = 0; p < g->nparts && s == NB_OK; ++p) {
+            if (!g->parts[p].local) continue;
+            f->cs = f->ps * (g->parts[p].nz() + 2);
+            size_t bytes = (size_t)f->cs * card * f->esz;
+            cudaError_t e = cudaMalloc(&f->base[p], bytes);
+            if (e != cudaSuccess) {
+                cudaGetLastError();
+                nb_set_error("nb_field_create: cudaMalloc(%zu) failed: %s", bytes, cudaGetErrorString(e));
+                s = NB_ENOMEM;
+                break;
+            }
+            f->bytes[p] = bytes;
+            if (outside == 0.0)
+                e = cudaMemsetAsync(f->base[p], 0, bytes, g->cs);
+            else
+                s = fill_const_raw(g, f->base[p], (int64_t)(bytes / f->esz), dt, outside, g->cs);
+            if (e != cudaSuccess) {
+                nb_set_error("cudaMemset failed: %s", cudaGetErrorString(e));
+                s = NB_ECUDA;
+            }
+        }
+        // component stride must be uniform across partitions for the kernels'
+        // per-partition arithmetic; it is per partition: store the local one
+        // (all local partitions share the formula cs = ps*(nz_p+2)).
+    }
+    if (s != NB_OK) {
+        for (auto p : f->base)
+            if (p) cudaFree(p);
+        delete f;
+        return s;
+    }
+    g->nfields++;
+    *out = f;
+    return NB_OK;
+}
+
+// component stride of partition p (dense): ps * (nz_p + 2)
+static inline int64_t dense_cs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
+
+extern "C" nb_status nb_field_destroy(nb_field *f) {
+    if (!f) return NB_OK;
+    DeviceGuard dg(f->g->device);
+    cudaStreamSynchronize(f->g->cs);
+    cudaStreamSynchronize(f->g->hs);
+    for (auto p : f->base)
+        if (p) cudaFree(p);
+    f->g->nfields--;
+    delete f;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_field_partition_ptr(const nb_field *f, int32_t p, void **ptr, int64_t *pitch,
+                                            int64_t *pstride, int64_t *cstride) {
+    if (!f || p < 0 || p >= f->g->nparts) NB_FAIL(NB_EINVAL, "nb_field_partition_ptr: bad arguments");
+    if (!f->g->parts[p].local) NB_FAIL(NB_EINVAL, "partition %d is not local", p);
+    if (ptr) *ptr = f->base[p];
+    if (pitch) *pitch = f->pitch;
+    if (pstride) *pstride = f->ps;
+    if (cstride) *cstride = f->g->sparse ? f->cs : dense_cs(f, p);
+    return NB_OK;
+}
+
+static size_t logical_bytes(const nb_field *f) {
+    return (size_t)f->g->nx * f->g->ny * f->g->nz * f->card * f->esz;
+}
+
+extern "C" nb_status nb_field_upload(nb_field *f, const void *host, int64_t nbytes) {
+    if (!f || !host) NB_FAIL(NB_EINVAL, "nb_field_upload: NULL argument");
+    if ((size_t)nbytes != logical_bytes(f))
+        NB_FAIL(NB_EINVAL, "nb_field_upload: %lld bytes, expected %zu", (long long)nbytes, logical_bytes(f));
+    nb_grid *g = f->g;
+    DeviceGuard dg(g->device);
+    if (g->sparse) return nb_sparse_upload(f, host);
+    const char *h = (const char *)host;
+    size_t row = (size_t)g->nx * f->esz, plane = row * g->ny;
+    for (int p = 0; p < g->nparts; ++p) {
+        if (!g->parts[p].local) continue;
+        const NbPart &q = g->parts[p];
+        for (int c = 0; c < f->card; ++c) {
+            char *dst = f->base[p] + ((int64_t)c * dense_cs(f, p) + f->ps) * f->esz;
+            const char *src = h + ((size_t)c * g->nz + q.z0) * plane;
+            NB_CUDA(cudaMemcpy2DAsync(dst, f->pitch * f->esz, src, row, row, (size_t)g->ny * q.nz(),
+                                      cudaMemcpyHostToDevice, g->cs));
+        }
+    }
+    return NB_OK;
+}
+
+extern "C" nb_status nb_field_download(const nb_field *f, void *host, int64_t nbytes) {
+    if (!f || !host) NB_FAIL(NB_EINVAL, "nb_field_download: NULL argument");
+    if ((size_t)nbytes != logical_bytes(f))
+        NB_FAIL(NB_EINVAL, "nb_field_download: %lld bytes, expected %zu", (long long)nbytes, logical_bytes(f));
+    nb_grid *g = f->g;
+    DeviceGuard dg(g->device);
+    if (g->sparse) return nb_sparse_download(f, host);
+    char *h = (char *)host;
+    size_t row = (size_t)g->nx * f->esz, plane = row * g->ny;
+    for (int p = 0; p < g->nparts; ++p) {
+        if (!g->parts[p].local) continue;
+        const NbPart &q = g->parts[p];
+        for (int c = 0; c < f->card; ++c) {
+            const char *src = f->base[p] + ((int64_t)c * dense_cs(f, p) + f->ps) * f->esz;
+            char *dst = h + ((size_t)c * g->nz + q.z0) * plane;
+            NB_CUDA(cudaMemcpy2DAsync(dst, row, src, f->pitch * f->esz, row, (size_t)g->ny * q.nz(),
+                                      cudaMemcpyDeviceToHost, g->cs));
+        }
+    }
+    NB_CUDA(cudaStreamSynchronize(g->cs));
+    return NB_OK;
+}
+
+// ---- counter-based fill (same generator as synth/, own implementation) -----
+__device__ __forceinline__ uint64_t nb_mix64(uint64_t z) {
+    z ^= z >> 30;
+    z *= 0xBF58476D1CE4E5B9ull;
+    z ^= z >> 27;
+    z *= 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    return z;
+}
+
+__device__ __forceinline__ double nb_gen(int kind, uint64_t seed, uint64_t gidx, double a, double b,
+                                         int x, int y, int z, double h) {
+    if (kind == NB_FILL_CONST) return a;
+    if (kind == NB_FILL_POISSON_RHS) {
+        // b = (h*h) * (((gy*gz + gx*gz) + gx*gy) * 2), g(t) = t*(1-t), t = (i+1)*h
+        double tx = __dmul_rn((double)(x + 1), h), ty = __dmul_rn((double)(y + 1), h),
+               tz = __dmul_rn((double)(z + 1), h);
+        double gx = __dmul_rn(tx, __dsub_rn(1.0, tx)), gy = __dmul_rn(ty, __dsub_rn(1.0, ty)),
+               gz = __dmul_rn(tz, __dsub_rn(1.0, tz));
+        double f = __dadd_rn(__dadd_rn(__dmul_rn(gy, gz), __dmul_rn(gx, gz)), __dmul_rn(gx, gy));
+        f = __dmul_rn(f, 2.0);
+        return __dmul_rn(__dmul_rn(h, h), f);
+    }
+    uint64_t hsh = nb_mix64(seed * 0x9E3779B97F4A7C15ull + gidx + 1ull);
+    if (kind == NB_FILL_UNIFORM) {
+        double u = (double)(hsh >> 11) * 0x1p-53;
+        return __dadd_rn(a, __dmul_rn(__dsub_rn(b, a), u));
+    }
+    // INT_UNIFORM: a + (h mod (b - a + 1))
+    int64_t lo = (int64_t)a, hi = (int64_t)b;
+    uint64_t span = (uint64_t)(hi - lo + 1);
+    return (double)((int64_t)(hsh % span) + lo);
+}
+
+template <typename T>
+__global__ void k_fill_gen(T *base, PGeo g, int64_t cstride, int card, int kind, uint64_t seed,
+                           double a, double b, double h) {
+    int x = blockIdx.x * blockDim.x + threadIdx.x;
+    int y = blockIdx.y;
+    int zl = blockIdx.z % g.nzl;
+    int c = blockIdx.z / g.nzl;
+    if (x >= g.nx || c >= card) return;
+    int z = g.z0 + zl;
+    uint64_t gidx = (uint64_t)x + (uint64_t)g.nx * ((uint64_t)y + (uint64_t)g.ny * ((uint64_t)z + (uint64_t)g.NZ * c));
+    double v = nb_gen(kind, seed, gidx, a, b, x, y, z, h);
+    base[(int64_t)c * cstride + (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x] = (T)v;
+}
+
+extern "C" nb_status nb_field_fill(nb_field *f, nb_fill kind, uint64_t seed, double a, double b) {
+    if (!f) NB_FAIL(NB_EINVAL, "nb_field_fill: NULL field");
+    if (kind < NB_FILL_CONST || kind > NB_FILL_POISSON_RHS) NB_FAIL(NB_EINVAL, "bad fill kind");
+    nb_grid *g = f->g;
+    if (kind == NB_FILL_INT_UNIFORM && !(b >= a)) NB_FAIL(NB_EINVAL, "INT_UNIFORM needs b >= a");
+    if (kind == NB_FILL_POISSON_RHS && !(g->nx == g->ny && g->ny == g->nz))
+        NB_FAIL(NB_EUNSUPPORTED, "POISSON_RHS is defined on cubic grids");
+    DeviceGuard dg(g->device);
+    if (g->sparse) return nb_sparse_fill(f, kind, seed, a, b);
+    double h = 1.0 / (double)(g->nx + 1);
+    for (int p = 0; p < g->nparts; ++p) {
+        if (!g->parts[p].local) continue;
+        PGeo geo = pgeo(f, p);
+        dim3 blk(128), grd((g->nx + 127) / 128, g->ny, geo.nzl * f->card);
+        LaunchScope ls(g, g->cs, "k_fill_gen");
+        if (f->dt == NB_F64)
+            k_fill_gen<double><<<grd, blk, 0, g->cs>>>((double *)f->base[p], geo, dense_cs(f, p), f->card,
+                                                        kind, seed, a, b, h);
+        else
+            k_fill_gen<float><<<grd, blk, 0, g->cs>>>((float *)f->base[p], geo, dense_cs(f, p), f->card,
+                                                       kind, seed, a, b, h);
+        NB_TRY(nb_launch_check("k_fill_gen"));
+    }
+    return NB_OK;
+}
+
+// ===========================================================================
+// halo update (PAPER.md L246 haloUpdate, L252 explicit transfers, L256:
+// 2 transfers per component, no marshalling)
+// ===========================================================================
+// Components [c0, c1).  send_up: my last plane -> upper neighbour's low halo;
+// send_down: my first plane -> lower neighbour's high halo.
+nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down,
+                                  cudaStream_t s) {
+    nb_grid *g = f->g;
+    size_t pbytes = (size_t)f->ps * f->esz;
+    bool any_remote = false;
+    for (int p = 0; p < g->nparts; ++p) {
+        if (!g->parts[p].local) continue;
+        const NbPart &q = g->parts[p];
+        for (int c = c0; c < c1; ++c) {
+            if (send_up && q.hi >= 0) {
+                const char *src = f->base[p] + ((int64_t)c * dense_cs(f, p) + (int64_t)q.nz() * f->ps) * f->esz;
+                if (g->parts[q.hi].local) {
+                    char *dst = f->base[q.hi] + ((int64_t)c * dense_cs(f, q.hi)) * f->esz;  // zl = -1
+                    NB_CUDA(cudaMemcpyAsync(dst, src, pbytes, cudaMemcpyDeviceToDevice, s));
+                } else {
+                    any_remote = true;
+                }
+            }
+            if (send_down && q.lo >= 0) {
+                const char *src = f->base[p] + ((int64_t)c * dense_cs(f, p) + f->ps) * f->esz;
+                if (g->parts[q.lo].local) {
+                    int nzn = g->parts[q.lo].nz();
+                    char *dst = f->base[q.lo] + ((int64_t)c * dense_cs(f, q.lo) + (int64_t)(nzn + 1) * f->ps) * f->esz;
+                    NB_CUDA(cudaMemcpyAsync(dst, src, pbytes, cudaMemcpyDeviceToDevice, s));
+                } else {
+                    any_remote = true;
+                }
+            }
+        }
+    }
+    if (!any_remote) return NB_OK;
+    // cross-process transfers: grouped NCCL send/recv over NVLink
+    NB_TRY(nb_nccl_group(g, true));
+    for (int p = 0; p < g->nparts; ++p) {
+        if (!g->parts[p].local) continue;
+        const NbPart &q = g->parts[p];
+        for (int c = c0; c < c1; ++c) {
+            if (q.hi >= 0 && !g->parts[q.hi].local) {
+                int peer = nb_part_owner(g, q.hi);
+                if (send_up) {
+                    const char *src = f->base[p] + ((int64_t)c * dense_cs(f, p) + (int64_t)q.nz() * f->ps) * f->esz;
+                    NB_TRY(nb_nccl_send(g, src, pbytes, peer, s));
+                }
+                if (send_down) {  // the upper neighbour sends me its first plane -> my high halo
+                    char *dst = f->base[p] + ((int64_t)c * dense_cs(f, p) + (int64_t)(q.nz() + 1) * f->ps) * f->esz;
+                    NB_TRY(nb_nccl_recv(g, dst, pbytes, peer, s));
+                }
+            }
+            if (q.lo >= 0 && !g->parts[q.lo].local) {
+                int peer = nb_part_owner(g, q.lo);
+                if (send_down) {
+                    const char *src = f->base[p] + ((int64_t)c * dense_cs(f, p) + f->ps) * f->esz;
+                    NB_TRY(nb_nccl_send(g, src, pbytes, peer, s));
+                }
+                if (send_up) {  // the lower neighbour sends me its last plane -> my low halo
+                    char *dst = f->base[p] + ((int64_t)c * dense_cs(f, p)) * f->esz;
+                    NB_TRY(nb_nccl_recv(g, dst, pbytes, peer, s));
+                }
+            }
+        }
+    }
+    NB_TRY(nb_nccl_group(g, false));
+    return NB_OK;
+}
+
+nb_status nb_sparse_halo_update(nb_field *f);
+
+extern "C" nb_status nb_halo_update(nb_field *f) {
+    if (!f) NB_FAIL(NB_EINVAL, "nb_halo_update: NULL field");
+    DeviceGuard dg(f->g->device);
+    if (f->g->sparse) return nb_sparse_halo_update(f);
+    return nb_halo_exchange_planes(f, 0, f->card, true, true, f->g->cs);
+}
+
+// ===========================================================================
+// map operations (eq. L104): y <- a*x + b*y on plane ranges, 128-bit vectors
+// ===========================================================================
+// The per-element arithmetic is fixed: b == 0: a*x ; b == 1: fma(a, x, y) ;
+// otherwise fma(a, x, b*y).
+template <typename T, int BMODE>
+__device__ __forceinline__ T axpby_cell(T a, T x, T b, T y) {
+    if (BMODE == 0) return a * x;
+    if (BMODE == 1) return fma(a, x, y);
+    return fma(a, x, b * y);
+}
+
+template <typename T, typename V, int BMODE>
+__global__ void __launch_bounds__(256) k_axpby(const T *__restrict__ x, T *__restrict__ y, int64_t nvec,
+                                               T a, T b) {
+    constexpr int W = sizeof(V) / sizeof(T);
+    const V *xv = reinterpret_cast<const V *>(x);
+    V *yv = reinterpret_cast<V *>(y);
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nvec;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        V xi = __ldcs(xv + i);
+        V yi;
+        if (BMODE != 0) yi = __ldcs(yv + i);
+        T *xs = reinterpret_cast<T *>(&xi);
+        T *ys = reinterpret_cast<T *>(&yi);
+        V o;
+        T *os = reinterpret_cast<T *>(&o);
+#pragma unroll
+        for (int k = 0; k < W; ++k) os[k] = axpby_cell<T, BMODE>(a, xs[k], b, BMODE ? ys[k] : T(0));
+        __stcs(yv + i, o);
+    }
+}
+
+// plane ranges [zb, ze) of a view in partition p (dense)
+std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v) {
+    const NbPart &q = g->parts[p];
+    int nz = q.nz();
+    int lo = q.lo >= 0 ? 1 : 0, hi = q.hi >= 0 ? 1 : 0;
+    std::vector<std::pair<int, int>> r;
+    if (v == NB_VIEW_STANDARD) {
+        r.push_back({0, nz});
+    } else if (v == NB_VIEW_INTERNAL) {
+        if (nz - hi > lo) r.push_back({lo, nz - hi});
+    } else {
+        if (lo) r.push_back({0, 1});
+        if (hi && !(lo && nz == 1)) r.push_back({nz - 1, nz});
+    }
+    return r;
+}
+
+static nb_status check_pair(const nb_field *x, const nb_field *y) {
+    if (!x || !y) NB_FAIL(NB_EINVAL, "NULL field");
+    if (x->g != y->g) NB_FAIL(NB_EMISMATCH, "fields belong to different grids");
+    if (x->dt != y->dt || x->card != y->card) NB_FAIL(NB_EMISMATCH, "dtype / cardinality mismatch");
+    return NB_OK;
+}
+
+nb_status nb_sparse_axpby(double a, const nb_field *x, double b, nb_field *y, nb_view v);
+
+template <typename T, typename V>
+static nb_status launch_axpby(nb_grid *g, const T *x, T *y, int64_t n, double a, double b) {
+    if (n <= 0) return NB_OK;
+    constexpr int W = sizeof(V) / sizeof(T);
+    int64_t nvec = n / W;  // plane ranges are multiples of 32 elements
+    int blocks = (int)std::min<int64_t>((nvec + 255) / 256, 148 * 8);
+    LaunchScope ls(g, g->cs, "k_axpby");
+    int mode = (b == 0.0) ? 0 : (b == 1.0 ? 1 : 2);
+    if (mode == 0)
+        k_axpby<T, V, 0><<<blocks, 256, 0, g->cs>>>(x, y, nvec, (T)a, (T)b);
+    else if (mode == 1)
+        k_axpby<T, V, 1><<<blocks, 256, 0, g->cs>>>(x, y, nvec, (T)a, (T)b);
+    else
+        k_axpby<T, V, 2><<<blocks, 256, 0, g->cs>>>(x, y, nvec, (T)a, (T)b);
+    return nb_launch_check("k_axpby");
+}
+
+extern "C" nb_status nb_axpby(double a, const nb_field *x, double b, nb_field *y, nb_view v) {
+    NB_TRY(check_pair(x, y));
+    if (v < NB_VIEW_STANDARD || v > NB_VIEW_BOUNDARY) NB_FAIL(NB_EINVAL, "bad view");
+    nb_grid *g = x->g;
+    DeviceGuard dg(g->device);
+    if (g->sparse) return nb_sparse_axpby(a, x, b, y, v);
+    for (int p = 0; p < g->nparts; ++p) {
+        if (!g->parts[p].local) continue;
+        for (auto rg : view_ranges(g, p, v)) {
+            for (int c = 0; c < x->card; ++c) {
+                int64_t off = (int64_t)c * dense_cs(x, p) + (int64_t)(rg.first + 1) * x->ps;
+                int64_t n = (int64_t)(rg.second - rg.first) * x->ps;
+                if (x->dt == NB_F64)
+                    NB_TRY((launch_axpby<double, double2>(g, (const double *)x->base[p] + off,
+                                                          (double *)y->base[p] + off, n, a, b)));
+                else
+                    NB_TRY((launch_axpby<float, float4>(g, (const float *)x->base[p] + off,
+                                                        (float *)y->base[p] + off, n, a, b)));
+            }
+        }
+    }
+    return NB_OK;
+}
+
+extern "C" nb_status nb_axpy(double a, const nb_field *x, nb_field *y, nb_view v) {
+    return nb_axpby(a, x, 1.0, y, v);
+}
+
+// ===========================================================================
+// reduce (eq. L129): canonical tiles -> plane sums -> total
+// ===========================================================================
+template <typename T>
+__global__ void __launch_bounds__(256) k_dot(const T *__restrict__ x, const T *__restrict__ y, PGeo g,
+                                             int64_t cstride, int zb, int ze, double *tp, int T_tiles) {
+    constexpr int ZC = 16;
+    __shared__ TileStage<ZC> st;
+    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
+    const int nchunk = (ze - zb + ZC - 1) / ZC;
+    const int c = blockIdx.z / nchunk, ch = blockIdx.z % nchunk;
+    const int zs = zb + ch * ZC, zend = min(ze, zs + ZC);
+    const bool valid = xi < g.nx && yi < g.ny;
+    const int64_t o = (int64_t)c * cstride + (int64_t)yi * g.pitch + xi;
+    for (int z = zs; z < zend; ++z) {
+        double v = 0.0;
+        if (valid) {
+            int64_t i = o + (int64_t)(z + 1) * g.ps;
+            v = __dmul_rn((double)__ldcs(x + i), (double)__ldcs(y + i));
+        }
+        tile_stage_put<ZC>(st, z - zs, v);
+    }
+    __syncthreads();
+    tile_stage_flush<ZC>(st, zend - zs, tp, (int64_t)c * g.NZ + g.z0 + zs, T_tiles,
+                         blockIdx.y * gridDim.x + blockIdx.x);
+}
+
+// ---- finalize: plane sums (one CTA per plane) + last-block total ----------
+__device__ void apply_final(int mode, double total, void *state, double *dots, int slot) {
+    if (mode == FIN_STORE) {
+        dots[slot] = total;
+        return;
+    }
+    CgScal *s = (CgScal *)state;
+    if (mode == FIN_CG_INIT) {
+        s->rr = total;
+        s->rr0 = total;
+        s->status = (total == 0.0) ? 2 : 0;
+        s->alpha = 0.0;
+        s->alpha_prev = 0.0;
+        s->beta = 0.0;
+        s->pending = 0;
+        s->iters = 0;
+        return;
+    }
+    if (s->status != 0) return;
+    if (mode == FIN_CG_PQ) {
+        s->pq = total;
+        s->pending = 0;  // phase A applied the deferred x update
+        if (!(total > 0.0))
+            s->status = 3;
+        else
+            s->alpha = s->rr / total;
+    } else if (mode == FIN_CG_RR) {
+        s->beta = total / s->rr;
+        s->rr = total;
+        s->alpha_prev = s->alpha;
+        s->pending = 1;
+        s->iters += 1;
+        if (total == 0.0)
+            s->status = 2;
+        else if (s->rtol2 > 0.0 && total <= s->rtol2 * s->rr0)
+            s->status = 1;
+    }
+}
+
+// blocks: one per plane in [p0, p1) of each component range; planes are
+// indexed c*NZ + z.  If `final_planes` > 0 the last block to finish sums
+// psum[0, final_planes) and applies the mode.
+__global__ void __launch_bounds__(RED_THREADS) k_finalize(const double *tp, int T, double *psum,
+                                                          int NZ, int z0, int zn, int card,
+                                                          unsigned int *counter, int final_planes,
+                                                          int mode, void *state, double *dots,
+                                                          int slot) {
+    __shared__ double sh[RED_THREADS];
+    __shared__ int last;
+    int b = blockIdx.x;
+    int c = b / zn, z = z0 + b % zn;
+    int plane = c * NZ + z;
+    double s = block_tree_sum(tp + (int64_t)plane * T, T, sh);
+    if (threadIdx.x == 0) psum[plane] = s;
+    if (final_planes <= 0) return;
+    __threadfence();
+    if (threadIdx.x == 0) {
+        unsigned int t = atomicAdd(counter, 1u);
+        last = (t == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    // canonical tree over all planes (volatile-free: psum written by other
+    // blocks before their fence + atomic; read through L2)
+    const int t = threadIdx.x;
+    double acc = 0.0;
+    for (int i = t; i < final_planes; i += RED_THREADS) acc = __dadd_rn(acc, __ldcg(psum + i));
+    sh[t] = acc;
+    __syncthreads();
+    for (int k = RED_THREADS / 2; k > 0; k >>= 1) {
+        if (t < k) sh[t] = __dadd_rn(sh[t], sh[t + k]);
+        __syncthreads();
+    }
+    if (t == 0) {
+        *counter = 0u;
+        apply_final(mode, sh[0], state, dots, slot);
+    }
+}
+
+__global__ void __launch_bounds__(RED_THREADS) k_final_only(const double *psum, int planes, int mode,
+                                                            void *state, double *dots, int slot) {
+    __shared__ double sh[RED_THREADS];
+    double s = block_tree_sum(psum, planes, sh);
+    if (threadIdx.x == 0) apply_final(mode, s, state, dots, slot);
+}
+
+// Reduce the tile partials of `card` components (planes c*NZ + z) into the
+// final value.  Single process: one launch (plane sums + last-block total).
+// Multi-process: local plane sums -> NCCL all-reduce of the (disjoint,
+// zero-padded) plane-sum vector -> fixed-order total on every rank.
+nb_status nb_reduce_finalize(nb_grid *g, int card, int mode, void *state, int slot) {
+    int planes = card * g->nz;
+    cudaStream_t s = g->cs;
+    bool dist = g->comm && g->comm->world > 1;
+    if (!dist) {
+        LaunchScope ls(g, s, "k_finalize");
+        k_finalize<<<planes, RED_THREADS, 0, s>>>(g->tp, g->T, g->psum, g->nz, 0, g->nz, card, g->counter,
+                                                  planes, mode, state, g->dots, slot);
+        return nb_launch_check("k_finalize");
+    }
+    int z0 = g->parts[g->first_local].z0, z1 = g->parts[g->first_local + g->nlocal - 1].z1;
+    {
+        LaunchScope ls(g, s, "k_finalize");
+        k_finalize<<<card * (z1 - z0), RED_THREADS, 0, s>>>(g->tp, g->T, g->psum_send, g->nz, z0, z1 - z0,
+                                                            card, g->counter, 0, mode, state, g->dots, slot);
+        NB_TRY(nb_launch_check("k_finalize"));
+    }
+    NB_TRY(nb_nccl_allreduce_sum(g, g->psum_send, g->psum, planes, s));
+    LaunchScope ls(g, s, "k_final_only");
+    k_final_only<<<1, RED_THREADS, 0, s>>>(g->psum, planes, mode, state, g->dots, slot);
+    return nb_launch_check("k_final_only");
+}
+
+nb_status nb_sparse_dot_partials(const nb_field *x, const nb_field *y);
+
+nb_status nb_dot_partials(const nb_field *x, const nb_field *y) {
+    nb_grid *g = x->g;
+    if (g->sparse) return nb_sparse_dot_partials(x, y);
+    for (int p = 0; p < g->nparts; ++p) {
+        if (!g->parts[p].local) continue;
+        PGeo geo = pgeo(x, p);
+        int nchunk = (geo.nzl + 15) / 16;
+        dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, nchunk * x->card);
+        LaunchScope ls(g, g->cs, "k_dot");
+        if (x->dt == NB_F64)
+            k_dot<double><<<grd, blk, 0, g->cs>>>((const double *)x->base[p], (const double *)y->base[p], geo,
+                                                   dense_cs(x, p), 0, geo.nzl, g->tp, g->T);
+        else
+            k_dot<float><<<grd, blk, 0, g->cs>>>((const float *)x->base[p], (const float *)y->base[p], geo,
+                                                  dense_cs(x, p), 0, geo.nzl, g->tp, g->T);
+        NB_TRY(nb_launch_check("k_dot"));
+    }
+    return NB_OK;
+}
+
+extern "C" nb_status nb_dot(const nb_field *x, const nb_field *y, double *host_out) {
+    NB_TRY(check_pair(x, y));
+    if (!host_out) NB_FAIL(NB_EINVAL, "nb_dot: host_out is NULL");
+    nb_grid *g = x->g;
+    if (x->card > g->max_card) NB_FAIL(NB_EUNSUPPORTED, "nb_dot: cardinality > %d", g->max_card);
+    DeviceGuard dg(g->device);
+    NB_TRY(nb_dot_partials(x, y));
+    NB_TRY(nb_reduce_finalize(g, x->card, FIN_STORE, nullptr, 0));
+    NB_CUDA(cudaMemcpyAsync(host_out, g->dots, sizeof(double), cudaMemcpyDeviceToHost, g->cs));
+    NB_CUDA(cudaStreamSynchronize(g->cs));
+    return NB_OK;
+}
+
+// ===========================================================================
+// measurement
+// ===========================================================================
+extern "C" nb_status nb_profile_enable(nb_grid *g, int32_t enable) {
+    if (!g) NB_FAIL(NB_EINVAL, "NULL grid");
+    if (enable) {  // start a fresh record
+        DeviceGuard dg(g->device);
+        cudaStreamSynchronize(g->cs);
+        for (auto &r : g->prof) {
+            cudaEventDestroy(r.a);
+            cudaEventDestroy(r.b);
+        }
+        g->prof.clear();
+    }
+    g->profiling = enable != 0;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_profile_read(nb_grid *g, const char *name, int64_t *launches, double *total_ms) {
+    if (!g || !name) NB_FAIL(NB_EINVAL, "NULL argument");
+    DeviceGuard dg(g->device);
+    NB_CUDA(cudaStreamSynchronize(g->cs));
+    NB_CUDA(cudaStreamSynchronize(g->hs));
+    int64_t n = 0;
+    double ms = 0.0;
+    for (auto &r : g->prof) {
+        if (!strstr(r.name, name)) continue;
+        float t = 0.f;
+        NB_CUDA(cudaEventElapsedTime(&t, r.a, r.b));
+        ms += t;
+        ++n;
+    }
+    if (launches) *launches = n;
+    if (total_ms) *total_ms = ms;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_launch_count(const nb_grid *g, int64_t *count) {
+    if (!g || !count) NB_FAIL(NB_EINVAL, "NULL argument");
+    *count = g->launches;
+    return NB_OK;
+}

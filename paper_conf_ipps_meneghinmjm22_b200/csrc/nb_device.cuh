@@ -1,0 +1,64 @@
+// nb_device.cuh — device helpers shared by the kernels of libnb.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+
+#include "nb_internal.cuh"
+
+// xor-butterfly warp sum (offsets 16, 8, 4, 2, 1).  IEEE addition is
+// commutative, so every lane ends with the same bits: the value is a fixed
+// function of the 32 inputs.
+__device__ __forceinline__ double warp_sum_canon(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v = __dadd_rn(v, __shfl_xor_sync(0xffffffffu, v, o));
+    return v;
+}
+
+// Canonical block tree over n values v[0..n) (stride `stride`) computed by a
+// block of RED_THREADS threads: thread t sums v[t], v[t+256], ... in order,
+// then a fixed halving tree.  Must be called by all RED_THREADS threads;
+// `sh` is RED_THREADS doubles of shared memory.  Returns the sum in all
+// threads.
+__device__ __forceinline__ double block_tree_sum(const double *v, int64_t n, double *sh) {
+    const int t = threadIdx.x;
+    double acc = 0.0;
+    for (int64_t i = t; i < n; i += RED_THREADS) acc = __dadd_rn(acc, v[i]);
+    sh[t] = acc;
+    __syncthreads();
+#pragma unroll
+    for (int s = RED_THREADS / 2; s > 0; s >>= 1) {
+        if (t < s) sh[t] = __dadd_rn(sh[t], sh[t + s]);
+        __syncthreads();
+    }
+    double r = sh[0];
+    __syncthreads();
+    return r;
+}
+
+// Per-chunk tile-partial staging for z-march kernels with blockDim
+// (DOT_TX, DOT_TY): warp w = threadIdx.y owns one x-row of the tile.
+// After the chunk, tile value = ((w0 + w1) + w2) + ... + w7 per plane.
+template <int ZC>
+struct TileStage {
+    double w[ZC][DOT_TY];
+};
+
+template <int ZC>
+__device__ __forceinline__ void tile_stage_put(TileStage<ZC> &st, int zi, double v) {
+    v = warp_sum_canon(v);
+    if (threadIdx.x == 0) st.w[zi][threadIdx.y] = v;
+}
+
+// write the tile partials of planes [0, nplanes) of the chunk; plane index in
+// the global tile-partial array = pbase + zi.  Call after __syncthreads().
+template <int ZC>
+__device__ __forceinline__ void tile_stage_flush(const TileStage<ZC> &st, int nplanes,
+                                                 double *tp, int64_t pbase, int T, int tile) {
+    int t = threadIdx.y * DOT_TX + threadIdx.x;
+    if (t < nplanes) {
+        double s = st.w[t][0];
+#pragma unroll
+        for (int w = 1; w < DOT_TY; ++w) s = __dadd_rn(s, st.w[t][w]);
+        tp[(pbase + t) * (int64_t)T + tile] = s;
+    }
+}

@@ -1,0 +1,226 @@
+// nb_internal.cuh — shared internals of libnb (B200 / sm_100a).
+//
+// Everything here is product code; nothing is shared with oracle/.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <string>
+#include <vector>
+
+#include "nb.h"
+
+// ---------------------------------------------------------------------------
+// error plumbing (no exception crosses the ABI)
+// ---------------------------------------------------------------------------
+void nb_set_error(const char *fmt, ...);
+
+#define NB_FAIL(code, ...)            \
+    do {                              \
+        nb_set_error(__VA_ARGS__);    \
+        return (code);                \
+    } while (0)
+
+#define NB_CUDA(call)                                                                     \
+    do {                                                                                  \
+        cudaError_t _e = (call);                                                          \
+        if (_e != cudaSuccess)                                                            \
+            NB_FAIL(NB_ECUDA, "%s failed: %s (%s:%d)", #call, cudaGetErrorString(_e),     \
+                    __FILE__, __LINE__);                                                  \
+    } while (0)
+
+#define NB_TRY(call)                      \
+    do {                                  \
+        nb_status _s = (call);            \
+        if (_s != NB_OK) return _s;       \
+    } while (0)
+
+// ---------------------------------------------------------------------------
+// canonical dot tiling: every plane
+// (c, z) is cut into DOT_TX x DOT_TY tiles; inside a tile each warp owns one
+// x-row (lane = x), reduced by the xor-butterfly 16,8,4,2,1; the 8 warp
+// values are added in increasing y; tiles of a plane and then planes are
+// added by the fixed 256-wide block tree of nb_tree_sum.  Nothing depends on
+// the partition count or on which kernel produced the tile value.
+// ---------------------------------------------------------------------------
+constexpr int DOT_TX = 32;
+constexpr int DOT_TY = 8;
+constexpr int RED_THREADS = 256;
+
+// LBM lattice size
+constexpr int Q19 = 19;
+
+struct nb_comm {
+    int world = 1, rank = 0, device = 0;
+    void *nccl = nullptr;  // ncclComm_t
+};
+
+struct NbPart {
+    int device = 0;
+    int local = 1;
+    int z0 = 0, z1 = 0;  // global planes [z0, z1)
+    int lo = -1, hi = -1;  // neighbour partition across the low / high z face (-1: none)
+    // element-sparse grids
+    int64_t n_act = 0;       // active cells in the partition
+    int64_t a0 = 0;          // global compact index of its first active cell
+    int64_t n_lo_bnd = 0;    // active cells on the partition's first plane
+    int64_t n_hi_bnd = 0;    // active cells on the partition's last plane
+    int64_t halo_lo = 0;     // cells in the low halo (= previous part's last plane)
+    int64_t halo_hi = 0;     // cells in the high halo (= next part's first plane)
+    int nz() const { return z1 - z0; }
+};
+
+struct ProfRec {
+    const char *name;
+    cudaEvent_t a, b;
+};
+
+// sparse partition device data (element-sparse grid)
+struct NbSparsePart {
+    int32_t *conn = nullptr;     // [6][n_act] neighbour local slot (incl. halo), -1 = outside
+    int32_t *coord = nullptr;    // [n_act] packed (x | y<<16), local plane id in plane_of
+    int32_t *plane_of = nullptr; // [n_act] local plane zl
+    int64_t *plane_start = nullptr;  // host copy: [nz+1] local slot offsets per plane
+    std::vector<int64_t> h_plane_start;
+    int32_t *tile_of = nullptr;  // [n_act] canonical dot tile id within (c, z)
+};
+
+struct nb_grid {
+    int nx = 0, ny = 0, nz = 0;
+    int nparts = 1;
+    std::vector<NbPart> parts;
+    int first_local = 0, nlocal = 0;
+    nb_comm *comm = nullptr;
+    int device = 0;
+    bool sparse = false;
+    cudaStream_t cs = nullptr, hs = nullptr;
+    bool own_cs = false, own_hs = false;
+    // deterministic reduction scratch
+    int tiles_x = 0, tiles_y = 0, T = 0;  // dot tiles per plane
+    int max_card = 3;
+    double *tp = nullptr;         // [max_card*nz][T] tile partials
+    double *psum = nullptr;       // [max_card*nz] plane sums
+    double *psum_send = nullptr;  // [max_card*nz] (multi-process)
+    double *dots = nullptr;       // [NB_DOT_SLOTS] reduce results
+    unsigned int *counter = nullptr;
+    int nfields = 0, nsolvers = 0;
+    bool profiling = false;
+    std::vector<ProfRec> prof;
+    int64_t launches = 0;
+    // element-sparse
+    std::vector<NbSparsePart> sp;
+    std::vector<int64_t> plane_count;  // [nz] active per global plane
+};
+
+constexpr int NB_DOT_SLOTS = 1024;
+
+struct nb_field {
+    nb_grid *g = nullptr;
+    nb_dtype dt = NB_F64;
+    int card = 1;
+    double outside = 0.0;
+    size_t esz = 8;
+    int64_t pitch = 0, ps = 0, cs = 0;  // elements: row pitch, plane stride, component stride
+    std::vector<char *> base;          // per partition (local only)
+    std::vector<size_t> bytes;
+};
+
+// per-partition geometry handed to kernels (dense)
+struct PGeo {
+    int nx, ny, nzl;  // nzl: planes of the partition
+    int z0, NZ;       // first global plane, global plane count
+    int64_t pitch, ps;
+};
+
+inline PGeo pgeo(const nb_field *f, int g) {
+    const NbPart &p = f->g->parts[g];
+    PGeo r;
+    r.nx = f->g->nx;
+    r.ny = f->g->ny;
+    r.nzl = p.nz();
+    r.z0 = p.z0;
+    r.NZ = f->g->nz;
+    r.pitch = f->pitch;
+    r.ps = f->ps;
+    return r;
+}
+
+// pointer to plane zl (may be -1 or nzl: halo) of component c of partition g
+template <typename T>
+inline T *plane_ptr(const nb_field *f, int g, int c, int zl) {
+    return reinterpret_cast<T *>(f->base[g]) + (int64_t)c * f->cs + (int64_t)(zl + 1) * f->ps;
+}
+
+// ---------------------------------------------------------------------------
+// launch bookkeeping: profiling events + launch counter
+// ---------------------------------------------------------------------------
+struct LaunchScope {
+    nb_grid *g;
+    cudaStream_t s;
+    const char *name;
+    cudaEvent_t a = nullptr, b = nullptr;
+    LaunchScope(nb_grid *g_, cudaStream_t s_, const char *n) : g(g_), s(s_), name(n) {
+        g->launches++;
+        if (g->profiling) {
+            cudaEventCreate(&a);
+            cudaEventCreate(&b);
+            cudaEventRecord(a, s);
+        }
+    }
+    ~LaunchScope() {
+        if (g->profiling) {
+            cudaEventRecord(b, s);
+            g->prof.push_back({name, a, b});
+        }
+    }
+};
+
+// kernels / helpers implemented in the .cu files
+nb_status nb_launch_check(const char *what);
+nb_status nb_reduce_finalize(nb_grid *g, int planes, int mode, void *state, int slot);
+
+// finalize modes
+enum {
+    FIN_STORE = 0,    // dots[slot] = total
+    FIN_CG_INIT = 1,  // rr = rr0 = total
+    FIN_CG_PQ = 2,    // alpha = rr / total
+    FIN_CG_RR = 3,    // beta = total / rr ...
+};
+
+struct CgScal {
+    double rr, rr0, alpha, alpha_prev, beta, pq, rtol2;
+    int32_t iters, status, pending, pad;
+};
+
+// halo helpers (nb_api.cu)
+nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down,
+                                  cudaStream_t s);
+nb_status nb_nccl_allreduce_sum(nb_grid *g, const double *send, double *recv, size_t n,
+                                cudaStream_t s);
+nb_status nb_nccl_group(nb_grid *g, bool start);
+nb_status nb_nccl_send(nb_grid *g, const void *buf, size_t bytes, int peer, cudaStream_t s);
+nb_status nb_nccl_recv(nb_grid *g, void *buf, size_t bytes, int peer, cudaStream_t s);
+
+int nb_part_owner(const nb_grid *g, int part);
+
+// halo overlap events of a schedule (multi-process)
+struct HaloSync {
+    cudaEvent_t eb = nullptr, eh = nullptr;
+};
+
+#include <map>
+struct nb_cg {
+    nb_grid *g = nullptr;
+    nb_field *x = nullptr;
+    const nb_field *b = nullptr;
+    nb_field *r = nullptr, *p[2] = {nullptr, nullptr}, *q = nullptr;
+    CgScal *sc = nullptr;
+    nb_cg_params prm{};
+    int64_t k = 0;  // iterations enqueued
+    std::map<std::pair<int, int>, std::pair<cudaGraphExec_t, int64_t>> graphs;  // (count, parity) -> graph, kernels
+    HaloSync hs;
+    bool finished = false;
+};
+

@@ -1,0 +1,358 @@
+// nb_lbm.cu — D3Q19 BGK lattice Boltzmann, twoPop pull scheme, fused
+// collide-and-stream (§VI-A: "Collide and streaming steps
+// are fused into a single kernel", twoPop "works on two buffers ... swapped").
+//
+// Per cell (the formulas are the SURVEY.md §8(c) c6 reading):
+//   f_i = fin_i(x - c_i)                 (pull: own-compute rule, L246)
+//       | fin_opp(i)(x) + 6 w_i rho_w (c_i . u_lid)[lid]   (half-way bounce-back)
+//   rho = sum f_i ; u = sum c_i f_i / rho
+//   feq_i = w_i rho (1 + 3 c.u + 4.5 (c.u)^2 - 1.5 |u|^2)
+//   fout_i(x) = f_i - omega (f_i - feq_i)
+// fp32 storage and arithmetic, SoA [c][zl][y][x].  Algorithmic traffic
+// 19 loads + 19 stores of 4 B = 152 B per cell per step.
+//
+// Velocity order (halo-contiguous): 0 rest; 1-4 (+-x, +-y); 5-8 xy diagonals;
+// 9-13 c_z = +1; 14-18 c_z = -1.
+#include <algorithm>
+
+#include "nb_device.cuh"
+#include "nb_internal.cuh"
+
+namespace {
+__device__ __host__ constexpr int CXv(int i) {
+    constexpr int t[19] = {0, 1, -1, 0, 0, 1, -1, 1, -1, 0, 1, -1, 0, 0, 0, -1, 1, 0, 0};
+    return t[i];
+}
+__device__ __host__ constexpr int CYv(int i) {
+    constexpr int t[19] = {0, 0, 0, 1, -1, 1, -1, -1, 1, 0, 0, 0, 1, -1, 0, 0, 0, -1, 1};
+    return t[i];
+}
+__device__ __host__ constexpr int CZv(int i) {
+    constexpr int t[19] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 1, 1, 1, 1, 1, -1, -1, -1, -1, -1};
+    return t[i];
+}
+__device__ __host__ constexpr int OPPv(int i) {
+    constexpr int t[19] = {0, 2, 1, 4, 3, 6, 5, 8, 7, 14, 15, 16, 17, 18, 9, 10, 11, 12, 13};
+    return t[i];
+}
+__device__ __host__ constexpr float Wv(int i) {
+    return i == 0 ? 1.0f / 3.0f : (CXv(i) * CXv(i) + CYv(i) * CYv(i) + CZv(i) * CZv(i) == 1 ? 1.0f / 18.0f : 1.0f / 36.0f);
+}
+}  // namespace
+
+struct LbmArgs {
+    const float *fin;
+    float *fout;
+    PGeo g;
+    int64_t cs;          // component stride of this partition
+    float omega, ulid, rho_w;
+    int periodic;
+    float *rem_lo;       // lower neighbour's fout, component 0, plane zl = nz_lo (its high halo)
+    int64_t rem_lo_cs;
+    float *rem_hi;       // upper neighbour's fout, component 0, plane zl = -1 (its low halo)
+    int64_t rem_hi_cs;
+};
+
+template <bool PERIODIC>
+__global__ void __launch_bounds__(128) k_lbm_d3q19(LbmArgs A, int zb) {
+    const int x = blockIdx.x * blockDim.x + threadIdx.x;
+    const int y = blockIdx.y;
+    const int zl = zb + blockIdx.z;
+    const PGeo &g = A.g;
+    if (x >= g.nx) return;
+    const int gz = g.z0 + zl;
+    const int64_t cell = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+    float f[Q19];
+#pragma unroll
+    for (int i = 0; i < Q19; ++i) {
+        int sx = x - CXv(i), sy = y - CYv(i), szl = zl - CZv(i);
+        if (PERIODIC) {
+            sx = sx < 0 ? sx + g.nx : (sx >= g.nx ? sx - g.nx : sx);
+            sy = sy < 0 ? sy + g.ny : (sy >= g.ny ? sy - g.ny : sy);
+            f[i] = __ldg(A.fin + (int64_t)i * A.cs + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx);
+        } else {
+            const int sgz = gz - CZv(i);
+            const bool inside = sx >= 0 && sx < g.nx && sy >= 0 && sy < g.ny && sgz >= 0 && sgz < g.NZ;
+            if (inside) {
+                f[i] = __ldg(A.fin + (int64_t)i * A.cs + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx);
+            } else {
+                float v = __ldg(A.fin + (int64_t)OPPv(i) * A.cs + cell);
+                if (CXv(i) != 0 && sy == g.ny && sx >= 0 && sx < g.nx && sgz >= 0 && sgz < g.NZ)
+                    v = v + 6.0f * Wv(i) * A.rho_w * ((float)CXv(i) * A.ulid);
+                f[i] = v;
+            }
+        }
+    }
+    float rho = 0.f, jx = 0.f, jy = 0.f, jz = 0.f;
+#pragma unroll
+    for (int i = 0; i < Q19; ++i) {
+        rho += f[i];
+        if (CXv(i) == 1) jx += f[i];
+        if (CXv(i) == -1) jx -= f[i];
+        if (CYv(i) == 1) jy += f[i];
+        if (CYv(i) == -1) jy -= f[i];
+        if (CZv(i) == 1) jz += f[i];
+        if (CZv(i) == -1) jz -= f[i];
+    }
+    const float ux = jx / rho, uy = jy / rho, uz = jz / rho;
+    const float usq = ux * ux + uy * uy + uz * uz;
+    const float om = A.omega;
+    float o[Q19];
+#pragma unroll
+    for (int i = 0; i < Q19; ++i) {
+        float cu = (float)CXv(i) * ux + (float)CYv(i) * uy + (float)CZv(i) * uz;
+        float feq = Wv(i) * rho * (1.0f + 3.0f * cu + 4.5f * cu * cu - 1.5f * usq);
+        o[i] = f[i] - om * (f[i] - feq);
+        __stcs(A.fout + (int64_t)i * A.cs + cell, o[i]);
+    }
+    // halo transfer fused into the producing kernel: outgoing populations
+    // of the boundary planes go straight into the neighbours' halo planes
+    const int64_t row = (int64_t)y * g.pitch + x;
+    if (zl == 0 && A.rem_lo) {
+#pragma unroll
+        for (int i = 14; i < 19; ++i) A.rem_lo[(int64_t)i * A.rem_lo_cs + row] = o[i];
+    }
+    if (zl == g.nzl - 1 && A.rem_hi) {
+#pragma unroll
+        for (int i = 9; i < 14; ++i) A.rem_hi[(int64_t)i * A.rem_hi_cs + row] = o[i];
+    }
+}
+
+__global__ void __launch_bounds__(128) k_lbm_init(float *f, PGeo g, int64_t cs, float rho, float ux, float uy,
+                                                  float uz) {
+    const int x = blockIdx.x * blockDim.x + threadIdx.x, y = blockIdx.y, zl = (int)blockIdx.z - 1;
+    if (x >= g.nx) return;
+    const int64_t cell = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+    const float usq = ux * ux + uy * uy + uz * uz;
+#pragma unroll
+    for (int i = 0; i < Q19; ++i) {
+        float cu = (float)CXv(i) * ux + (float)CYv(i) * uy + (float)CZv(i) * uz;
+        f[(int64_t)i * cs + cell] = Wv(i) * rho * (1.0f + 3.0f * cu + 4.5f * cu * cu - 1.5f * usq);
+    }
+}
+
+__global__ void __launch_bounds__(128) k_lbm_macro(const float *f, float *rho_o, float *u_o, PGeo g, int64_t cs,
+                                                   int64_t cs_rho, int64_t cs_u) {
+    const int x = blockIdx.x * blockDim.x + threadIdx.x, y = blockIdx.y, zl = blockIdx.z;
+    if (x >= g.nx) return;
+    const int64_t cell = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+    float rho = 0.f, jx = 0.f, jy = 0.f, jz = 0.f;
+#pragma unroll
+    for (int i = 0; i < Q19; ++i) {
+        float v = f[(int64_t)i * cs + cell];
+        rho += v;
+        jx += (float)CXv(i) * v;
+        jy += (float)CYv(i) * v;
+        jz += (float)CZv(i) * v;
+    }
+    (void)cs_rho;
+    rho_o[cell] = rho;
+    u_o[cell] = jx / rho;
+    u_o[cs_u + cell] = jy / rho;
+    u_o[2 * cs_u + cell] = jz / rho;
+}
+
+static inline int64_t lcs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
+
+static nb_status lbm_check(const nb_field *f) {
+    if (!f) NB_FAIL(NB_EINVAL, "NULL field");
+    if (f->dt != NB_F32 || f->card != Q19) NB_FAIL(NB_EMISMATCH, "LBM needs an fp32 field of cardinality 19");
+    if (f->g->sparse) NB_FAIL(NB_EUNSUPPORTED, "LBM on element-sparse grids is not built yet (SURVEY f2)");
+    return NB_OK;
+}
+
+extern "C" nb_status nb_lbm_init(nb_field *f, double rho0, const double u0[3]) {
+    NB_TRY(lbm_check(f));
+    if (!u0) NB_FAIL(NB_EINVAL, "u0 is NULL");
+    nb_grid *g = f->g;
+    cudaSetDevice(g->device);
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        PGeo geo = pgeo(f, p);
+        dim3 blk(128), grd((g->nx + 127) / 128, g->ny, geo.nzl + 2);  // halo planes too
+        LaunchScope ls(g, g->cs, "k_lbm_init");
+        k_lbm_init<<<grd, blk, 0, g->cs>>>((float *)f->base[p], geo, lcs(f, p), (float)rho0, (float)u0[0],
+                                           (float)u0[1], (float)u0[2]);
+        NB_TRY(nb_launch_check("k_lbm_init"));
+    }
+    return NB_OK;
+}
+
+// neighbours for the LBM (ring when periodic)
+static int lbm_lo(const nb_grid *g, int p, bool per) {
+    if (g->parts[p].lo >= 0) return g->parts[p].lo;
+    return per ? g->nparts - 1 : -1;
+}
+static int lbm_hi(const nb_grid *g, int p, bool per) {
+    if (g->parts[p].hi >= 0) return g->parts[p].hi;
+    return per ? 0 : -1;
+}
+
+// Halo of the 10 populations that cross z faces: my last plane's c_z=+1
+// populations (9..13) -> upper neighbour's low halo; my first plane's c_z=-1
+// populations (14..18) -> lower neighbour's high halo.  Local partners:
+// device copies; remote partners: grouped NCCL send/recv.
+static nb_status lbm_halo(nb_field *f, bool per, cudaStream_t s) {
+    nb_grid *g = f->g;
+    size_t pb = (size_t)f->ps * 4;
+    bool remote = false;
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        int hi = lbm_hi(g, p, per), lo = lbm_lo(g, p, per);
+        int nz = g->parts[p].nz();
+        float *b = (float *)f->base[p];
+        if (hi >= 0) {
+            if (g->parts[hi].local) {
+                float *d = (float *)f->base[hi];
+                for (int i = 9; i < 14; ++i)
+                    NB_CUDA(cudaMemcpyAsync(d + i * lcs(f, hi), b + i * lcs(f, p) + (int64_t)nz * f->ps, pb,
+                                            cudaMemcpyDeviceToDevice, s));
+            } else {
+                remote = true;
+            }
+        }
+        if (lo >= 0) {
+            if (g->parts[lo].local) {
+                float *d = (float *)f->base[lo];
+                int nzl = g->parts[lo].nz();
+                for (int i = 14; i < 19; ++i)
+                    NB_CUDA(cudaMemcpyAsync(d + i * lcs(f, lo) + (int64_t)(nzl + 1) * f->ps, b + i * lcs(f, p) + f->ps,
+                                            pb, cudaMemcpyDeviceToDevice, s));
+            } else {
+                remote = true;
+            }
+        }
+    }
+    if (!remote) return NB_OK;
+    NB_TRY(nb_nccl_group(g, true));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        int hi = lbm_hi(g, p, per), lo = lbm_lo(g, p, per);
+        int nz = g->parts[p].nz();
+        float *b = (float *)f->base[p];
+        if (hi >= 0 && !g->parts[hi].local) {
+            int peer = nb_part_owner(g, hi);
+            for (int i = 9; i < 14; ++i) NB_TRY(nb_nccl_send(g, b + i * lcs(f, p) + (int64_t)nz * f->ps, pb, peer, s));
+            for (int i = 14; i < 19; ++i)
+                NB_TRY(nb_nccl_recv(g, b + i * lcs(f, p) + (int64_t)(nz + 1) * f->ps, pb, peer, s));
+        }
+        if (lo >= 0 && !g->parts[lo].local) {
+            int peer = nb_part_owner(g, lo);
+            for (int i = 14; i < 19; ++i) NB_TRY(nb_nccl_send(g, b + i * lcs(f, p) + f->ps, pb, peer, s));
+            for (int i = 9; i < 14; ++i) NB_TRY(nb_nccl_recv(g, b + i * lcs(f, p), pb, peer, s));
+        }
+    }
+    NB_TRY(nb_nccl_group(g, false));
+    return NB_OK;
+}
+
+static nb_status launch_lbm(nb_grid *g, int p, nb_field *fin, nb_field *fout, const nb_lbm_params *prm, int zb,
+                            int ze, bool remote_stores) {
+    if (ze <= zb) return NB_OK;
+    bool per = prm->bc == NB_LBM_PERIODIC;
+    LbmArgs A;
+    A.fin = (const float *)fin->base[p];
+    A.fout = (float *)fout->base[p];
+    A.g = pgeo(fin, p);
+    A.cs = lcs(fin, p);
+    A.omega = (float)prm->omega;
+    A.ulid = (float)prm->u_lid;
+    A.rho_w = (float)prm->rho_w;
+    A.periodic = per;
+    A.rem_lo = A.rem_hi = nullptr;
+    A.rem_lo_cs = A.rem_hi_cs = 0;
+    if (remote_stores) {
+        int lo = lbm_lo(g, p, per), hi = lbm_hi(g, p, per);
+        if (zb == 0 && lo >= 0 && g->parts[lo].local) {
+            A.rem_lo = (float *)fout->base[lo] + (int64_t)(g->parts[lo].nz() + 1) * fout->ps;
+            A.rem_lo_cs = lcs(fout, lo);
+        }
+        if (ze == g->parts[p].nz() && hi >= 0 && g->parts[hi].local) {
+            A.rem_hi = (float *)fout->base[hi];
+            A.rem_hi_cs = lcs(fout, hi);
+        }
+    }
+    dim3 blk(128), grd((g->nx + 127) / 128, g->ny, ze - zb);
+    LaunchScope ls(g, g->cs, "k_lbm_d3q19");
+    if (per)
+        k_lbm_d3q19<true><<<grd, blk, 0, g->cs>>>(A, zb);
+    else
+        k_lbm_d3q19<false><<<grd, blk, 0, g->cs>>>(A, zb);
+    return nb_launch_check("k_lbm_d3q19");
+}
+
+extern "C" nb_status nb_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm_params *prm, int32_t nsteps,
+                                 nb_occ occ) {
+    if (!pfin || !pfout || !prm) NB_FAIL(NB_EINVAL, "nb_lbm_step: NULL argument");
+    nb_field *fin = *pfin, *fout = *pfout;
+    NB_TRY(lbm_check(fin));
+    NB_TRY(lbm_check(fout));
+    if (fin->g != fout->g) NB_FAIL(NB_EMISMATCH, "fin and fout belong to different grids");
+    if (fin == fout) NB_FAIL(NB_EINVAL, "twoPop needs two distinct buffers");
+    if (nsteps < 0) NB_FAIL(NB_EINVAL, "nsteps < 0");
+    if (prm->bc != NB_LBM_CAVITY && prm->bc != NB_LBM_PERIODIC) NB_FAIL(NB_EINVAL, "bad bc");
+    nb_grid *g = fin->g;
+    cudaSetDevice(g->device);
+    const bool per = prm->bc == NB_LBM_PERIODIC;
+    const bool dist = g->comm && g->comm->world > 1;
+    // make fin's halos current (covers states written by upload/init)
+    NB_TRY(lbm_halo(fin, per, g->cs));
+    HaloSync hs;
+    if (dist) {
+        NB_CUDA(cudaEventCreateWithFlags(&hs.eb, cudaEventDisableTiming));
+        NB_CUDA(cudaEventCreateWithFlags(&hs.eh, cudaEventDisableTiming));
+    }
+    nb_status st = NB_OK;
+    for (int t = 0; t < nsteps && st == NB_OK; ++t) {
+        // boundary planes first (their outputs are the next step's halos)
+        for (int p = g->first_local; p < g->first_local + g->nlocal && st == NB_OK; ++p) {
+            int nz = g->parts[p].nz();
+            bool blo = lbm_lo(g, p, per) >= 0, bhi = lbm_hi(g, p, per) >= 0;
+            if (occ == NB_OCC_NONE || (!blo && !bhi)) {
+                st = launch_lbm(g, p, fin, fout, prm, 0, nz, true);
+            } else {
+                if (blo) st = launch_lbm(g, p, fin, fout, prm, 0, 1, true);
+                if (st == NB_OK && bhi && !(blo && nz == 1)) st = launch_lbm(g, p, fin, fout, prm, nz - 1, nz, true);
+            }
+        }
+        if (st != NB_OK) break;
+        if (dist) {  // remote halos on the halo stream, overlapped with the interior
+            cudaEventRecord(hs.eb, g->cs);
+            cudaStreamWaitEvent(g->hs, hs.eb, 0);
+            st = lbm_halo(fout, per, g->hs);
+            cudaEventRecord(hs.eh, g->hs);
+            if (occ == NB_OCC_NONE) cudaStreamWaitEvent(g->cs, hs.eh, 0);
+        }
+        for (int p = g->first_local; p < g->first_local + g->nlocal && st == NB_OK; ++p) {
+            int nz = g->parts[p].nz();
+            bool blo = lbm_lo(g, p, per) >= 0, bhi = lbm_hi(g, p, per) >= 0;
+            if (occ == NB_OCC_NONE || (!blo && !bhi)) continue;
+            st = launch_lbm(g, p, fin, fout, prm, blo ? 1 : 0, bhi ? nz - 1 : nz, false);
+        }
+        if (dist && occ != NB_OCC_NONE) cudaStreamWaitEvent(g->cs, hs.eh, 0);
+        std::swap(fin, fout);
+    }
+    if (hs.eb) {
+        cudaEventDestroy(hs.eb);
+        cudaEventDestroy(hs.eh);
+    }
+    *pfin = fin;
+    *pfout = fout;
+    return st;
+}
+
+extern "C" nb_status nb_lbm_macroscopic(const nb_field *f, nb_field *rho, nb_field *u) {
+    NB_TRY(lbm_check(f));
+    if (!rho || !u) NB_FAIL(NB_EINVAL, "NULL field");
+    if (rho->g != f->g || u->g != f->g) NB_FAIL(NB_EMISMATCH, "fields belong to different grids");
+    if (rho->dt != NB_F32 || u->dt != NB_F32 || rho->card != 1 || u->card != 3)
+        NB_FAIL(NB_EMISMATCH, "rho: fp32 card 1, u: fp32 card 3");
+    nb_grid *g = f->g;
+    cudaSetDevice(g->device);
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        PGeo geo = pgeo(f, p);
+        dim3 blk(128), grd((g->nx + 127) / 128, g->ny, geo.nzl);
+        LaunchScope ls(g, g->cs, "k_lbm_macro");
+        k_lbm_macro<<<grd, blk, 0, g->cs>>>((const float *)f->base[p], (float *)rho->base[p], (float *)u->base[p], geo,
+                                            lcs(f, p), lcs(rho, p), lcs(u, p));
+        NB_TRY(nb_launch_check("k_lbm_macro"));
+    }
+    return NB_OK;
+}

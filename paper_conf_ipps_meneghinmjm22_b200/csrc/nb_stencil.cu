@@ -1,0 +1,741 @@
+// nb_stencil.cu — 7-point stencil, the config-C1 map-stencil-reduce loop and
+// the matrix-free Poisson CG on dense grids.
+//
+// Paper: Listing 2 7-point Laplacian, Fig. 4a chain
+// apxpy -> laplace -> dot (L268-L280), CG with UpdateP first (L161-L163,
+// L460), OCC variants (L293-L331).  DESIGN.md "Kernels" gives the roofline of
+// every kernel; "CG schedule" the 64 B/cell/iteration two-phase schedule.
+//
+// Per-cell arithmetic is fixed:
+//   s = ((((x[-x] + x[+x]) + x[-y]) + x[+y]) + x[-z]) + x[+z]
+//   L(x) = fma(-6, x_c, s)          A(p) = -L(p) = fma(6, p_c, -s)
+//   UpdateP: p = fma(beta, p_old, r)   x-update: x = fma(alpha, p, x)
+//   r-update: r = fma(-alpha, q, r)    C1 map: x = fma(a, y, x)
+// Every kernel that touches a cell runs these same expressions, so the
+// result does not depend on the partition count or the OCC schedule.
+#include <algorithm>
+#include <map>
+#include <vector>
+
+#include "nb_device.cuh"
+#include "nb_internal.cuh"
+
+std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v);
+nb_status nb_dot_partials(const nb_field *x, const nb_field *y);
+nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v);
+
+static inline int64_t dcs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
+
+constexpr int ZC = 32;  // planes per CTA in the z-march kernels
+
+static dim3 zmarch_grid(const nb_grid *g, int nplanes) {
+    return dim3(g->tiles_x, g->tiles_y, (nplanes + ZC - 1) / ZC);
+}
+
+// ===========================================================================
+// 7-point Laplacian y = L(x) on planes [zb, ze) (z-march: each thread keeps
+// the z-1, z, z+1 values of its column in registers; x/y neighbours come
+// from L1).  Algorithmic traffic: read x + write y = 2*sizeof(T) per cell.
+// ===========================================================================
+template <typename T>
+__global__ void __launch_bounds__(256) k_laplace7(const T *__restrict__ x, T *__restrict__ y, PGeo g,
+                                                  int zb, int ze, T outside) {
+    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
+    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
+    if (xi >= g.nx || yi >= g.ny || zs >= zend) return;
+    const int64_t o = (int64_t)yi * g.pitch + xi;
+    const T *px = x + o + g.ps;  // plane zl = 0
+    const bool hxm = xi > 0, hxp = xi < g.nx - 1, hym = yi > 0, hyp = yi < g.ny - 1;
+    T below = px[(int64_t)(zs - 1) * g.ps];
+    T center = px[(int64_t)zs * g.ps];
+    for (int z = zs; z < zend; ++z) {
+        const T *pc = px + (int64_t)z * g.ps;
+        T above = pc[g.ps];
+        T xm = hxm ? pc[-1] : outside;
+        T xp = hxp ? pc[1] : outside;
+        T ym = hym ? pc[-g.pitch] : outside;
+        T yp = hyp ? pc[g.pitch] : outside;
+        T s = xm + xp;
+        s = s + ym;
+        s = s + yp;
+        s = s + below;
+        s = s + above;
+        __stcs(y + o + (int64_t)(z + 1) * g.ps, fma(T(-6), center, s));
+        below = center;
+        center = above;
+    }
+}
+
+extern "C" nb_status nb_laplace7(const nb_field *x, nb_field *y, nb_view v) {
+    if (!x || !y) NB_FAIL(NB_EINVAL, "nb_laplace7: NULL field");
+    if (x->g != y->g) NB_FAIL(NB_EMISMATCH, "fields belong to different grids");
+    if (x->dt != y->dt || x->card != 1 || y->card != 1)
+        NB_FAIL(NB_EMISMATCH, "nb_laplace7 needs two scalar fields of one dtype");
+    nb_grid *g = x->g;
+    if (g->sparse) return nb_sparse_laplace7(x, y, v);
+    cudaSetDevice(g->device);
+    for (int p = 0; p < g->nparts; ++p) {
+        if (!g->parts[p].local) continue;
+        PGeo geo = pgeo(x, p);
+        for (auto rg : view_ranges(g, p, v)) {
+            dim3 blk(DOT_TX, DOT_TY), grd = zmarch_grid(g, rg.second - rg.first);
+            LaunchScope ls(g, g->cs, "k_laplace7");
+            if (x->dt == NB_F64)
+                k_laplace7<double><<<grd, blk, 0, g->cs>>>((const double *)x->base[p], (double *)y->base[p],
+                                                           geo, rg.first, rg.second, x->outside);
+            else
+                k_laplace7<float><<<grd, blk, 0, g->cs>>>((const float *)x->base[p], (float *)y->base[p], geo,
+                                                          rg.first, rg.second, (float)x->outside);
+            NB_TRY(nb_launch_check("k_laplace7"));
+        }
+    }
+    return NB_OK;
+}
+
+// ===========================================================================
+// "map then stencil then reduce" fused z-march (the Fig. 4a chain and CG
+// phase A share it).  The map output u = fma(m, v, w) is recomputed at every
+// neighbour inside the partition (never read back from memory), and read
+// from the stored u buffer on halo planes, where it was written by the
+// neighbour's boundary map.  MODE:
+//   MSR_C1: u = x_new = fma(a, y, x); out = y_new = L(u); dot = u*out
+//   MSR_CG: u = p_new = fma(beta, p_old, r); out = q = A(u); dot = u*q; also
+//           applies the deferred x += alpha_prev * p_old when DOMAP
+// ===========================================================================
+enum { MSR_C1 = 0, MSR_CG = 1 };
+
+struct MsrArgs {
+    const double *w;   // C1: x_in ; CG: r
+    const double *v;   // C1: y_in ; CG: p_old
+    double *u;         // C1: x_out ; CG: p_new   (halo planes read from here)
+    double *out;       // C1: y_out ; CG: unused
+    double *xs;        // CG: solution x (deferred update) ; C1: unused
+    double m;          // C1: a ; CG: beta
+    double ap;         // CG: alpha_prev
+    int pending;       // CG: apply deferred x update
+    const CgScal *sc;  // CG: status gate (may be NULL)
+};
+
+template <int MODE, bool RECOMPUTE, bool DOMAP>
+__global__ void __launch_bounds__(256) k_msr(MsrArgs A, PGeo g, int zb, int ze, double *tp, int T) {
+    __shared__ TileStage<ZC> st;
+    if (A.sc && A.sc->status != 0) return;
+    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
+    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
+    const bool valid = xi < g.nx && yi < g.ny;
+    const int64_t o = (int64_t)(valid ? yi : 0) * g.pitch + (valid ? xi : 0) + g.ps;  // zl = 0
+    const bool hxm = valid && xi > 0, hxp = valid && xi < g.nx - 1;
+    const bool hym = valid && yi > 0, hyp = valid && yi < g.ny - 1;
+    double m = A.m, ap = A.ap;
+    int pending = A.pending;
+    if (MODE == MSR_CG) {  // beta, alpha_prev, pending live on the device
+        m = A.sc->beta;
+        ap = A.sc->alpha_prev;
+        pending = A.sc->pending;
+    }
+    // map output at (plane zl, element index i): recomputed inside the slab
+    auto U = [&](int zl, int64_t i) -> double {
+        if (!RECOMPUTE || zl < 0 || zl >= g.nzl) return A.u[i];
+        return fma(m, A.v[i], A.w[i]);
+    };
+    double below = 0.0, center = 0.0, v_c = 0.0, w_c = 0.0;
+    if (valid) {
+        below = U(zs - 1, o + (int64_t)(zs - 1) * g.ps);
+        int64_t ic = o + (int64_t)zs * g.ps;
+        v_c = A.v[ic];
+        w_c = A.w[ic];
+        center = RECOMPUTE ? fma(m, v_c, w_c) : A.u[ic];
+    }
+    for (int z = zs; z < zend; ++z) {
+        double prod = 0.0;
+        double v_a = 0.0, w_a = 0.0, above = 0.0;
+        if (valid) {
+            const int64_t ic = o + (int64_t)z * g.ps, ia = ic + g.ps;
+            if (RECOMPUTE && z + 1 < g.nzl) {
+                v_a = A.v[ia];
+                w_a = A.w[ia];
+                above = fma(m, v_a, w_a);
+            } else {
+                above = A.u[ia];
+                if (DOMAP && z + 1 < g.nzl) {
+                    v_a = A.v[ia];
+                    w_a = A.w[ia];
+                }
+            }
+            double xm = hxm ? U(z, ic - 1) : 0.0;
+            double xp = hxp ? U(z, ic + 1) : 0.0;
+            double ym = hym ? U(z, ic - g.pitch) : 0.0;
+            double yp = hyp ? U(z, ic + g.pitch) : 0.0;
+            double s = __dadd_rn(xm, xp);
+            s = __dadd_rn(s, ym);
+            s = __dadd_rn(s, yp);
+            s = __dadd_rn(s, below);
+            s = __dadd_rn(s, above);
+            double res;
+            if (MODE == MSR_C1) {
+                res = fma(-6.0, center, s);
+                __stcs(A.out + ic, res);
+            } else {
+                res = fma(6.0, center, -s);
+            }
+            if (DOMAP) {
+                A.u[ic] = center;
+                if (MODE == MSR_CG && pending) A.xs[ic] = fma(ap, v_c, A.xs[ic]);
+            }
+            prod = __dmul_rn(center, res);
+        }
+        tile_stage_put<ZC>(st, z - zs, prod);
+        below = center;
+        center = above;
+        v_c = v_a;
+        w_c = w_a;
+    }
+    __syncthreads();
+    if (zs < zend)
+        tile_stage_flush<ZC>(st, zend - zs, tp, (int64_t)g.z0 + zs, T, blockIdx.y * gridDim.x + blockIdx.x);
+}
+
+// map only: u = fma(m, v, w) on planes [zb, ze) (+ CG deferred x update);
+// boundary planes are also stored into the neighbour partition's halo plane
+// (rem_lo: lower neighbour's high halo, rem_hi: upper neighbour's low halo)
+// — the halo transfer fused into the producing kernel.
+template <int MODE>
+__global__ void __launch_bounds__(256) k_map_u(MsrArgs A, PGeo g, int zb, int ze, double *rem_lo,
+                                               double *rem_hi) {
+    if (A.sc && A.sc->status != 0) return;
+    double m = A.m, ap = A.ap;
+    int pending = A.pending;
+    if (MODE == MSR_CG) {
+        m = A.sc->beta;
+        ap = A.sc->alpha_prev;
+        pending = A.sc->pending;
+    }
+    const int xi = blockIdx.x * blockDim.x + threadIdx.x, yi = blockIdx.y;
+    if (xi >= g.nx) return;
+    for (int z = zb + blockIdx.z; z < ze; z += gridDim.z) {
+        const int64_t row = (int64_t)yi * g.pitch + xi;
+        const int64_t ic = row + (int64_t)(z + 1) * g.ps;
+        double vc = A.v[ic];
+        double u = fma(m, vc, A.w[ic]);
+        A.u[ic] = u;
+        if (z == 0 && rem_lo) rem_lo[row] = u;
+        if (z == g.nzl - 1 && rem_hi) rem_hi[row] = u;
+        if (MODE == MSR_CG && pending) A.xs[ic] = fma(ap, vc, A.xs[ic]);
+    }
+}
+
+// CG phase B: q = A(p_new) from stored p_new (halo planes included),
+// r = fma(-alpha, q, r), dot r*r.
+__global__ void __launch_bounds__(256) k_cg_B(const double *__restrict__ p, double *__restrict__ r, PGeo g,
+                                              int zb, int ze, const CgScal *sc, double *tp, int T) {
+    __shared__ TileStage<ZC> st;
+    if (sc->status != 0) return;
+    const double alpha = sc->alpha;
+    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
+    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
+    const bool valid = xi < g.nx && yi < g.ny;
+    const int64_t o = (int64_t)(valid ? yi : 0) * g.pitch + (valid ? xi : 0) + g.ps;
+    const bool hxm = valid && xi > 0, hxp = valid && xi < g.nx - 1;
+    const bool hym = valid && yi > 0, hyp = valid && yi < g.ny - 1;
+    double below = 0.0, center = 0.0;
+    if (valid) {
+        below = p[o + (int64_t)(zs - 1) * g.ps];
+        center = p[o + (int64_t)zs * g.ps];
+    }
+    for (int z = zs; z < zend; ++z) {
+        double prod = 0.0, above = 0.0;
+        if (valid) {
+            const int64_t ic = o + (int64_t)z * g.ps;
+            above = p[ic + g.ps];
+            double xm = hxm ? p[ic - 1] : 0.0;
+            double xp = hxp ? p[ic + 1] : 0.0;
+            double ym = hym ? p[ic - g.pitch] : 0.0;
+            double yp = hyp ? p[ic + g.pitch] : 0.0;
+            double s = __dadd_rn(xm, xp);
+            s = __dadd_rn(s, ym);
+            s = __dadd_rn(s, yp);
+            s = __dadd_rn(s, below);
+            s = __dadd_rn(s, above);
+            double q = fma(6.0, center, -s);
+            double rn = fma(-alpha, q, __ldcs(r + ic));
+            __stcs(r + ic, rn);
+            prod = __dmul_rn(rn, rn);
+        }
+        tile_stage_put<ZC>(st, z - zs, prod);
+        below = center;
+        center = above;
+    }
+    __syncthreads();
+    if (zs < zend)
+        tile_stage_flush<ZC>(st, zend - zs, tp, (int64_t)g.z0 + zs, T, blockIdx.y * gridDim.x + blockIdx.x);
+}
+
+// CG set-up: r = b - A(x) (x halo current), dot r*r
+__global__ void __launch_bounds__(256) k_cg_init(const double *__restrict__ x, const double *__restrict__ b,
+                                                 double *__restrict__ r, PGeo g, int zb, int ze, double outside,
+                                                 double *tp, int T) {
+    __shared__ TileStage<ZC> st;
+    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
+    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
+    const bool valid = xi < g.nx && yi < g.ny;
+    const int64_t o = (int64_t)(valid ? yi : 0) * g.pitch + (valid ? xi : 0) + g.ps;
+    const bool hxm = valid && xi > 0, hxp = valid && xi < g.nx - 1;
+    const bool hym = valid && yi > 0, hyp = valid && yi < g.ny - 1;
+    double below = 0.0, center = 0.0;
+    if (valid) {
+        below = x[o + (int64_t)(zs - 1) * g.ps];
+        center = x[o + (int64_t)zs * g.ps];
+    }
+    for (int z = zs; z < zend; ++z) {
+        double prod = 0.0, above = 0.0;
+        if (valid) {
+            const int64_t ic = o + (int64_t)z * g.ps;
+            above = x[ic + g.ps];
+            double xm = hxm ? x[ic - 1] : outside;
+            double xp = hxp ? x[ic + 1] : outside;
+            double ym = hym ? x[ic - g.pitch] : outside;
+            double yp = hyp ? x[ic + g.pitch] : outside;
+            double s = __dadd_rn(xm, xp);
+            s = __dadd_rn(s, ym);
+            s = __dadd_rn(s, yp);
+            s = __dadd_rn(s, below);
+            s = __dadd_rn(s, above);
+            double ax = fma(6.0, center, -s);
+            double rv = __dsub_rn(b[ic], ax);
+            r[ic] = rv;
+            prod = __dmul_rn(rv, rv);
+        }
+        tile_stage_put<ZC>(st, z - zs, prod);
+        below = center;
+        center = above;
+    }
+    __syncthreads();
+    if (zs < zend)
+        tile_stage_flush<ZC>(st, zend - zs, tp, (int64_t)g.z0 + zs, T, blockIdx.y * gridDim.x + blockIdx.x);
+}
+
+// x += alpha_prev * p_last if an update is pending (p_last chosen by the
+// device iteration count, since convergence may stop the count early)
+__global__ void __launch_bounds__(256) k_cg_flush(double *x, const double *p0, const double *p1, int64_t n,
+                                                  CgScal *sc) {
+    if (!sc->pending) return;
+    const double *p = (sc->iters & 1) ? p1 : p0;
+    const double a = sc->alpha_prev;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        x[i] = fma(a, p[i], x[i]);
+}
+
+__global__ void k_cg_flush_done(CgScal *sc) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) sc->pending = 0;
+}
+
+// ===========================================================================
+// schedules
+// ===========================================================================
+// Boundary-plane ranges of partition p that face another partition.
+static std::vector<int> bnd_planes(const nb_grid *g, int p) {
+    std::vector<int> r;
+    const NbPart &q = g->parts[p];
+    if (q.lo >= 0) r.push_back(0);
+    if (q.hi >= 0 && !(q.lo >= 0 && q.nz() == 1)) r.push_back(q.nz() - 1);
+    return r;
+}
+
+// pointer to plane zl of partition p of a scalar field
+static double *pl(const nb_field *f, int p, int zl) {
+    return (double *)f->base[p] + (int64_t)(zl + 1) * f->ps;
+}
+
+// launch k_map_u on the planes of `planes` (or all when all==true), with
+// fused stores into neighbour halos of `ufield` for local neighbours
+static nb_status launch_map_u(nb_grid *g, int mode, int p, MsrArgs A, const nb_field *ufield, int zb, int ze) {
+    const NbPart &q = g->parts[p];
+    PGeo geo = pgeo(ufield, p);
+    double *rem_lo = nullptr, *rem_hi = nullptr;
+    if (zb == 0 && q.lo >= 0 && g->parts[q.lo].local) rem_lo = pl(ufield, q.lo, g->parts[q.lo].nz());
+    if (ze == q.nz() && q.hi >= 0 && g->parts[q.hi].local) rem_hi = pl(ufield, q.hi, -1);
+    dim3 blk(128), grd((g->nx + 127) / 128, g->ny, std::min(ze - zb, 64));
+    LaunchScope ls(g, g->cs, "k_map_u");
+    if (mode == MSR_C1)
+        k_map_u<MSR_C1><<<grd, blk, 0, g->cs>>>(A, geo, zb, ze, rem_lo, rem_hi);
+    else
+        k_map_u<MSR_CG><<<grd, blk, 0, g->cs>>>(A, geo, zb, ze, rem_lo, rem_hi);
+    return nb_launch_check("k_map_u");
+}
+
+template <int MODE, bool RC, bool DM>
+static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int zb, int ze) {
+    if (ze <= zb) return NB_OK;
+    dim3 blk(DOT_TX, DOT_TY), grd = zmarch_grid(g, ze - zb);
+    LaunchScope ls(g, g->cs, MODE == MSR_C1 ? "k_msr_c1" : "k_msr_cgA");
+    k_msr<MODE, RC, DM><<<grd, blk, 0, g->cs>>>(A, pgeo(f, p), zb, ze, g->tp, g->T);
+    return nb_launch_check("k_msr");
+}
+
+// cross-process halo of the map output after the boundary maps (NCCL on the
+// halo stream, overlapped with the internal work of the compute stream)
+
+static bool is_dist(const nb_grid *g) { return g->comm && g->comm->world > 1; }
+
+static nb_status dist_halo_begin(nb_grid *g, nb_field *u, HaloSync &hsync) {
+    if (!is_dist(g)) return NB_OK;
+    if (!hsync.eb) {
+        NB_CUDA(cudaEventCreateWithFlags(&hsync.eb, cudaEventDisableTiming));
+        NB_CUDA(cudaEventCreateWithFlags(&hsync.eh, cudaEventDisableTiming));
+    }
+    NB_CUDA(cudaEventRecord(hsync.eb, g->cs));
+    NB_CUDA(cudaStreamWaitEvent(g->hs, hsync.eb, 0));
+    NB_TRY(nb_halo_exchange_planes(u, 0, 1, true, true, g->hs));
+    NB_CUDA(cudaEventRecord(hsync.eh, g->hs));
+    return NB_OK;
+}
+static nb_status dist_halo_wait(nb_grid *g, HaloSync &hsync) {
+    if (!is_dist(g)) return NB_OK;
+    NB_CUDA(cudaStreamWaitEvent(g->cs, hsync.eh, 0));
+    return NB_OK;
+}
+
+// per-partition arguments: MsrArgs holds partition pointers, so the step is
+// run partition by partition through this adaptor
+struct MsrFields {
+    const nb_field *w, *v;
+    nb_field *u, *out, *xs;
+};
+
+template <int MODE>
+static nb_status msr_step_fields(nb_grid *g, nb_occ occ, MsrFields F, double m, double ap, int pending,
+                                 const CgScal *sc, HaloSync &hs) {
+    // maps
+    auto args = [&](int p) {
+        MsrArgs A;
+        A.w = (const double *)F.w->base[p];
+        A.v = (const double *)F.v->base[p];
+        A.u = (double *)F.u->base[p];
+        A.out = F.out ? (double *)F.out->base[p] : nullptr;
+        A.xs = F.xs ? (double *)F.xs->base[p] : nullptr;
+        A.m = m;
+        A.ap = ap;
+        A.pending = pending;
+        A.sc = sc;
+        return A;
+    };
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbPart &q = g->parts[p];
+        if (occ == NB_OCC_NONE || occ == NB_OCC_STANDARD) {
+            NB_TRY(launch_map_u(g, MODE, p, args(p), F.u, 0, q.nz()));
+        } else {
+            for (int z : bnd_planes(g, p)) NB_TRY(launch_map_u(g, MODE, p, args(p), F.u, z, z + 1));
+        }
+    }
+    NB_TRY(dist_halo_begin(g, F.u, hs));
+    if (occ == NB_OCC_NONE) NB_TRY(dist_halo_wait(g, hs));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        auto in = view_ranges(g, p, occ == NB_OCC_NONE ? NB_VIEW_STANDARD : NB_VIEW_INTERNAL);
+        for (auto rg : in) {
+            if (occ == NB_OCC_NONE || occ == NB_OCC_STANDARD)
+                NB_TRY((launch_msr<MODE, false, false>(g, p, args(p), F.u, rg.first, rg.second)));
+            else
+                NB_TRY((launch_msr<MODE, true, true>(g, p, args(p), F.u, rg.first, rg.second)));
+        }
+    }
+    if (occ == NB_OCC_NONE) return NB_OK;
+    NB_TRY(dist_halo_wait(g, hs));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        for (int z : bnd_planes(g, p)) {
+            if (occ == NB_OCC_STANDARD)
+                NB_TRY((launch_msr<MODE, false, false>(g, p, args(p), F.u, z, z + 1)));
+            else
+                NB_TRY((launch_msr<MODE, true, false>(g, p, args(p), F.u, z, z + 1)));
+        }
+    }
+    return NB_OK;
+}
+
+// ===========================================================================
+// config C1: map -> stencil -> reduce loop (Fig. 4a)
+// ===========================================================================
+extern "C" nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, int32_t iters, nb_occ occ,
+                                           double *dots_out) {
+    if (!x || !y || !dots_out) NB_FAIL(NB_EINVAL, "nb_map_stencil_reduce: NULL argument");
+    if (x->g != y->g) NB_FAIL(NB_EMISMATCH, "fields belong to different grids");
+    if (x->dt != NB_F64 || y->dt != NB_F64 || x->card != 1 || y->card != 1)
+        NB_FAIL(NB_EMISMATCH, "nb_map_stencil_reduce needs scalar fp64 fields");
+    if (iters < 0 || iters > NB_DOT_SLOTS) NB_FAIL(NB_EINVAL, "iters must be in [0, %d]", NB_DOT_SLOTS);
+    if (occ < NB_OCC_NONE || occ > NB_OCC_TWO_WAY) NB_FAIL(NB_EINVAL, "bad occ");
+    nb_grid *g = x->g;
+    if (g->sparse) NB_FAIL(NB_EUNSUPPORTED, "nb_map_stencil_reduce: dense grids only");
+    if (x->outside != 0.0) NB_FAIL(NB_EUNSUPPORTED, "nb_map_stencil_reduce: outside value must be 0");
+    cudaSetDevice(g->device);
+    // ping-pong partners (the stencil reads neighbours of x and y while the
+    // step writes new x and y)
+    nb_field *x2 = nullptr, *y2 = nullptr;
+    NB_TRY(nb_field_create(g, NB_F64, 1, 0.0, &x2));
+    nb_status st = nb_field_create(g, NB_F64, 1, 0.0, &y2);
+    HaloSync hs;
+    nb_field *xin = x, *yin = y, *xo = x2, *yo = y2;
+    for (int k = 0; k < iters && st == NB_OK; ++k) {
+        MsrFields F{xin, yin, xo, yo, nullptr};
+        st = msr_step_fields<MSR_C1>(g, occ, F, a, 0.0, 0, nullptr, hs);
+        if (st == NB_OK) st = nb_reduce_finalize(g, 1, FIN_STORE, nullptr, k);
+        std::swap(xin, xo);
+        std::swap(yin, yo);
+    }
+    if (st == NB_OK && xin != x) {  // odd iteration count: results live in the partners
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            size_t bytes = x->bytes[p];
+            cudaMemcpyAsync(x->base[p], xin->base[p], bytes, cudaMemcpyDeviceToDevice, g->cs);
+            cudaMemcpyAsync(y->base[p], yin->base[p], bytes, cudaMemcpyDeviceToDevice, g->cs);
+        }
+    }
+    if (st == NB_OK && iters > 0) {
+        cudaError_t e = cudaMemcpyAsync(dots_out, g->dots, sizeof(double) * iters, cudaMemcpyDeviceToHost, g->cs);
+        if (e != cudaSuccess) {
+            nb_set_error("cudaMemcpyAsync: %s", cudaGetErrorString(e));
+            st = NB_ECUDA;
+        }
+    }
+    cudaError_t e = cudaStreamSynchronize(g->cs);
+    if (st == NB_OK && e != cudaSuccess) {
+        nb_set_error("nb_map_stencil_reduce: %s", cudaGetErrorString(e));
+        st = NB_ECUDA;
+    }
+    if (hs.eb) {
+        cudaEventDestroy(hs.eb);
+        cudaEventDestroy(hs.eh);
+    }
+    nb_field_destroy(x2);
+    nb_field_destroy(y2);
+    return st;
+}
+
+// ===========================================================================
+// CG (Listing 3, UpdateP first L460) — two-phase schedule, 64 B/cell/iter:
+//   phase A: p_new = r + beta p_old (recomputed at neighbours), x += alpha_prev
+//            p_old (deferred), q = A p_new, <p_new, q>       40 B/cell
+//   finalize: alpha = rr / <p,q>
+//   phase B: q = A p_new (recomputed from stored p_new), r -= alpha q, <r,r>
+//                                                            24 B/cell
+//   finalize: beta = rr'/rr, ...
+// ===========================================================================
+nb_status nb_fem_cg_hooks(nb_cg *cg, int what);  // nb_fem.cu
+nb_status nb_sparse_cg_hooks(nb_cg *cg, int what);
+
+static nb_status cg_enqueue_iteration(nb_cg *cg) {
+    nb_grid *g = cg->g;
+    int64_t k = cg->k + 1;  // iteration number being enqueued
+    nb_field *pn = cg->p[k & 1], *po = cg->p[(k + 1) & 1];
+    if (cg->prm.op == NB_OP_FEM27) return nb_fem_cg_hooks(cg, (int)(k & 1));
+    if (g->sparse) return nb_sparse_cg_hooks(cg, (int)(k & 1));
+    // phase A (beta, alpha_prev and pending are read on the device from sc)
+    MsrFields F{cg->r, po, pn, nullptr, cg->x};
+    NB_TRY(msr_step_fields<MSR_CG>(g, cg->prm.occ, F, 0.0, 0.0, 0, cg->sc, cg->hs));
+    NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_PQ, cg->sc, 0));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        PGeo geo = pgeo(pn, p);
+        dim3 blk(DOT_TX, DOT_TY), grd = zmarch_grid(g, geo.nzl);
+        LaunchScope ls(g, g->cs, "k_cg_B");
+        k_cg_B<<<grd, blk, 0, g->cs>>>((const double *)pn->base[p], (double *)cg->r->base[p], geo, 0, geo.nzl,
+                                       cg->sc, g->tp, g->T);
+        NB_TRY(nb_launch_check("k_cg_B"));
+    }
+    NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_RR, cg->sc, 0));
+    cg->k = k;
+    return NB_OK;
+}
+
+static nb_status cg_check(const nb_field *x, const nb_field *b, const nb_cg_params *prm) {
+    if (!x || !b || !prm) NB_FAIL(NB_EINVAL, "nb_cg: NULL argument");
+    if (x->g != b->g) NB_FAIL(NB_EMISMATCH, "x and b belong to different grids");
+    if (x->dt != NB_F64 || b->dt != NB_F64) NB_FAIL(NB_EMISMATCH, "CG runs in fp64");
+    int card = prm->op == NB_OP_FEM27 ? 3 : 1;
+    if (x->card != card || b->card != card) NB_FAIL(NB_EMISMATCH, "CG operator needs cardinality %d", card);
+    if (prm->op != NB_OP_LAPLACE7 && prm->op != NB_OP_FEM27) NB_FAIL(NB_EINVAL, "bad operator");
+    if (prm->occ < NB_OCC_NONE || prm->occ > NB_OCC_TWO_WAY) NB_FAIL(NB_EINVAL, "bad occ");
+    if (prm->op == NB_OP_FEM27 && x->g->sparse) NB_FAIL(NB_EUNSUPPORTED, "FEM on sparse grids");
+    if (x->outside != 0.0) NB_FAIL(NB_EUNSUPPORTED, "CG: x must have outside value 0 (homogeneous Dirichlet)");
+    return NB_OK;
+}
+
+nb_status nb_fem_cg_init(nb_cg *cg);           // nb_fem.cu
+nb_status nb_sparse_cg_init(nb_cg *cg);        // nb_sparse.cu
+nb_status nb_sparse_cg_flush(nb_cg *cg);
+
+extern "C" nb_status nb_cg_create(nb_field *x, const nb_field *b, const nb_cg_params *prm, nb_cg **out) {
+    if (!out) NB_FAIL(NB_EINVAL, "nb_cg_create: out is NULL");
+    *out = nullptr;
+    NB_TRY(cg_check(x, b, prm));
+    nb_grid *g = x->g;
+    cudaSetDevice(g->device);
+    nb_cg *cg = new nb_cg();
+    cg->g = g;
+    cg->x = x;
+    cg->b = b;
+    cg->prm = *prm;
+    int card = x->card;
+    nb_status s = nb_field_create(g, NB_F64, card, 0.0, &cg->r);
+    if (s == NB_OK) s = nb_field_create(g, NB_F64, card, 0.0, &cg->p[0]);
+    if (s == NB_OK) s = nb_field_create(g, NB_F64, card, 0.0, &cg->p[1]);
+    if (s == NB_OK && (prm->op == NB_OP_FEM27 || g->sparse)) s = nb_field_create(g, NB_F64, card, 0.0, &cg->q);
+    if (s == NB_OK && cudaMalloc(&cg->sc, sizeof(CgScal)) != cudaSuccess) {
+        nb_set_error("cudaMalloc scalars failed");
+        s = NB_ENOMEM;
+    }
+    if (s == NB_OK) {
+        CgScal h{};
+        h.rtol2 = prm->rtol * prm->rtol;
+        cudaMemcpyAsync(cg->sc, &h, sizeof(CgScal), cudaMemcpyHostToDevice, g->cs);
+        // r = b - A x and rr0 (x's halo first)
+        s = nb_halo_update(x);
+        if (s == NB_OK) {
+            if (prm->op == NB_OP_FEM27) {
+                s = nb_fem_cg_init(cg);
+            } else if (g->sparse) {
+                s = nb_sparse_cg_init(cg);
+            } else {
+                for (int p = g->first_local; p < g->first_local + g->nlocal && s == NB_OK; ++p) {
+                    PGeo geo = pgeo(x, p);
+                    dim3 blk(DOT_TX, DOT_TY), grd = zmarch_grid(g, geo.nzl);
+                    LaunchScope ls(g, g->cs, "k_cg_init");
+                    k_cg_init<<<grd, blk, 0, g->cs>>>((const double *)x->base[p], (const double *)b->base[p],
+                                                      (double *)cg->r->base[p], geo, 0, geo.nzl, x->outside,
+                                                      g->tp, g->T);
+                    s = nb_launch_check("k_cg_init");
+                }
+                if (s == NB_OK) s = nb_reduce_finalize(g, 1, FIN_CG_INIT, cg->sc, 0);
+            }
+        }
+    }
+    g->nsolvers++;
+    if (s != NB_OK) {
+        nb_cg_destroy(cg);
+        return s;
+    }
+    *out = cg;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_cg_iterate(nb_cg *cg, int32_t iters) {
+    if (!cg) NB_FAIL(NB_EINVAL, "nb_cg_iterate: NULL solver");
+    if (cg->finished) NB_FAIL(NB_ESTATE, "nb_cg_iterate after nb_cg_finish");
+    if (iters < 0) NB_FAIL(NB_EINVAL, "iters < 0");
+    nb_grid *g = cg->g;
+    cudaSetDevice(g->device);
+    // eager path: profiling, multi-process (NCCL inside), or tiny counts
+    bool eager = g->profiling || is_dist(g) || getenv("NB_NO_GRAPH") != nullptr;
+    if (eager) {
+        for (int i = 0; i < iters; ++i) NB_TRY(cg_enqueue_iteration(cg));
+        return NB_OK;
+    }
+    // graph path: graphs of up to CHUNK iterations, keyed by (count, parity)
+    const int CHUNK = 16;
+    int done = 0;
+    while (done < iters) {
+        int n = std::min(CHUNK, iters - done);
+        auto key = std::make_pair(n, (int)(cg->k & 1));
+        auto it = cg->graphs.find(key);
+        if (it == cg->graphs.end()) {
+            cudaGraph_t graph;
+            int64_t l0 = g->launches, k0 = cg->k;
+            NB_CUDA(cudaStreamBeginCapture(g->cs, cudaStreamCaptureModeThreadLocal));
+            nb_status s = NB_OK;
+            for (int i = 0; i < n && s == NB_OK; ++i) s = cg_enqueue_iteration(cg);
+            cudaError_t e = cudaStreamEndCapture(g->cs, &graph);
+            int64_t nl = g->launches - l0;
+            g->launches = l0;
+            cg->k = k0;
+            if (s != NB_OK) return s;
+            if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "graph capture failed: %s", cudaGetErrorString(e));
+            cudaGraphExec_t exec;
+            e = cudaGraphInstantiate(&exec, graph, 0);
+            cudaGraphDestroy(graph);
+            if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "graph instantiate failed: %s", cudaGetErrorString(e));
+            it = cg->graphs.emplace(key, std::make_pair(exec, nl)).first;
+        }
+        NB_CUDA(cudaGraphLaunch(it->second.first, g->cs));
+        g->launches += it->second.second;
+        cg->k += n;
+        done += n;
+    }
+    return NB_OK;
+}
+
+extern "C" nb_status nb_cg_finish(nb_cg *cg, nb_cg_result *res) {
+    if (!cg) NB_FAIL(NB_EINVAL, "nb_cg_finish: NULL solver");
+    nb_grid *g = cg->g;
+    cudaSetDevice(g->device);
+    if (!cg->finished) {
+        if (g->sparse && cg->prm.op != NB_OP_FEM27) {
+            NB_TRY(nb_sparse_cg_flush(cg));
+        } else {
+            for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+                int64_t n = (int64_t)cg->x->bytes[p] / 8;
+                LaunchScope ls(g, g->cs, "k_cg_flush");
+                k_cg_flush<<<148 * 4, 256, 0, g->cs>>>((double *)cg->x->base[p], (const double *)cg->p[0]->base[p],
+                                                      (const double *)cg->p[1]->base[p], n, cg->sc);
+                NB_TRY(nb_launch_check("k_cg_flush"));
+            }
+        }
+        k_cg_flush_done<<<1, 32, 0, g->cs>>>(cg->sc);
+        NB_TRY(nb_launch_check("k_cg_flush_done"));
+        cg->finished = true;
+    }
+    CgScal h;
+    NB_CUDA(cudaMemcpyAsync(&h, cg->sc, sizeof(CgScal), cudaMemcpyDeviceToHost, g->cs));
+    NB_CUDA(cudaStreamSynchronize(g->cs));
+    if (res) {
+        res->iters = h.iters;
+        res->converged = h.status;
+        res->rr0 = h.rr0;
+        res->rr = h.rr;
+    }
+    return NB_OK;
+}
+
+nb_status nb_cg_status(nb_cg *cg, int *status, int *iters) {
+    CgScal h;
+    NB_CUDA(cudaMemcpyAsync(&h, cg->sc, sizeof(CgScal), cudaMemcpyDeviceToHost, cg->g->cs));
+    NB_CUDA(cudaStreamSynchronize(cg->g->cs));
+    *status = h.status;
+    *iters = h.iters;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_cg_destroy(nb_cg *cg) {
+    if (!cg) return NB_OK;
+    cudaSetDevice(cg->g->device);
+    cudaStreamSynchronize(cg->g->cs);
+    for (auto &kv : cg->graphs) cudaGraphExecDestroy(kv.second.first);
+    if (cg->hs.eb) {
+        cudaEventDestroy(cg->hs.eb);
+        cudaEventDestroy(cg->hs.eh);
+    }
+    nb_field_destroy(cg->r);
+    nb_field_destroy(cg->p[0]);
+    nb_field_destroy(cg->p[1]);
+    nb_field_destroy(cg->q);
+    if (cg->sc) cudaFree(cg->sc);
+    cg->g->nsolvers--;
+    delete cg;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_cg_solve(nb_field *x, const nb_field *b, const nb_cg_params *prm, nb_cg_result *res) {
+    nb_cg *cg = nullptr;
+    NB_TRY(nb_cg_create(x, b, prm, &cg));
+    int every = prm->check_every > 0 ? prm->check_every : 16;
+    int done = 0;
+    nb_status s = NB_OK;
+    while (done < prm->max_iter && s == NB_OK) {
+        int n = std::min(every, prm->max_iter - done);
+        s = nb_cg_iterate(cg, n);
+        done += n;
+        if (s == NB_OK && prm->rtol > 0.0 && done < prm->max_iter) {
+            int st = 0, it = 0;
+            s = nb_cg_status(cg, &st, &it);
+            if (st != 0) break;
+        }
+    }
+    if (s == NB_OK) s = nb_cg_finish(cg, res);
+    nb_cg_destroy(cg);
+    return s;
+}
