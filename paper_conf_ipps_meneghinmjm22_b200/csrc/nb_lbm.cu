@@ -14,6 +14,7 @@
 // Velocity order (halo-contiguous): 0 rest; 1-4 (+-x, +-y); 5-8 xy diagonals;
 // 9-13 c_z = +1; 14-18 c_z = -1.
 #include <algorithm>
+#include <cstring>
 
 #include "nb_device.cuh"
 #include "nb_internal.cuh"
@@ -41,48 +42,18 @@ __device__ __host__ constexpr float Wv(int i) {
 }  // namespace
 
 struct LbmArgs {
-    const float *fin;
-    float *fout;
+    const float *fin[Q19];   // component base pointers (plane zl = -1, row 0)
+    float *fout[Q19];
+    float *rem_lo[Q19];      // lower neighbour's fout components at its high halo plane (14..18 used)
+    float *rem_hi[Q19];      // upper neighbour's fout components at its low halo plane (9..13 used)
     PGeo g;
-    int64_t cs;          // component stride of this partition
     float omega, ulid, rho_w;
-    int periodic;
-    float *rem_lo;       // lower neighbour's fout, component 0, plane zl = nz_lo (its high halo)
-    int64_t rem_lo_cs;
-    float *rem_hi;       // upper neighbour's fout, component 0, plane zl = -1 (its low halo)
-    int64_t rem_hi_cs;
 };
 
-template <bool PERIODIC>
-__global__ void __launch_bounds__(128) k_lbm_d3q19(LbmArgs A, int zb) {
-    const int x = blockIdx.x * blockDim.x + threadIdx.x;
-    const int y = blockIdx.y;
-    const int zl = zb + blockIdx.z;
-    const PGeo &g = A.g;
-    if (x >= g.nx) return;
-    const int gz = g.z0 + zl;
-    const int64_t cell = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
-    float f[Q19];
-#pragma unroll
-    for (int i = 0; i < Q19; ++i) {
-        int sx = x - CXv(i), sy = y - CYv(i), szl = zl - CZv(i);
-        if (PERIODIC) {
-            sx = sx < 0 ? sx + g.nx : (sx >= g.nx ? sx - g.nx : sx);
-            sy = sy < 0 ? sy + g.ny : (sy >= g.ny ? sy - g.ny : sy);
-            f[i] = __ldg(A.fin + (int64_t)i * A.cs + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx);
-        } else {
-            const int sgz = gz - CZv(i);
-            const bool inside = sx >= 0 && sx < g.nx && sy >= 0 && sy < g.ny && sgz >= 0 && sgz < g.NZ;
-            if (inside) {
-                f[i] = __ldg(A.fin + (int64_t)i * A.cs + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx);
-            } else {
-                float v = __ldg(A.fin + (int64_t)OPPv(i) * A.cs + cell);
-                if (CXv(i) != 0 && sy == g.ny && sx >= 0 && sx < g.nx && sgz >= 0 && sgz < g.NZ)
-                    v = v + 6.0f * Wv(i) * A.rho_w * ((float)CXv(i) * A.ulid);
-                f[i] = v;
-            }
-        }
-    }
+// BGK collision of the gathered populations and the streaming store (shared
+// by the interior fast path and the boundary path: same code, same bits)
+__device__ __forceinline__ void lbm_collide_store(const float (&f)[Q19], const LbmArgs &A, int64_t cell,
+                                                  int zl, int64_t row) {
     float rho = 0.f, jx = 0.f, jy = 0.f, jz = 0.f;
 #pragma unroll
     for (int i = 0; i < Q19; ++i) {
@@ -103,19 +74,62 @@ __global__ void __launch_bounds__(128) k_lbm_d3q19(LbmArgs A, int zb) {
         float cu = (float)CXv(i) * ux + (float)CYv(i) * uy + (float)CZv(i) * uz;
         float feq = Wv(i) * rho * (1.0f + 3.0f * cu + 4.5f * cu * cu - 1.5f * usq);
         o[i] = f[i] - om * (f[i] - feq);
-        __stcs(A.fout + (int64_t)i * A.cs + cell, o[i]);
+        __stcs(A.fout[i] + cell, o[i]);
     }
-    // halo transfer fused into the producing kernel: outgoing populations
-    // of the boundary planes go straight into the neighbours' halo planes
+    // halo transfer fused into the producing kernel: outgoing populations of
+    // the boundary planes go straight into the neighbours' halo planes
+    if (zl == 0 && A.rem_lo[14]) {
+#pragma unroll
+        for (int i = 14; i < 19; ++i) A.rem_lo[i][row] = o[i];
+    }
+    if (zl == A.g.nzl - 1 && A.rem_hi[9]) {
+#pragma unroll
+        for (int i = 9; i < 14; ++i) A.rem_hi[i][row] = o[i];
+    }
+}
+
+template <bool PERIODIC>
+__global__ void __launch_bounds__(128) k_lbm_d3q19(LbmArgs A, int zb) {
+    const int x = blockIdx.x * blockDim.x + threadIdx.x;
+    const int y = blockIdx.y;
+    const int zl = zb + blockIdx.z;
+    const PGeo &g = A.g;
+    if (x >= g.nx) return;
+    const int gz = g.z0 + zl;
     const int64_t row = (int64_t)y * g.pitch + x;
-    if (zl == 0 && A.rem_lo) {
+    const int64_t cell = (int64_t)(zl + 1) * g.ps + row;
+    float f[Q19];
+    const bool interior = x > 0 && x < g.nx - 1 && y > 0 && y < g.ny - 1 &&
+                          (PERIODIC || (gz > 0 && gz < g.NZ - 1));
+    if (interior) {
+        // every source is in the slab or its halo planes: 19 independent
+        // loads at uniform offsets
 #pragma unroll
-        for (int i = 14; i < 19; ++i) A.rem_lo[(int64_t)i * A.rem_lo_cs + row] = o[i];
-    }
-    if (zl == g.nzl - 1 && A.rem_hi) {
+        for (int i = 0; i < Q19; ++i)
+            f[i] = __ldg(A.fin[i] + cell - (int64_t)CZv(i) * g.ps - (int64_t)CYv(i) * g.pitch - CXv(i));
+    } else {
 #pragma unroll
-        for (int i = 9; i < 14; ++i) A.rem_hi[(int64_t)i * A.rem_hi_cs + row] = o[i];
+        for (int i = 0; i < Q19; ++i) {
+            int sx = x - CXv(i), sy = y - CYv(i), szl = zl - CZv(i);
+            if (PERIODIC) {
+                sx = sx < 0 ? sx + g.nx : (sx >= g.nx ? sx - g.nx : sx);
+                sy = sy < 0 ? sy + g.ny : (sy >= g.ny ? sy - g.ny : sy);
+                f[i] = __ldg(A.fin[i] + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx);
+            } else {
+                // in-domain neighbour, or half-way bounce-back from the
+                // opposite population of this cell (+ moving-lid term)
+                const int sgz = gz - CZv(i);
+                const bool inside = sx >= 0 && sx < g.nx && sy >= 0 && sy < g.ny && sgz >= 0 && sgz < g.NZ;
+                const float *src = inside ? A.fin[i] + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx
+                                          : A.fin[OPPv(i)] + cell;
+                float v = __ldg(src);
+                if (CXv(i) != 0 && sy == g.ny && sx >= 0 && sx < g.nx && sgz >= 0 && sgz < g.NZ)
+                    v = v + 6.0f * Wv(i) * A.rho_w * ((float)CXv(i) * A.ulid);
+                f[i] = v;
+            }
+        }
     }
+    lbm_collide_store(f, A, cell, zl, row);
 }
 
 __global__ void __launch_bounds__(128) k_lbm_init(float *f, PGeo g, int64_t cs, float rho, float ux, float uy,
@@ -248,26 +262,23 @@ static nb_status launch_lbm(nb_grid *g, int p, nb_field *fin, nb_field *fout, co
     if (ze <= zb) return NB_OK;
     bool per = prm->bc == NB_LBM_PERIODIC;
     LbmArgs A;
-    A.fin = (const float *)fin->base[p];
-    A.fout = (float *)fout->base[p];
+    memset(&A, 0, sizeof(A));
+    for (int i = 0; i < Q19; ++i) {
+        A.fin[i] = (const float *)fin->base[p] + (int64_t)i * lcs(fin, p);
+        A.fout[i] = (float *)fout->base[p] + (int64_t)i * lcs(fout, p);
+    }
     A.g = pgeo(fin, p);
-    A.cs = lcs(fin, p);
     A.omega = (float)prm->omega;
     A.ulid = (float)prm->u_lid;
     A.rho_w = (float)prm->rho_w;
-    A.periodic = per;
-    A.rem_lo = A.rem_hi = nullptr;
-    A.rem_lo_cs = A.rem_hi_cs = 0;
     if (remote_stores) {
         int lo = lbm_lo(g, p, per), hi = lbm_hi(g, p, per);
-        if (zb == 0 && lo >= 0 && g->parts[lo].local) {
-            A.rem_lo = (float *)fout->base[lo] + (int64_t)(g->parts[lo].nz() + 1) * fout->ps;
-            A.rem_lo_cs = lcs(fout, lo);
-        }
-        if (ze == g->parts[p].nz() && hi >= 0 && g->parts[hi].local) {
-            A.rem_hi = (float *)fout->base[hi];
-            A.rem_hi_cs = lcs(fout, hi);
-        }
+        if (zb == 0 && lo >= 0 && g->parts[lo].local)
+            for (int i = 14; i < 19; ++i)
+                A.rem_lo[i] = (float *)fout->base[lo] + (int64_t)i * lcs(fout, lo) +
+                              (int64_t)(g->parts[lo].nz() + 1) * fout->ps;
+        if (ze == g->parts[p].nz() && hi >= 0 && g->parts[hi].local)
+            for (int i = 9; i < 14; ++i) A.rem_hi[i] = (float *)fout->base[hi] + (int64_t)i * lcs(fout, hi);
     }
     dim3 blk(128), grd((g->nx + 127) / 128, g->ny, ze - zb);
     LaunchScope ls(g, g->cs, "k_lbm_d3q19");

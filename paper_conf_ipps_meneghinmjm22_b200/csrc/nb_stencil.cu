@@ -19,6 +19,7 @@
 
 #include "nb_device.cuh"
 #include "nb_internal.cuh"
+#include "nb_zmarch.cuh"
 
 std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v);
 nb_status nb_dot_partials(const nb_field *x, const nb_field *y);
@@ -26,44 +27,40 @@ nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v);
 
 static inline int64_t dcs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
 
-constexpr int ZC = 32;  // planes per CTA in the z-march kernels
-
-static dim3 zmarch_grid(const nb_grid *g, int nplanes) {
-    return dim3(g->tiles_x, g->tiles_y, (nplanes + ZC - 1) / ZC);
-}
 
 // ===========================================================================
-// 7-point Laplacian y = L(x) on planes [zb, ze) (z-march: each thread keeps
-// the z-1, z, z+1 values of its column in registers; x/y neighbours come
-// from L1).  Algorithmic traffic: read x + write y = 2*sizeof(T) per cell.
+// 7-point Laplacian y = L(x) (Listing 2).  Algorithmic traffic: read x +
+// write y = 2*sizeof(T) per cell.
 // ===========================================================================
-template <typename T>
-__global__ void __launch_bounds__(256) k_laplace7(const T *__restrict__ x, T *__restrict__ y, PGeo g,
-                                                  int zb, int ze, T outside) {
-    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
-    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
-    if (xi >= g.nx || yi >= g.ny || zs >= zend) return;
-    const int64_t o = (int64_t)yi * g.pitch + xi;
-    const T *px = x + o + g.ps;  // plane zl = 0
-    const bool hxm = xi > 0, hxp = xi < g.nx - 1, hym = yi > 0, hyp = yi < g.ny - 1;
-    T below = px[(int64_t)(zs - 1) * g.ps];
-    T center = px[(int64_t)zs * g.ps];
-    for (int z = zs; z < zend; ++z) {
-        const T *pc = px + (int64_t)z * g.ps;
-        T above = pc[g.ps];
-        T xm = hxm ? pc[-1] : outside;
-        T xp = hxp ? pc[1] : outside;
-        T ym = hym ? pc[-g.pitch] : outside;
-        T yp = hyp ? pc[g.pitch] : outside;
-        T s = xm + xp;
-        s = s + ym;
-        s = s + yp;
-        s = s + below;
-        s = s + above;
-        __stcs(y + o + (int64_t)(z + 1) * g.ps, fma(T(-6), center, s));
-        below = center;
-        center = above;
+template <typename TT>
+struct Lap7Op {
+    using T = TT;
+    struct Raw {
+        TT a;
+    };
+    static constexpr bool DOT = false;
+    const TT *x;
+    TT *y;
+    TT outv;
+    __device__ bool skip() const { return false; }
+    __device__ void init() {}
+    __device__ TT outside() const { return outv; }
+    __device__ Raw raw(int, int64_t i, bool) const { return {x[i]}; }
+    __device__ TT val(int, const Raw &r) const { return r.a; }
+    __device__ TT nval(int, int64_t i) const { return x[i]; }
+    __device__ double cell(int, int64_t i, TT c, TT s, const Raw &) {
+        __stcs(y + i, fma(TT(-6), c, s));
+        return 0.0;
     }
+};
+
+template <class Op, bool SMEM = false>
+static nb_status launch_zmarch(nb_grid *g, const char *name, Op op, PGeo geo, int zb, int ze) {
+    if (ze <= zb) return NB_OK;
+    dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
+    LaunchScope ls(g, g->cs, name);
+    k_zmarch<Op, SMEM><<<grd, blk, 0, g->cs>>>(op, geo, zb, ze, g->tp, g->T);
+    return nb_launch_check(name);
 }
 
 extern "C" nb_status nb_laplace7(const nb_field *x, nb_field *y, nb_view v) {
@@ -78,15 +75,14 @@ extern "C" nb_status nb_laplace7(const nb_field *x, nb_field *y, nb_view v) {
         if (!g->parts[p].local) continue;
         PGeo geo = pgeo(x, p);
         for (auto rg : view_ranges(g, p, v)) {
-            dim3 blk(DOT_TX, DOT_TY), grd = zmarch_grid(g, rg.second - rg.first);
-            LaunchScope ls(g, g->cs, "k_laplace7");
             if (x->dt == NB_F64)
-                k_laplace7<double><<<grd, blk, 0, g->cs>>>((const double *)x->base[p], (double *)y->base[p],
-                                                           geo, rg.first, rg.second, x->outside);
+                NB_TRY(launch_zmarch(g, "k_laplace7",
+                                     Lap7Op<double>{(const double *)x->base[p], (double *)y->base[p], x->outside},
+                                     geo, rg.first, rg.second));
             else
-                k_laplace7<float><<<grd, blk, 0, g->cs>>>((const float *)x->base[p], (float *)y->base[p], geo,
-                                                          rg.first, rg.second, (float)x->outside);
-            NB_TRY(nb_launch_check("k_laplace7"));
+                NB_TRY(launch_zmarch(g, "k_laplace7",
+                                     Lap7Op<float>{(const float *)x->base[p], (float *)y->base[p], (float)x->outside},
+                                     geo, rg.first, rg.second));
         }
     }
     return NB_OK;
@@ -117,83 +113,58 @@ struct MsrArgs {
 };
 
 template <int MODE, bool RECOMPUTE, bool DOMAP>
-__global__ void __launch_bounds__(256) k_msr(MsrArgs A, PGeo g, int zb, int ze, double *tp, int T) {
-    __shared__ TileStage<ZC> st;
-    if (A.sc && A.sc->status != 0) return;
-    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
-    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
-    const bool valid = xi < g.nx && yi < g.ny;
-    const int64_t o = (int64_t)(valid ? yi : 0) * g.pitch + (valid ? xi : 0) + g.ps;  // zl = 0
-    const bool hxm = valid && xi > 0, hxp = valid && xi < g.nx - 1;
-    const bool hym = valid && yi > 0, hyp = valid && yi < g.ny - 1;
-    double m = A.m, ap = A.ap;
-    int pending = A.pending;
-    if (MODE == MSR_CG) {  // beta, alpha_prev, pending live on the device
-        m = A.sc->beta;
-        ap = A.sc->alpha_prev;
-        pending = A.sc->pending;
-    }
-    // map output at (plane zl, element index i): recomputed inside the slab
-    auto U = [&](int zl, int64_t i) -> double {
-        if (!RECOMPUTE || zl < 0 || zl >= g.nzl) return A.u[i];
-        return fma(m, A.v[i], A.w[i]);
+struct MsrOp {
+    using T = double;
+    struct Raw {
+        double v, w, x;  // v: map input (or stored u on halo planes), w, x: see cell()
     };
-    double below = 0.0, center = 0.0, v_c = 0.0, w_c = 0.0;
-    if (valid) {
-        below = U(zs - 1, o + (int64_t)(zs - 1) * g.ps);
-        int64_t ic = o + (int64_t)zs * g.ps;
-        v_c = A.v[ic];
-        w_c = A.w[ic];
-        center = RECOMPUTE ? fma(m, v_c, w_c) : A.u[ic];
-    }
-    for (int z = zs; z < zend; ++z) {
-        double prod = 0.0;
-        double v_a = 0.0, w_a = 0.0, above = 0.0;
-        if (valid) {
-            const int64_t ic = o + (int64_t)z * g.ps, ia = ic + g.ps;
-            if (RECOMPUTE && z + 1 < g.nzl) {
-                v_a = A.v[ia];
-                w_a = A.w[ia];
-                above = fma(m, v_a, w_a);
-            } else {
-                above = A.u[ia];
-                if (DOMAP && z + 1 < g.nzl) {
-                    v_a = A.v[ia];
-                    w_a = A.w[ia];
-                }
-            }
-            double xm = hxm ? U(z, ic - 1) : 0.0;
-            double xp = hxp ? U(z, ic + 1) : 0.0;
-            double ym = hym ? U(z, ic - g.pitch) : 0.0;
-            double yp = hyp ? U(z, ic + g.pitch) : 0.0;
-            double s = __dadd_rn(xm, xp);
-            s = __dadd_rn(s, ym);
-            s = __dadd_rn(s, yp);
-            s = __dadd_rn(s, below);
-            s = __dadd_rn(s, above);
-            double res;
-            if (MODE == MSR_C1) {
-                res = fma(-6.0, center, s);
-                __stcs(A.out + ic, res);
-            } else {
-                res = fma(6.0, center, -s);
-            }
-            if (DOMAP) {
-                A.u[ic] = center;
-                if (MODE == MSR_CG && pending) A.xs[ic] = fma(ap, v_c, A.xs[ic]);
-            }
-            prod = __dmul_rn(center, res);
+    static constexpr bool DOT = true;
+    MsrArgs A;
+    int nzl;
+    double m, ap;
+    int pending;
+    __device__ bool skip() const { return A.sc && A.sc->status != 0; }
+    __device__ void init() {
+        m = A.m;
+        ap = A.ap;
+        pending = A.pending;
+        if (MODE == MSR_CG) {  // beta, alpha_prev, pending live on the device
+            m = A.sc->beta;
+            ap = A.sc->alpha_prev;
+            pending = A.sc->pending;
         }
-        tile_stage_put<ZC>(st, z - zs, prod);
-        below = center;
-        center = above;
-        v_c = v_a;
-        w_c = w_a;
     }
-    __syncthreads();
-    if (zs < zend)
-        tile_stage_flush<ZC>(st, zend - zs, tp, (int64_t)g.z0 + zs, T, blockIdx.y * gridDim.x + blockIdx.x);
-}
+    __device__ double outside() const { return 0.0; }
+    __device__ bool stored(int zl) const { return !RECOMPUTE || zl < 0 || zl >= nzl; }
+    // map output: recomputed inside the slab, read back on halo planes
+    __device__ Raw raw(int zl, int64_t i, bool own) const {
+        Raw r{0.0, 0.0, 0.0};
+        if (stored(zl)) {
+            r.v = A.u[i];
+        } else {
+            r.v = A.v[i];
+            r.w = A.w[i];
+            if (MODE == MSR_CG && DOMAP && own && pending) r.x = A.xs[i];
+        }
+        return r;
+    }
+    __device__ double val(int zl, const Raw &r) const { return stored(zl) ? r.v : fma(m, r.v, r.w); }
+    __device__ double nval(int zl, int64_t i) const { return val(zl, raw(zl, i, false)); }
+    __device__ double cell(int, int64_t i, double c, double s, const Raw &rc) {
+        double res;
+        if (MODE == MSR_C1) {
+            res = fma(-6.0, c, s);
+            __stcs(A.out + i, res);
+        } else {
+            res = fma(6.0, c, -s);
+        }
+        if (DOMAP) {
+            A.u[i] = c;
+            if (MODE == MSR_CG && pending) A.xs[i] = fma(ap, rc.v, rc.x);
+        }
+        return __dmul_rn(c, res);
+    }
+};
 
 // map only: u = fma(m, v, w) on planes [zb, ze) (+ CG deferred x update);
 // boundary planes are also stored into the neighbour partition's halo plane
@@ -226,93 +197,53 @@ __global__ void __launch_bounds__(256) k_map_u(MsrArgs A, PGeo g, int zb, int ze
 
 // CG phase B: q = A(p_new) from stored p_new (halo planes included),
 // r = fma(-alpha, q, r), dot r*r.
-__global__ void __launch_bounds__(256) k_cg_B(const double *__restrict__ p, double *__restrict__ r, PGeo g,
-                                              int zb, int ze, const CgScal *sc, double *tp, int T) {
-    __shared__ TileStage<ZC> st;
-    if (sc->status != 0) return;
-    const double alpha = sc->alpha;
-    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
-    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
-    const bool valid = xi < g.nx && yi < g.ny;
-    const int64_t o = (int64_t)(valid ? yi : 0) * g.pitch + (valid ? xi : 0) + g.ps;
-    const bool hxm = valid && xi > 0, hxp = valid && xi < g.nx - 1;
-    const bool hym = valid && yi > 0, hyp = valid && yi < g.ny - 1;
-    double below = 0.0, center = 0.0;
-    if (valid) {
-        below = p[o + (int64_t)(zs - 1) * g.ps];
-        center = p[o + (int64_t)zs * g.ps];
+struct CgBOp {
+    using T = double;
+    struct Raw {
+        double p, r;
+    };
+    static constexpr bool DOT = true;
+    const double *p;
+    double *r;
+    const CgScal *sc;
+    double alpha;
+    __device__ bool skip() const { return sc->status != 0; }
+    __device__ void init() { alpha = sc->alpha; }
+    __device__ double outside() const { return 0.0; }
+    __device__ Raw raw(int, int64_t i, bool own) const { return {p[i], own ? __ldcs(r + i) : 0.0}; }
+    __device__ double val(int, const Raw &q) const { return q.p; }
+    __device__ double nval(int, int64_t i) const { return p[i]; }
+    __device__ double cell(int, int64_t i, double c, double s, const Raw &rc) {
+        double q = fma(6.0, c, -s);
+        double rn = fma(-alpha, q, rc.r);
+        __stcs(r + i, rn);
+        return __dmul_rn(rn, rn);
     }
-    for (int z = zs; z < zend; ++z) {
-        double prod = 0.0, above = 0.0;
-        if (valid) {
-            const int64_t ic = o + (int64_t)z * g.ps;
-            above = p[ic + g.ps];
-            double xm = hxm ? p[ic - 1] : 0.0;
-            double xp = hxp ? p[ic + 1] : 0.0;
-            double ym = hym ? p[ic - g.pitch] : 0.0;
-            double yp = hyp ? p[ic + g.pitch] : 0.0;
-            double s = __dadd_rn(xm, xp);
-            s = __dadd_rn(s, ym);
-            s = __dadd_rn(s, yp);
-            s = __dadd_rn(s, below);
-            s = __dadd_rn(s, above);
-            double q = fma(6.0, center, -s);
-            double rn = fma(-alpha, q, __ldcs(r + ic));
-            __stcs(r + ic, rn);
-            prod = __dmul_rn(rn, rn);
-        }
-        tile_stage_put<ZC>(st, z - zs, prod);
-        below = center;
-        center = above;
-    }
-    __syncthreads();
-    if (zs < zend)
-        tile_stage_flush<ZC>(st, zend - zs, tp, (int64_t)g.z0 + zs, T, blockIdx.y * gridDim.x + blockIdx.x);
-}
+};
 
 // CG set-up: r = b - A(x) (x halo current), dot r*r
-__global__ void __launch_bounds__(256) k_cg_init(const double *__restrict__ x, const double *__restrict__ b,
-                                                 double *__restrict__ r, PGeo g, int zb, int ze, double outside,
-                                                 double *tp, int T) {
-    __shared__ TileStage<ZC> st;
-    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
-    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
-    const bool valid = xi < g.nx && yi < g.ny;
-    const int64_t o = (int64_t)(valid ? yi : 0) * g.pitch + (valid ? xi : 0) + g.ps;
-    const bool hxm = valid && xi > 0, hxp = valid && xi < g.nx - 1;
-    const bool hym = valid && yi > 0, hyp = valid && yi < g.ny - 1;
-    double below = 0.0, center = 0.0;
-    if (valid) {
-        below = x[o + (int64_t)(zs - 1) * g.ps];
-        center = x[o + (int64_t)zs * g.ps];
+struct CgInitOp {
+    using T = double;
+    struct Raw {
+        double x, b;
+    };
+    static constexpr bool DOT = true;
+    const double *x, *b;
+    double *r;
+    double outv;
+    __device__ bool skip() const { return false; }
+    __device__ void init() {}
+    __device__ double outside() const { return outv; }
+    __device__ Raw raw(int, int64_t i, bool own) const { return {x[i], own ? b[i] : 0.0}; }
+    __device__ double val(int, const Raw &q) const { return q.x; }
+    __device__ double nval(int, int64_t i) const { return x[i]; }
+    __device__ double cell(int, int64_t i, double c, double s, const Raw &rc) {
+        double ax = fma(6.0, c, -s);
+        double rv = __dsub_rn(rc.b, ax);
+        r[i] = rv;
+        return __dmul_rn(rv, rv);
     }
-    for (int z = zs; z < zend; ++z) {
-        double prod = 0.0, above = 0.0;
-        if (valid) {
-            const int64_t ic = o + (int64_t)z * g.ps;
-            above = x[ic + g.ps];
-            double xm = hxm ? x[ic - 1] : outside;
-            double xp = hxp ? x[ic + 1] : outside;
-            double ym = hym ? x[ic - g.pitch] : outside;
-            double yp = hyp ? x[ic + g.pitch] : outside;
-            double s = __dadd_rn(xm, xp);
-            s = __dadd_rn(s, ym);
-            s = __dadd_rn(s, yp);
-            s = __dadd_rn(s, below);
-            s = __dadd_rn(s, above);
-            double ax = fma(6.0, center, -s);
-            double rv = __dsub_rn(b[ic], ax);
-            r[ic] = rv;
-            prod = __dmul_rn(rv, rv);
-        }
-        tile_stage_put<ZC>(st, z - zs, prod);
-        below = center;
-        center = above;
-    }
-    __syncthreads();
-    if (zs < zend)
-        tile_stage_flush<ZC>(st, zend - zs, tp, (int64_t)g.z0 + zs, T, blockIdx.y * gridDim.x + blockIdx.x);
-}
+};
 
 // x += alpha_prev * p_last if an update is pending (p_last chosen by the
 // device iteration count, since convergence may stop the count early)
@@ -365,11 +296,13 @@ static nb_status launch_map_u(nb_grid *g, int mode, int p, MsrArgs A, const nb_f
 
 template <int MODE, bool RC, bool DM>
 static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int zb, int ze) {
-    if (ze <= zb) return NB_OK;
-    dim3 blk(DOT_TX, DOT_TY), grd = zmarch_grid(g, ze - zb);
-    LaunchScope ls(g, g->cs, MODE == MSR_C1 ? "k_msr_c1" : "k_msr_cgA");
-    k_msr<MODE, RC, DM><<<grd, blk, 0, g->cs>>>(A, pgeo(f, p), zb, ze, g->tp, g->T);
-    return nb_launch_check("k_msr");
+    MsrOp<MODE, RC, DM> op;
+    op.A = A;
+    op.nzl = g->parts[p].nz();
+    // recompute: the map output of every cell is computed once per CTA into
+    // the staged tile; stored input: neighbours straight from L1
+    return launch_zmarch<MsrOp<MODE, RC, DM>, RC>(g, MODE == MSR_C1 ? "k_msr_c1" : "k_msr_cgA", op, pgeo(f, p),
+                                                  zb, ze);
 }
 
 // cross-process halo of the map output after the boundary maps (NCCL on the
@@ -532,11 +465,8 @@ static nb_status cg_enqueue_iteration(nb_cg *cg) {
     NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_PQ, cg->sc, 0));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         PGeo geo = pgeo(pn, p);
-        dim3 blk(DOT_TX, DOT_TY), grd = zmarch_grid(g, geo.nzl);
-        LaunchScope ls(g, g->cs, "k_cg_B");
-        k_cg_B<<<grd, blk, 0, g->cs>>>((const double *)pn->base[p], (double *)cg->r->base[p], geo, 0, geo.nzl,
-                                       cg->sc, g->tp, g->T);
-        NB_TRY(nb_launch_check("k_cg_B"));
+        CgBOp op{(const double *)pn->base[p], (double *)cg->r->base[p], cg->sc, 0.0};
+        NB_TRY(launch_zmarch(g, "k_cg_B", op, geo, 0, geo.nzl));
     }
     NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_RR, cg->sc, 0));
     cg->k = k;
@@ -594,12 +524,9 @@ extern "C" nb_status nb_cg_create(nb_field *x, const nb_field *b, const nb_cg_pa
             } else {
                 for (int p = g->first_local; p < g->first_local + g->nlocal && s == NB_OK; ++p) {
                     PGeo geo = pgeo(x, p);
-                    dim3 blk(DOT_TX, DOT_TY), grd = zmarch_grid(g, geo.nzl);
-                    LaunchScope ls(g, g->cs, "k_cg_init");
-                    k_cg_init<<<grd, blk, 0, g->cs>>>((const double *)x->base[p], (const double *)b->base[p],
-                                                      (double *)cg->r->base[p], geo, 0, geo.nzl, x->outside,
-                                                      g->tp, g->T);
-                    s = nb_launch_check("k_cg_init");
+                    CgInitOp op{(const double *)x->base[p], (const double *)b->base[p], (double *)cg->r->base[p],
+                                x->outside};
+                    s = launch_zmarch(g, "k_cg_init", op, geo, 0, geo.nzl);
                 }
                 if (s == NB_OK) s = nb_reduce_finalize(g, 1, FIN_CG_INIT, cg->sc, 0);
             }
