@@ -212,6 +212,10 @@ nb_status nb_cg_create(nb_field *x, const nb_field *b, const nb_cg_params *param
 /* Enqueue `iters` CG iterations (graph-launched; converged state turns
  * later iterations into no-ops).  No sync. */
 nb_status nb_cg_iterate(nb_cg *cg, int32_t iters);
+/* Capture (without running anything) the CUDA graphs that
+ * nb_cg_iterate(cg, iters) will launch from the current state, so that the
+ * first call does not pay for graph instantiation. */
+nb_status nb_cg_prepare(nb_cg *cg, int32_t iters);
 /* Apply the deferred x update and read the scalars back.  Synchronises. */
 nb_status nb_cg_finish(nb_cg *cg, nb_cg_result *result);
 nb_status nb_cg_destroy(nb_cg *cg);

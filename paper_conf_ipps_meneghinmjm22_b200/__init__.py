@@ -95,6 +95,7 @@ SIGNATURES = {
     "nb_map_stencil_reduce": ([P, P, D, I32, I32, P], I32),
     "nb_cg_create": ([P, P, P, PP], I32),
     "nb_cg_iterate": ([P, I32], I32),
+    "nb_cg_prepare": ([P, I32], I32),
     "nb_cg_finish": ([P, P], I32),
     "nb_cg_destroy": ([P], I32),
     "nb_cg_solve": ([P, P, P, P], I32),
@@ -388,6 +389,10 @@ class CG:
 
     def iterate(self, n: int):
         _check(lib().nb_cg_iterate(self.handle, int(n)))
+
+    def prepare(self, n: int):
+        """Build the CUDA graphs iterate(n) will launch (no GPU work)."""
+        _check(lib().nb_cg_prepare(self.handle, int(n)))
 
     def finish(self) -> CgResult:
         r = CgResult()

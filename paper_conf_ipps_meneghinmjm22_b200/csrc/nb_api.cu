@@ -341,6 +341,21 @@ extern "C" nb_status nb_grid_create_dense(const int32_t dims[3], int32_t nparts,
 
 void nb_sparse_free(nb_grid *g);  // nb_sparse.cu
 
+nb_status nb_grid_scratch(nb_grid *g, nb_dtype dt, int card, int slot, nb_field **out) {
+    auto key = std::make_pair((int)dt * 1000 + card, slot);
+    auto it = g->scratch.find(key);
+    if (it != g->scratch.end()) {
+        *out = it->second;
+        return NB_OK;
+    }
+    nb_field *f = nullptr;
+    NB_TRY(nb_field_create(g, dt, card, 0.0, &f));
+    g->nfields--;  // owned by the grid
+    g->scratch[key] = f;
+    *out = f;
+    return NB_OK;
+}
+
 extern "C" nb_status nb_grid_destroy(nb_grid *g) {
     if (!g) return NB_OK;
     if (g->nfields > 0 || g->nsolvers > 0)
@@ -349,6 +364,11 @@ extern "C" nb_status nb_grid_destroy(nb_grid *g) {
     DeviceGuard dg(g->device);
     if (g->cs) cudaStreamSynchronize(g->cs);
     if (g->hs) cudaStreamSynchronize(g->hs);
+    for (auto &kv : g->scratch) {
+        g->nfields++;
+        nb_field_destroy(kv.second);
+    }
+    g->scratch.clear();
     for (auto &r : g->prof) {
         cudaEventDestroy(r.a);
         cudaEventDestroy(r.b);

@@ -8,6 +8,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <string>
+#include <map>
 #include <vector>
 
 #include "nb.h"
@@ -109,6 +110,8 @@ struct nb_grid {
     bool profiling = false;
     std::vector<ProfRec> prof;
     int64_t launches = 0;
+    // internal scratch fields (ping-pong partners), not counted in nfields
+    std::map<std::pair<int, int>, struct nb_field *> scratch;
     // element-sparse
     std::vector<NbSparsePart> sp;
     std::vector<int64_t> plane_count;  // [nz] active per global plane
@@ -193,6 +196,9 @@ struct CgScal {
     double rr, rr0, alpha, alpha_prev, beta, pq, rtol2;
     int32_t iters, status, pending, pad;
 };
+
+// cached internal field of the grid (slot distinguishes several of one kind)
+nb_status nb_grid_scratch(nb_grid *g, nb_dtype dt, int card, int slot, nb_field **out);
 
 // halo helpers (nb_api.cu)
 nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down,

@@ -54,12 +54,28 @@ struct Lap7Op {
     }
 };
 
+// z-march variant: lookahead L (0: load plane z+1 at step z; 1: prefetch
+// plane z+2 at step z).  NB_ZM_L overrides for experiments ("0"/"1").
+static int zm_lookahead(bool smem) {
+    static int env[2] = {-2, -2};
+    int k = smem ? 1 : 0;
+    if (env[k] == -2) {
+        const char *e = getenv(smem ? "NB_ZM_LS" : "NB_ZM_L");
+        env[k] = e ? atoi(e) : -1;
+    }
+    if (env[k] >= 0) return env[k];
+    return smem ? 1 : 0;
+}
+
 template <class Op, bool SMEM = false>
 static nb_status launch_zmarch(nb_grid *g, const char *name, Op op, PGeo geo, int zb, int ze) {
     if (ze <= zb) return NB_OK;
     dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
     LaunchScope ls(g, g->cs, name);
-    k_zmarch<Op, SMEM><<<grd, blk, 0, g->cs>>>(op, geo, zb, ze, g->tp, g->T);
+    if (zm_lookahead(SMEM) == 1)
+        k_zmarch<Op, SMEM, 1><<<grd, blk, 0, g->cs>>>(op, geo, zb, ze, g->tp, g->T);
+    else
+        k_zmarch<Op, SMEM, 0><<<grd, blk, 0, g->cs>>>(op, geo, zb, ze, g->tp, g->T);
     return nb_launch_check(name);
 }
 
@@ -402,8 +418,8 @@ extern "C" nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, i
     // ping-pong partners (the stencil reads neighbours of x and y while the
     // step writes new x and y)
     nb_field *x2 = nullptr, *y2 = nullptr;
-    NB_TRY(nb_field_create(g, NB_F64, 1, 0.0, &x2));
-    nb_status st = nb_field_create(g, NB_F64, 1, 0.0, &y2);
+    NB_TRY(nb_grid_scratch(g, NB_F64, 1, 0, &x2));
+    nb_status st = nb_grid_scratch(g, NB_F64, 1, 1, &y2);
     HaloSync hs;
     nb_field *xin = x, *yin = y, *xo = x2, *yo = y2;
     for (int k = 0; k < iters && st == NB_OK; ++k) {
@@ -436,8 +452,6 @@ extern "C" nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, i
         cudaEventDestroy(hs.eb);
         cudaEventDestroy(hs.eh);
     }
-    nb_field_destroy(x2);
-    nb_field_destroy(y2);
     return st;
 }
 
@@ -541,49 +555,79 @@ extern "C" nb_status nb_cg_create(nb_field *x, const nb_field *b, const nb_cg_pa
     return NB_OK;
 }
 
+static bool cg_eager(const nb_grid *g) {
+    return g->profiling || is_dist(g) || getenv("NB_NO_GRAPH") != nullptr;
+}
+
+constexpr int CG_GRAPH_CHUNK = 16;
+
+// the CUDA graph of n iterations starting at parity `par` (captured once)
+static nb_status cg_graph(nb_cg *cg, int n, int par, std::pair<cudaGraphExec_t, int64_t> **out) {
+    nb_grid *g = cg->g;
+    auto key = std::make_pair(n, par);
+    auto it = cg->graphs.find(key);
+    if (it == cg->graphs.end()) {
+        cudaGraph_t graph;
+        int64_t l0 = g->launches, k0 = cg->k;
+        cg->k = par;  // parity of the first captured iteration is (par + 1) & 1
+        NB_CUDA(cudaStreamBeginCapture(g->cs, cudaStreamCaptureModeThreadLocal));
+        nb_status s = NB_OK;
+        for (int i = 0; i < n && s == NB_OK; ++i) s = cg_enqueue_iteration(cg);
+        cudaError_t e = cudaStreamEndCapture(g->cs, &graph);
+        int64_t nl = g->launches - l0;
+        g->launches = l0;
+        cg->k = k0;
+        if (s != NB_OK) return s;
+        if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "graph capture failed: %s", cudaGetErrorString(e));
+        cudaGraphExec_t exec;
+        e = cudaGraphInstantiate(&exec, graph, 0);
+        cudaGraphDestroy(graph);
+        if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "graph instantiate failed: %s", cudaGetErrorString(e));
+        it = cg->graphs.emplace(key, std::make_pair(exec, nl)).first;
+    }
+    *out = &it->second;
+    return NB_OK;
+}
+
+// walk the chunks nb_cg_iterate(iters) will use; launch them or only build them
+static nb_status cg_run_chunks(nb_cg *cg, int32_t iters, bool launch) {
+    nb_grid *g = cg->g;
+    int64_t k = cg->k;
+    int done = 0;
+    while (done < iters) {
+        int n = std::min(CG_GRAPH_CHUNK, iters - done);
+        std::pair<cudaGraphExec_t, int64_t> *gr = nullptr;
+        NB_TRY(cg_graph(cg, n, (int)(k & 1), &gr));
+        if (launch) {
+            NB_CUDA(cudaGraphLaunch(gr->first, g->cs));
+            g->launches += gr->second;
+        }
+        k += n;
+        done += n;
+    }
+    if (launch) cg->k = k;
+    return NB_OK;
+}
+
 extern "C" nb_status nb_cg_iterate(nb_cg *cg, int32_t iters) {
     if (!cg) NB_FAIL(NB_EINVAL, "nb_cg_iterate: NULL solver");
     if (cg->finished) NB_FAIL(NB_ESTATE, "nb_cg_iterate after nb_cg_finish");
     if (iters < 0) NB_FAIL(NB_EINVAL, "iters < 0");
     nb_grid *g = cg->g;
     cudaSetDevice(g->device);
-    // eager path: profiling, multi-process (NCCL inside), or tiny counts
-    bool eager = g->profiling || is_dist(g) || getenv("NB_NO_GRAPH") != nullptr;
-    if (eager) {
+    if (cg_eager(g)) {  // profiling (per-launch events) or multi-process (NCCL inside)
         for (int i = 0; i < iters; ++i) NB_TRY(cg_enqueue_iteration(cg));
         return NB_OK;
     }
-    // graph path: graphs of up to CHUNK iterations, keyed by (count, parity)
-    const int CHUNK = 16;
-    int done = 0;
-    while (done < iters) {
-        int n = std::min(CHUNK, iters - done);
-        auto key = std::make_pair(n, (int)(cg->k & 1));
-        auto it = cg->graphs.find(key);
-        if (it == cg->graphs.end()) {
-            cudaGraph_t graph;
-            int64_t l0 = g->launches, k0 = cg->k;
-            NB_CUDA(cudaStreamBeginCapture(g->cs, cudaStreamCaptureModeThreadLocal));
-            nb_status s = NB_OK;
-            for (int i = 0; i < n && s == NB_OK; ++i) s = cg_enqueue_iteration(cg);
-            cudaError_t e = cudaStreamEndCapture(g->cs, &graph);
-            int64_t nl = g->launches - l0;
-            g->launches = l0;
-            cg->k = k0;
-            if (s != NB_OK) return s;
-            if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "graph capture failed: %s", cudaGetErrorString(e));
-            cudaGraphExec_t exec;
-            e = cudaGraphInstantiate(&exec, graph, 0);
-            cudaGraphDestroy(graph);
-            if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "graph instantiate failed: %s", cudaGetErrorString(e));
-            it = cg->graphs.emplace(key, std::make_pair(exec, nl)).first;
-        }
-        NB_CUDA(cudaGraphLaunch(it->second.first, g->cs));
-        g->launches += it->second.second;
-        cg->k += n;
-        done += n;
-    }
-    return NB_OK;
+    return cg_run_chunks(cg, iters, true);
+}
+
+extern "C" nb_status nb_cg_prepare(nb_cg *cg, int32_t iters) {
+    if (!cg) NB_FAIL(NB_EINVAL, "nb_cg_prepare: NULL solver");
+    if (iters < 0) NB_FAIL(NB_EINVAL, "iters < 0");
+    cudaSetDevice(cg->g->device);
+    if (cg_eager(cg->g)) return NB_OK;
+    return cg_run_chunks(cg, iters, false);
 }
 
 extern "C" nb_status nb_cg_finish(nb_cg *cg, nb_cg_result *res) {

@@ -41,7 +41,7 @@ __device__ __forceinline__ double add_rn<double>(double a, double b) { return __
 template <>
 __device__ __forceinline__ float add_rn<float>(float a, float b) { return __fadd_rn(a, b); }
 
-template <class Op, bool SMEM>
+template <class Op, bool SMEM, int L>
 __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_zmarch(Op op, PGeo g, int zb, int ze, double *tp, int T) {
     using V = typename Op::T;
     using Raw = typename Op::Raw;
@@ -80,12 +80,12 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_zmarch(Op op, PGeo g, int zb
     if (valid) {
         below = op.val(zs - 1, op.raw(zs - 1, o + (int64_t)(zs - 1) * g.ps, false));
         rc = op.raw(zs, o + (int64_t)zs * g.ps, true);
-        r1 = op.raw(zs + 1, o + (int64_t)(zs + 1) * g.ps, true);
+        if (L == 1) r1 = op.raw(zs + 1, o + (int64_t)(zs + 1) * g.ps, true);
     }
     if (r0in) g0c = op.raw(zs, ro0 + (int64_t)(zs) * g.ps, false);
     if (r1in) g1c = op.raw(zs, ro1 + (int64_t)(zs) * g.ps, false);
-    if (r0in && zs + 1 < zend) g0n = op.raw(zs + 1, ro0 + (int64_t)(zs + 1) * g.ps, false);
-    if (r1in && zs + 1 < zend) g1n = op.raw(zs + 1, ro1 + (int64_t)(zs + 1) * g.ps, false);
+    if (L == 1 && r0in && zs + 1 < zend) g0n = op.raw(zs + 1, ro0 + (int64_t)(zs + 1) * g.ps, false);
+    if (L == 1 && r1in && zs + 1 < zend) g1n = op.raw(zs + 1, ro1 + (int64_t)(zs + 1) * g.ps, false);
     if (valid) center = op.val(zs, rc);
     if (SMEM) {
         sU[0][ty + 1][tx + 1] = center;
@@ -94,11 +94,18 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_zmarch(Op op, PGeo g, int zb
     for (int z = zs; z < zend; ++z) {
         const int b = SMEM ? ((z - zs) & 1) : 0;
         const int64_t ic = o + (int64_t)z * g.ps;
-        // prefetch plane z+2 (own column) and the ring of plane z+2
-        if (valid && z + 2 <= zend) r2 = op.raw(z + 2, ic + 2 * g.ps, true);
+        // L = 1: prefetch plane z+2 (own column and ring) while plane z is
+        // computed; L = 0: load plane z+1 now
         Raw g0f{}, g1f{};
-        if (r0in && z + 2 < zend) g0f = op.raw(z + 2, ro0 + (int64_t)(z + 2) * g.ps, false);
-        if (r1in && z + 2 < zend) g1f = op.raw(z + 2, ro1 + (int64_t)(z + 2) * g.ps, false);
+        if (L == 1) {
+            if (valid && z + 2 <= zend) r2 = op.raw(z + 2, ic + 2 * g.ps, true);
+            if (r0in && z + 2 < zend) g0f = op.raw(z + 2, ro0 + (int64_t)(z + 2) * g.ps, false);
+            if (r1in && z + 2 < zend) g1f = op.raw(z + 2, ro1 + (int64_t)(z + 2) * g.ps, false);
+        } else {
+            if (valid) r1 = op.raw(z + 1, ic + g.ps, true);
+            if (r0in && z + 1 < zend) g0n = op.raw(z + 1, ro0 + (int64_t)(z + 1) * g.ps, false);
+            if (r1in && z + 1 < zend) g1n = op.raw(z + 1, ro1 + (int64_t)(z + 1) * g.ps, false);
+        }
         const V above = valid ? op.val(z + 1, r1) : out;
         if (SMEM) __syncthreads();
         double prod = 0.0;
@@ -130,9 +137,11 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_zmarch(Op op, PGeo g, int zb
         below = center;
         center = above;
         rc = r1;
-        r1 = r2;
-        g0n = g0f;
-        g1n = g1f;
+        if (L == 1) {
+            r1 = r2;
+            g0n = g0f;
+            g1n = g1f;
+        }
     }
     if (Op::DOT) {
         __syncthreads();

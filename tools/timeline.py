@@ -1,0 +1,51 @@
+"""CUPTI kernel timeline (torch.profiler) of a few CG iterations / LBM steps:
+per-kernel device durations and the idle gaps between consecutive kernels.
+  python tools/timeline.py [n] [iters] [cg|lbm] [--out gpurun_out/timeline.json]"""
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+from torch.profiler import ProfilerActivity, profile  # noqa: E402
+
+import paper_conf_ipps_meneghinmjm22_b200 as nb  # noqa: E402
+
+n = int(sys.argv[1]) if len(sys.argv) > 1 else 512
+iters = int(sys.argv[2]) if len(sys.argv) > 2 else 8
+what = sys.argv[3] if len(sys.argv) > 3 else "cg"
+g = nb.Grid((n, n, n))
+if what == "cg":
+    b, x = nb.Field(g), nb.Field(g)
+    b.fill(nb.FILL_POISSON_RHS)
+    x.fill_const(0.0)
+    cg = nb.CG(x, b)
+    cg.iterate(16)
+    g.sync()
+    with profile(activities=[ProfilerActivity.CUDA]) as prof:
+        cg.iterate(iters)
+        g.sync()
+    cg.finish()
+    cg.close()
+else:
+    fa, fb = nb.Field(g, "f32", 19), nb.Field(g, "f32", 19)
+    nb.nb_lbm_init(fa, 1.0, (0, 0, 0))
+    fa, fb = nb.nb_lbm_step(fa, fb, 0.7886, 2)
+    g.sync()
+    with profile(activities=[ProfilerActivity.CUDA]) as prof:
+        fa, fb = nb.nb_lbm_step(fa, fb, 0.7886, iters)
+        g.sync()
+evs = [e for e in prof.events() if e.device_type == torch.autograd.DeviceType.CUDA]
+ks = sorted([(e.time_range.start, e.time_range.end, e.name) for e in evs])
+rows = []
+for i, (s, e, name) in enumerate(ks):
+    gap = s - ks[i - 1][1] if i else 0.0
+    rows.append({"name": name[:50], "start_us": s - ks[0][0], "dur_us": e - s, "gap_us": gap})
+tot = ks[-1][1] - ks[0][0]
+busy = sum(r["dur_us"] for r in rows)
+summary = {"span_us": tot, "busy_us": busy, "idle_us": tot - busy, "kernels": len(rows)}
+print(json.dumps(summary))
+for r in rows[:24]:
+    print(f"{r['name']:50s} dur {r['dur_us']:9.1f} us  gap {r['gap_us']:7.1f} us")
+if "--out" in sys.argv:
+    json.dump({"summary": summary, "kernels": rows}, open(sys.argv[sys.argv.index("--out") + 1], "w"), indent=1)
