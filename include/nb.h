@@ -106,6 +106,28 @@ nb_status nb_partition_plan(int32_t nz, int32_t nparts, int32_t *z_begin);
 nb_status nb_partition_plan_weighted(int32_t nz, const int64_t *counts, int32_t nparts,
                                      int32_t *z_begin);
 
+/* One halo message of the z-slab decomposition (each
+ * partition talks to its two neighbours; 2 transfers per component, no
+ * marshalling). */
+typedef struct {
+    int32_t src_part, dst_part;  /* global partition ids                          */
+    int32_t src_rank, dst_rank;  /* owning processes (equal: a device copy)       */
+    int32_t src_plane;           /* local plane of src sent (0 or nz_src-1)        */
+    int32_t dst_plane;           /* halo plane of dst written (-1 or nz_dst)       */
+    int32_t up;                  /* 1: src's top plane -> dst's low halo; 0: down */
+} nb_halo_msg;
+/* Pure host logic: the halo messages of an nparts-slab decomposition of nz
+ * planes owned by `world` processes (partition p on rank p/(nparts/world)),
+ * restricted to those `rank` sends or receives (rank = -1: all), in the
+ * canonical order every rank posts them in (so point-to-point sends and
+ * receives between two ranks match in order): neighbour pairs (p, p+1) in
+ * increasing p — with periodic != 0 also the ring pair (nparts-1, 0) — and
+ * within a pair the up message before the down message.  count receives the
+ * number of messages; out may be NULL to query it; NB_EINVAL if cap is too
+ * small. */
+nb_status nb_halo_plan(int32_t nz, int32_t nparts, int32_t world, int32_t rank, int32_t periodic,
+                       nb_halo_msg *out, int32_t cap, int32_t *count);
+
 /* Dense grid of dims = {Nx, Ny, Nz} cells split into nparts z-slabs.
  * comm == NULL: every partition lives in this process; device_ids[nparts]
  *   gives each partition's device and must name ONE device (virtual

@@ -73,6 +73,7 @@ SIGNATURES = {
     "nb_comm_destroy": ([P], I32),
     "nb_partition_plan": ([I32, I32, P], I32),
     "nb_partition_plan_weighted": ([I32, P, I32, P], I32),
+    "nb_halo_plan": ([I32, I32, I32, I32, I32, P, I32, P], I32),
     "nb_grid_create_dense": ([P, I32, P, P, PP], I32),
     "nb_grid_create_sparse": ([P, P, I32, P, P, PP], I32),
     "nb_grid_destroy": ([P], I32),
@@ -168,6 +169,20 @@ def nb_partition_plan_weighted(counts, nparts: int) -> list:
     zb = (C.c_int32 * (nparts + 1))()
     _check(lib().nb_partition_plan_weighted(len(c), c.ctypes.data_as(P), nparts, zb))
     return list(zb)
+
+
+class HaloMsg(C.Structure):
+    _fields_ = [("src_part", C.c_int32), ("dst_part", C.c_int32), ("src_rank", C.c_int32),
+                ("dst_rank", C.c_int32), ("src_plane", C.c_int32), ("dst_plane", C.c_int32), ("up", C.c_int32)]
+
+
+def nb_halo_plan(nz: int, nparts: int, world: int = 1, rank: int = -1, periodic: bool = False) -> list:
+    """Halo messages (dicts) this rank posts, in the canonical order."""
+    n = C.c_int32()
+    _check(lib().nb_halo_plan(nz, nparts, world, rank, int(periodic), None, 0, C.byref(n)))
+    arr = (HaloMsg * max(n.value, 1))()
+    _check(lib().nb_halo_plan(nz, nparts, world, rank, int(periodic), arr, n.value, C.byref(n)))
+    return [{k: getattr(m, k) for k, _ in HaloMsg._fields_} for m in arr[:n.value]]
 
 
 # ---------------------------------------------------------------------------

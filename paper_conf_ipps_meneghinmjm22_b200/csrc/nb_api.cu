@@ -243,6 +243,86 @@ extern "C" nb_status nb_partition_plan_weighted(int32_t nz, const int64_t *count
     return NB_OK;
 }
 
+extern "C" nb_status nb_halo_plan(int32_t nz, int32_t nparts, int32_t world, int32_t rank, int32_t periodic,
+                                   nb_halo_msg *out, int32_t cap, int32_t *count) {
+    if (!count || nparts < 1 || world < 1 || nparts % world != 0 || rank < -1 || rank >= world)
+        NB_FAIL(NB_EINVAL, "nb_halo_plan: bad arguments");
+    std::vector<int32_t> zb(nparts + 1);
+    NB_TRY(nb_partition_plan(nz, nparts, zb.data()));
+    const int k = nparts / world;
+    int n = 0;
+    auto emit = [&](int src, int dst, int up) -> bool {
+        int sr = src / k, dr = dst / k;
+        if (rank != -1 && sr != rank && dr != rank) return true;
+        if (out) {
+            if (n >= cap) return false;
+            nb_halo_msg &m = out[n];
+            m.src_part = src;
+            m.dst_part = dst;
+            m.src_rank = sr;
+            m.dst_rank = dr;
+            m.src_plane = up ? zb[src + 1] - zb[src] - 1 : 0;
+            m.dst_plane = up ? -1 : zb[dst + 1] - zb[dst];
+            m.up = up;
+        }
+        ++n;
+        return true;
+    };
+    for (int p = 0; p < nparts; ++p) {
+        int q = p + 1;
+        if (q == nparts) {
+            if (!periodic) break;
+            q = 0;
+        }
+        // pair (p below, q above): p's top -> q's low halo; q's bottom -> p's high halo
+        if (!emit(p, q, 1) || !emit(q, p, 0)) NB_FAIL(NB_EINVAL, "nb_halo_plan: cap %d too small", cap);
+    }
+    *count = n;
+    return NB_OK;
+}
+
+// Execute the halo messages of field f for this process: local messages are
+// device copies, remote ones grouped NCCL send/recv on stream s.  comps(up)
+// gives the component range [c0, c1) carried by up / down messages.
+nb_status nb_halo_run(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int c1d, cudaStream_t s) {
+    nb_grid *g = f->g;
+    int world = g->comm ? g->comm->world : 1, rank = g->comm ? g->comm->rank : 0;
+    int cnt = 0;
+    NB_TRY(nb_halo_plan(g->nz, g->nparts, world, rank, periodic, nullptr, 0, &cnt));
+    std::vector<nb_halo_msg> msgs(cnt);
+    NB_TRY(nb_halo_plan(g->nz, g->nparts, world, rank, periodic, msgs.data(), cnt, &cnt));
+    size_t pb = (size_t)f->ps * f->esz;
+    auto cs_of = [&](int p) { return f->ps * (g->parts[p].nz() + 2); };
+    auto plane_addr = [&](int p, int c, int zl) {
+        return f->base[p] + ((int64_t)c * cs_of(p) + (int64_t)(zl + 1) * f->ps) * f->esz;
+    };
+    bool remote = false;
+    for (auto &m : msgs) {
+        int c0 = m.up ? c0u : c0d, c1 = m.up ? c1u : c1d;
+        if (m.src_rank == rank && m.dst_rank == rank) {
+            for (int c = c0; c < c1; ++c)
+                NB_CUDA(cudaMemcpyAsync(plane_addr(m.dst_part, c, m.dst_plane), plane_addr(m.src_part, c, m.src_plane),
+                                        pb, cudaMemcpyDeviceToDevice, s));
+        } else {
+            remote = true;
+        }
+    }
+    if (!remote) return NB_OK;
+    NB_TRY(nb_nccl_group(g, true));
+    for (auto &m : msgs) {
+        if (m.src_rank == rank && m.dst_rank == rank) continue;
+        int c0 = m.up ? c0u : c0d, c1 = m.up ? c1u : c1d;
+        for (int c = c0; c < c1; ++c) {
+            if (m.src_rank == rank)
+                NB_TRY(nb_nccl_send(g, plane_addr(m.src_part, c, m.src_plane), pb, m.dst_rank, s));
+            else
+                NB_TRY(nb_nccl_recv(g, plane_addr(m.dst_part, c, m.dst_plane), pb, m.src_rank, s));
+        }
+    }
+    NB_TRY(nb_nccl_group(g, false));
+    return NB_OK;
+}
+
 // ===========================================================================
 // grid
 // ===========================================================================
@@ -683,67 +763,7 @@ extern "C" nb_status nb_field_fill(nb_field *f, nb_fill kind, uint64_t seed, dou
 // send_down: my first plane -> lower neighbour's high halo.
 nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down,
                                   cudaStream_t s) {
-    nb_grid *g = f->g;
-    size_t pbytes = (size_t)f->ps * f->esz;
-    bool any_remote = false;
-    for (int p = 0; p < g->nparts; ++p) {
-        if (!g->parts[p].local) continue;
-        const NbPart &q = g->parts[p];
-        for (int c = c0; c < c1; ++c) {
-            if (send_up && q.hi >= 0) {
-                const char *src = f->base[p] + ((int64_t)c * dense_cs(f, p) + (int64_t)q.nz() * f->ps) * f->esz;
-                if (g->parts[q.hi].local) {
-                    char *dst = f->base[q.hi] + ((int64_t)c * dense_cs(f, q.hi)) * f->esz;  // zl = -1
-                    NB_CUDA(cudaMemcpyAsync(dst, src, pbytes, cudaMemcpyDeviceToDevice, s));
-                } else {
-                    any_remote = true;
-                }
-            }
-            if (send_down && q.lo >= 0) {
-                const char *src = f->base[p] + ((int64_t)c * dense_cs(f, p) + f->ps) * f->esz;
-                if (g->parts[q.lo].local) {
-                    int nzn = g->parts[q.lo].nz();
-                    char *dst = f->base[q.lo] + ((int64_t)c * dense_cs(f, q.lo) + (int64_t)(nzn + 1) * f->ps) * f->esz;
-                    NB_CUDA(cudaMemcpyAsync(dst, src, pbytes, cudaMemcpyDeviceToDevice, s));
-                } else {
-                    any_remote = true;
-                }
-            }
-        }
-    }
-    if (!any_remote) return NB_OK;
-    // cross-process transfers: grouped NCCL send/recv over NVLink
-    NB_TRY(nb_nccl_group(g, true));
-    for (int p = 0; p < g->nparts; ++p) {
-        if (!g->parts[p].local) continue;
-        const NbPart &q = g->parts[p];
-        for (int c = c0; c < c1; ++c) {
-            if (q.hi >= 0 && !g->parts[q.hi].local) {
-                int peer = nb_part_owner(g, q.hi);
-                if (send_up) {
-                    const char *src = f->base[p] + ((int64_t)c * dense_cs(f, p) + (int64_t)q.nz() * f->ps) * f->esz;
-                    NB_TRY(nb_nccl_send(g, src, pbytes, peer, s));
-                }
-                if (send_down) {  // the upper neighbour sends me its first plane -> my high halo
-                    char *dst = f->base[p] + ((int64_t)c * dense_cs(f, p) + (int64_t)(q.nz() + 1) * f->ps) * f->esz;
-                    NB_TRY(nb_nccl_recv(g, dst, pbytes, peer, s));
-                }
-            }
-            if (q.lo >= 0 && !g->parts[q.lo].local) {
-                int peer = nb_part_owner(g, q.lo);
-                if (send_down) {
-                    const char *src = f->base[p] + ((int64_t)c * dense_cs(f, p) + f->ps) * f->esz;
-                    NB_TRY(nb_nccl_send(g, src, pbytes, peer, s));
-                }
-                if (send_up) {  // the lower neighbour sends me its last plane -> my low halo
-                    char *dst = f->base[p] + ((int64_t)c * dense_cs(f, p)) * f->esz;
-                    NB_TRY(nb_nccl_recv(g, dst, pbytes, peer, s));
-                }
-            }
-        }
-    }
-    NB_TRY(nb_nccl_group(g, false));
-    return NB_OK;
+    return nb_halo_run(f, false, send_up ? c0 : 0, send_up ? c1 : 0, send_down ? c0 : 0, send_down ? c1 : 0, s);
 }
 
 nb_status nb_sparse_halo_update(nb_field *f);

@@ -203,6 +203,7 @@ nb_status nb_grid_scratch(nb_grid *g, nb_dtype dt, int card, int slot, nb_field 
 // halo helpers (nb_api.cu)
 nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down,
                                   cudaStream_t s);
+nb_status nb_halo_run(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int c1d, cudaStream_t s);
 nb_status nb_nccl_allreduce_sum(nb_grid *g, const double *send, double *recv, size_t n,
                                 cudaStream_t s);
 nb_status nb_nccl_group(nb_grid *g, bool start);

@@ -203,59 +203,10 @@ static int lbm_hi(const nb_grid *g, int p, bool per) {
 
 // Halo of the 10 populations that cross z faces: my last plane's c_z=+1
 // populations (9..13) -> upper neighbour's low halo; my first plane's c_z=-1
-// populations (14..18) -> lower neighbour's high halo.  Local partners:
-// device copies; remote partners: grouped NCCL send/recv.
-static nb_status lbm_halo(nb_field *f, bool per, cudaStream_t s) {
-    nb_grid *g = f->g;
-    size_t pb = (size_t)f->ps * 4;
-    bool remote = false;
-    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
-        int hi = lbm_hi(g, p, per), lo = lbm_lo(g, p, per);
-        int nz = g->parts[p].nz();
-        float *b = (float *)f->base[p];
-        if (hi >= 0) {
-            if (g->parts[hi].local) {
-                float *d = (float *)f->base[hi];
-                for (int i = 9; i < 14; ++i)
-                    NB_CUDA(cudaMemcpyAsync(d + i * lcs(f, hi), b + i * lcs(f, p) + (int64_t)nz * f->ps, pb,
-                                            cudaMemcpyDeviceToDevice, s));
-            } else {
-                remote = true;
-            }
-        }
-        if (lo >= 0) {
-            if (g->parts[lo].local) {
-                float *d = (float *)f->base[lo];
-                int nzl = g->parts[lo].nz();
-                for (int i = 14; i < 19; ++i)
-                    NB_CUDA(cudaMemcpyAsync(d + i * lcs(f, lo) + (int64_t)(nzl + 1) * f->ps, b + i * lcs(f, p) + f->ps,
-                                            pb, cudaMemcpyDeviceToDevice, s));
-            } else {
-                remote = true;
-            }
-        }
-    }
-    if (!remote) return NB_OK;
-    NB_TRY(nb_nccl_group(g, true));
-    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
-        int hi = lbm_hi(g, p, per), lo = lbm_lo(g, p, per);
-        int nz = g->parts[p].nz();
-        float *b = (float *)f->base[p];
-        if (hi >= 0 && !g->parts[hi].local) {
-            int peer = nb_part_owner(g, hi);
-            for (int i = 9; i < 14; ++i) NB_TRY(nb_nccl_send(g, b + i * lcs(f, p) + (int64_t)nz * f->ps, pb, peer, s));
-            for (int i = 14; i < 19; ++i)
-                NB_TRY(nb_nccl_recv(g, b + i * lcs(f, p) + (int64_t)(nz + 1) * f->ps, pb, peer, s));
-        }
-        if (lo >= 0 && !g->parts[lo].local) {
-            int peer = nb_part_owner(g, lo);
-            for (int i = 14; i < 19; ++i) NB_TRY(nb_nccl_send(g, b + i * lcs(f, p) + f->ps, pb, peer, s));
-            for (int i = 9; i < 14; ++i) NB_TRY(nb_nccl_recv(g, b + i * lcs(f, p), pb, peer, s));
-        }
-    }
-    NB_TRY(nb_nccl_group(g, false));
-    return NB_OK;
-}
+// populations (14..18) -> lower neighbour's high halo (ring when periodic).
+// Local partners: device copies; remote partners: grouped NCCL send/recv in
+// the canonical order of nb_halo_plan.
+static nb_status lbm_halo(nb_field *f, bool per, cudaStream_t s) { return nb_halo_run(f, per, 9, 14, 14, 19, s); }
 
 static nb_status launch_lbm(nb_grid *g, int p, nb_field *fin, nb_field *fout, const nb_lbm_params *prm, int zb,
                             int ze, bool remote_stores) {
