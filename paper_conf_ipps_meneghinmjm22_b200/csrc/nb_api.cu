@@ -326,14 +326,14 @@ nb_status nb_halo_run(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int
 // ===========================================================================
 // grid
 // ===========================================================================
-static nb_status grid_alloc_common(nb_grid *g) {
+nb_status nb_grid_alloc_common(nb_grid *g) {
     DeviceGuard dg(g->device);
     NB_CUDA(cudaStreamCreateWithFlags(&g->cs, cudaStreamNonBlocking));
     NB_CUDA(cudaStreamCreateWithFlags(&g->hs, cudaStreamNonBlocking));
     g->own_cs = g->own_hs = true;
     g->tiles_x = (g->nx + DOT_TX - 1) / DOT_TX;
     g->tiles_y = (g->ny + DOT_TY - 1) / DOT_TY;
-    g->T = g->tiles_x * g->tiles_y;
+    if (!g->sparse) g->T = g->tiles_x * g->tiles_y;  // sparse: set by the builder (segments per plane)
     size_t planes = (size_t)g->max_card * g->nz;
     NB_CUDA(cudaMalloc(&g->tp, sizeof(double) * planes * g->T));
     NB_CUDA(cudaMalloc(&g->psum, sizeof(double) * planes));
@@ -404,7 +404,7 @@ extern "C" nb_status nb_grid_create_dense(const int32_t dims[3], int32_t nparts,
     g->ny = dims[1];
     g->nz = dims[2];
     nb_status s = nb_grid_setup_parts(g, zb.data(), nparts, device_ids, comm);
-    if (s == NB_OK) s = grid_alloc_common(g);
+    if (s == NB_OK) s = nb_grid_alloc_common(g);
     if (s != NB_OK) {
         nb_grid_destroy(g);
         return s;
@@ -628,7 +628,7 @@ extern "C" nb_status nb_field_partition_ptr(const nb_field *f, int32_t p, void *
     if (ptr) *ptr = f->base[p];
     if (pitch) *pitch = f->pitch;
     if (pstride) *pstride = f->ps;
-    if (cstride) *cstride = f->g->sparse ? f->cs : dense_cs(f, p);
+    if (cstride) *cstride = f->g->sparse ? f->pcs[p] : dense_cs(f, p);
     return NB_OK;
 }
 
@@ -681,40 +681,7 @@ extern "C" nb_status nb_field_download(const nb_field *f, void *host, int64_t nb
     return NB_OK;
 }
 
-// ---- counter-based fill (same generator as synth/, own implementation) -----
-__device__ __forceinline__ uint64_t nb_mix64(uint64_t z) {
-    z ^= z >> 30;
-    z *= 0xBF58476D1CE4E5B9ull;
-    z ^= z >> 27;
-    z *= 0x94D049BB133111EBull;
-    z ^= z >> 31;
-    return z;
-}
-
-__device__ __forceinline__ double nb_gen(int kind, uint64_t seed, uint64_t gidx, double a, double b,
-                                         int x, int y, int z, double h) {
-    if (kind == NB_FILL_CONST) return a;
-    if (kind == NB_FILL_POISSON_RHS) {
-        // b = (h*h) * (((gy*gz + gx*gz) + gx*gy) * 2), g(t) = t*(1-t), t = (i+1)*h
-        double tx = __dmul_rn((double)(x + 1), h), ty = __dmul_rn((double)(y + 1), h),
-               tz = __dmul_rn((double)(z + 1), h);
-        double gx = __dmul_rn(tx, __dsub_rn(1.0, tx)), gy = __dmul_rn(ty, __dsub_rn(1.0, ty)),
-               gz = __dmul_rn(tz, __dsub_rn(1.0, tz));
-        double f = __dadd_rn(__dadd_rn(__dmul_rn(gy, gz), __dmul_rn(gx, gz)), __dmul_rn(gx, gy));
-        f = __dmul_rn(f, 2.0);
-        return __dmul_rn(__dmul_rn(h, h), f);
-    }
-    uint64_t hsh = nb_mix64(seed * 0x9E3779B97F4A7C15ull + gidx + 1ull);
-    if (kind == NB_FILL_UNIFORM) {
-        double u = (double)(hsh >> 11) * 0x1p-53;
-        return __dadd_rn(a, __dmul_rn(__dsub_rn(b, a), u));
-    }
-    // INT_UNIFORM: a + (h mod (b - a + 1))
-    int64_t lo = (int64_t)a, hi = (int64_t)b;
-    uint64_t span = (uint64_t)(hi - lo + 1);
-    return (double)((int64_t)(hsh % span) + lo);
-}
-
+// ---- counter-based fill: nb_gen in nb_device.cuh ----------------------------
 template <typename T>
 __global__ void k_fill_gen(T *base, PGeo g, int64_t cstride, int card, int kind, uint64_t seed,
                            double a, double b, double h) {

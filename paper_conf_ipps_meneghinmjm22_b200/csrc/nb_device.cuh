@@ -62,3 +62,38 @@ __device__ __forceinline__ void tile_stage_flush(const TileStage<ZC> &st, int np
         tp[(pbase + t) * (int64_t)T + tile] = s;
     }
 }
+
+// ---- counter-based fill (same generator as synth/, own implementation) -----
+__device__ __forceinline__ uint64_t nb_mix64(uint64_t z) {
+    z ^= z >> 30;
+    z *= 0xBF58476D1CE4E5B9ull;
+    z ^= z >> 27;
+    z *= 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    return z;
+}
+
+__device__ __forceinline__ double nb_gen(int kind, uint64_t seed, uint64_t gidx, double a, double b,
+                                         int x, int y, int z, double h) {
+    if (kind == NB_FILL_CONST) return a;
+    if (kind == NB_FILL_POISSON_RHS) {
+        // b = (h*h) * (((gy*gz + gx*gz) + gx*gy) * 2), g(t) = t*(1-t), t = (i+1)*h
+        double tx = __dmul_rn((double)(x + 1), h), ty = __dmul_rn((double)(y + 1), h),
+               tz = __dmul_rn((double)(z + 1), h);
+        double gx = __dmul_rn(tx, __dsub_rn(1.0, tx)), gy = __dmul_rn(ty, __dsub_rn(1.0, ty)),
+               gz = __dmul_rn(tz, __dsub_rn(1.0, tz));
+        double f = __dadd_rn(__dadd_rn(__dmul_rn(gy, gz), __dmul_rn(gx, gz)), __dmul_rn(gx, gy));
+        f = __dmul_rn(f, 2.0);
+        return __dmul_rn(__dmul_rn(h, h), f);
+    }
+    uint64_t hsh = nb_mix64(seed * 0x9E3779B97F4A7C15ull + gidx + 1ull);
+    if (kind == NB_FILL_UNIFORM) {
+        double u = (double)(hsh >> 11) * 0x1p-53;
+        return __dadd_rn(a, __dmul_rn(__dsub_rn(b, a), u));
+    }
+    // INT_UNIFORM: a + (h mod (b - a + 1))
+    int64_t lo = (int64_t)a, hi = (int64_t)b;
+    uint64_t span = (uint64_t)(hi - lo + 1);
+    return (double)((int64_t)(hsh % span) + lo);
+}
+

@@ -78,14 +78,18 @@ struct ProfRec {
     cudaEvent_t a, b;
 };
 
-// sparse partition device data (element-sparse grid)
+// element-sparse partition: the active cells of the
+// slab in (z, y, x) order.  Field buffers hold [halo_lo | own | halo_hi]
+// per component: halo_lo = the lower neighbour's last-plane cells, halo_hi =
+// the upper neighbour's first-plane cells (same (y, x) order), so every halo
+// transfer is one contiguous segment (no marshalling).
 struct NbSparsePart {
-    int32_t *conn = nullptr;     // [6][n_act] neighbour local slot (incl. halo), -1 = outside
-    int32_t *coord = nullptr;    // [n_act] packed (x | y<<16), local plane id in plane_of
-    int32_t *plane_of = nullptr; // [n_act] local plane zl
-    int64_t *plane_start = nullptr;  // host copy: [nz+1] local slot offsets per plane
-    std::vector<int64_t> h_plane_start;
-    int32_t *tile_of = nullptr;  // [n_act] canonical dot tile id within (c, z)
+    int64_t hl = 0, n = 0, hh = 0, cs = 0;  // halo lo / own / halo hi cells; component stride
+    std::vector<int64_t> pstart;            // own-slot offset of each local plane [nz_p + 1]
+    int64_t *d_pstart = nullptr;            // device copy
+    int32_t *conn = nullptr;                // [6][n] buffer index of the neighbour, -1 = outside
+    int32_t *coord = nullptr;               // [n] x | y << 16
+    int max_plane = 0;                      // max active cells in one local plane
 };
 
 struct nb_grid {
@@ -115,6 +119,7 @@ struct nb_grid {
     // element-sparse
     std::vector<NbSparsePart> sp;
     std::vector<int64_t> plane_count;  // [nz] active per global plane
+    int64_t n_active = 0;
 };
 
 constexpr int NB_DOT_SLOTS = 1024;
@@ -128,6 +133,7 @@ struct nb_field {
     int64_t pitch = 0, ps = 0, cs = 0;  // elements: row pitch, plane stride, component stride
     std::vector<char *> base;          // per partition (local only)
     std::vector<size_t> bytes;
+    std::vector<int64_t> pcs;          // per-partition component stride (elements)
 };
 
 // per-partition geometry handed to kernels (dense)
@@ -197,6 +203,9 @@ struct CgScal {
     int32_t iters, status, pending, pad;
 };
 
+nb_status nb_grid_alloc_common(nb_grid *g);
+nb_status nb_grid_setup_parts(nb_grid *g, const int32_t *zb, int32_t nparts, const int32_t *device_ids,
+                              nb_comm *comm);
 // cached internal field of the grid (slot distinguishes several of one kind)
 nb_status nb_grid_scratch(nb_grid *g, nb_dtype dt, int card, int slot, nb_field **out);
 

@@ -1,23 +1,662 @@
-// nb_sparse.cu — element-sparse grid.  Placeholder:
-// the element-sparse grid is the next §8 row (a9) to build.
+// nb_sparse.cu — element-sparse grid ("element-sparse, where
+// only cells of interest are stored with their connectivity table"; L256:
+// boundary cells in contiguous segments, two transfers per partition, no
+// marshalling; L472: dense vs sparse trade-off).  SURVEY.md §8(a) a9.
+//
+// Layout per partition and component: [halo_lo | own | halo_hi] where own =
+// the slab's active cells in (z, y, x) order, halo_lo / halo_hi = the active
+// cells of the neighbours' adjacent planes in (y, x) order.  The connectivity
+// table conn[d][j] (d = -x, +x, -y, +y, -z, +z) holds the buffer index of the
+// neighbour of own cell j, or -1 for an inactive / out-of-domain neighbour
+// (read as outside).  Built on the device: an exclusive scan (CUB) of the
+// slab mask numbers the active cells directly in buffer order.
+//
+// Canonical dot order (sparse): per plane (c, z), the plane's active cells
+// in (y, x) order are cut into 256-cell segments; a segment is reduced by
+// xor-butterflies over warps then the 8 warps in order; segment values, then
+// plane sums, by the fixed block tree of nb_reduce_finalize.  Independent of
+// the partitioning (a plane's cells and their order do not depend on it).
+#include <cub/device/device_scan.cuh>
+#include <cub/iterator/transform_input_iterator.cuh>
+
+#include <algorithm>
+#include <vector>
+
+#include "nb_device.cuh"
 #include "nb_internal.cuh"
 
-void nb_sparse_free(nb_grid *g) { (void)g; }
-nb_status nb_sparse_field_alloc(nb_field *) { NB_FAIL(NB_EUNSUPPORTED, "element-sparse grid not built yet"); }
-nb_status nb_sparse_upload(nb_field *, const void *) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
-nb_status nb_sparse_download(const nb_field *, void *) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
-nb_status nb_sparse_fill(nb_field *, nb_fill, uint64_t, double, double) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
-nb_status nb_sparse_halo_update(nb_field *) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
-nb_status nb_sparse_axpby(double, const nb_field *, double, nb_field *, nb_view) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
-nb_status nb_sparse_dot_partials(const nb_field *, const nb_field *) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
-nb_status nb_sparse_laplace7(const nb_field *, nb_field *, nb_view) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
-nb_status nb_sparse_cg_hooks(nb_cg *, int) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
-nb_status nb_sparse_cg_init(nb_cg *) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
-nb_status nb_sparse_cg_flush(nb_cg *) { NB_FAIL(NB_EUNSUPPORTED, "sparse"); }
+constexpr int SEG = 256;
+
+std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v);
+
+namespace {
+struct MaskToInt {
+    __host__ __device__ int operator()(uint8_t v) const { return v ? 1 : 0; }
+};
+}  // namespace
+
+void nb_sparse_free(nb_grid *g) {
+    for (auto &s : g->sp) {
+        cudaFree(s.conn);
+        cudaFree(s.coord);
+        cudaFree(s.d_pstart);
+        s.conn = s.coord = nullptr;
+        s.d_pstart = nullptr;
+    }
+}
+
+__global__ void k_sp_conn(const uint8_t *__restrict__ mask, const int32_t *__restrict__ map, int nx, int ny,
+                          int slab_z0, int nslab, int z0, int NZ, int hl, int64_t n, int32_t *conn, int32_t *coord) {
+    const int x = blockIdx.x * blockDim.x + threadIdx.x, y = blockIdx.y, z = z0 + blockIdx.z;
+    if (x >= nx) return;
+    const int64_t plane = (int64_t)nx * ny;
+    const int64_t cell = (int64_t)(z - slab_z0) * plane + (int64_t)y * nx + x;
+    if (!mask[cell]) return;
+    const int64_t j = (int64_t)map[cell] - hl;
+    coord[j] = x | (y << 16);
+    const int dx[6] = {-1, 1, 0, 0, 0, 0}, dy[6] = {0, 0, -1, 1, 0, 0}, dz[6] = {0, 0, 0, 0, -1, 1};
+#pragma unroll
+    for (int d = 0; d < 6; ++d) {
+        int xx = x + dx[d], yy = y + dy[d], zz = z + dz[d];
+        int32_t v = -1;
+        if (xx >= 0 && xx < nx && yy >= 0 && yy < ny && zz >= 0 && zz < NZ && zz - slab_z0 >= 0 &&
+            zz - slab_z0 < nslab) {
+            int64_t nc = (int64_t)(zz - slab_z0) * plane + (int64_t)yy * nx + xx;
+            if (mask[nc]) v = map[nc];
+        }
+        conn[(int64_t)d * n + j] = v;
+    }
+}
 
 extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t *active, int32_t nparts,
                                            const int32_t *device_ids, nb_comm *comm, nb_grid **out) {
-    (void)dims; (void)active; (void)nparts; (void)device_ids; (void)comm;
-    if (out) *out = nullptr;
-    NB_FAIL(NB_EUNSUPPORTED, "element-sparse grid not built yet");
+    if (!out || !dims || !active) NB_FAIL(NB_EINVAL, "nb_grid_create_sparse: NULL argument");
+    *out = nullptr;
+    if (dims[0] < 1 || dims[1] < 1 || dims[2] < 1 || dims[0] > 65535 || dims[1] > 32767)
+        NB_FAIL(NB_EINVAL, "nb_grid_create_sparse: bad dims");
+    const int nx = dims[0], ny = dims[1], nz = dims[2];
+    const int64_t plane = (int64_t)nx * ny;
+    std::vector<int64_t> counts(nz, 0);
+    for (int z = 0; z < nz; ++z) {
+        const uint8_t *m = active + z * plane;
+        int64_t c = 0;
+        for (int64_t i = 0; i < plane; ++i) c += m[i] != 0;
+        counts[z] = c;
+    }
+    if (nparts < 1 || nparts > nz) NB_FAIL(NB_EINVAL, "nb_grid_create_sparse: bad nparts %d", nparts);
+    std::vector<int32_t> zb(nparts + 1);
+    NB_TRY(nb_partition_plan_weighted(nz, counts.data(), nparts, zb.data()));
+    if (nparts > 1)
+        for (int p = 0; p < nparts; ++p)
+            if (zb[p + 1] - zb[p] < 2) NB_FAIL(NB_EUNSUPPORTED, "sparse slab %d has < 2 planes", p);
+    nb_grid *g = new nb_grid();
+    g->sparse = true;
+    g->nx = nx;
+    g->ny = ny;
+    g->nz = nz;
+    g->plane_count = counts;
+    int64_t maxc = 1;
+    for (auto c : counts) {
+        g->n_active += c;
+        maxc = std::max(maxc, c);
+    }
+    g->T = (int)((maxc + SEG - 1) / SEG);
+    nb_status s = nb_grid_setup_parts(g, zb.data(), nparts, device_ids, comm);
+    if (s == NB_OK) s = nb_grid_alloc_common(g);
+    if (s != NB_OK) {
+        nb_grid_destroy(g);
+        return s;
+    }
+    g->sp.resize(nparts);
+    int64_t a0 = 0;
+    for (int p = 0; p < nparts; ++p) {
+        NbPart &q = g->parts[p];
+        q.a0 = a0;
+        q.n_act = 0;
+        for (int z = q.z0; z < q.z1; ++z) q.n_act += counts[z];
+        a0 += q.n_act;
+        q.n_lo_bnd = q.lo >= 0 ? counts[q.z0] : 0;
+        q.n_hi_bnd = q.hi >= 0 ? counts[q.z1 - 1] : 0;
+        q.halo_lo = q.lo >= 0 ? counts[q.z0 - 1] : 0;
+        q.halo_hi = q.hi >= 0 ? counts[q.z1] : 0;
+        NbSparsePart &sp = g->sp[p];
+        sp.hl = q.halo_lo;
+        sp.n = q.n_act;
+        sp.hh = q.halo_hi;
+        sp.cs = std::max<int64_t>(32, (sp.hl + sp.n + sp.hh + 31) / 32 * 32);
+        sp.pstart.assign(q.nz() + 1, 0);
+        for (int z = q.z0; z < q.z1; ++z) {
+            sp.pstart[z - q.z0 + 1] = sp.pstart[z - q.z0] + counts[z];
+            sp.max_plane = std::max<int>(sp.max_plane, (int)counts[z]);
+        }
+    }
+    cudaSetDevice(g->device);
+    for (int p = g->first_local; p < g->first_local + g->nlocal && s == NB_OK; ++p) {
+        NbPart &q = g->parts[p];
+        NbSparsePart &sp = g->sp[p];
+        const int slab_z0 = q.z0 - (q.lo >= 0 ? 1 : 0), slab_z1 = q.z1 + (q.hi >= 0 ? 1 : 0);
+        const int nslab = slab_z1 - slab_z0;
+        const int64_t ncell = (int64_t)nslab * plane;
+        uint8_t *d_mask = nullptr;
+        int32_t *d_map = nullptr;
+        void *tmp = nullptr;
+        size_t tmp_bytes = 0;
+        auto fail = [&](const char *what, cudaError_t e) {
+            nb_set_error("nb_grid_create_sparse: %s: %s", what, cudaGetErrorString(e));
+            s = NB_ECUDA;
+        };
+        cudaError_t e;
+        if ((e = cudaMalloc(&d_mask, ncell)) != cudaSuccess) fail("cudaMalloc mask", e);
+        if (s == NB_OK && (e = cudaMalloc(&d_map, ncell * 4)) != cudaSuccess) fail("cudaMalloc map", e);
+        if (s == NB_OK && (e = cudaMemcpyAsync(d_mask, active + (int64_t)slab_z0 * plane, ncell,
+                                               cudaMemcpyHostToDevice, g->cs)) != cudaSuccess)
+            fail("mask upload", e);
+        cub::TransformInputIterator<int, MaskToInt, const uint8_t *> it(d_mask, MaskToInt());
+        if (s == NB_OK) {
+            cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, it, d_map, ncell, g->cs);
+            if ((e = cudaMalloc(&tmp, tmp_bytes)) != cudaSuccess) fail("cudaMalloc scan temp", e);
+        }
+        if (s == NB_OK && (e = cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, it, d_map, ncell, g->cs)) != cudaSuccess)
+            fail("scan", e);
+        if (s == NB_OK && (e = cudaMalloc(&sp.conn, sizeof(int32_t) * 6 * std::max<int64_t>(sp.n, 1))) != cudaSuccess)
+            fail("cudaMalloc conn", e);
+        if (s == NB_OK && (e = cudaMalloc(&sp.coord, sizeof(int32_t) * std::max<int64_t>(sp.n, 1))) != cudaSuccess)
+            fail("cudaMalloc coord", e);
+        if (s == NB_OK && (e = cudaMalloc(&sp.d_pstart, sizeof(int64_t) * sp.pstart.size())) != cudaSuccess)
+            fail("cudaMalloc pstart", e);
+        if (s == NB_OK)
+            cudaMemcpyAsync(sp.d_pstart, sp.pstart.data(), sizeof(int64_t) * sp.pstart.size(), cudaMemcpyHostToDevice,
+                            g->cs);
+        if (s == NB_OK && q.nz() > 0) {
+            dim3 blk(128), grd((nx + 127) / 128, ny, q.nz());
+            LaunchScope ls(g, g->cs, "k_sp_conn");
+            k_sp_conn<<<grd, blk, 0, g->cs>>>(d_mask, d_map, nx, ny, slab_z0, nslab, q.z0, nz, (int)sp.hl, sp.n,
+                                              sp.conn, sp.coord);
+            s = nb_launch_check("k_sp_conn");
+        }
+        cudaStreamSynchronize(g->cs);
+        cudaFree(d_mask);
+        cudaFree(d_map);
+        cudaFree(tmp);
+    }
+    if (s != NB_OK) {
+        nb_grid_destroy(g);
+        return s;
+    }
+    *out = g;
+    return NB_OK;
+}
+
+// ---------------------------------------------------------------------------
+// fields
+// ---------------------------------------------------------------------------
+template <typename T>
+__global__ void k_sp_fill_const(T *p, int64_t n, T v) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = v;
+}
+
+nb_status nb_sparse_field_alloc(nb_field *f) {
+    nb_grid *g = f->g;
+    f->pcs.assign(g->nparts, 0);
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbSparsePart &sp = g->sp[p];
+        f->pcs[p] = sp.cs;
+        size_t bytes = (size_t)sp.cs * f->card * f->esz;
+        cudaError_t e = cudaMalloc(&f->base[p], bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            NB_FAIL(NB_ENOMEM, "nb_field_create (sparse): cudaMalloc(%zu) failed", bytes);
+        }
+        f->bytes[p] = bytes;
+        if (f->outside == 0.0) {
+            NB_CUDA(cudaMemsetAsync(f->base[p], 0, bytes, g->cs));
+        } else {
+            int64_t n = (int64_t)(bytes / f->esz);
+            LaunchScope ls(g, g->cs, "k_fill_const");
+            if (f->dt == NB_F64)
+                k_sp_fill_const<double><<<296, 256, 0, g->cs>>>((double *)f->base[p], n, f->outside);
+            else
+                k_sp_fill_const<float><<<296, 256, 0, g->cs>>>((float *)f->base[p], n, (float)f->outside);
+            NB_TRY(nb_launch_check("k_fill_const"));
+        }
+    }
+    f->cs = f->pcs[g->first_local];
+    return NB_OK;
+}
+
+// plane-organised launch over own slots: grid (segments, planes), 256 threads
+static dim3 sp_grid(const NbSparsePart &sp, int nplanes) {
+    return dim3((unsigned)std::max(1, (sp.max_plane + SEG - 1) / SEG), (unsigned)std::max(1, nplanes));
+}
+
+// gather / scatter between a dense slab [z][y][x] and the own region
+template <typename T>
+__global__ void k_sp_gather(const T *__restrict__ dense, T *__restrict__ own, const int32_t *coord,
+                            const int64_t *pstart, int nx, int ny, int zb) {
+    const int zl = zb + blockIdx.y;
+    const int64_t j = pstart[zl] + (int64_t)blockIdx.x * SEG + threadIdx.x;
+    if (j >= pstart[zl + 1]) return;
+    const int c = coord[j], x = c & 0xffff, y = c >> 16;
+    own[j] = dense[((int64_t)zl * ny + y) * nx + x];
+}
+
+template <typename T>
+__global__ void k_sp_scatter(T *__restrict__ dense, const T *__restrict__ own, const int32_t *coord,
+                             const int64_t *pstart, int nx, int ny, int zb) {
+    const int zl = zb + blockIdx.y;
+    const int64_t j = pstart[zl] + (int64_t)blockIdx.x * SEG + threadIdx.x;
+    if (j >= pstart[zl + 1]) return;
+    const int c = coord[j], x = c & 0xffff, y = c >> 16;
+    dense[((int64_t)zl * ny + y) * nx + x] = own[j];
+}
+
+nb_status nb_sparse_upload(nb_field *f, const void *host) {
+    nb_grid *g = f->g;
+    const int64_t plane = (int64_t)g->nx * g->ny;
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbPart &q = g->parts[p];
+        const NbSparsePart &sp = g->sp[p];
+        size_t slab = (size_t)plane * q.nz() * f->esz;
+        void *tmp = nullptr;
+        NB_CUDA(cudaMallocAsync(&tmp, std::max<size_t>(slab, 1), g->cs));
+        for (int c = 0; c < f->card; ++c) {
+            const char *src = (const char *)host + ((size_t)c * g->nz + q.z0) * plane * f->esz;
+            NB_CUDA(cudaMemcpyAsync(tmp, src, slab, cudaMemcpyHostToDevice, g->cs));
+            char *own = f->base[p] + ((int64_t)c * sp.cs + sp.hl) * f->esz;
+            LaunchScope ls(g, g->cs, "k_sp_gather");
+            if (f->dt == NB_F64)
+                k_sp_gather<double><<<sp_grid(sp, q.nz()), SEG, 0, g->cs>>>((const double *)tmp, (double *)own, sp.coord,
+                                                                            sp.d_pstart, g->nx, g->ny, 0);
+            else
+                k_sp_gather<float><<<sp_grid(sp, q.nz()), SEG, 0, g->cs>>>((const float *)tmp, (float *)own, sp.coord,
+                                                                           sp.d_pstart, g->nx, g->ny, 0);
+            NB_TRY(nb_launch_check("k_sp_gather"));
+        }
+        NB_CUDA(cudaFreeAsync(tmp, g->cs));
+    }
+    NB_CUDA(cudaStreamSynchronize(g->cs));
+    return NB_OK;
+}
+
+nb_status nb_sparse_download(const nb_field *f, void *host) {
+    nb_grid *g = f->g;
+    const int64_t plane = (int64_t)g->nx * g->ny;
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbPart &q = g->parts[p];
+        const NbSparsePart &sp = g->sp[p];
+        size_t slab = (size_t)plane * q.nz() * f->esz;
+        void *tmp = nullptr;
+        NB_CUDA(cudaMallocAsync(&tmp, std::max<size_t>(slab, 1), g->cs));
+        for (int c = 0; c < f->card; ++c) {
+            int64_t n = (int64_t)(slab / f->esz);
+            {
+                LaunchScope ls(g, g->cs, "k_fill_const");
+                if (f->dt == NB_F64)
+                    k_sp_fill_const<double><<<296, 256, 0, g->cs>>>((double *)tmp, n, f->outside);
+                else
+                    k_sp_fill_const<float><<<296, 256, 0, g->cs>>>((float *)tmp, n, (float)f->outside);
+            }
+            const char *own = f->base[p] + ((int64_t)c * sp.cs + sp.hl) * f->esz;
+            LaunchScope ls(g, g->cs, "k_sp_scatter");
+            if (f->dt == NB_F64)
+                k_sp_scatter<double><<<sp_grid(sp, q.nz()), SEG, 0, g->cs>>>((double *)tmp, (const double *)own,
+                                                                             sp.coord, sp.d_pstart, g->nx, g->ny, 0);
+            else
+                k_sp_scatter<float><<<sp_grid(sp, q.nz()), SEG, 0, g->cs>>>((float *)tmp, (const float *)own, sp.coord,
+                                                                            sp.d_pstart, g->nx, g->ny, 0);
+            NB_TRY(nb_launch_check("k_sp_scatter"));
+            char *dst = (char *)host + ((size_t)c * g->nz + q.z0) * plane * f->esz;
+            NB_CUDA(cudaMemcpyAsync(dst, tmp, slab, cudaMemcpyDeviceToHost, g->cs));
+        }
+        NB_CUDA(cudaFreeAsync(tmp, g->cs));
+    }
+    NB_CUDA(cudaStreamSynchronize(g->cs));
+    return NB_OK;
+}
+
+template <typename T>
+__global__ void k_sp_fill(T *own, const int32_t *coord, const int64_t *pstart, int z0, int nx, int ny, int NZ,
+                          int nzp, int64_t cs, int kind, uint64_t seed, double a, double b, double h) {
+    const int zl = blockIdx.y % nzp, c = blockIdx.y / nzp;
+    const int64_t j = pstart[zl] + (int64_t)blockIdx.x * SEG + threadIdx.x;
+    if (j >= pstart[zl + 1]) return;
+    const int cc = coord[j], x = cc & 0xffff, y = cc >> 16, z = z0 + zl;
+    uint64_t gidx = (uint64_t)x + (uint64_t)nx * ((uint64_t)y + (uint64_t)ny * ((uint64_t)z + (uint64_t)NZ * c));
+    own[(int64_t)c * cs + j] = (T)nb_gen(kind, seed, gidx, a, b, x, y, z, h);
+}
+
+nb_status nb_sparse_fill(nb_field *f, nb_fill kind, uint64_t seed, double a, double b) {
+    nb_grid *g = f->g;
+    double h = 1.0 / (double)(g->nx + 1);
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbPart &q = g->parts[p];
+        const NbSparsePart &sp = g->sp[p];
+        if (q.nz() == 0) continue;
+        dim3 grd = sp_grid(sp, q.nz() * f->card);
+        LaunchScope ls(g, g->cs, "k_sp_fill");
+        if (f->dt == NB_F64)
+            k_sp_fill<double><<<grd, SEG, 0, g->cs>>>((double *)f->base[p] + sp.hl, sp.coord, sp.d_pstart, q.z0, g->nx,
+                                                      g->ny, g->nz, q.nz(), sp.cs, kind, seed, a, b, h);
+        else
+            k_sp_fill<float><<<grd, SEG, 0, g->cs>>>((float *)f->base[p] + sp.hl, sp.coord, sp.d_pstart, q.z0, g->nx,
+                                                     g->ny, g->nz, q.nz(), sp.cs, kind, seed, a, b, h);
+        NB_TRY(nb_launch_check("k_sp_fill"));
+    }
+    return NB_OK;
+}
+
+// ---------------------------------------------------------------------------
+// halo: contiguous segments (the neighbour's adjacent plane), plan order
+// ---------------------------------------------------------------------------
+nb_status nb_sparse_halo_update(nb_field *f) {
+    nb_grid *g = f->g;
+    int world = g->comm ? g->comm->world : 1, rank = g->comm ? g->comm->rank : 0;
+    int cnt = 0;
+    NB_TRY(nb_halo_plan(g->nz, g->nparts, world, rank, 0, nullptr, 0, &cnt));
+    std::vector<nb_halo_msg> msgs(cnt);
+    NB_TRY(nb_halo_plan(g->nz, g->nparts, world, rank, 0, msgs.data(), cnt, &cnt));
+    // message geometry from the sparse partitions (src segment, dst halo region)
+    auto src_off = [&](const nb_halo_msg &m) -> int64_t {  // element offset in src buffer (component 0)
+        const NbSparsePart &sp = g->sp[m.src_part];
+        const NbPart &q = g->parts[m.src_part];
+        return m.up ? sp.hl + sp.n - g->plane_count[q.z1 - 1] : sp.hl;
+    };
+    auto dst_off = [&](const nb_halo_msg &m) -> int64_t {
+        const NbSparsePart &sp = g->sp[m.dst_part];
+        return m.up ? 0 : sp.hl + sp.n;
+    };
+    auto count = [&](const nb_halo_msg &m) -> int64_t {
+        const NbPart &q = g->parts[m.src_part];
+        return g->plane_count[m.up ? q.z1 - 1 : q.z0];
+    };
+    bool remote = false;
+    for (auto &m : msgs) {
+        if (m.src_rank == rank && m.dst_rank == rank) {
+            for (int c = 0; c < f->card; ++c) {
+                const char *src = f->base[m.src_part] + ((int64_t)c * f->pcs[m.src_part] + src_off(m)) * f->esz;
+                char *dst = f->base[m.dst_part] + ((int64_t)c * f->pcs[m.dst_part] + dst_off(m)) * f->esz;
+                if (count(m) > 0)
+                    NB_CUDA(cudaMemcpyAsync(dst, src, count(m) * f->esz, cudaMemcpyDeviceToDevice, g->cs));
+            }
+        } else {
+            remote = true;
+        }
+    }
+    if (!remote) return NB_OK;
+    NB_TRY(nb_nccl_group(g, true));
+    for (auto &m : msgs) {
+        if (m.src_rank == rank && m.dst_rank == rank) continue;
+        if (count(m) == 0) continue;
+        for (int c = 0; c < f->card; ++c) {
+            if (m.src_rank == rank)
+                NB_TRY(nb_nccl_send(g, f->base[m.src_part] + ((int64_t)c * f->pcs[m.src_part] + src_off(m)) * f->esz,
+                                    count(m) * f->esz, m.dst_rank, g->cs));
+            else
+                NB_TRY(nb_nccl_recv(g, f->base[m.dst_part] + ((int64_t)c * f->pcs[m.dst_part] + dst_off(m)) * f->esz,
+                                    count(m) * f->esz, m.src_rank, g->cs));
+        }
+    }
+    NB_TRY(nb_nccl_group(g, false));
+    return NB_OK;
+}
+
+// ---------------------------------------------------------------------------
+// maps (same per-element arithmetic as the dense k_axpby)
+// ---------------------------------------------------------------------------
+template <typename T>
+__global__ void k_sp_axpby(const T *__restrict__ x, T *__restrict__ y, int64_t n, T a, T b, int mode) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        T xv = x[i];
+        if (mode == 0)
+            y[i] = a * xv;
+        else if (mode == 1)
+            y[i] = fma(a, xv, y[i]);
+        else
+            y[i] = fma(a, xv, b * y[i]);
+    }
+}
+
+nb_status nb_sparse_axpby(double a, const nb_field *x, double b, nb_field *y, nb_view v) {
+    nb_grid *g = x->g;
+    int mode = (b == 0.0) ? 0 : (b == 1.0 ? 1 : 2);
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbSparsePart &sp = g->sp[p];
+        for (auto rg : view_ranges(g, p, v)) {
+            int64_t j0 = sp.pstart[rg.first], j1 = sp.pstart[rg.second];
+            for (int c = 0; c < x->card; ++c) {
+                int64_t off = (int64_t)c * sp.cs + sp.hl + j0, n = j1 - j0;
+                if (n <= 0) continue;
+                int blocks = (int)std::min<int64_t>((n + 255) / 256, 148 * 8);
+                LaunchScope ls(g, g->cs, "k_sp_axpby");
+                if (x->dt == NB_F64)
+                    k_sp_axpby<double><<<blocks, 256, 0, g->cs>>>((const double *)x->base[p] + off,
+                                                                  (double *)y->base[p] + off, n, a, b, mode);
+                else
+                    k_sp_axpby<float><<<blocks, 256, 0, g->cs>>>((const float *)x->base[p] + off,
+                                                                 (float *)y->base[p] + off, n, (float)a, (float)b, mode);
+                NB_TRY(nb_launch_check("k_sp_axpby"));
+            }
+        }
+    }
+    return NB_OK;
+}
+
+// ---------------------------------------------------------------------------
+// plane-segment kernels: stencil / dot / CG phases.  Block = one 256-cell
+// segment of one plane; the dot value of the segment is the canonical one.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ double seg_sum(double v, double *sw) {
+    v = warp_sum_canon(v);
+    const int w = threadIdx.x >> 5;
+    if ((threadIdx.x & 31) == 0) sw[w] = v;
+    __syncthreads();
+    double s = sw[0];
+#pragma unroll
+    for (int k = 1; k < SEG / 32; ++k) s = __dadd_rn(s, sw[k]);
+    return s;
+}
+
+enum { SPK_DOT = 0, SPK_LAP = 1, SPK_CG_INIT = 2, SPK_CG_MAP = 3, SPK_CG_Q = 4, SPK_CG_R = 5, SPK_CG_FLUSH = 6 };
+
+struct SpArgs {
+    const int64_t *pstart;
+    const int32_t *conn;
+    int64_t n;       // own cells (conn stride)
+    int64_t hl;      // own-region offset in the buffers
+    int zb;          // first local plane of this launch
+    int plane0;      // global plane index of local plane 0 (+ c*NZ)
+    int T;
+    double *tp;
+    double outside;
+    const double *a;  // kernel-specific operands (buffer base pointers)
+    const double *b;
+    double *c;
+    double *d;
+    CgScal *sc;
+};
+
+template <typename T>
+__device__ __forceinline__ T sp_nsum(const T *x, const int32_t *conn, int64_t n, int64_t j, T outside) {
+    // canonical order -x, +x, -y, +y, -z, +z (as the dense kernels)
+    T s;
+#pragma unroll
+    for (int d = 0; d < 6; ++d) {
+        int32_t k = conn[(int64_t)d * n + j];
+        T v = k >= 0 ? x[k] : outside;
+        s = d == 0 ? v : s + v;
+    }
+    return s;
+}
+
+template <int K>
+__global__ void __launch_bounds__(SEG) k_sp(SpArgs A) {
+    __shared__ double sw[SEG / 32];
+    if (K >= SPK_CG_MAP && K <= SPK_CG_R && A.sc->status != 0) return;
+    const int zl = A.zb + blockIdx.y;
+    const int64_t j0 = A.pstart[zl], j1 = A.pstart[zl + 1];
+    const int64_t j = j0 + (int64_t)blockIdx.x * SEG + threadIdx.x;
+    const bool valid = j < j1;
+    const int64_t i = A.hl + j;  // buffer index of own cell j
+    double prod = 0.0;
+    if (valid) {
+        if (K == SPK_DOT) {
+            prod = __dmul_rn(A.a[i], A.b[i]);
+        } else if (K == SPK_CG_INIT) {  // r = b - A x
+            double s = sp_nsum(A.a, A.conn, A.n, j, A.outside);
+            double r = __dsub_rn(A.b[i], fma(6.0, A.a[i], -s));
+            A.c[i] = r;
+            prod = __dmul_rn(r, r);
+        } else if (K == SPK_CG_MAP) {  // x += alpha_prev p_old (pending); p = r + beta p_old
+            double po = A.c[i];
+            if (A.sc->pending) A.d[i] = fma(A.sc->alpha_prev, po, A.d[i]);
+            A.c[i] = fma(A.sc->beta, po, A.a[i]);
+        } else if (K == SPK_CG_Q) {  // q = A p, <p, q>
+            double s = sp_nsum(A.a, A.conn, A.n, j, 0.0);
+            double pc = A.a[i];
+            double q = fma(6.0, pc, -s);
+            A.c[i] = q;
+            prod = __dmul_rn(pc, q);
+        } else if (K == SPK_CG_R) {  // r -= alpha q, <r, r>
+            double r = fma(-A.sc->alpha, A.a[i], A.c[i]);
+            A.c[i] = r;
+            prod = __dmul_rn(r, r);
+        }
+    }
+    if (K == SPK_DOT || K == SPK_CG_INIT || K == SPK_CG_Q || K == SPK_CG_R) {
+        double s = seg_sum(prod, sw);
+        if (threadIdx.x == 0) A.tp[(int64_t)(A.plane0 + zl) * A.T + blockIdx.x] = s;
+    }
+}
+
+template <typename T>
+__global__ void __launch_bounds__(SEG) k_sp_lap(const T *x, T *y, const int64_t *pstart, const int32_t *conn, int64_t n,
+                                                int64_t hl, int zb, T outside) {
+    const int zl = zb + blockIdx.y;
+    const int64_t j = pstart[zl] + (int64_t)blockIdx.x * SEG + threadIdx.x;
+    if (j >= pstart[zl + 1]) return;
+    T s = sp_nsum(x, conn, n, j, outside);
+    y[hl + j] = fma(T(-6), x[hl + j], s);
+}
+
+template <int K>
+static nb_status sp_launch(nb_grid *g, int p, int zb, int ze, SpArgs A, int plane_base, const char *name) {
+    if (ze <= zb) return NB_OK;
+    const NbSparsePart &sp = g->sp[p];
+    A.pstart = sp.d_pstart;
+    A.conn = sp.conn;
+    A.n = sp.n;
+    A.hl = sp.hl;
+    A.zb = zb;
+    A.plane0 = plane_base + g->parts[p].z0;
+    A.T = g->T;
+    A.tp = g->tp;
+    dim3 grd((unsigned)g->T, (unsigned)(ze - zb));
+    LaunchScope ls(g, g->cs, name);
+    k_sp<K><<<grd, SEG, 0, g->cs>>>(A);
+    return nb_launch_check(name);
+}
+
+nb_status nb_sparse_dot_partials(const nb_field *x, const nb_field *y) {
+    nb_grid *g = x->g;
+    if (x->dt != NB_F64) NB_FAIL(NB_EUNSUPPORTED, "sparse dot: fp64 fields");
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbSparsePart &sp = g->sp[p];
+        for (int c = 0; c < x->card; ++c) {
+            SpArgs A{};
+            A.a = (const double *)x->base[p] + (int64_t)c * sp.cs;
+            A.b = (const double *)y->base[p] + (int64_t)c * sp.cs;
+            NB_TRY(sp_launch<SPK_DOT>(g, p, 0, g->parts[p].nz(), A, c * g->nz, "k_sp_dot"));
+        }
+    }
+    return NB_OK;
+}
+
+nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v) {
+    nb_grid *g = x->g;
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbSparsePart &sp = g->sp[p];
+        for (auto rg : view_ranges(g, p, v)) {
+            dim3 grd((unsigned)g->T, (unsigned)(rg.second - rg.first));
+            LaunchScope ls(g, g->cs, "k_sp_lap");
+            if (x->dt == NB_F64)
+                k_sp_lap<double><<<grd, SEG, 0, g->cs>>>((const double *)x->base[p], (double *)y->base[p], sp.d_pstart,
+                                                         sp.conn, sp.n, sp.hl, rg.first, x->outside);
+            else
+                k_sp_lap<float><<<grd, SEG, 0, g->cs>>>((const float *)x->base[p], (float *)y->base[p], sp.d_pstart,
+                                                        sp.conn, sp.n, sp.hl, rg.first, (float)x->outside);
+            NB_TRY(nb_launch_check("k_sp_lap"));
+        }
+    }
+    return NB_OK;
+}
+
+// ---------------------------------------------------------------------------
+// sparse CG: three passes per iteration (104 B per active cell incl. the
+// 24 B connectivity): map (x deferred update, p = r + beta p) -> halo(p) ->
+// q = A p, <p,q> -> alpha -> r -= alpha q, <r,r> -> beta
+// ---------------------------------------------------------------------------
+nb_status nb_sparse_cg_init(nb_cg *cg) {
+    nb_grid *g = cg->g;
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        SpArgs A{};
+        A.a = (const double *)cg->x->base[p];
+        A.b = (const double *)cg->b->base[p];
+        A.c = (double *)cg->r->base[p];
+        A.outside = cg->x->outside;
+        NB_TRY(sp_launch<SPK_CG_INIT>(g, p, 0, g->parts[p].nz(), A, 0, "k_sp_cg_init"));
+    }
+    return nb_reduce_finalize(g, 1, FIN_CG_INIT, cg->sc, 0);
+}
+
+nb_status nb_sparse_cg_hooks(nb_cg *cg, int parity) {
+    (void)parity;
+    nb_grid *g = cg->g;
+    nb_field *p_ = cg->p[0];
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        SpArgs A{};
+        A.a = (const double *)cg->r->base[p];
+        A.c = (double *)p_->base[p];
+        A.d = (double *)cg->x->base[p];
+        A.sc = cg->sc;
+        NB_TRY(sp_launch<SPK_CG_MAP>(g, p, 0, g->parts[p].nz(), A, 0, "k_sp_cg_map"));
+    }
+    NB_TRY(nb_sparse_halo_update(p_));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        SpArgs A{};
+        A.a = (const double *)p_->base[p];
+        A.c = (double *)cg->q->base[p];
+        A.sc = cg->sc;
+        NB_TRY(sp_launch<SPK_CG_Q>(g, p, 0, g->parts[p].nz(), A, 0, "k_sp_cg_q"));
+    }
+    NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_PQ, cg->sc, 0));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        SpArgs A{};
+        A.a = (const double *)cg->q->base[p];
+        A.c = (double *)cg->r->base[p];
+        A.sc = cg->sc;
+        NB_TRY(sp_launch<SPK_CG_R>(g, p, 0, g->parts[p].nz(), A, 0, "k_sp_cg_r"));
+    }
+    NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_RR, cg->sc, 0));
+    cg->k += 1;
+    return NB_OK;
+}
+
+__global__ void k_sp_cg_flush(double *x, const double *p, int64_t n, const CgScal *sc) {
+    if (!sc->pending) return;
+    const double a = sc->alpha_prev;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        x[i] = fma(a, p[i], x[i]);
+}
+
+nb_status nb_sparse_cg_flush(nb_cg *cg) {
+    nb_grid *g = cg->g;
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbSparsePart &sp = g->sp[p];
+        LaunchScope ls(g, g->cs, "k_sp_cg_flush");
+        k_sp_cg_flush<<<296, 256, 0, g->cs>>>((double *)cg->x->base[p] + sp.hl, (const double *)cg->p[0]->base[p] + sp.hl,
+                                              sp.n, cg->sc);
+        NB_TRY(nb_launch_check("k_sp_cg_flush"));
+    }
+    return NB_OK;
 }
