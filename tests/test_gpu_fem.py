@@ -1,0 +1,107 @@
+"""GPU parity of the matrix-free Q1 linear-elastic operator and its CG
+ against the oracle."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_meneghinmjm22_b200 as nb
+import synth
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    import __graft_entry__
+    __graft_entry__.build()
+    assert nb.nb_device_count() > 0
+
+
+def grid(dims, parts=1):
+    return nb.Grid(dims, nparts=parts, devices=[0] * parts)
+
+
+@pytest.mark.parametrize("dims,parts", [((9, 7, 8), 1), ((12, 11, 10), 2), ((33, 9, 12), 3)])
+def test_fem_apply_vs_oracle(dims, parts):
+    u = synth.uniform(dims, card=3, seed=2)
+    exp = oracle.fem_apply(u, 1.0, 0.3)
+    with grid(dims, parts) as g:
+        fu, fy = nb.Field(g, card=3), nb.Field(g, card=3)
+        fu.upload(u)
+        fu.halo_update()
+        nb.nb_fem27_apply(fu, fy, 1.0, 0.3)
+        got = fy.download()
+        fu.close(), fy.close()
+    assert np.max(np.abs(got - exp)) <= 1e-13 * np.max(np.abs(exp))
+
+
+def test_fem_apply_partition_invariant_bitwise():
+    dims = (17, 13, 16)
+    u = synth.uniform(dims, card=3, seed=3)
+    ref = None
+    for parts in (1, 2, 4):
+        with grid(dims, parts) as g:
+            fu, fy = nb.Field(g, card=3), nb.Field(g, card=3)
+            fu.upload(u)
+            fu.halo_update()
+            nb.nb_fem27_apply(fu, fy, 1.0, 0.3)
+            got = fy.download()
+            fu.close(), fy.close()
+        ref = got if ref is None else ref
+        assert np.array_equal(got, ref), parts
+
+
+def test_fem_rigid_translation_and_rhs():
+    dims = (10, 9, 8)
+    nx, ny, nz = dims
+    with grid(dims) as g:
+        fu, fy, fb = nb.Field(g, card=3), nb.Field(g, card=3), nb.Field(g, card=3)
+        # rigid translation in x: zero force away from the Dirichlet layer
+        u = np.zeros((3, nz, ny, nx))
+        u[0] = 1.0
+        fu.upload(u)
+        nb.nb_fem27_apply(fu, fy)
+        y = fy.download()
+        assert np.max(np.abs(y[:, 2:])) < 1e-13
+        nb.nb_fem27_rhs(fb, 1.0)
+        b = fb.download()
+        assert np.array_equal(b, oracle.fem_rhs(dims, 1.0))
+        assert abs(b[2].sum() - (nx - 1) * (ny - 1)) < 1e-12
+        for f in (fu, fy, fb):
+            f.close()
+
+
+def run_fem_cg(dims, parts, iters, rtol=0.0):
+    with grid(dims, parts) as g:
+        fb, fx = nb.Field(g, card=3), nb.Field(g, card=3)
+        nb.nb_fem27_rhs(fb, 1.0)
+        fx.upload(np.zeros((3,) + dims[::-1]))
+        r = nb.nb_cg_solve(fx, fb, max_iter=iters, rtol=rtol, op=nb.OP_FEM27, check_every=16)
+        x = fx.download()
+        fb.close(), fx.close()
+    return x, r
+
+
+def test_fem_cg_vs_oracle_iterates_and_partitions():
+    dims = (10, 9, 12)
+    b = oracle.fem_rhs(dims, 1.0)
+    xo, ro, _ = oracle.cg(b, max_iter=25, op=oracle.OP_FEM27)
+    ref = None
+    for parts in (1, 2, 3):
+        x, r = run_fem_cg(dims, parts, 25)
+        assert r.iters == 25
+        assert np.max(np.abs(x - xo)) <= 1e-10 * np.max(np.abs(xo))
+        if ref is None:
+            ref = (x, r.rr)
+        assert np.array_equal(x, ref[0]) and r.rr == ref[1], parts
+
+
+def test_fem_cg_converges():
+    dims = (8, 8, 8)
+    x, r = run_fem_cg(dims, 2, 2000, rtol=1e-10)
+    assert r.converged == 1
+    b = oracle.fem_rhs(dims, 1.0)
+    res = oracle.fem_apply(x, 1.0, 0.3) - b
+    assert np.max(np.abs(res)) <= 1e-8 * np.max(np.abs(b))
+    assert np.all(x[:, 0] == 0.0)        # Dirichlet plane stays fixed
+    assert x[2, -1].mean() > 0           # the top moves outward (+z) under the pressure
