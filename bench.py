@@ -298,6 +298,128 @@ def bench_lbm_run(n, steps, warmup, world, local, occ="standard"):
     return res
 
 
+SPARSE_BYTES = {"k_sp_cg_map": 40, "k_sp_cg_q": 40, "k_sp_cg_r": 24}  # per active cell (q: p 8 + conn 24 + q 8)
+FEM_BYTES = {"k_fem_map": 120, "k_fem_cg_q": 48, "k_fem_r": 72}     # per node, 3 fp64 components
+FEM_FLOPS_PER_NODE = 306  # 153 nonzero stencil coefficients x 2
+FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12  # SMs x FP64 lanes x 2 x max clock
+
+
+def _profiled_kernels(g, run, names):
+    g.profile(True)
+    run()
+    out = {}
+    for nm in names:
+        k, ms = g.profile_read(nm)
+        out[nm] = (k, ms)
+    g.profile(False)
+    return out
+
+
+def bench_sparse_run(n, steps, warmup, world, local):
+    """C4 (configs[3]): element-sparse sphere (~30 % of the n^3 box), 7-point
+    CG fp64, active-balanced z cuts."""
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    import synth
+    mask = synth.sphere_mask(n)
+    nact = int(mask.sum(dtype="int64"))
+    comm = nb.Comm.from_torch_distributed(local) if world > 1 else None
+    g = nb.Grid((n, n, n), nparts=world, comm=comm, active=mask) if comm else \
+        nb.Grid((n, n, n), nparts=1, devices=[local], active=mask)
+    stream = torch.cuda.ExternalStream(g.stream())
+    b, x = nb.Field(g), nb.Field(g)
+    b.fill_uniform(seed=4)
+    x.fill_const(0.0)
+    cg = nb.CG(x, b)
+    cg.iterate(warmup)
+    cg.prepare(steps)
+    g.sync()
+    l0 = g.launch_count()
+    ms, clocks = timed(world, stream, lambda: cg.iterate(steps), local)
+    launches = g.launch_count() - l0
+    cg.finish()
+    cg.close()
+    x.fill_const(0.0)
+    cg = nb.CG(x, b)
+    prof = _profiled_kernels(g, lambda: cg.iterate(5), list(SPARSE_BYTES))
+    cg.finish()
+    cg.close()
+    hbm, peak_kind = peaks()
+    t = ms / 1e3
+    local_act = nact // world
+    dom = max(prof, key=lambda k: prof[k][1])
+    dk, dms = prof[dom]
+    achieved = SPARSE_BYTES[dom] * local_act / (dms / max(dk, 1) / 1e3) / 1e9
+    b.close(), x.close()
+    g.close()
+    if comm:
+        comm.close()
+    per_cell = sum(SPARSE_BYTES.values())
+    return {"value": nact * steps / t / 1e6, "unit": "MLUPS (active cells)", "n_gpus": world, "steps": steps,
+            "ms_per_step": ms / steps, "scaling": "strong", "dtype": "f64",
+            "config": {"workload": f"C4 element-sparse sphere r=0.41528N in {n}^3 ({nact} active, "
+                                   f"{nact / n ** 3:.2%}), 7-point CG fp64 (configs[3])",
+                       "schedule": f"3 passes, {per_cell} B/active cell/iter incl. 24 B connectivity"},
+            "hbm_gbs": per_cell * nact * steps / t / 1e9, "hbm_frac": per_cell * nact * steps / t / 1e9 / hbm,
+            "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                         "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": ncu_traffic(dom),
+                         "kernel_ms": {k: v[1] / max(v[0], 1) for k, v in prof.items()}},
+            "gpu_launches": int(launches), "clocks": clocks}
+
+
+def bench_fem_run(n, steps, warmup, world, local):
+    """C5 (configs[4]): matrix-free Q1 linear-elastic CG on n^3 nodes x 3 fp64."""
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    comm = nb.Comm.from_torch_distributed(local) if world > 1 else None
+    dims = (n, n, n)
+    g = nb.Grid(dims, nparts=world, comm=comm) if comm else nb.Grid(dims, nparts=1, devices=[local])
+    stream = torch.cuda.ExternalStream(g.stream())
+    b, x = nb.Field(g, card=3), nb.Field(g, card=3)
+    nb.nb_fem27_rhs(b, 1.0)
+    x.fill_const(0.0)
+    cg = nb.CG(x, b, op=nb.OP_FEM27)
+    cg.iterate(warmup)
+    cg.prepare(steps)
+    g.sync()
+    l0 = g.launch_count()
+    ms, clocks = timed(world, stream, lambda: cg.iterate(steps), local)
+    launches = g.launch_count() - l0
+    cg.finish()
+    cg.close()
+    x.fill_const(0.0)
+    cg = nb.CG(x, b, op=nb.OP_FEM27)
+    prof = _profiled_kernels(g, lambda: cg.iterate(5), list(FEM_BYTES))
+    cg.finish()
+    cg.close()
+    hbm, peak_kind = peaks()
+    t = ms / 1e3
+    nodes = n ** 3
+    local_nodes = nodes // world
+    qk, qms = prof["k_fem_cg_q"]
+    q_avg = qms / max(qk, 1) / 1e3
+    flops = FEM_FLOPS_PER_NODE * local_nodes / q_avg / 1e12
+    per_node = sum(FEM_BYTES.values())
+    b.close(), x.close()
+    g.close()
+    if comm:
+        comm.close()
+    return {"value": nodes * steps / t / 1e6, "unit": "MLUPS (nodes)", "n_gpus": world, "steps": steps,
+            "ms_per_step": ms / steps, "scaling": "strong", "dtype": "f64",
+            "config": {"workload": f"C5 FEM Q1 linear elastic CG, {n}^3 nodes x 3 fp64, E=1 nu=0.3, "
+                                   "Dirichlet z=0, pressure 1 on z=N-1 (configs[4])",
+                       "schedule": f"3 passes, {per_node} B/node/iter"},
+            "hbm_gbs": per_node * nodes * steps / t / 1e9, "hbm_frac": per_node * nodes * steps / t / 1e9 / hbm,
+            "roofline": {"bound": "alu", "kernel": "k_fem_cg_q", "achieved": flops, "peak": FP64_PEAK_TFLOPS,
+                         "unit": "TFLOP/s", "frac": flops / FP64_PEAK_TFLOPS,
+                         "peak_kind": "derived: 148 SMs x 64 FP64 lanes x 2 flop x 1.965 GHz",
+                         "traffic": ncu_traffic("k_fem_cg_q"),
+                         "kernel_ms": {k: v[1] / max(v[0], 1) for k, v in prof.items()}},
+            "gpu_launches": int(launches), "clocks": clocks}
+
+
 def bench_c1(local):
     """Config C1 (64^3 fp64, 10 map-stencil-reduce iterations, 1 GPU): a
     launch/latency-bound case.  Timed per synchronous nb_map_stencil_reduce
@@ -400,7 +522,7 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="nb", choices=["nb", "reference"])
-    ap.add_argument("--workload", default="cg", choices=["cg", "lbm"])
+    ap.add_argument("--workload", default="cg", choices=["cg", "lbm", "sparse", "fem"])
     ap.add_argument("--n", type=int, default=512)
     ap.add_argument("--occ", default="two_way", choices=list(("none", "standard", "extended", "two_way")))
     ap.add_argument("--prof-steps", type=int, default=10)
@@ -422,9 +544,16 @@ def main():
         out = bench_cg(args, world, rank, local)
         if world == 1 and not args.no_extras:
             lbm = bench_lbm_run(args.n, 20, 3, 1, local)
-            out["also"] = {"lbm_d3q19": lbm, "c1": bench_c1(local)}
+            out["also"] = {"lbm_d3q19": lbm, "c1": bench_c1(local),
+                           "sparse_c4": bench_sparse_run(args.n, 20, 3, 1, local),
+                           "fem_c5": bench_fem_run(384, 20, 3, 1, local)}
             out["cpu_baseline"] = cpu_baseline_cg(args.n)
             out["also"]["lbm_d3q19"]["cpu_baseline"] = cpu_baseline_lbm()
+    elif args.workload in ("sparse", "fem"):
+        fn = bench_sparse_run if args.workload == "sparse" else bench_fem_run
+        r = fn(args.n if args.workload == "sparse" else min(args.n, 384), args.steps, args.warmup, world, local)
+        out = {"metric": METRIC, "higher_is_better": True, "vs_baseline": None, "data": "synthetic",
+               "warmup": args.warmup, **r}
     else:
         r = bench_lbm_run(args.n, args.steps, args.warmup, world, local, occ=args.occ if args.occ in
                           ("none", "standard") else "standard")

@@ -86,6 +86,15 @@ static nb_status fem_upload_constants(double E, double nu) {
             for (int i = 0; i < 3; ++i)
                 for (int j = 0; j < 3; ++j) S[o * 9 + i * 3 + j] += ke[(3 * a + i) * 24 + 3 * b + j];
         }
+    // structural zeros of the assembled stencil: the coupling of components
+    // i != j at offset o vanishes unless o_i != 0 and o_j != 0 (odd symmetry
+    // of the tensor-product element); store them as exact zeros
+    for (int o = 0; o < 27; ++o) {
+        const int oc[3] = {o % 3 - 1, (o / 3) % 3 - 1, o / 9 - 1};
+        for (int i = 0; i < 3; ++i)
+            for (int j = 0; j < 3; ++j)
+                if (i != j && (oc[i] == 0 || oc[j] == 0)) S[o * 9 + i * 3 + j] = 0.0;
+    }
     NB_CUDA(cudaMemcpyToSymbol(c_ke, ke, sizeof(ke)));
     NB_CUDA(cudaMemcpyToSymbol(c_S, S, sizeof(S)));
     g_fem_E = E;
@@ -114,14 +123,16 @@ __device__ __forceinline__ void fem_node(const double *__restrict__ u, int64_t c
             const int64_t m = c0 + (int64_t)oz * g.ps + (int64_t)oy * g.pitch + ox;
             const double u0 = u[m], u1 = u[cs + m], u2 = u[2 * cs + m];
             const double *S = c_S + o * 9;
+            // 153 structurally nonzero coefficients (diagonal blocks always;
+            // i-j coupling only where o_i != 0 and o_j != 0): 306 flop/node
             acc0 = fma(S[0], u0, acc0);
-            acc0 = fma(S[1], u1, acc0);
-            acc0 = fma(S[2], u2, acc0);
-            acc1 = fma(S[3], u0, acc1);
+            if (ox != 0 && oy != 0) acc0 = fma(S[1], u1, acc0);
+            if (ox != 0 && oz != 0) acc0 = fma(S[2], u2, acc0);
+            if (oy != 0 && ox != 0) acc1 = fma(S[3], u0, acc1);
             acc1 = fma(S[4], u1, acc1);
-            acc1 = fma(S[5], u2, acc1);
-            acc2 = fma(S[6], u0, acc2);
-            acc2 = fma(S[7], u1, acc2);
+            if (oy != 0 && oz != 0) acc1 = fma(S[5], u2, acc1);
+            if (oz != 0 && ox != 0) acc2 = fma(S[6], u0, acc2);
+            if (oz != 0 && oy != 0) acc2 = fma(S[7], u1, acc2);
             acc2 = fma(S[8], u2, acc2);
         }
     } else {

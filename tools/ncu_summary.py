@@ -36,9 +36,11 @@ def load(rep):
                 val = float(r[i].replace(",", "")) if r[i] else 0.0
                 u = units[i]
                 if v in ("dram_read", "dram_write"):
-                    val *= {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}.get(u, 1)
+                    val *= {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
+                            "B": 1, "KB": 1e3, "MB": 1e6, "GB": 1e9}.get(u, 1)
                 if v == "ms":
-                    val *= {"nsecond": 1e-6, "usecond": 1e-3, "msecond": 1, "second": 1e3}.get(u, 1)
+                    val *= {"nsecond": 1e-6, "ns": 1e-6, "usecond": 1e-3, "us": 1e-3, "msecond": 1, "ms": 1,
+                            "second": 1e3, "s": 1e3}.get(u, 1)
                 d[v] = val
         stalls = []
         for i in stall_cols:

@@ -28,4 +28,29 @@ if "lbm" in what:
     g.sync()
     fa.close(), fb.close()
     g.close()
+if "sparse" in what:
+    import synth
+    m = synth.sphere_mask(n)
+    g = nb.Grid((n, n, n), active=m)
+    b, x = nb.Field(g), nb.Field(g)
+    b.fill_uniform(seed=4)
+    x.fill_const(0.0)
+    cg = nb.CG(x, b)
+    cg.iterate(3)
+    cg.finish()
+    cg.close()
+    b.close(), x.close()
+    g.close()
+if "fem" in what:
+    nf = min(n, 384)
+    g = nb.Grid((nf, nf, nf))
+    b, x = nb.Field(g, card=3), nb.Field(g, card=3)
+    nb.nb_fem27_rhs(b, 1.0)
+    x.fill_const(0.0)
+    cg = nb.CG(x, b, op=nb.OP_FEM27)
+    cg.iterate(3)
+    cg.finish()
+    cg.close()
+    b.close(), x.close()
+    g.close()
 print("prof driver done")

@@ -1,0 +1,18 @@
+#!/bin/bash
+# GPU-box profiling pass for one round: launch list of the bench command and
+# one ncu --set full capture per hot kernel.  Usage: tools/profile_round.sh r1
+set -u
+R=${1:-r1}
+mkdir -p gpurun_out
+# every launch of the default bench workload (cold-cache, serialised: compare shares)
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv \
+    --log-file gpurun_out/launches_${R}.csv python bench.py --steps 3 --warmup 3 --no-extras \
+    > gpurun_out/launches_${R}.log 2>&1
+# full sections of each hot kernel (2-4 launches each)
+timeout 900 ncu --set full --clock-control none --import-source on \
+    -k regex:"k_zmarch|k_finalize|k_lbm_d3q19" -c 12 -o gpurun_out/prof_${R}_dense \
+    python tools/prof_driver.py 512 cg,lbm > gpurun_out/prof_${R}_dense.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on \
+    -k regex:"k_sp<|k_fem<|k_fem_map|k_fem_r" -c 14 -o gpurun_out/prof_${R}_sparse_fem \
+    python tools/prof_driver.py 512 sparse,fem > gpurun_out/prof_${R}_sparse_fem.log 2>&1
+echo profile done
