@@ -24,7 +24,7 @@ __all__ = [
     "OCC_NONE", "OCC_STANDARD", "OCC_EXTENDED", "OCC_TWO_WAY",
 ]
 
-LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libnb.so")
+LIB_PATH = os.environ.get("NB_LIB") or os.path.join(os.path.dirname(os.path.abspath(__file__)), "libnb.so")
 
 NB_OK, NB_EINVAL, NB_ENOMEM, NB_ECUDA, NB_ENCCL, NB_EMISMATCH, NB_EUNSUPPORTED, NB_ESTATE = range(8)
 NB_F32, NB_F64 = 0, 1

@@ -14,8 +14,11 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-OUT = os.path.join(PKG, "libnb.so")
-BUILD = os.path.join(ROOT, "build", "nb")
+# experiment variants: NB_VARIANT="ZR=4" builds libnb_ZR4.so with -DNB_ZR=4
+VARIANT = os.environ.get("NB_VARIANT", "")
+_VTAG = VARIANT.replace("=", "").replace(",", "_")
+OUT = os.path.join(PKG, f"libnb_{_VTAG}.so" if VARIANT else "libnb.so")
+BUILD = os.path.join(ROOT, "build", f"nb_{_VTAG}" if VARIANT else "nb")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 NVCC_FLAGS = [
@@ -23,7 +26,7 @@ NVCC_FLAGS = [
     "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3",
     "--expt-relaxed-constexpr", "-Xptxas", "-v",
     f"-I{os.path.join(ROOT, 'include')}", f"-I{CSRC}",
-]
+] + [f"-DNB_{d}" for d in VARIANT.split(",") if d]
 
 
 def _compile(src: str) -> str:

@@ -14,6 +14,7 @@
 
 #include "nb_device.cuh"
 #include "nb_internal.cuh"
+#include "nb_zmarch.cuh"
 
 // ===========================================================================
 // errors, version
@@ -849,28 +850,34 @@ extern "C" nb_status nb_axpy(double a, const nb_field *x, nb_field *y, nb_view v
 // ===========================================================================
 // reduce (eq. L129): canonical tiles -> plane sums -> total
 // ===========================================================================
+// canonical dot tiles (the order of nb_zmarch.cuh): warp = ZR rows, per lane
+// rows sequential, butterfly, then the warps of a 32 x 8 tile in order
 template <typename T>
-__global__ void __launch_bounds__(256) k_dot(const T *__restrict__ x, const T *__restrict__ y, PGeo g,
-                                             int64_t cstride, int zb, int ze, double *tp, int T_tiles) {
-    constexpr int ZC = 16;
-    __shared__ TileStage<ZC> st;
-    const int xi = blockIdx.x * DOT_TX + threadIdx.x, yi = blockIdx.y * DOT_TY + threadIdx.y;
-    const int nchunk = (ze - zb + ZC - 1) / ZC;
+__global__ void __launch_bounds__(32 * ZW) k_dot(const T *__restrict__ x, const T *__restrict__ y, PGeo g,
+                                                 int64_t cstride, int nchunk, double *tp, int T_tiles, int tiles_y) {
+    constexpr int ZR = ZR_STO, ZTY = ZW * ZR;
+    __shared__ double sw[ZC][ZW];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int xi = blockIdx.x * DOT_TX + lane, yr = blockIdx.y * ZTY + w * ZR;
     const int c = blockIdx.z / nchunk, ch = blockIdx.z % nchunk;
-    const int zs = zb + ch * ZC, zend = min(ze, zs + ZC);
-    const bool valid = xi < g.nx && yi < g.ny;
-    const int64_t o = (int64_t)c * cstride + (int64_t)yi * g.pitch + xi;
+    const int zs = ch * ZC, zend = min(g.nzl, zs + ZC);
+    const int64_t o = (int64_t)c * cstride + (int64_t)yr * g.pitch + xi + g.ps;
     for (int z = zs; z < zend; ++z) {
-        double v = 0.0;
-        if (valid) {
-            int64_t i = o + (int64_t)(z + 1) * g.ps;
-            v = __dmul_rn((double)__ldcs(x + i), (double)__ldcs(y + i));
+        double col = 0.0;
+#pragma unroll
+        for (int j = 0; j < ZR; ++j) {
+            double prod = 0.0;
+            if (xi < g.nx && yr + j < g.ny) {
+                const int64_t i = o + (int64_t)z * g.ps + (int64_t)j * g.pitch;
+                prod = __dmul_rn((double)__ldcs(x + i), (double)__ldcs(y + i));
+            }
+            col = j == 0 ? prod : __dadd_rn(col, prod);
         }
-        tile_stage_put<ZC>(st, z - zs, v);
+        col = warp_sum_canon(col);
+        if (lane == 0) sw[z - zs][w] = col;
     }
     __syncthreads();
-    tile_stage_flush<ZC>(st, zend - zs, tp, (int64_t)c * g.NZ + g.z0 + zs, T_tiles,
-                         blockIdx.y * gridDim.x + blockIdx.x);
+    zm_flush<ZR>(sw, zend - zs, tp, (int64_t)c * g.NZ + g.z0 + zs, T_tiles, gridDim.x, tiles_y, blockIdx.x, blockIdx.y);
 }
 
 // ---- finalize: plane sums (one CTA per plane) + last-block total ----------
@@ -995,15 +1002,15 @@ nb_status nb_dot_partials(const nb_field *x, const nb_field *y) {
     for (int p = 0; p < g->nparts; ++p) {
         if (!g->parts[p].local) continue;
         PGeo geo = pgeo(x, p);
-        int nchunk = (geo.nzl + 15) / 16;
-        dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, nchunk * x->card);
+        int nchunk = (geo.nzl + ZC - 1) / ZC;
+        dim3 blk(32 * ZW), grd(g->tiles_x, (g->ny + ZW * ZR_STO - 1) / (ZW * ZR_STO), nchunk * x->card);
         LaunchScope ls(g, g->cs, "k_dot");
         if (x->dt == NB_F64)
             k_dot<double><<<grd, blk, 0, g->cs>>>((const double *)x->base[p], (const double *)y->base[p], geo,
-                                                   dense_cs(x, p), 0, geo.nzl, g->tp, g->T);
+                                                   dense_cs(x, p), nchunk, g->tp, g->T, g->tiles_y);
         else
             k_dot<float><<<grd, blk, 0, g->cs>>>((const float *)x->base[p], (const float *)y->base[p], geo,
-                                                  dense_cs(x, p), 0, geo.nzl, g->tp, g->T);
+                                                  dense_cs(x, p), nchunk, g->tp, g->T, g->tiles_y);
         NB_TRY(nb_launch_check("k_dot"));
     }
     return NB_OK;

@@ -21,6 +21,13 @@
 #include "nb_internal.cuh"
 #include "nb_zmarch.cuh"
 
+#ifndef NB_ZL_SMEM
+#define NB_ZL_SMEM 1
+#endif
+#ifndef NB_ZL_L1
+#define NB_ZL_L1 0
+#endif
+
 std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v);
 nb_status nb_dot_partials(const nb_field *x, const nb_field *y);
 nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v);
@@ -38,7 +45,7 @@ struct Lap7Op {
     struct Raw {
         TT a;
     };
-    static constexpr bool DOT = false;
+    static constexpr bool DOT = false, MAP = false;
     const TT *x;
     TT *y;
     TT outv;
@@ -54,28 +61,15 @@ struct Lap7Op {
     }
 };
 
-// z-march variant: lookahead L (0: load plane z+1 at step z; 1: prefetch
-// plane z+2 at step z).  NB_ZM_L overrides for experiments ("0"/"1").
-static int zm_lookahead(bool smem) {
-    static int env[2] = {-2, -2};
-    int k = smem ? 1 : 0;
-    if (env[k] == -2) {
-        const char *e = getenv(smem ? "NB_ZM_LS" : "NB_ZM_L");
-        env[k] = e ? atoi(e) : -1;
-    }
-    if (env[k] >= 0) return env[k];
-    return smem ? 1 : 0;
-}
-
 template <class Op, bool SMEM = false>
 static nb_status launch_zmarch(nb_grid *g, const char *name, Op op, PGeo geo, int zb, int ze) {
     if (ze <= zb) return NB_OK;
-    dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
+    constexpr int ZR = Op::MAP ? ZR_MAP : ZR_STO;
+    constexpr int ZTY = ZW * ZR;
+    dim3 blk(32 * ZW), grd(g->tiles_x, (g->ny + ZTY - 1) / ZTY, (ze - zb + ZC - 1) / ZC);
     LaunchScope ls(g, g->cs, name);
-    if (zm_lookahead(SMEM) == 1)
-        k_zmarch<Op, SMEM, 1><<<grd, blk, 0, g->cs>>>(op, geo, zb, ze, g->tp, g->T);
-    else
-        k_zmarch<Op, SMEM, 0><<<grd, blk, 0, g->cs>>>(op, geo, zb, ze, g->tp, g->T);
+    constexpr int L = SMEM ? NB_ZL_SMEM : NB_ZL_L1;
+    k_zmarch<Op, SMEM, L, ZR><<<grd, blk, 0, g->cs>>>(op, geo, zb, ze, g->tp, g->T, g->tiles_y);
     return nb_launch_check(name);
 }
 
@@ -134,7 +128,7 @@ struct MsrOp {
     struct Raw {
         double v, w, x;  // v: map input (or stored u on halo planes), w, x: see cell()
     };
-    static constexpr bool DOT = true;
+    static constexpr bool DOT = true, MAP = true;  // every MsrOp variant: one canonical <u, res> order
     MsrArgs A;
     int nzl;
     double m, ap;
@@ -218,7 +212,7 @@ struct CgBOp {
     struct Raw {
         double p, r;
     };
-    static constexpr bool DOT = true;
+    static constexpr bool DOT = true, MAP = false;
     const double *p;
     double *r;
     const CgScal *sc;
@@ -243,7 +237,7 @@ struct CgInitOp {
     struct Raw {
         double x, b;
     };
-    static constexpr bool DOT = true;
+    static constexpr bool DOT = true, MAP = false;
     const double *x, *b;
     double *r;
     double outv;
