@@ -1,0 +1,112 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py
+times (single partition, default OCC, graph-launched CG), on outputs the
+oracle can compute: whole-grid oracle CG iterations where the oracle takes
+seconds (C2 512^3, C4 sparse 512^3), and sampled outputs computed one by one
+on small oracle blocks elsewhere (C3 LBM 512^3, C5 FEM 384^3)."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_meneghinmjm22_b200 as nb
+import synth
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    import __graft_entry__
+    __graft_entry__.build()
+    assert nb.nb_device_count() > 0
+
+
+def test_c2_poisson_cg_512_vs_oracle():
+    """C2: 512^3 fp64, b = h^2 f (manufactured), x0 = 0: 3 CG iterations on
+    the GPU (bench path: nb_cg_create / iterate / finish, graphs) vs the oracle."""
+    n, k = 512, 3
+    b = synth.poisson_poly_rhs((n, n, n))
+    xo, ro, hist = oracle.cg(b, max_iter=k)
+    with nb.Grid((n, n, n)) as g:
+        fb, fx = nb.Field(g), nb.Field(g)
+        fb.fill(nb.FILL_POISSON_RHS)
+        fx.fill_const(0.0)
+        cg = nb.CG(fx, fb)
+        cg.prepare(k)
+        cg.iterate(k)
+        r = cg.finish()
+        cg.close()
+        x = fx.download()
+        fb.close(), fx.close()
+    assert r.iters == k
+    assert abs(r.rr0 - hist[0]) <= 1e-12 * hist[0]
+    assert abs(r.rr - ro.rr) <= 1e-10 * ro.rr
+    assert np.max(np.abs(x - xo)) <= 1e-11 * np.max(np.abs(xo))
+
+
+def test_c4_sparse_cg_512_vs_oracle():
+    n, k = 512, 2
+    m = synth.sphere_mask(n)
+    b = np.where(m, synth.uniform((n, n, n), seed=4), 0.0)
+    xo, ro, hist = oracle.cg(b, max_iter=k, op=oracle.OP_SPARSE7, mask=m)
+    with nb.Grid((n, n, n), active=m) as g:
+        fb, fx = nb.Field(g), nb.Field(g)
+        fb.fill_uniform(seed=4)
+        fx.fill_const(0.0)
+        r = nb.nb_cg_solve(fx, fb, max_iter=k)
+        x = fx.download()
+        fb.close(), fx.close()
+    assert r.iters == k
+    assert abs(r.rr0 - hist[0]) <= 1e-12 * hist[0]
+    assert abs(r.rr - ro.rr) <= 1e-10 * ro.rr
+    assert np.max(np.abs(x - xo)) <= 1e-11 * np.max(np.abs(xo))
+
+
+def _lbm_slab_oracle(f, z, omega, nz):
+    """Oracle step for plane z of the full grid from the planes z-1..z+1 of
+    the state f ([19][nz][ny][nx] fp32, global), computed on a 3-plane slab
+    (2 planes at the global faces): every source of plane z lies in the
+    slab, and the slab's own z faces coincide with the global ones where
+    the slab is cut by them."""
+    z0, z1 = max(z - 1, 0), min(z + 2, nz)
+    sub = oracle.lbm_step(f[:, z0:z1], omega)
+    return sub[:, z - z0]
+
+
+def test_c3_lbm_512_sampled_planes_vs_oracle():
+    n = 512
+    omega = oracle.lbm_omega(n)
+    planes = [0, 1, 255, 510, 511]
+    with nb.Grid((n, n, n)) as g:
+        a, b = nb.Field(g, "f32", 19), nb.Field(g, "f32", 19)
+        nb.nb_lbm_init(a, 1.0, (0.0, 0.0, 0.0))
+        a, b = nb.nb_lbm_step(a, b, omega, 3)  # a non-trivial state near the lid
+        f = a.download()
+        a, b = nb.nb_lbm_step(a, b, omega, 1)
+        f1 = a.download()
+        a.close(), b.close()
+    for z in planes:
+        exp = _lbm_slab_oracle(f, z, omega, n)
+        got = f1[:, z].astype(np.float64)
+        assert np.max(np.abs(got - exp) / np.abs(exp)) <= 1e-5, z
+    assert np.max(np.abs(f1[:, :, -1] - f[:, :, -1])) > 1e-6  # the lid drives the flow
+
+
+def test_c5_fem_384_sampled_nodes_vs_oracle():
+    n = 384
+    rng = np.random.default_rng(0)
+    pts = [(0, 0, 0), (n - 1, n - 1, n - 1), (1, 2, 1), (n // 2, n // 2, n // 2), (0, 200, 383), (383, 0, 1)]
+    pts += [tuple(int(v) for v in rng.integers(0, n, 3)) for _ in range(10)]
+    with nb.Grid((n, n, n)) as g:
+        u, y = nb.Field(g, card=3), nb.Field(g, card=3)
+        u.fill_uniform(seed=5)
+        nb.nb_fem27_apply(u, y)
+        ug, yg = u.download(), y.download()
+        u.close(), y.close()
+    for (x, yy, z) in pts:
+        sl = [slice(max(c - 1, 0), min(c + 2, n)) for c in (z, yy, x)]
+        blk = ug[:, sl[0], sl[1], sl[2]]
+        exp = oracle.fem_apply(blk, 1.0, 0.3, dirichlet_z0=(sl[0].start == 0))
+        loc = (z - sl[0].start, yy - sl[1].start, x - sl[2].start)
+        e = exp[:, loc[0], loc[1], loc[2]]
+        got = yg[:, z, yy, x]
+        assert np.max(np.abs(got - e)) <= 1e-13 * max(1.0, np.max(np.abs(e))), (x, yy, z)
