@@ -90,6 +90,9 @@ struct NbSparsePart {
     int32_t *conn = nullptr;                // [6][n] buffer index of the neighbour, -1 = outside
     int32_t *coord = nullptr;               // [n] x | y << 16
     int max_plane = 0;                      // max active cells in one local plane
+    // non-empty 256-cell dot segments, plane-major: entry = zl << 16 | seg
+    int32_t *d_seg = nullptr;
+    std::vector<int64_t> seg_start;         // first segment of each local plane [nz_p + 1]
 };
 
 struct nb_grid {

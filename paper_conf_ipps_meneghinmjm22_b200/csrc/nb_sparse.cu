@@ -40,8 +40,10 @@ void nb_sparse_free(nb_grid *g) {
         cudaFree(s.conn);
         cudaFree(s.coord);
         cudaFree(s.d_pstart);
+        cudaFree(s.d_seg);
         s.conn = s.coord = nullptr;
         s.d_pstart = nullptr;
+        s.d_seg = nullptr;
     }
 }
 
@@ -84,6 +86,8 @@ extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t 
         counts[z] = c;
     }
     if (nparts < 1 || nparts > nz) NB_FAIL(NB_EINVAL, "nb_grid_create_sparse: bad nparts %d", nparts);
+    if (nz > 65535 || plane > (int64_t)SEG * 65535)
+        NB_FAIL(NB_EUNSUPPORTED, "nb_grid_create_sparse: segment table limits (nz <= 65535, Nx*Ny <= 16.7M)");
     std::vector<int32_t> zb(nparts + 1);
     NB_TRY(nb_partition_plan_weighted(nz, counts.data(), nparts, zb.data()));
     if (nparts > 1)
@@ -125,8 +129,10 @@ extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t 
         sp.hh = q.halo_hi;
         sp.cs = std::max<int64_t>(32, (sp.hl + sp.n + sp.hh + 31) / 32 * 32);
         sp.pstart.assign(q.nz() + 1, 0);
+        sp.seg_start.assign(q.nz() + 1, 0);
         for (int z = q.z0; z < q.z1; ++z) {
             sp.pstart[z - q.z0 + 1] = sp.pstart[z - q.z0] + counts[z];
+            sp.seg_start[z - q.z0 + 1] = sp.seg_start[z - q.z0] + (counts[z] + SEG - 1) / SEG;
             sp.max_plane = std::max<int>(sp.max_plane, (int)counts[z]);
         }
     }
@@ -167,6 +173,13 @@ extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t 
         if (s == NB_OK)
             cudaMemcpyAsync(sp.d_pstart, sp.pstart.data(), sizeof(int64_t) * sp.pstart.size(), cudaMemcpyHostToDevice,
                             g->cs);
+        std::vector<int32_t> segs;
+        for (int zl = 0; zl < q.nz(); ++zl)
+            for (int64_t k = 0; k < sp.seg_start[zl + 1] - sp.seg_start[zl]; ++k) segs.push_back((zl << 16) | (int)k);
+        if (s == NB_OK && (e = cudaMalloc(&sp.d_seg, sizeof(int32_t) * std::max<size_t>(segs.size(), 1))) != cudaSuccess)
+            fail("cudaMalloc seg", e);
+        if (s == NB_OK && !segs.empty())
+            cudaMemcpyAsync(sp.d_seg, segs.data(), sizeof(int32_t) * segs.size(), cudaMemcpyHostToDevice, g->cs);
         if (s == NB_OK && q.nz() > 0) {
             dim3 blk(128), grd((nx + 127) / 128, ny, q.nz());
             LaunchScope ls(g, g->cs, "k_sp_conn");
@@ -460,11 +473,12 @@ __device__ __forceinline__ double seg_sum(double v, double *sw) {
 enum { SPK_DOT = 0, SPK_LAP = 1, SPK_CG_INIT = 2, SPK_CG_MAP = 3, SPK_CG_Q = 4, SPK_CG_R = 5, SPK_CG_FLUSH = 6 };
 
 struct SpArgs {
+    const int32_t *seg;  // segment table of the partition
+    int64_t seg0;        // first table entry of this launch
     const int64_t *pstart;
     const int32_t *conn;
     int64_t n;       // own cells (conn stride)
     int64_t hl;      // own-region offset in the buffers
-    int zb;          // first local plane of this launch
     int plane0;      // global plane index of local plane 0 (+ c*NZ)
     int T;
     double *tp;
@@ -493,9 +507,10 @@ template <int K>
 __global__ void __launch_bounds__(SEG) k_sp(SpArgs A) {
     __shared__ double sw[SEG / 32];
     if (K >= SPK_CG_MAP && K <= SPK_CG_R && A.sc->status != 0) return;
-    const int zl = A.zb + blockIdx.y;
+    const int e = A.seg[A.seg0 + blockIdx.x];  // non-empty segment: plane << 16 | index
+    const int zl = e >> 16, sg = e & 0xffff;
     const int64_t j0 = A.pstart[zl], j1 = A.pstart[zl + 1];
-    const int64_t j = j0 + (int64_t)blockIdx.x * SEG + threadIdx.x;
+    const int64_t j = j0 + (int64_t)sg * SEG + threadIdx.x;
     const bool valid = j < j1;
     const int64_t i = A.hl + j;  // buffer index of own cell j
     double prod = 0.0;
@@ -525,35 +540,39 @@ __global__ void __launch_bounds__(SEG) k_sp(SpArgs A) {
     }
     if (K == SPK_DOT || K == SPK_CG_INIT || K == SPK_CG_Q || K == SPK_CG_R) {
         double s = seg_sum(prod, sw);
-        if (threadIdx.x == 0) A.tp[(int64_t)(A.plane0 + zl) * A.T + blockIdx.x] = s;
+        if (threadIdx.x == 0) A.tp[(int64_t)(A.plane0 + zl) * A.T + sg] = s;
     }
 }
 
 template <typename T>
-__global__ void __launch_bounds__(SEG) k_sp_lap(const T *x, T *y, const int64_t *pstart, const int32_t *conn, int64_t n,
-                                                int64_t hl, int zb, T outside) {
-    const int zl = zb + blockIdx.y;
-    const int64_t j = pstart[zl] + (int64_t)blockIdx.x * SEG + threadIdx.x;
+__global__ void __launch_bounds__(SEG) k_sp_lap(const T *x, T *y, const int32_t *seg, int64_t seg0, const int64_t *pstart,
+                                                const int32_t *conn, int64_t n, int64_t hl, T outside) {
+    const int e = seg[seg0 + blockIdx.x];
+    const int zl = e >> 16;
+    const int64_t j = pstart[zl] + (int64_t)(e & 0xffff) * SEG + threadIdx.x;
     if (j >= pstart[zl + 1]) return;
     T s = sp_nsum(x, conn, n, j, outside);
     y[hl + j] = fma(T(-6), x[hl + j], s);
 }
 
+// launch over the non-empty segments of local planes [zb, ze)
 template <int K>
 static nb_status sp_launch(nb_grid *g, int p, int zb, int ze, SpArgs A, int plane_base, const char *name) {
     if (ze <= zb) return NB_OK;
     const NbSparsePart &sp = g->sp[p];
+    const int64_t s0 = sp.seg_start[zb], s1 = sp.seg_start[ze];
+    if (s1 <= s0) return NB_OK;
+    A.seg = sp.d_seg;
+    A.seg0 = s0;
     A.pstart = sp.d_pstart;
     A.conn = sp.conn;
     A.n = sp.n;
     A.hl = sp.hl;
-    A.zb = zb;
     A.plane0 = plane_base + g->parts[p].z0;
     A.T = g->T;
     A.tp = g->tp;
-    dim3 grd((unsigned)g->T, (unsigned)(ze - zb));
     LaunchScope ls(g, g->cs, name);
-    k_sp<K><<<grd, SEG, 0, g->cs>>>(A);
+    k_sp<K><<<(unsigned)(s1 - s0), SEG, 0, g->cs>>>(A);
     return nb_launch_check(name);
 }
 
@@ -577,14 +596,17 @@ nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v) {
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         const NbSparsePart &sp = g->sp[p];
         for (auto rg : view_ranges(g, p, v)) {
-            dim3 grd((unsigned)g->T, (unsigned)(rg.second - rg.first));
+            const int64_t s0 = sp.seg_start[rg.first], s1 = sp.seg_start[rg.second];
+            if (s1 <= s0) continue;
             LaunchScope ls(g, g->cs, "k_sp_lap");
             if (x->dt == NB_F64)
-                k_sp_lap<double><<<grd, SEG, 0, g->cs>>>((const double *)x->base[p], (double *)y->base[p], sp.d_pstart,
-                                                         sp.conn, sp.n, sp.hl, rg.first, x->outside);
+                k_sp_lap<double><<<(unsigned)(s1 - s0), SEG, 0, g->cs>>>((const double *)x->base[p], (double *)y->base[p],
+                                                                         sp.d_seg, s0, sp.d_pstart, sp.conn, sp.n,
+                                                                         sp.hl, x->outside);
             else
-                k_sp_lap<float><<<grd, SEG, 0, g->cs>>>((const float *)x->base[p], (float *)y->base[p], sp.d_pstart,
-                                                        sp.conn, sp.n, sp.hl, rg.first, (float)x->outside);
+                k_sp_lap<float><<<(unsigned)(s1 - s0), SEG, 0, g->cs>>>((const float *)x->base[p], (float *)y->base[p],
+                                                                        sp.d_seg, s0, sp.d_pstart, sp.conn, sp.n, sp.hl,
+                                                                        (float)x->outside);
             NB_TRY(nb_launch_check("k_sp_lap"));
         }
     }

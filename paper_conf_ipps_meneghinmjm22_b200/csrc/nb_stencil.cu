@@ -176,6 +176,150 @@ struct MsrOp {
     }
 };
 
+// ===========================================================================
+// Specialised recompute kernel (the CG phase-A / C1 hot path): the same
+// arithmetic and canonical dot order as k_zmarch<MsrOp<MODE, true, DOMAP>,
+// SMEM, L=1, ZR=1>, written with per-array pointers advanced by one plane per
+// step, a CTA-uniform fast path for tiles whose cells and ring are all inside
+// the domain, and halo-plane selection by CTA-uniform branches — about a
+// third of the generic kernel's instructions per cell.
+// ===========================================================================
+template <int MODE, bool DOMAP, bool FULL>
+__device__ __forceinline__ void msr_fast_body(const MsrArgs &A, const PGeo &g, int zs, int zend, double m, double ap,
+                                              bool dox, double (*sU)[DOT_TY + 2][DOT_TX + 2], double (*sw)[ZW]) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int x0 = blockIdx.x * DOT_TX, y0 = blockIdx.y * DOT_TY;
+    const int xi = x0 + lane, yi = y0 + w;
+    const int nzl = g.nzl;
+    const int64_t ps = g.ps;
+    const bool valid = FULL || (xi < g.nx && yi < g.ny);
+    // ring roles: warp 0 / 7 -> rows y0-1 / y0+8, lane 0 / 31 -> columns x0-1 / x0+32
+    const bool hasR = (w == 0 || w == DOT_TY - 1), hasC = (lane == 0 || lane == 31);
+    const int ry = w == 0 ? y0 - 1 : y0 + DOT_TY, rx = lane == 0 ? x0 - 1 : x0 + DOT_TX;
+    const bool rin = hasR && (FULL || (xi < g.nx && ry >= 0 && ry < g.ny));
+    const bool cin = hasC && (FULL || (rx >= 0 && rx < g.nx && yi < g.ny));
+    // element offsets of plane zs-1 (halo or in-slab), advanced by ps per step
+    int64_t eo = valid ? (int64_t)zs * ps + (int64_t)yi * g.pitch + xi : 0;
+    int64_t er = rin ? (int64_t)(zs + 1) * ps + (int64_t)ry * g.pitch + xi : 0;
+    int64_t ec = cin ? (int64_t)(zs + 1) * ps + (int64_t)yi * g.pitch + rx : 0;
+    auto U = [&](int zl, int64_t e) -> double {  // map output at plane zl (uniform halo test)
+        return (zl < 0 || zl >= nzl) ? A.u[e] : fma(m, A.v[e], A.w[e]);
+    };
+    double below = 0.0, center = 0.0, vc = 0.0, xc = 0.0;
+    // raw loads of plane zs+1 (own and ring) and of plane zs (ring)
+    double va = 0.0, wa = 0.0, xa = 0.0, rv = 0.0, rw = 0.0, cv = 0.0, cw = 0.0;
+    if (valid) {
+        below = U(zs - 1, eo);
+        eo += ps;  // plane zs
+        vc = A.v[eo];
+        center = fma(m, vc, A.w[eo]);
+        if (dox) xc = A.xs[eo];
+        if (zs + 1 < nzl) {
+            va = A.v[eo + ps];
+            wa = A.w[eo + ps];
+            if (dox) xa = A.xs[eo + ps];
+        } else {
+            va = A.u[eo + ps];
+        }
+    }
+    sU[0][w + 1][lane + 1] = center;
+    if (hasR) sU[0][w == 0 ? 0 : DOT_TY + 1][lane + 1] = rin ? fma(m, A.v[er], A.w[er]) : 0.0;
+    if (hasC) sU[0][w + 1][lane == 0 ? 0 : DOT_TX + 1] = cin ? fma(m, A.v[ec], A.w[ec]) : 0.0;
+    if (zs + 1 < zend) {
+        if (rin) { rv = A.v[er + ps]; rw = A.w[er + ps]; }
+        if (cin) { cv = A.v[ec + ps]; cw = A.w[ec + ps]; }
+    }
+    for (int z = zs; z < zend; ++z) {
+        const int b = (z - zs) & 1;
+        // prefetch plane z+2 (own) and the ring of plane z+2
+        double vb = 0.0, wb = 0.0, xb = 0.0, rvb = 0.0, rwb = 0.0, cvb = 0.0, cwb = 0.0;
+        if (z + 2 <= zend) {
+            if (z + 2 < nzl) {
+                if (valid) {
+                    vb = A.v[eo + 2 * ps];
+                    wb = A.w[eo + 2 * ps];
+                    if (dox) xb = A.xs[eo + 2 * ps];
+                }
+            } else if (valid) {
+                vb = A.u[eo + 2 * ps];
+            }
+        }
+        if (z + 2 < zend) {
+            if (rin) { rvb = A.v[er + 2 * ps]; rwb = A.w[er + 2 * ps]; }
+            if (cin) { cvb = A.v[ec + 2 * ps]; cwb = A.w[ec + 2 * ps]; }
+        }
+        const double above = (z + 1 < nzl) ? fma(m, va, wa) : va;
+        __syncthreads();
+        double prod = 0.0;
+        if (valid) {
+            double s = __dadd_rn(sU[b][w + 1][lane], sU[b][w + 1][lane + 2]);
+            s = __dadd_rn(s, sU[b][w][lane + 1]);
+            s = __dadd_rn(s, sU[b][w + 2][lane + 1]);
+            s = __dadd_rn(s, below);
+            s = __dadd_rn(s, above);
+            double res;
+            if (MODE == MSR_C1) {
+                res = fma(-6.0, center, s);
+                __stcs(A.out + eo, res);
+            } else {
+                res = fma(6.0, center, -s);
+            }
+            if (DOMAP) {
+                A.u[eo] = center;
+                if (dox) A.xs[eo] = fma(ap, vc, xc);
+            }
+            prod = __dmul_rn(center, res);
+        }
+        prod = warp_sum_canon(prod);
+        if (lane == 0) sw[z - zs][w] = prod;
+        if (z + 1 < zend) {
+            sU[b ^ 1][w + 1][lane + 1] = above;
+            if (hasR) sU[b ^ 1][w == 0 ? 0 : DOT_TY + 1][lane + 1] = rin ? fma(m, rv, rw) : 0.0;
+            if (hasC) sU[b ^ 1][w + 1][lane == 0 ? 0 : DOT_TX + 1] = cin ? fma(m, cv, cw) : 0.0;
+        }
+        below = center;
+        center = above;
+        vc = va;
+        xc = xa;
+        va = vb;
+        wa = wb;
+        xa = xb;
+        rv = rvb;
+        rw = rwb;
+        cv = cvb;
+        cw = cwb;
+        eo += ps;
+        er += ps;
+        ec += ps;
+    }
+}
+
+template <int MODE, bool DOMAP>
+__global__ void __launch_bounds__(DOT_TX *DOT_TY) k_msr_fast(MsrArgs A, PGeo g, int zb, int ze, double *tp, int T,
+                                                           int tiles_y) {
+    __shared__ double sU[2][DOT_TY + 2][DOT_TX + 2];
+    __shared__ double sw[ZC][ZW];
+    if (A.sc && A.sc->status != 0) return;
+    double m = A.m, ap = A.ap;
+    int pending = A.pending;
+    if (MODE == MSR_CG) {
+        m = A.sc->beta;
+        ap = A.sc->alpha_prev;
+        pending = A.sc->pending;
+    }
+    const bool dox = MODE == MSR_CG && DOMAP && pending;
+    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
+    const int x0 = blockIdx.x * DOT_TX, y0 = blockIdx.y * DOT_TY;
+    // all own cells and all ring cells inside the domain (CTA-uniform)
+    const bool full = x0 >= 1 && y0 >= 1 && x0 + DOT_TX + 1 <= g.nx && y0 + DOT_TY + 1 <= g.ny;
+    if (full)
+        msr_fast_body<MODE, DOMAP, true>(A, g, zs, zend, m, ap, dox, sU, sw);
+    else
+        msr_fast_body<MODE, DOMAP, false>(A, g, zs, zend, m, ap, dox, sU, sw);
+    __syncthreads();
+    zm_flush<1>(sw, zend - zs, tp, (int64_t)g.z0 + zs, T, gridDim.x, tiles_y, blockIdx.x, blockIdx.y);
+}
+
 // map only: u = fma(m, v, w) on planes [zb, ze) (+ CG deferred x update);
 // boundary planes are also stored into the neighbour partition's halo plane
 // (rem_lo: lower neighbour's high halo, rem_hi: upper neighbour's low halo)
@@ -306,13 +450,21 @@ static nb_status launch_map_u(nb_grid *g, int mode, int p, MsrArgs A, const nb_f
 
 template <int MODE, bool RC, bool DM>
 static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int zb, int ze) {
+    if (ze <= zb) return NB_OK;
+    const char *name = MODE == MSR_C1 ? "k_msr_c1" : "k_msr_cgA";
+    if (RC && ZR_MAP == 1 && !getenv("NB_GENERIC_MSR")) {
+        // specialised recompute kernel (same arithmetic and dot order)
+        dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
+        LaunchScope ls(g, g->cs, name);
+        k_msr_fast<MODE, DM><<<grd, blk, 0, g->cs>>>(A, pgeo(f, p), zb, ze, g->tp, g->T, g->tiles_y);
+        return nb_launch_check(name);
+    }
     MsrOp<MODE, RC, DM> op;
     op.A = A;
     op.nzl = g->parts[p].nz();
     // recompute: the map output of every cell is computed once per CTA into
     // the staged tile; stored input: neighbours straight from L1
-    return launch_zmarch<MsrOp<MODE, RC, DM>, RC>(g, MODE == MSR_C1 ? "k_msr_c1" : "k_msr_cgA", op, pgeo(f, p),
-                                                  zb, ze);
+    return launch_zmarch<MsrOp<MODE, RC, DM>, RC>(g, name, op, pgeo(f, p), zb, ze);
 }
 
 // cross-process halo of the map output after the boundary maps (NCCL on the
