@@ -229,6 +229,7 @@ __device__ __forceinline__ void msr_fast_body(const MsrArgs &A, const PGeo &g, i
         if (rin) { rv = A.v[er + ps]; rw = A.w[er + ps]; }
         if (cin) { cv = A.v[ec + ps]; cw = A.w[ec + ps]; }
     }
+#pragma unroll 2
     for (int z = zs; z < zend; ++z) {
         const int b = (z - zs) & 1;
         // prefetch plane z+2 (own) and the ring of plane z+2

@@ -46,7 +46,10 @@
 #ifndef NB_ZR_STO
 #define NB_ZR_STO 2
 #endif
-constexpr int ZC = 32;                  // planes per CTA
+#ifndef NB_ZC
+#define NB_ZC 32
+#endif
+constexpr int ZC = NB_ZC;               // planes per CTA
 constexpr int ZW = 8;                   // warps per CTA
 constexpr int ZR_MAP = NB_ZR_MAP, ZR_STO = NB_ZR_STO;
 static_assert(DOT_TY % ZR_MAP == 0 && DOT_TY % ZR_STO == 0, "ZR must divide the dot tile height");

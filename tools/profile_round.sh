@@ -10,9 +10,9 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --
     > gpurun_out/launches_${R}.log 2>&1
 # full sections of each hot kernel (2-4 launches each)
 timeout 900 ncu --set full --clock-control none --import-source on \
-    -k regex:"k_zmarch|k_finalize|k_lbm_d3q19" -c 12 -o gpurun_out/prof_${R}_dense \
+    -k regex:"k_msr_fast|k_zmarch|k_finalize|k_lbm_d3q19" -c 12 -o gpurun_out/prof_${R}_dense \
     python tools/prof_driver.py 512 cg,lbm > gpurun_out/prof_${R}_dense.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on \
-    -k regex:"k_sp<|k_fem<|k_fem_map|k_fem_r" -c 14 -o gpurun_out/prof_${R}_sparse_fem \
+    -k regex:"^k_sp$|^k_fem$|k_fem_map|k_fem_r$" -c 16 -o gpurun_out/prof_${R}_sparse_fem \
     python tools/prof_driver.py 512 sparse,fem > gpurun_out/prof_${R}_sparse_fem.log 2>&1
 echo profile done
