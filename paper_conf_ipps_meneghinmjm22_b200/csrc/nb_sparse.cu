@@ -459,22 +459,12 @@ nb_status nb_sparse_axpby(double a, const nb_field *x, double b, nb_field *y, nb
 // plane-segment kernels: stencil / dot / CG phases.  Block = one 256-cell
 // segment of one plane; the dot value of the segment is the canonical one.
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ double seg_sum(double v, double *sw) {
-    v = warp_sum_canon(v);
-    const int w = threadIdx.x >> 5;
-    if ((threadIdx.x & 31) == 0) sw[w] = v;
-    __syncthreads();
-    double s = sw[0];
-#pragma unroll
-    for (int k = 1; k < SEG / 32; ++k) s = __dadd_rn(s, sw[k]);
-    return s;
-}
-
 enum { SPK_DOT = 0, SPK_LAP = 1, SPK_CG_INIT = 2, SPK_CG_MAP = 3, SPK_CG_Q = 4, SPK_CG_R = 5, SPK_CG_FLUSH = 6 };
 
 struct SpArgs {
     const int32_t *seg;  // segment table of the partition
     int64_t seg0;        // first table entry of this launch
+    int64_t nseg;        // table entries of this launch
     const int64_t *pstart;
     const int32_t *conn;
     int64_t n;       // own cells (conn stride)
@@ -503,44 +493,115 @@ __device__ __forceinline__ T sp_nsum(const T *x, const int32_t *conn, int64_t n,
     return s;
 }
 
+// NSB segments per block: thread t handles cell t of each of them, so every
+// thread has NSB independent loads per operand in flight; each segment keeps
+// its own canonical reduction (butterfly per warp, then the 8 warps).
+constexpr int NSB = 4;
+
 template <int K>
 __global__ void __launch_bounds__(SEG) k_sp(SpArgs A) {
-    __shared__ double sw[SEG / 32];
+    __shared__ double sw[NSB][SEG / 32];
     if (K >= SPK_CG_MAP && K <= SPK_CG_R && A.sc->status != 0) return;
-    const int e = A.seg[A.seg0 + blockIdx.x];  // non-empty segment: plane << 16 | index
-    const int zl = e >> 16, sg = e & 0xffff;
-    const int64_t j0 = A.pstart[zl], j1 = A.pstart[zl + 1];
-    const int64_t j = j0 + (int64_t)sg * SEG + threadIdx.x;
-    const bool valid = j < j1;
-    const int64_t i = A.hl + j;  // buffer index of own cell j
-    double prod = 0.0;
-    if (valid) {
-        if (K == SPK_DOT) {
-            prod = __dmul_rn(A.a[i], A.b[i]);
-        } else if (K == SPK_CG_INIT) {  // r = b - A x
-            double s = sp_nsum(A.a, A.conn, A.n, j, A.outside);
-            double r = __dsub_rn(A.b[i], fma(6.0, A.a[i], -s));
-            A.c[i] = r;
-            prod = __dmul_rn(r, r);
-        } else if (K == SPK_CG_MAP) {  // x += alpha_prev p_old (pending); p = r + beta p_old
-            double po = A.c[i];
-            if (A.sc->pending) A.d[i] = fma(A.sc->alpha_prev, po, A.d[i]);
-            A.c[i] = fma(A.sc->beta, po, A.a[i]);
-        } else if (K == SPK_CG_Q) {  // q = A p, <p, q>
-            double s = sp_nsum(A.a, A.conn, A.n, j, 0.0);
-            double pc = A.a[i];
-            double q = fma(6.0, pc, -s);
-            A.c[i] = q;
-            prod = __dmul_rn(pc, q);
-        } else if (K == SPK_CG_R) {  // r -= alpha q, <r, r>
-            double r = fma(-A.sc->alpha, A.a[i], A.c[i]);
-            A.c[i] = r;
-            prod = __dmul_rn(r, r);
+    const int t = threadIdx.x;
+    int zl[NSB], sg[NSB];
+    int64_t i[NSB], jj[NSB];
+    bool valid[NSB];
+#pragma unroll
+    for (int k = 0; k < NSB; ++k) {
+        const int64_t q = (int64_t)blockIdx.x * NSB + k;
+        zl[k] = -1;
+        sg[k] = 0;
+        valid[k] = false;
+        jj[k] = 0;
+        if (q < A.nseg) {
+            const int e = A.seg[A.seg0 + q];  // non-empty segment: plane << 16 | index
+            zl[k] = e >> 16;
+            sg[k] = e & 0xffff;
+            jj[k] = A.pstart[zl[k]] + (int64_t)sg[k] * SEG + t;
+            valid[k] = jj[k] < A.pstart[zl[k] + 1];
+        }
+        i[k] = A.hl + jj[k];  // buffer index of own cell
+    }
+    double prod[NSB];
+    if (K == SPK_DOT) {
+        double a[NSB], b[NSB];
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) {
+            a[k] = valid[k] ? A.a[i[k]] : 0.0;
+            b[k] = valid[k] ? A.b[i[k]] : 0.0;
+        }
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) prod[k] = __dmul_rn(a[k], b[k]);
+    } else if (K == SPK_CG_INIT || K == SPK_CG_Q) {  // CG_INIT: r = b - A x; CG_Q: q = A p, <p, q>
+        double s[NSB], c[NSB], bb[NSB];
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) {
+            s[k] = valid[k] ? sp_nsum(A.a, A.conn, A.n, jj[k], K == SPK_CG_INIT ? A.outside : 0.0) : 0.0;
+            c[k] = valid[k] ? A.a[i[k]] : 0.0;
+            bb[k] = (K == SPK_CG_INIT && valid[k]) ? A.b[i[k]] : 0.0;
+        }
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) {
+            prod[k] = 0.0;
+            if (!valid[k]) continue;
+            const double ac = fma(6.0, c[k], -s[k]);
+            if (K == SPK_CG_INIT) {
+                const double r = __dsub_rn(bb[k], ac);
+                A.c[i[k]] = r;
+                prod[k] = __dmul_rn(r, r);
+            } else {
+                A.c[i[k]] = ac;
+                prod[k] = __dmul_rn(c[k], ac);
+            }
+        }
+    } else if (K == SPK_CG_MAP) {  // x += alpha_prev p_old (pending); p = r + beta p_old
+        const int pending = A.sc->pending;
+        const double beta = A.sc->beta, ap = A.sc->alpha_prev;
+        double po[NSB], rr[NSB], xx[NSB];
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) {
+            po[k] = valid[k] ? A.c[i[k]] : 0.0;
+            rr[k] = valid[k] ? A.a[i[k]] : 0.0;
+            xx[k] = (valid[k] && pending) ? A.d[i[k]] : 0.0;
+        }
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) {
+            prod[k] = 0.0;
+            if (!valid[k]) continue;
+            if (pending) A.d[i[k]] = fma(ap, po[k], xx[k]);
+            A.c[i[k]] = fma(beta, po[k], rr[k]);
+        }
+    } else {  // SPK_CG_R: r -= alpha q, <r, r>
+        const double alpha = A.sc->alpha;
+        double qq[NSB], rr[NSB];
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) {
+            qq[k] = valid[k] ? A.a[i[k]] : 0.0;
+            rr[k] = valid[k] ? A.c[i[k]] : 0.0;
+        }
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) {
+            prod[k] = 0.0;
+            if (!valid[k]) continue;
+            const double r = fma(-alpha, qq[k], rr[k]);
+            A.c[i[k]] = r;
+            prod[k] = __dmul_rn(r, r);
         }
     }
     if (K == SPK_DOT || K == SPK_CG_INIT || K == SPK_CG_Q || K == SPK_CG_R) {
-        double s = seg_sum(prod, sw);
-        if (threadIdx.x == 0) A.tp[(int64_t)(A.plane0 + zl) * A.T + sg] = s;
+        const int w = t >> 5;
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) {
+            const double v = warp_sum_canon(prod[k]);
+            if ((t & 31) == 0) sw[k][w] = v;
+        }
+        __syncthreads();
+        if (t < NSB && zl[t] >= 0) {
+            double s = sw[t][0];
+#pragma unroll
+            for (int ww = 1; ww < SEG / 32; ++ww) s = __dadd_rn(s, sw[t][ww]);
+            A.tp[(int64_t)(A.plane0 + zl[t]) * A.T + sg[t]] = s;
+        }
     }
 }
 
@@ -564,6 +625,7 @@ static nb_status sp_launch(nb_grid *g, int p, int zb, int ze, SpArgs A, int plan
     if (s1 <= s0) return NB_OK;
     A.seg = sp.d_seg;
     A.seg0 = s0;
+    A.nseg = s1 - s0;
     A.pstart = sp.d_pstart;
     A.conn = sp.conn;
     A.n = sp.n;
@@ -572,7 +634,7 @@ static nb_status sp_launch(nb_grid *g, int p, int zb, int ze, SpArgs A, int plan
     A.T = g->T;
     A.tp = g->tp;
     LaunchScope ls(g, g->cs, name);
-    k_sp<K><<<(unsigned)(s1 - s0), SEG, 0, g->cs>>>(A);
+    k_sp<K><<<(unsigned)((s1 - s0 + NSB - 1) / NSB), SEG, 0, g->cs>>>(A);
     return nb_launch_check(name);
 }
 
