@@ -16,3 +16,8 @@ timeout 900 ncu --set full --clock-control none --import-source on \
     -k regex:"^k_sp$|^k_fem$|k_fem_map|k_fem_r$" -c 16 -o gpurun_out/prof_${R}_sparse_fem \
     python tools/prof_driver.py 512 sparse,fem > gpurun_out/prof_${R}_sparse_fem.log 2>&1
 echo profile done
+# kernel timelines (CUPTI via torch.profiler): 1 partition and 4 virtual partitions
+timeout 300 python tools/timeline.py 512 8 cg 1 --out gpurun_out/timeline_${R}_cg_p1.json > /dev/null 2>&1
+timeout 300 python tools/timeline.py 512 8 cg 4 --out gpurun_out/timeline_${R}_cg_p4.json > /dev/null 2>&1
+timeout 300 python tools/timeline.py 512 4 lbm 4 --out gpurun_out/timeline_${R}_lbm_p4.json > /dev/null 2>&1
+echo timelines done

@@ -14,7 +14,8 @@ import paper_conf_ipps_meneghinmjm22_b200 as nb  # noqa: E402
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 512
 iters = int(sys.argv[2]) if len(sys.argv) > 2 else 8
 what = sys.argv[3] if len(sys.argv) > 3 else "cg"
-g = nb.Grid((n, n, n))
+parts = int(sys.argv[4]) if len(sys.argv) > 4 and not sys.argv[4].startswith("--") else 1
+g = nb.Grid((n, n, n), nparts=parts, devices=[0] * parts)
 if what == "cg":
     b, x = nb.Field(g), nb.Field(g)
     b.fill(nb.FILL_POISSON_RHS)
@@ -43,7 +44,8 @@ for i, (s, e, name) in enumerate(ks):
     rows.append({"name": name[:50], "start_us": s - ks[0][0], "dur_us": e - s, "gap_us": gap})
 tot = ks[-1][1] - ks[0][0]
 busy = sum(r["dur_us"] for r in rows)
-summary = {"span_us": tot, "busy_us": busy, "idle_us": tot - busy, "kernels": len(rows)}
+summary = {"what": what, "n": n, "parts": parts, "iters": iters, "span_us": tot, "busy_us": busy,
+           "idle_us": tot - busy, "kernels": len(rows)}
 print(json.dumps(summary))
 for r in rows[:24]:
     print(f"{r['name']:50s} dur {r['dur_us']:9.1f} us  gap {r['gap_us']:7.1f} us")
