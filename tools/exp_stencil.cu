@@ -82,6 +82,79 @@ __global__ void v2(const double *__restrict__ p, double *__restrict__ r, double 
     }
 }
 
+
+// V3: z-march, per-plane products staged in shared memory, butterflies of
+// all ZC planes batched at the end of the chunk (independent chains)
+template <int ZC>
+__global__ void v3(const double *__restrict__ p, double *__restrict__ r, double a, double *tp) {
+    __shared__ double sp[ZC][8][32];
+    __shared__ double sw[ZC][8];
+    const int x = blockIdx.x * 32 + threadIdx.x, y = blockIdx.y * 8 + threadIdx.y;
+    const int zs = blockIdx.z * ZC;
+    long i = (long)(zs + 1) * PS + (long)y * NX + x;
+    double below = p[i - PS], c = p[i];
+    for (int z = zs; z < zs + ZC; ++z, i += PS) {
+        double above = p[i + PS];
+        double s = (x > 0 ? p[i - 1] : 0.0) + (x < NX - 1 ? p[i + 1] : 0.0);
+        s += (y > 0 ? p[i - NX] : 0.0);
+        s += (y < NY - 1 ? p[i + NX] : 0.0);
+        s += below;
+        s += above;
+        double q = fma(6.0, c, -s);
+        double rn = fma(-a, q, r[i]);
+        r[i] = rn;
+        sp[z - zs][threadIdx.y][threadIdx.x] = rn * rn;
+        below = c;
+        c = above;
+    }
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < ZC; ++k) {
+        double v = wsum(sp[k][threadIdx.y][threadIdx.x]);
+        if (threadIdx.x == 0) sw[k][threadIdx.y] = v;
+    }
+    __syncthreads();
+    int t = threadIdx.y * 32 + threadIdx.x;
+    if (t < ZC) {
+        double s = sw[t][0];
+        for (int k = 1; k < 8; ++k) s += sw[t][k];
+        tp[(long)(zs + t) * 1024 + blockIdx.y * 16 + blockIdx.x] = s;
+    }
+}
+
+// V4: v2 with the z loop unrolled by 2
+template <int ZC>
+__global__ void v4(const double *__restrict__ p, double *__restrict__ r, double a, double *tp) {
+    __shared__ double sw[ZC][8];
+    const int x = blockIdx.x * 32 + threadIdx.x, y = blockIdx.y * 8 + threadIdx.y;
+    const int zs = blockIdx.z * ZC;
+    long i = (long)(zs + 1) * PS + (long)y * NX + x;
+    double below = p[i - PS], c = p[i];
+#pragma unroll 2
+    for (int z = zs; z < zs + ZC; ++z, i += PS) {
+        double above = p[i + PS];
+        double s = (x > 0 ? p[i - 1] : 0.0) + (x < NX - 1 ? p[i + 1] : 0.0);
+        s += (y > 0 ? p[i - NX] : 0.0);
+        s += (y < NY - 1 ? p[i + NX] : 0.0);
+        s += below;
+        s += above;
+        double q = fma(6.0, c, -s);
+        double rn = fma(-a, q, r[i]);
+        r[i] = rn;
+        double v = wsum(rn * rn);
+        if (threadIdx.x == 0) sw[z - zs][threadIdx.y] = v;
+        below = c;
+        c = above;
+    }
+    __syncthreads();
+    int t = threadIdx.y * 32 + threadIdx.x;
+    if (t < ZC) {
+        double s = sw[t][0];
+        for (int k = 1; k < 8; ++k) s += sw[t][k];
+        tp[(long)(zs + t) * 1024 + blockIdx.y * 16 + blockIdx.x] = s;
+    }
+}
+
 template <typename F>
 float timeit(F f, int reps = 20) {
     cudaEvent_t a, b;
@@ -115,6 +188,12 @@ int main() {
     rep("v2 zmarch32 dot", timeit([&] { v2<true, 32><<<dim3(16, 64, NZ / 32), b>>>(p, r, 1e-3, tp); }));
     rep("v2 zmarch8 dot", timeit([&] { v2<true, 8><<<dim3(16, 64, NZ / 8), b>>>(p, r, 1e-3, tp); }));
     rep("v2 zmarch4 dot", timeit([&] { v2<true, 4><<<dim3(16, 64, NZ / 4), b>>>(p, r, 1e-3, tp); }));
+    rep("v3 staged8", timeit([&] { v3<8><<<dim3(16, 64, NZ / 8), b>>>(p, r, 1e-3, tp); }));
+    rep("v3 staged16", timeit([&] { v3<16><<<dim3(16, 64, NZ / 16), b>>>(p, r, 1e-3, tp); }));
+    rep("v4 unroll2 zc32", timeit([&] { v4<32><<<dim3(16, 64, NZ / 32), b>>>(p, r, 1e-3, tp); }));
+    rep("v0 stream (again)", timeit([&] { v0<<<148 * 16, 256>>>(p, r, 1e-3, n); }));
+    rep("v2 zmarch32 nodot (again)", timeit([&] { v2<false, 32><<<dim3(16, 64, NZ / 32), b>>>(p, r, 1e-3, tp); }));
+    rep("v2 zmarch32 dot (again)", timeit([&] { v2<true, 32><<<dim3(16, 64, NZ / 32), b>>>(p, r, 1e-3, tp); }));
     cudaError_t e = cudaDeviceSynchronize();
     printf("status %s\n", cudaGetErrorString(e));
     return 0;
