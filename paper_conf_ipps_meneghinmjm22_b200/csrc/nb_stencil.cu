@@ -31,6 +31,9 @@
 std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v);
 nb_status nb_dot_partials(const nb_field *x, const nb_field *y);
 nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v);
+bool nb_tma_enabled();
+nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x, bool domap,
+                     int zb, int ze, const CgScal *sc);
 
 static inline int64_t dcs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
 
@@ -453,6 +456,8 @@ template <int MODE, bool RC, bool DM>
 static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int zb, int ze) {
     if (ze <= zb) return NB_OK;
     const char *name = MODE == MSR_C1 ? "k_msr_c1" : "k_msr_cgA";
+    if (MODE == MSR_CG && RC && ZR_MAP == 1 && nb_tma_enabled())  // TMA-staged phase A
+        return nb_cgA_tma(g, pgeo(f, p), A.w, A.v, A.u, A.xs, DM, zb, ze, A.sc);
     if (RC && ZR_MAP == 1 && !getenv("NB_GENERIC_MSR")) {
         // specialised recompute kernel (same arithmetic and dot order)
         dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
