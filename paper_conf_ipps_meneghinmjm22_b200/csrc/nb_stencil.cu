@@ -32,6 +32,7 @@ std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v)
 nb_status nb_dot_partials(const nb_field *x, const nb_field *y);
 nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v);
 bool nb_tma_enabled();
+nb_status nb_cgB_tma(nb_grid *g, const PGeo &geo, const double *p, double *r, int zb, int ze, const CgScal *sc);
 nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x, bool domap,
                      int zb, int ze, const CgScal *sc);
 
@@ -631,6 +632,10 @@ static nb_status cg_enqueue_iteration(nb_cg *cg) {
     NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_PQ, cg->sc, 0));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         PGeo geo = pgeo(pn, p);
+        if (ZR_STO == 1 && nb_tma_enabled()) {  // TMA-staged phase B
+            NB_TRY(nb_cgB_tma(g, geo, (const double *)pn->base[p], (double *)cg->r->base[p], 0, geo.nzl, cg->sc));
+            continue;
+        }
         CgBOp op{(const double *)pn->base[p], (double *)cg->r->base[p], cg->sc, 0.0};
         NB_TRY(launch_zmarch(g, "k_cg_B", op, geo, 0, geo.nzl));
     }

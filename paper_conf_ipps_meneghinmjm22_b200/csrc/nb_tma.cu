@@ -161,6 +161,85 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY)
 }
 
 // ---------------------------------------------------------------------------
+// CG phase B, TMA-staged: q = A p_new from the stored p_new (36 x 10 box per
+// plane, halo planes included), r -= alpha q (32 x 8 box of r per plane),
+// per-plane tile partial of r*r in the ZR = 1 canonical order (butterfly per
+// row, rows in increasing y).
+// ---------------------------------------------------------------------------
+struct __align__(128) CgBStage {
+    double p[BY][BX];
+    double pad0[(TPAD - BY * BX * 8) / 8];
+    double r[DOT_TY][DOT_TX];
+};
+
+__global__ void __launch_bounds__(DOT_TX *DOT_TY)
+    k_cgB_tma(const __grid_constant__ CUtensorMap m_p, const __grid_constant__ CUtensorMap m_r, double *r, PGeo g,
+              int zb, int ze, const CgScal *sc, double *tp, int T) {
+    __shared__ CgBStage st[NSTAGE];
+    __shared__ __align__(8) uint64_t bar[NSTAGE];
+    __shared__ double sw[TZC][DOT_TY];
+    if (sc->status != 0) return;
+    const double alpha = sc->alpha;
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const int x0 = blockIdx.x * DOT_TX, y0 = blockIdx.y * DOT_TY;
+    const int xi = x0 + lane, yi = y0 + w;
+    const int zs = zb + blockIdx.z * TZC, zend = min(ze, zs + TZC);
+    const bool valid = xi < g.nx && yi < g.ny;
+    auto stage_of = [&](int zl) { return (zl - zs + 1) & (NSTAGE - 1); };
+    auto parity_of = [&](int zl) { return (uint32_t)(((zl - zs + 1) / NSTAGE) & 1); };
+    auto issue = [&](int zl) {
+        CgBStage &s = st[stage_of(zl)];
+        uint64_t *b = &bar[stage_of(zl)];
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        const bool wr = zl >= zs && zl < zend;
+        mbar_expect_tx(b, BY * BX * 8 + (wr ? DOT_TY * DOT_TX * 8 : 0));
+        tma_load_3d(&s.p[0][0], &m_p, b, x0 - 2, y0 - 1, zl + 1);
+        if (wr) tma_load_3d(&s.r[0][0], &m_r, b, x0, y0, zl + 1);
+    };
+    if (tid == 0) {
+        for (int k = 0; k < NSTAGE; ++k) mbar_init(&bar[k], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (tid == 0)
+        for (int zl = zs - 1; zl <= min(zs + 2, zend); ++zl) issue(zl);
+    mbar_wait(&bar[stage_of(zs - 1)], parity_of(zs - 1));
+    mbar_wait(&bar[stage_of(zs)], parity_of(zs));
+    double below = st[stage_of(zs - 1)].p[w + 1][lane + 2];
+    double center = st[stage_of(zs)].p[w + 1][lane + 2];
+    const int64_t o = (int64_t)yi * g.pitch + xi + g.ps;
+    for (int z = zs; z < zend; ++z) {
+        mbar_wait(&bar[stage_of(z + 1)], parity_of(z + 1));
+        const CgBStage &sz = st[stage_of(z)];
+        const double above = st[stage_of(z + 1)].p[w + 1][lane + 2];
+        double prod = 0.0;
+        if (valid) {
+            double s = __dadd_rn(sz.p[w + 1][lane + 1], sz.p[w + 1][lane + 3]);
+            s = __dadd_rn(s, sz.p[w][lane + 2]);
+            s = __dadd_rn(s, sz.p[w + 2][lane + 2]);
+            s = __dadd_rn(s, below);
+            s = __dadd_rn(s, above);
+            const double q = fma(6.0, center, -s);
+            const double rn = fma(-alpha, q, sz.r[w][lane]);
+            __stcs(r + o + (int64_t)z * g.ps, rn);
+            prod = __dmul_rn(rn, rn);
+        }
+        prod = warp_sum_canon(prod);
+        if (lane == 0) sw[z - zs][w] = prod;
+        below = center;
+        center = above;
+        __syncthreads();
+        if (tid == 0 && z + 3 <= zend) issue(z + 3);
+    }
+    if (tid < zend - zs) {
+        double s = sw[tid][0];
+#pragma unroll
+        for (int k = 1; k < DOT_TY; ++k) s = __dadd_rn(s, sw[tid][k]);
+        tp[((int64_t)g.z0 + zs + tid) * T + blockIdx.y * gridDim.x + blockIdx.x] = s;
+    }
+}
+
+// ---------------------------------------------------------------------------
 // host side: tensor maps (cached per buffer and geometry)
 // ---------------------------------------------------------------------------
 typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
@@ -241,4 +320,16 @@ nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double 
     else
         k_cgA_tma<false><<<grd, blk, 0, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T, g->tiles_y);
     return nb_launch_check("k_cgA_tma");
+}
+
+// CG phase B on planes [zb, ze) of a partition (stored p_new, r)
+nb_status nb_cgB_tma(nb_grid *g, const PGeo &geo, const double *p, double *r, int zb, int ze, const CgScal *sc) {
+    if (ze <= zb) return NB_OK;
+    CUtensorMap mp, mr;
+    NB_TRY(tmap_for(p, geo, 0, &mp));
+    NB_TRY(tmap_for(r, geo, 1, &mr));
+    dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + TZC - 1) / TZC);
+    LaunchScope ls(g, g->cs, "k_cg_B");
+    k_cgB_tma<<<grd, blk, 0, g->cs>>>(mp, mr, r, geo, zb, ze, sc, g->tp, g->T);
+    return nb_launch_check("k_cgB_tma");
 }

@@ -44,7 +44,7 @@
 #define NB_ZR_MAP 1
 #endif
 #ifndef NB_ZR_STO
-#define NB_ZR_STO 2
+#define NB_ZR_STO 1
 #endif
 #ifndef NB_ZC
 #define NB_ZC 32
