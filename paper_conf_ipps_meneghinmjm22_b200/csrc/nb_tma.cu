@@ -21,6 +21,7 @@
 
 #include "nb_device.cuh"
 #include "nb_internal.cuh"
+#include "nb_tma.cuh"
 
 #ifndef NB_ZC
 #define NB_ZC 32
@@ -40,35 +41,6 @@ struct __align__(128) CgAStage {
     double xs[DOT_TY][DOT_TX];  // x of the own cells
 };
 static_assert(sizeof(double) * BY * BX < TPAD && TPAD % 128 == 0, "stage tile padding");
-
-__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
-    uint32_t done;
-    do {
-        asm volatile(
-            "{\n\t.reg .pred p;\n\t"
-            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-            "selp.u32 %0, 1, 0, p;\n\t}"
-            : "=r"(done)
-            : "r"(smem_u32(bar)), "r"(parity)
-            : "memory");
-    } while (!done);
-}
-__device__ __forceinline__ void tma_load_3d(void *dst, const CUtensorMap *map, uint64_t *bar, int c0, int c1, int c2) {
-    asm volatile(
-        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::
-            "r"(smem_u32(dst)),
-        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(c2), "r"(smem_u32(bar))
-        : "memory");
-}
 
 template <bool DOMAP>
 __global__ void __launch_bounds__(DOT_TX *DOT_TY)
@@ -266,7 +238,7 @@ static std::mutex g_tmap_mu;
 static std::map<std::tuple<const void *, int, int, int, int64_t, int>, CUtensorMap> g_tmaps;
 
 // box: 0 = (tile + ring) 36 x 10 x 1 (x from x0-2), 1 = own tile 32 x 8 x 1
-static nb_status tmap_for(const void *base, const PGeo &g, int box, CUtensorMap *out) {
+nb_status tmap_for(const void *base, const PGeo &g, int box, CUtensorMap *out) {
     std::lock_guard<std::mutex> lk(g_tmap_mu);
     auto key = std::make_tuple(base, g.nx, g.ny, g.nzl, g.pitch, box);
     auto it = g_tmaps.find(key);
