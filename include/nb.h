@@ -163,6 +163,14 @@ nb_status nb_grid_partition_info(const nb_grid *grid, int32_t g, nb_part_info *o
  * library's own.  Either may be NULL to keep the current one. */
 nb_status nb_grid_set_streams(nb_grid *grid, void *compute_stream, void *halo_stream);
 nb_status nb_grid_get_stream(const nb_grid *grid, void **compute_stream);
+/* Halo transport for partitions of this process: NB_HALO_FUSED (default)
+ * stores boundary-plane outputs straight into the neighbour's halo from the
+ * producing kernel; NB_HALO_STREAM issues them as device copies on the halo
+ * stream, ordered by events and overlapped with the interior kernels (the
+ * cross-process path always uses the halo stream, with NCCL). */
+#define NB_HALO_FUSED 0
+#define NB_HALO_STREAM 1
+nb_status nb_grid_set_halo_mode(nb_grid *grid, int32_t mode);
 /* synchronises: waits for all work of the grid, reports async errors */
 nb_status nb_sync(nb_grid *grid);
 

@@ -33,6 +33,7 @@ OCC_NONE, OCC_STANDARD, OCC_EXTENDED, OCC_TWO_WAY = 0, 1, 2, 3
 FILL_CONST, FILL_UNIFORM, FILL_INT_UNIFORM, FILL_POISSON_RHS = 0, 1, 2, 3
 OP_LAPLACE7, OP_FEM27 = 0, 1
 LBM_CAVITY, LBM_PERIODIC = 0, 1
+HALO_FUSED, HALO_STREAM = 0, 1
 OCC_NAMES = {"none": OCC_NONE, "standard": OCC_STANDARD, "extended": OCC_EXTENDED, "two_way": OCC_TWO_WAY}
 
 
@@ -82,6 +83,7 @@ SIGNATURES = {
     "nb_grid_set_streams": ([P, P, P], I32),
     "nb_grid_get_stream": ([P, PP], I32),
     "nb_sync": ([P], I32),
+    "nb_grid_set_halo_mode": ([P, I32], I32),
     "nb_field_create": ([P, I32, I32, D, PP], I32),
     "nb_field_destroy": ([P], I32),
     "nb_field_upload": ([P, P, I64], I32),
@@ -262,6 +264,11 @@ class Grid:
 
     def sync(self):
         _check(lib().nb_sync(self.handle))
+
+    def set_halo_mode(self, mode: int):
+        """HALO_FUSED (stores from the boundary kernels) or HALO_STREAM
+        (device copies on the halo stream, overlapped with the interior)."""
+        _check(lib().nb_grid_set_halo_mode(self.handle, int(mode)))
 
     def launch_count(self) -> int:
         n = C.c_int64()

@@ -514,6 +514,13 @@ extern "C" nb_status nb_grid_get_stream(const nb_grid *g, void **cs) {
     return NB_OK;
 }
 
+extern "C" nb_status nb_grid_set_halo_mode(nb_grid *g, int32_t mode) {
+    if (!g) NB_FAIL(NB_EINVAL, "NULL grid");
+    if (mode != NB_HALO_FUSED && mode != NB_HALO_STREAM) NB_FAIL(NB_EINVAL, "bad halo mode %d", mode);
+    g->halo_mode = mode;
+    return NB_OK;
+}
+
 extern "C" nb_status nb_sync(nb_grid *g) {
     if (!g) NB_FAIL(NB_EINVAL, "NULL grid");
     DeviceGuard dg(g->device);

@@ -114,6 +114,7 @@ struct nb_grid {
     double *dots = nullptr;       // [NB_DOT_SLOTS] reduce results
     unsigned int *counter = nullptr;
     int nfields = 0, nsolvers = 0;
+    int halo_mode = 0;  // NB_HALO_FUSED / NB_HALO_STREAM
     bool profiling = false;
     std::vector<ProfRec> prof;
     int64_t launches = 0;
@@ -223,6 +224,10 @@ nb_status nb_nccl_send(nb_grid *g, const void *buf, size_t bytes, int peer, cuda
 nb_status nb_nccl_recv(nb_grid *g, void *buf, size_t bytes, int peer, cudaStream_t s);
 
 int nb_part_owner(const nb_grid *g, int part);
+// halos travel on the halo stream (multi-process, or NB_HALO_STREAM)
+inline bool nb_halo_on_stream(const nb_grid *g) {
+    return (g->comm && g->comm->world > 1) || g->halo_mode == NB_HALO_STREAM;
+}
 
 // halo overlap events of a schedule (multi-process)
 struct HaloSync {

@@ -253,7 +253,7 @@ extern "C" nb_status nb_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm
     nb_grid *g = fin->g;
     cudaSetDevice(g->device);
     const bool per = prm->bc == NB_LBM_PERIODIC;
-    const bool dist = g->comm && g->comm->world > 1;
+    const bool dist = nb_halo_on_stream(g);  // halos on the halo stream (NCCL or device copies)
     // make fin's halos current (covers states written by upload/init)
     NB_TRY(lbm_halo(fin, per, g->cs));
     HaloSync hs;
@@ -268,14 +268,14 @@ extern "C" nb_status nb_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm
             int nz = g->parts[p].nz();
             bool blo = lbm_lo(g, p, per) >= 0, bhi = lbm_hi(g, p, per) >= 0;
             if (occ == NB_OCC_NONE || (!blo && !bhi)) {
-                st = launch_lbm(g, p, fin, fout, prm, 0, nz, true);
+                st = launch_lbm(g, p, fin, fout, prm, 0, nz, !dist);
             } else {
-                if (blo) st = launch_lbm(g, p, fin, fout, prm, 0, 1, true);
-                if (st == NB_OK && bhi && !(blo && nz == 1)) st = launch_lbm(g, p, fin, fout, prm, nz - 1, nz, true);
+                if (blo) st = launch_lbm(g, p, fin, fout, prm, 0, 1, !dist);
+                if (st == NB_OK && bhi && !(blo && nz == 1)) st = launch_lbm(g, p, fin, fout, prm, nz - 1, nz, !dist);
             }
         }
         if (st != NB_OK) break;
-        if (dist) {  // remote halos on the halo stream, overlapped with the interior
+        if (dist) {  // halos on the halo stream, overlapped with the interior
             cudaEventRecord(hs.eb, g->cs);
             cudaStreamWaitEvent(g->hs, hs.eb, 0);
             st = lbm_halo(fout, per, g->hs);

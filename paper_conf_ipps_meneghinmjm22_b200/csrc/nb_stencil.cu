@@ -442,8 +442,10 @@ static nb_status launch_map_u(nb_grid *g, int mode, int p, MsrArgs A, const nb_f
     const NbPart &q = g->parts[p];
     PGeo geo = pgeo(ufield, p);
     double *rem_lo = nullptr, *rem_hi = nullptr;
-    if (zb == 0 && q.lo >= 0 && g->parts[q.lo].local) rem_lo = pl(ufield, q.lo, g->parts[q.lo].nz());
-    if (ze == q.nz() && q.hi >= 0 && g->parts[q.hi].local) rem_hi = pl(ufield, q.hi, -1);
+    if (!nb_halo_on_stream(g)) {  // fused halo: store straight into the neighbour
+        if (zb == 0 && q.lo >= 0 && g->parts[q.lo].local) rem_lo = pl(ufield, q.lo, g->parts[q.lo].nz());
+        if (ze == q.nz() && q.hi >= 0 && g->parts[q.hi].local) rem_hi = pl(ufield, q.hi, -1);
+    }
     dim3 blk(128), grd((g->nx + 127) / 128, g->ny, std::min(ze - zb, 64));
     LaunchScope ls(g, g->cs, "k_map_u");
     if (mode == MSR_C1)
@@ -474,13 +476,15 @@ static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int
     return launch_zmarch<MsrOp<MODE, RC, DM>, RC>(g, name, op, pgeo(f, p), zb, ze);
 }
 
-// cross-process halo of the map output after the boundary maps (NCCL on the
-// halo stream, overlapped with the internal work of the compute stream)
+// halo of the map output after the boundary maps on the halo stream (NCCL
+// across processes, device copies within one), overlapped with the internal
+// work of the compute stream and joined by an event before the boundary
+// stencils
 
 static bool is_dist(const nb_grid *g) { return g->comm && g->comm->world > 1; }
 
 static nb_status dist_halo_begin(nb_grid *g, nb_field *u, HaloSync &hsync) {
-    if (!is_dist(g)) return NB_OK;
+    if (!nb_halo_on_stream(g)) return NB_OK;
     if (!hsync.eb) {
         NB_CUDA(cudaEventCreateWithFlags(&hsync.eb, cudaEventDisableTiming));
         NB_CUDA(cudaEventCreateWithFlags(&hsync.eh, cudaEventDisableTiming));
@@ -492,7 +496,7 @@ static nb_status dist_halo_begin(nb_grid *g, nb_field *u, HaloSync &hsync) {
     return NB_OK;
 }
 static nb_status dist_halo_wait(nb_grid *g, HaloSync &hsync) {
-    if (!is_dist(g)) return NB_OK;
+    if (!nb_halo_on_stream(g)) return NB_OK;
     NB_CUDA(cudaStreamWaitEvent(g->cs, hsync.eh, 0));
     return NB_OK;
 }

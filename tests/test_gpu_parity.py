@@ -417,3 +417,31 @@ def test_errors_are_reported_not_crashing():
     with pytest.raises(nb.NbError) as e:
         nb.Grid((8, 8, 3), nparts=2, devices=[0, 0])
     assert e.value.status == nb.NB_EUNSUPPORTED
+
+
+# ---- halo transport: fused stores vs copies on the halo stream -------------
+def test_halo_stream_mode_bitwise_equals_fused():
+    """NB_HALO_STREAM (device copies on the halo stream, ordered by events and
+    overlapped with the interior) must give the same bits as the fused halo
+    stores, for CG, C1 and LBM under every OCC mode."""
+    dims = (45, 19, 37)
+    bh = synth.uniform(dims, seed=3)
+    f0 = lbm_state(dims, 8)
+    for occ in (nb.OCC_NONE, nb.OCC_STANDARD, nb.OCC_EXTENDED):
+        outs = []
+        for mode in (nb.HALO_FUSED, nb.HALO_STREAM):
+            with grid(dims, 3) as g:
+                g.set_halo_mode(mode)
+                b = field(g, bh)
+                x = field(g, np.zeros(dims[::-1]))
+                r = nb.nb_cg_solve(x, b, max_iter=9, occ=occ)
+                y = field(g, np.zeros(dims[::-1]))
+                x2 = field(g, bh)
+                d = nb.nb_map_stencil_reduce(x2, y, 0.125, 4, occ)
+                a, c = field(g, f0, "f32", 19), field(g, dtype="f32", card=19)
+                a2, _ = nb.nb_lbm_step(a, c, 1.2, 4, occ=min(occ, nb.OCC_STANDARD))
+                outs.append((x.download(), r.rr, x2.download(), y.download(), d, a2.download()))
+                for f in (b, x, y, x2, a, c):
+                    f.close()
+        for u, v in zip(outs[0], outs[1]):
+            assert np.array_equal(u, v), occ

@@ -15,7 +15,9 @@ n = int(sys.argv[1]) if len(sys.argv) > 1 else 512
 iters = int(sys.argv[2]) if len(sys.argv) > 2 else 8
 what = sys.argv[3] if len(sys.argv) > 3 else "cg"
 parts = int(sys.argv[4]) if len(sys.argv) > 4 and not sys.argv[4].startswith("--") else 1
+hmode = int(sys.argv[5]) if len(sys.argv) > 5 and not sys.argv[5].startswith("--") else 0
 g = nb.Grid((n, n, n), nparts=parts, devices=[0] * parts)
+g.set_halo_mode(hmode)
 if what == "cg":
     b, x = nb.Field(g), nb.Field(g)
     b.fill(nb.FILL_POISSON_RHS)
@@ -38,14 +40,38 @@ else:
         g.sync()
 evs = [e for e in prof.events() if e.device_type == torch.autograd.DeviceType.CUDA]
 ks = sorted([(e.time_range.start, e.time_range.end, e.name) for e in evs])
+# halo copies vs kernels: fraction of copy time overlapped by a running kernel
+copies = [(s, e) for s, e, nm in ks if "Memcpy" in nm or "memcpy" in nm]
+kern = [(s, e) for s, e, nm in ks if not ("Memcpy" in nm or "memcpy" in nm)]
+cov = 0.0
+for cs_, ce_ in copies:
+    segs = sorted((max(cs_, s), min(ce_, e)) for s, e in kern if s < ce_ and e > cs_)
+    t, cur = 0.0, cs_
+    for s, e in segs:
+        s = max(s, cur)
+        if e > s:
+            t += e - s
+            cur = e
+    cov += t
+copy_t = sum(e - s for s, e in copies)
 rows = []
 for i, (s, e, name) in enumerate(ks):
     gap = s - ks[i - 1][1] if i else 0.0
     rows.append({"name": name[:50], "start_us": s - ks[0][0], "dur_us": e - s, "gap_us": gap})
 tot = ks[-1][1] - ks[0][0]
-busy = sum(r["dur_us"] for r in rows)
-summary = {"what": what, "n": n, "parts": parts, "iters": iters, "span_us": tot, "busy_us": busy,
-           "idle_us": tot - busy, "kernels": len(rows)}
+# busy = union of device activity (kernels and copies may overlap)
+busy, cur = 0.0, None
+for s_, e_, _ in ks:
+    if cur is None or s_ > cur[1]:
+        if cur:
+            busy += cur[1] - cur[0]
+        cur = [s_, e_]
+    else:
+        cur[1] = max(cur[1], e_)
+busy += cur[1] - cur[0] if cur else 0.0
+summary = {"what": what, "n": n, "parts": parts, "halo_mode": hmode, "iters": iters, "span_us": tot,
+           "busy_us": busy, "idle_us": tot - busy, "kernels": len(rows), "halo_copies": len(copies),
+           "halo_copy_us": copy_t, "halo_copy_overlapped_frac": (cov / copy_t) if copy_t else None}
 print(json.dumps(summary))
 for r in rows[:24]:
     print(f"{r['name']:50s} dur {r['dur_us']:9.1f} us  gap {r['gap_us']:7.1f} us")
