@@ -93,6 +93,29 @@ nb_status nb_comm_create(int32_t world, int32_t rank, const uint8_t id[128], int
                          nb_comm **out);
 nb_status nb_comm_destroy(nb_comm *comm);
 
+/* Peer-memory transport (PAPER.md L252-L256 explicit GPU-to-GPU transfers,
+ * SURVEY.md §8(e) "P2P stores from the boundary kernel"): no NCCL on the
+ * data path.  Every field partition adjacent to this rank's slabs, and every
+ * rank's reduction buffer and flag words, are mapped into this process with
+ * CUDA IPC; boundary kernels store their halo planes straight into the
+ * neighbour's halo (over NVLink / NVSwitch, or locally when several
+ * processes share one GPU), plane sums of a reduction are stored into every
+ * rank, and completion is a system-scope release store of a counter that
+ * the consumer's kernel acquires.  Ordering is stream order + these flags.
+ *
+ * ag(ctx, send, bytes, recv): host allgather used ONLY during setup and
+ * teardown (IPC handle exchange, barrier): every rank passes `bytes` bytes,
+ * recv receives world*bytes bytes ordered by rank; return 0 on success.
+ * It is called from inside nb_grid_create_*, nb_grid_destroy,
+ * nb_field_create and nb_field_destroy, which therefore become collective:
+ * every rank makes the same calls in the same order.  world <= 16.
+ * Comm and callback must outlive every grid built on them. */
+typedef int32_t (*nb_allgather_fn)(void *ctx, const void *send, int64_t bytes, void *recv);
+nb_status nb_comm_create_peer(int32_t world, int32_t rank, int32_t device, nb_allgather_fn ag, void *ctx,
+                              nb_comm **out);
+/* 1 if comm uses the peer-memory transport, 0 if NCCL */
+nb_status nb_comm_is_peer(const nb_comm *comm, int32_t *is_peer);
+
 /* ---- grid (PAPER.md L81-L88 Domain, L244 Grid, L256 1-D decomposition) -- */
 /* Pure host logic (no GPU needed): the z-slab partition of a1 — partition g
  * owns planes [z_begin[g], z_begin[g+1]); the first (nz mod nparts)

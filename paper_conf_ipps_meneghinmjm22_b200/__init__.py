@@ -72,6 +72,8 @@ SIGNATURES = {
     "nb_comm_unique_id": ([P], I32),
     "nb_comm_create": ([I32, I32, P, I32, PP], I32),
     "nb_comm_destroy": ([P], I32),
+    "nb_comm_create_peer": ([I32, I32, I32, P, P, PP], I32),
+    "nb_comm_is_peer": ([P, P], I32),
     "nb_partition_plan": ([I32, I32, P], I32),
     "nb_partition_plan_weighted": ([I32, P, I32, P], I32),
     "nb_halo_plan": ([I32, I32, I32, I32, I32, P, I32, P], I32),
@@ -188,14 +190,53 @@ def nb_halo_plan(nz: int, nparts: int, world: int = 1, rank: int = -1, periodic:
 
 
 # ---------------------------------------------------------------------------
-class Comm:
-    """One process per GPU: an NCCL communicator created inside libnb.  The
-    128-byte unique id is broadcast with torch.distributed (plumbing)."""
+# host allgather callback of the peer-memory transport (include/nb.h)
+ALLGATHER_FN = C.CFUNCTYPE(C.c_int32, C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p)
 
-    def __init__(self, world: int, rank: int, device: int, uid: bytes):
+
+def _torch_allgather(world: int, group):
+    """nb_allgather_fn over a CPU (gloo) torch.distributed group: setup-time
+    plumbing only (IPC handles, teardown barriers), never on the data path."""
+    import traceback
+
+    import torch
+    import torch.distributed as dist
+
+    def ag(ctx, send, nbytes, recv):
+        try:
+            mine = torch.frombuffer(bytearray(C.string_at(send, nbytes)), dtype=torch.uint8)
+            outs = [torch.empty(nbytes, dtype=torch.uint8) for _ in range(world)]
+            dist.all_gather(outs, mine, group=group)
+            data = b"".join(o.numpy().tobytes() for o in outs)
+            C.memmove(recv, data, len(data))
+            return 0
+        except Exception:  # reported to libnb as a failed collective
+            traceback.print_exc()
+            return 1
+
+    return ALLGATHER_FN(ag)
+
+
+class Comm:
+    """One process per GPU.  transport="peer" (default): libnb's
+    peer-memory transport — CUDA IPC mappings of the neighbours' halos and of
+    every rank's reduction buffer, kernels store across GPUs and signal with
+    device flags; torch.distributed (gloo) only exchanges IPC handles at
+    setup.  transport="nccl": an NCCL communicator inside libnb (the 128-byte
+    unique id is broadcast with torch.distributed)."""
+
+    def __init__(self, world: int, rank: int, device: int, uid: bytes | None = None, allgather=None):
         self.handle = P()
-        buf = (C.c_uint8 * 128).from_buffer_copy(uid)
-        _check(lib().nb_comm_create(world, rank, buf, device, C.byref(self.handle)))
+        self._ag = None
+        if allgather is not None:
+            self._ag = allgather  # keep the callback alive as long as the comm
+            _check(lib().nb_comm_create_peer(world, rank, device, C.cast(allgather, C.c_void_p), None,
+                                             C.byref(self.handle)))
+            self.transport = "peer"
+        else:
+            buf = (C.c_uint8 * 128).from_buffer_copy(uid)
+            _check(lib().nb_comm_create(world, rank, buf, device, C.byref(self.handle)))
+            self.transport = "nccl"
         self.world, self.rank, self.device = world, rank, device
 
     @staticmethod
@@ -205,10 +246,19 @@ class Comm:
         return bytes(buf)
 
     @classmethod
-    def from_torch_distributed(cls, device: int):
-        import torch
+    def from_torch_distributed(cls, device: int, transport: str | None = None):
+        """Build the communicator of the current torch.distributed world;
+        transport defaults to $NB_TRANSPORT or "peer"."""
         import torch.distributed as dist
+        transport = transport or os.environ.get("NB_TRANSPORT", "peer")
         world, rank = dist.get_world_size(), dist.get_rank()
+        if transport == "peer":
+            group = dist.new_group(backend="gloo") if dist.get_backend() != "gloo" else None
+            comm = cls(world, rank, device, allgather=_torch_allgather(world, group))
+            comm._group = group
+            return comm
+        if transport != "nccl":
+            raise ValueError(f"transport must be 'peer' or 'nccl', got {transport!r}")
         uid = [cls.unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
         return cls(world, rank, device, uid[0])

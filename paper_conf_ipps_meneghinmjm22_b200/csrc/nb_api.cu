@@ -46,18 +46,6 @@ nb_status nb_launch_check(const char *what) {
     return NB_OK;
 }
 
-struct DeviceGuard {
-    int prev = -1;
-    explicit DeviceGuard(int d) {
-        cudaGetDevice(&prev);
-        if (prev != d) cudaSetDevice(d);
-    }
-    ~DeviceGuard() {
-        int cur = -1;
-        cudaGetDevice(&cur);
-        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
-    }
-};
 
 // ===========================================================================
 // NCCL, loaded at run time (no link-time dependency; one process per GPU)
@@ -285,6 +273,37 @@ extern "C" nb_status nb_halo_plan(int32_t nz, int32_t nparts, int32_t world, int
 // Execute the halo messages of field f for this process: local messages are
 // device copies, remote ones grouped NCCL send/recv on stream s.  comps(up)
 // gives the component range [c0, c1) carried by up / down messages.
+// ---------------------------------------------------------------------------
+// batched device-local plane copies: up to MAX (dst, src, bytes) descriptors
+// per launch, passed by value; blocks are dealt to descriptors by a prefix of
+// block counts.  16-byte vectors when every address and size allows it, else
+// 4-byte words (every field element is >= 4 bytes).
+// ---------------------------------------------------------------------------
+
+__global__ void __launch_bounds__(256) k_halo_copy(const __grid_constant__ CopyBatch cb) {
+    const uint32_t b = blockIdx.x;
+    int d = 0;
+    while (d + 1 < cb.n && cb.bstart[d + 1] <= b) ++d;
+    const uint64_t w0 = (uint64_t)(b - cb.bstart[d]) * CopyBatch::CHUNK;
+    const uint64_t w1 = min(w0 + CopyBatch::CHUNK, cb.words[d]);
+    if ((cb.vec >> d) & 1u) {
+        const uint4 *s = (const uint4 *)cb.src[d];
+        uint4 *t = (uint4 *)cb.dst[d];
+        for (uint64_t i = w0 + threadIdx.x; i < w1; i += 256) t[i] = __ldcs(s + i);
+    } else {
+        const uint32_t *s = (const uint32_t *)cb.src[d];
+        uint32_t *t = (uint32_t *)cb.dst[d];
+        for (uint64_t i = w0 + threadIdx.x; i < w1; i += 256) t[i] = __ldcs(s + i);
+    }
+}
+
+nb_status nb_launch_copy_batch(nb_grid *g, const CopyBatch &cb, cudaStream_t s) {
+    if (!cb.n || !cb.bstart[cb.n]) return NB_OK;
+    LaunchScope ls(g, s, "k_halo_copy");
+    k_halo_copy<<<cb.bstart[cb.n], 256, 0, s>>>(cb);
+    return nb_launch_check("k_halo_copy");
+}
+
 nb_status nb_halo_run(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int c1d, cudaStream_t s) {
     nb_grid *g = f->g;
     int world = g->comm ? g->comm->world : 1, rank = g->comm ? g->comm->rank : 0;
@@ -297,17 +316,47 @@ nb_status nb_halo_run(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int
     auto plane_addr = [&](int p, int c, int zl) {
         return f->base[p] + ((int64_t)c * cs_of(p) + (int64_t)(zl + 1) * f->ps) * f->esz;
     };
+    if (nb_is_peer(g)) {
+        // peer memory: a "ready" round (the neighbours finished reading the
+        // halos about to be overwritten), my planes stored straight into the
+        // neighbours' (IPC-mapped) halos, a "done" round
+        NB_TRY(nb_peer_round(g, periodic, s));
+        CopyBatch cb;
+        for (auto &m : msgs) {
+            if (m.src_rank != rank) continue;  // the sender writes
+            int c0 = m.up ? c0u : c0d, c1 = m.up ? c1u : c1d;
+            for (int c = c0; c < c1; ++c) {
+                if (cb.n == CopyBatch::MAX) {
+                    NB_TRY(nb_launch_copy_batch(g, cb, s));
+                    cb = CopyBatch();
+                }
+                cb.add(plane_addr(m.dst_part, c, m.dst_plane), plane_addr(m.src_part, c, m.src_plane), pb);
+            }
+        }
+        if (cb.n) NB_TRY(nb_launch_copy_batch(g, cb, s));
+        return nb_peer_round(g, periodic, s);
+    }
     bool remote = false;
+    // every device-local plane of the exchange goes into ONE batched copy
+    // launch (a per-plane cudaMemcpyAsync costs ~4 us of host enqueue each,
+    // which serialised the halo stream behind the host on LBM's 5-population
+    // messages)
+    CopyBatch cb;
     for (auto &m : msgs) {
         int c0 = m.up ? c0u : c0d, c1 = m.up ? c1u : c1d;
         if (m.src_rank == rank && m.dst_rank == rank) {
-            for (int c = c0; c < c1; ++c)
-                NB_CUDA(cudaMemcpyAsync(plane_addr(m.dst_part, c, m.dst_plane), plane_addr(m.src_part, c, m.src_plane),
-                                        pb, cudaMemcpyDeviceToDevice, s));
+            for (int c = c0; c < c1; ++c) {
+                if (cb.n == CopyBatch::MAX) {
+                    NB_TRY(nb_launch_copy_batch(g, cb, s));
+                    cb = CopyBatch();
+                }
+                cb.add(plane_addr(m.dst_part, c, m.dst_plane), plane_addr(m.src_part, c, m.src_plane), pb);
+            }
         } else {
             remote = true;
         }
     }
+    if (cb.n) NB_TRY(nb_launch_copy_batch(g, cb, s));
     if (!remote) return NB_OK;
     NB_TRY(nb_nccl_group(g, true));
     for (auto &m : msgs) {
@@ -346,6 +395,7 @@ nb_status nb_grid_alloc_common(nb_grid *g) {
     NB_CUDA(cudaMemset(g->psum_send, 0, sizeof(double) * planes));
     NB_CUDA(cudaMemset(g->dots, 0, sizeof(double) * NB_DOT_SLOTS));
     NB_CUDA(cudaMemset(g->counter, 0, sizeof(unsigned int) * 16));
+    if (nb_is_peer(g)) NB_TRY(nb_peer_grid_setup(g));  // collective
     return NB_OK;
 }
 
@@ -450,6 +500,7 @@ extern "C" nb_status nb_grid_destroy(nb_grid *g) {
         nb_field_destroy(kv.second);
     }
     g->scratch.clear();
+    nb_peer_grid_teardown(g);  // collective (peer transport)
     for (auto &r : g->prof) {
         cudaEventDestroy(r.a);
         cudaEventDestroy(r.b);
@@ -603,9 +654,11 @@ extern "C" nb_status nb_field_create(nb_grid *g, nb_dtype dt, int32_t card, doub
         // per-partition arithmetic; it is per partition: store the local one
         // (all local partitions share the formula cs = ps*(nz_p+2)).
     }
+    f->mapped.assign(g->nparts, 0);
+    if (s == NB_OK && nb_is_peer(g)) s = nb_peer_field_map(f);  // collective
     if (s != NB_OK) {
-        for (auto p : f->base)
-            if (p) cudaFree(p);
+        for (size_t p = 0; p < f->base.size(); ++p)
+            if (f->base[p] && !f->mapped[p]) cudaFree(f->base[p]);
         delete f;
         return s;
     }
@@ -622,8 +675,9 @@ extern "C" nb_status nb_field_destroy(nb_field *f) {
     DeviceGuard dg(f->g->device);
     cudaStreamSynchronize(f->g->cs);
     cudaStreamSynchronize(f->g->hs);
-    for (auto p : f->base)
-        if (p) cudaFree(p);
+    if (nb_is_peer(f->g)) nb_peer_field_unmap(f);  // collective: closes the mappings, then a barrier
+    for (size_t p = 0; p < f->base.size(); ++p)
+        if (f->base[p] && !(p < f->mapped.size() && f->mapped[p])) cudaFree(f->base[p]);
     f->g->nfields--;
     delete f;
     return NB_OK;
@@ -888,43 +942,6 @@ __global__ void __launch_bounds__(32 * ZW) k_dot(const T *__restrict__ x, const 
 }
 
 // ---- finalize: plane sums (one CTA per plane) + last-block total ----------
-__device__ void apply_final(int mode, double total, void *state, double *dots, int slot) {
-    if (mode == FIN_STORE) {
-        dots[slot] = total;
-        return;
-    }
-    CgScal *s = (CgScal *)state;
-    if (mode == FIN_CG_INIT) {
-        s->rr = total;
-        s->rr0 = total;
-        s->status = (total == 0.0) ? 2 : 0;
-        s->alpha = 0.0;
-        s->alpha_prev = 0.0;
-        s->beta = 0.0;
-        s->pending = 0;
-        s->iters = 0;
-        return;
-    }
-    if (s->status != 0) return;
-    if (mode == FIN_CG_PQ) {
-        s->pq = total;
-        s->pending = 0;  // phase A applied the deferred x update
-        if (!(total > 0.0))
-            s->status = 3;
-        else
-            s->alpha = s->rr / total;
-    } else if (mode == FIN_CG_RR) {
-        s->beta = total / s->rr;
-        s->rr = total;
-        s->alpha_prev = s->alpha;
-        s->pending = 1;
-        s->iters += 1;
-        if (total == 0.0)
-            s->status = 2;
-        else if (s->rtol2 > 0.0 && total <= s->rtol2 * s->rr0)
-            s->status = 1;
-    }
-}
 
 // blocks: one per plane in [p0, p1) of each component range; planes are
 // indexed c*NZ + z.  If `final_planes` > 0 the last block to finish sums
@@ -963,7 +980,7 @@ __global__ void __launch_bounds__(RED_THREADS) k_finalize(const double *tp, int 
     }
     if (t == 0) {
         *counter = 0u;
-        apply_final(mode, sh[0], state, dots, slot);
+        nb_apply_final(mode, sh[0], state, dots, slot);
     }
 }
 
@@ -971,7 +988,7 @@ __global__ void __launch_bounds__(RED_THREADS) k_final_only(const double *psum, 
                                                             void *state, double *dots, int slot) {
     __shared__ double sh[RED_THREADS];
     double s = block_tree_sum(psum, planes, sh);
-    if (threadIdx.x == 0) apply_final(mode, s, state, dots, slot);
+    if (threadIdx.x == 0) nb_apply_final(mode, s, state, dots, slot);
 }
 
 // Reduce the tile partials of `card` components (planes c*NZ + z) into the
@@ -988,6 +1005,7 @@ nb_status nb_reduce_finalize(nb_grid *g, int card, int mode, void *state, int sl
                                                   planes, mode, state, g->dots, slot);
         return nb_launch_check("k_finalize");
     }
+    if (nb_is_peer(g)) return nb_peer_reduce_finalize(g, card, mode, state, slot);
     int z0 = g->parts[g->first_local].z0, z1 = g->parts[g->first_local + g->nlocal - 1].z1;
     {
         LaunchScope ls(g, s, "k_finalize");

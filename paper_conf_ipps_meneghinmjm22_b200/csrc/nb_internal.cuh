@@ -53,9 +53,50 @@ constexpr int RED_THREADS = 256;
 // LBM lattice size
 constexpr int Q19 = 19;
 
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int d) {
+        cudaGetDevice(&prev);
+        if (prev != d) cudaSetDevice(d);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+// largest world of the peer-memory transport (flag slots, kernel params)
+constexpr int NB_MAX_WORLD = 16;
+
 struct nb_comm {
     int world = 1, rank = 0, device = 0;
-    void *nccl = nullptr;  // ncclComm_t
+    void *nccl = nullptr;  // ncclComm_t (NCCL transport)
+    // peer-memory transport (nb_comm_create_peer): host allgather used only
+    // at setup (IPC handle exchange) and as the teardown barrier
+    bool peer = false;
+    nb_allgather_fn ag = nullptr;
+    void *ag_ctx = nullptr;
+};
+
+// Per-grid state of the peer-memory transport (nb_peer.cu).  Every rank's
+// flag words and reduction buffers are mapped into every other rank (CUDA
+// IPC over NVLink / NVSwitch); kernels store halos and plane sums straight
+// into the peer and raise a flag with a system-scope release store.
+//   flags[0]      raised by the lower neighbour (its up-going halo is in)
+//   flags[1]      raised by the upper neighbour (its down-going halo is in)
+//   flags[2 + r]  raised by rank r (its plane sums of the current reduction)
+//   ctr[0]        reductions done (parity selects the psum2 half)
+//   ctr[1], [2]   halo signals sent up / down;  ctr[3], [4] halo signals
+//                 awaited from below / above (device counters: CUDA-graph
+//                 replay safe)
+struct NbPeer {
+    uint64_t *flags = nullptr;
+    uint64_t *ctr = nullptr;
+    double *psum2 = nullptr;  // [2][planes]
+    int planes = 0;
+    std::vector<uint64_t *> rflags;  // [world] each rank's flags (self: local)
+    std::vector<double *> rpsum;     // [world] each rank's psum2 (self: local)
 };
 
 struct NbPart {
@@ -124,6 +165,7 @@ struct nb_grid {
     std::vector<NbSparsePart> sp;
     std::vector<int64_t> plane_count;  // [nz] active per global plane
     int64_t n_active = 0;
+    NbPeer *peer = nullptr;  // peer-memory transport (multi-process)
 };
 
 constexpr int NB_DOT_SLOTS = 1024;
@@ -138,7 +180,11 @@ struct nb_field {
     std::vector<char *> base;          // per partition (local only)
     std::vector<size_t> bytes;
     std::vector<int64_t> pcs;          // per-partition component stride (elements)
+    std::vector<char> mapped;          // per partition: base is a peer's buffer (CUDA IPC)
 };
+
+// partition p's buffer of f is addressable from this process (local or mapped)
+inline bool nb_reachable(const nb_field *f, int p) { return p >= 0 && f->base[p] != nullptr; }
 
 // per-partition geometry handed to kernels (dense)
 struct PGeo {
@@ -207,11 +253,77 @@ struct CgScal {
     int32_t iters, status, pending, pad;
 };
 
+// apply a reduction's total: store it, or advance the CG scalars (the
+// convergence gate of SURVEY.md §8(c) c5 lives here, on the device)
+__device__ __forceinline__ void nb_apply_final(int mode, double total, void *state, double *dots, int slot) {
+    if (mode == FIN_STORE) {
+        dots[slot] = total;
+        return;
+    }
+    CgScal *s = (CgScal *)state;
+    if (mode == FIN_CG_INIT) {
+        s->rr = total;
+        s->rr0 = total;
+        s->status = (total == 0.0) ? 2 : 0;
+        s->alpha = 0.0;
+        s->alpha_prev = 0.0;
+        s->beta = 0.0;
+        s->pending = 0;
+        s->iters = 0;
+        return;
+    }
+    if (s->status != 0) return;
+    if (mode == FIN_CG_PQ) {
+        s->pq = total;
+        s->pending = 0;  // phase A applied the deferred x update
+        if (!(total > 0.0))
+            s->status = 3;
+        else
+            s->alpha = s->rr / total;
+    } else if (mode == FIN_CG_RR) {
+        s->beta = total / s->rr;
+        s->rr = total;
+        s->alpha_prev = s->alpha;
+        s->pending = 1;
+        s->iters += 1;
+        if (total == 0.0)
+            s->status = 2;
+        else if (s->rtol2 > 0.0 && total <= s->rtol2 * s->rr0)
+            s->status = 1;
+    }
+}
+
 nb_status nb_grid_alloc_common(nb_grid *g);
 nb_status nb_grid_setup_parts(nb_grid *g, const int32_t *zb, int32_t nparts, const int32_t *device_ids,
                               nb_comm *comm);
 // cached internal field of the grid (slot distinguishes several of one kind)
 nb_status nb_grid_scratch(nb_grid *g, nb_dtype dt, int card, int slot, nb_field **out);
+
+// Batched plane copies (one launch for all device-local / peer-mapped halo
+// planes of an exchange): up to MAX (dst, src, bytes) descriptors passed by
+// value; blocks are dealt to descriptors by a prefix of block counts.
+// 16-byte vectors when every address and size allows it, else 4-byte words.
+struct CopyBatch {
+    static constexpr int MAX = 48;
+    static constexpr int CHUNK = 256 * 4;  // vectors per block
+    void *dst[MAX];
+    const void *src[MAX];
+    uint64_t words[MAX];     // number of 16-byte (vec) or 4-byte words
+    uint32_t bstart[MAX + 1];
+    uint32_t vec;            // bit i: descriptor i uses 16-byte words
+    int n = 0;
+    CopyBatch() : vec(0) { bstart[0] = 0; }
+    void add(void *d, const void *s_, size_t bytes) {
+        bool v = ((uintptr_t)d % 16 == 0) && ((uintptr_t)s_ % 16 == 0) && (bytes % 16 == 0);
+        dst[n] = d;
+        src[n] = s_;
+        words[n] = v ? bytes / 16 : bytes / 4;
+        if (v) vec |= 1u << n;
+        bstart[n + 1] = bstart[n] + (uint32_t)((words[n] + CHUNK - 1) / CHUNK);
+        ++n;
+    }
+};
+nb_status nb_launch_copy_batch(nb_grid *g, const CopyBatch &cb, cudaStream_t s);
 
 // halo helpers (nb_api.cu)
 nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down,
@@ -224,10 +336,27 @@ nb_status nb_nccl_send(nb_grid *g, const void *buf, size_t bytes, int peer, cuda
 nb_status nb_nccl_recv(nb_grid *g, void *buf, size_t bytes, int peer, cudaStream_t s);
 
 int nb_part_owner(const nb_grid *g, int part);
-// halos travel on the halo stream (multi-process, or NB_HALO_STREAM)
-inline bool nb_halo_on_stream(const nb_grid *g) {
-    return (g->comm && g->comm->world > 1) || g->halo_mode == NB_HALO_STREAM;
-}
+// multi-process with the peer-memory transport
+inline bool nb_is_peer(const nb_grid *g) { return g->comm && g->comm->world > 1 && g->comm->peer; }
+// multi-process with the NCCL transport
+inline bool nb_is_nccl(const nb_grid *g) { return g->comm && g->comm->world > 1 && !g->comm->peer; }
+// halos travel on the halo stream (NCCL transport, or NB_HALO_STREAM);
+// otherwise the boundary kernels store them straight into the neighbour
+// (same process, or a peer's buffer mapped through CUDA IPC)
+inline bool nb_halo_on_stream(const nb_grid *g) { return nb_is_nccl(g) || g->halo_mode == NB_HALO_STREAM; }
+
+// peer-memory transport (nb_peer.cu)
+nb_status nb_peer_grid_setup(nb_grid *g);
+void nb_peer_grid_teardown(nb_grid *g);
+nb_status nb_peer_field_map(struct nb_field *f);
+nb_status nb_peer_field_unmap(struct nb_field *f);
+// halo signal to / wait for the neighbouring ranks (periodic: ring too)
+nb_status nb_peer_signal(nb_grid *g, bool periodic, cudaStream_t s);
+nb_status nb_peer_wait(nb_grid *g, bool periodic, cudaStream_t s);
+// signal + wait in one launch
+nb_status nb_peer_round(nb_grid *g, bool periodic, cudaStream_t s);
+nb_status nb_peer_barrier(nb_comm *c);
+nb_status nb_peer_reduce_finalize(nb_grid *g, int card, int mode, void *state, int slot);
 
 // halo overlap events of a schedule (multi-process)
 struct HaloSync {

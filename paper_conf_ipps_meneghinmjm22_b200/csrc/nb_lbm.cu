@@ -224,11 +224,11 @@ static nb_status launch_lbm(nb_grid *g, int p, nb_field *fin, nb_field *fout, co
     A.rho_w = (float)prm->rho_w;
     if (remote_stores) {
         int lo = lbm_lo(g, p, per), hi = lbm_hi(g, p, per);
-        if (zb == 0 && lo >= 0 && g->parts[lo].local)
+        if (zb == 0 && nb_reachable(fout, lo))
             for (int i = 14; i < 19; ++i)
                 A.rem_lo[i] = (float *)fout->base[lo] + (int64_t)i * lcs(fout, lo) +
                               (int64_t)(g->parts[lo].nz() + 1) * fout->ps;
-        if (ze == g->parts[p].nz() && hi >= 0 && g->parts[hi].local)
+        if (ze == g->parts[p].nz() && nb_reachable(fout, hi))
             for (int i = 9; i < 14; ++i) A.rem_hi[i] = (float *)fout->base[hi] + (int64_t)i * lcs(fout, hi);
     }
     dim3 blk(128), grd((g->nx + 127) / 128, g->ny, ze - zb);
@@ -275,20 +275,26 @@ extern "C" nb_status nb_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm
             }
         }
         if (st != NB_OK) break;
-        if (dist) {  // halos on the halo stream, overlapped with the interior
-            cudaEventRecord(hs.eb, g->cs);
-            cudaStreamWaitEvent(g->hs, hs.eb, 0);
-            st = lbm_halo(fout, per, g->hs);
-            cudaEventRecord(hs.eh, g->hs);
-            if (occ == NB_OCC_NONE) cudaStreamWaitEvent(g->cs, hs.eh, 0);
-        }
+        // the halo stream starts after the boundary planes (event eb); the
+        // interior kernels are ENQUEUED before the halo transfer so the host
+        // never holds them back behind the transfer's API calls
+        if (dist) cudaEventRecord(hs.eb, g->cs);
+        // peer transport: the boundary kernels stored the halos into the
+        // neighbours' fout; tell them (their wait follows their interior)
+        if (st == NB_OK && nb_is_peer(g)) st = nb_peer_signal(g, per, g->cs);
         for (int p = g->first_local; p < g->first_local + g->nlocal && st == NB_OK; ++p) {
             int nz = g->parts[p].nz();
             bool blo = lbm_lo(g, p, per) >= 0, bhi = lbm_hi(g, p, per) >= 0;
             if (occ == NB_OCC_NONE || (!blo && !bhi)) continue;
             st = launch_lbm(g, p, fin, fout, prm, blo ? 1 : 0, bhi ? nz - 1 : nz, false);
         }
-        if (dist && occ != NB_OCC_NONE) cudaStreamWaitEvent(g->cs, hs.eh, 0);
+        if (dist && st == NB_OK) {  // halos on the halo stream, overlapped with the interior
+            cudaStreamWaitEvent(g->hs, hs.eb, 0);
+            st = lbm_halo(fout, per, g->hs);
+            cudaEventRecord(hs.eh, g->hs);
+            cudaStreamWaitEvent(g->cs, hs.eh, 0);
+        }
+        if (st == NB_OK && nb_is_peer(g)) st = nb_peer_wait(g, per, g->cs);
         std::swap(fin, fout);
     }
     if (hs.eb) {

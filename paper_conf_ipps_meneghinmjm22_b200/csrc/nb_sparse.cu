@@ -383,19 +383,30 @@ nb_status nb_sparse_halo_update(nb_field *f) {
         const NbPart &q = g->parts[m.src_part];
         return g->plane_count[m.up ? q.z1 - 1 : q.z0];
     };
+    // device-local segments, and with the peer transport every segment this
+    // rank sends (into the neighbour's IPC-mapped halo), in one batched launch
+    const bool peer = nb_is_peer(g);
+    if (peer) NB_TRY(nb_peer_round(g, false, g->cs));  // neighbours done reading these halos
     bool remote = false;
+    CopyBatch cb;
     for (auto &m : msgs) {
-        if (m.src_rank == rank && m.dst_rank == rank) {
-            for (int c = 0; c < f->card; ++c) {
+        const bool mine = m.src_rank == rank && (peer || m.dst_rank == rank);
+        if (mine) {
+            for (int c = 0; c < f->card && count(m) > 0; ++c) {
                 const char *src = f->base[m.src_part] + ((int64_t)c * f->pcs[m.src_part] + src_off(m)) * f->esz;
                 char *dst = f->base[m.dst_part] + ((int64_t)c * f->pcs[m.dst_part] + dst_off(m)) * f->esz;
-                if (count(m) > 0)
-                    NB_CUDA(cudaMemcpyAsync(dst, src, count(m) * f->esz, cudaMemcpyDeviceToDevice, g->cs));
+                if (cb.n == CopyBatch::MAX) {
+                    NB_TRY(nb_launch_copy_batch(g, cb, g->cs));
+                    cb = CopyBatch();
+                }
+                cb.add(dst, src, count(m) * f->esz);
             }
-        } else {
+        } else if (!(m.src_rank == rank && m.dst_rank == rank)) {
             remote = true;
         }
     }
+    if (cb.n) NB_TRY(nb_launch_copy_batch(g, cb, g->cs));
+    if (peer) return nb_peer_round(g, false, g->cs);
     if (!remote) return NB_OK;
     NB_TRY(nb_nccl_group(g, true));
     for (auto &m : msgs) {

@@ -443,8 +443,8 @@ static nb_status launch_map_u(nb_grid *g, int mode, int p, MsrArgs A, const nb_f
     PGeo geo = pgeo(ufield, p);
     double *rem_lo = nullptr, *rem_hi = nullptr;
     if (!nb_halo_on_stream(g)) {  // fused halo: store straight into the neighbour
-        if (zb == 0 && q.lo >= 0 && g->parts[q.lo].local) rem_lo = pl(ufield, q.lo, g->parts[q.lo].nz());
-        if (ze == q.nz() && q.hi >= 0 && g->parts[q.hi].local) rem_hi = pl(ufield, q.hi, -1);
+        if (zb == 0 && nb_reachable(ufield, q.lo)) rem_lo = pl(ufield, q.lo, g->parts[q.lo].nz());
+        if (ze == q.nz() && nb_reachable(ufield, q.hi)) rem_hi = pl(ufield, q.hi, -1);
     }
     dim3 blk(128), grd((g->nx + 127) / 128, g->ny, std::min(ze - zb, 64));
     LaunchScope ls(g, g->cs, "k_map_u");
@@ -481,22 +481,31 @@ static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int
 // work of the compute stream and joined by an event before the boundary
 // stencils
 
-static bool is_dist(const nb_grid *g) { return g->comm && g->comm->world > 1; }
 
-static nb_status dist_halo_begin(nb_grid *g, nb_field *u, HaloSync &hsync) {
-    if (!nb_halo_on_stream(g)) return NB_OK;
+// mark: the boundary maps are enqueued (event eb on the compute stream);
+// begin: the halo stream waits for eb and transfers.  Between the two the
+// internal stencils are enqueued, so the host never holds them back behind
+// the transfer's API calls.
+static nb_status dist_halo_mark(nb_grid *g, HaloSync &hsync) {
+    if (!nb_halo_on_stream(g)) return NB_OK;  // (peer transport: nothing to mark)
     if (!hsync.eb) {
         NB_CUDA(cudaEventCreateWithFlags(&hsync.eb, cudaEventDisableTiming));
         NB_CUDA(cudaEventCreateWithFlags(&hsync.eh, cudaEventDisableTiming));
     }
     NB_CUDA(cudaEventRecord(hsync.eb, g->cs));
+    return NB_OK;
+}
+static nb_status dist_halo_begin(nb_grid *g, nb_field *u, HaloSync &hsync) {
+    // peer transport: the boundary maps already stored the halo into the
+    // neighbours; tell them
+    if (!nb_halo_on_stream(g)) return nb_is_peer(g) ? nb_peer_signal(g, false, g->cs) : NB_OK;
     NB_CUDA(cudaStreamWaitEvent(g->hs, hsync.eb, 0));
     NB_TRY(nb_halo_exchange_planes(u, 0, 1, true, true, g->hs));
     NB_CUDA(cudaEventRecord(hsync.eh, g->hs));
     return NB_OK;
 }
 static nb_status dist_halo_wait(nb_grid *g, HaloSync &hsync) {
-    if (!nb_halo_on_stream(g)) return NB_OK;
+    if (!nb_halo_on_stream(g)) return nb_is_peer(g) ? nb_peer_wait(g, false, g->cs) : NB_OK;
     NB_CUDA(cudaStreamWaitEvent(g->cs, hsync.eh, 0));
     return NB_OK;
 }
@@ -533,8 +542,11 @@ static nb_status msr_step_fields(nb_grid *g, nb_occ occ, MsrFields F, double m, 
             for (int z : bnd_planes(g, p)) NB_TRY(launch_map_u(g, MODE, p, args(p), F.u, z, z + 1));
         }
     }
-    NB_TRY(dist_halo_begin(g, F.u, hs));
-    if (occ == NB_OCC_NONE) NB_TRY(dist_halo_wait(g, hs));
+    NB_TRY(dist_halo_mark(g, hs));
+    if (occ == NB_OCC_NONE) {
+        NB_TRY(dist_halo_begin(g, F.u, hs));
+        NB_TRY(dist_halo_wait(g, hs));
+    }
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         auto in = view_ranges(g, p, occ == NB_OCC_NONE ? NB_VIEW_STANDARD : NB_VIEW_INTERNAL);
         for (auto rg : in) {
@@ -545,6 +557,7 @@ static nb_status msr_step_fields(nb_grid *g, nb_occ occ, MsrFields F, double m, 
         }
     }
     if (occ == NB_OCC_NONE) return NB_OK;
+    NB_TRY(dist_halo_begin(g, F.u, hs));
     NB_TRY(dist_halo_wait(g, hs));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         for (int z : bnd_planes(g, p)) {
@@ -717,7 +730,7 @@ extern "C" nb_status nb_cg_create(nb_field *x, const nb_field *b, const nb_cg_pa
 }
 
 static bool cg_eager(const nb_grid *g) {
-    return g->profiling || is_dist(g) || getenv("NB_NO_GRAPH") != nullptr;
+    return g->profiling || nb_is_nccl(g) || getenv("NB_NO_GRAPH") != nullptr;
 }
 
 constexpr int CG_GRAPH_CHUNK = 16;

@@ -41,8 +41,12 @@ else:
 evs = [e for e in prof.events() if e.device_type == torch.autograd.DeviceType.CUDA]
 ks = sorted([(e.time_range.start, e.time_range.end, e.name) for e in evs])
 # halo copies vs kernels: fraction of copy time overlapped by a running kernel
-copies = [(s, e) for s, e, nm in ks if "Memcpy" in nm or "memcpy" in nm]
-kern = [(s, e) for s, e, nm in ks if not ("Memcpy" in nm or "memcpy" in nm)]
+def is_copy(nm):
+    return "Memcpy" in nm or "memcpy" in nm or "k_halo_copy" in nm
+
+
+copies = [(s, e) for s, e, nm in ks if is_copy(nm)]
+kern = [(s, e) for s, e, nm in ks if not is_copy(nm)]
 cov = 0.0
 for cs_, ce_ in copies:
     segs = sorted((max(cs_, s), min(ce_, e)) for s, e in kern if s < ce_ and e > cs_)
@@ -76,4 +80,5 @@ print(json.dumps(summary))
 for r in rows[:24]:
     print(f"{r['name']:50s} dur {r['dur_us']:9.1f} us  gap {r['gap_us']:7.1f} us")
 if "--out" in sys.argv:
-    json.dump({"summary": summary, "kernels": rows}, open(sys.argv[sys.argv.index("--out") + 1], "w"), indent=1)
+    with open(sys.argv[sys.argv.index("--out") + 1], "w") as fh:
+        json.dump({"summary": summary, "kernels": rows}, fh, indent=1)
