@@ -99,12 +99,26 @@ def setup_dist(args):
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     import torch
+    # one process per GPU; if there are fewer GPUs than local ranks (a
+    # single-GPU box exercising the multi-process path) ranks share GPUs and
+    # the timing plumbing uses gloo (NCCL refuses two ranks on one GPU)
+    ndev = max(torch.cuda.device_count(), 1)
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
+    global _SHARED_GPU
+    _SHARED_GPU = local_world > ndev
+    local = local % ndev
     torch.cuda.set_device(local)
     if world > 1:
         import torch.distributed as dist
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if _SHARED_GPU:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     return world, rank, local
+
+
+_SHARED_GPU = False
 
 
 def barrier(world):
@@ -118,7 +132,7 @@ def max_over_ranks(world, v):
         return v
     import torch
     import torch.distributed as dist
-    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    t = torch.tensor([v], dtype=torch.float64, device="cpu" if _SHARED_GPU else "cuda")
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
