@@ -208,6 +208,21 @@ nb_status nb_sync(nb_grid *grid);
 nb_status nb_field_create(nb_grid *grid, nb_dtype dtype, int32_t cardinality, double outside_value,
                           nb_field **out);
 nb_status nb_field_destroy(nb_field *field);
+/* Borrowed storage (SURVEY.md §8(b) "field (borrowed)": PyTorch owns the
+ * memory).  Pure host logic: the number of elements partition g of a field
+ * of `cardinality` components occupies in the layout above (dense:
+ * pitch*Ny*(nz_g+2)*card; sparse: (halo_lo+n_g+halo_hi, padded)*card). */
+nb_status nb_field_required_elems(const nb_grid *grid, int32_t cardinality, int32_t g, int64_t *n);
+/* A field over caller-owned device buffers: dev_ptrs[i] backs the i-th
+ * partition owned by this process (partitions in increasing order), each at
+ * least nb_field_required_elems elements of dtype, 16-byte aligned, on the
+ * grid's device.  The call writes outside_value into the halo planes /
+ * segments (stream-ordered) and leaves the own cells as they are; the
+ * library never frees the buffers — the caller keeps them alive until
+ * nb_field_destroy.  NB_EINVAL for NULL, misaligned or non-device pointers.
+ * With the peer transport the call is collective, like nb_field_create. */
+nb_status nb_field_wrap(nb_grid *grid, nb_dtype dtype, int32_t cardinality, double outside_value,
+                        void *const *dev_ptrs, nb_field **out);
 /* host: dense logical view, nbytes = Nx*Ny*Nz*card*sizeof(dtype); inactive
  * cells of sparse grids are ignored on upload and read back as outside.
  * Upload is stream-ordered (host buffer must stay valid until nb_sync);
@@ -237,6 +252,9 @@ nb_status nb_laplace7(const nb_field *x, nb_field *y, nb_view view);
  * fixed order that does not depend on the partition count (DESIGN.md
  * "Deterministic reductions").  Synchronises; *host_out receives the value. */
 nb_status nb_dot(const nb_field *x, const nb_field *y, double *host_out);
+/* The same value written to device memory dev_out (one double, on the grid's
+ * device), stream-ordered on the compute stream; does not synchronise. */
+nb_status nb_dot_dev(const nb_field *x, const nb_field *y, double *dev_out);
 
 /* Config C1 (Fig. 4a): for k < iters: x <- x + a*y;
  * y <- L(x); dots[k] = <x, y>.  Halo on x (L280).  dots_out: host [iters].

@@ -88,6 +88,8 @@ SIGNATURES = {
     "nb_grid_set_halo_mode": ([P, I32], I32),
     "nb_field_create": ([P, I32, I32, D, PP], I32),
     "nb_field_destroy": ([P], I32),
+    "nb_field_required_elems": ([P, I32, I32, P], I32),
+    "nb_field_wrap": ([P, I32, I32, D, P, PP], I32),
     "nb_field_upload": ([P, P, I64], I32),
     "nb_field_download": ([P, P, I64], I32),
     "nb_field_fill": ([P, I32, U64, D, D], I32),
@@ -97,6 +99,7 @@ SIGNATURES = {
     "nb_axpby": ([D, P, D, P, I32], I32),
     "nb_laplace7": ([P, P, I32], I32),
     "nb_dot": ([P, P, P], I32),
+    "nb_dot_dev": ([P, P, P], I32),
     "nb_map_stencil_reduce": ([P, P, D, I32, I32, P], I32),
     "nb_cg_create": ([P, P, P, PP], I32),
     "nb_cg_iterate": ([P, I32], I32),
@@ -279,7 +282,9 @@ class Grid:
         if comm is None:
             devs = [0] * self.nparts if devices is None else list(devices)
             dv = (C.c_int32 * self.nparts)(*devs)
+            self.device = int(devs[0])
         else:
+            self.device = int(comm.device)
             k = self.nparts // comm.world
             dv = (C.c_int32 * max(k, 1))(*([comm.device] * max(k, 1)))
         self.handle = P()
@@ -349,14 +354,41 @@ class Field:
     """Field of `card` components (PAPER.md L58-L63 newField<T>(cardinality,
     outsideDomainValue)); SoA layout with z halo planes."""
 
-    def __init__(self, grid: Grid, dtype="f64", card: int = 1, outside: float = 0.0):
+    def __init__(self, grid: Grid, dtype="f64", card: int = 1, outside: float = 0.0, _buffers=None):
         self.grid = grid
         self.dt = _dtype_code(dtype)
         self.np_dtype = _DT[self.dt]
         self.card = int(card)
         self.outside = float(outside)
         self.handle = P()
-        _check(lib().nb_field_create(grid.handle, self.dt, self.card, self.outside, C.byref(self.handle)))
+        self.buffers = _buffers  # borrowed storage (kept alive with the field)
+        if _buffers is None:
+            _check(lib().nb_field_create(grid.handle, self.dt, self.card, self.outside, C.byref(self.handle)))
+        else:
+            ptrs = (C.c_void_p * len(_buffers))(*[b.data_ptr() for b in _buffers])
+            _check(lib().nb_field_wrap(grid.handle, self.dt, self.card, self.outside, ptrs, C.byref(self.handle)))
+
+    @staticmethod
+    def required_elems(grid: Grid, card: int, part: int) -> int:
+        n = C.c_int64()
+        _check(lib().nb_field_required_elems(grid.handle, int(card), int(part), C.byref(n)))
+        return n.value
+
+    @classmethod
+    def wrap(cls, grid: Grid, buffers, dtype="f64", card: int = 1, outside: float = 0.0):
+        """Field over caller-owned torch CUDA tensors, one per local partition
+        (each >= required_elems elements; torch keeps ownership)."""
+        return cls(grid, dtype, card, outside, _buffers=list(buffers))
+
+    @classmethod
+    def empty_torch(cls, grid: Grid, dtype="f64", card: int = 1, outside: float = 0.0):
+        """Allocate the partitions with torch.empty on the grid's device and wrap them."""
+        import torch
+        tdt = torch.float64 if _dtype_code(dtype) == 1 else torch.float32
+        dev = torch.device("cuda", grid.device)
+        bufs = [torch.empty(cls.required_elems(grid, card, p), dtype=tdt, device=dev)
+                for p in range(grid.nparts) if grid.partition_info(p)["local"]]
+        return cls.wrap(grid, bufs, dtype, card, outside)
 
     @property
     def shape(self):
@@ -438,6 +470,12 @@ def nb_dot(x: Field, y: Field) -> float:
     out = C.c_double()
     _check(lib().nb_dot(_h(x), _h(y), C.byref(out)))
     return out.value
+
+
+def nb_dot_dev(x: Field, y: Field, out_ptr: int) -> None:
+    """<x, y> written to the device double at out_ptr (e.g. a torch tensor's
+    data_ptr()), stream-ordered; no synchronisation."""
+    _check(lib().nb_dot_dev(_h(x), _h(y), P(out_ptr)))
 
 
 def nb_map_stencil_reduce(x: Field, y: Field, a: float = 0.125, iters: int = 10, occ: int = OCC_TWO_WAY):

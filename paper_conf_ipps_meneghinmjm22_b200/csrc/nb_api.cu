@@ -667,6 +667,95 @@ extern "C" nb_status nb_field_create(nb_grid *g, nb_dtype dt, int32_t card, doub
     return NB_OK;
 }
 
+// ---- borrowed storage (SURVEY.md §8(b) "field (borrowed)") ---------------
+static int64_t dense_pitch(const nb_grid *g) { return ((int64_t)g->nx + 31) / 32 * 32; }
+
+static nb_status required_elems(const nb_grid *g, int card, int p, int64_t *n) {
+    if (p < 0 || p >= g->nparts) NB_FAIL(NB_EINVAL, "partition %d out of range", p);
+    if (g->sparse)
+        *n = g->sp[p].cs * card;
+    else
+        *n = dense_pitch(g) * g->ny * (g->parts[p].nz() + 2) * card;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_field_required_elems(const nb_grid *g, int32_t card, int32_t p, int64_t *n) {
+    if (!g || !n || card < 1 || card > 64) NB_FAIL(NB_EINVAL, "nb_field_required_elems: bad arguments");
+    return required_elems(g, card, p, n);
+}
+
+extern "C" nb_status nb_field_wrap(nb_grid *g, nb_dtype dt, int32_t card, double outside, void *const *dev_ptrs,
+                                   nb_field **out) {
+    if (!g || !out || !dev_ptrs) NB_FAIL(NB_EINVAL, "nb_field_wrap: NULL argument");
+    *out = nullptr;
+    if (dt != NB_F32 && dt != NB_F64) NB_FAIL(NB_EINVAL, "nb_field_wrap: bad dtype %d", (int)dt);
+    if (card < 1 || card > 64) NB_FAIL(NB_EINVAL, "nb_field_wrap: cardinality %d", card);
+    for (int i = 0; i < g->nlocal; ++i) {
+        const void *ptr = dev_ptrs[i];
+        if (!ptr || (uintptr_t)ptr % 16) NB_FAIL(NB_EINVAL, "nb_field_wrap: dev_ptrs[%d] is NULL or not 16-byte aligned", i);
+        cudaPointerAttributes at;
+        if (cudaPointerGetAttributes(&at, ptr) != cudaSuccess || at.type != cudaMemoryTypeDevice ||
+            at.device != g->device) {
+            cudaGetLastError();
+            NB_FAIL(NB_EINVAL, "nb_field_wrap: dev_ptrs[%d] is not device memory of device %d", i, g->device);
+        }
+    }
+    DeviceGuard dg(g->device);
+    nb_field *f = new nb_field();
+    f->g = g;
+    f->dt = dt;
+    f->card = card;
+    f->outside = outside;
+    f->esz = dt == NB_F64 ? 8 : 4;
+    f->borrowed = true;
+    f->base.assign(g->nparts, nullptr);
+    f->bytes.assign(g->nparts, 0);
+    f->pcs.assign(g->nparts, 0);
+    f->mapped.assign(g->nparts, 0);
+    if (!g->sparse) {
+        f->pitch = dense_pitch(g);
+        f->ps = f->pitch * g->ny;
+    }
+    nb_status s = NB_OK;
+    for (int i = 0; i < g->nlocal && s == NB_OK; ++i) {
+        const int p = g->first_local + i;
+        int64_t n = 0;
+        required_elems(g, card, p, &n);
+        f->base[p] = (char *)dev_ptrs[i];
+        f->bytes[p] = (size_t)n * f->esz;
+        // the halo planes / segments start as outside (what nb_field_create
+        // gives); own cells keep the caller's data
+        if (g->sparse) {
+            const NbSparsePart &sp = g->sp[p];
+            f->pcs[p] = sp.cs;
+            for (int c = 0; c < card && s == NB_OK; ++c) {
+                char *b = f->base[p] + (size_t)c * sp.cs * f->esz;
+                s = fill_const_raw(g, b, sp.hl, dt, outside, g->cs);
+                if (s == NB_OK) s = fill_const_raw(g, b + (size_t)(sp.hl + sp.n) * f->esz, sp.cs - sp.hl - sp.n, dt,
+                                                   outside, g->cs);
+            }
+        } else {
+            const int64_t cs = f->ps * (g->parts[p].nz() + 2);
+            f->pcs[p] = cs;
+            for (int c = 0; c < card && s == NB_OK; ++c) {
+                char *b = f->base[p] + (size_t)c * cs * f->esz;
+                s = fill_const_raw(g, b, f->ps, dt, outside, g->cs);
+                if (s == NB_OK)
+                    s = fill_const_raw(g, b + (size_t)(cs - f->ps) * f->esz, f->ps, dt, outside, g->cs);
+            }
+        }
+    }
+    f->cs = f->pcs[g->first_local];
+    if (s == NB_OK && nb_is_peer(g)) s = nb_peer_field_map(f);  // collective
+    if (s != NB_OK) {
+        delete f;
+        return s;
+    }
+    g->nfields++;
+    *out = f;
+    return NB_OK;
+}
+
 // component stride of partition p (dense): ps * (nz_p + 2)
 static inline int64_t dense_cs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
 
@@ -676,8 +765,9 @@ extern "C" nb_status nb_field_destroy(nb_field *f) {
     cudaStreamSynchronize(f->g->cs);
     cudaStreamSynchronize(f->g->hs);
     if (nb_is_peer(f->g)) nb_peer_field_unmap(f);  // collective: closes the mappings, then a barrier
-    for (size_t p = 0; p < f->base.size(); ++p)
-        if (f->base[p] && !(p < f->mapped.size() && f->mapped[p])) cudaFree(f->base[p]);
+    if (!f->borrowed)
+        for (size_t p = 0; p < f->base.size(); ++p)
+            if (f->base[p] && !(p < f->mapped.size() && f->mapped[p])) cudaFree(f->base[p]);
     f->g->nfields--;
     delete f;
     return NB_OK;
@@ -1051,6 +1141,18 @@ extern "C" nb_status nb_dot(const nb_field *x, const nb_field *y, double *host_o
     NB_TRY(nb_reduce_finalize(g, x->card, FIN_STORE, nullptr, 0));
     NB_CUDA(cudaMemcpyAsync(host_out, g->dots, sizeof(double), cudaMemcpyDeviceToHost, g->cs));
     NB_CUDA(cudaStreamSynchronize(g->cs));
+    return NB_OK;
+}
+
+extern "C" nb_status nb_dot_dev(const nb_field *x, const nb_field *y, double *dev_out) {
+    NB_TRY(check_pair(x, y));
+    if (!dev_out) NB_FAIL(NB_EINVAL, "nb_dot_dev: dev_out is NULL");
+    nb_grid *g = x->g;
+    if (x->card > g->max_card) NB_FAIL(NB_EUNSUPPORTED, "nb_dot_dev: cardinality > %d", g->max_card);
+    DeviceGuard dg(g->device);
+    NB_TRY(nb_dot_partials(x, y));
+    NB_TRY(nb_reduce_finalize(g, x->card, FIN_STORE, nullptr, 0));
+    NB_CUDA(cudaMemcpyAsync(dev_out, g->dots, sizeof(double), cudaMemcpyDeviceToDevice, g->cs));
     return NB_OK;
 }
 

@@ -181,6 +181,8 @@ struct nb_field {
     std::vector<size_t> bytes;
     std::vector<int64_t> pcs;          // per-partition component stride (elements)
     std::vector<char> mapped;          // per partition: base is a peer's buffer (CUDA IPC)
+    bool borrowed = false;             // nb_field_wrap: caller-owned buffers (never freed)
+    std::vector<uint64_t> map_off;     // per mapped partition: offset inside the peer's allocation
 };
 
 // partition p's buffer of f is addressable from this process (local or mapped)

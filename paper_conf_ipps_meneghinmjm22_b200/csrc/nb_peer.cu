@@ -29,6 +29,8 @@
 #include "nb_device.cuh"
 #include "nb_internal.cuh"
 
+#include <cuda.h>
+
 #include <cstring>
 
 nb_status nb_launch_check(const char *what);
@@ -149,19 +151,51 @@ static std::vector<int> remote_neighbour_parts(const nb_grid *g) {
     return v;
 }
 
+// start of the cudaMalloc allocation holding p (borrowed buffers of
+// nb_field_wrap may sit inside a larger, e.g. PyTorch caching-allocator, block)
+typedef CUresult (*GetAddressRangeFn)(CUdeviceptr *, size_t *, CUdeviceptr);
+static nb_status alloc_base(const void *p, const char **base) {
+    static GetAddressRangeFn fn = nullptr;
+    if (!fn) {
+        void *q = nullptr;
+        cudaDriverEntryPointQueryResult r;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &q, cudaEnableDefault, &r) != cudaSuccess ||
+            r != cudaDriverEntryPointSuccess || !q)
+            NB_FAIL(NB_ECUDA, "cuMemGetAddressRange unavailable");
+        fn = (GetAddressRangeFn)q;
+    }
+    CUdeviceptr b = 0;
+    size_t sz = 0;
+    if (fn(&b, &sz, (CUdeviceptr)p) != CUDA_SUCCESS) NB_FAIL(NB_ECUDA, "cuMemGetAddressRange failed");
+    *base = (const char *)b;
+    return NB_OK;
+}
+
+struct IpcRec {
+    cudaIpcMemHandle_t h;
+    uint64_t offset;  // of the partition buffer inside the exported allocation
+};
+
 nb_status nb_peer_field_map(nb_field *f) {
     nb_grid *g = f->g;
     nb_comm *c = g->comm;
     const int k = g->nlocal;
     f->mapped.assign(g->nparts, 0);
-    std::vector<cudaIpcMemHandle_t> mine(k), all((size_t)k * c->world);
-    for (int i = 0; i < k; ++i) NB_CUDA(cudaIpcGetMemHandle(&mine[i], f->base[g->first_local + i]));
-    NB_TRY(peer_allgather(c, mine.data(), (int64_t)sizeof(cudaIpcMemHandle_t) * k, all.data()));
+    std::vector<IpcRec> mine(k), all((size_t)k * c->world);
+    for (int i = 0; i < k; ++i) {
+        const char *p = f->base[g->first_local + i], *b = p;
+        if (f->borrowed) NB_TRY(alloc_base(p, &b));
+        NB_CUDA(cudaIpcGetMemHandle(&mine[i].h, (void *)b));
+        mine[i].offset = (uint64_t)(p - b);
+    }
+    NB_TRY(peer_allgather(c, mine.data(), (int64_t)sizeof(IpcRec) * k, all.data()));
     for (int p : remote_neighbour_parts(g)) {
         void *ptr = nullptr;
-        NB_CUDA(cudaIpcOpenMemHandle(&ptr, all[p], cudaIpcMemLazyEnablePeerAccess));  // p = owner*k + index
-        f->base[p] = (char *)ptr;
+        NB_CUDA(cudaIpcOpenMemHandle(&ptr, all[p].h, cudaIpcMemLazyEnablePeerAccess));  // p = owner*k + index
+        f->base[p] = (char *)ptr + all[p].offset;
         f->mapped[p] = 1;
+        f->map_off.resize(g->nparts, 0);
+        f->map_off[p] = all[p].offset;
         if (g->sparse) f->pcs[p] = g->sp[p].cs;
     }
     return NB_OK;
@@ -170,7 +204,7 @@ nb_status nb_peer_field_map(nb_field *f) {
 nb_status nb_peer_field_unmap(nb_field *f) {
     for (size_t p = 0; p < f->mapped.size(); ++p) {
         if (!f->mapped[p]) continue;
-        cudaIpcCloseMemHandle(f->base[p]);
+        cudaIpcCloseMemHandle(f->base[p] - (p < f->map_off.size() ? f->map_off[p] : 0));
         f->base[p] = nullptr;
         f->mapped[p] = 0;
     }

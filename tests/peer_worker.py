@@ -175,6 +175,21 @@ def fem_cg(g):
 
 compare("fem cg", (12, 11, 14), 2, fem_cg)
 
+# ---- borrowed (torch-owned) storage: IPC handle of the enclosing allocation + offset
+def wrapped_cg(g):
+    pad = torch.empty(7, dtype=torch.float64, device=f"cuda:{DEV}")  # noqa: F841 (offsets the next blocks)
+    b, x = nb.Field.empty_torch(g), nb.Field.empty_torch(g)
+    b.fill(nb.FILL_POISSON_RHS)
+    x.fill_const(0.0)
+    r = nb.nb_cg_solve(x, b, max_iter=15, rtol=0.0, occ=nb.OCC_TWO_WAY)
+    out = [x.download()]
+    b.close(), x.close()
+    return out, [r.rr, r.iters]
+
+
+compare("wrapped cg", (20, 20, 20), 2, wrapped_cg)
+
+
 # ---- the peer path really ran: its kernels were launched ---------------------
 g = nb.Grid((32, 32, 32), nparts=2, comm=COMM)
 b, x = nb.Field(g), nb.Field(g)
