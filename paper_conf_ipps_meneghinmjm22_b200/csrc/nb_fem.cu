@@ -16,13 +16,33 @@
 // gather element by element (a, then b, then j).  The classification depends
 // only on the global node position, so results are partition independent.
 #include <cmath>
+#include <cstdlib>
+#include <algorithm>
 #include <cstring>
+#include <vector>
 
 #include "nb_device.cuh"
 #include "nb_internal.cuh"
+#include "nb_tma.cuh"
 
 __constant__ double c_ke[24 * 24];      // element stiffness, row-major
 __constant__ double c_S[27 * 9];        // interior stencil blocks [o][i][j]
+__constant__ const double *c_cls;       // surface-class stencils [FEM_NCLS][27 * 9] (device memory)
+
+// Surface nodes: y_n = sum over the EXISTING elements around n of K_e u_e
+// (an element exists iff its 8 nodes are in the box).  Along one axis, a
+// node at coordinate t of N nodes belongs to the elements starting at t - d,
+// d in {0, 1}, with 0 <= t - d <= N - 2: the set is {0} at t = 0, {1} at
+// t = N - 1, {0, 1} inside and {} when N = 1 — 4 axis states.  Per (x, y, z)
+// state and "drop the z = 0 Dirichlet columns" (nodes at gz = 1), the
+// assembled 27-block stencil of the existing elements is precomputed once
+// (host, fp64), so a surface node costs one 27-point pass instead of the
+// 8 x 8 element-pair gather.
+constexpr int FEM_NCLS = 4 * 4 * 4 * 2;
+__device__ __forceinline__ int fem_axis_state(int t, int n) {
+    if (n == 1) return 3;
+    return t == 0 ? 0 : (t == n - 1 ? 1 : 2);
+}
 
 std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v);
 nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down, cudaStream_t s);
@@ -95,6 +115,26 @@ static nb_status fem_upload_constants(double E, double nu) {
             for (int j = 0; j < 3; ++j)
                 if (i != j && (oc[i] == 0 || oc[j] == 0)) S[o * 9 + i * 3 + j] = 0.0;
     }
+    std::vector<double> cls((size_t)FEM_NCLS * 243, 0.0);
+    for (int k = 0; k < FEM_NCLS; ++k) {
+        const int drop = k & 1, st[3] = {k >> 5, (k >> 3) & 3, (k >> 1) & 3};  // x, y, z axis states
+        auto has = [&](int axis, int d) { return st[axis] == 2 || (st[axis] == 0 && d == 0) || (st[axis] == 1 && d == 1); };
+        double *C = cls.data() + (size_t)k * 243;
+        for (int a = 0; a < 8; ++a) {  // node n is corner a of the element starting at n - off(a)
+            if (!has(0, a & 1) || !has(1, (a >> 1) & 1) || !has(2, (a >> 2) & 1)) continue;
+            for (int b = 0; b < 8; ++b) {
+                const int ox = (b & 1) - (a & 1), oy = ((b >> 1) & 1) - ((a >> 1) & 1), oz = ((b >> 2) & 1) - ((a >> 2) & 1);
+                if (drop && oz == -1) continue;  // Dirichlet column (z = 0)
+                const int o = (oz + 1) * 9 + (oy + 1) * 3 + (ox + 1);
+                for (int i = 0; i < 3; ++i)
+                    for (int j = 0; j < 3; ++j) C[o * 9 + i * 3 + j] += ke[(3 * a + i) * 24 + 3 * b + j];
+            }
+        }
+    }
+    static double *d_cls = nullptr;
+    if (!d_cls) NB_CUDA(cudaMalloc(&d_cls, sizeof(double) * cls.size()));
+    NB_CUDA(cudaMemcpy(d_cls, cls.data(), sizeof(double) * cls.size(), cudaMemcpyHostToDevice));
+    NB_CUDA(cudaMemcpyToSymbol(c_cls, &d_cls, sizeof(d_cls)));
     NB_CUDA(cudaMemcpyToSymbol(c_ke, ke, sizeof(ke)));
     NB_CUDA(cudaMemcpyToSymbol(c_S, S, sizeof(S)));
     g_fem_E = E;
@@ -136,25 +176,28 @@ __device__ __forceinline__ void fem_node(const double *__restrict__ u, int64_t c
             acc2 = fma(S[8], u2, acc2);
         }
     } else {
-        for (int a = 0; a < 8; ++a) {
-            const int ex = x - (a & 1), ey = y - ((a >> 1) & 1), ez = gz - ((a >> 2) & 1);
-            if (ex < 0 || ey < 0 || ez < 0 || ex > g.nx - 2 || ey > g.ny - 2 || ez > g.NZ - 2) continue;
-            for (int b = 0; b < 8; ++b) {
-                const int mx = ex + (b & 1), my = ey + ((b >> 1) & 1), mz = ez + ((b >> 2) & 1);
-                if (mz == 0) continue;  // Dirichlet column
-                const int64_t m = (int64_t)(mz - g.z0 + 1) * g.ps + (int64_t)my * g.pitch + mx;
-                const double u0 = u[m], u1 = u[cs + m], u2 = u[2 * cs + m];
-                const double *K = c_ke + (3 * a) * 24 + 3 * b;
-                acc0 = fma(K[0], u0, acc0);
-                acc0 = fma(K[1], u1, acc0);
-                acc0 = fma(K[2], u2, acc0);
-                acc1 = fma(K[24], u0, acc1);
-                acc1 = fma(K[25], u1, acc1);
-                acc1 = fma(K[26], u2, acc1);
-                acc2 = fma(K[48], u0, acc2);
-                acc2 = fma(K[49], u1, acc2);
-                acc2 = fma(K[50], u2, acc2);
-            }
+        // surface class stencil (positions outside the box have no element
+        // and are skipped; their coefficients are zero)
+        const int cls = ((fem_axis_state(x, g.nx) * 4 + fem_axis_state(y, g.ny)) * 4 + fem_axis_state(gz, g.NZ)) * 2 +
+                        (gz == 1 ? 1 : 0);
+        const double *__restrict__ C = c_cls + (size_t)cls * 243;
+#pragma unroll
+        for (int o = 0; o < 27; ++o) {
+            const int ox = o % 3 - 1, oy = (o / 3) % 3 - 1, oz = o / 9 - 1;
+            const int mx = x + ox, my = y + oy, mz = gz + oz;
+            if (mx < 0 || my < 0 || mz < 0 || mx >= g.nx || my >= g.ny || mz >= g.NZ) continue;
+            const int64_t m = c0 + (int64_t)oz * g.ps + (int64_t)oy * g.pitch + ox;
+            const double u0 = u[m], u1 = u[cs + m], u2 = u[2 * cs + m];
+            const double *K = C + o * 9;
+            acc0 = fma(__ldg(K + 0), u0, acc0);
+            acc0 = fma(__ldg(K + 1), u1, acc0);
+            acc0 = fma(__ldg(K + 2), u2, acc0);
+            acc1 = fma(__ldg(K + 3), u0, acc1);
+            acc1 = fma(__ldg(K + 4), u1, acc1);
+            acc1 = fma(__ldg(K + 5), u2, acc1);
+            acc2 = fma(__ldg(K + 6), u0, acc2);
+            acc2 = fma(__ldg(K + 7), u1, acc2);
+            acc2 = fma(__ldg(K + 8), u2, acc2);
         }
     }
     out[0] = acc0;
@@ -218,6 +261,529 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_fem(FemArgs A, PGeo g, int z
     }
 }
 
+// ---------------------------------------------------------------------------
+// z-marching interior operator (the hot kernel of C5).  A thread owns one
+// (x, y) column of a 32x8 tile for ZC planes.  Each u plane is loaded ONCE
+// (9 positions x 3 components) and feeds three outputs: plane k-1 (offset
+// oz = +1, which completes it), plane k (oz = 0) and plane k+1 (oz = -1,
+// which starts it).  Every output therefore receives exactly the FMA chain
+// of fem_node's interior path — o = (oz, oy, ox) lexicographic, then j, the
+// same structural zeros skipped — so the result is bit-identical to
+// fem_node while loading 27 values per node instead of 81 (the L1 / LSU
+// pipe, not the FP64 pipe, bounded the one-node-per-thread kernel).
+// Nodes outside the interior (column on an x/y face, gz < 2 or gz > NZ-2)
+// take fem_node.
+// ---------------------------------------------------------------------------
+template <int O>
+__device__ __forceinline__ void fem_blk(const double (&v)[3], double (&acc)[3]) {
+    constexpr int ox = O % 3 - 1, oy = (O / 3) % 3 - 1, oz = O / 9 - 1;
+    const double *S = c_S + O * 9;
+    acc[0] = fma(S[0], v[0], acc[0]);
+    if (ox != 0 && oy != 0) acc[0] = fma(S[1], v[1], acc[0]);
+    if (ox != 0 && oz != 0) acc[0] = fma(S[2], v[2], acc[0]);
+    if (oy != 0 && ox != 0) acc[1] = fma(S[3], v[0], acc[1]);
+    acc[1] = fma(S[4], v[1], acc[1]);
+    if (oy != 0 && oz != 0) acc[1] = fma(S[5], v[2], acc[1]);
+    if (oz != 0 && ox != 0) acc[2] = fma(S[6], v[0], acc[2]);
+    if (oz != 0 && oy != 0) acc[2] = fma(S[7], v[1], acc[2]);
+    acc[2] = fma(S[8], v[2], acc[2]);
+}
+
+// all 9 in-plane positions of one oz block, in (oy, ox) order
+template <int OZ>
+__device__ __forceinline__ void fem_plane_blocks(const double (&v)[9][3], double (&acc)[3]) {
+    fem_blk<(OZ + 1) * 9 + 0>(v[0], acc);
+    fem_blk<(OZ + 1) * 9 + 1>(v[1], acc);
+    fem_blk<(OZ + 1) * 9 + 2>(v[2], acc);
+    fem_blk<(OZ + 1) * 9 + 3>(v[3], acc);
+    fem_blk<(OZ + 1) * 9 + 4>(v[4], acc);
+    fem_blk<(OZ + 1) * 9 + 5>(v[5], acc);
+    fem_blk<(OZ + 1) * 9 + 6>(v[6], acc);
+    fem_blk<(OZ + 1) * 9 + 7>(v[7], acc);
+    fem_blk<(OZ + 1) * 9 + 8>(v[8], acc);
+}
+
+// load plane k (element offset `base` = centre of the column in that plane)
+// and apply it: aA (output k-1) += oz=+1, aB (output k) += oz=0, aC (output
+// k+1) = oz=-1 from zero.  cen receives the centre values.
+template <bool DA, bool DB>
+__device__ __forceinline__ void fem_plane(const double *__restrict__ u, int64_t cs, int64_t base, int64_t pitch,
+                                          double (&aA)[3], double (&aB)[3], double (&aC)[3], double (&cen)[3]) {
+    double v[9][3];
+#pragma unroll
+    for (int q = 0; q < 9; ++q) {
+        const int64_t m = base + (int64_t)(q / 3 - 1) * pitch + (q % 3 - 1);
+        v[q][0] = __ldg(u + m);
+        v[q][1] = __ldg(u + cs + m);
+        v[q][2] = __ldg(u + 2 * cs + m);
+    }
+#pragma unroll
+    for (int c = 0; c < 3; ++c) cen[c] = v[4][c];
+    if (DA) fem_plane_blocks<1>(v, aA);
+    if (DB) fem_plane_blocks<0>(v, aB);
+    aC[0] = aC[1] = aC[2] = 0.0;
+    fem_plane_blocks<-1>(v, aC);
+}
+
+template <int K, int ZC>
+__global__ void __launch_bounds__(DOT_TX *DOT_TY, 2) k_fem_z(FemArgs A, PGeo g, int zb0, int ze0, double *tp, int T) {
+    __shared__ double sw[ZC][3][DOT_TY];
+    if (K == FEM_CG_Q && A.sc->status != 0) return;
+    const int x = blockIdx.x * DOT_TX + threadIdx.x, y = blockIdx.y * DOT_TY + threadIdx.y;
+    const int zs = zb0 + blockIdx.z * ZC, zend = min(zs + ZC, ze0);
+    const bool valid = x < g.nx && y < g.ny;
+    const bool colint = x >= 1 && x <= g.nx - 2 && y >= 1 && y <= g.ny - 2;
+    // fast planes: interior in z as well (gz in [2, NZ-2])
+    int fa = max(zs, 2 - g.z0), fb = min(zend, g.NZ - 1 - g.z0);
+    if (!colint || fb < fa) fb = fa;
+    const double *__restrict__ u = A.u;
+    const int64_t cs = A.cs, col = (int64_t)y * g.pitch + x;
+    double aA[3], aB[3], aC[3], cprev[3], ccur[3];
+    if (fa < fb) {  // preload planes fa-1 (starts output fa) and fa
+        fem_plane<false, false>(u, cs, (int64_t)fa * g.ps + col, g.pitch, aA, aB, aC, cprev);
+#pragma unroll
+        for (int c = 0; c < 3; ++c) aB[c] = aC[c];
+        fem_plane<false, true>(u, cs, (int64_t)(fa + 1) * g.ps + col, g.pitch, aA, aB, aC, ccur);
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+            aA[c] = aB[c];
+            aB[c] = aC[c];
+        }
+    }
+    for (int zl = zs; zl < zend; ++zl) {
+        double o[3] = {0.0, 0.0, 0.0}, uc[3] = {0.0, 0.0, 0.0};
+        const int64_t c0 = (int64_t)(zl + 1) * g.ps + col;
+        if (zl >= fa && zl < fb) {
+            // plane zl+1 completes output zl (held in aA)
+            double cnext[3];
+            fem_plane<true, true>(u, cs, (int64_t)(zl + 2) * g.ps + col, g.pitch, aA, aB, aC, cnext);
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                o[c] = aA[c];
+                uc[c] = ccur[c];
+                aA[c] = aB[c];
+                aB[c] = aC[c];
+                ccur[c] = cnext[c];
+            }
+        } else if (valid) {
+            fem_node(u, cs, g, x, y, zl, o);
+            if (K == FEM_CG_Q) {
+                uc[0] = u[c0];
+                uc[1] = u[cs + c0];
+                uc[2] = u[2 * cs + c0];
+            }
+        }
+        double prod[3] = {0.0, 0.0, 0.0};
+        if (valid) {
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                const int64_t i = c * cs + c0;
+                if (K == FEM_CG_INIT) {
+                    const double r = __dsub_rn(A.b[i], o[c]);
+                    A.y[i] = r;
+                    prod[c] = __dmul_rn(r, r);
+                } else {
+                    A.y[i] = o[c];
+                    if (K == FEM_CG_Q) prod[c] = __dmul_rn(uc[c], o[c]);
+                }
+            }
+        }
+        if (K != FEM_APPLY) {
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                const double v = warp_sum_canon(prod[c]);
+                if (threadIdx.x == 0) sw[zl - zs][c][threadIdx.y] = v;
+            }
+        }
+    }
+    (void)cprev;
+    if (K == FEM_APPLY) return;
+    __syncthreads();
+    const int t = threadIdx.y * DOT_TX + threadIdx.x;
+    if (t < 3 * (zend - zs)) {
+        const int zi = t / 3, c = t % 3;
+        double s = sw[zi][c][0];
+#pragma unroll
+        for (int w = 1; w < DOT_TY; ++w) s = __dadd_rn(s, sw[zi][c][w]);
+        tp[((int64_t)c * g.NZ + g.z0 + zs + zi) * T + blockIdx.y * gridDim.x + blockIdx.x] = s;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// TMA-staged z-march (default): the CTA streams its tile's planes (36 x 10
+// box per component, tile + ring, fetched by one elected thread with
+// cp.async.bulk.tensor into a 4-stage shared-memory ring completed through
+// mbarrier transaction bytes) — the per-thread global-load latency that
+// stalled k_fem_z disappears; threads read the 27 values of a plane from
+// shared memory position by position (3 registers live), so the kernel is
+// small enough for 3 CTAs per SM.  Same FMA chains as fem_node (bitwise).
+// ---------------------------------------------------------------------------
+constexpr int FBX = DOT_TX + 4, FBY = DOT_TY + 2;  // box starts at x0 - 2 (16-byte aligned)
+constexpr int FTPAD = 2944;                         // 36*10*8 = 2880 rounded up to 128
+constexpr int FNST = 4;
+#ifndef NB_FEM_NR
+#define NB_FEM_NR 2  // rows per thread of the TMA kernel
+#endif
+
+struct __align__(128) FemStage {
+    double c[3][FTPAD / 8];
+};
+
+// ---- surface nodes, converged: one thread per node ----------------------
+// Surface nodes (an x / y face column, or gz < 2, or gz = NZ-1) are ~2 % of
+// the nodes but put one divergent lane into ~17 % of the streaming kernel's
+// warps; they are computed first by this kernel (fem_node, raw operator
+// output into A.y) and the streaming kernel only reads them back.
+struct FemSurf {
+    int ncol_edge;  // edge columns of the (x, y) plane
+    int nin;        // interior columns (x in [1, nx-2], y in [1, ny-2])
+    int nzs;        // z-surface planes of the launch range
+    int zlist[3];   // their local plane indices
+};
+
+__device__ __forceinline__ void fem_edge_col(int e, int nx, int ny, int &x, int &y) {
+    if (e < nx) {
+        x = e;
+        y = 0;
+        return;
+    }
+    e -= nx;
+    if (ny > 1) {
+        if (e < nx) {
+            x = e;
+            y = ny - 1;
+            return;
+        }
+        e -= nx;
+    }
+    if (nx > 1) {
+        y = 1 + e / 2;
+        x = (e & 1) ? nx - 1 : 0;
+    } else {
+        y = 1 + e;
+        x = 0;
+    }
+}
+
+template <int K>
+__global__ void __launch_bounds__(128) k_fem_surface(FemArgs A, PGeo g, int zb, int ze, FemSurf S) {
+    if (K == FEM_CG_Q && A.sc->status != 0) return;
+    const int nzl = ze - zb;
+    const int64_t n1 = (int64_t)S.ncol_edge * nzl, n2 = (int64_t)S.nin * S.nzs;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n1 + n2; i += (int64_t)gridDim.x * blockDim.x) {
+        int x, y, zl;
+        if (i < n1) {
+            fem_edge_col((int)(i / nzl), g.nx, g.ny, x, y);
+            zl = zb + (int)(i % nzl);
+        } else {
+            const int64_t k = i - n1;
+            const int c = (int)(k % S.nin);
+            zl = S.zlist[k / S.nin];
+            x = 1 + c % (g.nx - 2);
+            y = 1 + c / (g.nx - 2);
+        }
+        double o[3];
+        fem_node(A.u, A.cs, g, x, y, zl, o);
+        const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+        A.y[c0] = o[0];
+        A.y[A.cs + c0] = o[1];
+        A.y[2 * A.cs + c0] = o[2];
+    }
+}
+
+// ---- face columns (x or y on the box surface), z-marching -----------------
+// One thread per face column and chunk of FZC planes: every u plane is read
+// once (its in-box positions of the 3 x 3 neighbourhood) and feeds the three
+// outputs it touches, each with its own surface-class stencil; per output
+// the in-box positions arrive in o order with all 9 coefficients — the FMA
+// chain of fem_node's surface path (bitwise), at ~1/3 of its loads.
+constexpr int FZC = 4;
+
+__device__ __forceinline__ const double *fem_cls_ptr(int x, int y, int gz, const PGeo &g) {
+    const int cls = ((fem_axis_state(x, g.nx) * 4 + fem_axis_state(y, g.ny)) * 4 + fem_axis_state(gz, g.NZ)) * 2 +
+                    (gz == 1 ? 1 : 0);
+    return c_cls + (size_t)cls * 243;
+}
+
+// contributions of one plane k (global gz_k) to output accumulators whose
+// class stencils are CA (output k-1, offset oz = +1), CB (k, 0), CC (k+1, -1)
+__device__ __forceinline__ void fem_face_plane(const double *__restrict__ u, int64_t cs, const PGeo &g, int x, int y,
+                                               int k, const double *CA, const double *CB, const double *CC,
+                                               double (&aA)[3], double (&aB)[3], double (&aC)[3], double (&cen)[3]) {
+    const int64_t base = (int64_t)(k + 1) * g.ps + (int64_t)y * g.pitch + x;
+    aC[0] = aC[1] = aC[2] = 0.0;
+#pragma unroll
+    for (int q = 0; q < 9; ++q) {
+        const int oy = q / 3 - 1, ox = q % 3 - 1;
+        const int mx = x + ox, my = y + oy;
+        if (mx < 0 || my < 0 || mx >= g.nx || my >= g.ny) continue;
+        const int64_t m = base + (int64_t)oy * g.pitch + ox;
+        const double v0 = u[m], v1 = u[cs + m], v2 = u[2 * cs + m];
+        if (q == 4) {
+            cen[0] = v0;
+            cen[1] = v1;
+            cen[2] = v2;
+        }
+        const double *K;
+#define FEM_FACE_APPLY(CP, OZ, ACC)                                       \
+    if (CP) {                                                             \
+        K = CP + ((OZ + 1) * 9 + q) * 9;                                  \
+        ACC[0] = fma(__ldg(K + 0), v0, ACC[0]);                           \
+        ACC[0] = fma(__ldg(K + 1), v1, ACC[0]);                           \
+        ACC[0] = fma(__ldg(K + 2), v2, ACC[0]);                           \
+        ACC[1] = fma(__ldg(K + 3), v0, ACC[1]);                           \
+        ACC[1] = fma(__ldg(K + 4), v1, ACC[1]);                           \
+        ACC[1] = fma(__ldg(K + 5), v2, ACC[1]);                           \
+        ACC[2] = fma(__ldg(K + 6), v0, ACC[2]);                           \
+        ACC[2] = fma(__ldg(K + 7), v1, ACC[2]);                           \
+        ACC[2] = fma(__ldg(K + 8), v2, ACC[2]);                           \
+    }
+        FEM_FACE_APPLY(CA, 1, aA)
+        FEM_FACE_APPLY(CB, 0, aB)
+        FEM_FACE_APPLY(CC, -1, aC)
+#undef FEM_FACE_APPLY
+    }
+}
+
+__device__ __forceinline__ void fem_face_col(int c, const PGeo &g, int &x, int &y) {
+    const int nyf = g.nx > 2 ? (g.nx - 2) * (g.ny > 1 ? 2 : 1) : 0;  // y-face columns (x interior)
+    if (c < nyf) {
+        x = 1 + c % (g.nx - 2);
+        y = (c / (g.nx - 2)) ? g.ny - 1 : 0;
+    } else {
+        c -= nyf;
+        y = c % g.ny;
+        x = (c / g.ny) ? g.nx - 1 : 0;
+    }
+}
+
+template <int K>
+__global__ void __launch_bounds__(64) k_fem_faces(FemArgs A, PGeo g, int zb, int ze, int ncols) {
+    if (K == FEM_CG_Q && A.sc->status != 0) return;
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= ncols) return;
+    int x, y;
+    fem_face_col(c, g, x, y);
+    const int zs = zb + blockIdx.y * FZC, zend = min(zs + FZC, ze);
+    const double *__restrict__ u = A.u;
+    double aA[3] = {0.0, 0.0, 0.0}, aB[3] = {0.0, 0.0, 0.0}, aC[3], cen[3], cprev[3] = {0.0, 0.0, 0.0};
+    // planes zs-1 .. zend (in-box only: the halo planes beyond the global box are skipped)
+    for (int k = zs - 1; k <= zend; ++k) {
+        const int gk = g.z0 + k;
+        const int oA = k - 1, oB = k, oC = k + 1;  // outputs touched (local planes)
+        const bool inA = oA >= zs && oA < zend, inB = oB >= zs && oB < zend, inC = oC >= zs && oC < zend;
+        if (gk < 0 || gk >= g.NZ) {  // outside the box: no contribution, just rotate
+            aC[0] = aC[1] = aC[2] = 0.0;
+            cen[0] = cen[1] = cen[2] = 0.0;
+        } else {
+            const double *CA = inA && g.z0 + oA > 0 ? fem_cls_ptr(x, y, g.z0 + oA, g) : nullptr;
+            const double *CB = inB && g.z0 + oB > 0 ? fem_cls_ptr(x, y, g.z0 + oB, g) : nullptr;
+            const double *CC = inC && g.z0 + oC > 0 ? fem_cls_ptr(x, y, g.z0 + oC, g) : nullptr;
+            fem_face_plane(u, A.cs, g, x, y, k, CA, CB, CC, aA, aB, aC, cen);
+        }
+        if (inA) {  // output k-1 complete
+            const int64_t c0 = (int64_t)(oA + 1) * g.ps + (int64_t)y * g.pitch + x;
+            const bool ident = g.z0 + oA == 0;  // Dirichlet identity row
+#pragma unroll
+            for (int cc = 0; cc < 3; ++cc) A.y[cc * A.cs + c0] = ident ? cprev[cc] : aA[cc];
+        }
+#pragma unroll
+        for (int cc = 0; cc < 3; ++cc) {
+            aA[cc] = aB[cc];
+            aB[cc] = aC[cc];
+            cprev[cc] = cen[cc];
+        }
+    }
+}
+
+// ---- streaming interior kernel ---------------------------------------------
+// Thread = NR adjacent rows of one x column.  Coefficient-major order: for
+// each in-plane position q and each oz block, every coefficient (held in a
+// uniform register) is applied to the NR rows back to back, so a constant
+// load serves NR nodes.  Per output, positions still arrive in (oy, ox)
+// order with the oz blocks in plane order: fem_node's interior FMA chain
+// (bitwise).
+template <int O, int NR>
+__device__ __forceinline__ void fem_blkN(const double (&v)[NR][3], double (&acc)[NR][3]) {
+    constexpr int ox = O % 3 - 1, oy = (O / 3) % 3 - 1, oz = O / 9 - 1;
+    const double *S = c_S + O * 9;
+#pragma unroll
+    for (int r = 0; r < NR; ++r) acc[r][0] = fma(S[0], v[r][0], acc[r][0]);
+    if (ox != 0 && oy != 0)
+#pragma unroll
+        for (int r = 0; r < NR; ++r) acc[r][0] = fma(S[1], v[r][1], acc[r][0]);
+    if (ox != 0 && oz != 0)
+#pragma unroll
+        for (int r = 0; r < NR; ++r) acc[r][0] = fma(S[2], v[r][2], acc[r][0]);
+    if (oy != 0 && ox != 0)
+#pragma unroll
+        for (int r = 0; r < NR; ++r) acc[r][1] = fma(S[3], v[r][0], acc[r][1]);
+#pragma unroll
+    for (int r = 0; r < NR; ++r) acc[r][1] = fma(S[4], v[r][1], acc[r][1]);
+    if (oy != 0 && oz != 0)
+#pragma unroll
+        for (int r = 0; r < NR; ++r) acc[r][1] = fma(S[5], v[r][2], acc[r][1]);
+    if (oz != 0 && ox != 0)
+#pragma unroll
+        for (int r = 0; r < NR; ++r) acc[r][2] = fma(S[6], v[r][0], acc[r][2]);
+    if (oz != 0 && oy != 0)
+#pragma unroll
+        for (int r = 0; r < NR; ++r) acc[r][2] = fma(S[7], v[r][1], acc[r][2]);
+#pragma unroll
+    for (int r = 0; r < NR; ++r) acc[r][2] = fma(S[8], v[r][2], acc[r][2]);
+}
+
+template <int NR>
+struct FemAcc {
+    double a[NR][3], b[NR][3], c[NR][3];  // outputs k-1 (oz=+1), k (oz=0), k+1 (oz=-1)
+};
+
+template <int NR, int Q>
+__device__ __forceinline__ void fem_q(const FemStage &st, int sidx, bool da, bool db, FemAcc<NR> &A,
+                                      double (&cen)[NR][3]) {
+    constexpr int off = (Q / 3 - 1) * FBX + (Q % 3 - 1);
+    double v[NR][3];
+#pragma unroll
+    for (int r = 0; r < NR; ++r)
+#pragma unroll
+        for (int c = 0; c < 3; ++c) v[r][c] = st.c[c][sidx + r * FBX + off];
+    if (Q == 4)
+#pragma unroll
+        for (int r = 0; r < NR; ++r)
+#pragma unroll
+            for (int c = 0; c < 3; ++c) cen[r][c] = v[r][c];
+    if (da) fem_blkN<18 + Q, NR>(v, A.a);
+    if (db) fem_blkN<9 + Q, NR>(v, A.b);
+    fem_blkN<Q, NR>(v, A.c);
+}
+
+template <int K, int ZC, int NR>
+__global__ void __launch_bounds__(DOT_TX *(DOT_TY / NR), 8 / NR + 1)
+    k_fem_tma(const __grid_constant__ CUtensorMap m0, const __grid_constant__ CUtensorMap m1,
+              const __grid_constant__ CUtensorMap m2, FemArgs A, PGeo g, int zb0, int ze0, double *tp, int T) {
+    constexpr int NT = DOT_TX * (DOT_TY / NR);
+    __shared__ FemStage st[FNST];
+    __shared__ __align__(8) uint64_t bar[FNST];
+    __shared__ double sw[ZC][3][DOT_TY];
+    if (K == FEM_CG_Q && A.sc->status != 0) return;
+    const int tid = threadIdx.y * DOT_TX + threadIdx.x;
+    const int x0 = blockIdx.x * DOT_TX, y0 = blockIdx.y * DOT_TY;
+    const int x = x0 + threadIdx.x, ya = y0 + threadIdx.y * NR;  // rows ya .. ya+NR-1
+    const int zs = zb0 + blockIdx.z * ZC, zend = min(zs + ZC, ze0);
+    const int nplanes = zend - zs + 2;  // planes zs-1 .. zend
+    const bool xin = x < g.nx, xint = x >= 1 && x <= g.nx - 2;
+    const int fa = max(zs, 2 - g.z0), fb = min(zend, g.NZ - 1 - g.z0);  // fast outputs [fa, fb)
+    bool anyfast = false;
+#pragma unroll
+    for (int r = 0; r < NR; ++r) anyfast |= xint && ya + r >= 1 && ya + r <= g.ny - 2;
+    const int sidx = (threadIdx.y * NR + 1) * FBX + threadIdx.x + 2;
+    auto issue = [&](int j) {  // plane zs-1+j -> stage j % FNST
+        FemStage &S = st[j % FNST];
+        uint64_t *b = &bar[j % FNST];
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_expect_tx(b, 3 * FBX * FBY * 8);
+        const int tz = zs + j;  // tensor z of plane zl = zl + 1
+        tma_load_3d(&S.c[0][0], &m0, b, x0 - 2, y0 - 1, tz);
+        tma_load_3d(&S.c[1][0], &m1, b, x0 - 2, y0 - 1, tz);
+        tma_load_3d(&S.c[2][0], &m2, b, x0 - 2, y0 - 1, tz);
+    };
+    if (tid == 0) {
+        for (int k = 0; k < FNST; ++k) mbar_init(&bar[k], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (tid == 0)
+        for (int j = 0; j < min(FNST, nplanes); ++j) issue(j);
+    FemAcc<NR> acc;
+    double csave[NR][3];
+#pragma unroll
+    for (int r = 0; r < NR; ++r)
+#pragma unroll
+        for (int c = 0; c < 3; ++c) acc.a[r][c] = acc.b[r][c] = csave[r][c] = 0.0;
+#pragma unroll 3
+    for (int j = 0; j < nplanes; ++j) {
+        mbar_wait(&bar[j % FNST], (uint32_t)((j / FNST) & 1));
+        const FemStage &S = st[j % FNST];
+        const bool da = j >= 2, db = j >= 1;  // CTA-uniform
+        double cen[NR][3];
+        if (anyfast) {
+#pragma unroll
+            for (int r = 0; r < NR; ++r) acc.c[r][0] = acc.c[r][1] = acc.c[r][2] = 0.0;
+            fem_q<NR, 0>(S, sidx, da, db, acc, cen);
+            fem_q<NR, 1>(S, sidx, da, db, acc, cen);
+            fem_q<NR, 2>(S, sidx, da, db, acc, cen);
+            fem_q<NR, 3>(S, sidx, da, db, acc, cen);
+            fem_q<NR, 4>(S, sidx, da, db, acc, cen);
+            fem_q<NR, 5>(S, sidx, da, db, acc, cen);
+            fem_q<NR, 6>(S, sidx, da, db, acc, cen);
+            fem_q<NR, 7>(S, sidx, da, db, acc, cen);
+            fem_q<NR, 8>(S, sidx, da, db, acc, cen);
+        }
+        if (da) {  // output plane zl = zs + j - 2 is complete
+            const int zl = zs + j - 2;
+            const bool zfast = zl >= fa && zl < fb;
+#pragma unroll
+            for (int r = 0; r < NR; ++r) {
+                const int y = ya + r;
+                const bool valid = xin && y < g.ny;
+                const bool fast = zfast && xint && y >= 1 && y <= g.ny - 2;
+                const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+                double o[3] = {acc.a[r][0], acc.a[r][1], acc.a[r][2]};
+                double uc[3] = {csave[r][0], csave[r][1], csave[r][2]};
+                if (valid && !fast) {  // computed by k_fem_surface
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) {
+                        o[c] = A.y[c * A.cs + c0];
+                        if (K == FEM_CG_Q) uc[c] = A.u[c * A.cs + c0];
+                    }
+                }
+                double prod[3] = {0.0, 0.0, 0.0};
+                if (valid) {
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) {
+                        const int64_t i = c * A.cs + c0;
+                        if (K == FEM_CG_INIT) {
+                            const double rr = __dsub_rn(A.b[i], o[c]);
+                            A.y[i] = rr;
+                            prod[c] = __dmul_rn(rr, rr);
+                        } else {
+                            if (fast) A.y[i] = o[c];
+                            if (K == FEM_CG_Q) prod[c] = __dmul_rn(uc[c], o[c]);
+                        }
+                    }
+                }
+                if (K != FEM_APPLY) {
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) {
+                        const double v = warp_sum_canon(prod[c]);
+                        if (threadIdx.x == 0) sw[zl - zs][c][threadIdx.y * NR + r] = v;
+                    }
+                }
+            }
+        }
+        if (anyfast) {
+#pragma unroll
+            for (int r = 0; r < NR; ++r)
+#pragma unroll
+                for (int c = 0; c < 3; ++c) {
+                    acc.a[r][c] = acc.b[r][c];
+                    acc.b[r][c] = acc.c[r][c];
+                    csave[r][c] = cen[r][c];
+                }
+        }
+        __syncthreads();  // stage j % FNST is free
+        if (tid == 0 && j + FNST < nplanes) issue(j + FNST);
+    }
+    if (K == FEM_APPLY) return;
+    for (int t = tid; t < 3 * (zend - zs); t += NT) {
+        const int zi = t / 3, c = t % 3;
+        double s = sw[zi][c][0];
+#pragma unroll
+        for (int w = 1; w < DOT_TY; ++w) s = __dadd_rn(s, sw[zi][c][w]);
+        tp[((int64_t)c * g.NZ + g.z0 + zs + zi) * T + blockIdx.y * gridDim.x + blockIdx.x] = s;
+    }
+}
+
 // CG map: x += alpha_prev p_old (pending), p = r + beta p_old (in place)
 __global__ void k_fem_map(double *x, double *p, const double *r, int64_t n, const CgScal *sc) {
     if (sc->status != 0) return;
@@ -268,9 +834,43 @@ template <int K>
 static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int zb, int ze, const char *name) {
     if (ze <= zb) return NB_OK;
     A.cs = fcs(f, p);
-    dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, ze - zb);
     LaunchScope ls(g, g->cs, name);
-    k_fem<K><<<grd, blk, 0, g->cs>>>(A, pgeo(f, p), zb, g->tp, g->T);
+    const PGeo geo = pgeo(f, p);
+    const char *variant = getenv("NB_FEM_KERNEL");  // "plain" | "zmarch" | default TMA
+    if (variant && !strcmp(variant, "plain")) {  // the one-node-per-thread reference kernel
+        dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, ze - zb);
+        k_fem<K><<<grd, blk, 0, g->cs>>>(A, geo, zb, g->tp, g->T);
+    } else if (!variant && nb_tma_enabled()) {
+        constexpr int ZC = 32, NR = NB_FEM_NR;
+        CUtensorMap m[3];
+        for (int c = 0; c < 3; ++c) NB_TRY(tmap_for(A.u + c * A.cs, geo, 0, &m[c]));
+        // surface nodes first (converged), then the streaming interior
+        FemSurf S{};
+        const int nx = geo.nx, ny = geo.ny;
+        S.ncol_edge = nx * std::min(ny, 2) + std::max(ny - 2, 0) * std::min(nx, 2);
+        S.nin = std::max(nx - 2, 0) * std::max(ny - 2, 0);
+        for (int zl = zb; zl < ze; ++zl) {
+            const int gz = geo.z0 + zl;
+            if (gz < 2 || gz > geo.NZ - 2) S.zlist[S.nzs++] = zl;
+        }
+        {
+            const int ncols = S.ncol_edge;
+            S.ncol_edge = 0;  // face columns: z-marching kernel; z-surface planes: per node
+            const int64_t n = (int64_t)S.nin * S.nzs;
+            if (n > 0) {
+                const int blocks = (int)std::min<int64_t>((n + 127) / 128, 1 << 30);
+                k_fem_surface<K><<<blocks, 128, 0, g->cs>>>(A, geo, zb, ze, S);
+            }
+            dim3 fg((ncols + 63) / 64, (ze - zb + FZC - 1) / FZC);
+            k_fem_faces<K><<<fg, 64, 0, g->cs>>>(A, geo, zb, ze, ncols);
+        }
+        dim3 blk(DOT_TX, DOT_TY / NR), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
+        k_fem_tma<K, ZC, NR><<<grd, blk, 0, g->cs>>>(m[0], m[1], m[2], A, geo, zb, ze, g->tp, g->T);
+    } else {
+        constexpr int ZC = 16;
+        dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
+        k_fem_z<K, ZC><<<grd, blk, 0, g->cs>>>(A, geo, zb, ze, g->tp, g->T);
+    }
     return nb_launch_check(name);
 }
 
