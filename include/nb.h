@@ -319,6 +319,53 @@ nb_status nb_fem27_apply(const nb_field *u, nb_field *y, double E, double nu);
 /* b = consistent nodal load of pressure p on the top (z = Nz-1) face */
 nb_status nb_fem27_rhs(nb_field *b, double pressure);
 
+/* ---- Skeleton (§V) ------------------
+ * Sequential user code — a list of Containers — is turned into a data
+ * dependency graph (L279-L290: nodes = Containers with operation type,
+ * data view and coherency flag; edges = RaW / WaR / WaW on shared data),
+ * then a multi-GPU graph (L292-L331: halo-update nodes before incoherent
+ * stencils; OCC = NONE / STANDARD (split stencil) / EXTENDED (also the maps
+ * before it) / TWO_WAY (also the maps and reduces after it, with the
+ * internal -> boundary reduce dependency); transitively redundant edges
+ * removed; scheduling hints "launch the internal nodes before the halo"),
+ * then a schedule (L333-L396: BFS levels, a stream per concurrent node of
+ * the widest level with parent-stream reuse, an event per cross-stream
+ * dependency, task order by BFS over data edges + hints).
+ * Containers: y = a x + b y (MapOp), y = L(x) (StencilOp, 7-point), and
+ * <x, y> -> result slot (ReduceOp, the deterministic dot). */
+typedef enum { NB_SK_AXPBY = 0, NB_SK_LAPLACE7 = 1, NB_SK_DOT = 2 } nb_container_op;
+typedef struct {
+    int32_t op;    /* nb_container_op                                         */
+    int32_t x, y;  /* field ids (any non-negative integers naming the data)    */
+    int32_t slot;  /* NB_SK_DOT: result slot in [0, 1024)                      */
+    double a, b;   /* NB_SK_AXPBY coefficients                                 */
+} nb_container;
+/* Pure host logic (no GPU): plan n containers for an nparts-slab grid and
+ * write the plan as JSON into json (cap bytes; json = NULL: only *len) —
+ * {"nodes": [{id, name, op, view, container, incoherent, finalize, level,
+ * stream, event, waits}], "data": [[from, to]...], "hints": [...],
+ * "order": [...], "streams": S, "events": E}. */
+nb_status nb_skeleton_plan(int32_t nparts, nb_occ occ, const nb_container *containers, int32_t n, char *json,
+                           int64_t cap, int64_t *len);
+typedef struct nb_skeleton nb_skeleton;
+/* A skeleton over a dense grid; the fields it is given must outlive it, and
+ * the grid cannot be destroyed while it lives (NB_ESTATE). */
+nb_status nb_skeleton_create(nb_grid *grid, nb_occ occ, nb_skeleton **out);
+nb_status nb_skeleton_axpby(nb_skeleton *sk, double a, nb_field *x, double b, nb_field *y);
+nb_status nb_skeleton_laplace7(nb_skeleton *sk, nb_field *x, nb_field *y);
+nb_status nb_skeleton_dot(nb_skeleton *sk, nb_field *x, nb_field *y, int32_t slot);
+/* builds the plan, streams and events (implicit in the first run) */
+nb_status nb_skeleton_compile(nb_skeleton *sk);
+/* enqueue every task in plan order on its stream (asynchronous; ordered
+ * after earlier work on the grid's compute stream, and later work on that
+ * stream is ordered after it) */
+nb_status nb_skeleton_run(nb_skeleton *sk);
+/* a ReduceOp result (synchronises) */
+nb_status nb_skeleton_result(nb_skeleton *sk, int32_t slot, double *host);
+/* the plan as JSON, as nb_skeleton_plan */
+nb_status nb_skeleton_describe(nb_skeleton *sk, char *json, int64_t cap, int64_t *len);
+nb_status nb_skeleton_destroy(nb_skeleton *sk);
+
 /* ---- measurement ------------------------------------------------------ */
 /* When enabled, every kernel launch is bracketed by CUDA events on the
  * launching stream (graph launch is bypassed).  nb_profile_read

@@ -62,6 +62,14 @@ class LbmParams(C.Structure):
     _fields_ = [("omega", C.c_double), ("u_lid", C.c_double), ("rho_w", C.c_double), ("bc", C.c_int32)]
 
 
+class Container(C.Structure):
+    _fields_ = [("op", C.c_int32), ("x", C.c_int32), ("y", C.c_int32), ("slot", C.c_int32),
+                ("a", C.c_double), ("b", C.c_double)]
+
+
+SK_AXPBY, SK_LAPLACE7, SK_DOT = 0, 1, 2
+
+
 # exported symbols and their ctypes signatures (the whole of include/nb.h)
 P, I32, I64, D, U64 = C.c_void_p, C.c_int32, C.c_int64, C.c_double, C.c_uint64
 PP = C.POINTER(C.c_void_p)
@@ -112,6 +120,16 @@ SIGNATURES = {
     "nb_lbm_macroscopic": ([P, P, P], I32),
     "nb_fem27_apply": ([P, P, D, D], I32),
     "nb_fem27_rhs": ([P, D], I32),
+    "nb_skeleton_plan": ([I32, I32, P, I32, P, I64, P], I32),
+    "nb_skeleton_create": ([P, I32, PP], I32),
+    "nb_skeleton_axpby": ([P, D, P, D, P], I32),
+    "nb_skeleton_laplace7": ([P, P, P], I32),
+    "nb_skeleton_dot": ([P, P, P, I32], I32),
+    "nb_skeleton_compile": ([P], I32),
+    "nb_skeleton_run": ([P], I32),
+    "nb_skeleton_result": ([P, I32, P], I32),
+    "nb_skeleton_describe": ([P, P, I64, P], I32),
+    "nb_skeleton_destroy": ([P], I32),
     "nb_profile_enable": ([P, I32], I32),
     "nb_profile_read": ([P, C.c_char_p, P, P], I32),
     "nb_launch_count": ([P, P], I32),
@@ -549,3 +567,75 @@ def nb_fem27_apply(u: Field, y: Field, E: float = 1.0, nu: float = 0.3):
 
 def nb_fem27_rhs(b: Field, pressure: float = 1.0):
     _check(lib().nb_fem27_rhs(_h(b), pressure))
+
+
+# ---- Skeleton (§V): sequential containers -> graph -> schedule ----
+def _json_out(call):
+    import json
+    n = C.c_int64()
+    _check(call(None, 0, C.byref(n)))
+    buf = C.create_string_buffer(n.value + 1)
+    _check(call(buf, n.value + 1, C.byref(n)))
+    return json.loads(buf.value.decode())
+
+
+def nb_skeleton_plan(nparts: int, occ: int, containers) -> dict:
+    """Pure host planning (no GPU).  containers: (op, x, y, a, b, slot)
+    tuples with integer field ids; returns the plan (nodes, data edges,
+    hints, task order, streams, events)."""
+    arr = (Container * max(len(containers), 1))()
+    for i, (op, x, y, a, b, slot) in enumerate(containers):
+        arr[i] = Container(op, x, y, slot, a, b)
+    return _json_out(lambda buf, cap, n: lib().nb_skeleton_plan(int(nparts), int(occ), arr, len(containers),
+                                                                 buf, cap, n))
+
+
+class Skeleton:
+    """Sequential user code over fields, executed by the Skeleton's
+    generated multi-GPU schedule (§V)."""
+
+    def __init__(self, grid: Grid, occ: int = OCC_TWO_WAY):
+        self.grid = grid
+        self.handle = P()
+        self.fields = []  # keep the fields alive as long as the skeleton
+        _check(lib().nb_skeleton_create(grid.handle, int(occ), C.byref(self.handle)))
+
+    def axpby(self, a: float, x: Field, b: float, y: Field):
+        self.fields += [x, y]
+        _check(lib().nb_skeleton_axpby(self.handle, float(a), _h(x), float(b), _h(y)))
+
+    def axpy(self, a: float, x: Field, y: Field):
+        self.axpby(a, x, 1.0, y)
+
+    def laplace7(self, x: Field, y: Field):
+        self.fields += [x, y]
+        _check(lib().nb_skeleton_laplace7(self.handle, _h(x), _h(y)))
+
+    def dot(self, x: Field, y: Field, slot: int):
+        self.fields += [x, y]
+        _check(lib().nb_skeleton_dot(self.handle, _h(x), _h(y), int(slot)))
+
+    def compile(self):
+        _check(lib().nb_skeleton_compile(self.handle))
+
+    def run(self):
+        _check(lib().nb_skeleton_run(self.handle))
+
+    def result(self, slot: int) -> float:
+        v = C.c_double()
+        _check(lib().nb_skeleton_result(self.handle, int(slot), C.byref(v)))
+        return v.value
+
+    def describe(self) -> dict:
+        return _json_out(lambda buf, cap, n: lib().nb_skeleton_describe(self.handle, buf, cap, n))
+
+    def close(self):
+        if self.handle:
+            _check(lib().nb_skeleton_destroy(self.handle))
+            self.handle = P()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

@@ -1111,25 +1111,40 @@ nb_status nb_reduce_finalize(nb_grid *g, int card, int mode, void *state, int sl
 
 nb_status nb_sparse_dot_partials(const nb_field *x, const nb_field *y);
 
-nb_status nb_dot_partials(const nb_field *x, const nb_field *y) {
+// canonical tile partials of <x, y> over the planes of view v (a plane's
+// partials do not depend on which launch produced them, so a split reduce —
+// internal planes, then boundary planes — fills the same tiles)
+nb_status nb_dot_partials_view(const nb_field *x, const nb_field *y, nb_view v) {
     nb_grid *g = x->g;
-    if (g->sparse) return nb_sparse_dot_partials(x, y);
+    if (g->sparse) {
+        if (v != NB_VIEW_STANDARD) NB_FAIL(NB_EUNSUPPORTED, "split reduce on element-sparse grids");
+        return nb_sparse_dot_partials(x, y);
+    }
     for (int p = 0; p < g->nparts; ++p) {
         if (!g->parts[p].local) continue;
-        PGeo geo = pgeo(x, p);
-        int nchunk = (geo.nzl + ZC - 1) / ZC;
-        dim3 blk(32 * ZW), grd(g->tiles_x, (g->ny + ZW * ZR_STO - 1) / (ZW * ZR_STO), nchunk * x->card);
-        LaunchScope ls(g, g->cs, "k_dot");
-        if (x->dt == NB_F64)
-            k_dot<double><<<grd, blk, 0, g->cs>>>((const double *)x->base[p], (const double *)y->base[p], geo,
-                                                   dense_cs(x, p), nchunk, g->tp, g->T, g->tiles_y);
-        else
-            k_dot<float><<<grd, blk, 0, g->cs>>>((const float *)x->base[p], (const float *)y->base[p], geo,
-                                                  dense_cs(x, p), nchunk, g->tp, g->T, g->tiles_y);
-        NB_TRY(nb_launch_check("k_dot"));
+        for (auto rg : view_ranges(g, p, v)) {
+            PGeo geo = pgeo(x, p);
+            const int64_t off = (int64_t)rg.first * geo.ps * x->esz;  // planes shift, every component alike
+            geo.z0 += rg.first;
+            geo.nzl = rg.second - rg.first;
+            int nchunk = (geo.nzl + ZC - 1) / ZC;
+            dim3 blk(32 * ZW), grd(g->tiles_x, (g->ny + ZW * ZR_STO - 1) / (ZW * ZR_STO), nchunk * x->card);
+            LaunchScope ls(g, g->cs, "k_dot");
+            if (x->dt == NB_F64)
+                k_dot<double><<<grd, blk, 0, g->cs>>>((const double *)(x->base[p] + off),
+                                                       (const double *)(y->base[p] + off), geo, dense_cs(x, p), nchunk,
+                                                       g->tp, g->T, g->tiles_y);
+            else
+                k_dot<float><<<grd, blk, 0, g->cs>>>((const float *)(x->base[p] + off),
+                                                      (const float *)(y->base[p] + off), geo, dense_cs(x, p), nchunk,
+                                                      g->tp, g->T, g->tiles_y);
+            NB_TRY(nb_launch_check("k_dot"));
+        }
     }
     return NB_OK;
 }
+
+nb_status nb_dot_partials(const nb_field *x, const nb_field *y) { return nb_dot_partials_view(x, y, NB_VIEW_STANDARD); }
 
 extern "C" nb_status nb_dot(const nb_field *x, const nb_field *y, double *host_out) {
     NB_TRY(check_pair(x, y));
