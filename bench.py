@@ -471,6 +471,52 @@ def bench_c1(local):
                                     "to host); latency-bound: 2 MB fields live in L2"}
 
 
+def bench_skeleton(local, n=512, parts=4, iters=10):
+    """the Skeleton's generated schedule (separate map / stencil /
+    reduce containers, halo nodes, Two-way OCC, BFS streams + events) against
+    the hand-written fused schedule of the same sequential code (the Fig. 4a
+    loop), on `parts` virtual partitions; bit-identical results
+    (test_gpu_skeleton.py), device time per iteration on the compute stream."""
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    g = nb.Grid((n, n, n), nparts=parts, devices=[local] * parts)
+    stream = torch.cuda.ExternalStream(g.stream())
+    x, y = nb.Field(g), nb.Field(g)
+    x.fill_uniform(seed=1)
+    y.fill_const(0.0)
+    sk = nb.Skeleton(g, nb.OCC_TWO_WAY)
+    for k in range(iters):
+        sk.axpy(0.125, y, x)
+        sk.laplace7(x, y)
+        sk.dot(x, y, k)
+    sk.compile()
+    plan = sk.describe()
+
+    def t(fn):
+        fn()
+        g.sync()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        fn()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        return ev0.elapsed_time(ev1) / iters
+
+    ms_sk = t(sk.run)
+    ms_fused = t(lambda: nb.nb_map_stencil_reduce(x, y, 0.125, iters, nb.OCC_TWO_WAY))
+    sk.close()
+    x.close(), y.close()
+    g.close()
+    cells = n ** 3
+    return {"workload": f"Fig. 4a loop (axpy, 7-pt, dot) x {iters}, {n}^3 fp64, {parts} partitions, Two-way OCC",
+            "skeleton_ms_per_iter": ms_sk, "fused_ms_per_iter": ms_fused,
+            "skeleton_gbs": 56 * cells / ms_sk / 1e6, "fused_gbs": 32 * cells / ms_fused / 1e6,
+            "nodes": len(plan["nodes"]), "streams": plan["streams"], "events": plan["events"],
+            "note": "skeleton = unfused containers (24 + 16 + 16 = 56 B/cell/iter), as Neon generates them; "
+                    "fused = one kernel per iteration (32 B/cell/iter)"}
+
+
 # ---------------------------------------------------------------------------
 def cpu_baseline_cg(n, iters=2):
     """The oracle (plain C, fp64, OpenMP over planes) on the host cores:
@@ -561,7 +607,8 @@ def main():
             lbm = bench_lbm_run(args.n, 20, 3, 1, local)
             out["also"] = {"lbm_d3q19": lbm, "c1": bench_c1(local),
                            "sparse_c4": bench_sparse_run(args.n, 20, 3, 1, local),
-                           "fem_c5": bench_fem_run(384, 20, 3, 1, local)}
+                           "fem_c5": bench_fem_run(384, 20, 3, 1, local),
+                           "skeleton_f1": bench_skeleton(local)}
             out["cpu_baseline"] = cpu_baseline_cg(args.n)
             out["also"]["lbm_d3q19"]["cpu_baseline"] = cpu_baseline_lbm()
     elif args.workload in ("sparse", "fem"):
