@@ -507,7 +507,10 @@ __device__ __forceinline__ T sp_nsum(const T *x, const int32_t *conn, int64_t n,
 // NSB segments per block: thread t handles cell t of each of them, so every
 // thread has NSB independent loads per operand in flight; each segment keeps
 // its own canonical reduction (butterfly per warp, then the 8 warps).
-constexpr int NSB = 4;
+#ifndef NB_SP_NSB
+#define NB_SP_NSB 4
+#endif
+constexpr int NSB = NB_SP_NSB;
 
 template <int K>
 __global__ void __launch_bounds__(SEG) k_sp(SpArgs A) {
@@ -544,12 +547,30 @@ __global__ void __launch_bounds__(SEG) k_sp(SpArgs A) {
 #pragma unroll
         for (int k = 0; k < NSB; ++k) prod[k] = __dmul_rn(a[k], b[k]);
     } else if (K == SPK_CG_INIT || K == SPK_CG_Q) {  // CG_INIT: r = b - A x; CG_Q: q = A p, <p, q>
-        double s[NSB], c[NSB], bb[NSB];
+        // all connectivity loads of the NSB cells first, then all gathers:
+        // one table + one gather latency per thread instead of NSB of each
+        const double outv = K == SPK_CG_INIT ? A.outside : 0.0;
+        int32_t nbr[NSB][6];
+#pragma unroll
+        for (int k = 0; k < NSB; ++k)
+#pragma unroll
+            for (int d = 0; d < 6; ++d) nbr[k][d] = valid[k] ? __ldg(A.conn + (int64_t)d * A.n + jj[k]) : -1;
+        double s[NSB], c[NSB], bb[NSB], v[NSB][6];
 #pragma unroll
         for (int k = 0; k < NSB; ++k) {
-            s[k] = valid[k] ? sp_nsum(A.a, A.conn, A.n, jj[k], K == SPK_CG_INIT ? A.outside : 0.0) : 0.0;
-            c[k] = valid[k] ? A.a[i[k]] : 0.0;
-            bb[k] = (K == SPK_CG_INIT && valid[k]) ? A.b[i[k]] : 0.0;
+            c[k] = valid[k] ? __ldg(A.a + i[k]) : 0.0;
+            bb[k] = (K == SPK_CG_INIT && valid[k]) ? __ldg(A.b + i[k]) : 0.0;
+        }
+#pragma unroll
+        for (int k = 0; k < NSB; ++k)
+#pragma unroll
+            for (int d = 0; d < 6; ++d) v[k][d] = nbr[k][d] >= 0 ? __ldg(A.a + nbr[k][d]) : outv;
+#pragma unroll
+        for (int k = 0; k < NSB; ++k) {  // canonical order -x, +x, -y, +y, -z, +z (sp_nsum)
+            double t = v[k][0];
+#pragma unroll
+            for (int d = 1; d < 6; ++d) t = t + v[k][d];
+            s[k] = valid[k] ? t : 0.0;
         }
 #pragma unroll
         for (int k = 0; k < NSB; ++k) {
