@@ -33,6 +33,8 @@ nb_status nb_dot_partials(const nb_field *x, const nb_field *y);
 nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v);
 bool nb_tma_enabled();
 nb_status nb_cgB_tma(nb_grid *g, const PGeo &geo, const double *p, double *r, int zb, int ze, const CgScal *sc);
+nb_status nb_c1_tma(nb_grid *g, const PGeo &geo, const double *xin, const double *yin, double *xout, double *yout,
+                    double a, bool domap, int zb, int ze);
 nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x, bool domap,
                      int zb, int ze, const CgScal *sc);
 
@@ -461,6 +463,10 @@ static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int
     const char *name = MODE == MSR_C1 ? "k_msr_c1" : "k_msr_cgA";
     if (MODE == MSR_CG && RC && ZR_MAP == 1 && nb_tma_enabled())  // TMA-staged phase A
         return nb_cgA_tma(g, pgeo(f, p), A.w, A.v, A.u, A.xs, DM, zb, ze, A.sc);
+    // TMA-staged C1 chain: large grids only (the 64^3 C1 config lives in L2,
+    // where the register/L1 kernel has lower latency per launch)
+    if (MODE == MSR_C1 && RC && ZR_MAP == 1 && nb_tma_enabled() && (int64_t)g->nx * g->ny * g->nz >= (1 << 21))
+        return nb_c1_tma(g, pgeo(f, p), A.w, A.v, A.u, A.out, A.m, DM, zb, ze);
     if (RC && ZR_MAP == 1 && !getenv("NB_GENERIC_MSR")) {
         // specialised recompute kernel (same arithmetic and dot order)
         dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);

@@ -42,17 +42,21 @@ struct __align__(128) CgAStage {
 };
 static_assert(sizeof(double) * BY * BX < TPAD && TPAD % 128 == 0, "stage tile padding");
 
-template <bool DOMAP>
+// C1 (C1 = true): the same map -> stencil -> reduce chain of Fig. 4a with
+// r -> x_in, p_old -> y_in, p_new -> x_out (u = fma(a, y_in, x_in)),
+// out = L(u) = fma(-6, u, s) stored to y_out, dot u * out, no deferred x.
+template <bool DOMAP, bool C1 = false>
 __global__ void __launch_bounds__(DOT_TX *DOT_TY)
     k_cgA_tma(const __grid_constant__ CUtensorMap m_r, const __grid_constant__ CUtensorMap m_po,
               const __grid_constant__ CUtensorMap m_pn, const __grid_constant__ CUtensorMap m_x, double *pn, double *xs,
-              PGeo g, int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_y) {
+              PGeo g, int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_y, double c1_a = 0.0,
+              double *c1_out = nullptr) {
     __shared__ CgAStage st[NSTAGE];
     __shared__ __align__(8) uint64_t bar[NSTAGE];
     __shared__ double sw[TZC][DOT_TY];
-    if (sc->status != 0) return;
-    const double beta = sc->beta, ap = sc->alpha_prev;
-    const bool dox = DOMAP && sc->pending;
+    if (!C1 && sc->status != 0) return;
+    const double beta = C1 ? c1_a : sc->beta, ap = C1 ? 0.0 : sc->alpha_prev;
+    const bool dox = !C1 && DOMAP && sc->pending;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const int x0 = blockIdx.x * DOT_TX, y0 = blockIdx.y * DOT_TY;
     const int xi = x0 + lane, yi = y0 + w;
@@ -105,8 +109,9 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY)
             s = __dadd_rn(s, U(z, w + 2, lane + 2));
             s = __dadd_rn(s, below);
             s = __dadd_rn(s, above);
-            const double q = fma(6.0, center, -s);
+            const double q = C1 ? fma(-6.0, center, s) : fma(6.0, center, -s);
             const int64_t e = o + (int64_t)z * g.ps;
+            if (C1) __stcs(c1_out + e, q);
             if (DOMAP) {
                 pn[e] = center;
                 if (dox) {
@@ -292,6 +297,26 @@ nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double 
     else
         k_cgA_tma<false><<<grd, blk, 0, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T, g->tiles_y);
     return nb_launch_check("k_cgA_tma");
+}
+
+// C1 map-stencil-reduce on planes [zb, ze): x_out = x_in + a y_in (stored
+// when domap), y_out = L(x_out), per-plane tile partials of x_out * y_out
+nb_status nb_c1_tma(nb_grid *g, const PGeo &geo, const double *xin, const double *yin, double *xout, double *yout,
+                    double a, bool domap, int zb, int ze) {
+    if (ze <= zb) return NB_OK;
+    CUtensorMap mx, my, mu;
+    NB_TRY(tmap_for(xin, geo, 0, &mx));
+    NB_TRY(tmap_for(yin, geo, 0, &my));
+    NB_TRY(tmap_for(xout, geo, 0, &mu));
+    dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + TZC - 1) / TZC);
+    LaunchScope ls(g, g->cs, "k_msr_c1");
+    if (domap)
+        k_cgA_tma<true, true><<<grd, blk, 0, g->cs>>>(mx, my, mu, mx, xout, nullptr, geo, zb, ze, nullptr, g->tp, g->T,
+                                                      g->tiles_y, a, yout);
+    else
+        k_cgA_tma<false, true><<<grd, blk, 0, g->cs>>>(mx, my, mu, mx, xout, nullptr, geo, zb, ze, nullptr, g->tp,
+                                                       g->T, g->tiles_y, a, yout);
+    return nb_launch_check("k_c1_tma");
 }
 
 // CG phase B on planes [zb, ze) of a partition (stored p_new, r)

@@ -107,3 +107,16 @@ def test_skeleton_state_errors():
             sk.dot(x, y, 0)  # compiled: no more containers
         sk.close()
         x.close(), y.close()
+
+
+@pytest.mark.parametrize("parts,occ", [(1, nb.OCC_TWO_WAY), (3, nb.OCC_TWO_WAY), (3, nb.OCC_NONE),
+                                       (2, nb.OCC_STANDARD)])
+def test_large_c1_tma_chain_bitwise_equals_skeleton(parts, occ):
+    """Above 2^21 cells the fused C1 chain runs on the TMA-staged kernel
+    (k_cgA_tma<., C1>); it must still equal the unfused generated schedule
+    bit for bit (ragged x / y tiles, several 32-plane chunks)."""
+    dims = (130, 129, 131)
+    x0 = synth.uniform(dims, seed=8)
+    xs, ys, ds, _ = run_skeleton(dims, parts, occ, x0, iters=3)
+    xf, yf, df = run_fused(dims, parts, occ, x0, iters=3)
+    assert np.array_equal(xs, xf) and np.array_equal(ys, yf) and np.array_equal(ds, df)
