@@ -59,6 +59,7 @@ def lib():
         L.or_cg.restype = i32
         L.or_lbm_lattice.argtypes = [P, P, P]
         L.or_lbm_step.argtypes = [i32, i32, i32, i32, d, d, d, P, P]
+        L.or_lbm_step_masked.argtypes = [i32, i32, i32, i32, d, d, d, P, P, P]
         L.or_lbm_macroscopic.argtypes = [i32, i32, i32, P, P, P]
         L.or_num_threads.restype = i32
         L.or_set_num_threads.argtypes = [i32]
@@ -204,13 +205,21 @@ def lbm_lattice():
 LBM_CAVITY, LBM_PERIODIC = 0, 1
 
 
-def lbm_step(fin, omega, u_lid=0.05, rho_w=1.0, bc=LBM_CAVITY):
-    """fin: [19][z][y][x] (any float dtype; computed in fp64) -> fout fp64."""
+def lbm_step(fin, omega, u_lid=0.05, rho_w=1.0, bc=LBM_CAVITY, active=None):
+    """fin: [19][z][y][x] (any float dtype; computed in fp64) -> fout fp64.
+    active: optional [z][y][x] mask of fluid cells (element-sparse domain,
+    bounce-back at inactive sources; inactive cells -> 0)."""
     fin = _f64(fin)
     _, nz, ny, nx = fin.shape
     fout = np.empty_like(fin)
-    lib().or_lbm_step(nx, ny, nz, int(bc), float(omega), float(u_lid), float(rho_w),
-                      _ptr(fin), _ptr(fout))
+    if active is None:
+        lib().or_lbm_step(nx, ny, nz, int(bc), float(omega), float(u_lid), float(rho_w),
+                          _ptr(fin), _ptr(fout))
+    else:
+        m = np.ascontiguousarray(active, dtype=np.uint8)
+        assert m.shape == (nz, ny, nx)
+        lib().or_lbm_step_masked(nx, ny, nz, int(bc), float(omega), float(u_lid), float(rho_w),
+                                 m.ctypes.data_as(C.c_void_p), _ptr(fin), _ptr(fout))
     return fout
 
 

@@ -472,8 +472,15 @@ void or_lbm_lattice(int *c /* 19*3 */, double *w /* 19 */, int *opp /* 19 */) {
     }
 }
 
-void or_lbm_step(int nx, int ny, int nz, int bc, double omega, double u_lid, double rho_w,
-                 const double *fin, double *fout) {
+/* D3Q19 pull step on an element-sparse domain ("bounce-
+ * back where the connectivity table gives -1"): active[z][y][x] != 0 marks
+ * fluid cells (NULL: every cell).  A population whose source x - c_i is not an
+ * active in-box cell bounces back (half-way, from the opposite population of
+ * this cell); the moving-lid term applies only to sources beyond the y = Ny
+ * face (the dense reading).  Inactive cells get fout = 0 (they are not
+ * stored; the host view reads them back as the outside value 0). */
+void or_lbm_step_masked(int nx, int ny, int nz, int bc, double omega, double u_lid, double rho_w,
+                        const unsigned char *active, const double *fin, double *fout) {
     int c[57], opp[19];
     double w[19];
     or_lbm_lattice(c, w, opp);
@@ -484,14 +491,22 @@ void or_lbm_step(int nx, int ny, int nz, int bc, double omega, double u_lid, dou
             for (int i = 0; i < nx; ++i) {
                 int64_t cell = IDX(i, j, k);
                 double f[19];
+                if (active && !active[cell]) {
+                    for (int q = 0; q < 19; ++q) fout[(int64_t)q * n + cell] = 0.0;
+                    continue;
+                }
                 for (int q = 0; q < 19; ++q) {
                     int si = i - c[3 * q], sj = j - c[3 * q + 1], sk = k - c[3 * q + 2];
                     if (bc == 1) {
                         si = (si + nx) % nx;
                         sj = (sj + ny) % ny;
                         sk = (sk + nz) % nz;
-                        f[q] = fin[(int64_t)q * n + IDX(si, sj, sk)];
-                    } else if (si >= 0 && si < nx && sj >= 0 && sj < ny && sk >= 0 && sk < nz) {
+                        if (active && !active[IDX(si, sj, sk)])
+                            f[q] = fin[(int64_t)opp[q] * n + cell];
+                        else
+                            f[q] = fin[(int64_t)q * n + IDX(si, sj, sk)];
+                    } else if (si >= 0 && si < nx && sj >= 0 && sj < ny && sk >= 0 && sk < nz &&
+                               (!active || active[IDX(si, sj, sk)])) {
                         f[q] = fin[(int64_t)q * n + IDX(si, sj, sk)];
                     } else {
                         double v = fin[(int64_t)opp[q] * n + cell];
@@ -515,6 +530,11 @@ void or_lbm_step(int nx, int ny, int nz, int bc, double omega, double u_lid, dou
                     fout[(int64_t)q * n + cell] = f[q] - omega * (f[q] - feq);
                 }
             }
+}
+
+void or_lbm_step(int nx, int ny, int nz, int bc, double omega, double u_lid, double rho_w,
+                 const double *fin, double *fout) {
+    or_lbm_step_masked(nx, ny, nz, bc, omega, u_lid, rho_w, 0, fin, fout);
 }
 
 /* rho and u (3 components) of a population field f: [19][z][y][x] */
