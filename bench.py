@@ -313,6 +313,47 @@ def bench_lbm_run(n, steps, warmup, world, local, occ="standard"):
     return res
 
 
+LBM_SPARSE_BYTES_PER_CELL = 152 + 18 * 4  # 19 loads + 19 stores fp32, + the 18-direction source table
+
+
+def bench_lbm_sparse_run(n, steps, warmup, local):
+    """D3Q19 on an element-sparse domain — the C4 sphere (30 % of
+    the n^3 box) as the fluid region, bounce-back on its surface, 1 GPU."""
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    import synth
+    m = synth.sphere_mask(n)
+    g = nb.Grid((n, n, n), devices=[local], active=m)
+    active = int(m.sum(dtype="int64"))
+    stream = torch.cuda.ExternalStream(g.stream())
+    st = {"a": nb.Field(g, "f32", 19), "b": nb.Field(g, "f32", 19)}
+    nb.nb_lbm_init(st["a"], 1.0, (0.01, 0.0, 0.0))
+    om = lbm_omega(n)
+
+    def run(k):
+        st["a"], st["b"] = nb.nb_lbm_step(st["a"], st["b"], om, k)
+    run(warmup)
+    g.sync()
+    ms, clocks = timed(1, stream, lambda: run(steps), local)
+    g.profile(True)
+    run(3)
+    nk, msk = g.profile_read("k_sp_lbm")
+    g.profile(False)
+    hbm, peak_kind = peaks()
+    k_ms = msk / max(nk, 1)
+    achieved = LBM_SPARSE_BYTES_PER_CELL * active / (k_ms / 1e3) / 1e9
+    st["a"].close(), st["b"].close()
+    g.close()
+    return {"workload": f"D3Q19 BGK on the element-sparse sphere ({active} active cells of {n}^3, 30 %), fp32, "
+                        "bounce-back at the surface (SURVEY f2)",
+            "value": active * steps / (ms / 1e3) / 1e6, "unit": "MLUPS (active cells)", "ms_per_step": ms / steps,
+            "roofline": {"bound": "hbm", "kernel": "k_sp_lbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                         "frac": achieved / hbm, "peak_kind": peak_kind,
+                         "algorithmic_bytes_per_cell": LBM_SPARSE_BYTES_PER_CELL, "launch_ms": k_ms},
+            "clocks": clocks}
+
+
 SPARSE_BYTES = {"k_sp_cg_map": 40, "k_sp_cg_q": 40, "k_sp_cg_r": 24}  # per active cell (q: p 8 + conn 24 + q 8)
 FEM_BYTES = {"k_fem_map": 120, "k_fem_cg_q": 48, "k_fem_r": 72}     # per node, 3 fp64 components
 FEM_FLOPS_PER_NODE = 306  # 153 nonzero stencil coefficients x 2 (SURVEY §8(a) a10)
@@ -608,7 +649,8 @@ def main():
             out["also"] = {"lbm_d3q19": lbm, "c1": bench_c1(local),
                            "sparse_c4": bench_sparse_run(args.n, 20, 3, 1, local),
                            "fem_c5": bench_fem_run(384, 20, 3, 1, local),
-                           "skeleton_f1": bench_skeleton(local)}
+                           "skeleton_f1": bench_skeleton(local),
+                           "lbm_sparse_f2": bench_lbm_sparse_run(args.n, 20, 3, local)}
             out["cpu_baseline"] = cpu_baseline_cg(args.n)
             out["also"]["lbm_d3q19"]["cpu_baseline"] = cpu_baseline_lbm()
     elif args.workload in ("sparse", "fem"):

@@ -129,6 +129,7 @@ struct NbSparsePart {
     std::vector<int64_t> pstart;            // own-slot offset of each local plane [nz_p + 1]
     int64_t *d_pstart = nullptr;            // device copy
     int32_t *conn = nullptr;                // [6][n] buffer index of the neighbour, -1 = outside
+    int32_t *conn19 = nullptr;              // D3Q19 pull sources [18][n] (lazy): -1 wall, -2 lid
     int32_t *coord = nullptr;               // [n] x | y << 16
     int max_plane = 0;                      // max active cells in one local plane
     // non-empty 256-cell dot segments, plane-major: entry = zl << 16 | seg
@@ -164,6 +165,7 @@ struct nb_grid {
     // element-sparse
     std::vector<NbSparsePart> sp;
     std::vector<int64_t> plane_count;  // [nz] active per global plane
+    std::vector<uint8_t> host_mask;    // [z][y][x] active cells (element-sparse; lazy tables)
     int64_t n_active = 0;
     NbPeer *peer = nullptr;  // peer-memory transport (multi-process)
 };

@@ -52,8 +52,7 @@ struct LbmArgs {
 
 // BGK collision of the gathered populations and the streaming store (shared
 // by the interior fast path and the boundary path: same code, same bits)
-__device__ __forceinline__ void lbm_collide_store(const float (&f)[Q19], const LbmArgs &A, int64_t cell,
-                                                  int zl, int64_t row) {
+__device__ __forceinline__ void lbm_collide(const float (&f)[Q19], float om, float (&o)[Q19]) {
     float rho = 0.f, jx = 0.f, jy = 0.f, jz = 0.f;
 #pragma unroll
     for (int i = 0; i < Q19; ++i) {
@@ -67,15 +66,20 @@ __device__ __forceinline__ void lbm_collide_store(const float (&f)[Q19], const L
     }
     const float ux = jx / rho, uy = jy / rho, uz = jz / rho;
     const float usq = ux * ux + uy * uy + uz * uz;
-    const float om = A.omega;
-    float o[Q19];
 #pragma unroll
     for (int i = 0; i < Q19; ++i) {
         float cu = (float)CXv(i) * ux + (float)CYv(i) * uy + (float)CZv(i) * uz;
         float feq = Wv(i) * rho * (1.0f + 3.0f * cu + 4.5f * cu * cu - 1.5f * usq);
         o[i] = f[i] - om * (f[i] - feq);
-        __stcs(A.fout[i] + cell, o[i]);
     }
+}
+
+__device__ __forceinline__ void lbm_collide_store(const float (&f)[Q19], const LbmArgs &A, int64_t cell,
+                                                  int zl, int64_t row) {
+    float o[Q19];
+    lbm_collide(f, A.omega, o);
+#pragma unroll
+    for (int i = 0; i < Q19; ++i) __stcs(A.fout[i] + cell, o[i]);
     // halo transfer fused into the producing kernel: outgoing populations of
     // the boundary planes go straight into the neighbours' halo planes
     if (zl == 0 && A.rem_lo[14]) {
@@ -171,7 +175,151 @@ static inline int64_t lcs(const nb_field *f, int p) { return f->ps * (f->g->part
 static nb_status lbm_check(const nb_field *f) {
     if (!f) NB_FAIL(NB_EINVAL, "NULL field");
     if (f->dt != NB_F32 || f->card != Q19) NB_FAIL(NB_EMISMATCH, "LBM needs an fp32 field of cardinality 19");
-    if (f->g->sparse) NB_FAIL(NB_EUNSUPPORTED, "LBM on element-sparse grids is not built yet (SURVEY f2)");
+    return NB_OK;
+}
+
+// ===========================================================================
+// D3Q19 on element-sparse domains ("the
+// domain is free-form", L248 element-sparse grid).  Same pull step, with the
+// sources looked up in an 18-direction connectivity table of the compact
+// (z, y, x) cell order: -1 = no fluid source (inactive cell or outside the
+// box: half-way bounce-back), -2 = beyond the moving lid (y = Ny face).
+// One thread per active cell; the collision is the dense kernel's (bitwise:
+// a full mask reproduces the dense grid).  Halos: the 5 populations with
+// c_z = +1 up, the 5 with c_z = -1 down, contiguous segments.
+// ===========================================================================
+nb_status nb_sparse_slab_map(nb_grid *g, int p, uint8_t **d_mask, int32_t **d_map, int *slab_z0, int *nslab);
+nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d);
+
+__global__ void k_sp_conn19(const uint8_t *__restrict__ mask, const int32_t *__restrict__ map, int nx, int ny,
+                            int slab_z0, int nslab, int z0, int NZ, int64_t hl, int64_t n, int32_t *conn19) {
+    const int x = blockIdx.x * blockDim.x + threadIdx.x, y = blockIdx.y, z = z0 + blockIdx.z;
+    if (x >= nx) return;
+    const int64_t plane = (int64_t)nx * ny;
+    const int64_t cell = (int64_t)(z - slab_z0) * plane + (int64_t)y * nx + x;
+    if (!mask[cell]) return;
+    const int64_t j = (int64_t)map[cell] - hl;
+#pragma unroll
+    for (int q = 1; q < Q19; ++q) {
+        const int sx = x - CXv(q), sy = y - CYv(q), sz = z - CZv(q);
+        int32_t v = -1;
+        if (sx >= 0 && sx < nx && sy >= 0 && sy < ny && sz >= 0 && sz < NZ && sz - slab_z0 >= 0 &&
+            sz - slab_z0 < nslab) {
+            const int64_t sc = (int64_t)(sz - slab_z0) * plane + (int64_t)sy * nx + sx;
+            if (mask[sc]) v = map[sc];
+        } else if (sy == ny && sx >= 0 && sx < nx && sz >= 0 && sz < NZ) {
+            v = -2;
+        }
+        conn19[(int64_t)(q - 1) * n + j] = v;
+    }
+}
+
+__global__ void __launch_bounds__(128) k_sp_lbm(const float *__restrict__ fin, float *__restrict__ fout, int64_t cs,
+                                                int64_t hl, int64_t n, const int32_t *__restrict__ conn19, float om,
+                                                float ulid, float rho_w) {
+    const int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (j >= n) return;
+    const int64_t own = hl + j;
+    int32_t src[Q19];
+#pragma unroll
+    for (int q = 1; q < Q19; ++q) src[q] = __ldg(conn19 + (int64_t)(q - 1) * n + j);
+    float f[Q19];
+    f[0] = __ldg(fin + own);
+#pragma unroll
+    for (int q = 1; q < Q19; ++q) {
+        const int32_t k = src[q];
+        float v = __ldg(k >= 0 ? fin + (int64_t)q * cs + k : fin + (int64_t)OPPv(q) * cs + own);
+        if (CXv(q) != 0 && k == -2) v = v + 6.0f * Wv(q) * rho_w * ((float)CXv(q) * ulid);
+        f[q] = v;
+    }
+    float o[Q19];
+    lbm_collide(f, om, o);
+#pragma unroll
+    for (int q = 0; q < Q19; ++q) __stcs(fout + (int64_t)q * cs + own, o[q]);
+}
+
+__global__ void k_sp_lbm_init(float *f, int64_t cs, float rho, float ux, float uy, float uz) {
+    const float usq = ux * ux + uy * uy + uz * uz;
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < cs; e += (int64_t)gridDim.x * blockDim.x) {
+#pragma unroll
+        for (int i = 0; i < Q19; ++i) {
+            float cu = (float)CXv(i) * ux + (float)CYv(i) * uy + (float)CZv(i) * uz;
+            f[(int64_t)i * cs + e] = Wv(i) * rho * (1.0f + 3.0f * cu + 4.5f * cu * cu - 1.5f * usq);
+        }
+    }
+}
+
+__global__ void k_sp_lbm_macro(const float *f, float *rho_o, float *u_o, int64_t cs, int64_t cs_rho, int64_t cs_u,
+                               int64_t hl, int64_t n) {
+    const int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (j >= n) return;
+    const int64_t e = hl + j;
+    float rho = 0.f, jx = 0.f, jy = 0.f, jz = 0.f;
+#pragma unroll
+    for (int i = 0; i < Q19; ++i) {
+        float v = f[(int64_t)i * cs + e];
+        rho += v;
+        jx += (float)CXv(i) * v;
+        jy += (float)CYv(i) * v;
+        jz += (float)CZv(i) * v;
+    }
+    (void)cs_rho;
+    rho_o[e] = rho;
+    u_o[e] = jx / rho;
+    u_o[cs_u + e] = jy / rho;
+    u_o[2 * cs_u + e] = jz / rho;
+}
+
+static nb_status sp_lbm_tables(nb_grid *g) {
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        NbSparsePart &sp = g->sp[p];
+        if (sp.conn19) continue;
+        uint8_t *d_mask = nullptr;
+        int32_t *d_map = nullptr;
+        int slab_z0 = 0, nslab = 0;
+        nb_status s = nb_sparse_slab_map(g, p, &d_mask, &d_map, &slab_z0, &nslab);
+        if (s == NB_OK && cudaMalloc(&sp.conn19, sizeof(int32_t) * 18 * std::max<int64_t>(sp.n, 1)) != cudaSuccess) {
+            cudaGetLastError();
+            nb_set_error("sparse LBM: cudaMalloc of the D3Q19 connectivity failed");
+            s = NB_ENOMEM;
+        }
+        if (s == NB_OK && g->parts[p].nz() > 0) {
+            dim3 blk(128), grd((g->nx + 127) / 128, g->ny, g->parts[p].nz());
+            LaunchScope ls(g, g->cs, "k_sp_conn19");
+            k_sp_conn19<<<grd, blk, 0, g->cs>>>(d_mask, d_map, g->nx, g->ny, slab_z0, nslab, g->parts[p].z0, g->nz,
+                                                 sp.hl, sp.n, sp.conn19);
+            s = nb_launch_check("k_sp_conn19");
+            cudaStreamSynchronize(g->cs);
+        }
+        cudaFree(d_mask);
+        cudaFree(d_map);
+        if (s != NB_OK) return s;
+    }
+    return NB_OK;
+}
+
+static nb_status sp_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm_params *prm, int nsteps) {
+    nb_field *fin = *pfin, *fout = *pfout;
+    nb_grid *g = fin->g;
+    if (prm->bc != NB_LBM_CAVITY)
+        NB_FAIL(NB_EUNSUPPORTED, "LBM on element-sparse grids: bounce-back (cavity) boundaries only");
+    NB_TRY(sp_lbm_tables(g));
+    NB_TRY(nb_sparse_halo_comps(fin, 9, 14, 14, 19));
+    for (int t = 0; t < nsteps; ++t) {
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbSparsePart &sp = g->sp[p];
+            if (sp.n == 0) continue;
+            LaunchScope ls(g, g->cs, "k_sp_lbm");
+            k_sp_lbm<<<(unsigned)((sp.n + 127) / 128), 128, 0, g->cs>>>(
+                (const float *)fin->base[p], (float *)fout->base[p], fin->pcs[p], sp.hl, sp.n, sp.conn19,
+                (float)prm->omega, (float)prm->u_lid, (float)prm->rho_w);
+            NB_TRY(nb_launch_check("k_sp_lbm"));
+        }
+        NB_TRY(nb_sparse_halo_comps(fout, 9, 14, 14, 19));
+        std::swap(fin, fout);
+    }
+    *pfin = fin;
+    *pfout = fout;
     return NB_OK;
 }
 
@@ -180,6 +328,15 @@ extern "C" nb_status nb_lbm_init(nb_field *f, double rho0, const double u0[3]) {
     if (!u0) NB_FAIL(NB_EINVAL, "u0 is NULL");
     nb_grid *g = f->g;
     cudaSetDevice(g->device);
+    if (g->sparse) {
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            LaunchScope ls(g, g->cs, "k_lbm_init");
+            k_sp_lbm_init<<<296, 256, 0, g->cs>>>((float *)f->base[p], f->pcs[p], (float)rho0, (float)u0[0],
+                                                  (float)u0[1], (float)u0[2]);
+            NB_TRY(nb_launch_check("k_sp_lbm_init"));
+        }
+        return NB_OK;
+    }
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         PGeo geo = pgeo(f, p);
         dim3 blk(128), grd((g->nx + 127) / 128, g->ny, geo.nzl + 2);  // halo planes too
@@ -252,6 +409,7 @@ extern "C" nb_status nb_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm
     if (prm->bc != NB_LBM_CAVITY && prm->bc != NB_LBM_PERIODIC) NB_FAIL(NB_EINVAL, "bad bc");
     nb_grid *g = fin->g;
     cudaSetDevice(g->device);
+    if (g->sparse) return sp_lbm_step(pfin, pfout, prm, nsteps);
     const bool per = prm->bc == NB_LBM_PERIODIC;
     const bool dist = nb_halo_on_stream(g);  // halos on the halo stream (NCCL or device copies)
     // make fin's halos current (covers states written by upload/init)
@@ -314,6 +472,18 @@ extern "C" nb_status nb_lbm_macroscopic(const nb_field *f, nb_field *rho, nb_fie
         NB_FAIL(NB_EMISMATCH, "rho: fp32 card 1, u: fp32 card 3");
     nb_grid *g = f->g;
     cudaSetDevice(g->device);
+    if (g->sparse) {
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbSparsePart &sp = g->sp[p];
+            if (sp.n == 0) continue;
+            LaunchScope ls(g, g->cs, "k_lbm_macro");
+            k_sp_lbm_macro<<<(unsigned)((sp.n + 127) / 128), 128, 0, g->cs>>>(
+                (const float *)f->base[p], (float *)rho->base[p], (float *)u->base[p], f->pcs[p], rho->pcs[p],
+                u->pcs[p], sp.hl, sp.n);
+            NB_TRY(nb_launch_check("k_sp_lbm_macro"));
+        }
+        return NB_OK;
+    }
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         PGeo geo = pgeo(f, p);
         dim3 blk(128), grd((g->nx + 127) / 128, g->ny, geo.nzl);

@@ -38,6 +38,8 @@ struct MaskToInt {
 void nb_sparse_free(nb_grid *g) {
     for (auto &s : g->sp) {
         cudaFree(s.conn);
+        cudaFree(s.conn19);
+        s.conn19 = nullptr;
         cudaFree(s.coord);
         cudaFree(s.d_pstart);
         cudaFree(s.d_seg);
@@ -99,6 +101,7 @@ extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t 
     g->ny = ny;
     g->nz = nz;
     g->plane_count = counts;
+    g->host_mask.assign(active, active + (size_t)nz * plane);
     int64_t maxc = 1;
     for (auto c : counts) {
         g->n_active += c;
@@ -359,10 +362,41 @@ nb_status nb_sparse_fill(nb_field *f, nb_fill kind, uint64_t seed, double a, dou
     return NB_OK;
 }
 
+// The compact index of partition p's slab with its halo planes (the map
+// nb_grid_create_sparse builds the connectivity from): device mask and
+// exclusive-scan map of planes [slab_z0, slab_z0 + nslab); caller frees.
+nb_status nb_sparse_slab_map(nb_grid *g, int p, uint8_t **d_mask, int32_t **d_map, int *slab_z0, int *nslab) {
+    const NbPart &q = g->parts[p];
+    const int64_t plane = (int64_t)g->nx * g->ny;
+    *slab_z0 = q.z0 - (q.lo >= 0 ? 1 : 0);
+    *nslab = q.z1 + (q.hi >= 0 ? 1 : 0) - *slab_z0;
+    const int64_t ncell = (int64_t)*nslab * plane;
+    *d_mask = nullptr;
+    *d_map = nullptr;
+    void *tmp = nullptr;
+    size_t tmp_bytes = 0;
+    NB_CUDA(cudaMalloc(d_mask, ncell));
+    NB_CUDA(cudaMalloc(d_map, ncell * 4));
+    NB_CUDA(cudaMemcpyAsync(*d_mask, g->host_mask.data() + (int64_t)*slab_z0 * plane, ncell, cudaMemcpyHostToDevice,
+                            g->cs));
+    cub::TransformInputIterator<int, MaskToInt, const uint8_t *> it(*d_mask, MaskToInt());
+    NB_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, it, *d_map, ncell, g->cs));
+    NB_CUDA(cudaMalloc(&tmp, tmp_bytes));
+    NB_CUDA(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, it, *d_map, ncell, g->cs));
+    NB_CUDA(cudaStreamSynchronize(g->cs));
+    cudaFree(tmp);
+    return NB_OK;
+}
+
 // ---------------------------------------------------------------------------
 // halo: contiguous segments (the neighbour's adjacent plane), plan order
 // ---------------------------------------------------------------------------
-nb_status nb_sparse_halo_update(nb_field *f) {
+nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d);
+nb_status nb_sparse_halo_update(nb_field *f) { return nb_sparse_halo_comps(f, 0, f->card, 0, f->card); }
+
+// components [c0u, c1u) travel up (last plane -> upper neighbour's low halo),
+// [c0d, c1d) down
+nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d) {
     nb_grid *g = f->g;
     int world = g->comm ? g->comm->world : 1, rank = g->comm ? g->comm->rank : 0;
     int cnt = 0;
@@ -391,8 +425,9 @@ nb_status nb_sparse_halo_update(nb_field *f) {
     CopyBatch cb;
     for (auto &m : msgs) {
         const bool mine = m.src_rank == rank && (peer || m.dst_rank == rank);
+        const int c0 = m.up ? c0u : c0d, c1 = m.up ? c1u : c1d;
         if (mine) {
-            for (int c = 0; c < f->card && count(m) > 0; ++c) {
+            for (int c = c0; c < c1 && count(m) > 0; ++c) {
                 const char *src = f->base[m.src_part] + ((int64_t)c * f->pcs[m.src_part] + src_off(m)) * f->esz;
                 char *dst = f->base[m.dst_part] + ((int64_t)c * f->pcs[m.dst_part] + dst_off(m)) * f->esz;
                 if (cb.n == CopyBatch::MAX) {
@@ -412,7 +447,8 @@ nb_status nb_sparse_halo_update(nb_field *f) {
     for (auto &m : msgs) {
         if (m.src_rank == rank && m.dst_rank == rank) continue;
         if (count(m) == 0) continue;
-        for (int c = 0; c < f->card; ++c) {
+        const int c0 = m.up ? c0u : c0d, c1 = m.up ? c1u : c1d;
+        for (int c = c0; c < c1; ++c) {
             if (m.src_rank == rank)
                 NB_TRY(nb_nccl_send(g, f->base[m.src_part] + ((int64_t)c * f->pcs[m.src_part] + src_off(m)) * f->esz,
                                     count(m) * f->esz, m.dst_rank, g->cs));
