@@ -82,8 +82,8 @@ def c1(seed, integer, occ):
 
 
 for occ in (nb.OCC_NONE, nb.OCC_STANDARD, nb.OCC_TWO_WAY):
-    compare(f"c1 int occ{occ}", (37, 21, 16), 2, c1(1, True, occ))
-compare("c1 real 4 parts", (40, 24, 20), 4, c1(2, False, nb.OCC_TWO_WAY))
+    compare(f"c1 int occ{occ}", (37, 21, 16), WORLD, c1(1, True, occ))
+compare("c1 real 4 parts", (40, 24, 20), 2 * WORLD, c1(2, False, nb.OCC_TWO_WAY))
 
 
 # ---- dot, laplace7 + halo update -------------------------------------------
@@ -99,8 +99,8 @@ def dot_lap(g):
     return out, [d]
 
 
-compare("dot+laplace7", (45, 19, 22), 2, dot_lap)
-compare("dot+laplace7 4 parts", (45, 19, 22), 4, dot_lap)
+compare("dot+laplace7", (45, 19, 22), WORLD, dot_lap)
+compare("dot+laplace7 4 parts", (45, 19, 22), 2 * WORLD, dot_lap)
 
 
 # ---- C2: Poisson CG ----------------------------------------------------------
@@ -120,8 +120,8 @@ def cg(occ, iters):
 
 
 for occ in (nb.OCC_NONE, nb.OCC_STANDARD, nb.OCC_EXTENDED, nb.OCC_TWO_WAY):
-    compare(f"cg occ{occ}", (32, 32, 32), 2, cg(occ, 21))
-compare("cg 4 parts", (32, 32, 32), 4, cg(nb.OCC_TWO_WAY, 37))
+    compare(f"cg occ{occ}", (32, 32, 32), WORLD, cg(occ, 21))
+compare("cg 4 parts", (32, 32, 32), 2 * WORLD, cg(nb.OCC_TWO_WAY, 37))
 
 
 # ---- C3: D3Q19 LBM (cavity and periodic) ------------------------------------
@@ -138,8 +138,8 @@ def lbm(bc, occ, steps):
 
 for bc in (nb.LBM_CAVITY, nb.LBM_PERIODIC):
     for occ in (nb.OCC_NONE, nb.OCC_STANDARD):
-        compare(f"lbm bc{bc} occ{occ}", (24, 20, 18), 2, lbm(bc, occ, 7))
-compare("lbm periodic 4 parts", (24, 20, 18), 4, lbm(nb.LBM_PERIODIC, nb.OCC_STANDARD, 6))
+        compare(f"lbm bc{bc} occ{occ}", (24, 20, 18), WORLD, lbm(bc, occ, 7))
+compare("lbm periodic 4 parts", (24, 20, 18), 2 * WORLD, lbm(nb.LBM_PERIODIC, nb.OCC_STANDARD, 6))
 
 
 # ---- C4: element-sparse CG ---------------------------------------------------
@@ -159,7 +159,7 @@ def sparse_cg(g):
     return out, [r.rr, r.iters, d]
 
 
-compare("sparse cg", (n, n, n), 2, sparse_cg, active=sphere)
+compare("sparse cg", (n, n, n), WORLD, sparse_cg, active=sphere)
 
 
 # ---- C5: FEM 27-point CG -----------------------------------------------------
@@ -173,7 +173,7 @@ def fem_cg(g):
     return out, [r.rr, r.iters]
 
 
-compare("fem cg", (12, 11, 14), 2, fem_cg)
+compare("fem cg", (12, 11, 14), WORLD, fem_cg)
 
 # ---- borrowed (torch-owned) storage: IPC handle of the enclosing allocation + offset
 def wrapped_cg(g):
@@ -187,11 +187,11 @@ def wrapped_cg(g):
     return out, [r.rr, r.iters]
 
 
-compare("wrapped cg", (20, 20, 20), 2, wrapped_cg)
+compare("wrapped cg", (20, 20, 20), WORLD, wrapped_cg)
 
 
 # ---- the peer path really ran: its kernels were launched ---------------------
-g = nb.Grid((32, 32, 32), nparts=2, comm=COMM)
+g = nb.Grid((32, 32, 32), nparts=WORLD, comm=COMM)
 b, x = nb.Field(g), nb.Field(g)
 b.fill(nb.FILL_POISSON_RHS)
 x.fill_const(0.0)

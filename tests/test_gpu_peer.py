@@ -32,12 +32,14 @@ def free_port():
         return s.getsockname()[1]
 
 
-def test_peer_transport_two_processes_bitwise():
-    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+@pytest.mark.parametrize("world", [2, 3])
+def test_peer_transport_multi_process_bitwise(world):
+    """world 3: the middle rank has two remote neighbours (distinct ranks)."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
            "--master-addr", "127.0.0.1", "--master-port", str(free_port()),
            os.path.join(ROOT, "tests", "peer_worker.py")]
     env = dict(os.environ, OMP_NUM_THREADS="1")
     p = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=900)
     out = p.stdout + p.stderr
     assert p.returncode == 0, out[-6000:]
-    assert out.count("PEER_OK") == 2, out[-6000:]
+    assert out.count("PEER_OK") == world, out[-6000:]
