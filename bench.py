@@ -313,6 +313,32 @@ def bench_lbm_run(n, steps, warmup, world, local, occ="standard"):
     return res
 
 
+def bench_lbm_aa_run(n, steps, warmup, local):
+    """the AA pattern — the C3 cavity on ONE population buffer
+    updated in place (half of twoPop's memory), 1 GPU."""
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    g = nb.Grid((n, n, n), devices=[local])
+    stream = torch.cuda.ExternalStream(g.stream())
+    f = nb.Field(g, "f32", 19)
+    nb.nb_lbm_init(f, 1.0, (0.0, 0.0, 0.0))
+    om = lbm_omega(n)
+    nb.nb_lbm_step_aa(f, om, warmup + (warmup & 1))
+    g.sync()
+    steps += steps & 1
+    ms, clocks = timed(1, stream, lambda: nb.nb_lbm_step_aa(f, om, steps), local)
+    hbm, peak_kind = peaks()
+    cells = n ** 3
+    gbs = LBM_BYTES_PER_CELL * cells * steps / (ms / 1e3) / 1e9
+    f.close()
+    g.close()
+    return {"workload": f"C3 D3Q19 cavity {n}^3 fp32, AA pattern (one in-place buffer, {19 * 4 * n ** 3 / 1e9:.1f} GB "
+                        f"instead of {2 * 19 * 4 * n ** 3 / 1e9:.1f} GB) (SURVEY f3)",
+            "value": cells * steps / (ms / 1e3) / 1e6, "unit": "MLUPS", "ms_per_step": ms / steps,
+            "hbm_gbs": gbs, "hbm_frac": gbs / hbm, "peak_kind": peak_kind, "clocks": clocks}
+
+
 LBM_SPARSE_BYTES_PER_CELL = 152 + 18 * 4  # 19 loads + 19 stores fp32, + the 18-direction source table
 
 
@@ -650,7 +676,8 @@ def main():
                            "sparse_c4": bench_sparse_run(args.n, 20, 3, 1, local),
                            "fem_c5": bench_fem_run(384, 20, 3, 1, local),
                            "skeleton_f1": bench_skeleton(local),
-                           "lbm_sparse_f2": bench_lbm_sparse_run(args.n, 20, 3, local)}
+                           "lbm_sparse_f2": bench_lbm_sparse_run(args.n, 20, 3, local),
+                           "lbm_aa_f3": bench_lbm_aa_run(args.n, 20, 4, local)}
             out["cpu_baseline"] = cpu_baseline_cg(args.n)
             out["also"]["lbm_d3q19"]["cpu_baseline"] = cpu_baseline_lbm()
     elif args.workload in ("sparse", "fem"):

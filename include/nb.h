@@ -309,6 +309,14 @@ nb_status nb_lbm_init(nb_field *f, double rho0, const double u0[3]);
  * Halo: 5 populations per side (c_z = +1 up, c_z = -1 down). */
 nb_status nb_lbm_step(nb_field **fin, nb_field **fout, const nb_lbm_params *params,
                       int32_t nsteps, nb_occ occ);
+/* AA pattern (PAPER.md L451 stlbm's AA variant): the
+ * same physics on ONE population field updated in place (half of twoPop's
+ * memory).  Even steps collide locally and store reversed; odd steps pull
+ * from and push to the neighbours' opposite slots.  nsteps must be even
+ * (NB_EINVAL otherwise) so f returns to the natural layout; the result then
+ * equals nsteps twoPop steps bit for bit.  Dense grids, fused halos (one
+ * process with virtual partitions, or the peer transport). */
+nb_status nb_lbm_step_aa(nb_field *f, const nb_lbm_params *params, int32_t nsteps);
 /* rho (card 1) and u (card 3) fp32 fields from f */
 nb_status nb_lbm_macroscopic(const nb_field *f, nb_field *rho, nb_field *u);
 

@@ -118,6 +118,7 @@ SIGNATURES = {
     "nb_lbm_init": ([P, D, P], I32),
     "nb_lbm_step": ([PP, PP, P, I32, I32], I32),
     "nb_lbm_macroscopic": ([P, P, P], I32),
+    "nb_lbm_step_aa": ([P, P, I32], I32),
     "nb_fem27_apply": ([P, P, D, D], I32),
     "nb_fem27_rhs": ([P, D], I32),
     "nb_skeleton_plan": ([I32, I32, P, I32, P, I64, P], I32),
@@ -555,6 +556,14 @@ def nb_lbm_step(fin: Field, fout: Field, omega: float, nsteps: int = 1, u_lid: f
     if a.value == fin.handle.value:
         return fin, fout
     return fout, fin
+
+
+def nb_lbm_step_aa(f: Field, omega: float, nsteps: int = 2, u_lid: float = 0.05, rho_w: float = 1.0,
+                   bc: int = LBM_CAVITY):
+    """AA pattern: nsteps (even) steps in place on ONE population field."""
+    prm = LbmParams(omega, u_lid, rho_w, bc)
+    _check(lib().nb_lbm_step_aa(_h(f), C.byref(prm), int(nsteps)))
+    return f
 
 
 def nb_lbm_macroscopic(f: Field, rho: Field, u: Field):

@@ -464,6 +464,157 @@ extern "C" nb_status nb_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm
     return st;
 }
 
+// ===========================================================================
+// AA pattern (PAPER.md L451 stlbm's AA / twoPop / Swap
+// variants): ONE population buffer, updated in place — half the memory of
+// twoPop, so twice the domain per GPU.  With P_t = twoPop's post-collision
+// populations (natural layout A[x][i] = P_t(x, i) at even times):
+//   even step: f_i = A[x - c_i][i]            (wall: A[x][opp(i)] + lid_i)
+//              collide -> o;  A[x + c_i][opp(i)] = o_i
+//                             (wall: A[x][i] = o_i + lid_opp(i))
+//   odd step:  f_i = A[x][opp(i)];  collide -> o;  A[x][i] = o_i  (local)
+// Every (location, slot) is read and written by one cell only, so the
+// update is race free in place.  The gathered values are exactly twoPop's
+// and the collision is shared, so 2k AA steps equal 2k twoPop steps bit for
+// bit.  Partitions: the even step needs twoPop's halo (c_z = +1 populations
+// up, -1 down) and stores the populations leaving the slab straight into
+// the neighbour's own boundary plane (reversed slots); the odd step is
+// local.
+// ===========================================================================
+struct LbmAAArgs {
+    float *f[Q19];       // component base pointers (plane zl = -1, row 0)
+    float *up[Q19];      // upper neighbour's components at its plane 0 (14..18 written)
+    float *dn[Q19];      // lower neighbour's components at its top plane (9..13 written)
+    PGeo g;
+    float omega, ulid, rho_w;
+};
+
+template <bool EVEN, bool PERIODIC>
+__global__ void __launch_bounds__(128) k_lbm_aa(LbmAAArgs A) {
+    const int x = blockIdx.x * blockDim.x + threadIdx.x;
+    const int y = blockIdx.y;
+    const int zl = blockIdx.z;
+    const PGeo &g = A.g;
+    if (x >= g.nx) return;
+    const int gz = g.z0 + zl;
+    const int64_t row = (int64_t)y * g.pitch + x;
+    const int64_t cell = (int64_t)(zl + 1) * g.ps + row;
+    float f[Q19], o[Q19];
+    if (!EVEN) {  // local: reversed slots in, natural slots out
+#pragma unroll
+        for (int i = 0; i < Q19; ++i) f[i] = __ldg(A.f[OPPv(i)] + cell);
+        lbm_collide(f, A.omega, o);
+#pragma unroll
+        for (int i = 0; i < Q19; ++i) __stcs(A.f[i] + cell, o[i]);
+        return;
+    }
+    // even, interior cell (every source and target inside the slab): 19
+    // independent loads and 19 stores at uniform offsets
+    if (x > 0 && x < g.nx - 1 && y > 0 && y < g.ny - 1 && zl > 0 && zl < g.nzl - 1) {
+#pragma unroll
+        for (int i = 0; i < Q19; ++i)
+            f[i] = __ldg(A.f[i] + cell - (int64_t)CZv(i) * g.ps - (int64_t)CYv(i) * g.pitch - CXv(i));
+        lbm_collide(f, A.omega, o);
+#pragma unroll
+        for (int i = 0; i < Q19; ++i)
+            __stcs(A.f[OPPv(i)] + cell + (int64_t)CZv(i) * g.ps + (int64_t)CYv(i) * g.pitch + CXv(i), o[i]);
+        return;
+    }
+    // even: twoPop's pull gather from the natural layout
+#pragma unroll
+    for (int i = 0; i < Q19; ++i) {
+        int sx = x - CXv(i), sy = y - CYv(i);
+        const int szl = zl - CZv(i), sgz = gz - CZv(i);
+        if (PERIODIC) {
+            sx = sx < 0 ? sx + g.nx : (sx >= g.nx ? sx - g.nx : sx);
+            sy = sy < 0 ? sy + g.ny : (sy >= g.ny ? sy - g.ny : sy);
+            f[i] = __ldg(A.f[i] + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx);
+        } else {
+            const bool inside = sx >= 0 && sx < g.nx && sy >= 0 && sy < g.ny && sgz >= 0 && sgz < g.NZ;
+            float v = __ldg(inside ? A.f[i] + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx
+                                   : A.f[OPPv(i)] + cell);
+            if (CXv(i) != 0 && sy == g.ny && sx >= 0 && sx < g.nx && sgz >= 0 && sgz < g.NZ)
+                v = v + 6.0f * Wv(i) * A.rho_w * ((float)CXv(i) * A.ulid);
+            f[i] = v;
+        }
+    }
+    lbm_collide(f, A.omega, o);
+    // push o_i to x + c_i, reversed slot; a wall reflects it into this cell
+#pragma unroll
+    for (int i = 0; i < Q19; ++i) {
+        int tx = x + CXv(i), ty = y + CYv(i);
+        const int tzl = zl + CZv(i), tgz = gz + CZv(i);
+        const int j = OPPv(i);
+        if (!PERIODIC && !(tx >= 0 && tx < g.nx && ty >= 0 && ty < g.ny && tgz >= 0 && tgz < g.NZ)) {
+            float v = o[i];  // read next step as population j of this cell (twoPop's bounce-back)
+            if (CXv(j) != 0 && ty == g.ny && tx >= 0 && tx < g.nx && tgz >= 0 && tgz < g.NZ)
+                v = v + 6.0f * Wv(j) * A.rho_w * ((float)CXv(j) * A.ulid);
+            A.f[i][cell] = v;
+            continue;
+        }
+        if (PERIODIC) {
+            tx = tx < 0 ? tx + g.nx : (tx >= g.nx ? tx - g.nx : tx);
+            ty = ty < 0 ? ty + g.ny : (ty >= g.ny ? ty - g.ny : ty);
+        }
+        const int64_t trow = (int64_t)ty * g.pitch + tx;
+        if (tzl >= 0 && tzl < g.nzl)
+            A.f[j][(int64_t)(tzl + 1) * g.ps + trow] = o[i];
+        else if (tzl == g.nzl)
+            A.up[j][trow] = o[i];  // upper neighbour's plane 0
+        else
+            A.dn[j][trow] = o[i];  // lower neighbour's top plane
+    }
+}
+
+extern "C" nb_status nb_lbm_step_aa(nb_field *f, const nb_lbm_params *prm, int32_t nsteps) {
+    if (!f || !prm) NB_FAIL(NB_EINVAL, "nb_lbm_step_aa: NULL argument");
+    NB_TRY(lbm_check(f));
+    if (nsteps < 0 || (nsteps & 1)) NB_FAIL(NB_EINVAL, "nb_lbm_step_aa: nsteps must be even (got %d)", nsteps);
+    if (prm->bc != NB_LBM_CAVITY && prm->bc != NB_LBM_PERIODIC) NB_FAIL(NB_EINVAL, "bad bc");
+    nb_grid *g = f->g;
+    if (g->sparse) NB_FAIL(NB_EUNSUPPORTED, "AA pattern on element-sparse grids is not built");
+    if (nb_halo_on_stream(g)) NB_FAIL(NB_EUNSUPPORTED, "AA pattern: fused (in-process / peer) halos only");
+    cudaSetDevice(g->device);
+    const bool per = prm->bc == NB_LBM_PERIODIC;
+    for (int t = 0; t < nsteps; ++t) {
+        const bool even = !(t & 1);
+        if (even) NB_TRY(nb_halo_run(f, per, 9, 14, 14, 19, g->cs));  // twoPop's halo: the pull sources
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            LbmAAArgs A;
+            memset(&A, 0, sizeof(A));
+            for (int i = 0; i < Q19; ++i) A.f[i] = (float *)f->base[p] + (int64_t)i * lcs(f, p);
+            A.g = pgeo(f, p);
+            A.omega = (float)prm->omega;
+            A.ulid = (float)prm->u_lid;
+            A.rho_w = (float)prm->rho_w;
+            const int lo = lbm_lo(g, p, per), hi = lbm_hi(g, p, per);
+            if (even) {
+                if (hi >= 0) {
+                    if (!nb_reachable(f, hi)) NB_FAIL(NB_EUNSUPPORTED, "AA pattern: neighbour not addressable");
+                    for (int i = 14; i < 19; ++i)
+                        A.up[i] = (float *)f->base[hi] + (int64_t)i * lcs(f, hi) + (int64_t)1 * f->ps;
+                }
+                if (lo >= 0) {
+                    if (!nb_reachable(f, lo)) NB_FAIL(NB_EUNSUPPORTED, "AA pattern: neighbour not addressable");
+                    for (int i = 9; i < 14; ++i)
+                        A.dn[i] = (float *)f->base[lo] + (int64_t)i * lcs(f, lo) + (int64_t)g->parts[lo].nz() * f->ps;
+                }
+            }
+            dim3 blk(128), grd((g->nx + 127) / 128, g->ny, A.g.nzl);
+            LaunchScope ls(g, g->cs, "k_lbm_aa");
+            if (even)
+                per ? k_lbm_aa<true, true><<<grd, blk, 0, g->cs>>>(A) : k_lbm_aa<true, false><<<grd, blk, 0, g->cs>>>(A);
+            else
+                per ? k_lbm_aa<false, true><<<grd, blk, 0, g->cs>>>(A)
+                    : k_lbm_aa<false, false><<<grd, blk, 0, g->cs>>>(A);
+            NB_TRY(nb_launch_check("k_lbm_aa"));
+        }
+        // peer transport: the even step stored into the neighbours' planes
+        if (even && nb_is_peer(g)) NB_TRY(nb_peer_round(g, per, g->cs));
+    }
+    return NB_OK;
+}
+
 extern "C" nb_status nb_lbm_macroscopic(const nb_field *f, nb_field *rho, nb_field *u) {
     NB_TRY(lbm_check(f));
     if (!rho || !u) NB_FAIL(NB_EINVAL, "NULL field");

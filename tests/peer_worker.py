@@ -142,6 +142,21 @@ for bc in (nb.LBM_CAVITY, nb.LBM_PERIODIC):
 compare("lbm periodic 4 parts", (24, 20, 18), 2 * WORLD, lbm(nb.LBM_PERIODIC, nb.OCC_STANDARD, 6))
 
 
+def lbm_aa(bc):
+    def fn(g):
+        a = nb.Field(g, "f32", 19)
+        nb.nb_lbm_init(a, 1.0, (0.01, -0.02, 0.015) if bc == nb.LBM_PERIODIC else (0.0, 0.0, 0.0))
+        nb.nb_lbm_step_aa(a, 0.9, 6, bc=bc)
+        out = [a.download()]
+        a.close()
+        return out, []
+    return fn
+
+
+for bc in (nb.LBM_CAVITY, nb.LBM_PERIODIC):
+    compare(f"lbm aa bc{bc}", (24, 20, 18), WORLD, lbm_aa(bc))
+
+
 # ---- C4: element-sparse CG ---------------------------------------------------
 n = 30
 zz, yy, xx = np.meshgrid(*(np.arange(n) + 0.5 - n / 2,) * 3, indexing="ij")
