@@ -60,6 +60,8 @@ def lib():
         L.or_lbm_lattice.argtypes = [P, P, P]
         L.or_lbm_step.argtypes = [i32, i32, i32, i32, d, d, d, P, P]
         L.or_lbm_step_masked.argtypes = [i32, i32, i32, i32, d, d, d, P, P, P]
+        L.or_d2q9_lattice.argtypes = [P, P, P]
+        L.or_d2q9_step.argtypes = [i32, i32, i32, d, d, i32, i32, i32, P, P]
         L.or_lbm_macroscopic.argtypes = [i32, i32, i32, P, P, P]
         L.or_num_threads.restype = i32
         L.or_set_num_threads.argtypes = [i32]
@@ -237,3 +239,26 @@ def lbm_omega(nx: int, u_lid: float = 0.05, re: float = 100.0) -> float:
     omega = 1/(3 nu + 1/2)."""
     nu = u_lid * nx / re
     return 1.0 / (3.0 * nu + 0.5)
+
+
+# ---- D2Q9 Karman vortex street (SURVEY.md §8(f) f4; readings in DESIGN.md §3)
+D2Q9_CHANNEL, D2Q9_PERIODIC = 0, 1
+
+
+def d2q9_lattice():
+    c = np.zeros(18, dtype=np.int32)
+    w = np.zeros(9, dtype=np.float64)
+    o = np.zeros(9, dtype=np.int32)
+    lib().or_d2q9_lattice(c.ctypes.data_as(C.c_void_p), w.ctypes.data_as(C.c_void_p), o.ctypes.data_as(C.c_void_p))
+    return c.reshape(9, 2), w, o
+
+
+def d2q9_step(fin, omega, u_in, cyl, bc=D2Q9_CHANNEL):
+    """fin: [9][y][x] -> fout fp64 (computed in fp64 from the given values);
+    cyl = (cx, cy, r) integers (r < 0: no cylinder)."""
+    fin = _f64(fin)
+    _, ny, nx = fin.shape
+    fout = np.empty_like(fin)
+    cx, cy, r = (int(v) for v in cyl)
+    lib().or_d2q9_step(nx, ny, int(bc), float(omega), float(u_in), cx, cy, r, _ptr(fin), _ptr(fout))
+    return fout

@@ -559,3 +559,70 @@ void or_lbm_macroscopic(int nx, int ny, int nz, const double *f, double *rho, do
         u[2 * n + cell] = mz / r;
     }
 }
+
+/* ---- D2Q9 Karman vortex street (Table I,
+ * L398-L439: "2D Karman Vortex Street LBM"; the lattice and boundaries are
+ * not stated — readings in DESIGN.md §3):
+ *   velocities 0 (0,0); 1 (1,0) 2 (-1,0) 3 (0,1) 4 (0,-1); 5 (1,1) 6 (-1,-1)
+ *   7 (1,-1) 8 (-1,1); w = 4/9, 1/9, 1/36; c_s^2 = 1/3.
+ *   solid cylinder: (x-cx)^2 + (y-cy)^2 <= r^2 (integers; r < 0: none), half-way
+ *   bounce-back; solid cells get fout = 0.
+ *   bc 0 (channel): y periodic; a source left of x = 0 gives the inflow
+ *   equilibrium f_i^eq(1, (u_in, 0)); a source right of x = nx-1 is clamped
+ *   to column nx-1 (zero-gradient outflow).  bc 1: periodic box.
+ *   f_i(x) = fin_i(x - c_i) (pull), BGK collide with omega. */
+void or_d2q9_lattice(int *c /* 9*2 */, double *w, int *opp) {
+    static const int cc[18] = {0, 0, 1, 0, -1, 0, 0, 1, 0, -1, 1, 1, -1, -1, 1, -1, -1, 1};
+    static const int oo[9] = {0, 2, 1, 4, 3, 6, 5, 8, 7};
+    for (int i = 0; i < 18; ++i) c[i] = cc[i];
+    for (int i = 0; i < 9; ++i) {
+        opp[i] = oo[i];
+        w[i] = i == 0 ? 4.0 / 9.0 : (i < 5 ? 1.0 / 9.0 : 1.0 / 36.0);
+    }
+}
+
+static double d2q9_feq(const int *c, const double *w, int i, double rho, double ux, double uy) {
+    double cu = c[2 * i] * ux + c[2 * i + 1] * uy;
+    return w[i] * rho * (1.0 + 3.0 * cu + 4.5 * cu * cu - 1.5 * (ux * ux + uy * uy));
+}
+
+void or_d2q9_step(int nx, int ny, int bc, double omega, double u_in, int cx, int cy, int r, const double *fin,
+                  double *fout) {
+    int c[18], opp[9];
+    double w[9];
+    or_d2q9_lattice(c, w, opp);
+    int64_t n = (int64_t)nx * ny;
+    #pragma omp parallel for schedule(static)
+    for (int y = 0; y < ny; ++y)
+        for (int x = 0; x < nx; ++x) {
+            int64_t cell = (int64_t)y * nx + x;
+            int64_t dx = x - cx, dy = y - cy;
+            if (r >= 0 && dx * dx + dy * dy <= (int64_t)r * r) {
+                for (int q = 0; q < 9; ++q) fout[q * n + cell] = 0.0;
+                continue;
+            }
+            double f[9];
+            for (int q = 0; q < 9; ++q) {
+                int sx = x - c[2 * q], sy = ((y - c[2 * q + 1]) % ny + ny) % ny;
+                if (bc == 1) sx = (sx % nx + nx) % nx;
+                if (sx < 0) {
+                    f[q] = d2q9_feq(c, w, q, 1.0, u_in, 0.0);
+                    continue;
+                }
+                if (sx >= nx) sx = nx - 1;
+                int64_t sdx = sx - cx, sdy = sy - cy;
+                if (r >= 0 && sdx * sdx + sdy * sdy <= (int64_t)r * r)
+                    f[q] = fin[opp[q] * n + cell];
+                else
+                    f[q] = fin[q * n + (int64_t)sy * nx + sx];
+            }
+            double rho = 0.0, mx = 0.0, my = 0.0;
+            for (int q = 0; q < 9; ++q) {
+                rho += f[q];
+                mx += c[2 * q] * f[q];
+                my += c[2 * q + 1] * f[q];
+            }
+            double ux = mx / rho, uy = my / rho;
+            for (int q = 0; q < 9; ++q) fout[q * n + cell] = f[q] - omega * (f[q] - d2q9_feq(c, w, q, rho, ux, uy));
+        }
+}
