@@ -339,6 +339,39 @@ def bench_lbm_aa_run(n, steps, warmup, local):
             "hbm_gbs": gbs, "hbm_frac": gbs / hbm, "peak_kind": peak_kind, "clocks": clocks}
 
 
+def bench_karman(local, steps=20):
+    """the 2-D Kármán vortex street of PAPER.md Table I (D2Q9,
+    fp32, 72 B/cell/step) at the table's four domain sizes, 1 GPU."""
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    hbm, peak_kind = peaks()
+    rows = []
+    for nx, ny in ((4096, 1024), (8192, 2048), (16384, 4096), (32768, 8192)):
+        g = nb.Grid((nx, ny, 1), devices=[local])
+        stream = torch.cuda.ExternalStream(g.stream())
+        st = {"a": nb.Field(g, "f32", 9), "b": nb.Field(g, "f32", 9)}
+        u = 0.08
+        cyl = (nx // 5, ny // 2, ny // 10)
+        omega = 1.0 / (3 * u * 2 * cyl[2] / 150.0 + 0.5)  # Re 150 on the diameter
+        nb.nb_d2q9_init(st["a"], 1.0, u, 0.0)
+
+        def run(k):
+            st["a"], st["b"] = nb.nb_d2q9_step(st["a"], st["b"], omega, u, cyl, k)
+        run(4)
+        g.sync()
+        ms, _ = timed(1, stream, lambda: run(steps), local)
+        cells = nx * ny
+        gbs = 72 * cells * steps / (ms / 1e3) / 1e9
+        rows.append({"domain": f"{nx}x{ny}", "mlups": cells * steps / (ms / 1e3) / 1e6, "ms_per_step": ms / steps,
+                     "hbm_gbs": gbs, "hbm_frac": gbs / hbm})
+        st["a"].close(), st["b"].close()
+        g.close()
+    return {"workload": "2-D Karman vortex street, D2Q9 BGK fp32, cylinder r = ny/10 at (nx/5, ny/2), Re 150 "
+                        "(PAPER.md Table I sizes; SURVEY f4)", "rows": rows, "peak_kind": peak_kind,
+            "paper_context": "Table I reports 33-206 'LUPS' on 1 A100 (units garbled in the extraction; context only)"}
+
+
 LBM_SPARSE_BYTES_PER_CELL = 152 + 18 * 4  # 19 loads + 19 stores fp32, + the 18-direction source table
 
 
@@ -677,7 +710,8 @@ def main():
                            "fem_c5": bench_fem_run(384, 20, 3, 1, local),
                            "skeleton_f1": bench_skeleton(local),
                            "lbm_sparse_f2": bench_lbm_sparse_run(args.n, 20, 3, local),
-                           "lbm_aa_f3": bench_lbm_aa_run(args.n, 20, 4, local)}
+                           "lbm_aa_f3": bench_lbm_aa_run(args.n, 20, 4, local),
+                           "karman_f4": bench_karman(local)}
             out["cpu_baseline"] = cpu_baseline_cg(args.n)
             out["also"]["lbm_d3q19"]["cpu_baseline"] = cpu_baseline_lbm()
     elif args.workload in ("sparse", "fem"):

@@ -320,6 +320,21 @@ nb_status nb_lbm_step_aa(nb_field *f, const nb_lbm_params *params, int32_t nstep
 /* rho (card 1) and u (card 3) fp32 fields from f */
 nb_status nb_lbm_macroscopic(const nb_field *f, nb_field *rho, nb_field *u);
 
+/* ---- D2Q9 Karman vortex street (Table I; SURVEY.md
+ * §8(f) f4).  A dense grid of one plane (Nz = 1), fields fp32 of
+ * cardinality 9 (velocities 0; +-x, +-y; (1,1) (-1,-1) (1,-1) (-1,1)).
+ * Solid cylinder (x-cx)^2 + (y-cy)^2 <= r^2 (r < 0: none) with half-way
+ * bounce-back (solid cells hold 0); bc 0 = channel: y periodic, inflow
+ * equilibrium (rho 1, u = (u_in, 0)) for sources left of x = 0,
+ * zero-gradient outflow at x = Nx-1; bc 1 = periodic box.  Pull + BGK fused,
+ * twoPop (the pointers swap after each step). */
+typedef struct {
+    double omega, u_in;
+    int32_t cx, cy, r, bc;
+} nb_d2q9_params;
+nb_status nb_d2q9_init(nb_field *f, double rho0, double ux, double uy);
+nb_status nb_d2q9_step(nb_field **fin, nb_field **fout, const nb_d2q9_params *params, int32_t nsteps);
+
 /* ---- FEM: Q1 hex linear elasticity, 27-point ------- */
 /* y = K u (card 3 fp64), Dirichlet u = 0 on the z = 0 plane (identity
  * rows/cols).  Reads u's halo planes: call nb_halo_update(u) first. */

@@ -119,6 +119,8 @@ SIGNATURES = {
     "nb_lbm_step": ([PP, PP, P, I32, I32], I32),
     "nb_lbm_macroscopic": ([P, P, P], I32),
     "nb_lbm_step_aa": ([P, P, I32], I32),
+    "nb_d2q9_init": ([P, D, D, D], I32),
+    "nb_d2q9_step": ([PP, PP, P, I32], I32),
     "nb_fem27_apply": ([P, P, D, D], I32),
     "nb_fem27_rhs": ([P, D], I32),
     "nb_skeleton_plan": ([I32, I32, P, I32, P, I64, P], I32),
@@ -564,6 +566,27 @@ def nb_lbm_step_aa(f: Field, omega: float, nsteps: int = 2, u_lid: float = 0.05,
     prm = LbmParams(omega, u_lid, rho_w, bc)
     _check(lib().nb_lbm_step_aa(_h(f), C.byref(prm), int(nsteps)))
     return f
+
+
+class D2q9Params(C.Structure):
+    _fields_ = [("omega", C.c_double), ("u_in", C.c_double), ("cx", C.c_int32), ("cy", C.c_int32),
+                ("r", C.c_int32), ("bc", C.c_int32)]
+
+
+D2Q9_CHANNEL, D2Q9_PERIODIC = 0, 1
+
+
+def nb_d2q9_init(f: Field, rho0: float = 1.0, ux: float = 0.0, uy: float = 0.0):
+    _check(lib().nb_d2q9_init(_h(f), rho0, ux, uy))
+
+
+def nb_d2q9_step(fin: Field, fout: Field, omega: float, u_in: float, cyl=(0, 0, -1), nsteps: int = 1,
+                 bc: int = D2Q9_CHANNEL):
+    """Kármán vortex street step(s); returns (fin, fout) after the swaps."""
+    prm = D2q9Params(omega, u_in, int(cyl[0]), int(cyl[1]), int(cyl[2]), int(bc))
+    a, b = P(fin.handle.value), P(fout.handle.value)
+    _check(lib().nb_d2q9_step(C.byref(a), C.byref(b), C.byref(prm), int(nsteps)))
+    return (fin, fout) if a.value == fin.handle.value else (fout, fin)
 
 
 def nb_lbm_macroscopic(f: Field, rho: Field, u: Field):
