@@ -658,8 +658,10 @@ def reference_arm(args, world, rank):
     import synth
     n = args.n
     b = synth.poisson_poly_rhs((n, n, n))
-    w = min(args.warmup, 1)
-    k = min(args.steps, 5)
+    # W untimed warm-up iterations, then K timed ones (capped at 400: ~0.35 s
+    # each on 16 host cores at 512^3, so the arm stays within a few minutes)
+    w = max(args.warmup, 3)
+    k = max(1, min(args.steps, 400))
     t0 = time.perf_counter()
     oracle.cg(b, max_iter=w)
     t1 = time.perf_counter()
