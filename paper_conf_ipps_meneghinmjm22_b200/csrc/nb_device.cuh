@@ -14,6 +14,51 @@ __device__ __forceinline__ double warp_sum_canon(double v) {
     return v;
 }
 
+// N canonical warp sums at once (transposed butterfly).  Bitwise equal to N
+// calls of warp_sum_canon: at every butterfly level each lane adds its
+// partner's partial of the SAME value to its own (own + partner), exactly
+// the pairs warp_sum_canon adds; the first log2(M) levels (M = N rounded up
+// to a power of two) only split the values between the two lanes of a pair
+// instead of computing both halves in both, so N values cost M - 1 + 5 -
+// log2(M) shuffles and adds instead of 5 N.  On return, the total of value i
+// is in the lanes with warp_multi_index<N>(lane) == i.
+template <int N>
+struct WarpMulti {
+    static constexpr int M = N <= 1 ? 1 : N <= 2 ? 2 : N <= 4 ? 4 : N <= 8 ? 8 : N <= 16 ? 16 : 32;
+};
+
+template <int N>
+__device__ __forceinline__ double warp_sum_multi(const double (&v)[N], int lane) {
+    constexpr int M = WarpMulti<N>::M;
+    double w[M];
+#pragma unroll
+    for (int i = 0; i < M; ++i) w[i] = i < N ? v[i] : 0.0;
+    int o = 16;
+#pragma unroll
+    for (int h = M / 2; h >= 1; h >>= 1, o >>= 1) {
+        const bool up = (lane & o) != 0;
+#pragma unroll
+        for (int i = 0; i < h; ++i) {
+            const double send = up ? w[i] : w[i + h];
+            const double keep = up ? w[i + h] : w[i];
+            w[i] = __dadd_rn(keep, __shfl_xor_sync(0xffffffffu, send, o));
+        }
+    }
+#pragma unroll
+    for (; o > 0; o >>= 1) w[0] = __dadd_rn(w[0], __shfl_xor_sync(0xffffffffu, w[0], o));
+    return w[0];
+}
+
+template <int N>
+__device__ __forceinline__ int warp_multi_index(int lane) {
+    constexpr int M = WarpMulti<N>::M;
+    int idx = 0, o = 16;
+#pragma unroll
+    for (int h = M / 2; h >= 1; h >>= 1, o >>= 1)
+        if (lane & o) idx += h;
+    return idx;
+}
+
 // Canonical block tree over n values v[0..n) (stride `stride`) computed by a
 // block of RED_THREADS threads: thread t sums v[t], v[t+256], ... in order,
 // then a fixed halving tree.  Must be called by all RED_THREADS threads;

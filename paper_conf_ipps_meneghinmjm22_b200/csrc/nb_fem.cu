@@ -19,6 +19,7 @@
 #include <cstdlib>
 #include <algorithm>
 #include <cstring>
+#include <type_traits>
 #include <vector>
 
 #include "nb_device.cuh"
@@ -27,7 +28,31 @@
 
 __constant__ double c_ke[24 * 24];      // element stiffness, row-major
 __constant__ double c_S[27 * 9];        // interior stencil blocks [o][i][j]
+__constant__ double c_cv[8];            // its 8 canonical values (see fem_cv_class)
+
+// Structure of the assembled interior stencil (cubic lattice, isotropic
+// material): S[o][i][j] = fem_cv_sign * cv[fem_cv_class] for 8 canonical
+// values cv, whatever (E, nu).  Diagonal entries depend on the number n of
+// nonzero offset components and on whether o_i != 0; off-diagonal entries
+// exist only where o_i != 0 and o_j != 0 and carry the sign of o_i o_j.
+// fem_upload_constants checks this against the assembled values.
+__host__ __device__ constexpr int fem_oc(int o, int i) { return i == 0 ? o % 3 - 1 : i == 1 ? (o / 3) % 3 - 1 : o / 9 - 1; }
+__host__ __device__ constexpr int fem_on(int o) { return (fem_oc(o, 0) != 0) + (fem_oc(o, 1) != 0) + (fem_oc(o, 2) != 0); }
+__host__ __device__ constexpr int fem_cv_class(int o, int i, int j) {
+    return i == j ? (fem_on(o) == 0   ? 0
+                     : fem_on(o) == 1 ? (fem_oc(o, i) ? 1 : 2)
+                     : fem_on(o) == 2 ? (fem_oc(o, i) ? 3 : 4)
+                                      : 5)
+                  : (fem_oc(o, i) && fem_oc(o, j)) ? (fem_on(o) == 2 ? 6 : 7) : -1;
+}
+__host__ __device__ constexpr int fem_cv_sign(int o, int i, int j) { return i == j ? 1 : fem_oc(o, i) * fem_oc(o, j); }
 __constant__ const double *c_cls;       // surface-class stencils [FEM_NCLS][27 * 9] (device memory)
+// the surface classes of grids with nx, ny, nz >= 3 (those with all axis
+// states in {0, 1, 2} and a non-Dirichlet z state), copied into constant
+// memory: a warp whose nodes share a class reads each coefficient with one
+// uniform constant-cache load instead of an L1 round trip
+constexpr int FEM_NFC = 27;
+__constant__ double c_fcls[FEM_NFC][243];
 
 // Surface nodes: y_n = sum over the EXISTING elements around n of K_e u_e
 // (an element exists iff its 8 nodes are in the box).  Along one axis, a
@@ -43,6 +68,27 @@ __device__ __forceinline__ int fem_axis_state(int t, int n) {
     if (n == 1) return 3;
     return t == 0 ? 0 : (t == n - 1 ? 1 : 2);
 }
+
+// constant-memory slot of surface class k = ((xs * 4 + ys) * 4 + zs) * 2 + drop,
+// or -1 (degenerate axis, or not a surface class): zs = 2 (drop 0 / 1) or 1
+__host__ __device__ __forceinline__ int fem_cslot(int k) {
+    const int xs = k >> 5, ys = (k >> 3) & 3, zs = (k >> 1) & 3, d = k & 1;
+    if (xs == 3 || ys == 3) return -1;
+    const int zk = (zs == 2 && !d) ? 0 : (zs == 1 && !d) ? 1 : (zs == 2 && d) ? 2 : -1;
+    if (zk < 0) return -1;
+    return zk * 9 + xs * 3 + ys;
+}
+static int fem_cslot_host(int k) { return fem_cslot(k); }
+
+// coefficient sources of a surface-class stencil
+struct FemCConst {
+    int slot;
+    __device__ __forceinline__ double operator()(int i) const { return c_fcls[slot][i]; }
+};
+struct FemCGlob {
+    const double *__restrict__ p;
+    __device__ __forceinline__ double operator()(int i) const { return __ldg(p + i); }
+};
 
 std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v);
 nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down, cudaStream_t s);
@@ -106,15 +152,36 @@ static nb_status fem_upload_constants(double E, double nu) {
             for (int i = 0; i < 3; ++i)
                 for (int j = 0; j < 3; ++j) S[o * 9 + i * 3 + j] += ke[(3 * a + i) * 24 + 3 * b + j];
         }
-    // structural zeros of the assembled stencil: the coupling of components
-    // i != j at offset o vanishes unless o_i != 0 and o_j != 0 (odd symmetry
-    // of the tensor-product element); store them as exact zeros
-    for (int o = 0; o < 27; ++o) {
-        const int oc[3] = {o % 3 - 1, (o / 3) % 3 - 1, o / 9 - 1};
+    // structural zeros of the assembled stencil (the coupling of components
+    // i != j at offset o vanishes unless o_i != 0 and o_j != 0) are stored as
+    // exact zeros, and every other entry as +-cv[class] (fem_cv_class): the
+    // symmetric copies agree to rounding, which is checked here; storing them
+    // exactly equal lets the streaming kernel hold 8 values in registers
+    double cv[8];
+    bool have[8] = {};
+    for (int o = 0; o < 27; ++o)
         for (int i = 0; i < 3; ++i)
-            for (int j = 0; j < 3; ++j)
-                if (i != j && (oc[i] == 0 || oc[j] == 0)) S[o * 9 + i * 3 + j] = 0.0;
-    }
+            for (int j = 0; j < 3; ++j) {
+                const int k = fem_cv_class(o, i, j);
+                double &e = S[o * 9 + i * 3 + j];
+                if (k < 0) {
+                    e = 0.0;
+                    continue;
+                }
+                const double v = e * fem_cv_sign(o, i, j);
+                if (!have[k]) {
+                    cv[k] = v;
+                    have[k] = true;
+                } else if (std::fabs(v - cv[k]) > 1e-13 * std::fabs(cv[k])) {
+                    NB_FAIL(NB_EINVAL, "FEM stencil symmetry check failed (o=%d i=%d j=%d)", o, i, j);
+                }
+            }
+    for (int o = 0; o < 27; ++o)
+        for (int i = 0; i < 3; ++i)
+            for (int j = 0; j < 3; ++j) {
+                const int k = fem_cv_class(o, i, j);
+                if (k >= 0) S[o * 9 + i * 3 + j] = fem_cv_sign(o, i, j) > 0 ? cv[k] : -cv[k];
+            }
     std::vector<double> cls((size_t)FEM_NCLS * 243, 0.0);
     for (int k = 0; k < FEM_NCLS; ++k) {
         const int drop = k & 1, st[3] = {k >> 5, (k >> 3) & 3, (k >> 1) & 3};  // x, y, z axis states
@@ -135,23 +202,78 @@ static nb_status fem_upload_constants(double E, double nu) {
     if (!d_cls) NB_CUDA(cudaMalloc(&d_cls, sizeof(double) * cls.size()));
     NB_CUDA(cudaMemcpy(d_cls, cls.data(), sizeof(double) * cls.size(), cudaMemcpyHostToDevice));
     NB_CUDA(cudaMemcpyToSymbol(c_cls, &d_cls, sizeof(d_cls)));
+    {
+        std::vector<double> fc((size_t)FEM_NFC * 243, 0.0);
+        for (int k = 0; k < FEM_NCLS; ++k) {
+            const int sl = fem_cslot_host(k);
+            if (sl >= 0) std::copy(cls.begin() + (size_t)k * 243, cls.begin() + (size_t)(k + 1) * 243, fc.begin() + (size_t)sl * 243);
+        }
+        NB_CUDA(cudaMemcpyToSymbol(c_fcls, fc.data(), sizeof(double) * fc.size()));
+    }
     NB_CUDA(cudaMemcpyToSymbol(c_ke, ke, sizeof(ke)));
     NB_CUDA(cudaMemcpyToSymbol(c_S, S, sizeof(S)));
+    NB_CUDA(cudaMemcpyToSymbol(c_cv, cv, sizeof(cv)));
     g_fem_E = E;
     g_fem_nu = nu;
     return NB_OK;
 }
 
-// K u at node (x, y, zl) of the partition; u: component base pointer and
-// stride; returns the 3 components.  Dirichlet nodes (global z = 0) read 0.
-__device__ __forceinline__ void fem_node(const double *__restrict__ u, int64_t cs, const PGeo &g, int x, int y, int zl,
-                                         double out[3]) {
+// Operator input accessors: u(c, m, zl) = component c at element offset m,
+// which lies in local plane zl.
+struct FemUPlain {  // a stored field
+    const double *__restrict__ u;
+    int64_t cs;
+    __device__ __forceinline__ double operator()(int c, int64_t m, int) const { return u[c * cs + m]; }
+};
+// p_new of the fused CG phase A: fma(beta, p_old, r) inside the slab (the
+// arithmetic of k_fem_map), the exchanged p_new on the halo planes
+struct FemUCgA {
+    const double *__restrict__ r, *__restrict__ po, *__restrict__ pn;
+    int64_t cs;
+    double beta;
+    int nzl;
+    __device__ __forceinline__ double operator()(int c, int64_t m, int zl) const {
+        const int64_t i = c * cs + m;
+        return (zl < 0 || zl >= nzl) ? pn[i] : fma(beta, po[i], r[i]);
+    }
+};
+
+// surface path of fem_node: the class stencil C over the in-box positions
+template <class CF, class U>
+__device__ __forceinline__ void fem_node_surf(const CF &C, const U &u, const PGeo &g, int x, int y, int zl,
+                                              double &acc0, double &acc1, double &acc2) {
+    const int gz = g.z0 + zl;
+    const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+#pragma unroll
+    for (int o = 0; o < 27; ++o) {
+        const int ox = o % 3 - 1, oy = (o / 3) % 3 - 1, oz = o / 9 - 1;
+        const int mx = x + ox, my = y + oy, mz = gz + oz;
+        if (mx < 0 || my < 0 || mz < 0 || mx >= g.nx || my >= g.ny || mz >= g.NZ) continue;
+        const int64_t m = c0 + (int64_t)oz * g.ps + (int64_t)oy * g.pitch + ox;
+        const double u0 = u(0, m, zl + oz), u1 = u(1, m, zl + oz), u2 = u(2, m, zl + oz);
+        const int K = o * 9;
+        acc0 = fma(C(K + 0), u0, acc0);
+        acc0 = fma(C(K + 1), u1, acc0);
+        acc0 = fma(C(K + 2), u2, acc0);
+        acc1 = fma(C(K + 3), u0, acc1);
+        acc1 = fma(C(K + 4), u1, acc1);
+        acc1 = fma(C(K + 5), u2, acc1);
+        acc2 = fma(C(K + 6), u0, acc2);
+        acc2 = fma(C(K + 7), u1, acc2);
+        acc2 = fma(C(K + 8), u2, acc2);
+    }
+}
+
+// K u at node (x, y, zl) of the partition; returns the 3 components.
+// Dirichlet nodes (global z = 0) are identity rows.
+template <class U>
+__device__ __forceinline__ void fem_node(const U &u, const PGeo &g, int x, int y, int zl, double out[3]) {
     const int gz = g.z0 + zl;
     const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
     if (gz == 0) {  // identity row
-        out[0] = u[c0];
-        out[1] = u[cs + c0];
-        out[2] = u[2 * cs + c0];
+        out[0] = u(0, c0, zl);
+        out[1] = u(1, c0, zl);
+        out[2] = u(2, c0, zl);
         return;
     }
     double acc0 = 0.0, acc1 = 0.0, acc2 = 0.0;
@@ -161,7 +283,7 @@ __device__ __forceinline__ void fem_node(const double *__restrict__ u, int64_t c
         for (int o = 0; o < 27; ++o) {
             const int ox = o % 3 - 1, oy = (o / 3) % 3 - 1, oz = o / 9 - 1;
             const int64_t m = c0 + (int64_t)oz * g.ps + (int64_t)oy * g.pitch + ox;
-            const double u0 = u[m], u1 = u[cs + m], u2 = u[2 * cs + m];
+            const double u0 = u(0, m, zl + oz), u1 = u(1, m, zl + oz), u2 = u(2, m, zl + oz);
             const double *S = c_S + o * 9;
             // 153 structurally nonzero coefficients (diagonal blocks always;
             // i-j coupling only where o_i != 0 and o_j != 0): 306 flop/node
@@ -180,25 +302,11 @@ __device__ __forceinline__ void fem_node(const double *__restrict__ u, int64_t c
         // and are skipped; their coefficients are zero)
         const int cls = ((fem_axis_state(x, g.nx) * 4 + fem_axis_state(y, g.ny)) * 4 + fem_axis_state(gz, g.NZ)) * 2 +
                         (gz == 1 ? 1 : 0);
-        const double *__restrict__ C = c_cls + (size_t)cls * 243;
-#pragma unroll
-        for (int o = 0; o < 27; ++o) {
-            const int ox = o % 3 - 1, oy = (o / 3) % 3 - 1, oz = o / 9 - 1;
-            const int mx = x + ox, my = y + oy, mz = gz + oz;
-            if (mx < 0 || my < 0 || mz < 0 || mx >= g.nx || my >= g.ny || mz >= g.NZ) continue;
-            const int64_t m = c0 + (int64_t)oz * g.ps + (int64_t)oy * g.pitch + ox;
-            const double u0 = u[m], u1 = u[cs + m], u2 = u[2 * cs + m];
-            const double *K = C + o * 9;
-            acc0 = fma(__ldg(K + 0), u0, acc0);
-            acc0 = fma(__ldg(K + 1), u1, acc0);
-            acc0 = fma(__ldg(K + 2), u2, acc0);
-            acc1 = fma(__ldg(K + 3), u0, acc1);
-            acc1 = fma(__ldg(K + 4), u1, acc1);
-            acc1 = fma(__ldg(K + 5), u2, acc1);
-            acc2 = fma(__ldg(K + 6), u0, acc2);
-            acc2 = fma(__ldg(K + 7), u1, acc2);
-            acc2 = fma(__ldg(K + 8), u2, acc2);
-        }
+        const int sl = fem_cslot(cls);
+        if (sl >= 0)
+            fem_node_surf(FemCConst{sl}, u, g, x, y, zl, acc0, acc1, acc2);
+        else
+            fem_node_surf(FemCGlob{c_cls + (size_t)cls * 243}, u, g, x, y, zl, acc0, acc1, acc2);
     }
     out[0] = acc0;
     out[1] = acc1;
@@ -209,7 +317,9 @@ __device__ __forceinline__ void fem_node(const double *__restrict__ u, int64_t c
 // have z = 0 neighbours, handled by the surface (element) path above since
 // the interior test requires gz >= 2.
 
-enum { FEM_APPLY = 0, FEM_CG_Q = 1, FEM_CG_INIT = 2 };
+// FEM_CG_A: the fused CG phase A (p_new = r + beta p_old, deferred
+// x += alpha_prev p_old, q = K p_new, <p_new, q>) of the TMA schedule
+enum { FEM_APPLY = 0, FEM_CG_Q = 1, FEM_CG_INIT = 2, FEM_CG_A = 3 };
 
 struct FemArgs {
     const double *u;   // stencil input (x or p)
@@ -217,20 +327,31 @@ struct FemArgs {
     double *y;         // output (y / q / r)
     int64_t cs;
     const CgScal *sc;
+    // FEM_CG_A only: u = p_new is formed on the fly from r and p_old
+    const double *r, *po;
+    double *pn, *x;
 };
+
+template <int K>
+__device__ __forceinline__ void fem_node_k(const FemArgs &A, const PGeo &g, int x, int y, int zl, double out[3]) {
+    if constexpr (K == FEM_CG_A)
+        fem_node(FemUCgA{A.r, A.po, A.pn, A.cs, A.sc->beta, g.nzl}, g, x, y, zl, out);
+    else
+        fem_node(FemUPlain{A.u, A.cs}, g, x, y, zl, out);
+}
 
 // one CTA = one 32x8 tile of one plane (canonical dot tiles, per component)
 template <int K>
 __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_fem(FemArgs A, PGeo g, int zb, double *tp, int T) {
     __shared__ double sw[3][DOT_TY];
-    if (K == FEM_CG_Q && A.sc->status != 0) return;
+    if ((K == FEM_CG_Q || K == FEM_CG_A) && A.sc->status != 0) return;
     const int x = blockIdx.x * DOT_TX + threadIdx.x, y = blockIdx.y * DOT_TY + threadIdx.y;
     const int zl = zb + blockIdx.z;
     const bool valid = x < g.nx && y < g.ny;
     double prod[3] = {0.0, 0.0, 0.0};
     if (valid) {
         double o[3];
-        fem_node(A.u, A.cs, g, x, y, zl, o);
+        fem_node(FemUPlain{A.u, A.cs}, g, x, y, zl, o);
         const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
 #pragma unroll
         for (int c = 0; c < 3; ++c) {
@@ -328,7 +449,7 @@ __device__ __forceinline__ void fem_plane(const double *__restrict__ u, int64_t 
 template <int K, int ZC>
 __global__ void __launch_bounds__(DOT_TX *DOT_TY, 2) k_fem_z(FemArgs A, PGeo g, int zb0, int ze0, double *tp, int T) {
     __shared__ double sw[ZC][3][DOT_TY];
-    if (K == FEM_CG_Q && A.sc->status != 0) return;
+    if ((K == FEM_CG_Q || K == FEM_CG_A) && A.sc->status != 0) return;
     const int x = blockIdx.x * DOT_TX + threadIdx.x, y = blockIdx.y * DOT_TY + threadIdx.y;
     const int zs = zb0 + blockIdx.z * ZC, zend = min(zs + ZC, ze0);
     const bool valid = x < g.nx && y < g.ny;
@@ -366,7 +487,7 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY, 2) k_fem_z(FemArgs A, PGeo g, 
                 ccur[c] = cnext[c];
             }
         } else if (valid) {
-            fem_node(u, cs, g, x, y, zl, o);
+            fem_node(FemUPlain{u, cs}, g, x, y, zl, o);
             if (K == FEM_CG_Q) {
                 uc[0] = u[c0];
                 uc[1] = u[cs + c0];
@@ -424,6 +545,18 @@ constexpr int FNST = 4;
 #ifndef NB_FEM_NR
 #define NB_FEM_NR 2  // rows per thread of the TMA kernel
 #endif
+#ifndef NB_FEM_MINB
+#define NB_FEM_MINB 5  // CTAs per SM of the TMA kernel (apply / init / q)
+#endif
+#ifndef NB_FEM_NR_A
+#define NB_FEM_NR_A 1  // rows per thread of the fused CG phase A (8 warps per CTA: latency hiding)
+#endif
+#ifndef NB_FEM_NST_A
+#define NB_FEM_NST_A 2  // ring stages of the fused CG phase A (6 component boxes each)
+#endif
+#ifndef NB_FEM_MINB_A
+#define NB_FEM_MINB_A 3
+#endif
 
 struct __align__(128) FemStage {
     double c[3][FTPAD / 8];
@@ -467,14 +600,14 @@ __device__ __forceinline__ void fem_edge_col(int e, int nx, int ny, int &x, int 
 
 template <int K>
 __global__ void __launch_bounds__(128) k_fem_surface(FemArgs A, PGeo g, int zb, int ze, FemSurf S) {
-    if (K == FEM_CG_Q && A.sc->status != 0) return;
+    if ((K == FEM_CG_Q || K == FEM_CG_A) && A.sc->status != 0) return;
     const int nzl = ze - zb;
     const int64_t n1 = (int64_t)S.ncol_edge * nzl, n2 = (int64_t)S.nin * S.nzs;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n1 + n2; i += (int64_t)gridDim.x * blockDim.x) {
         int x, y, zl;
-        if (i < n1) {
-            fem_edge_col((int)(i / nzl), g.nx, g.ny, x, y);
-            zl = zb + (int)(i % nzl);
+        if (i < n1) {  // edge columns: consecutive threads walk along a face (coalesced on y faces)
+            fem_edge_col((int)(i % S.ncol_edge), g.nx, g.ny, x, y);
+            zl = zb + (int)(i / S.ncol_edge);
         } else {
             const int64_t k = i - n1;
             const int c = (int)(k % S.nin);
@@ -483,7 +616,7 @@ __global__ void __launch_bounds__(128) k_fem_surface(FemArgs A, PGeo g, int zb, 
             y = 1 + c / (g.nx - 2);
         }
         double o[3];
-        fem_node(A.u, A.cs, g, x, y, zl, o);
+        fem_node_k<K>(A, g, x, y, zl, o);
         const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
         A.y[c0] = o[0];
         A.y[A.cs + c0] = o[1];
@@ -499,16 +632,40 @@ __global__ void __launch_bounds__(128) k_fem_surface(FemArgs A, PGeo g, int zb, 
 // chain of fem_node's surface path (bitwise), at ~1/3 of its loads.
 constexpr int FZC = 4;
 
-__device__ __forceinline__ const double *fem_cls_ptr(int x, int y, int gz, const PGeo &g) {
+// class code of the output at (x, y, gz): constant slot >= 0, or -1 - class
+// (global table)
+constexpr int FEM_NOCLS = -1000000;
+__device__ __forceinline__ int fem_cls_code(int x, int y, int gz, const PGeo &g) {
     const int cls = ((fem_axis_state(x, g.nx) * 4 + fem_axis_state(y, g.ny)) * 4 + fem_axis_state(gz, g.NZ)) * 2 +
                     (gz == 1 ? 1 : 0);
-    return c_cls + (size_t)cls * 243;
+    const int sl = fem_cslot(cls);
+    return sl >= 0 ? sl : -1 - cls;
+}
+
+template <class CF>
+__device__ __forceinline__ void fem_face_blk(const CF &C, int K, double v0, double v1, double v2, double (&acc)[3]) {
+    acc[0] = fma(C(K + 0), v0, acc[0]);
+    acc[0] = fma(C(K + 1), v1, acc[0]);
+    acc[0] = fma(C(K + 2), v2, acc[0]);
+    acc[1] = fma(C(K + 3), v0, acc[1]);
+    acc[1] = fma(C(K + 4), v1, acc[1]);
+    acc[1] = fma(C(K + 5), v2, acc[1]);
+    acc[2] = fma(C(K + 6), v0, acc[2]);
+    acc[2] = fma(C(K + 7), v1, acc[2]);
+    acc[2] = fma(C(K + 8), v2, acc[2]);
+}
+
+__device__ __forceinline__ void fem_face_apply(int code, int K, double v0, double v1, double v2, double (&acc)[3]) {
+    if (code >= 0)
+        fem_face_blk(FemCConst{code}, K, v0, v1, v2, acc);
+    else if (code != FEM_NOCLS)
+        fem_face_blk(FemCGlob{c_cls + (size_t)(-1 - code) * 243}, K, v0, v1, v2, acc);
 }
 
 // contributions of one plane k (global gz_k) to output accumulators whose
-// class stencils are CA (output k-1, offset oz = +1), CB (k, 0), CC (k+1, -1)
-__device__ __forceinline__ void fem_face_plane(const double *__restrict__ u, int64_t cs, const PGeo &g, int x, int y,
-                                               int k, const double *CA, const double *CB, const double *CC,
+// class codes are CA (output k-1, offset oz = +1), CB (k, 0), CC (k+1, -1)
+template <class U>
+__device__ __forceinline__ void fem_face_plane(const U &u, const PGeo &g, int x, int y, int k, int CA, int CB, int CC,
                                                double (&aA)[3], double (&aB)[3], double (&aC)[3], double (&cen)[3]) {
     const int64_t base = (int64_t)(k + 1) * g.ps + (int64_t)y * g.pitch + x;
     aC[0] = aC[1] = aC[2] = 0.0;
@@ -518,30 +675,15 @@ __device__ __forceinline__ void fem_face_plane(const double *__restrict__ u, int
         const int mx = x + ox, my = y + oy;
         if (mx < 0 || my < 0 || mx >= g.nx || my >= g.ny) continue;
         const int64_t m = base + (int64_t)oy * g.pitch + ox;
-        const double v0 = u[m], v1 = u[cs + m], v2 = u[2 * cs + m];
+        const double v0 = u(0, m, k), v1 = u(1, m, k), v2 = u(2, m, k);
         if (q == 4) {
             cen[0] = v0;
             cen[1] = v1;
             cen[2] = v2;
         }
-        const double *K;
-#define FEM_FACE_APPLY(CP, OZ, ACC)                                       \
-    if (CP) {                                                             \
-        K = CP + ((OZ + 1) * 9 + q) * 9;                                  \
-        ACC[0] = fma(__ldg(K + 0), v0, ACC[0]);                           \
-        ACC[0] = fma(__ldg(K + 1), v1, ACC[0]);                           \
-        ACC[0] = fma(__ldg(K + 2), v2, ACC[0]);                           \
-        ACC[1] = fma(__ldg(K + 3), v0, ACC[1]);                           \
-        ACC[1] = fma(__ldg(K + 4), v1, ACC[1]);                           \
-        ACC[1] = fma(__ldg(K + 5), v2, ACC[1]);                           \
-        ACC[2] = fma(__ldg(K + 6), v0, ACC[2]);                           \
-        ACC[2] = fma(__ldg(K + 7), v1, ACC[2]);                           \
-        ACC[2] = fma(__ldg(K + 8), v2, ACC[2]);                           \
-    }
-        FEM_FACE_APPLY(CA, 1, aA)
-        FEM_FACE_APPLY(CB, 0, aB)
-        FEM_FACE_APPLY(CC, -1, aC)
-#undef FEM_FACE_APPLY
+        fem_face_apply(CA, (18 + q) * 9, v0, v1, v2, aA);
+        fem_face_apply(CB, (9 + q) * 9, v0, v1, v2, aB);
+        fem_face_apply(CC, q * 9, v0, v1, v2, aC);
     }
 }
 
@@ -557,15 +699,9 @@ __device__ __forceinline__ void fem_face_col(int c, const PGeo &g, int &x, int &
     }
 }
 
-template <int K>
-__global__ void __launch_bounds__(64) k_fem_faces(FemArgs A, PGeo g, int zb, int ze, int ncols) {
-    if (K == FEM_CG_Q && A.sc->status != 0) return;
-    const int c = blockIdx.x * blockDim.x + threadIdx.x;
-    if (c >= ncols) return;
-    int x, y;
-    fem_face_col(c, g, x, y);
-    const int zs = zb + blockIdx.y * FZC, zend = min(zs + FZC, ze);
-    const double *__restrict__ u = A.u;
+template <class U>
+__device__ __forceinline__ void fem_face_col_run(const U &u, const FemArgs &A, const PGeo &g, int x, int y, int zs,
+                                                 int zend) {
     double aA[3] = {0.0, 0.0, 0.0}, aB[3] = {0.0, 0.0, 0.0}, aC[3], cen[3], cprev[3] = {0.0, 0.0, 0.0};
     // planes zs-1 .. zend (in-box only: the halo planes beyond the global box are skipped)
     for (int k = zs - 1; k <= zend; ++k) {
@@ -576,10 +712,10 @@ __global__ void __launch_bounds__(64) k_fem_faces(FemArgs A, PGeo g, int zb, int
             aC[0] = aC[1] = aC[2] = 0.0;
             cen[0] = cen[1] = cen[2] = 0.0;
         } else {
-            const double *CA = inA && g.z0 + oA > 0 ? fem_cls_ptr(x, y, g.z0 + oA, g) : nullptr;
-            const double *CB = inB && g.z0 + oB > 0 ? fem_cls_ptr(x, y, g.z0 + oB, g) : nullptr;
-            const double *CC = inC && g.z0 + oC > 0 ? fem_cls_ptr(x, y, g.z0 + oC, g) : nullptr;
-            fem_face_plane(u, A.cs, g, x, y, k, CA, CB, CC, aA, aB, aC, cen);
+            const int CA = inA && g.z0 + oA > 0 ? fem_cls_code(x, y, g.z0 + oA, g) : FEM_NOCLS;
+            const int CB = inB && g.z0 + oB > 0 ? fem_cls_code(x, y, g.z0 + oB, g) : FEM_NOCLS;
+            const int CC = inC && g.z0 + oC > 0 ? fem_cls_code(x, y, g.z0 + oC, g) : FEM_NOCLS;
+            fem_face_plane(u, g, x, y, k, CA, CB, CC, aA, aB, aC, cen);
         }
         if (inA) {  // output k-1 complete
             const int64_t c0 = (int64_t)(oA + 1) * g.ps + (int64_t)y * g.pitch + x;
@@ -596,6 +732,20 @@ __global__ void __launch_bounds__(64) k_fem_faces(FemArgs A, PGeo g, int zb, int
     }
 }
 
+template <int K>
+__global__ void __launch_bounds__(64) k_fem_faces(FemArgs A, PGeo g, int zb, int ze, int ncols) {
+    if ((K == FEM_CG_Q || K == FEM_CG_A) && A.sc->status != 0) return;
+    const int c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c >= ncols) return;
+    int x, y;
+    fem_face_col(c, g, x, y);
+    const int zs = zb + blockIdx.y * FZC, zend = min(zs + FZC, ze);
+    if constexpr (K == FEM_CG_A)
+        fem_face_col_run(FemUCgA{A.r, A.po, A.pn, A.cs, A.sc->beta, g.nzl}, A, g, x, y, zs, zend);
+    else
+        fem_face_col_run(FemUPlain{A.u, A.cs}, A, g, x, y, zs, zend);
+}
+
 // ---- streaming interior kernel ---------------------------------------------
 // Thread = NR adjacent rows of one x column.  Coefficient-major order: for
 // each in-plane position q and each oz block, every coefficient (held in a
@@ -603,196 +753,317 @@ __global__ void __launch_bounds__(64) k_fem_faces(FemArgs A, PGeo g, int zb, int
 // load serves NR nodes.  Per output, positions still arrive in (oy, ox)
 // order with the oz blocks in plane order: fem_node's interior FMA chain
 // (bitwise).
-template <int O, int NR>
-__device__ __forceinline__ void fem_blkN(const double (&v)[NR][3], double (&acc)[NR][3]) {
-    constexpr int ox = O % 3 - 1, oy = (O / 3) % 3 - 1, oz = O / 9 - 1;
-    const double *S = c_S + O * 9;
+template <int O, int I, int J, int NR>
+__device__ __forceinline__ void fem_cvfma(const double (&cv)[8], const double (&v)[NR][3], double (&acc)[NR][3]) {
+    constexpr int k = fem_cv_class(O, I, J);
+    if constexpr (k >= 0) {
+        const double c = fem_cv_sign(O, I, J) > 0 ? cv[k] : -cv[k];
 #pragma unroll
-    for (int r = 0; r < NR; ++r) acc[r][0] = fma(S[0], v[r][0], acc[r][0]);
-    if (ox != 0 && oy != 0)
-#pragma unroll
-        for (int r = 0; r < NR; ++r) acc[r][0] = fma(S[1], v[r][1], acc[r][0]);
-    if (ox != 0 && oz != 0)
-#pragma unroll
-        for (int r = 0; r < NR; ++r) acc[r][0] = fma(S[2], v[r][2], acc[r][0]);
-    if (oy != 0 && ox != 0)
-#pragma unroll
-        for (int r = 0; r < NR; ++r) acc[r][1] = fma(S[3], v[r][0], acc[r][1]);
-#pragma unroll
-    for (int r = 0; r < NR; ++r) acc[r][1] = fma(S[4], v[r][1], acc[r][1]);
-    if (oy != 0 && oz != 0)
-#pragma unroll
-        for (int r = 0; r < NR; ++r) acc[r][1] = fma(S[5], v[r][2], acc[r][1]);
-    if (oz != 0 && ox != 0)
-#pragma unroll
-        for (int r = 0; r < NR; ++r) acc[r][2] = fma(S[6], v[r][0], acc[r][2]);
-    if (oz != 0 && oy != 0)
-#pragma unroll
-        for (int r = 0; r < NR; ++r) acc[r][2] = fma(S[7], v[r][1], acc[r][2]);
-#pragma unroll
-    for (int r = 0; r < NR; ++r) acc[r][2] = fma(S[8], v[r][2], acc[r][2]);
+        for (int r = 0; r < NR; ++r) acc[r][I] = fma(c, v[r][J], acc[r][I]);
+    }
 }
 
-template <int NR>
-struct FemAcc {
-    double a[NR][3], b[NR][3], c[NR][3];  // outputs k-1 (oz=+1), k (oz=0), k+1 (oz=-1)
-};
+template <int O, int NR>
+__device__ __forceinline__ void fem_blkN(const double (&cv)[8], const double (&v)[NR][3], double (&acc)[NR][3]) {
+    fem_cvfma<O, 0, 0, NR>(cv, v, acc);
+    fem_cvfma<O, 0, 1, NR>(cv, v, acc);
+    fem_cvfma<O, 0, 2, NR>(cv, v, acc);
+    fem_cvfma<O, 1, 0, NR>(cv, v, acc);
+    fem_cvfma<O, 1, 1, NR>(cv, v, acc);
+    fem_cvfma<O, 1, 2, NR>(cv, v, acc);
+    fem_cvfma<O, 2, 0, NR>(cv, v, acc);
+    fem_cvfma<O, 2, 1, NR>(cv, v, acc);
+    fem_cvfma<O, 2, 2, NR>(cv, v, acc);
+}
 
-template <int NR, int Q>
-__device__ __forceinline__ void fem_q(const FemStage &st, int sidx, bool da, bool db, FemAcc<NR> &A,
-                                      double (&cen)[NR][3]) {
+// in-plane position Q of the current plane (stage S: 3 component tiles)
+// applied to the three outputs it touches: aA (output k-1, oz = +1), aB
+// (output k, oz = 0), aC (output k+1, oz = -1); DA / DB: outputs k-1 / k exist
+template <int NR, int Q, bool DA, bool DB>
+__device__ __forceinline__ void fem_q(const double (&cv)[8], const double *S, int sidx, double (&aA)[NR][3],
+                                      double (&aB)[NR][3], double (&aC)[NR][3]) {
     constexpr int off = (Q / 3 - 1) * FBX + (Q % 3 - 1);
     double v[NR][3];
 #pragma unroll
     for (int r = 0; r < NR; ++r)
 #pragma unroll
-        for (int c = 0; c < 3; ++c) v[r][c] = st.c[c][sidx + r * FBX + off];
-    if (Q == 4)
+        for (int c = 0; c < 3; ++c) v[r][c] = S[c * (FTPAD / 8) + sidx + r * FBX + off];
+    if constexpr (DA) fem_blkN<18 + Q, NR>(cv, v, aA);
+    if constexpr (DB) fem_blkN<9 + Q, NR>(cv, v, aB);
+    fem_blkN<Q, NR>(cv, v, aC);
+}
+
+// tensor maps: u = the stencil input (x / p), or r for FEM_CG_A, which also
+// streams p_old (po) and, on halo planes, the exchanged p_new (pn)
+struct FemMaps {
+    CUtensorMap u[3], po[3], pn[3];
+};
+
+template <int K>
+struct FemTmaCfg {
+    static constexpr bool CGA = K == FEM_CG_A;
+    static constexpr int NR = CGA ? NB_FEM_NR_A : NB_FEM_NR;  // rows per thread
+    static constexpr int NT = DOT_TX * (DOT_TY / NR);         // threads per CTA
+    static constexpr int NST = CGA ? NB_FEM_NST_A : FNST;     // ring stages
+    static constexpr int SD = (CGA ? 6 : 3) * (FTPAD / 8);    // doubles per stage
+    static constexpr int SMEM = (NST * SD + (CGA ? 6 * (FTPAD / 8) : 0)) * 8;  // dynamic shared memory bytes
+    static constexpr int MINB = CGA ? NB_FEM_MINB_A : NB_FEM_MINB;  // CTAs per SM
+};
+
+// Per-CTA state of the streaming kernel.  A thread owns NR rows of one x
+// column of a 32 x 8 tile and marches ZC output planes; plane j of the
+// chunk (local plane zs - 1 + j) arrives in ring stage j % NST.
+template <int K, int ZC>
+struct FemTma {
+    using Cfg = FemTmaCfg<K>;
+    static constexpr bool CGA = Cfg::CGA;
+    static constexpr int NR = Cfg::NR, NT = Cfg::NT, NST = Cfg::NST, SD = Cfg::SD, CP = FTPAD / 8;
+    const FemMaps &M;
+    const FemArgs &A;
+    const PGeo &g;
+    double *fsm;
+    uint64_t *bar;
+    double (*sw)[3][DOT_TY];  // [output parity][component][tile row]
+    double *tp;
+    int T;
+    int tid, lane, x0, y0, x, ya, zs, zend, nplanes, fa, fb, sidx;
+    bool xin, xint, anyfast, dox;
+    double beta, ap;
+    double cv[8];  // canonical stencil values (registers for the whole kernel)
+
+    __device__ __forceinline__ bool halo(int zl) const { return zl < 0 || zl >= g.nzl; }
+
+    __device__ __forceinline__ void issue(int j) const {  // plane zs-1+j -> stage j % NST
+        double *S = fsm + (j % NST) * SD;
+        uint64_t *b = &bar[j % NST];
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        const int zl = zs - 1 + j, tz = zl + 1;
+        if (CGA && !halo(zl)) {
+            mbar_expect_tx(b, 6 * FBX * FBY * 8);
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                tma_load_3d(S + c * CP, &M.u[c], b, x0 - 2, y0 - 1, tz);
+                tma_load_3d(S + (3 + c) * CP, &M.po[c], b, x0 - 2, y0 - 1, tz);
+            }
+        } else {
+            mbar_expect_tx(b, 3 * FBX * FBY * 8);
+#pragma unroll
+            for (int c = 0; c < 3; ++c) tma_load_3d(S + c * CP, CGA ? &M.pn[c] : &M.u[c], b, x0 - 2, y0 - 1, tz);
+        }
+    }
+
+    // plane j: its contributions to outputs j-2 (aA), j-1 (aB), j (aC, fresh);
+    // output j-2 is then complete (centre values cP, of plane j-1); cC
+    // receives this plane's centre values.
+    // FEM_CG_A: the raw stage (r, p_old) is first turned into p_new in one of
+    // two p_new buffers (double-buffered: one barrier per plane), so the
+    // stage is refilled while the FMAs run; the deferred x update is applied
+    // after the FMAs, which hide the latency of the x loads.
+    template <bool DA, bool DB>
+    __device__ __forceinline__ void step(int j, double (&aA)[NR][3], double (&aB)[NR][3], double (&aC)[NR][3],
+                                         const double (&cP)[NR][3], double (&cC)[NR][3]) const {
+        const int zin = zs - 1 + j;  // local plane held by this stage
+        const bool own = zin >= zs && zin < zend;
+        const double *S = fsm + (j % NST) * SD;  // stencil input tiles of this plane
+        double xo[NR][3], pc[NR][3];               // CGA: x and p_old of the own centres
+        if constexpr (CGA) {
+            if (own && dox) {
+#pragma unroll
+                for (int r = 0; r < NR; ++r) {
+                    const int64_t c0 = (int64_t)(zin + 1) * g.ps + (int64_t)(ya + r) * g.pitch + x;
+                    const bool v = xin && ya + r < g.ny;
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) xo[r][c] = v ? __ldcs(A.x + c * A.cs + c0) : 0.0;
+                }
+            }
+            mbar_wait(&bar[j % NST], (uint32_t)((j / NST) & 1));
+            double *P = fsm + NST * SD + (j & 1) * 3 * CP;  // p_new tiles (double-buffered)
+            if (!halo(zin)) {  // CTA-uniform
+                for (int c = 0; c < 3; ++c)
+                    for (int e = tid; e < FBX * FBY; e += NT) P[c * CP + e] = fma(beta, S[(3 + c) * CP + e], S[c * CP + e]);
+#pragma unroll
+                for (int r = 0; r < NR; ++r)
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) pc[r][c] = S[(3 + c) * CP + sidx + r * FBX];
+            } else {
+                for (int e = tid; e < 3 * CP; e += NT) P[e] = S[e];
+            }
+            __syncthreads();  // p_new tiles ready; the raw stage is free; step j-1's dot rows are in sw
+            if (tid == 0 && j + NST < nplanes) issue(j + NST);
+            if (j >= 3) flush(zs + j - 3, tp, T);
+            S = P;
+        } else {
+            if (j >= 3) flush(zs + j - 3, tp, T);  // the previous step's output (barrier passed)
+            mbar_wait(&bar[j % NST], (uint32_t)((j / NST) & 1));
+        }
+        if (anyfast) {
+#pragma unroll
+            for (int r = 0; r < NR; ++r) aC[r][0] = aC[r][1] = aC[r][2] = 0.0;
+            fem_q<NR, 0, DA, DB>(cv, S, sidx, aA, aB, aC);
+            fem_q<NR, 1, DA, DB>(cv, S, sidx, aA, aB, aC);
+            fem_q<NR, 2, DA, DB>(cv, S, sidx, aA, aB, aC);
+            fem_q<NR, 3, DA, DB>(cv, S, sidx, aA, aB, aC);
+            fem_q<NR, 4, DA, DB>(cv, S, sidx, aA, aB, aC);
+            fem_q<NR, 5, DA, DB>(cv, S, sidx, aA, aB, aC);
+            fem_q<NR, 6, DA, DB>(cv, S, sidx, aA, aB, aC);
+            fem_q<NR, 7, DA, DB>(cv, S, sidx, aA, aB, aC);
+            fem_q<NR, 8, DA, DB>(cv, S, sidx, aA, aB, aC);
+        }
 #pragma unroll
         for (int r = 0; r < NR; ++r)
 #pragma unroll
-            for (int c = 0; c < 3; ++c) cen[r][c] = v[r][c];
-    if (da) fem_blkN<18 + Q, NR>(v, A.a);
-    if (db) fem_blkN<9 + Q, NR>(v, A.b);
-    fem_blkN<Q, NR>(v, A.c);
-}
-
-template <int K, int ZC, int NR>
-__global__ void __launch_bounds__(DOT_TX *(DOT_TY / NR), 8 / NR + 1)
-    k_fem_tma(const __grid_constant__ CUtensorMap m0, const __grid_constant__ CUtensorMap m1,
-              const __grid_constant__ CUtensorMap m2, FemArgs A, PGeo g, int zb0, int ze0, double *tp, int T) {
-    constexpr int NT = DOT_TX * (DOT_TY / NR);
-    __shared__ FemStage st[FNST];
-    __shared__ __align__(8) uint64_t bar[FNST];
-    __shared__ double sw[ZC][3][DOT_TY];
-    if (K == FEM_CG_Q && A.sc->status != 0) return;
-    const int tid = threadIdx.y * DOT_TX + threadIdx.x;
-    const int x0 = blockIdx.x * DOT_TX, y0 = blockIdx.y * DOT_TY;
-    const int x = x0 + threadIdx.x, ya = y0 + threadIdx.y * NR;  // rows ya .. ya+NR-1
-    const int zs = zb0 + blockIdx.z * ZC, zend = min(zs + ZC, ze0);
-    const int nplanes = zend - zs + 2;  // planes zs-1 .. zend
-    const bool xin = x < g.nx, xint = x >= 1 && x <= g.nx - 2;
-    const int fa = max(zs, 2 - g.z0), fb = min(zend, g.NZ - 1 - g.z0);  // fast outputs [fa, fb)
-    bool anyfast = false;
+            for (int c = 0; c < 3; ++c) cC[r][c] = S[c * CP + sidx + r * FBX];
+        if constexpr (CGA) {
+            if (own) {  // own plane: store p_new and the deferred x += alpha_prev p_old
 #pragma unroll
-    for (int r = 0; r < NR; ++r) anyfast |= xint && ya + r >= 1 && ya + r <= g.ny - 2;
-    const int sidx = (threadIdx.y * NR + 1) * FBX + threadIdx.x + 2;
-    auto issue = [&](int j) {  // plane zs-1+j -> stage j % FNST
-        FemStage &S = st[j % FNST];
-        uint64_t *b = &bar[j % FNST];
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        mbar_expect_tx(b, 3 * FBX * FBY * 8);
-        const int tz = zs + j;  // tensor z of plane zl = zl + 1
-        tma_load_3d(&S.c[0][0], &m0, b, x0 - 2, y0 - 1, tz);
-        tma_load_3d(&S.c[1][0], &m1, b, x0 - 2, y0 - 1, tz);
-        tma_load_3d(&S.c[2][0], &m2, b, x0 - 2, y0 - 1, tz);
-    };
-    if (tid == 0) {
-        for (int k = 0; k < FNST; ++k) mbar_init(&bar[k], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    if (tid == 0)
-        for (int j = 0; j < min(FNST, nplanes); ++j) issue(j);
-    FemAcc<NR> acc;
-    double csave[NR][3];
+                for (int r = 0; r < NR; ++r) {
+                    const int y = ya + r;
+                    if (xin && y < g.ny) {
+                        const int64_t c0 = (int64_t)(zin + 1) * g.ps + (int64_t)y * g.pitch + x;
 #pragma unroll
-    for (int r = 0; r < NR; ++r)
-#pragma unroll
-        for (int c = 0; c < 3; ++c) acc.a[r][c] = acc.b[r][c] = csave[r][c] = 0.0;
-#pragma unroll 3
-    for (int j = 0; j < nplanes; ++j) {
-        mbar_wait(&bar[j % FNST], (uint32_t)((j / FNST) & 1));
-        const FemStage &S = st[j % FNST];
-        const bool da = j >= 2, db = j >= 1;  // CTA-uniform
-        double cen[NR][3];
-        if (anyfast) {
-#pragma unroll
-            for (int r = 0; r < NR; ++r) acc.c[r][0] = acc.c[r][1] = acc.c[r][2] = 0.0;
-            fem_q<NR, 0>(S, sidx, da, db, acc, cen);
-            fem_q<NR, 1>(S, sidx, da, db, acc, cen);
-            fem_q<NR, 2>(S, sidx, da, db, acc, cen);
-            fem_q<NR, 3>(S, sidx, da, db, acc, cen);
-            fem_q<NR, 4>(S, sidx, da, db, acc, cen);
-            fem_q<NR, 5>(S, sidx, da, db, acc, cen);
-            fem_q<NR, 6>(S, sidx, da, db, acc, cen);
-            fem_q<NR, 7>(S, sidx, da, db, acc, cen);
-            fem_q<NR, 8>(S, sidx, da, db, acc, cen);
-        }
-        if (da) {  // output plane zl = zs + j - 2 is complete
-            const int zl = zs + j - 2;
-            const bool zfast = zl >= fa && zl < fb;
-#pragma unroll
-            for (int r = 0; r < NR; ++r) {
-                const int y = ya + r;
-                const bool valid = xin && y < g.ny;
-                const bool fast = zfast && xint && y >= 1 && y <= g.ny - 2;
-                const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
-                double o[3] = {acc.a[r][0], acc.a[r][1], acc.a[r][2]};
-                double uc[3] = {csave[r][0], csave[r][1], csave[r][2]};
-                if (valid && !fast) {  // computed by k_fem_surface
-#pragma unroll
-                    for (int c = 0; c < 3; ++c) {
-                        o[c] = A.y[c * A.cs + c0];
-                        if (K == FEM_CG_Q) uc[c] = A.u[c * A.cs + c0];
-                    }
-                }
-                double prod[3] = {0.0, 0.0, 0.0};
-                if (valid) {
-#pragma unroll
-                    for (int c = 0; c < 3; ++c) {
-                        const int64_t i = c * A.cs + c0;
-                        if (K == FEM_CG_INIT) {
-                            const double rr = __dsub_rn(A.b[i], o[c]);
-                            A.y[i] = rr;
-                            prod[c] = __dmul_rn(rr, rr);
-                        } else {
-                            if (fast) A.y[i] = o[c];
-                            if (K == FEM_CG_Q) prod[c] = __dmul_rn(uc[c], o[c]);
+                        for (int c = 0; c < 3; ++c) {
+                            __stcs(A.pn + c * A.cs + c0, cC[r][c]);
+                            if (dox) __stcs(A.x + c * A.cs + c0, fma(ap, pc[r][c], xo[r][c]));
                         }
-                    }
-                }
-                if (K != FEM_APPLY) {
-#pragma unroll
-                    for (int c = 0; c < 3; ++c) {
-                        const double v = warp_sum_canon(prod[c]);
-                        if (threadIdx.x == 0) sw[zl - zs][c][threadIdx.y * NR + r] = v;
                     }
                 }
             }
         }
-        if (anyfast) {
-#pragma unroll
-            for (int r = 0; r < NR; ++r)
-#pragma unroll
-                for (int c = 0; c < 3; ++c) {
-                    acc.a[r][c] = acc.b[r][c];
-                    acc.b[r][c] = acc.c[r][c];
-                    csave[r][c] = cen[r][c];
-                }
+        if constexpr (DA) epilogue(j - 2 + zs, aA, cP);
+        if constexpr (!CGA) {
+            __syncthreads();  // stage j % NST is free
+            if (tid == 0 && j + NST < nplanes) issue(j + NST);
         }
-        __syncthreads();  // stage j % FNST is free
-        if (tid == 0 && j + FNST < nplanes) issue(j + FNST);
     }
-    if (K == FEM_APPLY) return;
-    for (int t = tid; t < 3 * (zend - zs); t += NT) {
-        const int zi = t / 3, c = t % 3;
-        double s = sw[zi][c][0];
+
+    // tile partials of output zl (its 8 row sums, after a barrier): rows in
+    // increasing y; sw is double-buffered by output parity
+    __device__ __forceinline__ void flush(int zl, double *tp, int T) const {
+        if (K != FEM_APPLY && tid < 3) {
+            const double(*w)[DOT_TY] = sw[(zl - zs) & 1];
+            double s = w[tid][0];
 #pragma unroll
-        for (int w = 1; w < DOT_TY; ++w) s = __dadd_rn(s, sw[zi][c][w]);
-        tp[((int64_t)c * g.NZ + g.z0 + zs + zi) * T + blockIdx.y * gridDim.x + blockIdx.x] = s;
+            for (int k = 1; k < DOT_TY; ++k) s = __dadd_rn(s, w[tid][k]);
+            tp[((int64_t)tid * g.NZ + g.z0 + zl) * T + blockIdx.y * gridDim.x + blockIdx.x] = s;
+        }
     }
+
+    // output plane zl: store (or, for surface nodes, read back), dot partials
+    __device__ __forceinline__ void epilogue(int zl, const double (&o3)[NR][3], const double (&cen)[NR][3]) const {
+        const bool zfast = zl >= fa && zl < fb;
+        double prod[NR * 3];
+#pragma unroll
+        for (int r = 0; r < NR; ++r) {
+            const int y = ya + r;
+            const bool valid = xin && y < g.ny;
+            const bool fast = zfast && xint && y >= 1 && y <= g.ny - 2;
+            const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+            double o[3] = {o3[r][0], o3[r][1], o3[r][2]};
+            if (valid && !fast)  // computed by k_fem_surface / k_fem_faces
+#pragma unroll
+                for (int c = 0; c < 3; ++c) o[c] = A.y[c * A.cs + c0];
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                double pr = 0.0;
+                if (valid) {
+                    const int64_t i = c * A.cs + c0;
+                    if (K == FEM_CG_INIT) {
+                        const double rr = __dsub_rn(A.b[i], o[c]);
+                        A.y[i] = rr;
+                        pr = __dmul_rn(rr, rr);
+                    } else {
+                        if (fast) __stcs(A.y + i, o[c]);
+                        if (K == FEM_CG_Q || CGA) pr = __dmul_rn(cen[r][c], o[c]);
+                    }
+                }
+                prod[r * 3 + c] = pr;
+            }
+        }
+        if (K != FEM_APPLY) {
+            constexpr int NV = NR * 3, M2 = WarpMulti<NV>::M;
+            const double v = warp_sum_multi<NV>(prod, lane);
+            const int i = warp_multi_index<NV>(lane);
+            if (i < NV && (lane & (32 / M2 - 1)) == 0) sw[(zl - zs) & 1][i % 3][threadIdx.y * NR + i / 3] = v;
+        }
+    }
+};
+
+template <int K, int ZC, int NR>
+__global__ void __launch_bounds__(FemTmaCfg<K>::NT, FemTmaCfg<K>::MINB)
+    k_fem_tma(const __grid_constant__ FemMaps M, FemArgs A, PGeo g, int zb0, int ze0, double *tp, int T) {
+    using Cfg = FemTmaCfg<K>;
+    static_assert(Cfg::NR == NR, "rows per thread");
+    extern __shared__ __align__(128) double fsm[];
+    __shared__ __align__(8) uint64_t bar[Cfg::NST];
+    __shared__ double sw[2][3][DOT_TY];
+    if ((K == FEM_CG_Q || K == FEM_CG_A) && A.sc->status != 0) return;
+    FemTma<K, ZC> t{M, A, g, fsm, bar, sw, tp, T};
+    t.tid = threadIdx.y * DOT_TX + threadIdx.x;
+    t.lane = threadIdx.x;
+    t.x0 = blockIdx.x * DOT_TX;
+    t.y0 = blockIdx.y * DOT_TY;
+    t.x = t.x0 + threadIdx.x;
+    t.ya = t.y0 + threadIdx.y * NR;  // rows ya .. ya+NR-1
+    t.zs = zb0 + blockIdx.z * ZC;
+    t.zend = min(t.zs + ZC, ze0);
+    t.nplanes = t.zend - t.zs + 2;  // planes zs-1 .. zend
+    t.xin = t.x < g.nx;
+    t.xint = t.x >= 1 && t.x <= g.nx - 2;
+    t.fa = max(t.zs, 2 - g.z0);  // fast outputs [fa, fb)
+    t.fb = min(t.zend, g.NZ - 1 - g.z0);
+    t.anyfast = false;
+#pragma unroll
+    for (int r = 0; r < NR; ++r) t.anyfast |= t.xint && t.ya + r >= 1 && t.ya + r <= g.ny - 2;
+    t.sidx = (threadIdx.y * NR + 1) * FBX + threadIdx.x + 2;
+    t.beta = t.ap = 0.0;
+    t.dox = false;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) t.cv[k] = c_cv[k];
+    if constexpr (K == FEM_CG_A) {
+        t.beta = A.sc->beta;
+        t.ap = A.sc->alpha_prev;
+        t.dox = A.sc->pending != 0;
+    }
+    if (t.tid == 0) {
+        for (int k = 0; k < Cfg::NST; ++k) mbar_init(&bar[k], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (t.tid == 0)
+        for (int j = 0; j < min(Cfg::NST, t.nplanes); ++j) t.issue(j);
+    // accumulators and centre values rotate through three register sets:
+    // the plane loop is unrolled by three so the rotation is free
+    double a0[NR][3], a1[NR][3], a2[NR][3], c0[NR][3], c1[NR][3], c2[NR][3];
+#pragma unroll
+    for (int r = 0; r < NR; ++r)
+#pragma unroll
+        for (int c = 0; c < 3; ++c) a0[r][c] = a1[r][c] = a2[r][c] = c0[r][c] = c1[r][c] = c2[r][c] = 0.0;
+    // plane 0 starts output 0 (a1 after rotation), plane 1 ...
+    t.template step<false, false>(0, a2, a0, a1, c2, c0);
+    t.template step<false, true>(1, a0, a1, a2, c0, c1);
+    int j = 2;
+#pragma unroll 1
+    for (; j + 2 < t.nplanes; j += 3) {
+        t.template step<true, true>(j, a1, a2, a0, c1, c2);
+        t.template step<true, true>(j + 1, a2, a0, a1, c2, c0);
+        t.template step<true, true>(j + 2, a0, a1, a2, c0, c1);
+    }
+    if (j < t.nplanes) t.template step<true, true>(j, a1, a2, a0, c1, c2);
+    if (j + 1 < t.nplanes) t.template step<true, true>(j + 1, a2, a0, a1, c2, c0);
+    if constexpr (K == FEM_CG_A) __syncthreads();
+    t.flush(t.zend - 1, tp, T);  // the last output (after a barrier)
 }
 
-// CG map: x += alpha_prev p_old (pending), p = r + beta p_old (in place)
-__global__ void k_fem_map(double *x, double *p, const double *r, int64_t n, const CgScal *sc) {
+// CG map: x += alpha_prev p_old (pending, when dox), p_new = r + beta p_old
+__global__ void k_fem_map(double *x, double *pn, const double *po, const double *r, int64_t n, const CgScal *sc,
+                          int dox) {
     if (sc->status != 0) return;
     const double beta = sc->beta, ap = sc->alpha_prev;
-    const int pending = sc->pending;
+    const int pending = dox && sc->pending;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const double po = p[i];
-        if (pending) x[i] = fma(ap, po, x[i]);
-        p[i] = fma(beta, po, r[i]);
+        const double pv = po[i];
+        if (pending) x[i] = fma(ap, pv, x[i]);
+        pn[i] = fma(beta, pv, r[i]);
     }
 }
 
@@ -834,16 +1105,25 @@ template <int K>
 static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int zb, int ze, const char *name) {
     if (ze <= zb) return NB_OK;
     A.cs = fcs(f, p);
-    LaunchScope ls(g, g->cs, name);
     const PGeo geo = pgeo(f, p);
     const char *variant = getenv("NB_FEM_KERNEL");  // "plain" | "zmarch" | default TMA
     if (variant && !strcmp(variant, "plain")) {  // the one-node-per-thread reference kernel
         dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, ze - zb);
+        LaunchScope ls(g, g->cs, name);
         k_fem<K><<<grd, blk, 0, g->cs>>>(A, geo, zb, g->tp, g->T);
     } else if (!variant && nb_tma_enabled()) {
-        constexpr int ZC = 32, NR = NB_FEM_NR;
-        CUtensorMap m[3];
-        for (int c = 0; c < 3; ++c) NB_TRY(tmap_for(A.u + c * A.cs, geo, 0, &m[c]));
+        using Cfg = FemTmaCfg<K>;
+        constexpr int ZC = 32, NR = Cfg::NR;
+        FemMaps M;
+        if constexpr (K == FEM_CG_A) {
+            for (int c = 0; c < 3; ++c) {
+                NB_TRY(tmap_for(A.r + c * A.cs, geo, 0, &M.u[c]));
+                NB_TRY(tmap_for(A.po + c * A.cs, geo, 0, &M.po[c]));
+                NB_TRY(tmap_for(A.pn + c * A.cs, geo, 0, &M.pn[c]));
+            }
+        } else {
+            for (int c = 0; c < 3; ++c) NB_TRY(tmap_for(A.u + c * A.cs, geo, 0, &M.u[c]));
+        }
         // surface nodes first (converged), then the streaming interior
         FemSurf S{};
         const int nx = geo.nx, ny = geo.ny;
@@ -854,21 +1134,37 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
             if (gz < 2 || gz > geo.NZ - 2) S.zlist[S.nzs++] = zl;
         }
         {
-            const int ncols = S.ncol_edge;
-            S.ncol_edge = 0;  // face columns: z-marching kernel; z-surface planes: per node
-            const int64_t n = (int64_t)S.nin * S.nzs;
+            // face columns: one thread per node, consecutive threads along a
+            // face (default; 0.19 ms at 384^3 for all surface nodes), or the
+            // z-marching column kernel (NB_FEM_FACES=col; 0.22 ms); z-surface
+            // planes: one thread per node
+            const bool faces_node = !(getenv("NB_FEM_FACES") && !strcmp(getenv("NB_FEM_FACES"), "col"));
+            const int ncols = faces_node ? 0 : S.ncol_edge;
+            if (!faces_node) S.ncol_edge = 0;
+            const int64_t n = (int64_t)S.ncol_edge * (ze - zb) + (int64_t)S.nin * S.nzs;
             if (n > 0) {
                 const int blocks = (int)std::min<int64_t>((n + 127) / 128, 1 << 30);
+                LaunchScope ls(g, g->cs, "k_fem_surface");
                 k_fem_surface<K><<<blocks, 128, 0, g->cs>>>(A, geo, zb, ze, S);
             }
-            dim3 fg((ncols + 63) / 64, (ze - zb + FZC - 1) / FZC);
-            k_fem_faces<K><<<fg, 64, 0, g->cs>>>(A, geo, zb, ze, ncols);
+            if (ncols > 0) {
+                dim3 fg((ncols + 63) / 64, (ze - zb + FZC - 1) / FZC);
+                LaunchScope ls(g, g->cs, "k_fem_faces");
+                k_fem_faces<K><<<fg, 64, 0, g->cs>>>(A, geo, zb, ze, ncols);
+            }
+        }
+        static unsigned attr_set = 0;  // per device: dynamic shared memory above 48 KB
+        if (g->device < 32 && !(attr_set & (1u << g->device))) {
+            NB_CUDA(cudaFuncSetAttribute(k_fem_tma<K, ZC, NR>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
+            attr_set |= 1u << g->device;
         }
         dim3 blk(DOT_TX, DOT_TY / NR), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
-        k_fem_tma<K, ZC, NR><<<grd, blk, 0, g->cs>>>(m[0], m[1], m[2], A, geo, zb, ze, g->tp, g->T);
+        LaunchScope ls(g, g->cs, name);
+        k_fem_tma<K, ZC, NR><<<grd, blk, Cfg::SMEM, g->cs>>>(M, A, geo, zb, ze, g->tp, g->T);
     } else {
         constexpr int ZC = 16;
         dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
+        LaunchScope ls(g, g->cs, name);
         k_fem_z<K, ZC><<<grd, blk, 0, g->cs>>>(A, geo, zb, ze, g->tp, g->T);
     }
     return nb_launch_check(name);
@@ -943,34 +1239,62 @@ nb_status nb_fem_cg_init(nb_cg *cg) {
     return nb_reduce_finalize(g, 3, FIN_CG_INIT, cg->sc, 0);
 }
 
+// fused schedule (default): boundary planes of p_new -> halo(p_new) ->
+// surface nodes + fused phase A -> alpha -> r -= alpha q, <r,r> -> beta
+// (216 B/node/iter).  With NB_FEM_KERNEL (reference kernels) or NB_FEM_3PASS:
+// map -> halo(p_new) -> q = K p_new -> alpha -> r -> beta (240 B/node/iter).
+// Both compute the same values in the same order (bitwise).
+static bool fem_fused() { return !getenv("NB_FEM_KERNEL") && !getenv("NB_FEM_3PASS") && nb_tma_enabled(); }
+
 nb_status nb_fem_cg_hooks(nb_cg *cg, int parity) {
-    (void)parity;
     nb_grid *g = cg->g;
-    nb_field *p_ = cg->p[0];
+    nb_field *pn = cg->p[parity], *po = cg->p[parity ^ 1];
+    const bool fused = fem_fused();
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
-        // own planes of all 3 components (halo planes excluded)
+        const NbPart &q = g->parts[p];
+        std::vector<int> planes;  // own planes to map first
+        if (fused) {
+            if (q.lo >= 0) planes.push_back(0);
+            if (q.hi >= 0 && q.nz() > 1) planes.push_back(q.nz() - 1);
+        }
         for (int c = 0; c < 3; ++c) {
-            int64_t off = (int64_t)c * fcs(p_, p) + p_->ps, n = (int64_t)g->parts[p].nz() * p_->ps;
-            LaunchScope ls(g, g->cs, "k_fem_map");
-            k_fem_map<<<148 * 8, 256, 0, g->cs>>>((double *)cg->x->base[p] + off, (double *)p_->base[p] + off,
-                                                  (const double *)cg->r->base[p] + off, n, cg->sc);
-            NB_TRY(nb_launch_check("k_fem_map"));
+            auto run = [&](int z0, int nz, int dox) -> nb_status {
+                const int64_t off = (int64_t)c * fcs(pn, p) + (int64_t)(z0 + 1) * pn->ps, n = (int64_t)nz * pn->ps;
+                LaunchScope ls(g, g->cs, "k_fem_map");
+                k_fem_map<<<fused ? 148 : 148 * 8, 256, 0, g->cs>>>(
+                    (double *)cg->x->base[p] + off, (double *)pn->base[p] + off, (const double *)po->base[p] + off,
+                    (const double *)cg->r->base[p] + off, n, cg->sc, dox);
+                return nb_launch_check("k_fem_map");
+            };
+            if (fused) {
+                for (int z : planes) NB_TRY(run(z, 1, 0));
+            } else {
+                NB_TRY(run(0, q.nz(), 1));
+            }
         }
     }
-    NB_TRY(nb_halo_exchange_planes(p_, 0, 3, true, true, g->cs));
+    NB_TRY(nb_halo_exchange_planes(pn, 0, 3, true, true, g->cs));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         FemArgs A{};
-        A.u = (const double *)p_->base[p];
         A.y = (double *)cg->q->base[p];
         A.sc = cg->sc;
-        NB_TRY(fem_launch<FEM_CG_Q>(g, p, A, p_, 0, g->parts[p].nz(), "k_fem_cg_q"));
+        if (fused) {
+            A.r = (const double *)cg->r->base[p];
+            A.po = (const double *)po->base[p];
+            A.pn = (double *)pn->base[p];
+            A.x = (double *)cg->x->base[p];
+            NB_TRY(fem_launch<FEM_CG_A>(g, p, A, pn, 0, g->parts[p].nz(), "k_fem_cg_a"));
+        } else {
+            A.u = (const double *)pn->base[p];
+            NB_TRY(fem_launch<FEM_CG_Q>(g, p, A, pn, 0, g->parts[p].nz(), "k_fem_cg_q"));
+        }
     }
     NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
-        PGeo geo = pgeo(p_, p);
+        PGeo geo = pgeo(pn, p);
         dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, geo.nzl);
         LaunchScope ls(g, g->cs, "k_fem_r");
-        k_fem_r<<<grd, blk, 0, g->cs>>>((double *)cg->r->base[p], (const double *)cg->q->base[p], fcs(p_, p), geo, 0,
+        k_fem_r<<<grd, blk, 0, g->cs>>>((double *)cg->r->base[p], (const double *)cg->q->base[p], fcs(pn, p), geo, 0,
                                         cg->sc, g->tp, g->T);
         NB_TRY(nb_launch_check("k_fem_r"));
     }

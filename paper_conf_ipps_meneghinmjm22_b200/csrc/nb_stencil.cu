@@ -821,8 +821,8 @@ extern "C" nb_status nb_cg_finish(nb_cg *cg, nb_cg_result *res) {
             for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
                 int64_t n = (int64_t)cg->x->bytes[p] / 8;
                 LaunchScope ls(g, g->cs, "k_cg_flush");
-                // dense Poisson CG ping-pongs p by parity; FEM keeps one p buffer
-                const double *p1 = (const double *)cg->p[cg->prm.op == NB_OP_FEM27 ? 0 : 1]->base[p];
+                // p ping-pongs by iteration parity (dense Poisson and FEM)
+                const double *p1 = (const double *)cg->p[1]->base[p];
                 k_cg_flush<<<148 * 4, 256, 0, g->cs>>>((double *)cg->x->base[p], (const double *)cg->p[0]->base[p], p1,
                                                       n, cg->sc);
                 NB_TRY(nb_launch_check("k_cg_flush"));

@@ -116,11 +116,17 @@ def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
     CG dots."""
     u = synth.uniform(dims, card=3, seed=9)
     out = {}
-    for variant in (None, "zmarch", "plain"):
-        if variant:
-            monkeypatch.setenv("NB_FEM_KERNEL", variant)
-        else:
-            monkeypatch.delenv("NB_FEM_KERNEL", raising=False)
+    # kernel variants (NB_FEM_KERNEL), the z-marching face-column kernel
+    # (NB_FEM_FACES=col) and the 3-pass CG schedule (NB_FEM_3PASS: map ->
+    # q = K p -> r) against the default fused schedule
+    envs = {None: {}, "zmarch": {"NB_FEM_KERNEL": "zmarch"}, "plain": {"NB_FEM_KERNEL": "plain"},
+            "faces_col": {"NB_FEM_FACES": "col"}, "3pass": {"NB_FEM_3PASS": "1"}}
+    for variant, env in envs.items():
+        for k in ("NB_FEM_KERNEL", "NB_FEM_FACES", "NB_FEM_3PASS"):
+            if k in env:
+                monkeypatch.setenv(k, env[k])
+            else:
+                monkeypatch.delenv(k, raising=False)
         with grid(dims, parts) as g:
             fu, fy = nb.Field(g, card=3), nb.Field(g, card=3)
             fu.upload(u)
@@ -134,6 +140,6 @@ def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
             out[variant] = (y, fx.download(), r.rr)
             for f in (fu, fy, fb, fx):
                 f.close()
-    for v in ("zmarch", "plain"):
+    for v in ("zmarch", "plain", "faces_col", "3pass"):
         assert np.array_equal(out[None][0], out[v][0]), v
         assert np.array_equal(out[None][1], out[v][1]) and out[None][2] == out[v][2], v
