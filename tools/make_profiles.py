@@ -60,7 +60,9 @@ tp = os.path.join(OUT, "ncu_traffic.json")
 if os.path.exists(tp):
     traffic = json.load(open(tp))
 for rep in sorted(os.listdir(GO)):
-    if not (rep.startswith(f"prof_{R}_") and rep.endswith(".ncu-rep")):
+    if not (rep.startswith(f"prof_{R}_") and rep.endswith((".ncu-rep", ".raw.csv"))):
+        continue
+    if rep.endswith(".ncu-rep") and os.path.exists(os.path.join(GO, rep.replace(".ncu-rep", ".raw.csv"))):
         continue
     res = ncu_summary.load(os.path.join(GO, rep))
     out = [f"# ncu --set full --clock-control none summary of {rep} ({R})",
@@ -76,7 +78,7 @@ for rep in sorted(os.listdir(GO)):
         per[lab].append(d.get("dram_read", 0) + d.get("dram_write", 0))
     for lab, v in per.items():
         traffic[lab] = max(v)  # the steady-state launch (x update active) is the largest
-    open(os.path.join(OUT, rep.replace(".ncu-rep", ".txt")), "w").write("\n".join(out) + "\n")
+    open(os.path.join(OUT, rep.replace(".ncu-rep", ".txt").replace(".raw.csv", ".txt")), "w").write("\n".join(out) + "\n")
 json.dump(traffic, open(tp, "w"), indent=1, sort_keys=True)
 print("\n".join(lines))
 print(json.dumps(traffic, indent=1))

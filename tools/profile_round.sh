@@ -16,8 +16,14 @@ timeout 900 ncu --set full --clock-control none --import-source on \
     -k regex:"k_lbm_d3q19" -s 1 -c 2 -o gpurun_out/prof_${R}_lbm \
     python tools/prof_driver.py 512 lbm > gpurun_out/prof_${R}_lbm.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on \
-    -k regex:"^k_sp$|k_fem_tma|k_fem_faces|k_fem_surface|k_fem_map|k_fem_r$" -c 20 -o gpurun_out/prof_${R}_sparse_fem \
+    -k regex:"^k_sp$|k_fem_tma|k_fem_faces|k_fem_surface|k_fem_map|k_fem_r$" -c 24 -o gpurun_out/prof_${R}_sparse_fem \
     python tools/prof_driver.py 512 sparse,fem > gpurun_out/prof_${R}_sparse_fem.log 2>&1
+# raw pages exported here; the reports themselves stay on the box (gpurun
+# copies back at most 64 MiB)
+for rep in gpurun_out/prof_${R}_*.ncu-rep; do
+    ncu -i "$rep" --page raw --csv > "${rep%.ncu-rep}.raw.csv" 2>/dev/null
+    rm -f "$rep"
+done
 echo profile done
 # kernel timelines (CUPTI via torch.profiler): 1 partition and 4 virtual partitions
 timeout 300 python tools/timeline.py 512 8 cg 1 --out gpurun_out/timeline_${R}_cg_p1.json > /dev/null 2>&1
