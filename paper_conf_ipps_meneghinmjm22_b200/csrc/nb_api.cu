@@ -500,6 +500,7 @@ extern "C" nb_status nb_grid_destroy(nb_grid *g) {
         nb_field_destroy(kv.second);
     }
     g->scratch.clear();
+    if (g->c1_exec) cudaGraphExecDestroy(g->c1_exec);
     nb_peer_grid_teardown(g);  // collective (peer transport)
     for (auto &r : g->prof) {
         cudaEventDestroy(r.a);

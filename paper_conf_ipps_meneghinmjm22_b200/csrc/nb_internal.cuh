@@ -162,6 +162,13 @@ struct nb_grid {
     int64_t launches = 0;
     // internal scratch fields (ping-pong partners), not counted in nfields
     std::map<std::pair<int, int>, struct nb_field *> scratch;
+    // CUDA graph of the last nb_map_stencil_reduce loop (key: x, y base
+    // pointers, a, iterations, OCC mode) and its kernel count
+    cudaGraphExec_t c1_exec = nullptr;
+    const void *c1_x = nullptr, *c1_y = nullptr;
+    double c1_a = 0.0;
+    int c1_iters = -1, c1_occ = -1;
+    int64_t c1_launches = 0;
     // element-sparse
     std::vector<NbSparsePart> sp;
     std::vector<int64_t> plane_count;  // [nz] active per global plane

@@ -303,7 +303,7 @@ __device__ __forceinline__ void msr_fast_body(const MsrArgs &A, const PGeo &g, i
 
 template <int MODE, bool DOMAP>
 __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_msr_fast(MsrArgs A, PGeo g, int zb, int ze, double *tp, int T,
-                                                           int tiles_y) {
+                                                           int tiles_y, int zc) {
     __shared__ double sU[2][DOT_TY + 2][DOT_TX + 2];
     __shared__ double sw[ZC][ZW];
     if (A.sc && A.sc->status != 0) return;
@@ -315,7 +315,7 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_msr_fast(MsrArgs A, PGeo g, 
         pending = A.sc->pending;
     }
     const bool dox = MODE == MSR_CG && DOMAP && pending;
-    const int zs = zb + blockIdx.z * ZC, zend = min(ze, zs + ZC);
+    const int zs = zb + blockIdx.z * zc, zend = min(ze, zs + zc);  // zc <= ZC planes per CTA
     const int x0 = blockIdx.x * DOT_TX, y0 = blockIdx.y * DOT_TY;
     // all own cells and all ring cells inside the domain (CTA-uniform)
     const bool full = x0 >= 1 && y0 >= 1 && x0 + DOT_TX + 1 <= g.nx && y0 + DOT_TY + 1 <= g.ny;
@@ -468,10 +468,14 @@ static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int
     if (MODE == MSR_C1 && RC && ZR_MAP == 1 && nb_tma_enabled() && (int64_t)g->nx * g->ny * g->nz >= (1 << 21))
         return nb_c1_tma(g, pgeo(f, p), A.w, A.v, A.u, A.out, A.m, DM, zb, ze);
     if (RC && ZR_MAP == 1 && !getenv("NB_GENERIC_MSR")) {
-        // specialised recompute kernel (same arithmetic and dot order)
-        dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
+        // specialised recompute kernel (same arithmetic and dot order); planes
+        // per CTA halved while the launch has fewer than two CTAs per SM (the
+        // dot partials are per plane and tile: results do not depend on it)
+        int zc = ZC;
+        while (zc > 2 && (int64_t)g->tiles_x * g->tiles_y * ((ze - zb + zc - 1) / zc) < 2 * 148) zc /= 2;
+        dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + zc - 1) / zc);
         LaunchScope ls(g, g->cs, name);
-        k_msr_fast<MODE, DM><<<grd, blk, 0, g->cs>>>(A, pgeo(f, p), zb, ze, g->tp, g->T, g->tiles_y);
+        k_msr_fast<MODE, DM><<<grd, blk, 0, g->cs>>>(A, pgeo(f, p), zb, ze, g->tp, g->T, g->tiles_y, zc);
         return nb_launch_check(name);
     }
     MsrOp<MODE, RC, DM> op;
@@ -598,12 +602,61 @@ extern "C" nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, i
     nb_status st = nb_grid_scratch(g, NB_F64, 1, 1, &y2);
     HaloSync hs;
     nb_field *xin = x, *yin = y, *xo = x2, *yo = y2;
-    for (int k = 0; k < iters && st == NB_OK; ++k) {
-        MsrFields F{xin, yin, xo, yo, nullptr};
-        st = msr_step_fields<MSR_C1>(g, occ, F, a, 0.0, 0, nullptr, hs);
-        if (st == NB_OK) st = nb_reduce_finalize(g, 1, FIN_STORE, nullptr, k);
-        std::swap(xin, xo);
-        std::swap(yin, yo);
+    auto loop = [&]() -> nb_status {
+        nb_status s = NB_OK;
+        for (int k = 0; k < iters && s == NB_OK; ++k) {
+            MsrFields F{xin, yin, xo, yo, nullptr};
+            s = msr_step_fields<MSR_C1>(g, occ, F, a, 0.0, 0, nullptr, hs);
+            if (s == NB_OK) s = nb_reduce_finalize(g, 1, FIN_STORE, nullptr, k);
+            std::swap(xin, xo);
+            std::swap(yin, yo);
+        }
+        return s;
+    };
+    // the loop is launch-latency bound at small sizes (C1: 64^3): replay it
+    // as one CUDA graph (rebuilt when fields, a, iterations or OCC change),
+    // except under per-launch profiling, NCCL or event-ordered halo streams,
+    // and across processes (the peer reductions alternate buffers by a host
+    // counter that a replay would not advance)
+    const bool graph = st == NB_OK && iters > 0 && !g->profiling && !nb_halo_on_stream(g) && !nb_is_peer(g) &&
+                       !getenv("NB_NO_GRAPH");
+    if (graph) {
+        const int fl = g->first_local;
+        const bool hit = g->c1_exec && g->c1_x == x->base[fl] && g->c1_y == y->base[fl] && g->c1_a == a &&
+                         g->c1_iters == iters && g->c1_occ == (int)occ;
+        if (!hit) {
+            if (g->c1_exec) cudaGraphExecDestroy(g->c1_exec);
+            g->c1_exec = nullptr;
+            const int64_t l0 = g->launches;
+            cudaGraph_t gr;
+            NB_CUDA(cudaStreamBeginCapture(g->cs, cudaStreamCaptureModeThreadLocal));
+            st = loop();
+            cudaError_t e = cudaStreamEndCapture(g->cs, &gr);
+            g->c1_launches = g->launches - l0;
+            g->launches = l0;
+            if (st == NB_OK && e != cudaSuccess) NB_FAIL(NB_ECUDA, "C1 graph capture: %s", cudaGetErrorString(e));
+            if (st == NB_OK) {
+                e = cudaGraphInstantiate(&g->c1_exec, gr, 0);
+                cudaGraphDestroy(gr);
+                if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "C1 graph instantiate: %s", cudaGetErrorString(e));
+                g->c1_x = x->base[fl];
+                g->c1_y = y->base[fl];
+                g->c1_a = a;
+                g->c1_iters = iters;
+                g->c1_occ = (int)occ;
+            }
+        } else {  // the replay ends where the captured loop ended
+            for (int k = 0; k < iters; ++k) {
+                std::swap(xin, xo);
+                std::swap(yin, yo);
+            }
+        }
+        if (st == NB_OK) {
+            NB_CUDA(cudaGraphLaunch(g->c1_exec, g->cs));
+            g->launches += g->c1_launches;
+        }
+    } else {
+        st = loop();
     }
     if (st == NB_OK && xin != x) {  // odd iteration count: results live in the partners
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {

@@ -49,7 +49,7 @@ template <bool DOMAP, bool C1 = false>
 __global__ void __launch_bounds__(DOT_TX *DOT_TY)
     k_cgA_tma(const __grid_constant__ CUtensorMap m_r, const __grid_constant__ CUtensorMap m_po,
               const __grid_constant__ CUtensorMap m_pn, const __grid_constant__ CUtensorMap m_x, double *pn, double *xs,
-              PGeo g, int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_y, double c1_a = 0.0,
+              PGeo g, int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_y, int zc, double c1_a = 0.0,
               double *c1_out = nullptr) {
     __shared__ CgAStage st[NSTAGE];
     __shared__ __align__(8) uint64_t bar[NSTAGE];
@@ -60,7 +60,7 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY)
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const int x0 = blockIdx.x * DOT_TX, y0 = blockIdx.y * DOT_TY;
     const int xi = x0 + lane, yi = y0 + w;
-    const int zs = zb + blockIdx.z * TZC, zend = min(ze, zs + TZC);
+    const int zs = zb + blockIdx.z * zc, zend = min(ze, zs + zc);  // zc <= TZC planes per CTA
     const int nzl = g.nzl;
     const bool valid = xi < g.nx && yi < g.ny;
     auto halo = [&](int zl) { return zl < 0 || zl >= nzl; };
@@ -151,7 +151,7 @@ struct __align__(128) CgBStage {
 
 __global__ void __launch_bounds__(DOT_TX *DOT_TY)
     k_cgB_tma(const __grid_constant__ CUtensorMap m_p, const __grid_constant__ CUtensorMap m_r, double *r, PGeo g,
-              int zb, int ze, const CgScal *sc, double *tp, int T) {
+              int zb, int ze, const CgScal *sc, double *tp, int T, int zc) {
     __shared__ CgBStage st[NSTAGE];
     __shared__ __align__(8) uint64_t bar[NSTAGE];
     __shared__ double sw[TZC][DOT_TY];
@@ -160,7 +160,7 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY)
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const int x0 = blockIdx.x * DOT_TX, y0 = blockIdx.y * DOT_TY;
     const int xi = x0 + lane, yi = y0 + w;
-    const int zs = zb + blockIdx.z * TZC, zend = min(ze, zs + TZC);
+    const int zs = zb + blockIdx.z * zc, zend = min(ze, zs + zc);
     const bool valid = xi < g.nx && yi < g.ny;
     auto stage_of = [&](int zl) { return (zl - zs + 1) & (NSTAGE - 1); };
     auto parity_of = [&](int zl) { return (uint32_t)(((zl - zs + 1) / NSTAGE) & 1); };
@@ -219,6 +219,16 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY)
 // ---------------------------------------------------------------------------
 // host side: tensor maps (cached per buffer and geometry)
 // ---------------------------------------------------------------------------
+// planes per CTA: TZC, halved while the launch would have fewer than two
+// CTAs per SM (small grids, e.g. C1's 64^3: 16 tiles x 2 chunks = 32 CTAs);
+// the dot partials are per plane and tile, so results do not depend on it
+static int tma_zc(const nb_grid *g, int nplanes) {
+    const int64_t tiles = (int64_t)g->tiles_x * g->tiles_y;
+    int zc = TZC;
+    while (zc > 2 && tiles * ((nplanes + zc - 1) / zc) < 2 * 148) zc /= 2;
+    return zc;
+}
+
 typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
                                   const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -290,12 +300,13 @@ nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double 
     NB_TRY(tmap_for(po, geo, 0, &mpo));
     NB_TRY(tmap_for(pn, geo, 0, &mpn));
     NB_TRY(tmap_for(x, geo, 1, &mx));
-    dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + TZC - 1) / TZC);
+    const int zc = tma_zc(g, ze - zb);
+    dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, "k_msr_cgA");
     if (domap)
-        k_cgA_tma<true><<<grd, blk, 0, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T, g->tiles_y);
+        k_cgA_tma<true><<<grd, blk, 0, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T, g->tiles_y, zc);
     else
-        k_cgA_tma<false><<<grd, blk, 0, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T, g->tiles_y);
+        k_cgA_tma<false><<<grd, blk, 0, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T, g->tiles_y, zc);
     return nb_launch_check("k_cgA_tma");
 }
 
@@ -308,14 +319,15 @@ nb_status nb_c1_tma(nb_grid *g, const PGeo &geo, const double *xin, const double
     NB_TRY(tmap_for(xin, geo, 0, &mx));
     NB_TRY(tmap_for(yin, geo, 0, &my));
     NB_TRY(tmap_for(xout, geo, 0, &mu));
-    dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + TZC - 1) / TZC);
+    const int zc = tma_zc(g, ze - zb);
+    dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, "k_msr_c1");
     if (domap)
         k_cgA_tma<true, true><<<grd, blk, 0, g->cs>>>(mx, my, mu, mx, xout, nullptr, geo, zb, ze, nullptr, g->tp, g->T,
-                                                      g->tiles_y, a, yout);
+                                                      g->tiles_y, zc, a, yout);
     else
         k_cgA_tma<false, true><<<grd, blk, 0, g->cs>>>(mx, my, mu, mx, xout, nullptr, geo, zb, ze, nullptr, g->tp,
-                                                       g->T, g->tiles_y, a, yout);
+                                                       g->T, g->tiles_y, zc, a, yout);
     return nb_launch_check("k_c1_tma");
 }
 
@@ -325,8 +337,9 @@ nb_status nb_cgB_tma(nb_grid *g, const PGeo &geo, const double *p, double *r, in
     CUtensorMap mp, mr;
     NB_TRY(tmap_for(p, geo, 0, &mp));
     NB_TRY(tmap_for(r, geo, 1, &mr));
-    dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + TZC - 1) / TZC);
+    const int zc = tma_zc(g, ze - zb);
+    dim3 blk(DOT_TX * DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, "k_cg_B");
-    k_cgB_tma<<<grd, blk, 0, g->cs>>>(mp, mr, r, geo, zb, ze, sc, g->tp, g->T);
+    k_cgB_tma<<<grd, blk, 0, g->cs>>>(mp, mr, r, geo, zb, ze, sc, g->tp, g->T, zc);
     return nb_launch_check("k_cgB_tma");
 }

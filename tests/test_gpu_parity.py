@@ -215,6 +215,43 @@ def test_c1_exact_regime_bit_exact_vs_oracle():
         fx.close(), fy.close()
 
 
+@pytest.mark.parametrize("parts", [1, 3])
+def test_c1_graph_replay_and_rebuild_bit_exact(parts, monkeypatch):
+    """nb_map_stencil_reduce replays its loop as a CUDA graph: repeated calls
+    on the same fields (replay), odd iteration counts (results copied back
+    from the ping-pong partners), a changed scalar and changed fields
+    (rebuild) must all equal the oracle, and the eager path bit for bit."""
+    dims = (64, 40, 37)
+    x0 = synth.int_uniform(dims, seed=3)
+    # oracle: 4 + 4 iterations at a = 1/8, then 3 at a = 1/4 (dyadic scalars,
+    # integer start: every operation is exact, so the order cannot matter)
+    ox, oy, od1 = oracle.c1_loop(x0, 0.125, 4)
+    ox, oy, od2 = oracle.c1_loop(ox, 0.125, 4, y0=oy)
+    ox, oy, od3 = oracle.c1_loop(ox, 0.25, 3, y0=oy)
+    out = {}
+    for mode in ("graph", "eager"):
+        if mode == "eager":
+            monkeypatch.setenv("NB_NO_GRAPH", "1")
+        with grid(dims, parts) as g:
+            fx, fy = field(g, x0), field(g, np.zeros_like(x0))
+            d1 = nb.nb_map_stencil_reduce(fx, fy, 0.125, 4, nb.OCC_TWO_WAY)
+            d2 = nb.nb_map_stencil_reduce(fx, fy, 0.125, 4, nb.OCC_TWO_WAY)
+            d3 = nb.nb_map_stencil_reduce(fx, fy, 0.25, 3, nb.OCC_TWO_WAY)
+            gx, gy = fx.download(), fy.download()
+            # other fields on the same grid: the cached graph must not be reused
+            hx, hy = field(g, x0), field(g, np.zeros_like(x0))
+            e1 = nb.nb_map_stencil_reduce(hx, hy, 0.125, 4, nb.OCC_TWO_WAY)
+            assert np.array_equal(e1, d1)
+            out[mode] = (gx, gy, d1, d2, d3)
+            for f in (fx, fy, hx, hy):
+                f.close()
+        assert np.array_equal(gx, ox) and np.array_equal(gy, oy), mode
+        for d, o in ((d1, od1), (d2, od2), (d3, od3)):
+            assert np.max(np.abs(d - o) / np.abs(o)) <= 1e-12, mode
+    for a, b in zip(out["graph"], out["eager"]):
+        assert np.array_equal(a, b)
+
+
 def test_c1_real_regime_vs_oracle():
     dims = (45, 19, 37)
     x0 = synth.uniform(dims, seed=1)
