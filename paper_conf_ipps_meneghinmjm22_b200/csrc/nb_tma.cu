@@ -100,7 +100,12 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY)
     double center = U(zs, w + 1, lane + 2);
     const int64_t o = (int64_t)yi * g.pitch + xi + g.ps;  // (xi, yi, zl = 0)
     for (int z = zs; z < zend; ++z) {
-        mbar_wait(&bar[stage_of(z + 1)], parity_of(z + 1));
+        // one thread waits on the stage's mbarrier, the CTA barrier releases
+        // the others (no per-thread try_wait polling); the stage of plane
+        // z-1 is free once every thread passed this barrier
+        if (tid == 0) mbar_wait(&bar[stage_of(z + 1)], parity_of(z + 1));
+        __syncthreads();
+        if (tid == 0 && z + 3 <= zend) issue(z + 3);  // -> stage of plane z-1 (read before this barrier)
         const double above = U(z + 1, w + 1, lane + 2);
         double prod = 0.0;
         if (valid) {
@@ -125,9 +130,8 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY)
         if (lane == 0) sw[z - zs][w] = prod;
         below = center;
         center = above;
-        __syncthreads();  // the stage of plane z-1 is free (last read in the previous step)
-        if (tid == 0 && z + 3 <= zend) issue(z + 3);  // -> stage of plane z-1
     }
+    __syncthreads();  // sw complete
     // per-plane tile partials: the 8 row values in increasing y
     if (tid < zend - zs) {
         double s = sw[tid][0];
@@ -186,7 +190,9 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY)
     double center = st[stage_of(zs)].p[w + 1][lane + 2];
     const int64_t o = (int64_t)yi * g.pitch + xi + g.ps;
     for (int z = zs; z < zend; ++z) {
-        mbar_wait(&bar[stage_of(z + 1)], parity_of(z + 1));
+        if (tid == 0) mbar_wait(&bar[stage_of(z + 1)], parity_of(z + 1));
+        __syncthreads();
+        if (tid == 0 && z + 3 <= zend) issue(z + 3);  // -> stage of plane z-1 (read before this barrier)
         const CgBStage &sz = st[stage_of(z)];
         const double above = st[stage_of(z + 1)].p[w + 1][lane + 2];
         double prod = 0.0;
@@ -205,9 +211,8 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY)
         if (lane == 0) sw[z - zs][w] = prod;
         below = center;
         center = above;
-        __syncthreads();
-        if (tid == 0 && z + 3 <= zend) issue(z + 3);
     }
+    __syncthreads();
     if (tid < zend - zs) {
         double s = sw[tid][0];
 #pragma unroll
