@@ -547,9 +547,17 @@ __device__ __forceinline__ T sp_nsum(const T *x, const int32_t *conn, int64_t n,
 #define NB_SP_NSB 4
 #endif
 constexpr int NSB = NB_SP_NSB;
+#ifndef NB_SP_MINB
+#define NB_SP_MINB 0
+#endif
+#if NB_SP_MINB > 0
+#define NB_SP_LB __launch_bounds__(SEG, NB_SP_MINB)
+#else
+#define NB_SP_LB __launch_bounds__(SEG)
+#endif
 
 template <int K>
-__global__ void __launch_bounds__(SEG) k_sp(SpArgs A) {
+__global__ void NB_SP_LB k_sp(SpArgs A) {
     __shared__ double sw[NSB][SEG / 32];
     if (K >= SPK_CG_MAP && K <= SPK_CG_R && A.sc->status != 0) return;
     const int t = threadIdx.x;

@@ -1,0 +1,4 @@
+for L in "" paper_conf_ipps_meneghinmjm22_b200/libnb_FEM_NST_A3.so paper_conf_ipps_meneghinmjm22_b200/libnb_FEM_NST_A3_FEM_MINB_A2.so; do
+  for a in "70 12 1" "70 12 3"; do NB_LIB=$L python tools/fem_dump.py $a 2>&1 | tail -1; done
+  NB_LIB=$L python tools/fem_time.py 384 20 2>&1 | tail -1
+done > gpurun_out/fem_probe.log 2>&1
