@@ -38,48 +38,59 @@ constexpr int TZC = NB_ZC;  // planes per CTA (matches the z-march chunking)
 #ifndef NB_CG_NTX
 #define NB_CG_NTX 2  // dot tiles per CTA along x of the CG phases (2: 64 x 8 cells, 68 x 10 boxes)
 #endif
-constexpr int BY = DOT_TY + 2;
-constexpr int NSTAGE = 4;
-template <int NTX>
+#ifndef NB_CG_NTY
+#define NB_CG_NTY 1  // dot tiles per CTA along y
+#endif
+#ifndef NB_CG_NST
+#define NB_CG_NST 4  // ring stages
+#endif
+template <int NTX, int NTY = 1, int NST_ = 4>
 struct TmaGeo {
+    static constexpr int NST = NST_;                             // ring stages
     static constexpr int TW = DOT_TX * NTX;                      // CTA width (cells)
+    static constexpr int TH = DOT_TY * NTY;                      // CTA height (rows)
     static constexpr int BXW = TW + 4;                           // box width
-    static constexpr int BOX = BY * BXW;                         // box cells
+    static constexpr int BYH = TH + 2;                           // box height
+    static constexpr int BOX = BYH * BXW;                        // box cells
     static constexpr int BPAD = (BOX * 8 + 127) / 128 * 128 / 8;  // box stride (doubles, 128-B aligned)
-    static constexpr int OWN = DOT_TY * TW;                      // own-cell box
-    static constexpr int NT = TW * DOT_TY;                       // threads
+    static constexpr int OWN = TH * TW;                          // own-cell box
+    static constexpr int NT = TW * TH;                           // threads
+    static constexpr int MINB = NT >= 1024 ? 2 : 1;              // CTAs per SM the registers must allow
     static constexpr int SA = 2 * BPAD + OWN;                    // phase A stage (doubles)
     static constexpr int SB = BPAD + OWN;                        // phase B stage
 };
+using CgGeo = TmaGeo<NB_CG_NTX, NB_CG_NTY, NB_CG_NST>;
 
 // C1 (C1 = true): the same map -> stencil -> reduce chain of Fig. 4a with
 // r -> x_in, p_old -> y_in, p_new -> x_out (u = fma(a, y_in, x_in)),
 // out = L(u) = fma(-6, u, s) stored to y_out, dot u * out, no deferred x.
 // Stage layout (dynamic shared memory): a = r (in-slab planes) or the stored
 // p_new (halo planes), b = p_old, then x of the own cells.
-template <bool DOMAP, bool C1 = false, int NTX = 1>
-__global__ void __launch_bounds__(TmaGeo<NTX>::NT)
+template <bool DOMAP, bool C1, class G>
+__global__ void __launch_bounds__(G::NT, G::MINB)
     k_cgA_tma(const __grid_constant__ CUtensorMap m_r, const __grid_constant__ CUtensorMap m_po,
               const __grid_constant__ CUtensorMap m_pn, const __grid_constant__ CUtensorMap m_x, double *pn, double *xs,
               PGeo g, int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_x, int zc, double c1_a = 0.0,
               double *c1_out = nullptr) {
-    using G = TmaGeo<NTX>;
+    constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY, NSTAGE = G::NST;
     extern __shared__ __align__(128) double tsm[];
     __shared__ __align__(8) uint64_t bar[NSTAGE];
-    __shared__ double sw[TZC][NTX][DOT_TY];
+    __shared__ double sw[TZC][NTY * NTX][DOT_TY];
     if (!C1 && sc->status != 0) return;
     const double beta = C1 ? c1_a : sc->beta, ap = C1 ? 0.0 : sc->alpha_prev;
     const bool dox = !C1 && DOMAP && sc->pending;
-    const int tid = threadIdx.x, lane = tid & 31, w = (tid >> 5) % DOT_TY, tx = (tid >> 5) / DOT_TY;
-    const int x0 = blockIdx.x * G::TW, y0 = blockIdx.y * DOT_TY;
+    // warp -> (dot tile t = (ty, tx) of the CTA, row wr of that tile); w = CTA row
+    const int tid = threadIdx.x, lane = tid & 31, wr = (tid >> 5) % DOT_TY, t = (tid >> 5) / DOT_TY;
+    const int tx = t % NTX, ty = t / NTX, w = ty * DOT_TY + wr;
+    const int x0 = blockIdx.x * G::TW, y0 = blockIdx.y * G::TH;
     const int xi = x0 + tx * DOT_TX + lane, yi = y0 + w;
     const int cx = tx * DOT_TX + lane + 2;  // box column of the own cell
     const int zs = zb + blockIdx.z * zc, zend = min(ze, zs + zc);  // zc <= TZC planes per CTA
     const int nzl = g.nzl;
     const bool valid = xi < g.nx && yi < g.ny;
     auto halo = [&](int zl) { return zl < 0 || zl >= nzl; };
-    auto stage_of = [&](int zl) { return (zl - zs + 1) & (NSTAGE - 1); };
-    auto parity_of = [&](int zl) { return (uint32_t)(((zl - zs + 1) / NSTAGE) & 1); };
+    auto stage_of = [&](int zl) { return (int)((unsigned)(zl - zs + 1) % (unsigned)NSTAGE); };
+    auto parity_of = [&](int zl) { return ((unsigned)(zl - zs + 1) / (unsigned)NSTAGE) & 1u; };
     auto sa = [&](int zl) { return tsm + stage_of(zl) * G::SA; };
     auto sb = [&](int zl) { return tsm + stage_of(zl) * G::SA + G::BPAD; };
     auto sx = [&](int zl) { return tsm + stage_of(zl) * G::SA + 2 * G::BPAD; };
@@ -104,7 +115,7 @@ __global__ void __launch_bounds__(TmaGeo<NTX>::NT)
     }
     __syncthreads();
     if (tid == 0)
-        for (int zl = zs - 1; zl <= min(zs + 2, zend); ++zl) issue(zl);
+        for (int zl = zs - 1; zl <= min(zs + NSTAGE - 2, zend); ++zl) issue(zl);
     // p_new at box cell (yy, xx) of plane zl's stage
     auto U = [&](int zl, int yy, int xx) -> double {
         const int e = yy * G::BXW + xx;
@@ -121,7 +132,7 @@ __global__ void __launch_bounds__(TmaGeo<NTX>::NT)
         // z-1 is free once every thread passed this barrier
         if (tid == 0) mbar_wait(&bar[stage_of(z + 1)], parity_of(z + 1));
         __syncthreads();
-        if (tid == 0 && z + 3 <= zend) issue(z + 3);  // -> stage of plane z-1 (read before this barrier)
+        if (tid == 0 && z + NSTAGE - 1 <= zend) issue(z + NSTAGE - 1);  // -> stage of plane z-1 (read before this barrier)
         const double above = U(z + 1, w + 1, cx);
         double prod = 0.0;
         if (valid) {
@@ -140,18 +151,20 @@ __global__ void __launch_bounds__(TmaGeo<NTX>::NT)
             prod = __dmul_rn(center, q);
         }
         prod = warp_sum_canon(prod);
-        if (lane == 0) sw[z - zs][tx][w] = prod;
+        if (lane == 0) sw[z - zs][t][wr] = prod;
         below = center;
         center = above;
     }
     __syncthreads();  // sw complete
     // per-plane tile partials: the 8 row values in increasing y
-    if (tid < (zend - zs) * NTX) {
-        const int zi = tid / NTX, t = tid % NTX, tile_x = blockIdx.x * NTX + t;
-        double s = sw[zi][t][0];
+    if (tid < (zend - zs) * NTX * NTY) {
+        const int zi = tid / (NTX * NTY), tt = tid % (NTX * NTY);
+        const int tile_x = blockIdx.x * NTX + tt % NTX, tile_y = blockIdx.y * NTY + tt / NTX;
+        double s = sw[zi][tt][0];
 #pragma unroll
-        for (int k = 1; k < DOT_TY; ++k) s = __dadd_rn(s, sw[zi][t][k]);
-        if (tile_x < tiles_x) tp[((int64_t)g.z0 + zs + zi) * T + blockIdx.y * tiles_x + tile_x] = s;
+        for (int k = 1; k < DOT_TY; ++k) s = __dadd_rn(s, sw[zi][tt][k]);
+        if (tile_x < tiles_x && tile_y * DOT_TY < g.ny)
+            tp[((int64_t)g.z0 + zs + zi) * T + (int64_t)tile_y * tiles_x + tile_x] = s;
     }
 }
 
@@ -161,24 +174,26 @@ __global__ void __launch_bounds__(TmaGeo<NTX>::NT)
 // plane), per-plane tile partial of r*r in the ZR = 1 canonical order
 // (butterfly per row, rows in increasing y).
 // ---------------------------------------------------------------------------
-template <int NTX = 1>
-__global__ void __launch_bounds__(TmaGeo<NTX>::NT)
+template <class G>
+__global__ void __launch_bounds__(G::NT, G::MINB)
     k_cgB_tma(const __grid_constant__ CUtensorMap m_p, const __grid_constant__ CUtensorMap m_r, double *r, PGeo g,
               int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_x, int zc) {
-    using G = TmaGeo<NTX>;
+    constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY, NSTAGE = G::NST;
     extern __shared__ __align__(128) double tsm[];
     __shared__ __align__(8) uint64_t bar[NSTAGE];
-    __shared__ double sw[TZC][NTX][DOT_TY];
+    __shared__ double sw[TZC][NTY * NTX][DOT_TY];
     if (sc->status != 0) return;
     const double alpha = sc->alpha;
-    const int tid = threadIdx.x, lane = tid & 31, w = (tid >> 5) % DOT_TY, tx = (tid >> 5) / DOT_TY;
-    const int x0 = blockIdx.x * G::TW, y0 = blockIdx.y * DOT_TY;
+    // warp -> (dot tile t = (ty, tx) of the CTA, row wr of that tile); w = CTA row
+    const int tid = threadIdx.x, lane = tid & 31, wr = (tid >> 5) % DOT_TY, t = (tid >> 5) / DOT_TY;
+    const int tx = t % NTX, ty = t / NTX, w = ty * DOT_TY + wr;
+    const int x0 = blockIdx.x * G::TW, y0 = blockIdx.y * G::TH;
     const int xi = x0 + tx * DOT_TX + lane, yi = y0 + w;
     const int cx = tx * DOT_TX + lane + 2;
     const int zs = zb + blockIdx.z * zc, zend = min(ze, zs + zc);
     const bool valid = xi < g.nx && yi < g.ny;
-    auto stage_of = [&](int zl) { return (zl - zs + 1) & (NSTAGE - 1); };
-    auto parity_of = [&](int zl) { return (uint32_t)(((zl - zs + 1) / NSTAGE) & 1); };
+    auto stage_of = [&](int zl) { return (int)((unsigned)(zl - zs + 1) % (unsigned)NSTAGE); };
+    auto parity_of = [&](int zl) { return ((unsigned)(zl - zs + 1) / (unsigned)NSTAGE) & 1u; };
     auto sp = [&](int zl) { return tsm + stage_of(zl) * G::SB; };
     auto sr = [&](int zl) { return tsm + stage_of(zl) * G::SB + G::BPAD; };
     auto issue = [&](int zl) {
@@ -195,7 +210,7 @@ __global__ void __launch_bounds__(TmaGeo<NTX>::NT)
     }
     __syncthreads();
     if (tid == 0)
-        for (int zl = zs - 1; zl <= min(zs + 2, zend); ++zl) issue(zl);
+        for (int zl = zs - 1; zl <= min(zs + NSTAGE - 2, zend); ++zl) issue(zl);
     mbar_wait(&bar[stage_of(zs - 1)], parity_of(zs - 1));
     mbar_wait(&bar[stage_of(zs)], parity_of(zs));
     const int c = (w + 1) * G::BXW + cx;
@@ -205,7 +220,7 @@ __global__ void __launch_bounds__(TmaGeo<NTX>::NT)
     for (int z = zs; z < zend; ++z) {
         if (tid == 0) mbar_wait(&bar[stage_of(z + 1)], parity_of(z + 1));
         __syncthreads();
-        if (tid == 0 && z + 3 <= zend) issue(z + 3);  // -> stage of plane z-1 (read before this barrier)
+        if (tid == 0 && z + NSTAGE - 1 <= zend) issue(z + NSTAGE - 1);  // -> stage of plane z-1 (read before this barrier)
         const double *pz = sp(z);
         const double above = sp(z + 1)[c];
         double prod = 0.0;
@@ -221,17 +236,19 @@ __global__ void __launch_bounds__(TmaGeo<NTX>::NT)
             prod = __dmul_rn(rn, rn);
         }
         prod = warp_sum_canon(prod);
-        if (lane == 0) sw[z - zs][tx][w] = prod;
+        if (lane == 0) sw[z - zs][t][wr] = prod;
         below = center;
         center = above;
     }
     __syncthreads();
-    if (tid < (zend - zs) * NTX) {
-        const int zi = tid / NTX, t = tid % NTX, tile_x = blockIdx.x * NTX + t;
-        double s = sw[zi][t][0];
+    if (tid < (zend - zs) * NTX * NTY) {
+        const int zi = tid / (NTX * NTY), tt = tid % (NTX * NTY);
+        const int tile_x = blockIdx.x * NTX + tt % NTX, tile_y = blockIdx.y * NTY + tt / NTX;
+        double s = sw[zi][tt][0];
 #pragma unroll
-        for (int k = 1; k < DOT_TY; ++k) s = __dadd_rn(s, sw[zi][t][k]);
-        if (tile_x < tiles_x) tp[((int64_t)g.z0 + zs + zi) * T + blockIdx.y * tiles_x + tile_x] = s;
+        for (int k = 1; k < DOT_TY; ++k) s = __dadd_rn(s, sw[zi][tt][k]);
+        if (tile_x < tiles_x && tile_y * DOT_TY < g.ny)
+            tp[((int64_t)g.z0 + zs + zi) * T + (int64_t)tile_y * tiles_x + tile_x] = s;
     }
 }
 
@@ -271,11 +288,10 @@ static EncodeTiledFn encode_fn() {
 static std::mutex g_tmap_mu;
 static std::map<std::tuple<const void *, int, int, int, int64_t, int>, CUtensorMap> g_tmaps;
 
-// box = 2 (ntx - 1) + own: own = 0 -> (tile + ring) (32 ntx + 4) x 10 x 1
-// (x from x0-2), own = 1 -> own tile 32 ntx x 8 x 1; ntx dot tiles per CTA
-nb_status tmap_for(const void *base, const PGeo &g, int box, CUtensorMap *out) {
+// tensor map of a partition buffer with a bw x bh x 1 box (cached)
+nb_status tmap_box(const void *base, const PGeo &g, int bw, int bh, CUtensorMap *out) {
     std::lock_guard<std::mutex> lk(g_tmap_mu);
-    auto key = std::make_tuple(base, g.nx, g.ny, g.nzl, g.pitch, box);
+    auto key = std::make_tuple(base, g.nx, g.ny, g.nzl, g.pitch, bw * 1024 + bh);
     auto it = g_tmaps.find(key);
     if (it != g_tmaps.end()) {
         *out = it->second;
@@ -286,9 +302,7 @@ nb_status tmap_for(const void *base, const PGeo &g, int box, CUtensorMap *out) {
     CUtensorMap m;
     cuuint64_t dims[3] = {(cuuint64_t)g.nx, (cuuint64_t)g.ny, (cuuint64_t)(g.nzl + 2)};
     cuuint64_t strides[2] = {(cuuint64_t)g.pitch * 8, (cuuint64_t)g.ps * 8};
-    const int ntx = box / 2 + 1;
-    const bool own = box & 1;
-    cuuint32_t boxd[3] = {(cuuint32_t)(DOT_TX * ntx + (own ? 0 : 4)), (cuuint32_t)(own ? DOT_TY : BY), 1};
+    cuuint32_t boxd[3] = {(cuuint32_t)bw, (cuuint32_t)bh, 1};
     cuuint32_t es[3] = {1, 1, 1};
     CUresult r = fn(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<void *>(base), dims, strides, boxd, es,
                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
@@ -297,6 +311,11 @@ nb_status tmap_for(const void *base, const PGeo &g, int box, CUtensorMap *out) {
     g_tmaps[key] = m;
     *out = m;
     return NB_OK;
+}
+
+// box: 0 = (tile + ring) 36 x 10 x 1 (x from x0-2), 1 = own tile 32 x 8 x 1
+nb_status tmap_for(const void *base, const PGeo &g, int box, CUtensorMap *out) {
+    return box == 0 ? tmap_box(base, g, DOT_TX + 4, DOT_TY + 2, out) : tmap_box(base, g, DOT_TX, DOT_TY, out);
 }
 
 // drop cached maps of a freed buffer
@@ -324,23 +343,22 @@ static void tma_smem_attr(F *f, int bytes) {
     }
 }
 
-template <bool DOMAP, bool C1, int NTX>
+template <bool DOMAP, bool C1, class G>
 static nb_status launch_cgA(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x,
                             int zb, int ze, const CgScal *sc, double c1_a, double *c1_out, const char *label) {
-    using G = TmaGeo<NTX>;
     CUtensorMap mr, mpo, mpn, mx;
-    const int bx = 2 * (NTX - 1);
-    NB_TRY(tmap_for(r, geo, bx, &mr));
-    NB_TRY(tmap_for(po, geo, bx, &mpo));
-    NB_TRY(tmap_for(pn, geo, bx, &mpn));
-    NB_TRY(tmap_for(C1 ? r : x, geo, C1 ? bx : bx + 1, &mx));
+    NB_TRY(tmap_box(r, geo, G::BXW, G::BYH, &mr));
+    NB_TRY(tmap_box(po, geo, G::BXW, G::BYH, &mpo));
+    NB_TRY(tmap_box(pn, geo, G::BXW, G::BYH, &mpn));
+    NB_TRY(tmap_box(C1 ? r : x, geo, C1 ? G::BXW : G::TW, C1 ? G::BYH : G::TH, &mx));
     const int zc = tma_zc(g, ze - zb);
-    const int smem = NSTAGE * G::SA * 8;
-    tma_smem_attr(k_cgA_tma<DOMAP, C1, NTX>, smem);
-    dim3 blk(G::NT), grd((g->tiles_x + NTX - 1) / NTX, g->tiles_y, (ze - zb + zc - 1) / zc);
+    const int smem = G::NST * G::SA * 8;
+    tma_smem_attr(k_cgA_tma<DOMAP, C1, G>, smem);
+    constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY;
+    dim3 blk(G::NT), grd((g->tiles_x + NTX - 1) / NTX, (g->tiles_y + NTY - 1) / NTY, (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, label);
-    k_cgA_tma<DOMAP, C1, NTX><<<grd, blk, smem, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T,
-                                                         g->tiles_x, zc, c1_a, c1_out);
+    k_cgA_tma<DOMAP, C1, G><<<grd, blk, smem, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T,
+                                                       g->tiles_x, zc, c1_a, c1_out);
     return nb_launch_check(label);
 }
 
@@ -348,9 +366,8 @@ static nb_status launch_cgA(nb_grid *g, const PGeo &geo, const double *r, const 
 nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x, bool domap,
                      int zb, int ze, const CgScal *sc) {
     if (ze <= zb) return NB_OK;
-    constexpr int N = NB_CG_NTX;
-    return domap ? launch_cgA<true, false, N>(g, geo, r, po, pn, x, zb, ze, sc, 0.0, nullptr, "k_msr_cgA")
-                 : launch_cgA<false, false, N>(g, geo, r, po, pn, x, zb, ze, sc, 0.0, nullptr, "k_msr_cgA");
+    return domap ? launch_cgA<true, false, CgGeo>(g, geo, r, po, pn, x, zb, ze, sc, 0.0, nullptr, "k_msr_cgA")
+                 : launch_cgA<false, false, CgGeo>(g, geo, r, po, pn, x, zb, ze, sc, 0.0, nullptr, "k_msr_cgA");
 }
 
 // C1 map-stencil-reduce on planes [zb, ze): x_out = x_in + a y_in (stored
@@ -358,24 +375,23 @@ nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double 
 nb_status nb_c1_tma(nb_grid *g, const PGeo &geo, const double *xin, const double *yin, double *xout, double *yout,
                     double a, bool domap, int zb, int ze) {
     if (ze <= zb) return NB_OK;
-    constexpr int N = NB_CG_NTX;
-    return domap ? launch_cgA<true, true, N>(g, geo, xin, yin, xout, nullptr, zb, ze, nullptr, a, yout, "k_msr_c1")
-                 : launch_cgA<false, true, N>(g, geo, xin, yin, xout, nullptr, zb, ze, nullptr, a, yout, "k_msr_c1");
+    return domap ? launch_cgA<true, true, CgGeo>(g, geo, xin, yin, xout, nullptr, zb, ze, nullptr, a, yout, "k_msr_c1")
+                 : launch_cgA<false, true, CgGeo>(g, geo, xin, yin, xout, nullptr, zb, ze, nullptr, a, yout, "k_msr_c1");
 }
 
 // CG phase B on planes [zb, ze) of a partition (stored p_new, r)
 nb_status nb_cgB_tma(nb_grid *g, const PGeo &geo, const double *p, double *r, int zb, int ze, const CgScal *sc) {
     if (ze <= zb) return NB_OK;
-    constexpr int N = NB_CG_NTX;
-    using G = TmaGeo<N>;
+    using G = CgGeo;
     CUtensorMap mp, mr;
-    NB_TRY(tmap_for(p, geo, 2 * (N - 1), &mp));
-    NB_TRY(tmap_for(r, geo, 2 * (N - 1) + 1, &mr));
+    NB_TRY(tmap_box(p, geo, G::BXW, G::BYH, &mp));
+    NB_TRY(tmap_box(r, geo, G::TW, G::TH, &mr));
     const int zc = tma_zc(g, ze - zb);
-    const int smem = NSTAGE * G::SB * 8;
-    tma_smem_attr(k_cgB_tma<N>, smem);
-    dim3 blk(G::NT), grd((g->tiles_x + N - 1) / N, g->tiles_y, (ze - zb + zc - 1) / zc);
+    const int smem = G::NST * G::SB * 8;
+    tma_smem_attr(k_cgB_tma<G>, smem);
+    constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY;
+    dim3 blk(G::NT), grd((g->tiles_x + NTX - 1) / NTX, (g->tiles_y + NTY - 1) / NTY, (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, "k_cg_B");
-    k_cgB_tma<N><<<grd, blk, smem, g->cs>>>(mp, mr, r, geo, zb, ze, sc, g->tp, g->T, g->tiles_x, zc);
+    k_cgB_tma<G><<<grd, blk, smem, g->cs>>>(mp, mr, r, geo, zb, ze, sc, g->tp, g->T, g->tiles_x, zc);
     return nb_launch_check("k_cgB_tma");
 }
