@@ -244,10 +244,12 @@ def bench_cg(args, world, rank, local):
     e2e()  # warm
     ms_e, _ = timed(world, stream, e2e, local)
     out["e2e"] = {"value": cells * args.steps / (ms_e / 1e3) / 1e6, "unit": "MLUPS",
-                  "h2d_bytes_per_step": 2 * local_bytes, "d2h_bytes_per_step": local_bytes,
+                  "h2d_bytes_per_step": 2 * local_bytes / args.steps, "d2h_bytes_per_step": local_bytes / args.steps,
+                  "h2d_bytes_per_call": 2 * local_bytes, "d2h_bytes_per_call": local_bytes,
                   "note": "per rank: upload b and x0 (own slab) from pinned host, CG create (r = b - Ax0), "
                           "steps iterations, finish (deferred x update), download x (own slab); "
-                          "one e2e call per timed region, max over ranks"}
+                          "one e2e call (a whole solve of `steps` iterations) per timed region, max over ranks; "
+                          "bytes per step = bytes per call / steps"}
     b.close(), x.close()
     g.close()
     if comm:

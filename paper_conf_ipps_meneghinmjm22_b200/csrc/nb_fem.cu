@@ -834,8 +834,8 @@ struct FemTma {
     __device__ __forceinline__ bool halo(int zl) const { return zl < 0 || zl >= g.nzl; }
 
     __device__ __forceinline__ void issue(int j) const {  // plane zs-1+j -> stage j % NST
-        double *S = fsm + (j % NST) * SD;
-        uint64_t *b = &bar[j % NST];
+        double *S = fsm + ((unsigned)j % NST) * SD;
+        uint64_t *b = &bar[(unsigned)j % NST];
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         const int zl = zs - 1 + j, tz = zl + 1;
         if (CGA && !halo(zl)) {
@@ -864,7 +864,7 @@ struct FemTma {
                                          const double (&cP)[NR][3], double (&cC)[NR][3]) const {
         const int zin = zs - 1 + j;  // local plane held by this stage
         const bool own = zin >= zs && zin < zend;
-        const double *S = fsm + (j % NST) * SD;  // stencil input tiles of this plane
+        const double *S = fsm + ((unsigned)j % NST) * SD;  // stencil input tiles of this plane
         double xo[NR][3], pc[NR][3];               // CGA: x and p_old of the own centres
         if constexpr (CGA) {
             if (own && dox) {
@@ -876,7 +876,7 @@ struct FemTma {
                     for (int c = 0; c < 3; ++c) xo[r][c] = v ? __ldcs(A.x + c * A.cs + c0) : 0.0;
                 }
             }
-            mbar_wait(&bar[j % NST], (uint32_t)((j / NST) & 1));
+            mbar_wait(&bar[(unsigned)j % NST], ((unsigned)j / NST) & 1u);
             double *P = fsm + NST * SD + (j & 1) * 3 * CP;  // p_new tiles (double-buffered)
             if (!halo(zin)) {  // CTA-uniform
                 for (int c = 0; c < 3; ++c)
@@ -894,7 +894,7 @@ struct FemTma {
             S = P;
         } else {
             if (j >= 3) flush(zs + j - 3, tp, T);  // the previous step's output (barrier passed)
-            mbar_wait(&bar[j % NST], (uint32_t)((j / NST) & 1));
+            mbar_wait(&bar[(unsigned)j % NST], ((unsigned)j / NST) & 1u);
         }
         if (anyfast) {
 #pragma unroll
