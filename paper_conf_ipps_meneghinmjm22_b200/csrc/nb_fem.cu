@@ -238,19 +238,20 @@ struct FemUCgA {
     }
 };
 
-// surface path of fem_node: the class stencil C over the in-box positions
-template <class CF, class U>
-__device__ __forceinline__ void fem_node_surf(const CF &C, const U &u, const PGeo &g, int x, int y, int zl,
-                                              double &acc0, double &acc1, double &acc2) {
-    const int gz = g.z0 + zl;
-    const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+// surface path of fem_node: the class stencil C over the in-box positions.
+// L(ox, oy, oz, u0, u1, u2) fetches the 3 components at offset (ox, oy, oz):
+// every caller shares this loop, so the FMA chain (o order, then K + 0..8)
+// is the same whichever memory the values come from.
+template <class CF, class L>
+__device__ __forceinline__ void fem_node_surf_l(const CF &C, const PGeo &g, int x, int y, int gz, const L &load,
+                                                double &acc0, double &acc1, double &acc2) {
 #pragma unroll
     for (int o = 0; o < 27; ++o) {
         const int ox = o % 3 - 1, oy = (o / 3) % 3 - 1, oz = o / 9 - 1;
         const int mx = x + ox, my = y + oy, mz = gz + oz;
         if (mx < 0 || my < 0 || mz < 0 || mx >= g.nx || my >= g.ny || mz >= g.NZ) continue;
-        const int64_t m = c0 + (int64_t)oz * g.ps + (int64_t)oy * g.pitch + ox;
-        const double u0 = u(0, m, zl + oz), u1 = u(1, m, zl + oz), u2 = u(2, m, zl + oz);
+        double u0, u1, u2;
+        load(ox, oy, oz, u0, u1, u2);
         const int K = o * 9;
         acc0 = fma(C(K + 0), u0, acc0);
         acc0 = fma(C(K + 1), u1, acc0);
@@ -262,6 +263,27 @@ __device__ __forceinline__ void fem_node_surf(const CF &C, const U &u, const PGe
         acc2 = fma(C(K + 7), u1, acc2);
         acc2 = fma(C(K + 8), u2, acc2);
     }
+}
+
+template <class CF, class U>
+__device__ __forceinline__ void fem_node_surf(const CF &C, const U &u, const PGeo &g, int x, int y, int zl,
+                                              double &acc0, double &acc1, double &acc2) {
+    const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+    fem_node_surf_l(
+        C, g, x, y, g.z0 + zl,
+        [&](int ox, int oy, int oz, double &u0, double &u1, double &u2) {
+            const int64_t m = c0 + (int64_t)oz * g.ps + (int64_t)oy * g.pitch + ox;
+            u0 = u(0, m, zl + oz);
+            u1 = u(1, m, zl + oz);
+            u2 = u(2, m, zl + oz);
+        },
+        acc0, acc1, acc2);
+}
+
+// surface class of the node at (x, y, gz)
+__device__ __forceinline__ int fem_surf_cls(int x, int y, int gz, const PGeo &g) {
+    return ((fem_axis_state(x, g.nx) * 4 + fem_axis_state(y, g.ny)) * 4 + fem_axis_state(gz, g.NZ)) * 2 +
+           (gz == 1 ? 1 : 0);
 }
 
 // K u at node (x, y, zl) of the partition; returns the 3 components.
@@ -300,8 +322,7 @@ __device__ __forceinline__ void fem_node(const U &u, const PGeo &g, int x, int y
     } else {
         // surface class stencil (positions outside the box have no element
         // and are skipped; their coefficients are zero)
-        const int cls = ((fem_axis_state(x, g.nx) * 4 + fem_axis_state(y, g.ny)) * 4 + fem_axis_state(gz, g.NZ)) * 2 +
-                        (gz == 1 ? 1 : 0);
+        const int cls = fem_surf_cls(x, y, gz, g);
         const int sl = fem_cslot(cls);
         if (sl >= 0)
             fem_node_surf(FemCConst{sl}, u, g, x, y, zl, acc0, acc1, acc2);
@@ -622,6 +643,73 @@ __global__ void __launch_bounds__(128) k_fem_surface(FemArgs A, PGeo g, int zb, 
         A.y[A.cs + c0] = o[1];
         A.y[2 * A.cs + c0] = o[2];
     }
+}
+
+// ---- x-face columns, staged through shared memory ------------------------
+// The nodes of the x = 0 and x = nx-1 faces (y in [1, ny-2]) sit one per
+// row: a warp of them reads 32 different rows per load, and each value is
+// re-read by up to 9 neighbours — k_fem_surface spent most of its time in
+// these L1 wavefronts.  Here a CTA of 32 (y) x 8 (z) face nodes first copies
+// the 2 x 34 x 10 patch of the 3 components (p_new formed on the fly in CG
+// phase A) into shared memory with one load per value, then evaluates the
+// same class stencil (fem_node_surf_l: bitwise the global-memory path).
+constexpr int XF_Y = 32, XF_Z = 8;
+
+template <int K>
+__global__ void __launch_bounds__(XF_Y *XF_Z) k_fem_xface(FemArgs A, PGeo g, int zb, int ze) {
+    if ((K == FEM_CG_Q || K == FEM_CG_A) && A.sc->status != 0) return;
+    __shared__ double su[3][XF_Z + 2][XF_Y + 2][2];
+    const int face = blockIdx.z;
+    const int xa = face ? g.nx - 2 : 0;  // patch columns xa, xa + 1
+    const int x = face ? g.nx - 1 : 0;   // node column
+    const int ybase = blockIdx.x * XF_Y;  // patch rows ybase .. ybase + 33; nodes ybase + 1 ..
+    const int zbase = zb + blockIdx.y * XF_Z;  // node planes zbase ..; patch planes zbase - 1 ..
+    const int tid = threadIdx.x;
+    constexpr int NP = (XF_Z + 2) * (XF_Y + 2) * 2;
+    for (int e = tid; e < 3 * NP; e += XF_Y * XF_Z) {
+        const int c = e / NP, r = e % NP;
+        const int xx = r & 1, yy = (r >> 1) % (XF_Y + 2), zz = (r >> 1) / (XF_Y + 2);
+        const int yg = ybase + yy, zl = zbase - 1 + zz, gz = g.z0 + zl;
+        double v = 0.0;
+        if (yg < g.ny && xa + xx < g.nx && gz >= 0 && gz < g.NZ && zl <= g.nzl) {
+            const int64_t m = (int64_t)(zl + 1) * g.ps + (int64_t)yg * g.pitch + xa + xx;
+            if constexpr (K == FEM_CG_A)
+                v = FemUCgA{A.r, A.po, A.pn, A.cs, A.sc->beta, g.nzl}(c, m, zl);
+            else
+                v = A.u[c * A.cs + m];
+        }
+        su[c][zz][yy][xx] = v;
+    }
+    __syncthreads();
+    const int ty = tid % XF_Y, tz = tid / XF_Y;
+    const int y = ybase + 1 + ty, zl = zbase + tz, gz = g.z0 + zl;
+    if (y > g.ny - 2 || zl >= ze) return;
+    double o[3];
+    if (gz == 0) {  // Dirichlet identity row
+#pragma unroll
+        for (int c = 0; c < 3; ++c) o[c] = su[c][tz + 1][ty + 1][x - xa];
+    } else {
+        double a0 = 0.0, a1 = 0.0, a2 = 0.0;
+        auto load = [&](int ox, int oy, int oz, double &u0, double &u1, double &u2) {
+            const int zz = tz + 1 + oz, yy = ty + 1 + oy, xx = x + ox - xa;
+            u0 = su[0][zz][yy][xx];
+            u1 = su[1][zz][yy][xx];
+            u2 = su[2][zz][yy][xx];
+        };
+        const int cls = fem_surf_cls(x, y, gz, g);
+        const int sl = fem_cslot(cls);
+        if (sl >= 0)
+            fem_node_surf_l(FemCConst{sl}, g, x, y, gz, load, a0, a1, a2);
+        else
+            fem_node_surf_l(FemCGlob{c_cls + (size_t)cls * 243}, g, x, y, gz, load, a0, a1, a2);
+        o[0] = a0;
+        o[1] = a1;
+        o[2] = a2;
+    }
+    const int64_t c0 = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+    A.y[c0] = o[0];
+    A.y[A.cs + c0] = o[1];
+    A.y[2 * A.cs + c0] = o[2];
 }
 
 // ---- face columns (x or y on the box surface), z-marching -----------------
@@ -1138,9 +1226,19 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
             // face (default; 0.19 ms at 384^3 for all surface nodes), or the
             // z-marching column kernel (NB_FEM_FACES=col; 0.22 ms); z-surface
             // planes: one thread per node
-            const bool faces_node = !(getenv("NB_FEM_FACES") && !strcmp(getenv("NB_FEM_FACES"), "col"));
+            const char *fv = getenv("NB_FEM_FACES");
+            const bool faces_node = !(fv && !strcmp(fv, "col"));
+            // x-face columns through shared memory (default), unless
+            // NB_FEM_FACES=node keeps them in k_fem_surface
+            const bool xface = faces_node && !(fv && !strcmp(fv, "node")) && nx >= 2 && ny >= 3;
             const int ncols = faces_node ? 0 : S.ncol_edge;
             if (!faces_node) S.ncol_edge = 0;
+            if (xface) {
+                S.ncol_edge = 2 * nx;  // fem_edge_col lists the y = 0 and y = ny-1 rows first
+                dim3 xg((ny - 2 + XF_Y - 1) / XF_Y, (ze - zb + XF_Z - 1) / XF_Z, 2);
+                LaunchScope ls(g, g->cs, "k_fem_surface");
+                k_fem_xface<K><<<xg, XF_Y * XF_Z, 0, g->cs>>>(A, geo, zb, ze);
+            }
             const int64_t n = (int64_t)S.ncol_edge * (ze - zb) + (int64_t)S.nin * S.nzs;
             if (n > 0) {
                 const int blocks = (int)std::min<int64_t>((n + 127) / 128, 1 << 30);

@@ -107,7 +107,8 @@ def test_fem_cg_converges():
     assert x[2, -1].mean() > 0           # the top moves outward (+z) under the pressure
 
 
-@pytest.mark.parametrize("dims,parts", [((17, 13, 40), 1), ((34, 19, 37), 3), ((9, 10, 5), 1)])
+@pytest.mark.parametrize("dims,parts", [((17, 13, 40), 1), ((34, 19, 37), 3), ((9, 10, 5), 1), ((20, 70, 13), 2),
+                                        ((2, 9, 6), 1)])
 def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
     """The TMA-staged z-march (default), the register z-march and the
     one-node-per-thread kernel must agree bit for bit: each output receives
@@ -117,10 +118,13 @@ def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
     u = synth.uniform(dims, card=3, seed=9)
     out = {}
     # kernel variants (NB_FEM_KERNEL), the z-marching face-column kernel
-    # (NB_FEM_FACES=col) and the 3-pass CG schedule (NB_FEM_3PASS: map ->
-    # q = K p -> r) against the default fused schedule
+    # (NB_FEM_FACES=col), x-face nodes in the one-thread-per-node surface
+    # kernel instead of the shared-memory x-face kernel (NB_FEM_FACES=node)
+    # and the 3-pass CG schedule (NB_FEM_3PASS: map -> q = K p -> r)
+    # against the default fused schedule
     envs = {None: {}, "zmarch": {"NB_FEM_KERNEL": "zmarch"}, "plain": {"NB_FEM_KERNEL": "plain"},
-            "faces_col": {"NB_FEM_FACES": "col"}, "3pass": {"NB_FEM_3PASS": "1"}}
+            "faces_col": {"NB_FEM_FACES": "col"}, "faces_node": {"NB_FEM_FACES": "node"},
+            "3pass": {"NB_FEM_3PASS": "1"}}
     for variant, env in envs.items():
         for k in ("NB_FEM_KERNEL", "NB_FEM_FACES", "NB_FEM_3PASS"):
             if k in env:
@@ -140,6 +144,6 @@ def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
             out[variant] = (y, fx.download(), r.rr)
             for f in (fu, fy, fb, fx):
                 f.close()
-    for v in ("zmarch", "plain", "faces_col", "3pass"):
+    for v in ("zmarch", "plain", "faces_col", "faces_node", "3pass"):
         assert np.array_equal(out[None][0], out[v][0]), v
         assert np.array_equal(out[None][1], out[v][1]) and out[None][2] == out[v][2], v
