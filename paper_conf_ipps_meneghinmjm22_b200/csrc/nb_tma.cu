@@ -55,9 +55,15 @@ struct TmaGeo {
     static constexpr int BPAD = (BOX * 8 + 127) / 128 * 128 / 8;  // box stride (doubles, 128-B aligned)
     static constexpr int OWN = TH * TW;                          // own-cell box
     static constexpr int NT = TW * TH;                           // threads
-    static constexpr int MINB = NT >= 1024 ? 2 : 1;              // CTAs per SM the registers must allow
     static constexpr int SA = 2 * BPAD + OWN;                    // phase A stage (doubles)
     static constexpr int SB = BPAD + OWN;                        // phase B stage
+    // CTAs per SM the registers must allow: as many as the shared memory
+    // does (ring + ~5 KB static + 1 KB reserved per CTA of 228 KB per SM)
+    static constexpr int fit(int ring) {
+        const int by_smem = 233472 / (ring * 8 + 6 * 1024), by_threads = 2048 / NT;
+        return by_smem < by_threads ? by_smem : by_threads;
+    }
+    static constexpr int MINB_A = fit(NST * SA), MINB_B = fit(NST * SB);
 };
 using CgGeo = TmaGeo<NB_CG_NTX, NB_CG_NTY, NB_CG_NST>;
 
@@ -67,7 +73,7 @@ using CgGeo = TmaGeo<NB_CG_NTX, NB_CG_NTY, NB_CG_NST>;
 // Stage layout (dynamic shared memory): a = r (in-slab planes) or the stored
 // p_new (halo planes), b = p_old, then x of the own cells.
 template <bool DOMAP, bool C1, class G>
-__global__ void __launch_bounds__(G::NT, G::MINB)
+__global__ void __launch_bounds__(G::NT, G::MINB_A)
     k_cgA_tma(const __grid_constant__ CUtensorMap m_r, const __grid_constant__ CUtensorMap m_po,
               const __grid_constant__ CUtensorMap m_pn, const __grid_constant__ CUtensorMap m_x, double *pn, double *xs,
               PGeo g, int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_x, int zc, double c1_a = 0.0,
@@ -126,34 +132,49 @@ __global__ void __launch_bounds__(G::NT, G::MINB)
     double below = U(zs - 1, w + 1, cx);
     double center = U(zs, w + 1, cx);
     const int64_t o = (int64_t)yi * g.pitch + xi + g.ps;  // (xi, yi, zl = 0)
-    for (int z = zs; z < zend; ++z) {
-        // one thread waits on the stage's mbarrier, the CTA barrier releases
-        // the others (no per-thread try_wait polling); the stage of plane
-        // z-1 is free once every thread passed this barrier
-        if (tid == 0) mbar_wait(&bar[stage_of(z + 1)], parity_of(z + 1));
-        __syncthreads();
-        if (tid == 0 && z + NSTAGE - 1 <= zend) issue(z + NSTAGE - 1);  // -> stage of plane z-1 (read before this barrier)
-        const double above = U(z + 1, w + 1, cx);
-        double prod = 0.0;
-        if (valid) {
-            double s = __dadd_rn(U(z, w + 1, cx - 1), U(z, w + 1, cx + 1));
-            s = __dadd_rn(s, U(z, w, cx));
-            s = __dadd_rn(s, U(z, w + 2, cx));
-            s = __dadd_rn(s, below);
-            s = __dadd_rn(s, above);
-            const double q = C1 ? fma(-6.0, center, s) : fma(6.0, center, -s);
-            const int64_t e = o + (int64_t)z * g.ps;
-            if (C1) __stcs(c1_out + e, q);
-            if (DOMAP) {
-                pn[e] = center;
-                if (dox) xs[e] = fma(ap, sb(z)[(w + 1) * G::BXW + cx], sx(z)[w * G::TW + cx - 2]);
+    // The plane loop is unrolled by the ring depth: plane z = zq + k sits in
+    // stage (k + 1) % NSTAGE, a compile-time constant, so every shared-memory
+    // read is a fixed offset from the ring base.  Planes z in [zs, zend) are
+    // inside the slab (never halo); only the plane above may be a halo plane.
+    const int c = (w + 1) * G::BXW + cx;  // own cell in a box
+    double *pnp = DOMAP ? pn + o + (int64_t)zs * g.ps : nullptr;
+    double *xsp = dox ? xs + o + (int64_t)zs * g.ps : nullptr;
+    double *c1p = C1 ? c1_out + o + (int64_t)zs * g.ps : nullptr;
+    for (int zq = zs, q = 0; zq < zend; zq += NSTAGE, ++q) {
+#pragma unroll
+        for (int k = 0; k < NSTAGE; ++k) {
+            const int z = zq + k;
+            if (z >= zend) break;  // CTA-uniform
+            const int s0 = (k + 1) % NSTAGE, s1 = (k + 2) % NSTAGE;  // stages of planes z, z + 1
+            if (tid == 0) mbar_wait(&bar[s1], (unsigned)(q + (k + 2) / NSTAGE) & 1u);
+            __syncthreads();
+            if (tid == 0 && z + NSTAGE - 1 <= zend) issue(z + NSTAGE - 1);  // -> stage k (plane z-1)
+            const double *A1 = tsm + s1 * G::SA, *A0 = tsm + s0 * G::SA;
+            const double *B1 = A1 + G::BPAD, *B0 = A0 + G::BPAD;
+            const double above = z + 1 >= nzl ? A1[c] : fma(beta, B1[c], A1[c]);
+            double prod = 0.0;
+            if (valid) {
+                double s = __dadd_rn(fma(beta, B0[c - 1], A0[c - 1]), fma(beta, B0[c + 1], A0[c + 1]));
+                s = __dadd_rn(s, fma(beta, B0[c - G::BXW], A0[c - G::BXW]));
+                s = __dadd_rn(s, fma(beta, B0[c + G::BXW], A0[c + G::BXW]));
+                s = __dadd_rn(s, below);
+                s = __dadd_rn(s, above);
+                const double qv = C1 ? fma(-6.0, center, s) : fma(6.0, center, -s);
+                if (C1) __stcs(c1p, qv);
+                if (DOMAP) {
+                    *pnp = center;
+                    if (dox) *xsp = fma(ap, B0[c], (A0 + 2 * G::BPAD)[w * G::TW + cx - 2]);
+                }
+                prod = __dmul_rn(center, qv);
             }
-            prod = __dmul_rn(center, q);
+            if (DOMAP) pnp += g.ps;
+            if (dox) xsp += g.ps;
+            if (C1) c1p += g.ps;
+            prod = warp_sum_canon(prod);
+            if (lane == 0) sw[z - zs][t][wr] = prod;
+            below = center;
+            center = above;
         }
-        prod = warp_sum_canon(prod);
-        if (lane == 0) sw[z - zs][t][wr] = prod;
-        below = center;
-        center = above;
     }
     __syncthreads();  // sw complete
     // per-plane tile partials: the 8 row values in increasing y
@@ -175,7 +196,7 @@ __global__ void __launch_bounds__(G::NT, G::MINB)
 // (butterfly per row, rows in increasing y).
 // ---------------------------------------------------------------------------
 template <class G>
-__global__ void __launch_bounds__(G::NT, G::MINB)
+__global__ void __launch_bounds__(G::NT, G::MINB_B)
     k_cgB_tma(const __grid_constant__ CUtensorMap m_p, const __grid_constant__ CUtensorMap m_r, double *r, PGeo g,
               int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_x, int zc) {
     constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY, NSTAGE = G::NST;
@@ -217,28 +238,36 @@ __global__ void __launch_bounds__(G::NT, G::MINB)
     double below = sp(zs - 1)[c];
     double center = sp(zs)[c];
     const int64_t o = (int64_t)yi * g.pitch + xi + g.ps;
-    for (int z = zs; z < zend; ++z) {
-        if (tid == 0) mbar_wait(&bar[stage_of(z + 1)], parity_of(z + 1));
-        __syncthreads();
-        if (tid == 0 && z + NSTAGE - 1 <= zend) issue(z + NSTAGE - 1);  // -> stage of plane z-1 (read before this barrier)
-        const double *pz = sp(z);
-        const double above = sp(z + 1)[c];
-        double prod = 0.0;
-        if (valid) {
-            double s = __dadd_rn(pz[c - 1], pz[c + 1]);
-            s = __dadd_rn(s, pz[c - G::BXW]);
-            s = __dadd_rn(s, pz[c + G::BXW]);
-            s = __dadd_rn(s, below);
-            s = __dadd_rn(s, above);
-            const double q = fma(6.0, center, -s);
-            const double rn = fma(-alpha, q, sr(z)[w * G::TW + cx - 2]);
-            __stcs(r + o + (int64_t)z * g.ps, rn);
-            prod = __dmul_rn(rn, rn);
+    double *rp = r + o + (int64_t)zs * g.ps;
+    for (int zq = zs, q = 0; zq < zend; zq += NSTAGE, ++q) {
+#pragma unroll
+        for (int k = 0; k < NSTAGE; ++k) {
+            const int z = zq + k;
+            if (z >= zend) break;  // CTA-uniform
+            const int s0 = (k + 1) % NSTAGE, s1 = (k + 2) % NSTAGE;  // stages of planes z, z + 1
+            if (tid == 0) mbar_wait(&bar[s1], (unsigned)(q + (k + 2) / NSTAGE) & 1u);
+            __syncthreads();
+            if (tid == 0 && z + NSTAGE - 1 <= zend) issue(z + NSTAGE - 1);  // -> stage k (plane z-1)
+            const double *pz = tsm + s0 * G::SB;
+            const double above = (tsm + s1 * G::SB)[c];
+            double prod = 0.0;
+            if (valid) {
+                double s = __dadd_rn(pz[c - 1], pz[c + 1]);
+                s = __dadd_rn(s, pz[c - G::BXW]);
+                s = __dadd_rn(s, pz[c + G::BXW]);
+                s = __dadd_rn(s, below);
+                s = __dadd_rn(s, above);
+                const double qv = fma(6.0, center, -s);
+                const double rn = fma(-alpha, qv, (pz + G::BPAD)[w * G::TW + cx - 2]);
+                __stcs(rp, rn);
+                prod = __dmul_rn(rn, rn);
+            }
+            rp += g.ps;
+            prod = warp_sum_canon(prod);
+            if (lane == 0) sw[z - zs][t][wr] = prod;
+            below = center;
+            center = above;
         }
-        prod = warp_sum_canon(prod);
-        if (lane == 0) sw[z - zs][t][wr] = prod;
-        below = center;
-        center = above;
     }
     __syncthreads();
     if (tid < (zend - zs) * NTX * NTY) {
