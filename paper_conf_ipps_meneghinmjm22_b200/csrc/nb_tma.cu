@@ -141,10 +141,12 @@ __global__ void __launch_bounds__(G::NT, G::MINB_A)
     double *xsp = dox ? xs + o + (int64_t)zs * g.ps : nullptr;
     double *c1p = C1 ? c1_out + o + (int64_t)zs * g.ps : nullptr;
     for (int zq = zs, q = 0; zq < zend; zq += NSTAGE, ++q) {
+        double pv[NSTAGE];  // this group's per-plane row products, reduced together below
 #pragma unroll
         for (int k = 0; k < NSTAGE; ++k) {
             const int z = zq + k;
-            if (z >= zend) break;  // CTA-uniform
+            pv[k] = 0.0;
+            if (z >= zend) continue;  // CTA-uniform
             const int s0 = (k + 1) % NSTAGE, s1 = (k + 2) % NSTAGE;  // stages of planes z, z + 1
             if (tid == 0) mbar_wait(&bar[s1], (unsigned)(q + (k + 2) / NSTAGE) & 1u);
             __syncthreads();
@@ -170,11 +172,15 @@ __global__ void __launch_bounds__(G::NT, G::MINB_A)
             if (DOMAP) pnp += g.ps;
             if (dox) xsp += g.ps;
             if (C1) c1p += g.ps;
-            prod = warp_sum_canon(prod);
-            if (lane == 0) sw[z - zs][t][wr] = prod;
+            pv[k] = prod;
             below = center;
             center = above;
         }
+        // the NSTAGE row sums of the group in one transposed butterfly (bitwise
+        // equal to NSTAGE warp_sum_canon calls, a third of the shuffles)
+        const double v = warp_sum_multi<NSTAGE>(pv, lane);
+        const int i = warp_multi_index<NSTAGE>(lane);
+        if ((lane & (32 / WarpMulti<NSTAGE>::M - 1)) == 0 && i < NSTAGE && zq + i < zend) sw[zq + i - zs][t][wr] = v;
     }
     __syncthreads();  // sw complete
     // per-plane tile partials: the 8 row values in increasing y
@@ -240,10 +246,12 @@ __global__ void __launch_bounds__(G::NT, G::MINB_B)
     const int64_t o = (int64_t)yi * g.pitch + xi + g.ps;
     double *rp = r + o + (int64_t)zs * g.ps;
     for (int zq = zs, q = 0; zq < zend; zq += NSTAGE, ++q) {
+        double pv[NSTAGE];  // this group's per-plane row products, reduced together below
 #pragma unroll
         for (int k = 0; k < NSTAGE; ++k) {
             const int z = zq + k;
-            if (z >= zend) break;  // CTA-uniform
+            pv[k] = 0.0;
+            if (z >= zend) continue;  // CTA-uniform
             const int s0 = (k + 1) % NSTAGE, s1 = (k + 2) % NSTAGE;  // stages of planes z, z + 1
             if (tid == 0) mbar_wait(&bar[s1], (unsigned)(q + (k + 2) / NSTAGE) & 1u);
             __syncthreads();
@@ -263,11 +271,15 @@ __global__ void __launch_bounds__(G::NT, G::MINB_B)
                 prod = __dmul_rn(rn, rn);
             }
             rp += g.ps;
-            prod = warp_sum_canon(prod);
-            if (lane == 0) sw[z - zs][t][wr] = prod;
+            pv[k] = prod;
             below = center;
             center = above;
         }
+        // the NSTAGE row sums of the group in one transposed butterfly (bitwise
+        // equal to NSTAGE warp_sum_canon calls, a third of the shuffles)
+        const double v = warp_sum_multi<NSTAGE>(pv, lane);
+        const int i = warp_multi_index<NSTAGE>(lane);
+        if ((lane & (32 / WarpMulti<NSTAGE>::M - 1)) == 0 && i < NSTAGE && zq + i < zend) sw[zq + i - zs][t][wr] = v;
     }
     __syncthreads();
     if (tid < (zend - zs) * NTX * NTY) {
