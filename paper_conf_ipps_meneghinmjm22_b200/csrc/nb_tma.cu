@@ -137,6 +137,8 @@ __global__ void __launch_bounds__(G::NT, G::MINB_A)
     // read is a fixed offset from the ring base.  Planes z in [zs, zend) are
     // inside the slab (never halo); only the plane above may be a halo plane.
     const int c = (w + 1) * G::BXW + cx;  // own cell in a box
+    const int cown = 2 * G::BPAD + w * G::TW + cx - 2;  // own cell in the stage's x tile
+    const int64_t ps = g.ps;
     double *pnp = DOMAP ? pn + o + (int64_t)zs * g.ps : nullptr;
     double *xsp = dox ? xs + o + (int64_t)zs * g.ps : nullptr;
     double *c1p = C1 ? c1_out + o + (int64_t)zs * g.ps : nullptr;
@@ -165,13 +167,13 @@ __global__ void __launch_bounds__(G::NT, G::MINB_A)
                 if (C1) __stcs(c1p, qv);
                 if (DOMAP) {
                     *pnp = center;
-                    if (dox) *xsp = fma(ap, B0[c], (A0 + 2 * G::BPAD)[w * G::TW + cx - 2]);
+                    if (dox) *xsp = fma(ap, B0[c], A0[cown]);
                 }
                 prod = __dmul_rn(center, qv);
             }
-            if (DOMAP) pnp += g.ps;
-            if (dox) xsp += g.ps;
-            if (C1) c1p += g.ps;
+            if (DOMAP) pnp += ps;
+            if (dox) xsp += ps;
+            if (C1) c1p += ps;
             pv[k] = prod;
             below = center;
             center = above;
@@ -245,6 +247,8 @@ __global__ void __launch_bounds__(G::NT, G::MINB_B)
     double center = sp(zs)[c];
     const int64_t o = (int64_t)yi * g.pitch + xi + g.ps;
     double *rp = r + o + (int64_t)zs * g.ps;
+    const int cown = G::BPAD + w * G::TW + cx - 2;  // own cell in the stage's r tile
+    const int64_t ps = g.ps;
     for (int zq = zs, q = 0; zq < zend; zq += NSTAGE, ++q) {
         double pv[NSTAGE];  // this group's per-plane row products, reduced together below
 #pragma unroll
@@ -266,11 +270,11 @@ __global__ void __launch_bounds__(G::NT, G::MINB_B)
                 s = __dadd_rn(s, below);
                 s = __dadd_rn(s, above);
                 const double qv = fma(6.0, center, -s);
-                const double rn = fma(-alpha, qv, (pz + G::BPAD)[w * G::TW + cx - 2]);
+                const double rn = fma(-alpha, qv, pz[cown]);
                 __stcs(rp, rn);
                 prod = __dmul_rn(rn, rn);
             }
-            rp += g.ps;
+            rp += ps;
             pv[k] = prod;
             below = center;
             center = above;
