@@ -24,7 +24,7 @@ LABELS = [("k_cgA_tma", "k_msr_cgA"), ("k_cgB_tma", "k_cg_B"), ("k_msr_fast<1, 1
           ("k_sp<4>", "k_sp_cg_q"), ("k_sp<5>", "k_sp_cg_r"), ("k_sp<2>", "k_sp_cg_init"),
           ("k_fem_tma<1", "k_fem_cg_q"), ("k_fem_tma<2", "k_fem_cg_init"), ("k_fem_tma<3", "k_fem_cg_a"),
           ("k_fem_tma<0", "k_fem_apply"), ("k_fem_faces", "k_fem_faces"),
-          ("k_fem_surface", "k_fem_surface"), ("k_fem<1>", "k_fem_cg_q"), ("k_fem<2>", "k_fem_cg_init"),
+          ("k_fem_surface", "k_fem_surface"), ("k_fem_xface", "k_fem_xface"), ("k_fem<1>", "k_fem_cg_q"), ("k_fem<2>", "k_fem_cg_init"),
           ("k_fem_map", "k_fem_map"), ("k_fem_r(", "k_fem_r"), ("k_fem_rhs", "k_fem_rhs"),
           ("k_halo_copy", "k_halo_copy"), ("k_peer_ops", "k_peer_ops")]
 
