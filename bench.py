@@ -224,6 +224,9 @@ def bench_cg(args, world, rank, local):
         "gpu_launches": int(launches), "clocks": clocks,
         "cg_state": {"iters": res.iters, "rr0": res.rr0, "rr": res.rr},
     }
+    if _SHARED_GPU:
+        out["note"] = ("ranks share one GPU (fewer GPUs than ranks): kernels of different ranks overlap and "
+                       "the peer-flag waits spin, so per-kernel times and the roofline are not meaningful here")
     # ---- e2e: public API, host buffers, H2D and D2H inside the timed region
     # (every rank holds the dense host logical view; nb_field_upload /
     # download move only its own slab)
@@ -647,11 +650,19 @@ def bench_skeleton(local, n=512, parts=4, iters=10):
 
 
 # ---------------------------------------------------------------------------
+def _oracle_all_cores():
+    """The oracle runs on every host core (torchrun sets OMP_NUM_THREADS=1 in
+    each rank; the reference arm and cpu_baseline run on rank 0 alone)."""
+    import oracle
+    oracle.set_num_threads(os.cpu_count() or 1)
+    return oracle
+
+
 def cpu_baseline_cg(n, iters=2):
     """The oracle (plain C, fp64, OpenMP over planes) on the host cores:
     `iters` CG iterations on the full n^3 grid (setup subtracted)."""
-    import oracle
     import synth
+    oracle = _oracle_all_cores()
     b = synth.poisson_poly_rhs((n, n, n))
     t0 = time.perf_counter()
     oracle.cg(b, max_iter=0)
@@ -666,7 +677,7 @@ def cpu_baseline_cg(n, iters=2):
 def cpu_baseline_lbm(n=256, steps=2):
     import numpy as np
 
-    import oracle
+    oracle = _oracle_all_cores()
     c, w, _ = oracle.lbm_lattice()
     f = np.broadcast_to(w[:, None, None, None], (19, n, n, n)).astype(np.float32)
     om = lbm_omega(n)
@@ -683,8 +694,8 @@ def reference_arm(args, world, rank):
     config / metric / unit; each step = one CG iteration on the full grid."""
     if rank != 0:
         return None
-    import oracle
     import synth
+    oracle = _oracle_all_cores()
     n = args.n
     b = synth.poisson_poly_rhs((n, n, n))
     # W untimed warm-up iterations, then K timed ones (capped at 400: ~0.35 s
