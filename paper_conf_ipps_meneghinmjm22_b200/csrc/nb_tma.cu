@@ -300,14 +300,37 @@ __global__ void __launch_bounds__(G::NT, G::MINB_B)
 // ---------------------------------------------------------------------------
 // host side: tensor maps (cached per buffer and geometry)
 // ---------------------------------------------------------------------------
-// planes per CTA: TZC, halved while the launch would have fewer than two
-// CTAs per SM (small grids, e.g. C1's 64^3: 16 tiles x 2 chunks = 32 CTAs);
-// the dot partials are per plane and tile, so results do not depend on it
-static int tma_zc(const nb_grid *g, int nplanes) {
-    const int64_t tiles = (int64_t)g->tiles_x * g->tiles_y;
-    int zc = TZC;
-    while (zc > 2 && tiles * ((nplanes + zc - 1) / zc) < 2 * 148) zc /= 2;
-    return zc;
+// planes per CTA.  Every CTA marches zc planes (plus ~H planes of set-up:
+// the two z-halo planes of the ring and the first load's latency), so a
+// launch costs about ceil(CTAs / resident CTAs) x (zc + H).  zc is the
+// power-of-two divisor of TZC (down to 2) that minimises that estimate:
+// 512^3 on one GPU keeps 32 (19 waves of 444 CTAs); a 64-plane slab (512^3
+// on 8 GPUs) takes 16 (5 waves instead of 3 partly empty ones).  The dot
+// partials are per plane and tile, so results do not depend on zc.
+// NB_CG_ZC=<n> forces n.
+static int sm_count() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+    }
+    return n;
+}
+static int tma_zc(int ctas_per_plane, int nplanes, int ctas_per_sm) {
+    static int forced = -1;
+    if (forced < 0) forced = getenv("NB_CG_ZC") ? std::max(1, std::min(TZC, atoi(getenv("NB_CG_ZC")))) : 0;
+    if (forced) return forced;
+    const int64_t cap = (int64_t)sm_count() * ctas_per_sm;
+    constexpr double H = 3.0;
+    int best = TZC;
+    double best_cost = 1e300;
+    for (int zc = TZC; zc >= 2; zc /= 2) {
+        const int64_t n = (int64_t)ctas_per_plane * ((nplanes + zc - 1) / zc);
+        const double cost = (double)((n + cap - 1) / cap) * (std::min(zc, nplanes) + H);
+        if (cost < best_cost - 1e-9) best_cost = cost, best = zc;
+    }
+    return best;
 }
 
 typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
@@ -396,10 +419,10 @@ static nb_status launch_cgA(nb_grid *g, const PGeo &geo, const double *r, const 
     NB_TRY(tmap_box(po, geo, G::BXW, G::BYH, &mpo));
     NB_TRY(tmap_box(pn, geo, G::BXW, G::BYH, &mpn));
     NB_TRY(tmap_box(C1 ? r : x, geo, C1 ? G::BXW : G::TW, C1 ? G::BYH : G::TH, &mx));
-    const int zc = tma_zc(g, ze - zb);
+    constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY;
+    const int zc = tma_zc(((g->tiles_x + NTX - 1) / NTX) * ((g->tiles_y + NTY - 1) / NTY), ze - zb, G::MINB_A);
     const int smem = G::NST * G::SA * 8;
     tma_smem_attr(k_cgA_tma<DOMAP, C1, G>, smem);
-    constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY;
     dim3 blk(G::NT), grd((g->tiles_x + NTX - 1) / NTX, (g->tiles_y + NTY - 1) / NTY, (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, label);
     k_cgA_tma<DOMAP, C1, G><<<grd, blk, smem, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T,
@@ -431,10 +454,10 @@ nb_status nb_cgB_tma(nb_grid *g, const PGeo &geo, const double *p, double *r, in
     CUtensorMap mp, mr;
     NB_TRY(tmap_box(p, geo, G::BXW, G::BYH, &mp));
     NB_TRY(tmap_box(r, geo, G::TW, G::TH, &mr));
-    const int zc = tma_zc(g, ze - zb);
+    constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY;
+    const int zc = tma_zc(((g->tiles_x + NTX - 1) / NTX) * ((g->tiles_y + NTY - 1) / NTY), ze - zb, G::MINB_B);
     const int smem = G::NST * G::SB * 8;
     tma_smem_attr(k_cgB_tma<G>, smem);
-    constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY;
     dim3 blk(G::NT), grd((g->tiles_x + NTX - 1) / NTX, (g->tiles_y + NTY - 1) / NTY, (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, "k_cg_B");
     k_cgB_tma<G><<<grd, blk, smem, g->cs>>>(mp, mr, r, geo, zb, ze, sc, g->tp, g->T, g->tiles_x, zc);
