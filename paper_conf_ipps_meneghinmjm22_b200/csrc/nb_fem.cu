@@ -900,7 +900,9 @@ struct FemTmaCfg {
     static constexpr int NT = DOT_TX * (DOT_TY / NR);         // threads per CTA
     static constexpr int NST = CGA ? NB_FEM_NST_A : FNST;     // ring stages
     static constexpr int SD = (CGA ? 6 : 3) * (FTPAD / 8);    // doubles per stage
-    static constexpr int SMEM = (NST * SD + (CGA ? 6 * (FTPAD / 8) : 0)) * 8;  // dynamic shared memory bytes
+    // dynamic shared memory bytes: the ring, plus (FEM_CG_A) three p_new
+    // buffers of 3 component tiles
+    static constexpr int SMEM = (NST * SD + (CGA ? 9 * (FTPAD / 8) : 0)) * 8;
     static constexpr int MINB = CGA ? NB_FEM_MINB_A : NB_FEM_MINB;  // CTAs per SM
 };
 
@@ -971,7 +973,10 @@ struct FemTma {
                 }
             }
             mbar_wait(&bar[(unsigned)j % NST], ((unsigned)j / NST) & 1u);
-            double *P = fsm + NST * SD + (j & 1) * 3 * CP;  // p_new tiles (double-buffered)
+            // p_new tiles, three buffers: plane j's is formed here; plane j-1's
+            // stays readable for this step's epilogue (its centres are the dot's
+            // p_new), and is overwritten only at step j+2, past barrier j+1
+            double *P = fsm + NST * SD + ((unsigned)j % 3u) * 3 * CP;
             if (!halo(zin)) {  // CTA-uniform
                 for (int c = 0; c < 3; ++c)
                     for (int e = tid; e < FBX * FBY; e += NT) P[c * CP + e] = fma(beta, S[(3 + c) * CP + e], S[c * CP + e]);
@@ -1003,10 +1008,12 @@ struct FemTma {
             fem_q<NR, 7, DA, DB>(cv, S, sidx, aA, aB, aC);
             fem_q<NR, 8, DA, DB>(cv, S, sidx, aA, aB, aC);
         }
+        if constexpr (!CGA) {
 #pragma unroll
-        for (int r = 0; r < NR; ++r)
+            for (int r = 0; r < NR; ++r)
 #pragma unroll
-            for (int c = 0; c < 3; ++c) cC[r][c] = S[c * CP + sidx + r * FBX];
+                for (int c = 0; c < 3; ++c) cC[r][c] = S[c * CP + sidx + r * FBX];
+        }
         if constexpr (CGA) {
             if (own) {  // own plane: store p_new and the deferred x += alpha_prev p_old
 #pragma unroll
@@ -1016,14 +1023,26 @@ struct FemTma {
                         const int64_t c0 = (int64_t)(zin + 1) * g.ps + (int64_t)y * g.pitch + x;
 #pragma unroll
                         for (int c = 0; c < 3; ++c) {
-                            __stcs(A.pn + c * A.cs + c0, cC[r][c]);
+                            __stcs(A.pn + c * A.cs + c0, S[c * CP + sidx + r * FBX]);  // S = this plane's p_new tiles
                             if (dox) __stcs(A.x + c * A.cs + c0, fma(ap, pc[r][c], xo[r][c]));
                         }
                     }
                 }
             }
         }
-        if constexpr (DA) epilogue(j - 2 + zs, aA, cP);
+        if constexpr (DA) {
+            if constexpr (CGA) {  // centres of output j-2 = plane j-1, read back from its p_new buffer
+                const double *Pp = fsm + NST * SD + ((unsigned)(j + 2) % 3u) * 3 * CP;
+                double cen[NR][3];
+#pragma unroll
+                for (int r = 0; r < NR; ++r)
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) cen[r][c] = Pp[c * CP + sidx + r * FBX];
+                epilogue(j - 2 + zs, aA, cen);
+            } else {
+                epilogue(j - 2 + zs, aA, cP);
+            }
+        }
         if constexpr (!CGA) {
             __syncthreads();  // stage j % NST is free
             if (tid == 0 && j + NST < nplanes) issue(j + NST);
