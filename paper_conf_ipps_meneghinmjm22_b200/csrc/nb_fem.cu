@@ -1180,6 +1180,65 @@ __global__ void k_fem_map(double *x, double *pn, const double *po, const double 
     }
 }
 
+// CG residual update, z-marching: a CTA owns one 32 x 8 tile for FRZ planes;
+// the next plane's q and r are loaded while the current one is updated, and
+// the three component dots of a plane go through one transposed butterfly
+// (bitwise the three canonical butterflies of k_fem_r)
+constexpr int FRZ = 16;
+__global__ void __launch_bounds__(DOT_TX *DOT_TY) k_fem_rz(double *r, const double *q, int64_t cs, PGeo g, int zb, int ze,
+                                                          const CgScal *sc, double *tp, int T) {
+    __shared__ double sw[FRZ][3][DOT_TY];
+    if (sc->status != 0) return;
+    const double alpha = sc->alpha;
+    const int lane = threadIdx.x, w = threadIdx.y;
+    const int x = blockIdx.x * DOT_TX + lane, y = blockIdx.y * DOT_TY + w;
+    const int zs = zb + blockIdx.z * FRZ, zend = min(ze, zs + FRZ);
+    const bool valid = x < g.nx && y < g.ny;
+    const int64_t ps = g.ps, off = (int64_t)(zs + 1) * ps + (int64_t)y * g.pitch + x;
+    const double *qp = q + off;
+    double *rp = r + off;
+    double qn[3] = {0.0, 0.0, 0.0}, rn[3] = {0.0, 0.0, 0.0};
+    if (valid)
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+            qn[c] = __ldcs(qp + c * cs);
+            rn[c] = __ldcs(rp + c * cs);
+        }
+    for (int z = zs; z < zend; ++z) {
+        double qc[3], rc[3];
+#pragma unroll
+        for (int c = 0; c < 3; ++c) qc[c] = qn[c], rc[c] = rn[c];
+        if (valid && z + 1 < zend)
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                qn[c] = __ldcs(qp + ps + c * cs);
+                rn[c] = __ldcs(rp + ps + c * cs);
+            }
+        double prod[3] = {0.0, 0.0, 0.0};
+        if (valid)
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                const double v = fma(-alpha, qc[c], rc[c]);
+                __stcs(rp + c * cs, v);
+                prod[c] = __dmul_rn(v, v);
+            }
+        const double s = warp_sum_multi<3>(prod, lane);
+        const int i = warp_multi_index<3>(lane);
+        if ((lane & 7) == 0 && i < 3) sw[z - zs][i][w] = s;
+        qp += ps;
+        rp += ps;
+    }
+    __syncthreads();
+    const int t = w * DOT_TX + lane;
+    if (t < 3 * (zend - zs)) {
+        const int zi = t / 3, c = t % 3;
+        double s = sw[zi][c][0];
+#pragma unroll
+        for (int k = 1; k < DOT_TY; ++k) s = __dadd_rn(s, sw[zi][c][k]);
+        tp[((int64_t)c * g.NZ + g.z0 + zs + zi) * T + blockIdx.y * gridDim.x + blockIdx.x] = s;
+    }
+}
+
 // CG residual update r -= alpha q with per-component canonical tile dots
 __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_fem_r(double *r, const double *q, int64_t cs, PGeo g, int zb,
                                                          const CgScal *sc, double *tp, int T) {
@@ -1415,10 +1474,16 @@ nb_status nb_fem_cg_hooks(nb_cg *cg, int parity) {
     NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         PGeo geo = pgeo(pn, p);
-        dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, geo.nzl);
         LaunchScope ls(g, g->cs, "k_fem_r");
-        k_fem_r<<<grd, blk, 0, g->cs>>>((double *)cg->r->base[p], (const double *)cg->q->base[p], fcs(pn, p), geo, 0,
-                                        cg->sc, g->tp, g->T);
+        if (getenv("NB_FEM_R_PLANE")) {  // one CTA per tile and plane (the earlier kernel)
+            dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, geo.nzl);
+            k_fem_r<<<grd, blk, 0, g->cs>>>((double *)cg->r->base[p], (const double *)cg->q->base[p], fcs(pn, p), geo,
+                                            0, cg->sc, g->tp, g->T);
+        } else {
+            dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, (geo.nzl + FRZ - 1) / FRZ);
+            k_fem_rz<<<grd, blk, 0, g->cs>>>((double *)cg->r->base[p], (const double *)cg->q->base[p], fcs(pn, p), geo,
+                                             0, geo.nzl, cg->sc, g->tp, g->T);
+        }
         NB_TRY(nb_launch_check("k_fem_r"));
     }
     NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_RR, cg->sc, 0));

@@ -120,13 +120,14 @@ def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
     # kernel variants (NB_FEM_KERNEL), the z-marching face-column kernel
     # (NB_FEM_FACES=col), x-face nodes in the one-thread-per-node surface
     # kernel instead of the shared-memory x-face kernel (NB_FEM_FACES=node)
-    # and the 3-pass CG schedule (NB_FEM_3PASS: map -> q = K p -> r)
-    # against the default fused schedule
+    # and the 3-pass CG schedule (NB_FEM_3PASS: map -> q = K p -> r), and
+    # the one-CTA-per-plane residual kernel (NB_FEM_R_PLANE) against the
+    # default fused schedule
     envs = {None: {}, "zmarch": {"NB_FEM_KERNEL": "zmarch"}, "plain": {"NB_FEM_KERNEL": "plain"},
             "faces_col": {"NB_FEM_FACES": "col"}, "faces_node": {"NB_FEM_FACES": "node"},
-            "3pass": {"NB_FEM_3PASS": "1"}}
+            "3pass": {"NB_FEM_3PASS": "1"}, "r_plane": {"NB_FEM_R_PLANE": "1"}}
     for variant, env in envs.items():
-        for k in ("NB_FEM_KERNEL", "NB_FEM_FACES", "NB_FEM_3PASS"):
+        for k in ("NB_FEM_KERNEL", "NB_FEM_FACES", "NB_FEM_3PASS", "NB_FEM_R_PLANE"):
             if k in env:
                 monkeypatch.setenv(k, env[k])
             else:
@@ -144,6 +145,6 @@ def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
             out[variant] = (y, fx.download(), r.rr)
             for f in (fu, fy, fb, fx):
                 f.close()
-    for v in ("zmarch", "plain", "faces_col", "faces_node", "3pass"):
+    for v in ("zmarch", "plain", "faces_col", "faces_node", "3pass", "r_plane"):
         assert np.array_equal(out[None][0], out[v][0]), v
         assert np.array_equal(out[None][1], out[v][1]) and out[None][2] == out[v][2], v
