@@ -64,13 +64,19 @@ __device__ __forceinline__ void lbm_collide(const float (&f)[Q19], float om, flo
         if (CZv(i) == 1) jz += f[i];
         if (CZv(i) == -1) jz -= f[i];
     }
-    const float ux = jx / rho, uy = jy / rho, uz = jz / rho;
+    // one reciprocal instead of three divisions; feq = (w rho) (base + cu (3 + 4.5 cu))
+    // with base = 1 - 1.5 |u|^2 and w rho per weight class
+    const float ir = 1.0f / rho;
+    const float ux = jx * ir, uy = jy * ir, uz = jz * ir;
     const float usq = ux * ux + uy * uy + uz * uz;
+    const float base = 1.0f - 1.5f * usq;
+    const float r0 = (1.0f / 3.0f) * rho, r1 = (1.0f / 18.0f) * rho, r2 = (1.0f / 36.0f) * rho;
 #pragma unroll
     for (int i = 0; i < Q19; ++i) {
-        float cu = (float)CXv(i) * ux + (float)CYv(i) * uy + (float)CZv(i) * uz;
-        float feq = Wv(i) * rho * (1.0f + 3.0f * cu + 4.5f * cu * cu - 1.5f * usq);
-        o[i] = f[i] - om * (f[i] - feq);
+        const float cu = (float)CXv(i) * ux + (float)CYv(i) * uy + (float)CZv(i) * uz;
+        const float wr = i == 0 ? r0 : (CXv(i) * CXv(i) + CYv(i) * CYv(i) + CZv(i) * CZv(i) == 1 ? r1 : r2);
+        const float feq = wr * fmaf(cu, fmaf(4.5f, cu, 3.0f), base);
+        o[i] = fmaf(-om, f[i] - feq, f[i]);
     }
 }
 
