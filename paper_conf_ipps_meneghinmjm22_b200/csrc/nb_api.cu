@@ -501,6 +501,8 @@ extern "C" nb_status nb_grid_destroy(nb_grid *g) {
     }
     g->scratch.clear();
     if (g->c1_exec) cudaGraphExecDestroy(g->c1_exec);
+    cudaFree(g->c1_tp);
+    cudaFree(g->c1_psum);
     nb_peer_grid_teardown(g);  // collective (peer transport)
     for (auto &r : g->prof) {
         cudaEventDestroy(r.a);
@@ -1059,20 +1061,24 @@ __global__ void __launch_bounds__(RED_THREADS) k_finalize(const double *tp, int 
     if (!last) return;
     __threadfence();
     // canonical tree over all planes (volatile-free: psum written by other
-    // blocks before their fence + atomic; read through L2)
+    // blocks before their fence + atomic; read through L2); FIN_STORE_EACH:
+    // the same tree over each component's planes, one total per component
     const int t = threadIdx.x;
-    double acc = 0.0;
-    for (int i = t; i < final_planes; i += RED_THREADS) acc = __dadd_rn(acc, __ldcg(psum + i));
-    sh[t] = acc;
-    __syncthreads();
-    for (int k = RED_THREADS / 2; k > 0; k >>= 1) {
-        if (t < k) sh[t] = __dadd_rn(sh[t], sh[t + k]);
+    const int ncomp = mode == FIN_STORE_EACH ? card : 1;
+    const int per = final_planes / ncomp;
+    for (int cc = 0; cc < ncomp; ++cc) {
+        double acc = 0.0;
+        for (int i = t; i < per; i += RED_THREADS) acc = __dadd_rn(acc, __ldcg(psum + (int64_t)cc * per + i));
+        sh[t] = acc;
+        __syncthreads();
+        for (int k = RED_THREADS / 2; k > 0; k >>= 1) {
+            if (t < k) sh[t] = __dadd_rn(sh[t], sh[t + k]);
+            __syncthreads();
+        }
+        if (t == 0) nb_apply_final(mode == FIN_STORE_EACH ? FIN_STORE : mode, sh[0], state, dots, slot + cc);
         __syncthreads();
     }
-    if (t == 0) {
-        *counter = 0u;
-        nb_apply_final(mode, sh[0], state, dots, slot);
-    }
+    if (t == 0) *counter = 0u;
 }
 
 __global__ void __launch_bounds__(RED_THREADS) k_final_only(const double *psum, int planes, int mode,
@@ -1108,6 +1114,16 @@ nb_status nb_reduce_finalize(nb_grid *g, int card, int mode, void *state, int sl
     LaunchScope ls(g, s, "k_final_only");
     k_final_only<<<1, RED_THREADS, 0, s>>>(g->psum, planes, mode, state, g->dots, slot);
     return nb_launch_check("k_final_only");
+}
+
+// C1: one finalize for `iters` iterations whose tile partials sit in
+// consecutive [NZ][T] slices of g->c1_tp (single process)
+nb_status nb_c1_finalize_all(nb_grid *g, int iters) {
+    const int planes = iters * g->nz;
+    LaunchScope ls(g, g->cs, "k_finalize");
+    k_finalize<<<planes, RED_THREADS, 0, g->cs>>>(g->c1_tp, g->T, g->c1_psum, g->nz, 0, g->nz, iters, g->counter,
+                                                    planes, FIN_STORE_EACH, nullptr, g->dots, 0);
+    return nb_launch_check("k_finalize");
 }
 
 nb_status nb_sparse_dot_partials(const nb_field *x, const nb_field *y);

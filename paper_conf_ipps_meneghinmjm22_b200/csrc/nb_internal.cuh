@@ -169,6 +169,10 @@ struct nb_grid {
     double c1_a = 0.0;
     int c1_iters = -1, c1_occ = -1;
     int64_t c1_launches = 0;
+    // C1 tile partials / plane sums of all iterations of one call (single
+    // process: one finalize per call instead of one per iteration)
+    double *c1_tp = nullptr, *c1_psum = nullptr;
+    int64_t c1_cap = 0;  // doubles of c1_tp
     // element-sparse
     std::vector<NbSparsePart> sp;
     std::vector<int64_t> plane_count;  // [nz] active per global plane
@@ -257,6 +261,7 @@ enum {
     FIN_CG_INIT = 1,  // rr = rr0 = total
     FIN_CG_PQ = 2,    // alpha = rr / total
     FIN_CG_RR = 3,    // beta = total / rr ...
+    FIN_STORE_EACH = 4,  // dots[slot + c] = total of component c (card components)
 };
 
 struct CgScal {

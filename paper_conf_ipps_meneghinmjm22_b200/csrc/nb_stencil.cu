@@ -35,6 +35,7 @@ bool nb_tma_enabled();
 nb_status nb_cgB_tma(nb_grid *g, const PGeo &geo, const double *p, double *r, int zb, int ze, const CgScal *sc);
 nb_status nb_c1_tma(nb_grid *g, const PGeo &geo, const double *xin, const double *yin, double *xout, double *yout,
                     double a, bool domap, int zb, int ze);
+nb_status nb_c1_finalize_all(nb_grid *g, int iters);
 nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x, bool domap,
                      int zb, int ze, const CgScal *sc);
 
@@ -602,15 +603,35 @@ extern "C" nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, i
     nb_status st = nb_grid_scratch(g, NB_F64, 1, 1, &y2);
     HaloSync hs;
     nb_field *xin = x, *yin = y, *xo = x2, *yo = y2;
+    // single process: every iteration writes its tile partials into its own
+    // slice and ONE finalize produces all the dots (same trees, same bits as
+    // a finalize per iteration); across processes, one finalize per iteration
+    const bool defer = st == NB_OK && iters > 0 && !(g->comm && g->comm->world > 1) && !getenv("NB_C1_FIN_EACH");
+    if (defer) {
+        const int64_t need = (int64_t)iters * g->nz * g->T;
+        if (g->c1_cap < need) {
+            cudaFree(g->c1_tp);
+            cudaFree(g->c1_psum);
+            g->c1_tp = g->c1_psum = nullptr;
+            g->c1_cap = 0;
+            NB_CUDA(cudaMalloc(&g->c1_tp, sizeof(double) * need));
+            NB_CUDA(cudaMalloc(&g->c1_psum, sizeof(double) * iters * g->nz));
+            g->c1_cap = need;
+        }
+    }
     auto loop = [&]() -> nb_status {
         nb_status s = NB_OK;
+        double *tp0 = g->tp;
         for (int k = 0; k < iters && s == NB_OK; ++k) {
             MsrFields F{xin, yin, xo, yo, nullptr};
+            if (defer) g->tp = g->c1_tp + (int64_t)k * g->nz * g->T;  // this iteration's slice
             s = msr_step_fields<MSR_C1>(g, occ, F, a, 0.0, 0, nullptr, hs);
-            if (s == NB_OK) s = nb_reduce_finalize(g, 1, FIN_STORE, nullptr, k);
+            g->tp = tp0;
+            if (s == NB_OK && !defer) s = nb_reduce_finalize(g, 1, FIN_STORE, nullptr, k);
             std::swap(xin, xo);
             std::swap(yin, yo);
         }
+        if (s == NB_OK && defer) s = nb_c1_finalize_all(g, iters);
         return s;
     };
     // the loop is launch-latency bound at small sizes (C1: 64^3): replay it
