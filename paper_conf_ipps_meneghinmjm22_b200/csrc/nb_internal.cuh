@@ -167,7 +167,7 @@ struct nb_grid {
     cudaGraphExec_t c1_exec = nullptr;
     const void *c1_x = nullptr, *c1_y = nullptr;
     double c1_a = 0.0;
-    int c1_iters = -1, c1_occ = -1;
+    int c1_iters = -1, c1_occ = -1, c1_defer = -1;
     int64_t c1_launches = 0;
     // C1 tile partials / plane sums of all iterations of one call (single
     // process: one finalize per call instead of one per iteration)

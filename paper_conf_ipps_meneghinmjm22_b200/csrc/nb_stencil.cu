@@ -644,7 +644,7 @@ extern "C" nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, i
     if (graph) {
         const int fl = g->first_local;
         const bool hit = g->c1_exec && g->c1_x == x->base[fl] && g->c1_y == y->base[fl] && g->c1_a == a &&
-                         g->c1_iters == iters && g->c1_occ == (int)occ;
+                         g->c1_iters == iters && g->c1_occ == (int)occ && g->c1_defer == (int)defer;
         if (!hit) {
             if (g->c1_exec) cudaGraphExecDestroy(g->c1_exec);
             g->c1_exec = nullptr;
@@ -665,6 +665,7 @@ extern "C" nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, i
                 g->c1_a = a;
                 g->c1_iters = iters;
                 g->c1_occ = (int)occ;
+                g->c1_defer = (int)defer;
             }
         } else {  // the replay ends where the captured loop ended
             for (int k = 0; k < iters; ++k) {

@@ -229,9 +229,15 @@ def test_c1_graph_replay_and_rebuild_bit_exact(parts, monkeypatch):
     ox, oy, od2 = oracle.c1_loop(ox, 0.125, 4, y0=oy)
     ox, oy, od3 = oracle.c1_loop(ox, 0.25, 3, y0=oy)
     out = {}
-    for mode in ("graph", "eager"):
-        if mode == "eager":
+    for mode in ("graph", "graph_fin_each", "eager", "eager_fin_each"):
+        # the loop's dots: one finalize per call over per-iteration slices
+        # (default, single process) or one finalize per iteration
+        if mode.startswith("eager"):
             monkeypatch.setenv("NB_NO_GRAPH", "1")
+        if mode.endswith("fin_each"):
+            monkeypatch.setenv("NB_C1_FIN_EACH", "1")
+        else:
+            monkeypatch.delenv("NB_C1_FIN_EACH", raising=False)
         with grid(dims, parts) as g:
             fx, fy = field(g, x0), field(g, np.zeros_like(x0))
             d1 = nb.nb_map_stencil_reduce(fx, fy, 0.125, 4, nb.OCC_TWO_WAY)
@@ -248,8 +254,9 @@ def test_c1_graph_replay_and_rebuild_bit_exact(parts, monkeypatch):
         assert np.array_equal(gx, ox) and np.array_equal(gy, oy), mode
         for d, o in ((d1, od1), (d2, od2), (d3, od3)):
             assert np.max(np.abs(d - o) / np.abs(o)) <= 1e-12, mode
-    for a, b in zip(out["graph"], out["eager"]):
-        assert np.array_equal(a, b)
+    for m in ("graph_fin_each", "eager", "eager_fin_each"):
+        for a, b in zip(out["graph"], out[m]):
+            assert np.array_equal(a, b), m
 
 
 def test_c1_real_regime_vs_oracle():
