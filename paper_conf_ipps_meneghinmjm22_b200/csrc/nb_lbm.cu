@@ -99,7 +99,12 @@ __device__ __forceinline__ void lbm_collide_store(const float (&f)[Q19], const L
 }
 
 template <bool PERIODIC>
-__global__ void __launch_bounds__(128) k_lbm_d3q19(LbmArgs A, int zb) {
+// x-threads per CTA of the twoPop D3Q19 step (256: 3.18 -> 3.10 ms at
+// 512^3 against 128; 512 is slower, 3.75)
+#ifndef NB_LBM_BX
+#define NB_LBM_BX 256
+#endif
+__global__ void __launch_bounds__(NB_LBM_BX) k_lbm_d3q19(LbmArgs A, int zb) {
     const int x = blockIdx.x * blockDim.x + threadIdx.x;
     const int y = blockIdx.y;
     const int zl = zb + blockIdx.z;
@@ -394,7 +399,7 @@ static nb_status launch_lbm(nb_grid *g, int p, nb_field *fin, nb_field *fout, co
         if (ze == g->parts[p].nz() && nb_reachable(fout, hi))
             for (int i = 9; i < 14; ++i) A.rem_hi[i] = (float *)fout->base[hi] + (int64_t)i * lcs(fout, hi);
     }
-    dim3 blk(128), grd((g->nx + 127) / 128, g->ny, ze - zb);
+    dim3 blk(NB_LBM_BX), grd((g->nx + NB_LBM_BX - 1) / NB_LBM_BX, g->ny, ze - zb);
     LaunchScope ls(g, g->cs, "k_lbm_d3q19");
     if (per)
         k_lbm_d3q19<true><<<grd, blk, 0, g->cs>>>(A, zb);
@@ -496,7 +501,7 @@ struct LbmAAArgs {
 };
 
 template <bool EVEN, bool PERIODIC>
-__global__ void __launch_bounds__(128) k_lbm_aa(LbmAAArgs A) {
+__global__ void __launch_bounds__(128) k_lbm_aa(LbmAAArgs A) {  // 128 wide: 256 was slower here
     const int x = blockIdx.x * blockDim.x + threadIdx.x;
     const int y = blockIdx.y;
     const int zl = blockIdx.z;
