@@ -501,7 +501,10 @@ struct LbmAAArgs {
 };
 
 template <bool EVEN, bool PERIODIC>
-__global__ void __launch_bounds__(128) k_lbm_aa(LbmAAArgs A) {  // 128 wide: 256 was slower here
+#ifndef NB_AA_BX
+#define NB_AA_BX 32
+#endif
+__global__ void __launch_bounds__(NB_AA_BX) k_lbm_aa(LbmAAArgs A) {  // 32 wide: 3.44 ms/step at 512^3 (64: 3.62, 128: 3.69, 256: 4.0)
     const int x = blockIdx.x * blockDim.x + threadIdx.x;
     const int y = blockIdx.y;
     const int zl = blockIdx.z;
@@ -611,7 +614,7 @@ extern "C" nb_status nb_lbm_step_aa(nb_field *f, const nb_lbm_params *prm, int32
                         A.dn[i] = (float *)f->base[lo] + (int64_t)i * lcs(f, lo) + (int64_t)g->parts[lo].nz() * f->ps;
                 }
             }
-            dim3 blk(128), grd((g->nx + 127) / 128, g->ny, A.g.nzl);
+            dim3 blk(NB_AA_BX), grd((g->nx + NB_AA_BX - 1) / NB_AA_BX, g->ny, A.g.nzl);
             LaunchScope ls(g, g->cs, "k_lbm_aa");
             if (even)
                 per ? k_lbm_aa<true, true><<<grd, blk, 0, g->cs>>>(A) : k_lbm_aa<true, false><<<grd, blk, 0, g->cs>>>(A);
