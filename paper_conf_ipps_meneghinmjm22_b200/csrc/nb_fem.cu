@@ -620,7 +620,10 @@ __device__ __forceinline__ void fem_edge_col(int e, int nx, int ny, int &x, int 
 }
 
 template <int K>
-__global__ void __launch_bounds__(128) k_fem_surface(FemArgs A, PGeo g, int zb, int ze, FemSurf S) {
+#ifndef NB_FSURF_BX
+#define NB_FSURF_BX 128
+#endif
+__global__ void __launch_bounds__(NB_FSURF_BX) k_fem_surface(FemArgs A, PGeo g, int zb, int ze, FemSurf S) {
     if ((K == FEM_CG_Q || K == FEM_CG_A) && A.sc->status != 0) return;
     const int nzl = ze - zb;
     const int64_t n1 = (int64_t)S.ncol_edge * nzl, n2 = (int64_t)S.nin * S.nzs;
@@ -1325,9 +1328,9 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
             }
             const int64_t n = (int64_t)S.ncol_edge * (ze - zb) + (int64_t)S.nin * S.nzs;
             if (n > 0) {
-                const int blocks = (int)std::min<int64_t>((n + 127) / 128, 1 << 30);
+                const int blocks = (int)std::min<int64_t>((n + NB_FSURF_BX - 1) / NB_FSURF_BX, 1 << 30);
                 LaunchScope ls(g, g->cs, "k_fem_surface");
-                k_fem_surface<K><<<blocks, 128, 0, g->cs>>>(A, geo, zb, ze, S);
+                k_fem_surface<K><<<blocks, NB_FSURF_BX, 0, g->cs>>>(A, geo, zb, ze, S);
             }
             if (ncols > 0) {
                 dim3 fg((ncols + 63) / 64, (ze - zb + FZC - 1) / FZC);
