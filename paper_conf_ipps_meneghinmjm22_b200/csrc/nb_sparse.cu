@@ -559,24 +559,36 @@ constexpr int NSB = NB_SP_NSB;
 template <int K>
 __global__ void NB_SP_LB k_sp(SpArgs A) {
     __shared__ double sw[NSB][SEG / 32];
+#if NB_SP_EARLY_STATUS
     if (K >= SPK_CG_MAP && K <= SPK_CG_R && A.sc->status != 0) return;
+#endif
     const int t = threadIdx.x;
+    // the segment-table entries do not depend on the solver status: load
+    // them first so the status load and the table loads overlap (one
+    // dependent hop fewer before the connectivity / operand loads)
+    int e[NSB];
+#pragma unroll
+    for (int k = 0; k < NSB; ++k) {
+        const int64_t q = (int64_t)blockIdx.x * NSB + k;
+        e[k] = q < A.nseg ? __ldg(A.seg + A.seg0 + q) : -1;  // non-empty segment: plane << 16 | index
+    }
+#if !NB_SP_EARLY_STATUS
+    if (K >= SPK_CG_MAP && K <= SPK_CG_R && A.sc->status != 0) return;
+#endif
     int zl[NSB], sg[NSB];
     int64_t i[NSB], jj[NSB];
     bool valid[NSB];
 #pragma unroll
     for (int k = 0; k < NSB; ++k) {
-        const int64_t q = (int64_t)blockIdx.x * NSB + k;
         zl[k] = -1;
         sg[k] = 0;
         valid[k] = false;
         jj[k] = 0;
-        if (q < A.nseg) {
-            const int e = A.seg[A.seg0 + q];  // non-empty segment: plane << 16 | index
-            zl[k] = e >> 16;
-            sg[k] = e & 0xffff;
-            jj[k] = A.pstart[zl[k]] + (int64_t)sg[k] * SEG + t;
-            valid[k] = jj[k] < A.pstart[zl[k] + 1];
+        if (e[k] >= 0) {
+            zl[k] = e[k] >> 16;
+            sg[k] = e[k] & 0xffff;
+            jj[k] = __ldg(A.pstart + zl[k]) + (int64_t)sg[k] * SEG + t;
+            valid[k] = jj[k] < __ldg(A.pstart + zl[k] + 1);
         }
         i[k] = A.hl + jj[k];  // buffer index of own cell
     }
