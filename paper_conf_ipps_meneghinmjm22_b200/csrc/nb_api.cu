@@ -286,7 +286,7 @@ __global__ void __launch_bounds__(256) k_halo_copy(const __grid_constant__ CopyB
     while (d + 1 < cb.n && cb.bstart[d + 1] <= b) ++d;
     const uint64_t w0 = (uint64_t)(b - cb.bstart[d]) * CopyBatch::CHUNK;
     const uint64_t w1 = min(w0 + CopyBatch::CHUNK, cb.words[d]);
-    if ((cb.vec >> d) & 1u) {
+    if ((cb.vec >> d) & 1ull) {
         const uint4 *s = (const uint4 *)cb.src[d];
         uint4 *t = (uint4 *)cb.dst[d];
         for (uint64_t i = w0 + threadIdx.x; i < w1; i += 256) t[i] = __ldcs(s + i);
@@ -768,6 +768,8 @@ extern "C" nb_status nb_field_destroy(nb_field *f) {
     cudaStreamSynchronize(f->g->cs);
     cudaStreamSynchronize(f->g->hs);
     if (nb_is_peer(f->g)) nb_peer_field_unmap(f);  // collective: closes the mappings, then a barrier
+    for (size_t p = 0; p < f->base.size(); ++p)  // cached tensor maps over these buffers
+        if (f->base[p] && p < f->bytes.size()) nb_tma_forget_range(f->base[p], f->base[p] + f->bytes[p]);
     if (!f->borrowed)
         for (size_t p = 0; p < f->base.size(); ++p)
             if (f->base[p] && !(p < f->mapped.size() && f->mapped[p])) cudaFree(f->base[p]);
@@ -842,13 +844,17 @@ __global__ void k_fill_gen(T *base, PGeo g, int64_t cstride, int card, int kind,
                            double a, double b, double h) {
     int x = blockIdx.x * blockDim.x + threadIdx.x;
     int y = blockIdx.y;
-    int zl = blockIdx.z % g.nzl;
-    int c = blockIdx.z / g.nzl;
-    if (x >= g.nx || c >= card) return;
-    int z = g.z0 + zl;
-    uint64_t gidx = (uint64_t)x + (uint64_t)g.nx * ((uint64_t)y + (uint64_t)g.ny * ((uint64_t)z + (uint64_t)g.NZ * c));
-    double v = nb_gen(kind, seed, gidx, a, b, x, y, z, h);
-    base[(int64_t)c * cstride + (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x] = (T)v;
+    if (x >= g.nx) return;
+    // (plane, component) pairs grid-strided over blockIdx.z (gridDim.z <= 65535)
+    for (int64_t zc = blockIdx.z; zc < (int64_t)g.nzl * card; zc += gridDim.z) {
+        int zl = (int)(zc % g.nzl);
+        int c = (int)(zc / g.nzl);
+        int z = g.z0 + zl;
+        uint64_t gidx =
+            (uint64_t)x + (uint64_t)g.nx * ((uint64_t)y + (uint64_t)g.ny * ((uint64_t)z + (uint64_t)g.NZ * c));
+        double v = nb_gen(kind, seed, gidx, a, b, x, y, z, h);
+        base[(int64_t)c * cstride + (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x] = (T)v;
+    }
 }
 
 extern "C" nb_status nb_field_fill(nb_field *f, nb_fill kind, uint64_t seed, double a, double b) {
@@ -864,7 +870,7 @@ extern "C" nb_status nb_field_fill(nb_field *f, nb_fill kind, uint64_t seed, dou
     for (int p = 0; p < g->nparts; ++p) {
         if (!g->parts[p].local) continue;
         PGeo geo = pgeo(f, p);
-        dim3 blk(128), grd((g->nx + 127) / 128, g->ny, geo.nzl * f->card);
+        dim3 blk(128), grd((g->nx + 127) / 128, g->ny, (unsigned)std::min<int64_t>((int64_t)geo.nzl * f->card, 65535));
         LaunchScope ls(g, g->cs, "k_fill_gen");
         if (f->dt == NB_F64)
             k_fill_gen<double><<<grd, blk, 0, g->cs>>>((double *)f->base[p], geo, dense_cs(f, p), f->card,

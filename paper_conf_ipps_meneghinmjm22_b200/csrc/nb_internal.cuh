@@ -326,20 +326,23 @@ struct CopyBatch {
     const void *src[MAX];
     uint64_t words[MAX];     // number of 16-byte (vec) or 4-byte words
     uint32_t bstart[MAX + 1];
-    uint32_t vec;            // bit i: descriptor i uses 16-byte words
+    uint64_t vec;            // bit i: descriptor i uses 16-byte words
     int n = 0;
+    static_assert(MAX <= 64, "CopyBatch::vec holds one bit per descriptor");
     CopyBatch() : vec(0) { bstart[0] = 0; }
     void add(void *d, const void *s_, size_t bytes) {
         bool v = ((uintptr_t)d % 16 == 0) && ((uintptr_t)s_ % 16 == 0) && (bytes % 16 == 0);
         dst[n] = d;
         src[n] = s_;
         words[n] = v ? bytes / 16 : bytes / 4;
-        if (v) vec |= 1u << n;
+        if (v) vec |= 1ull << n;
         bstart[n + 1] = bstart[n] + (uint32_t)((words[n] + CHUNK - 1) / CHUNK);
         ++n;
     }
 };
 nb_status nb_launch_copy_batch(nb_grid *g, const CopyBatch &cb, cudaStream_t s);
+// drop cached TMA tensor maps whose base address lies in [lo, hi) (nb_tma.cu)
+void nb_tma_forget_range(const void *lo, const void *hi);
 
 // halo helpers (nb_api.cu)
 nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down,

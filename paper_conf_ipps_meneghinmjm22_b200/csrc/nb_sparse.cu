@@ -88,8 +88,9 @@ extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t 
         counts[z] = c;
     }
     if (nparts < 1 || nparts > nz) NB_FAIL(NB_EINVAL, "nb_grid_create_sparse: bad nparts %d", nparts);
-    if (nz > 65535 || plane > (int64_t)SEG * 65535)
-        NB_FAIL(NB_EUNSUPPORTED, "nb_grid_create_sparse: segment table limits (nz <= 65535, Nx*Ny <= 16.7M)");
+    // segment entries are int32 (zl << 16 | k) with -1 as the sentinel: zl <= 32767 keeps them >= 0
+    if (nz > 32767 || plane > (int64_t)SEG * 65535)
+        NB_FAIL(NB_EUNSUPPORTED, "nb_grid_create_sparse: segment table limits (nz <= 32767, Nx*Ny <= 16.7M)");
     std::vector<int32_t> zb(nparts + 1);
     NB_TRY(nb_partition_plan_weighted(nz, counts.data(), nparts, zb.data()));
     if (nparts > 1)

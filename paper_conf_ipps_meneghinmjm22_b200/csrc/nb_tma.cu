@@ -386,11 +386,13 @@ nb_status tmap_for(const void *base, const PGeo &g, int box, CUtensorMap *out) {
     return box == 0 ? tmap_box(base, g, DOT_TX + 4, DOT_TY + 2, out) : tmap_box(base, g, DOT_TX, DOT_TY, out);
 }
 
-// drop cached maps of a freed buffer
-void nb_tma_forget(const void *base) {
+// drop cached maps whose base lies in [lo, hi) (a freed or unwrapped buffer)
+void nb_tma_forget_range(const void *lo, const void *hi) {
     std::lock_guard<std::mutex> lk(g_tmap_mu);
-    for (auto it = g_tmaps.begin(); it != g_tmaps.end();)
-        it = std::get<0>(it->first) == base ? g_tmaps.erase(it) : std::next(it);
+    for (auto it = g_tmaps.begin(); it != g_tmaps.end();) {
+        const char *b = (const char *)std::get<0>(it->first);
+        it = (b >= (const char *)lo && b < (const char *)hi) ? g_tmaps.erase(it) : std::next(it);
+    }
 }
 
 bool nb_tma_enabled() {

@@ -489,3 +489,42 @@ def test_halo_stream_mode_bitwise_equals_fused():
                     f.close()
         for u, v in zip(outs[0], outs[1]):
             assert np.array_equal(u, v), occ
+
+
+def test_lbm_halo_stream_many_partitions_bitwise_equals_fused():
+    """HALO_STREAM LBM on 6 virtual partitions puts 10 messages x 5
+    populations = 50 plane copies into one exchange (more than 32 CopyBatch
+    descriptors); it must equal the fused halo stores bit for bit."""
+    dims = (24, 20, 30)
+    f0 = lbm_state(dims, 5)
+    outs = []
+    for mode in (nb.HALO_FUSED, nb.HALO_STREAM):
+        with grid(dims, 6) as g:
+            g.set_halo_mode(mode)
+            a, c = field(g, f0, "f32", 19), field(g, dtype="f32", card=19)
+            a2, _ = nb.nb_lbm_step(a, c, 1.1, 3, occ=nb.OCC_STANDARD)
+            outs.append(a2.download())
+            a.close(), c.close()
+    assert np.array_equal(outs[0], outs[1])
+    exp = f0.astype(np.float64)
+    for _ in range(3):
+        exp = oracle.lbm_step(exp, 1.1)
+    assert np.max(np.abs(outs[0] - exp) / np.abs(exp)) < 1e-5
+
+
+@pytest.mark.parametrize("parts,occ", [(1, nb.OCC_TWO_WAY), (3, nb.OCC_EXTENDED), (2, nb.OCC_NONE)])
+def test_large_c1_tma_chain_exact_regime_vs_oracle(parts, occ):
+    """Above 2^21 cells the fused C1 chain runs on the TMA-staged kernel
+    (k_cgA_tma<., C1>).  In the exact regime (integer x0, a = 1/8, SURVEY
+    §8(c) c9 pin 1) x_10 and y_10 must equal the oracle bit for bit."""
+    dims = (130, 129, 131)
+    assert dims[0] * dims[1] * dims[2] > 2 ** 21
+    x0 = synth.int_uniform(dims, seed=5)
+    ox, oy, od = oracle.c1_loop(x0, 0.125, 10)
+    with grid(dims, parts) as g:
+        fx, fy = field(g, x0), field(g, np.zeros_like(x0))
+        dots = nb.nb_map_stencil_reduce(fx, fy, 0.125, 10, occ)
+        assert np.array_equal(fx.download(), ox)
+        assert np.array_equal(fy.download(), oy)
+        assert np.max(np.abs(dots - od) / np.abs(od)) <= 1e-12
+        fx.close(), fy.close()

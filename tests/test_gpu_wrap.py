@@ -89,3 +89,32 @@ def test_wrap_rejects_bad_pointers():
             nb.Field.wrap(g, [t[1:]])  # 8-byte aligned only
         with pytest.raises(nb.NbError):
             nb.Field.wrap(g, [torch.empty(n, dtype=torch.float64)])  # host memory
+
+
+@pytest.mark.parametrize("card,parts", [(19, 2), (19, 3), (3, 7)])
+def test_halo_update_many_descriptors_fills_every_halo_plane(card, parts):
+    """nb_halo_update batches all device-local plane copies of one exchange
+    into ONE launch (CopyBatch): 19 components x 2 partitions is 38
+    descriptors, 19 x 3 is 76 (more than one batch) — every halo plane of
+    every component must equal the neighbour's boundary plane bit for bit
+    (descriptors 32..47 once copied only a quarter of their plane)."""
+    dims = (45, 19, 23)
+    h = synth.uniform(dims, card=card, seed=21)
+    with nb.Grid(dims, nparts=parts, devices=[0] * parts) as g:
+        f = nb.Field.empty_torch(g, card=card, outside=-3.0)
+        f.upload(h)
+        f.halo_update()
+        g.sync()
+        nx, ny, _ = dims
+        for p in range(parts):
+            info = g.partition_info(p)
+            z0, z1 = info["z_begin"], info["z_end"]
+            _, pitch, ps, cs = f.partition_ptr(p)
+            buf = f.buffers[p]
+            for c in range(card):
+                for zl, zg in ((-1, z0 - 1), (z1 - z0, z1)):
+                    plane = buf[c * cs + (zl + 1) * ps: c * cs + (zl + 2) * ps].view(ny, pitch)[:, :nx]
+                    got = plane.cpu().numpy()
+                    exp = h[c, zg] if 0 <= zg < dims[2] else np.full((ny, nx), -3.0)
+                    assert np.array_equal(got, exp), (p, c, zl)
+        f.close()

@@ -181,3 +181,58 @@ def test_fem_brute_force_assembled_matrix():
     assert res.converged == 1
     assert np.max(np.abs(Kd @ x.ravel() - b.ravel())) < 1e-11
     assert np.allclose(x.ravel(), np.linalg.solve(Kd, b.ravel()), atol=1e-10)
+
+
+# ---- Neumann load placement ("the z = N-1 plane had outward
+# pressure"; consistent nodal loads, tributary areas
+# 1 / 1/2 / 1/4) ------------------------------------------------------------
+@pytest.mark.parametrize("dims,dirichlet", [((5, 5, 5), True), ((6, 4, 3), True), ((6, 4, 3), False),
+                                            ((4, 5, 2), True)])
+def test_fem_rhs_exact_tributary_loads_on_top_plane(dims, dirichlet):
+    """b is zero except b_z on the top node plane z = Nz-1, where it is p at
+    interior nodes, p/2 on edges and p/4 at corners (dyadic: bit-exact).
+    A load on plane Nz-2, on an element's bottom nodes or in x/y fails."""
+    nx, ny, nz = dims
+    p = 3.0
+    b = oracle.fem_rhs(dims, p, dirichlet_z0=dirichlet)
+    assert np.all(b[0] == 0) and np.all(b[1] == 0)
+    assert np.all(b[2, :nz - 1] == 0)
+    ex = np.where((np.arange(nx) == 0) | (np.arange(nx) == nx - 1), 0.5, 1.0)
+    ey = np.where((np.arange(ny) == 0) | (np.arange(ny) == ny - 1), 0.5, 1.0)
+    expect = p * ey[:, None] * ex[None, :]  # [y][x] tributary area of the top face
+    assert np.array_equal(b[2, nz - 1], expect)
+
+
+def test_fem_rhs_virtual_work_on_stepped_mask():
+    """Consistent loads integrate every bilinear test function v(x, y, z)
+    exactly over the loaded faces: sum_a b_a v_a = p * sum_faces int v dA.
+    On a two-level step (columns x >= 3 cut at z = 2) the exposed top faces
+    are the upper plateau at z = 4 and the lower one at z = 2; v = z fixes
+    the plane of every face, v = x, y, x*y its position."""
+    nx, ny, nz = 6, 4, 5
+    mask = np.ones((nz, ny, nx), dtype=np.uint8)
+    mask[3:, :, 4:] = 0  # nodes x >= 4 exist only up to z = 2 -> elements ex >= 3 stop at ez = 1
+    p = 1.0
+    b = oracle.fem_rhs((nx, ny, nz), p, mask=mask)
+    assert np.all(b[:2] == 0)
+    zz, yy, xx = np.meshgrid(np.arange(nz), np.arange(ny), np.arange(nx), indexing="ij")
+    # exposed faces: [ex0, ex1) x [0, ny-1) at height z (analytic integrals of v over unit squares)
+    faces = [(0, 3, 4.0), (3, 5, 2.0)]
+
+    def integral(fn):
+        tot = 0.0
+        for x0, x1, z in faces:
+            for ex_ in range(x0, x1):
+                for ey_ in range(ny - 1):
+                    tot += fn(ex_, ey_, z)
+        return tot
+    tests = {
+        "1": (np.ones_like(xx, dtype=float), lambda x, y, z: 1.0),
+        "z": (zz.astype(float), lambda x, y, z: z),
+        "x": (xx.astype(float), lambda x, y, z: x + 0.5),
+        "y": (yy.astype(float), lambda x, y, z: y + 0.5),
+        "xy": ((xx * yy).astype(float), lambda x, y, z: (x + 0.5) * (y + 0.5)),
+        "xz": ((xx * zz).astype(float), lambda x, y, z: (x + 0.5) * z),
+    }
+    for name, (v, fn) in tests.items():
+        assert abs(float(np.sum(b[2] * v)) - p * integral(fn)) < 1e-12, name
