@@ -163,101 +163,137 @@ def ncu_traffic(kernel: str):
 
 
 # ---------------------------------------------------------------------------
-def bench_cg(args, world, rank, local):
+def comm_profile(g, iters):
+    """Per-iteration device time of the communication kernels from a profiled
+    (event-bracketed, eager) pass: reductions (k_finalize: plane sums, the
+    cross-rank exchange of the peer transport, alpha / beta) and halo
+    signalling / waiting (k_peer_*) or batched halo copies (k_halo_copy).
+    The halo planes themselves are stored by the boundary kernels (fused
+    transport), so their bytes are inside the compute kernels' time."""
+    out = {}
+    for key, name in (("reduction", "k_finalize"), ("halo_sync", "k_peer_"), ("halo_copy", "k_halo_copy")):
+        k, ms = g.profile_read(name)
+        out[key + "_ms_per_iter"] = ms / max(iters, 1)
+        out[key + "_launches_per_iter"] = k / max(iters, 1)
+    return out
+
+
+def bench_cg(args, world, rank, local, weak=False, with_e2e=True):
+    """C2 Poisson CG.  Strong scaling: the n^3 grid split over `world` ranks;
+    weak: n x n x (n * world), an n^3 slab per rank."""
     import numpy as np
     import torch
 
     import paper_conf_ipps_meneghinmjm22_b200 as nb
     n = args.n
-    dims = (n, n, n)
-    cells = n ** 3
+    dims = (n, n, n * world) if weak else (n, n, n)
+    cells = dims[0] * dims[1] * dims[2]
+    steps = args.steps
     comm = nb.Comm.from_torch_distributed(local) if world > 1 else None
     g = nb.Grid(dims, nparts=world, comm=comm) if comm else nb.Grid(dims, nparts=1, devices=[local])
     stream = torch.cuda.ExternalStream(g.stream())
     b, x = nb.Field(g), nb.Field(g)
-    b.fill(nb.FILL_POISSON_RHS)
+    if weak:  # POISSON_RHS needs a cube: a seeded uniform right-hand side
+        b.fill_uniform(seed=2)
+    else:
+        b.fill(nb.FILL_POISSON_RHS)
     x.fill_const(0.0)
     occ = nb.OCC_NAMES[args.occ]
     cg = nb.CG(x, b, occ=occ)
     cg.iterate(args.warmup)
-    cg.prepare(args.steps)  # graph instantiation outside the timed region
+    cg.prepare(steps)  # graph instantiation outside the timed region
     g.sync()
     l0 = g.launch_count()
-    ms, clocks = timed(world, stream, lambda: cg.iterate(args.steps), local)
+    ms, clocks = timed(world, stream, lambda: cg.iterate(steps), local)
     launches = g.launch_count() - l0
     res = cg.finish()
     cg.close()
     t = ms / 1e3
-    mlups = cells * args.steps / t / 1e6
+    mlups = cells * steps / t / 1e6
     hbm, peak_kind = peaks()
-    # per-kernel durations: a profiled (event-bracketed, eager) pass
+    # per-kernel durations: a profiled (event-bracketed, eager) pass; the
+    # roofline divides one iteration's algorithmic bytes by the SUM of that
+    # kernel's launches in one iteration (at N > 1 phase A is an interior
+    # launch plus boundary-plane launches)
     x.fill_const(0.0)
-    g.profile(True)
     cg = nb.CG(x, b, occ=occ)
-    cg.iterate(args.prof_steps)
+    cg.iterate(1)
+    g.profile(True)
+    it = args.prof_steps
+    cg.iterate(it)
     na, msa = g.profile_read("k_msr_cgA")
     nbb, msb = g.profile_read("k_cg_B")
-    nfin, msf = g.profile_read("k_finalize")
+    comm_t = comm_profile(g, it)
     g.profile(False)
     cg.finish()
     cg.close()
     local_cells = cells // world
-    a_avg, b_avg = msa / max(na, 1), msb / max(nbb, 1)
-    dom = ("k_msr_cgA", CG_A_BYTES, a_avg, na) if msa >= msb else ("k_cg_B", CG_B_BYTES, b_avg, nbb)
+    a_it, b_it = msa / it, msb / it
+    dom = ("k_msr_cgA", CG_A_BYTES, a_it, na / it) if msa >= msb else ("k_cg_B", CG_B_BYTES, b_it, nbb / it)
     achieved = dom[1] * local_cells / (dom[2] / 1e3) / 1e9
     tr = ncu_traffic(dom[0])
+    kind = "weak" if weak else "strong"
     out = {
-        "metric": METRIC, "value": mlups, "unit": "MLUPS", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "strong",
+        "metric": METRIC, "value": mlups, "unit": "MLUPS", "n_gpus": world, "steps": steps,
+        "warmup": args.warmup, "ms_per_step": ms / steps, "higher_is_better": True, "scaling": kind,
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"C2 Poisson FD CG 7-point fp64 {n}^3 dense (configs[1])",
-                   "rhs": "b = h^2 f, manufactured u* = g(x)g(y)g(z)", "x0": 0,
-                   "parts": world, "occ": args.occ, "schedule": "2-phase, 64 B/cell/iter",
-                   "l2": "inputs larger than L2 (5 fp64 fields of %.2f GB each)" % (cells * 8 / 1e9)},
-        "hbm_gbs": CG_BYTES_PER_CELL * cells * args.steps / t / 1e9,
-        "hbm_frac": CG_BYTES_PER_CELL * cells * args.steps / t / 1e9 / hbm,
+        "config": {"workload": (f"C2 Poisson FD CG 7-point fp64 {n}^3 per GPU, weak scaling "
+                                f"({dims[0]}x{dims[1]}x{dims[2]})" if weak else
+                                f"C2 Poisson FD CG 7-point fp64 {n}^3 dense (configs[1])"),
+                   "rhs": "uniform[-1,1) seed 2" if weak else "b = h^2 f, manufactured u* = g(x)g(y)g(z)",
+                   "x0": 0, "parts": world, "occ": args.occ, "schedule": "2-phase, 64 B/cell/iter",
+                   "l2": "inputs larger than L2 (5 fp64 fields of %.2f GB per GPU)" % (local_cells * 8 / 1e9)},
+        "hbm_gbs": CG_BYTES_PER_CELL * cells * steps / t / 1e9,
+        "hbm_frac": CG_BYTES_PER_CELL * cells * steps / t / 1e9 / hbm / world,
         "roofline": {"bound": "hbm", "kernel": dom[0], "achieved": achieved, "peak": hbm, "unit": "GB/s",
                      "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": tr,
-                     "algorithmic_bytes_per_launch": dom[1] * local_cells,
-                     "launch_ms": dom[2],
-                     "kernel_ms": {"k_msr_cgA": a_avg, "k_cg_B": b_avg, "k_finalize": msf / max(nfin, 1)}},
+                     "algorithmic_bytes_per_iter": dom[1] * local_cells,
+                     "kernel_ms_per_iter": dom[2], "launches_per_iter": dom[3],
+                     "per_rank": world > 1,
+                     "kernel_ms": {"k_msr_cgA": a_it, "k_cg_B": b_it}},
+        "comm": comm_t,
         "gpu_launches": int(launches), "clocks": clocks,
         "cg_state": {"iters": res.iters, "rr0": res.rr0, "rr": res.rr},
     }
     if _SHARED_GPU:
-        out["note"] = ("ranks share one GPU (fewer GPUs than ranks): kernels of different ranks overlap and "
-                       "the peer-flag waits spin, so per-kernel times and the roofline are not meaningful here")
-    # ---- e2e: public API, host buffers, H2D and D2H inside the timed region
-    # (every rank holds the dense host logical view; nb_field_upload /
-    # download move only its own slab)
-    import synth
-    bh = torch.from_numpy(synth.poisson_poly_rhs(dims).reshape(-1)).pin_memory()
-    xh = torch.zeros(cells, dtype=torch.float64).pin_memory()
-    local_bytes = cells * 8 // world
+        out["note"] = SHARED_NOTE
+    if with_e2e:
+        # ---- e2e: public API, host buffers, H2D and D2H inside the timed
+        # region (every rank holds the dense host logical view;
+        # nb_field_upload / download move only its own slab)
+        import synth
+        bh = torch.from_numpy(synth.poisson_poly_rhs(dims).reshape(-1)).pin_memory()
+        xh = torch.zeros(cells, dtype=torch.float64).pin_memory()
+        local_bytes = cells * 8 // world
 
-    def e2e():
-        b.upload_async(bh.data_ptr())
-        x.upload_async(xh.data_ptr())
-        s = nb.CG(x, b, occ=occ)
-        s.prepare(args.steps)
-        s.iterate(args.steps)
-        s.finish()
-        s.close()
-        x.download(xh)
-    e2e()  # warm
-    ms_e, _ = timed(world, stream, e2e, local)
-    out["e2e"] = {"value": cells * args.steps / (ms_e / 1e3) / 1e6, "unit": "MLUPS",
-                  "h2d_bytes_per_step": 2 * local_bytes / args.steps, "d2h_bytes_per_step": local_bytes / args.steps,
-                  "h2d_bytes_per_call": 2 * local_bytes, "d2h_bytes_per_call": local_bytes,
-                  "note": "per rank: upload b and x0 (own slab) from pinned host, CG create (r = b - Ax0), "
-                          "steps iterations, finish (deferred x update), download x (own slab); "
-                          "one e2e call (a whole solve of `steps` iterations) per timed region, max over ranks; "
-                          "bytes per step = bytes per call / steps"}
+        def e2e():
+            b.upload_async(bh.data_ptr())
+            x.upload_async(xh.data_ptr())
+            s = nb.CG(x, b, occ=occ)
+            s.prepare(steps)
+            s.iterate(steps)
+            s.finish()
+            s.close()
+            x.download(xh)
+        e2e()  # warm
+        ms_e, _ = timed(world, stream, e2e, local)
+        out["e2e"] = {"value": cells * steps / (ms_e / 1e3) / 1e6, "unit": "MLUPS",
+                      "h2d_bytes_per_step": 2 * local_bytes / steps, "d2h_bytes_per_step": local_bytes / steps,
+                      "h2d_bytes_per_call": 2 * local_bytes, "d2h_bytes_per_call": local_bytes,
+                      "note": "per rank: upload b and x0 (own slab) from pinned host, CG create (r = b - Ax0), "
+                              "steps iterations, finish (deferred x update), download x (own slab); "
+                              "one e2e call (a whole solve of `steps` iterations) per timed region, max over "
+                              "ranks; bytes per step = bytes per call / steps"}
     b.close(), x.close()
     g.close()
     if comm:
         comm.close()
     return out
+
+
+SHARED_NOTE = ("ranks share one GPU (fewer GPUs than ranks): kernels of different ranks overlap and the "
+               "peer-flag waits spin, so per-kernel times, communication times and the roofline are not "
+               "meaningful here")
 
 
 def lbm_omega(nx, u_lid=0.05, re=100.0):
@@ -289,13 +325,14 @@ def bench_lbm_run(n, steps, warmup, world, local, occ="standard"):
     g.profile(True)
     run(3)
     nk, msk = g.profile_read("k_lbm_d3q19")
+    comm_t = comm_profile(g, 3)
     g.profile(False)
     cells = n * n * n * world
     t = ms / 1e3
     hbm, peak_kind = peaks()
-    k_ms = msk / max(nk, 1) * (1 if world == 1 else 1)
     local_cells = n * n * n
-    # at N=1 with no OCC split one launch covers the whole grid
+    # per step: the sum of the step's launches (boundary planes + interior
+    # under Standard OCC at N > 1; one launch at N = 1)
     per_step_ms = msk / 3.0
     achieved = LBM_BYTES_PER_CELL * local_cells / (per_step_ms / 1e3) / 1e9
     res = {
@@ -308,9 +345,13 @@ def bench_lbm_run(n, steps, warmup, world, local, occ="standard"):
         "hbm_frac": LBM_BYTES_PER_CELL * cells * steps / t / 1e9 / hbm,
         "roofline": {"bound": "hbm", "kernel": "k_lbm_d3q19", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                      "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": ncu_traffic("k_lbm_d3q19"),
-                     "algorithmic_bytes_per_launch": LBM_BYTES_PER_CELL * local_cells, "launch_ms": k_ms},
+                     "algorithmic_bytes_per_step": LBM_BYTES_PER_CELL * local_cells,
+                     "kernel_ms_per_step": per_step_ms, "launches_per_step": nk / 3.0, "per_rank": world > 1},
+        "comm": comm_t,
         "gpu_launches": int(launches), "clocks": clocks,
     }
+    if _SHARED_GPU:
+        res["note"] = SHARED_NOTE
     st["a"].close(), st["b"].close()
     g.close()
     if comm:
@@ -436,13 +477,15 @@ def fp64_peak():
     return FP64_PEAK_DERIVED, "derived: 148 SMs x 64 FP64 lanes x 2 flop x 1.965 GHz"
 
 
-def _profiled_kernels(g, run, names):
+def _profiled_kernels(g, run, names, comm_iters=0):
     g.profile(True)
     run()
     out = {}
     for nm in names:
         k, ms = g.profile_read(nm)
         out[nm] = (k, ms)
+    if comm_iters:
+        out["comm"] = comm_profile(g, comm_iters)
     g.profile(False)
     return out
 
@@ -474,7 +517,10 @@ def bench_sparse_run(n, steps, warmup, world, local):
     cg.close()
     x.fill_const(0.0)
     cg = nb.CG(x, b)
-    prof = _profiled_kernels(g, lambda: cg.iterate(5), list(SPARSE_BYTES))
+    cg.iterate(1)
+    pit = 5
+    prof = _profiled_kernels(g, lambda: cg.iterate(pit), list(SPARSE_BYTES), comm_iters=pit)
+    comm_t = prof.pop("comm")
     cg.finish()
     cg.close()
     hbm, peak_kind = peaks()
@@ -482,7 +528,7 @@ def bench_sparse_run(n, steps, warmup, world, local):
     local_act = nact // world
     dom = max(prof, key=lambda k: prof[k][1])
     dk, dms = prof[dom]
-    achieved = SPARSE_BYTES[dom] * local_act / (dms / max(dk, 1) / 1e3) / 1e9
+    achieved = SPARSE_BYTES[dom] * local_act / (dms / pit / 1e3) / 1e9
     b.close(), x.close()
     g.close()
     if comm:
@@ -496,8 +542,11 @@ def bench_sparse_run(n, steps, warmup, world, local):
             "hbm_gbs": per_cell * nact * steps / t / 1e9, "hbm_frac": per_cell * nact * steps / t / 1e9 / hbm,
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm, "unit": "GB/s",
                          "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": ncu_traffic(dom),
-                         "kernel_ms": {k: v[1] / max(v[0], 1) for k, v in prof.items()}},
-            "gpu_launches": int(launches), "clocks": clocks}
+                         "per_rank": world > 1, "local_active_cells": local_act,
+                         "kernel_ms_per_iter": {k: v[1] / pit for k, v in prof.items()},
+                         "launches_per_iter": {k: v[0] / pit for k, v in prof.items()}},
+            "comm": comm_t, "gpu_launches": int(launches), "clocks": clocks,
+            **({"note": SHARED_NOTE} if _SHARED_GPU else {})}
 
 
 def bench_fem_run(n, steps, warmup, world, local):
@@ -525,7 +574,9 @@ def bench_fem_run(n, steps, warmup, world, local):
     x.fill_const(0.0)
     cg = nb.CG(x, b, op=nb.OP_FEM27)
     cg.iterate(1)  # the first iteration has no deferred x update: profile steady-state ones
-    prof = _profiled_kernels(g, lambda: cg.iterate(5), list(FEM_BYTES) + ["k_fem_surface"])
+    pit = 5
+    prof = _profiled_kernels(g, lambda: cg.iterate(pit), list(FEM_BYTES) + ["k_fem_surface"], comm_iters=pit)
+    comm_t = prof.pop("comm")
     cg.finish()
     cg.close()
     # K u alone (nb_fem27_apply): the FP64-ALU-bound stencil kernel
@@ -541,10 +592,10 @@ def bench_fem_run(n, steps, warmup, world, local):
     nodes = n ** 3
     local_nodes = nodes // world
     ak, ams = prof["k_fem_cg_a"]
-    a_avg = ams / max(ak, 1) / 1e3
+    a_avg = ams / pit / 1e3  # per iteration (interior + boundary launches)
     achieved = FEM_BYTES["k_fem_cg_a"] * local_nodes / a_avg / 1e9
     qk, qms = aprof["k_fem_apply"]
-    flops = FEM_FLOPS_PER_NODE * local_nodes / (qms / max(qk, 1) / 1e3) / 1e12
+    flops = FEM_FLOPS_PER_NODE * local_nodes / (qms / 5 / 1e3) / 1e12  # per nb_fem27_apply call
     per_node = sum(FEM_BYTES.values())
     b.close(), x.close()
     g.close()
@@ -559,12 +610,14 @@ def bench_fem_run(n, steps, warmup, world, local):
             "hbm_gbs": per_node * nodes * steps / t / 1e9, "hbm_frac": per_node * nodes * steps / t / 1e9 / hbm,
             "roofline": {"bound": "hbm", "kernel": "k_fem_cg_a", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                          "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": ncu_traffic("k_fem_cg_a"),
-                         "algorithmic_bytes_per_node": FEM_BYTES["k_fem_cg_a"],
-                         "kernel_ms": {k: v[1] / max(v[0], 1) for k, v in prof.items()}},
+                         "algorithmic_bytes_per_node": FEM_BYTES["k_fem_cg_a"], "per_rank": world > 1,
+                         "kernel_ms_per_iter": {k: v[1] / pit for k, v in prof.items()},
+                         "launches_per_iter": {k: v[0] / pit for k, v in prof.items()}},
             "apply_alu": {"bound": "alu", "kernel": "k_fem_apply (interior K u, surface nodes excluded)",
                           "achieved": flops, "peak": f64, "unit": "TFLOP/s", "frac": flops / f64,
                           "peak_kind": f64_kind, "flop_per_node": FEM_FLOPS_PER_NODE},
-            "gpu_launches": int(launches), "clocks": clocks}
+            "comm": comm_t, "gpu_launches": int(launches), "clocks": clocks,
+            **({"note": SHARED_NOTE} if _SHARED_GPU else {})}
 
 
 def bench_c1(local):
@@ -650,19 +703,39 @@ def bench_skeleton(local, n=512, parts=4, iters=10):
 
 
 # ---------------------------------------------------------------------------
-def _oracle_all_cores():
-    """The oracle runs on every host core (torchrun sets OMP_NUM_THREADS=1 in
-    each rank; the reference arm and cpu_baseline run on rank 0 alone)."""
+def host_info():
+    """CPU model, logical cores and RAM of the host running the oracle."""
+    model, mem = None, None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemTotal"):
+                mem = round(int(line.split()[1]) / 1024 / 1024, 1)
+                break
+    except OSError:
+        pass
+    return {"cpu_model": model, "logical_cores": os.cpu_count(), "ram_gib": mem,
+            "sched_affinity_cores": len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else None}
+
+
+def _oracle_threads(nthreads):
+    """The oracle on `nthreads` host threads (torchrun sets OMP_NUM_THREADS=1
+    in each rank; the reference arm and cpu_baseline run on rank 0 alone)."""
     import oracle
-    oracle.set_num_threads(os.cpu_count() or 1)
+    oracle.set_num_threads(nthreads)
     return oracle
 
 
-def cpu_baseline_cg(n, iters=2):
-    """The oracle (plain C, fp64, OpenMP over planes) on the host cores:
-    `iters` CG iterations on the full n^3 grid (setup subtracted)."""
+def _oracle_all_cores():
+    return _oracle_threads(os.cpu_count() or 1)
+
+
+def _time_oracle_cg(n, iters, nthreads):
     import synth
-    oracle = _oracle_all_cores()
+    oracle = _oracle_threads(nthreads)
     b = synth.poisson_poly_rhs((n, n, n))
     t0 = time.perf_counter()
     oracle.cg(b, max_iter=0)
@@ -670,23 +743,42 @@ def cpu_baseline_cg(n, iters=2):
     oracle.cg(b, max_iter=iters)
     t2 = time.perf_counter()
     per_iter = max((t2 - t1) - (t1 - t0), 1e-9) / iters
-    return {"value": n ** 3 / per_iter / 1e6, "unit": "MLUPS", "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": f"{iters} CG iterations on the full {n}^3 grid (oracle.cg, setup time subtracted)"}
+    return n ** 3 / per_iter / 1e6, oracle.num_threads(), per_iter
+
+
+def cpu_baseline_cg(n, iters=3):
+    """The oracle (plain C, fp64, OpenMP over planes), as it stands, on the
+    host cores: CG iterations on the full n^3 grid (setup subtracted), on
+    every core and on one thread (SURVEY §8(d) "CPU oracle timing")."""
+    v_all, cores, per_all = _time_oracle_cg(n, iters, os.cpu_count() or 1)
+    v_one, _, per_one = _time_oracle_cg(n, 1, 1)
+    return {"value": v_all, "unit": "MLUPS", "cores": cores, "kind": "oracle",
+            "sample": f"{iters} CG iterations on the full {n}^3 grid on {cores} threads, and 1 iteration on "
+                      "1 thread (oracle.cg; set-up time subtracted)",
+            "ms_per_iter": per_all * 1e3,
+            "one_thread": {"value": v_one, "unit": "MLUPS", "cores": 1, "ms_per_iter": per_one * 1e3},
+            "host": host_info()}
 
 
 def cpu_baseline_lbm(n=256, steps=2):
     import numpy as np
 
-    oracle = _oracle_all_cores()
-    c, w, _ = oracle.lbm_lattice()
-    f = np.broadcast_to(w[:, None, None, None], (19, n, n, n)).astype(np.float32)
-    om = lbm_omega(n)
-    t0 = time.perf_counter()
-    for _ in range(steps):
-        f = oracle.lbm_step(f, om)
-    dt = (time.perf_counter() - t0) / steps
-    return {"value": n ** 3 / dt / 1e6, "unit": "MLUPS", "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": f"{steps} cavity steps at {n}^3 (512^3 x 19 fp64 does not fit the bounded sample)"}
+    out = {}
+    for label, nth in (("all", os.cpu_count() or 1), ("one", 1)):
+        oracle = _oracle_threads(nth)
+        c, w, _ = oracle.lbm_lattice()
+        f = np.broadcast_to(w[:, None, None, None], (19, n, n, n)).astype(np.float32)
+        om = lbm_omega(n)
+        k = steps if label == "all" else 1
+        t0 = time.perf_counter()
+        for _ in range(k):
+            f = oracle.lbm_step(f, om)
+        out[label] = ((time.perf_counter() - t0) / k, oracle.num_threads())
+    dt, cores = out["all"]
+    return {"value": n ** 3 / dt / 1e6, "unit": "MLUPS", "cores": cores, "kind": "oracle",
+            "sample": f"{steps} cavity steps at {n}^3 on {cores} threads, 1 step on 1 thread "
+                      "(512^3 x 19 fp64 does not fit the bounded sample)",
+            "one_thread": {"value": n ** 3 / out["one"][0] / 1e6, "unit": "MLUPS", "cores": 1}}
 
 
 def reference_arm(args, world, rank):
@@ -715,8 +807,20 @@ def reference_arm(args, world, rank):
             "config": {"workload": f"C2 Poisson FD CG 7-point fp64 {n}^3 dense (configs[1])", "parts": 1},
             "cpu_baseline": {"value": v, "unit": "MLUPS", "cores": oracle.num_threads(), "kind": "oracle",
                              "sample": f"{k} CG iterations on the full {n}^3 grid after {w} warm-up "
-                                       "(time of cg(w+k) minus cg(w))"},
+                                       "(time of cg(w+k) minus cg(w))", "host": host_info()},
             "e2e": {"value": v, "unit": "MLUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+def relaunch_under_torchrun(args) -> int:
+    """`bench.py --gpus N` (N > 1) outside torchrun: start N ranks, one per
+    GPU, with torch.distributed.run on this node (rendezvous on 127.0.0.1)."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
 
 
 def main():
@@ -729,12 +833,18 @@ def main():
     ap.add_argument("--n", type=int, default=512)
     ap.add_argument("--occ", default="two_way", choices=list(("none", "standard", "extended", "two_way")))
     ap.add_argument("--prof-steps", type=int, default=10)
-    ap.add_argument("--no-extras", action="store_true", help="skip the LBM / C1 / cpu_baseline extras")
+    ap.add_argument("--no-extras", action="store_true", help="skip the extra workload lines and cpu_baseline")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch_under_torchrun(args))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
+    if world != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}; launch one rank per GPU "
+              "(python bench.py --gpus N starts them itself)", file=sys.stderr)
+        sys.exit(2)
     if args.impl == "reference":
         out = reference_arm(args, world, rank)
         if out is not None:
@@ -745,7 +855,7 @@ def main():
     __graft_entry__.build()
     if args.workload == "cg":
         out = bench_cg(args, world, rank, local)
-        if world == 1 and not args.no_extras:
+        if not args.no_extras and world == 1:
             lbm = bench_lbm_run(args.n, 20, 3, 1, local)
             out["also"] = {"lbm_d3q19": lbm, "c1": bench_c1(local),
                            "sparse_c4": bench_sparse_run(args.n, 20, 3, 1, local),
@@ -756,6 +866,16 @@ def main():
                            "karman_f4": bench_karman(local)}
             out["cpu_baseline"] = cpu_baseline_cg(args.n)
             out["also"]["lbm_d3q19"]["cpu_baseline"] = cpu_baseline_lbm()
+        elif not args.no_extras:
+            # N > 1: the scaling lines of SURVEY §8(d) — C2 weak (n^3 per GPU),
+            # C3 D3Q19 weak (n^3 per GPU), C4 and C5 strong — each with its
+            # per-rank dominant-kernel roofline and communication times
+            wa = argparse.Namespace(**vars(args))
+            wa.steps = min(args.steps, 50)
+            out["also"] = {"c2_weak": bench_cg(wa, world, rank, local, weak=True, with_e2e=False),
+                           "lbm_d3q19_weak": bench_lbm_run(args.n, 20, 3, world, local),
+                           "sparse_c4_strong": bench_sparse_run(args.n, 20, 3, world, local),
+                           "fem_c5_strong": bench_fem_run(384, 20, 3, world, local)}
     elif args.workload in ("sparse", "fem"):
         fn = bench_sparse_run if args.workload == "sparse" else bench_fem_run
         r = fn(args.n if args.workload == "sparse" else min(args.n, 384), args.steps, args.warmup, world, local)
