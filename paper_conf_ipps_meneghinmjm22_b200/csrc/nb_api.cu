@@ -299,6 +299,7 @@ __global__ void __launch_bounds__(256) k_halo_copy(const __grid_constant__ CopyB
 
 nb_status nb_launch_copy_batch(nb_grid *g, const CopyBatch &cb, cudaStream_t s) {
     if (!cb.n || !cb.bstart[cb.n]) return NB_OK;
+    NB_TRY(nb_delay_launch(g, 8, s));
     LaunchScope ls(g, s, "k_halo_copy");
     k_halo_copy<<<cb.bstart[cb.n], 256, 0, s>>>(cb);
     return nb_launch_check("k_halo_copy");

@@ -376,6 +376,10 @@ nb_status nb_peer_wait(nb_grid *g, bool periodic, cudaStream_t s);
 nb_status nb_peer_round(nb_grid *g, bool periodic, cudaStream_t s);
 nb_status nb_peer_barrier(nb_comm *c);
 nb_status nb_peer_reduce_finalize(nb_grid *g, int card, int mode, void *state, int slot);
+// schedule-robustness test knob (NB_DELAY_* environment, nb_peer.cu): the
+// delay in ns at injection point `bit` for this rank, and a spin kernel
+uint32_t nb_peer_delay(const nb_grid *g, uint32_t bit);
+nb_status nb_delay_launch(nb_grid *g, uint32_t bit, cudaStream_t s);
 
 // halo overlap events of a schedule (multi-process)
 struct HaloSync {

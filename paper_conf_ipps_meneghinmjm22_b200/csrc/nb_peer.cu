@@ -222,7 +222,47 @@ struct PeerOps {
     const uint64_t *wait[2];  // own flag words to await
     int wait_ctr[2];
     int nwait;
+    uint32_t delay_sig_ns, delay_wait_ns;  // schedule-robustness delays (nb_peer_delay)
+    uint32_t jitter;
 };
+
+// ---------------------------------------------------------------------------
+// Schedule-robustness delays (PAPER.md L252-L256,
+// L352-L363: halo transfers and reductions are ordered by events / flags
+// only, so any timing of the two sides must give the same bits).  Test
+// knob, read once from the environment:
+//   NB_DELAY_US     delay in microseconds (0: off)
+//   NB_DELAY_WHERE  bit mask: 1 before a halo signal (producer side), 2 after
+//                   a halo wait (consumer side), 4 before the reduction flags
+//                   of the cross-rank dot, 8 before every batched halo copy
+//                   (halo stream included)
+//   NB_DELAY_RANK   the rank that is delayed (-1 or unset: every rank)
+//   NB_DELAY_JITTER 1: each delay is drawn in [0, NB_DELAY_US] from the
+//                   global timer instead of fixed
+// ---------------------------------------------------------------------------
+struct DelayCfg {
+    uint32_t ns = 0, where = 0, jitter = 0;
+    int rank = -1;
+};
+static const DelayCfg &delay_cfg() {
+    static DelayCfg c = [] {
+        DelayCfg d;
+        if (const char *v = getenv("NB_DELAY_US")) d.ns = (uint32_t)(atof(v) * 1000.0);
+        if (const char *v = getenv("NB_DELAY_WHERE")) d.where = (uint32_t)atoi(v);
+        if (const char *v = getenv("NB_DELAY_RANK")) d.rank = atoi(v);
+        if (const char *v = getenv("NB_DELAY_JITTER")) d.jitter = (uint32_t)atoi(v);
+        return d;
+    }();
+    return c;
+}
+// delay in ns at injection point `bit` for this rank (0: none)
+uint32_t nb_peer_delay(const nb_grid *g, uint32_t bit) {
+    const DelayCfg &c = delay_cfg();
+    if (!c.ns || !(c.where & bit)) return 0;
+    const int rank = g->comm ? g->comm->rank : 0;
+    return (c.rank < 0 || c.rank == rank) ? c.ns : 0;
+}
+uint32_t nb_peer_jitter() { return delay_cfg().jitter; }
 
 __device__ __forceinline__ void st_release_sys(uint64_t *p, uint64_t v) {
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
@@ -255,9 +295,31 @@ __device__ void peer_spin(const uint64_t *flag, uint64_t want) {
     }
 }
 
+// spin for `ns` nanoseconds (jitter: a pseudo-random fraction of it)
+__device__ void delay_spin(uint32_t ns, uint32_t jitter) {
+    if (!ns) return;
+    uint64_t t0 = globaltimer_ns();
+    uint64_t d = ns;
+    if (jitter) d = (t0 * 0x9E3779B97F4A7C15ull >> 40) % (uint64_t)(ns + 1);
+    while (globaltimer_ns() - t0 < d) __nanosleep(256);
+}
+
+__global__ void k_delay(uint32_t ns, uint32_t jitter) {
+    if (threadIdx.x == 0) delay_spin(ns, jitter);
+}
+
+nb_status nb_delay_launch(nb_grid *g, uint32_t bit, cudaStream_t s) {
+    const uint32_t ns = nb_peer_delay(g, bit);
+    if (!ns) return NB_OK;
+    LaunchScope ls(g, s, "k_delay");
+    k_delay<<<1, 32, 0, s>>>(ns, nb_peer_jitter());
+    return nb_launch_check("k_delay");
+}
+
 __global__ void k_peer_ops(PeerOps o) {
     if (threadIdx.x != 0) return;
     if (o.nsig) {
+        delay_spin(o.delay_sig_ns, o.jitter);
         __threadfence_system();  // this stream's earlier peer stores are performed
         for (int i = 0; i < o.nsig; ++i) {
             const uint64_t v = o.ctr[o.sig_ctr[i]] + 1;
@@ -270,7 +332,10 @@ __global__ void k_peer_ops(PeerOps o) {
         o.ctr[o.wait_ctr[i]] = v;
         peer_spin(o.wait[i], v);
     }
-    if (o.nwait) __threadfence_system();
+    if (o.nwait) {
+        __threadfence_system();
+        delay_spin(o.delay_wait_ns, o.jitter);
+    }
 }
 
 // the ranks owning the partitions below / above this rank's slabs (-1: none)
@@ -313,6 +378,9 @@ static nb_status peer_ops(nb_grid *g, bool per, bool sig, bool wait, cudaStream_
         }
     }
     if (!o.nsig && !o.nwait) return NB_OK;
+    o.delay_sig_ns = nb_peer_delay(g, 1);
+    o.delay_wait_ns = nb_peer_delay(g, 2);
+    o.jitter = nb_peer_jitter();
     LaunchScope ls(g, s, sig && wait ? "k_peer_round" : sig ? "k_peer_signal" : "k_peer_wait");
     k_peer_ops<<<1, 32, 0, s>>>(o);
     return nb_launch_check("k_peer_ops");
@@ -333,6 +401,7 @@ struct PeerRed {
     const uint64_t *myflags;       // my flags[2 + r] base
     uint64_t *ctr;
     int world, rank;
+    uint32_t delay_ns, jitter;  // before raising the reduction flags (nb_peer_delay bit 4)
 };
 
 __global__ void __launch_bounds__(RED_THREADS) k_finalize_peer(const double *tp, int T, int NZ, int z0, int zn,
@@ -358,6 +427,7 @@ __global__ void __launch_bounds__(RED_THREADS) k_finalize_peer(const double *tp,
     if (!last) return;
     if (t == 0) {
         __threadfence_system();
+        delay_spin(R.delay_ns, R.jitter);
         const uint64_t seq = seq0 + 1;
         for (int r = 0; r < R.world; ++r)
             if (r != R.rank) st_release_sys(R.rflag[r], seq);
@@ -398,6 +468,8 @@ nb_status nb_peer_reduce_finalize(nb_grid *g, int card, int mode, void *state, i
     R.ctr = P->ctr;
     R.world = c->world;
     R.rank = c->rank;
+    R.delay_ns = nb_peer_delay(g, 4);
+    R.jitter = nb_peer_jitter();
     // planes outside [z0, z1) of psum2 are filled by the other ranks; zero
     // planes of components beyond card are never read (planes = card*NZ)
     LaunchScope ls(g, g->cs, "k_finalize");
