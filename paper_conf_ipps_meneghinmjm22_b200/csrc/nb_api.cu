@@ -306,6 +306,11 @@ nb_status nb_launch_copy_batch(nb_grid *g, const CopyBatch &cb, cudaStream_t s) 
 }
 
 nb_status nb_halo_run(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int c1d, cudaStream_t s) {
+    return nb_halo_run_mode(f, periodic, c0u, c1u, c0d, c1d, s, NB_HALO_GENERIC);
+}
+
+nb_status nb_halo_run_mode(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int c1d, cudaStream_t s,
+                           int mode) {
     nb_grid *g = f->g;
     int world = g->comm ? g->comm->world : 1, rank = g->comm ? g->comm->rank : 0;
     int cnt = 0;
@@ -320,8 +325,9 @@ nb_status nb_halo_run(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int
     if (nb_is_peer(g)) {
         // peer memory: a "ready" round (the neighbours finished reading the
         // halos about to be overwritten), my planes stored straight into the
-        // neighbours' (IPC-mapped) halos, a "done" round
-        NB_TRY(nb_peer_round(g, periodic, s));
+        // neighbours' (IPC-mapped) halos, a "done" round (NB_HALO_SEND: the
+        // copies and a signal only)
+        if (mode == NB_HALO_GENERIC) NB_TRY(nb_peer_round(g, periodic, s));
         CopyBatch cb;
         for (auto &m : msgs) {
             if (m.src_rank != rank) continue;  // the sender writes
@@ -335,7 +341,7 @@ nb_status nb_halo_run(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int
             }
         }
         if (cb.n) NB_TRY(nb_launch_copy_batch(g, cb, s));
-        return nb_peer_round(g, periodic, s);
+        return mode == NB_HALO_GENERIC ? nb_peer_round(g, periodic, s) : nb_peer_signal(g, periodic, s);
     }
     bool remote = false;
     // every device-local plane of the exchange goes into ONE batched copy
@@ -896,6 +902,32 @@ nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, boo
 }
 
 nb_status nb_sparse_halo_update(nb_field *f);
+
+// ---- split halo exchange (OCC of the sparse and FEM CG schedules) ---------
+nb_status nb_halo_split_begin(nb_field *f, int c0, int c1, HaloSync &hs) {
+    nb_grid *g = f->g;
+    auto run = [&](cudaStream_t s, int mode) {
+        return g->sparse ? nb_sparse_halo_run(f, c0, c1, c0, c1, s, mode)
+                         : nb_halo_run_mode(f, false, c0, c1, c0, c1, s, mode);
+    };
+    if (!nb_is_peer(g) && !nb_halo_on_stream(g)) return run(g->cs, NB_HALO_GENERIC);  // one process, stream order
+    if (!hs.eb) {
+        NB_CUDA(cudaEventCreateWithFlags(&hs.eb, cudaEventDisableTiming));
+        NB_CUDA(cudaEventCreateWithFlags(&hs.eh, cudaEventDisableTiming));
+    }
+    NB_CUDA(cudaEventRecord(hs.eb, g->cs));  // after the boundary-plane maps
+    NB_CUDA(cudaStreamWaitEvent(g->hs, hs.eb, 0));
+    NB_TRY(run(g->hs, NB_HALO_SEND));
+    NB_CUDA(cudaEventRecord(hs.eh, g->hs));
+    return NB_OK;
+}
+
+nb_status nb_halo_split_wait(nb_grid *g, HaloSync &hs) {
+    if (!nb_is_peer(g) && !nb_halo_on_stream(g)) return NB_OK;
+    if (nb_is_peer(g)) NB_TRY(nb_peer_wait(g, false, g->cs));  // the neighbours' planes are in
+    NB_CUDA(cudaStreamWaitEvent(g->cs, hs.eh, 0));               // join the halo stream
+    return NB_OK;
+}
 
 extern "C" nb_status nb_halo_update(nb_field *f) {
     if (!f) NB_FAIL(NB_EINVAL, "nb_halo_update: NULL field");

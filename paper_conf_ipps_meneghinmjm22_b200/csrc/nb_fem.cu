@@ -1458,8 +1458,14 @@ nb_status nb_fem_cg_hooks(nb_cg *cg, int parity) {
             }
         }
     }
-    NB_TRY(nb_halo_exchange_planes(pn, 0, 3, true, true, g->cs));
-    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+    // OCC (occ != NONE, fused schedule): the halo of
+    // p_new is sent right after the boundary-plane map; the planes whose
+    // neighbours are all own planes ([lo, nz - hi)) run phase A while it is
+    // in flight (they recompute p_new at their neighbours from r and p_old),
+    // then the boundary planes after the wait.  Same values, same order per
+    // node and per-plane dot partials: bitwise equal to the serial schedule.
+    const bool split = fused && cg->prm.occ != NB_OCC_NONE && g->nparts > 1;
+    auto phase = [&](int p, int zb, int ze) -> nb_status {
         FemArgs A{};
         A.y = (double *)cg->q->base[p];
         A.sc = cg->sc;
@@ -1468,10 +1474,26 @@ nb_status nb_fem_cg_hooks(nb_cg *cg, int parity) {
             A.po = (const double *)po->base[p];
             A.pn = (double *)pn->base[p];
             A.x = (double *)cg->x->base[p];
-            NB_TRY(fem_launch<FEM_CG_A>(g, p, A, pn, 0, g->parts[p].nz(), "k_fem_cg_a"));
-        } else {
-            A.u = (const double *)pn->base[p];
-            NB_TRY(fem_launch<FEM_CG_Q>(g, p, A, pn, 0, g->parts[p].nz(), "k_fem_cg_q"));
+            return fem_launch<FEM_CG_A>(g, p, A, pn, zb, ze, "k_fem_cg_a");
+        }
+        A.u = (const double *)pn->base[p];
+        return fem_launch<FEM_CG_Q>(g, p, A, pn, zb, ze, "k_fem_cg_q");
+    };
+    if (!split) {
+        NB_TRY(nb_halo_exchange_planes(pn, 0, 3, true, true, g->cs));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) NB_TRY(phase(p, 0, g->parts[p].nz()));
+    } else {
+        NB_TRY(nb_halo_split_begin(pn, 0, 3, cg->hs));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbPart &q = g->parts[p];
+            const int ib = q.lo >= 0 ? 1 : 0, ie = q.nz() - (q.hi >= 0 ? 1 : 0);
+            if (ie > ib) NB_TRY(phase(p, ib, ie));
+        }
+        NB_TRY(nb_halo_split_wait(g, cg->hs));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbPart &q = g->parts[p];
+            if (q.lo >= 0) NB_TRY(phase(p, 0, 1));
+            if (q.hi >= 0 && q.nz() > 1) NB_TRY(phase(p, q.nz() - 1, q.nz()));
         }
     }
     NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));

@@ -348,6 +348,14 @@ void nb_tma_forget_range(const void *lo, const void *hi);
 nb_status nb_halo_exchange_planes(nb_field *f, int c0, int c1, bool send_up, bool send_down,
                                   cudaStream_t s);
 nb_status nb_halo_run(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int c1d, cudaStream_t s);
+// halo modes: GENERIC = with the peer transport a "ready" round before and a
+// "done" round after the copies; SEND = the copies and a signal only (the
+// consumer waits; used where a reduction already orders the previous read
+// before the next write)
+enum { NB_HALO_GENERIC = 0, NB_HALO_SEND = 1 };
+nb_status nb_halo_run_mode(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int c1d, cudaStream_t s,
+                           int mode);
+nb_status nb_sparse_halo_run(nb_field *f, int c0u, int c1u, int c0d, int c1d, cudaStream_t s, int mode);
 nb_status nb_nccl_allreduce_sum(nb_grid *g, const double *send, double *recv, size_t n,
                                 cudaStream_t s);
 nb_status nb_nccl_group(nb_grid *g, bool start);
@@ -385,6 +393,12 @@ nb_status nb_delay_launch(nb_grid *g, uint32_t bit, cudaStream_t s);
 struct HaloSync {
     cudaEvent_t eb = nullptr, eh = nullptr;
 };
+// OCC split of a halo exchange of components [c0, c1) (sparse and FEM CG):
+// begin after the boundary-plane maps (the transfer runs on the halo stream
+// with the peer / NCCL transport or NB_HALO_STREAM, in stream order
+// otherwise); wait before the boundary-plane stencils
+nb_status nb_halo_split_begin(nb_field *f, int c0, int c1, HaloSync &hs);
+nb_status nb_halo_split_wait(nb_grid *g, HaloSync &hs);
 
 #include <map>
 struct nb_cg {

@@ -394,10 +394,17 @@ nb_status nb_sparse_slab_map(nb_grid *g, int p, uint8_t **d_mask, int32_t **d_ma
 // ---------------------------------------------------------------------------
 nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d);
 nb_status nb_sparse_halo_update(nb_field *f) { return nb_sparse_halo_comps(f, 0, f->card, 0, f->card); }
+nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d) {
+    return nb_sparse_halo_run(f, c0u, c1u, c0d, c1d, f->g->cs, NB_HALO_GENERIC);
+}
 
 // components [c0u, c1u) travel up (last plane -> upper neighbour's low halo),
-// [c0d, c1d) down
-nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d) {
+// [c0d, c1d) down; on stream s.  mode NB_HALO_GENERIC: with the peer
+// transport a "ready" round before and a "done" round after the copies;
+// NB_HALO_SEND: only the copies and a signal (the OCC split send of the CG
+// schedules, whose reductions already order every halo read before the
+// next write; the consumer calls nb_peer_wait)
+nb_status nb_sparse_halo_run(nb_field *f, int c0u, int c1u, int c0d, int c1d, cudaStream_t s, int mode) {
     nb_grid *g = f->g;
     int world = g->comm ? g->comm->world : 1, rank = g->comm ? g->comm->rank : 0;
     int cnt = 0;
@@ -421,7 +428,7 @@ nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d) 
     // device-local segments, and with the peer transport every segment this
     // rank sends (into the neighbour's IPC-mapped halo), in one batched launch
     const bool peer = nb_is_peer(g);
-    if (peer) NB_TRY(nb_peer_round(g, false, g->cs));  // neighbours done reading these halos
+    if (peer && mode == NB_HALO_GENERIC) NB_TRY(nb_peer_round(g, false, s));  // neighbours done reading these halos
     bool remote = false;
     CopyBatch cb;
     for (auto &m : msgs) {
@@ -432,7 +439,7 @@ nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d) 
                 const char *src = f->base[m.src_part] + ((int64_t)c * f->pcs[m.src_part] + src_off(m)) * f->esz;
                 char *dst = f->base[m.dst_part] + ((int64_t)c * f->pcs[m.dst_part] + dst_off(m)) * f->esz;
                 if (cb.n == CopyBatch::MAX) {
-                    NB_TRY(nb_launch_copy_batch(g, cb, g->cs));
+                    NB_TRY(nb_launch_copy_batch(g, cb, s));
                     cb = CopyBatch();
                 }
                 cb.add(dst, src, count(m) * f->esz);
@@ -441,8 +448,8 @@ nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d) 
             remote = true;
         }
     }
-    if (cb.n) NB_TRY(nb_launch_copy_batch(g, cb, g->cs));
-    if (peer) return nb_peer_round(g, false, g->cs);
+    if (cb.n) NB_TRY(nb_launch_copy_batch(g, cb, s));
+    if (peer) return mode == NB_HALO_GENERIC ? nb_peer_round(g, false, s) : nb_peer_signal(g, false, s);
     if (!remote) return NB_OK;
     NB_TRY(nb_nccl_group(g, true));
     for (auto &m : msgs) {
@@ -452,10 +459,10 @@ nb_status nb_sparse_halo_comps(nb_field *f, int c0u, int c1u, int c0d, int c1d) 
         for (int c = c0; c < c1; ++c) {
             if (m.src_rank == rank)
                 NB_TRY(nb_nccl_send(g, f->base[m.src_part] + ((int64_t)c * f->pcs[m.src_part] + src_off(m)) * f->esz,
-                                    count(m) * f->esz, m.dst_rank, g->cs));
+                                    count(m) * f->esz, m.dst_rank, s));
             else
                 NB_TRY(nb_nccl_recv(g, f->base[m.dst_part] + ((int64_t)c * f->pcs[m.dst_part] + dst_off(m)) * f->esz,
-                                    count(m) * f->esz, m.src_rank, g->cs));
+                                    count(m) * f->esz, m.src_rank, s));
         }
     }
     NB_TRY(nb_nccl_group(g, false));
@@ -782,25 +789,72 @@ nb_status nb_sparse_cg_init(nb_cg *cg) {
     return nb_reduce_finalize(g, 1, FIN_CG_INIT, cg->sc, 0);
 }
 
+// OCC with occ != NONE: the map of the boundary planes
+// (the neighbours' halos) first, the halo transfer of p started (on the halo
+// stream across processes, or with NB_HALO_STREAM), the interior map and
+// interior q pass enqueued while it is in flight, then the wait and the q
+// pass of the boundary planes.  Every cell runs the same arithmetic and the
+// dot partials are per plane, so all schedules give the same bits.
+// Extended / Two-way split the map as well (the reduce is per plane in any
+// case); Standard maps every plane before the transfer.
 nb_status nb_sparse_cg_hooks(nb_cg *cg, int parity) {
     (void)parity;
     nb_grid *g = cg->g;
     nb_field *p_ = cg->p[0];
-    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+    const nb_occ occ = cg->prm.occ;
+    const bool split = occ != NB_OCC_NONE && g->nparts > 1;
+    const bool split_map = split && occ != NB_OCC_STANDARD;
+    auto map_args = [&](int p) {
         SpArgs A{};
         A.a = (const double *)cg->r->base[p];
         A.c = (double *)p_->base[p];
         A.d = (double *)cg->x->base[p];
         A.sc = cg->sc;
-        NB_TRY(sp_launch<SPK_CG_MAP>(g, p, 0, g->parts[p].nz(), A, 0, "k_sp_cg_map"));
-    }
-    NB_TRY(nb_sparse_halo_update(p_));
-    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        return A;
+    };
+    auto q_args = [&](int p) {
         SpArgs A{};
         A.a = (const double *)p_->base[p];
         A.c = (double *)cg->q->base[p];
         A.sc = cg->sc;
-        NB_TRY(sp_launch<SPK_CG_Q>(g, p, 0, g->parts[p].nz(), A, 0, "k_sp_cg_q"));
+        return A;
+    };
+    // interior planes [ib, ie) of a partition: those whose neighbours are own planes
+    auto inner = [&](int p, int *ib, int *ie) {
+        const NbPart &q = g->parts[p];
+        *ib = q.lo >= 0 ? 1 : 0;
+        *ie = q.nz() - (q.hi >= 0 ? 1 : 0);
+        if (*ie < *ib) *ie = *ib;
+    };
+    auto bnd = [&](int p) {
+        const NbPart &q = g->parts[p];
+        std::vector<int> z;
+        if (q.lo >= 0) z.push_back(0);
+        if (q.hi >= 0 && q.nz() > 1) z.push_back(q.nz() - 1);
+        return z;
+    };
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        if (split_map) {
+            for (int z : bnd(p)) NB_TRY(sp_launch<SPK_CG_MAP>(g, p, z, z + 1, map_args(p), 0, "k_sp_cg_map"));
+        } else {
+            NB_TRY(sp_launch<SPK_CG_MAP>(g, p, 0, g->parts[p].nz(), map_args(p), 0, "k_sp_cg_map"));
+        }
+    }
+    if (!split) {
+        NB_TRY(nb_sparse_halo_update(p_));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+            NB_TRY(sp_launch<SPK_CG_Q>(g, p, 0, g->parts[p].nz(), q_args(p), 0, "k_sp_cg_q"));
+    } else {
+        NB_TRY(nb_halo_split_begin(p_, 0, 1, cg->hs));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            int ib, ie;
+            inner(p, &ib, &ie);
+            if (split_map) NB_TRY(sp_launch<SPK_CG_MAP>(g, p, ib, ie, map_args(p), 0, "k_sp_cg_map"));
+            NB_TRY(sp_launch<SPK_CG_Q>(g, p, ib, ie, q_args(p), 0, "k_sp_cg_q"));
+        }
+        NB_TRY(nb_halo_split_wait(g, cg->hs));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+            for (int z : bnd(p)) NB_TRY(sp_launch<SPK_CG_Q>(g, p, z, z + 1, q_args(p), 0, "k_sp_cg_q"));
     }
     NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_PQ, cg->sc, 0));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {

@@ -165,32 +165,39 @@ zz, yy, xx = np.meshgrid(*(np.arange(n) + 0.5 - n / 2,) * 3, indexing="ij")
 sphere = ((xx ** 2 + yy ** 2 + zz ** 2) <= (0.41528 * n) ** 2).astype(np.uint8)
 
 
-def sparse_cg(g):
-    b, x = nb.Field(g), nb.Field(g)
-    b.fill_uniform(4)
-    x.fill_const(0.0)
-    r = nb.nb_cg_solve(x, b, max_iter=12, rtol=0.0, check_every=4)
-    d = nb.nb_dot(b, b)
-    out = [x.download()]
-    b.close(), x.close()
-    return out, [r.rr, r.iters, d]
+def sparse_cg(occ):
+    def fn(g):
+        b, x = nb.Field(g), nb.Field(g)
+        b.fill_uniform(4)
+        x.fill_const(0.0)
+        r = nb.nb_cg_solve(x, b, max_iter=12, rtol=0.0, check_every=4, occ=occ)
+        d = nb.nb_dot(b, b)
+        out = [x.download()]
+        b.close(), x.close()
+        return out, [r.rr, r.iters, d]
+    return fn
 
 
-compare("sparse cg", (n, n, n), WORLD, sparse_cg, active=sphere)
+for occ in (nb.OCC_NONE, nb.OCC_STANDARD, nb.OCC_TWO_WAY):  # serial, and split around the halo (OCC)
+    compare(f"sparse cg occ{occ}", (n, n, n), WORLD, sparse_cg(occ), active=sphere)
 
 
 # ---- C5: FEM 27-point CG -----------------------------------------------------
-def fem_cg(g):
-    b, x = nb.Field(g, card=3), nb.Field(g, card=3)
-    nb.nb_fem27_rhs(b, 1.0)
-    x.fill_const(0.0)
-    r = nb.nb_cg_solve(x, b, max_iter=9, rtol=0.0, op=nb.OP_FEM27, check_every=3)
-    out = [x.download()]
-    b.close(), x.close()
-    return out, [r.rr, r.iters]
+def fem_cg(occ):
+    def fn(g):
+        b, x = nb.Field(g, card=3), nb.Field(g, card=3)
+        nb.nb_fem27_rhs(b, 1.0)
+        x.fill_const(0.0)
+        r = nb.nb_cg_solve(x, b, max_iter=9, rtol=0.0, op=nb.OP_FEM27, check_every=3, occ=occ)
+        out = [x.download()]
+        b.close(), x.close()
+        return out, [r.rr, r.iters]
+    return fn
 
 
-compare("fem cg", (12, 11, 14), WORLD, fem_cg)
+for occ in (nb.OCC_NONE, nb.OCC_TWO_WAY):
+    compare(f"fem cg occ{occ}", (12, 11, 14), WORLD, fem_cg(occ))
+compare("fem cg 4 parts", (12, 11, 16), 2 * WORLD, fem_cg(nb.OCC_TWO_WAY))
 
 # ---- borrowed (torch-owned) storage: IPC handle of the enclosing allocation + offset
 def wrapped_cg(g):

@@ -71,12 +71,13 @@ def test_fem_rigid_translation_and_rhs():
             f.close()
 
 
-def run_fem_cg(dims, parts, iters, rtol=0.0):
+def run_fem_cg(dims, parts, iters, rtol=0.0, occ=nb.OCC_TWO_WAY, halo=nb.HALO_FUSED):
     with grid(dims, parts) as g:
+        g.set_halo_mode(halo)
         fb, fx = nb.Field(g, card=3), nb.Field(g, card=3)
         nb.nb_fem27_rhs(fb, 1.0)
         fx.upload(np.zeros((3,) + dims[::-1]))
-        r = nb.nb_cg_solve(fx, fb, max_iter=iters, rtol=rtol, op=nb.OP_FEM27, check_every=16)
+        r = nb.nb_cg_solve(fx, fb, max_iter=iters, rtol=rtol, op=nb.OP_FEM27, check_every=16, occ=occ)
         x = fx.download()
         fb.close(), fx.close()
     return x, r
@@ -148,3 +149,23 @@ def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
     for v in ("zmarch", "plain", "faces_col", "faces_node", "3pass", "r_plane"):
         assert np.array_equal(out[None][0], out[v][0]), v
         assert np.array_equal(out[None][1], out[v][1]) and out[None][2] == out[v][2], v
+
+
+def test_fem_cg_occ_modes_bitwise_equal():
+    """OCC on the FEM CG: the p_new halo is
+    sent after the boundary-plane map while phase A runs on the planes whose
+    neighbours are own planes; the boundary planes follow the wait.  Every
+    OCC mode, partition count (2-plane slabs included) and halo transport
+    gives the serial schedule's bits."""
+    dims = (13, 11, 16)
+    ref = None
+    for parts in (1, 2, 4, 8):
+        for occ in (nb.OCC_NONE, nb.OCC_STANDARD, nb.OCC_TWO_WAY):
+            for halo in (nb.HALO_FUSED, nb.HALO_STREAM):
+                x, r = run_fem_cg(dims, parts, 9, occ=occ, halo=halo)
+                if ref is None:
+                    ref = (x, r.rr)
+                assert np.array_equal(x, ref[0]) and r.rr == ref[1], (parts, occ, halo)
+    b = oracle.fem_rhs(dims, 1.0)
+    xo, _, _ = oracle.cg(b, max_iter=9, op=oracle.OP_FEM27)
+    assert np.max(np.abs(ref[0] - xo)) <= 1e-10 * np.max(np.abs(xo))

@@ -133,12 +133,13 @@ def test_sparse_axpby_views():
         fx.close(), fy.close()
 
 
-def run_sparse_cg(m, b, parts, iters, rtol=0.0):
+def run_sparse_cg(m, b, parts, iters, rtol=0.0, occ=nb.OCC_TWO_WAY, halo=nb.HALO_FUSED):
     with sgrid(m, parts) as g:
+        g.set_halo_mode(halo)
         fb, fx = nb.Field(g), nb.Field(g)
         fb.upload(b)
         fx.upload(np.zeros_like(b))
-        r = nb.nb_cg_solve(fx, fb, max_iter=iters, rtol=rtol, check_every=8)
+        r = nb.nb_cg_solve(fx, fb, max_iter=iters, rtol=rtol, check_every=8, occ=occ)
         x = fx.download()
         fb.close(), fx.close()
     return x, r
@@ -170,3 +171,23 @@ def test_sparse_cg_converges_on_sphere():
     xo, ro, _ = oracle.cg(b, max_iter=300, op=oracle.OP_SPARSE7, mask=m, rtol=1e-12)
     assert abs(r.iters - ro.iters) <= 1
     assert np.max(np.abs(x.ravel()[act] - xo.ravel()[act])) <= 1e-10 * np.max(np.abs(xo))
+
+
+def test_sparse_cg_occ_modes_bitwise_equal():
+    """OCC on the sparse CG: boundary-plane map, halo of
+    p in flight while the interior map and q pass run, then the boundary q
+    pass.  Every OCC mode, partition count and halo transport (fused stream
+    order or copies on the halo stream) gives the serial schedule's bits."""
+    n = 26
+    m = sphere(n)
+    b = np.where(m, synth.uniform((n, n, n), seed=14), 0.0)
+    ref = None
+    for parts in (1, 2, 4):
+        for occ in (nb.OCC_NONE, nb.OCC_STANDARD, nb.OCC_EXTENDED, nb.OCC_TWO_WAY):
+            for halo in (nb.HALO_FUSED, nb.HALO_STREAM):
+                x, r = run_sparse_cg(m, b, parts, 11, occ=occ, halo=halo)
+                if ref is None:
+                    ref = (x, r.rr)
+                assert np.array_equal(x, ref[0]) and r.rr == ref[1], (parts, occ, halo)
+    xo, ro, _ = oracle.cg(b, max_iter=11, op=oracle.OP_SPARSE7, mask=m)
+    assert np.max(np.abs(ref[0] - xo)) <= 1e-11 * np.max(np.abs(xo))

@@ -16,9 +16,29 @@ iters = int(sys.argv[2]) if len(sys.argv) > 2 else 8
 what = sys.argv[3] if len(sys.argv) > 3 else "cg"
 parts = int(sys.argv[4]) if len(sys.argv) > 4 and not sys.argv[4].startswith("--") else 1
 hmode = int(sys.argv[5]) if len(sys.argv) > 5 and not sys.argv[5].startswith("--") else 0
-g = nb.Grid((n, n, n), nparts=parts, devices=[0] * parts)
+if what == "sparse":
+    import synth  # noqa: E402
+    g = nb.Grid((n, n, n), nparts=parts, devices=[0] * parts, active=synth.sphere_mask(n))
+else:
+    g = nb.Grid((n, n, n), nparts=parts, devices=[0] * parts)
 g.set_halo_mode(hmode)
-if what == "cg":
+if what in ("sparse", "fem"):  # C4 / C5 CG under Two-way OCC
+    card = 3 if what == "fem" else 1
+    b, x = nb.Field(g, card=card), nb.Field(g, card=card)
+    if what == "fem":
+        nb.nb_fem27_rhs(b, 1.0)
+    else:
+        b.fill_uniform(seed=4)
+    x.fill_const(0.0)
+    cg = nb.CG(x, b, op=nb.OP_FEM27 if what == "fem" else nb.OP_LAPLACE7)
+    cg.iterate(4)
+    g.sync()
+    with profile(activities=[ProfilerActivity.CUDA]) as prof:
+        cg.iterate(iters)
+        g.sync()
+    cg.finish()
+    cg.close()
+elif what == "cg":
     b, x = nb.Field(g), nb.Field(g)
     b.fill(nb.FILL_POISSON_RHS)
     x.fill_const(0.0)
