@@ -281,27 +281,45 @@ extern "C" nb_status nb_halo_plan(int32_t nz, int32_t nparts, int32_t world, int
 // ---------------------------------------------------------------------------
 
 __global__ void __launch_bounds__(256) k_halo_copy(const __grid_constant__ CopyBatch cb) {
-    const uint32_t b = blockIdx.x;
+    // grid-stride over the chunks: a capped grid leaves most SMs to the
+    // interior kernels the copy overlaps with (OCC)
+    const uint32_t total = cb.bstart[cb.n];
     int d = 0;
-    while (d + 1 < cb.n && cb.bstart[d + 1] <= b) ++d;
-    const uint64_t w0 = (uint64_t)(b - cb.bstart[d]) * CopyBatch::CHUNK;
-    const uint64_t w1 = min(w0 + CopyBatch::CHUNK, cb.words[d]);
-    if ((cb.vec >> d) & 1ull) {
-        const uint4 *s = (const uint4 *)cb.src[d];
-        uint4 *t = (uint4 *)cb.dst[d];
-        for (uint64_t i = w0 + threadIdx.x; i < w1; i += 256) t[i] = __ldcs(s + i);
-    } else {
-        const uint32_t *s = (const uint32_t *)cb.src[d];
-        uint32_t *t = (uint32_t *)cb.dst[d];
-        for (uint64_t i = w0 + threadIdx.x; i < w1; i += 256) t[i] = __ldcs(s + i);
+    for (uint32_t b = blockIdx.x; b < total; b += gridDim.x) {
+        while (d + 1 < cb.n && cb.bstart[d + 1] <= b) ++d;
+        const uint64_t w0 = (uint64_t)(b - cb.bstart[d]) * CopyBatch::CHUNK;
+        const uint64_t w1 = min(w0 + CopyBatch::CHUNK, cb.words[d]);
+        if ((cb.vec >> d) & 1ull) {
+            const uint4 *s = (const uint4 *)cb.src[d];
+            uint4 *t = (uint4 *)cb.dst[d];
+            for (uint64_t i = w0 + threadIdx.x; i < w1; i += 256) t[i] = __ldcs(s + i);
+        } else {
+            const uint32_t *s = (const uint32_t *)cb.src[d];
+            uint32_t *t = (uint32_t *)cb.dst[d];
+            for (uint64_t i = w0 + threadIdx.x; i < w1; i += 256) t[i] = __ldcs(s + i);
+        }
     }
+}
+
+// blocks of a batched halo copy on the halo stream: at most
+// NB_HALO_COPY_BLOCKS (default 128, under one block per SM) so the copy does
+// not take every SM away from the interior kernels it is meant to overlap;
+// on the compute stream (stream-ordered copies) the full grid
+static uint32_t halo_copy_blocks() {
+    static uint32_t cap = [] {
+        const char *v = getenv("NB_HALO_COPY_BLOCKS");
+        int c = v ? atoi(v) : 128;
+        return (uint32_t)(c > 0 ? c : 128);
+    }();
+    return cap;
 }
 
 nb_status nb_launch_copy_batch(nb_grid *g, const CopyBatch &cb, cudaStream_t s) {
     if (!cb.n || !cb.bstart[cb.n]) return NB_OK;
     NB_TRY(nb_delay_launch(g, 8, s));
     LaunchScope ls(g, s, "k_halo_copy");
-    k_halo_copy<<<cb.bstart[cb.n], 256, 0, s>>>(cb);
+    const uint32_t blocks = s == g->cs ? cb.bstart[cb.n] : std::min(cb.bstart[cb.n], halo_copy_blocks());
+    k_halo_copy<<<blocks, 256, 0, s>>>(cb);
     return nb_launch_check("k_halo_copy");
 }
 
@@ -386,7 +404,13 @@ nb_status nb_halo_run_mode(nb_field *f, bool periodic, int c0u, int c1u, int c0d
 nb_status nb_grid_alloc_common(nb_grid *g) {
     DeviceGuard dg(g->device);
     NB_CUDA(cudaStreamCreateWithFlags(&g->cs, cudaStreamNonBlocking));
-    NB_CUDA(cudaStreamCreateWithFlags(&g->hs, cudaStreamNonBlocking));
+    // the halo stream runs at the highest priority: its copies are small and
+    // sit on the critical path, so the block scheduler should start them as
+    // soon as an SM frees up instead of behind the interior kernel's
+    // remaining CTAs (OCC)
+    int prio_lo = 0, prio_hi = 0;
+    NB_CUDA(cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi));
+    NB_CUDA(cudaStreamCreateWithPriority(&g->hs, cudaStreamNonBlocking, prio_hi));
     g->own_cs = g->own_hs = true;
     g->tiles_x = (g->nx + DOT_TX - 1) / DOT_TX;
     g->tiles_y = (g->ny + DOT_TY - 1) / DOT_TY;

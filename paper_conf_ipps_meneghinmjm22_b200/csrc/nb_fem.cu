@@ -623,15 +623,19 @@ template <int K>
 #ifndef NB_FSURF_BX
 #define NB_FSURF_BX 128
 #endif
-__global__ void __launch_bounds__(NB_FSURF_BX) k_fem_surface(FemArgs A, PGeo g, int zb, int ze, FemSurf S) {
+__global__ void __launch_bounds__(NB_FSURF_BX) k_fem_surface(FemArgs A, PGeo g, int zb, int ze, FemSurf S,
+                                                              int zhi) {
     if ((K == FEM_CG_Q || K == FEM_CG_A) && A.sc->status != 0) return;
-    const int nzl = ze - zb;
+    // planes [zb, ze), or with zhi >= 0 the two planes zb and zhi (the
+    // boundary planes of a slab in one launch)
+    const int nzl = zhi >= 0 ? 2 : ze - zb;
     const int64_t n1 = (int64_t)S.ncol_edge * nzl, n2 = (int64_t)S.nin * S.nzs;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n1 + n2; i += (int64_t)gridDim.x * blockDim.x) {
         int x, y, zl;
         if (i < n1) {  // edge columns: consecutive threads walk along a face (coalesced on y faces)
             fem_edge_col((int)(i % S.ncol_edge), g.nx, g.ny, x, y);
             zl = zb + (int)(i / S.ncol_edge);
+            if (zhi >= 0 && zl > zb) zl = zhi;
         } else {
             const int64_t k = i - n1;
             const int c = (int)(k % S.nin);
@@ -659,14 +663,18 @@ __global__ void __launch_bounds__(NB_FSURF_BX) k_fem_surface(FemArgs A, PGeo g, 
 constexpr int XF_Y = 32, XF_Z = 8;
 
 template <int K>
-__global__ void __launch_bounds__(XF_Y *XF_Z) k_fem_xface(FemArgs A, PGeo g, int zb, int ze) {
+__global__ void __launch_bounds__(XF_Y *XF_Z) k_fem_xface(FemArgs A, PGeo g, int zb, int ze, int zhi) {
     if ((K == FEM_CG_Q || K == FEM_CG_A) && A.sc->status != 0) return;
+    if (zhi >= 0) {  // the two planes zb and zhi, one per blockIdx.y
+        if (blockIdx.y) zb = zhi;
+        ze = zb + 1;
+    }
     __shared__ double su[3][XF_Z + 2][XF_Y + 2][2];
     const int face = blockIdx.z;
     const int xa = face ? g.nx - 2 : 0;  // patch columns xa, xa + 1
     const int x = face ? g.nx - 1 : 0;   // node column
     const int ybase = blockIdx.x * XF_Y;  // patch rows ybase .. ybase + 33; nodes ybase + 1 ..
-    const int zbase = zb + blockIdx.y * XF_Z;  // node planes zbase ..; patch planes zbase - 1 ..
+    const int zbase = zhi >= 0 ? zb : zb + blockIdx.y * XF_Z;  // node planes zbase ..; patch planes zbase - 1 ..
     const int tid = threadIdx.x;
     constexpr int NP = (XF_Z + 2) * (XF_Y + 2) * 2;
     for (int e = tid; e < 3 * NP; e += XF_Y * XF_Z) {
@@ -1170,12 +1178,19 @@ __global__ void __launch_bounds__(FemTmaCfg<K>::NT, FemTmaCfg<K>::MINB)
     t.flush(t.zend - 1, tp, T);  // the last output (after a barrier)
 }
 
-// CG map: x += alpha_prev p_old (pending, when dox), p_new = r + beta p_old
-__global__ void k_fem_map(double *x, double *pn, const double *po, const double *r, int64_t n, const CgScal *sc,
-                          int dox) {
+// CG map: x += alpha_prev p_old (pending, when dox), p_new = r + beta p_old,
+// over `nseg` runs of n elements starting at off[blockIdx.y] (all boundary
+// planes x components of a partition in one launch)
+struct FemMapSegs {
+    int64_t off[8];
+};
+__global__ void k_fem_map(double *x, double *pn, const double *po, const double *r, FemMapSegs S, int64_t n,
+                          const CgScal *sc, int dox) {
     if (sc->status != 0) return;
     const double beta = sc->beta, ap = sc->alpha_prev;
     const int pending = dox && sc->pending;
+    const int64_t o = S.off[blockIdx.y];
+    x += o, pn += o, po += o, r += o;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const double pv = po[i];
         if (pending) x[i] = fma(ap, pv, x[i]);
@@ -1276,9 +1291,16 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_fem_r(double *r, const doubl
 
 static inline int64_t fcs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
 
+// what: FEM_SURF = only the surface-node kernels of the TMA path, FEM_BULK =
+// only the streaming kernel, FEM_ALL = both (the OCC schedule runs the
+// surface nodes of the interior planes while the halo is in flight)
+enum { FEM_SURF = 1, FEM_BULK = 2, FEM_ALL = 3 };
+
 template <int K>
-static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int zb, int ze, const char *name) {
+static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int zb, int ze, const char *name,
+                            int what = FEM_ALL, int zhi = -1) {
     if (ze <= zb) return NB_OK;
+    if (zhi >= 0 && (what != FEM_SURF || ze != zb + 1 || zhi <= zb)) NB_FAIL(NB_EINVAL, "fem_launch: bad plane pair");
     A.cs = fcs(f, p);
     const PGeo geo = pgeo(f, p);
     const char *variant = getenv("NB_FEM_KERNEL");  // "plain" | "zmarch" | default TMA
@@ -1308,7 +1330,9 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
             const int gz = geo.z0 + zl;
             if (gz < 2 || gz > geo.NZ - 2) S.zlist[S.nzs++] = zl;
         }
-        {
+        if (zhi >= 0 && (geo.z0 + zhi < 2 || geo.z0 + zhi > geo.NZ - 2)) S.zlist[S.nzs++] = zhi;
+        const int nzr = zhi >= 0 ? 2 : ze - zb;  // planes of the launch
+        if (what & FEM_SURF) {
             // face columns: one thread per node, consecutive threads along a
             // face (default; 0.19 ms at 384^3 for all surface nodes), or the
             // z-marching column kernel (NB_FEM_FACES=col; 0.22 ms); z-surface
@@ -1322,22 +1346,24 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
             if (!faces_node) S.ncol_edge = 0;
             if (xface) {
                 S.ncol_edge = 2 * nx;  // fem_edge_col lists the y = 0 and y = ny-1 rows first
-                dim3 xg((ny - 2 + XF_Y - 1) / XF_Y, (ze - zb + XF_Z - 1) / XF_Z, 2);
+                dim3 xg((ny - 2 + XF_Y - 1) / XF_Y, zhi >= 0 ? 2 : (ze - zb + XF_Z - 1) / XF_Z, 2);
                 LaunchScope ls(g, g->cs, "k_fem_surface");
-                k_fem_xface<K><<<xg, XF_Y * XF_Z, 0, g->cs>>>(A, geo, zb, ze);
+                k_fem_xface<K><<<xg, XF_Y * XF_Z, 0, g->cs>>>(A, geo, zb, ze, zhi);
             }
-            const int64_t n = (int64_t)S.ncol_edge * (ze - zb) + (int64_t)S.nin * S.nzs;
+            const int64_t n = (int64_t)S.ncol_edge * nzr + (int64_t)S.nin * S.nzs;
             if (n > 0) {
                 const int blocks = (int)std::min<int64_t>((n + NB_FSURF_BX - 1) / NB_FSURF_BX, 1 << 30);
                 LaunchScope ls(g, g->cs, "k_fem_surface");
-                k_fem_surface<K><<<blocks, NB_FSURF_BX, 0, g->cs>>>(A, geo, zb, ze, S);
+                k_fem_surface<K><<<blocks, NB_FSURF_BX, 0, g->cs>>>(A, geo, zb, ze, S, zhi);
             }
             if (ncols > 0) {
+                if (zhi >= 0) NB_FAIL(NB_EUNSUPPORTED, "plane pairs with the face-column kernel");
                 dim3 fg((ncols + 63) / 64, (ze - zb + FZC - 1) / FZC);
                 LaunchScope ls(g, g->cs, "k_fem_faces");
                 k_fem_faces<K><<<fg, 64, 0, g->cs>>>(A, geo, zb, ze, ncols);
             }
         }
+        if (!(what & FEM_BULK)) return NB_OK;
         static unsigned attr_set = 0;  // per device: dynamic shared memory above 48 KB
         if (g->device < 32 && !(attr_set & (1u << g->device))) {
             NB_CUDA(cudaFuncSetAttribute(k_fem_tma<K, ZC, NR>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
@@ -1437,35 +1463,42 @@ nb_status nb_fem_cg_hooks(nb_cg *cg, int parity) {
     const bool fused = fem_fused();
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         const NbPart &q = g->parts[p];
-        std::vector<int> planes;  // own planes to map first
+        // fused: only the boundary planes (the neighbours' halos; phase A
+        // forms p_new everywhere else), all planes x components in ONE launch
+        FemMapSegs S{};
+        int nseg = 0;
+        int64_t n = 0;
         if (fused) {
-            if (q.lo >= 0) planes.push_back(0);
-            if (q.hi >= 0 && q.nz() > 1) planes.push_back(q.nz() - 1);
-        }
-        for (int c = 0; c < 3; ++c) {
-            auto run = [&](int z0, int nz, int dox) -> nb_status {
-                const int64_t off = (int64_t)c * fcs(pn, p) + (int64_t)(z0 + 1) * pn->ps, n = (int64_t)nz * pn->ps;
-                LaunchScope ls(g, g->cs, "k_fem_map");
-                k_fem_map<<<fused ? 148 : 148 * 8, 256, 0, g->cs>>>(
-                    (double *)cg->x->base[p] + off, (double *)pn->base[p] + off, (const double *)po->base[p] + off,
-                    (const double *)cg->r->base[p] + off, n, cg->sc, dox);
-                return nb_launch_check("k_fem_map");
-            };
-            if (fused) {
-                for (int z : planes) NB_TRY(run(z, 1, 0));
-            } else {
-                NB_TRY(run(0, q.nz(), 1));
+            n = pn->ps;
+            for (int c = 0; c < 3; ++c) {
+                if (q.lo >= 0) S.off[nseg++] = (int64_t)c * fcs(pn, p) + pn->ps;
+                if (q.hi >= 0 && q.nz() > 1) S.off[nseg++] = (int64_t)c * fcs(pn, p) + (int64_t)q.nz() * pn->ps;
             }
+        } else {
+            n = (int64_t)q.nz() * pn->ps;
+            for (int c = 0; c < 3; ++c) S.off[nseg++] = (int64_t)c * fcs(pn, p) + pn->ps;
         }
+        if (!nseg) continue;
+        LaunchScope ls(g, g->cs, "k_fem_map");
+        k_fem_map<<<dim3(fused ? 148 : 148 * 8, nseg), 256, 0, g->cs>>>(
+            (double *)cg->x->base[p], (double *)pn->base[p], (const double *)po->base[p], (const double *)cg->r->base[p],
+            S, n, cg->sc, fused ? 0 : 1);
+        NB_TRY(nb_launch_check("k_fem_map"));
     }
-    // OCC (occ != NONE, fused schedule): the halo of
-    // p_new is sent right after the boundary-plane map; the planes whose
-    // neighbours are all own planes ([lo, nz - hi)) run phase A while it is
-    // in flight (they recompute p_new at their neighbours from r and p_old),
-    // then the boundary planes after the wait.  Same values, same order per
-    // node and per-plane dot partials: bitwise equal to the serial schedule.
-    const bool split = fused && cg->prm.occ != NB_OCC_NONE && g->nparts > 1;
-    auto phase = [&](int p, int zb, int ze) -> nb_status {
+    // OCC (occ != NONE, fused schedule, and a transfer
+    // that actually runs asynchronously: the peer or NCCL transport across
+    // processes, or NB_HALO_STREAM): the halo of p_new is sent right after
+    // the boundary-plane map, and the surface nodes of the planes whose
+    // neighbours are own planes ([lo, nz - hi)) are computed while it is in
+    // flight (they recompute p_new at their neighbours from r and p_old);
+    // after the wait the surface nodes of the boundary planes, then the
+    // streaming phase A over all planes in one launch.  Same values, same
+    // order per node and per-plane dot partials: bitwise equal to the serial
+    // schedule.  In one process with fused halos the copies are stream-
+    // ordered work with nothing to overlap, and the serial schedule runs.
+    const bool split = fused && cg->prm.occ != NB_OCC_NONE && g->nparts > 1 &&
+                       (nb_is_peer(g) || nb_halo_on_stream(g)) && nb_tma_enabled() && !getenv("NB_FEM_KERNEL");
+    auto args = [&](int p) {
         FemArgs A{};
         A.y = (double *)cg->q->base[p];
         A.sc = cg->sc;
@@ -1474,26 +1507,37 @@ nb_status nb_fem_cg_hooks(nb_cg *cg, int parity) {
             A.po = (const double *)po->base[p];
             A.pn = (double *)pn->base[p];
             A.x = (double *)cg->x->base[p];
-            return fem_launch<FEM_CG_A>(g, p, A, pn, zb, ze, "k_fem_cg_a");
+        } else {
+            A.u = (const double *)pn->base[p];
         }
-        A.u = (const double *)pn->base[p];
-        return fem_launch<FEM_CG_Q>(g, p, A, pn, zb, ze, "k_fem_cg_q");
+        return A;
     };
     if (!split) {
         NB_TRY(nb_halo_exchange_planes(pn, 0, 3, true, true, g->cs));
-        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) NB_TRY(phase(p, 0, g->parts[p].nz()));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            if (fused)
+                NB_TRY(fem_launch<FEM_CG_A>(g, p, args(p), pn, 0, g->parts[p].nz(), "k_fem_cg_a"));
+            else
+                NB_TRY(fem_launch<FEM_CG_Q>(g, p, args(p), pn, 0, g->parts[p].nz(), "k_fem_cg_q"));
+        }
     } else {
         NB_TRY(nb_halo_split_begin(pn, 0, 3, cg->hs));
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
             const NbPart &q = g->parts[p];
             const int ib = q.lo >= 0 ? 1 : 0, ie = q.nz() - (q.hi >= 0 ? 1 : 0);
-            if (ie > ib) NB_TRY(phase(p, ib, ie));
+            if (ie > ib) NB_TRY(fem_launch<FEM_CG_A>(g, p, args(p), pn, ib, ie, "k_fem_cg_a", FEM_SURF));
         }
         NB_TRY(nb_halo_split_wait(g, cg->hs));
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
             const NbPart &q = g->parts[p];
-            if (q.lo >= 0) NB_TRY(phase(p, 0, 1));
-            if (q.hi >= 0 && q.nz() > 1) NB_TRY(phase(p, q.nz() - 1, q.nz()));
+            // the surface nodes of both boundary planes in one launch per kernel
+            if (q.lo >= 0 && q.hi >= 0 && q.nz() > 1)
+                NB_TRY(fem_launch<FEM_CG_A>(g, p, args(p), pn, 0, 1, "k_fem_cg_a", FEM_SURF, q.nz() - 1));
+            else if (q.lo >= 0)
+                NB_TRY(fem_launch<FEM_CG_A>(g, p, args(p), pn, 0, 1, "k_fem_cg_a", FEM_SURF));
+            else if (q.hi >= 0)
+                NB_TRY(fem_launch<FEM_CG_A>(g, p, args(p), pn, q.nz() - 1, q.nz(), "k_fem_cg_a", FEM_SURF));
+            NB_TRY(fem_launch<FEM_CG_A>(g, p, args(p), pn, 0, q.nz(), "k_fem_cg_a", FEM_BULK));
         }
     }
     NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));

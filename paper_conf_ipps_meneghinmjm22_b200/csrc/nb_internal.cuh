@@ -135,6 +135,10 @@ struct NbSparsePart {
     // non-empty 256-cell dot segments, plane-major: entry = zl << 16 | seg
     int32_t *d_seg = nullptr;
     std::vector<int64_t> seg_start;         // first segment of each local plane [nz_p + 1]
+    // the segments of the boundary planes facing a neighbour (OCC: one
+    // launch for both), entries as d_seg (lazy)
+    int32_t *d_seg_bnd = nullptr;
+    int64_t n_seg_bnd = -1;
 };
 
 struct nb_grid {

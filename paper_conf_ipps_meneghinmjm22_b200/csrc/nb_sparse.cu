@@ -43,6 +43,9 @@ void nb_sparse_free(nb_grid *g) {
         cudaFree(s.coord);
         cudaFree(s.d_pstart);
         cudaFree(s.d_seg);
+        cudaFree(s.d_seg_bnd);
+        s.d_seg_bnd = nullptr;
+        s.n_seg_bnd = -1;
         s.conn = s.coord = nullptr;
         s.d_pstart = nullptr;
         s.d_seg = nullptr;
@@ -71,6 +74,8 @@ __global__ void k_sp_conn(const uint8_t *__restrict__ mask, const int32_t *__res
         conn[(int64_t)d * n + j] = v;
     }
 }
+
+static nb_status sp_bnd_segments(nb_grid *g, int p);
 
 extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t *active, int32_t nparts,
                                            const int32_t *device_ids, nb_comm *comm, nb_grid **out) {
@@ -184,6 +189,7 @@ extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t 
             fail("cudaMalloc seg", e);
         if (s == NB_OK && !segs.empty())
             cudaMemcpyAsync(sp.d_seg, segs.data(), sizeof(int32_t) * segs.size(), cudaMemcpyHostToDevice, g->cs);
+        if (s == NB_OK) s = sp_bnd_segments(g, p);  // built here: the CG hooks may run under graph capture
         if (s == NB_OK && q.nz() > 0) {
             dim3 blk(128), grd((nx + 127) / 128, ny, q.nz());
             LaunchScope ls(g, g->cs, "k_sp_conn");
@@ -734,6 +740,46 @@ static nb_status sp_launch(nb_grid *g, int p, int zb, int ze, SpArgs A, int plan
     return nb_launch_check(name);
 }
 
+// launch over an explicit list of segment entries (plane << 16 | index)
+template <int K>
+static nb_status sp_launch_list(nb_grid *g, int p, const int32_t *list, int64_t n, SpArgs A, int plane_base,
+                                const char *name) {
+    if (n <= 0) return NB_OK;
+    const NbSparsePart &sp = g->sp[p];
+    A.seg = list;
+    A.seg0 = 0;
+    A.nseg = n;
+    A.pstart = sp.d_pstart;
+    A.conn = sp.conn;
+    A.n = sp.n;
+    A.hl = sp.hl;
+    A.plane0 = plane_base + g->parts[p].z0;
+    A.T = g->T;
+    A.tp = g->tp;
+    LaunchScope ls(g, g->cs, name);
+    k_sp<K><<<(unsigned)((n + NSB - 1) / NSB), SEG, 0, g->cs>>>(A);
+    return nb_launch_check(name);
+}
+
+// the segments of partition p's boundary planes (those facing a neighbour);
+// built at grid creation (never under graph capture)
+static nb_status sp_bnd_segments(nb_grid *g, int p) {
+    NbSparsePart &sp = g->sp[p];
+    if (sp.n_seg_bnd >= 0) return NB_OK;
+    const NbPart &q = g->parts[p];
+    std::vector<int32_t> segs;
+    auto add = [&](int zl) {
+        for (int64_t k = 0; k < sp.seg_start[zl + 1] - sp.seg_start[zl]; ++k) segs.push_back((zl << 16) | (int)k);
+    };
+    if (q.lo >= 0) add(0);
+    if (q.hi >= 0 && q.nz() > 1) add(q.nz() - 1);
+    NB_CUDA(cudaMalloc(&sp.d_seg_bnd, sizeof(int32_t) * std::max<size_t>(segs.size(), 1)));
+    if (!segs.empty())
+        NB_CUDA(cudaMemcpy(sp.d_seg_bnd, segs.data(), sizeof(int32_t) * segs.size(), cudaMemcpyHostToDevice));
+    sp.n_seg_bnd = (int64_t)segs.size();
+    return NB_OK;
+}
+
 nb_status nb_sparse_dot_partials(const nb_field *x, const nb_field *y) {
     nb_grid *g = x->g;
     if (x->dt != NB_F64) NB_FAIL(NB_EUNSUPPORTED, "sparse dot: fp64 fields");
@@ -789,20 +835,23 @@ nb_status nb_sparse_cg_init(nb_cg *cg) {
     return nb_reduce_finalize(g, 1, FIN_CG_INIT, cg->sc, 0);
 }
 
-// OCC with occ != NONE: the map of the boundary planes
-// (the neighbours' halos) first, the halo transfer of p started (on the halo
-// stream across processes, or with NB_HALO_STREAM), the interior map and
-// interior q pass enqueued while it is in flight, then the wait and the q
-// pass of the boundary planes.  Every cell runs the same arithmetic and the
-// dot partials are per plane, so all schedules give the same bits.
-// Extended / Two-way split the map as well (the reduce is per plane in any
-// case); Standard maps every plane before the transfer.
+// OCC with occ != NONE and a transfer that actually
+// runs asynchronously (the peer or NCCL transport across processes, or
+// NB_HALO_STREAM): the map of the boundary planes (the neighbours' halos)
+// first, the halo transfer of p started on the halo stream, the interior map
+// and interior q pass enqueued while it is in flight, then the wait and the
+// q pass of the boundary planes (both planes in one launch).  Every cell runs
+// the same arithmetic and the dot partials are per plane, so all schedules
+// give the same bits.  Extended / Two-way split the map as well (the reduce
+// is per plane in any case); Standard maps every plane before the transfer.
+// In one process with fused halos the copies are stream-ordered work with
+// nothing to overlap, and the serial schedule runs.
 nb_status nb_sparse_cg_hooks(nb_cg *cg, int parity) {
     (void)parity;
     nb_grid *g = cg->g;
     nb_field *p_ = cg->p[0];
     const nb_occ occ = cg->prm.occ;
-    const bool split = occ != NB_OCC_NONE && g->nparts > 1;
+    const bool split = occ != NB_OCC_NONE && g->nparts > 1 && (nb_is_peer(g) || nb_halo_on_stream(g));
     const bool split_map = split && occ != NB_OCC_STANDARD;
     auto map_args = [&](int p) {
         SpArgs A{};
@@ -826,16 +875,10 @@ nb_status nb_sparse_cg_hooks(nb_cg *cg, int parity) {
         *ie = q.nz() - (q.hi >= 0 ? 1 : 0);
         if (*ie < *ib) *ie = *ib;
     };
-    auto bnd = [&](int p) {
-        const NbPart &q = g->parts[p];
-        std::vector<int> z;
-        if (q.lo >= 0) z.push_back(0);
-        if (q.hi >= 0 && q.nz() > 1) z.push_back(q.nz() - 1);
-        return z;
-    };
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         if (split_map) {
-            for (int z : bnd(p)) NB_TRY(sp_launch<SPK_CG_MAP>(g, p, z, z + 1, map_args(p), 0, "k_sp_cg_map"));
+            const NbSparsePart &sp = g->sp[p];
+            NB_TRY(sp_launch_list<SPK_CG_MAP>(g, p, sp.d_seg_bnd, sp.n_seg_bnd, map_args(p), 0, "k_sp_cg_map"));
         } else {
             NB_TRY(sp_launch<SPK_CG_MAP>(g, p, 0, g->parts[p].nz(), map_args(p), 0, "k_sp_cg_map"));
         }
@@ -853,8 +896,10 @@ nb_status nb_sparse_cg_hooks(nb_cg *cg, int parity) {
             NB_TRY(sp_launch<SPK_CG_Q>(g, p, ib, ie, q_args(p), 0, "k_sp_cg_q"));
         }
         NB_TRY(nb_halo_split_wait(g, cg->hs));
-        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
-            for (int z : bnd(p)) NB_TRY(sp_launch<SPK_CG_Q>(g, p, z, z + 1, q_args(p), 0, "k_sp_cg_q"));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbSparsePart &sp = g->sp[p];
+            NB_TRY(sp_launch_list<SPK_CG_Q>(g, p, sp.d_seg_bnd, sp.n_seg_bnd, q_args(p), 0, "k_sp_cg_q"));
+        }
     }
     NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_PQ, cg->sc, 0));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {

@@ -60,6 +60,7 @@ else:
         g.sync()
 evs = [e for e in prof.events() if e.device_type == torch.autograd.DeviceType.CUDA]
 ks = sorted([(e.time_range.start, e.time_range.end, e.name) for e in evs])
+streams = {}  # kernel name -> set of device streams (the halo stream shows up separately)
 # halo copies vs kernels: fraction of copy time overlapped by a running kernel
 def is_copy(nm):
     return "Memcpy" in nm or "memcpy" in nm or "k_halo_copy" in nm
@@ -96,9 +97,10 @@ busy += cur[1] - cur[0] if cur else 0.0
 summary = {"what": what, "n": n, "parts": parts, "halo_mode": hmode, "iters": iters, "span_us": tot,
            "busy_us": busy, "idle_us": tot - busy, "kernels": len(rows), "halo_copies": len(copies),
            "halo_copy_us": copy_t, "halo_copy_overlapped_frac": (cov / copy_t) if copy_t else None}
-print(json.dumps(summary))
-for r in rows[:24]:
-    print(f"{r['name']:50s} dur {r['dur_us']:9.1f} us  gap {r['gap_us']:7.1f} us")
 if "--out" in sys.argv:
     with open(sys.argv[sys.argv.index("--out") + 1], "w") as fh:
         json.dump({"summary": summary, "kernels": rows}, fh, indent=1)
+print(json.dumps(summary), flush=True)
+if "--quiet" not in sys.argv:
+    for r in rows[:24]:
+        print(f"{r['name']:50s} dur {r['dur_us']:9.1f} us  gap {r['gap_us']:7.1f} us")
