@@ -459,7 +459,11 @@ def bench_lbm_sparse_run(n, steps, warmup, local):
             "clocks": clocks}
 
 
-SPARSE_BYTES = {"k_sp_cg_map": 40, "k_sp_cg_q": 40, "k_sp_cg_r": 24}  # per active cell (q: p 8 + conn 24 + q 8)
+# per active cell: map reads r, p_old, x and writes x, p (40 B); q reads p and
+# the 16-byte segment-indexed neighbour entry and writes q (32 B; the six
+# neighbour values are cache hits of the same p stream); r reads q, r and
+# writes r (24 B)
+SPARSE_BYTES = {"k_sp_cg_map": 40, "k_sp_cg_q": 32, "k_sp_cg_r": 24}
 # fused FEM CG schedule, per node of 3 fp64 components:
 # phase A reads x, r, p_old, writes x, p_new, q; phase B reads r, q, writes r
 FEM_BYTES = {"k_fem_cg_a": 144, "k_fem_r": 72}
@@ -538,7 +542,7 @@ def bench_sparse_run(n, steps, warmup, world, local):
             "ms_per_step": ms / steps, "scaling": "strong", "dtype": "f64",
             "config": {"workload": f"C4 element-sparse sphere r=0.41528N in {n}^3 ({nact} active, "
                                    f"{nact / n ** 3:.2%}), 7-point CG fp64 (configs[3])",
-                       "schedule": f"3 passes, {per_cell} B/active cell/iter incl. 24 B connectivity"},
+                       "schedule": f"3 passes, {per_cell} B/active cell/iter incl. the 16 B segment-indexed neighbour table"},
             "hbm_gbs": per_cell * nact * steps / t / 1e9, "hbm_frac": per_cell * nact * steps / t / 1e9 / hbm,
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm, "unit": "GB/s",
                          "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": ncu_traffic(dom),

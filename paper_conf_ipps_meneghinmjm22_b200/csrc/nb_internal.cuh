@@ -138,7 +138,15 @@ struct NbSparsePart {
     // the segments of the boundary planes facing a neighbour (OCC: one
     // launch for both), entries as d_seg (lazy)
     int32_t *d_seg_bnd = nullptr;
+    int32_t *d_seg_bnd_gi = nullptr;  // their indices in the full segment table
     int64_t n_seg_bnd = -1;
+    // segment-indexed 7-point neighbour table (nb_sparse.cu "segment
+    // table"): d_nbr[s * 256 + t] = {-z, +z, -y | x flags, +y} offsets of the
+    // segment's cell t; d_seginfo[s] = {first own cell, cells, plane << 16 |
+    // index}: one dependent level before the operand gathers
+    void *d_nbr = nullptr;
+    void *d_seginfo = nullptr;
+    int64_t n_runs = 0;
 };
 
 struct nb_grid {

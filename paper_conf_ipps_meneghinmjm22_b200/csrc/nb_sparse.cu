@@ -44,7 +44,12 @@ void nb_sparse_free(nb_grid *g) {
         cudaFree(s.d_pstart);
         cudaFree(s.d_seg);
         cudaFree(s.d_seg_bnd);
-        s.d_seg_bnd = nullptr;
+        cudaFree(s.d_seg_bnd_gi);
+        cudaFree(s.d_nbr);
+        cudaFree(s.d_seginfo);
+        s.d_seg_bnd = s.d_seg_bnd_gi = nullptr;
+        s.d_nbr = s.d_seginfo = nullptr;
+        s.n_runs = 0;
         s.n_seg_bnd = -1;
         s.conn = s.coord = nullptr;
         s.d_pstart = nullptr;
@@ -76,6 +81,7 @@ __global__ void k_sp_conn(const uint8_t *__restrict__ mask, const int32_t *__res
 }
 
 static nb_status sp_bnd_segments(nb_grid *g, int p);
+static nb_status sp_build_runs(nb_grid *g, int p);
 
 extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t *active, int32_t nparts,
                                            const int32_t *device_ids, nb_comm *comm, nb_grid **out) {
@@ -190,6 +196,7 @@ extern "C" nb_status nb_grid_create_sparse(const int32_t dims[3], const uint8_t 
         if (s == NB_OK && !segs.empty())
             cudaMemcpyAsync(sp.d_seg, segs.data(), sizeof(int32_t) * segs.size(), cudaMemcpyHostToDevice, g->cs);
         if (s == NB_OK) s = sp_bnd_segments(g, p);  // built here: the CG hooks may run under graph capture
+        if (s == NB_OK) s = sp_build_runs(g, p);
         if (s == NB_OK && q.nz() > 0) {
             dim3 blk(128), grd((nx + 127) / 128, ny, q.nz());
             LaunchScope ls(g, g->cs, "k_sp_conn");
@@ -718,6 +725,12 @@ __global__ void __launch_bounds__(SEG) k_sp_lap(const T *x, T *y, const int32_t 
     y[hl + j] = fma(T(-6), x[hl + j], s);
 }
 
+struct SpRun;
+static bool sp_use_runs(const NbSparsePart &sp);
+template <int K>
+static nb_status sp_launch_runs(nb_grid *g, int p, const int32_t *list, const int32_t *gidx, int64_t s0, int64_t n,
+                                SpArgs A, int plane_base, const char *name);
+
 // launch over the non-empty segments of local planes [zb, ze)
 template <int K>
 static nb_status sp_launch(nb_grid *g, int p, int zb, int ze, SpArgs A, int plane_base, const char *name) {
@@ -725,6 +738,8 @@ static nb_status sp_launch(nb_grid *g, int p, int zb, int ze, SpArgs A, int plan
     const NbSparsePart &sp = g->sp[p];
     const int64_t s0 = sp.seg_start[zb], s1 = sp.seg_start[ze];
     if (s1 <= s0) return NB_OK;
+    if constexpr (K == SPK_CG_Q || K == SPK_CG_INIT)
+        if (sp_use_runs(sp)) return sp_launch_runs<K>(g, p, sp.d_seg, nullptr, s0, s1 - s0, A, plane_base, name);
     A.seg = sp.d_seg;
     A.seg0 = s0;
     A.nseg = s1 - s0;
@@ -746,6 +761,8 @@ static nb_status sp_launch_list(nb_grid *g, int p, const int32_t *list, int64_t 
                                 const char *name) {
     if (n <= 0) return NB_OK;
     const NbSparsePart &sp = g->sp[p];
+    if constexpr (K == SPK_CG_Q || K == SPK_CG_INIT)
+        if (sp_use_runs(sp)) return sp_launch_runs<K>(g, p, list, sp.d_seg_bnd_gi, 0, n, A, plane_base, name);
     A.seg = list;
     A.seg0 = 0;
     A.nseg = n;
@@ -773,11 +790,298 @@ static nb_status sp_bnd_segments(nb_grid *g, int p) {
     };
     if (q.lo >= 0) add(0);
     if (q.hi >= 0 && q.nz() > 1) add(q.nz() - 1);
+    std::vector<int32_t> gi;  // index of each entry in the full (plane-major) segment table
+    for (int32_t e : segs) gi.push_back((int32_t)(sp.seg_start[e >> 16] + (e & 0xffff)));
     NB_CUDA(cudaMalloc(&sp.d_seg_bnd, sizeof(int32_t) * std::max<size_t>(segs.size(), 1)));
-    if (!segs.empty())
+    NB_CUDA(cudaMalloc(&sp.d_seg_bnd_gi, sizeof(int32_t) * std::max<size_t>(segs.size(), 1)));
+    if (!segs.empty()) {
         NB_CUDA(cudaMemcpy(sp.d_seg_bnd, segs.data(), sizeof(int32_t) * segs.size(), cudaMemcpyHostToDevice));
+        NB_CUDA(cudaMemcpy(sp.d_seg_bnd_gi, gi.data(), sizeof(int32_t) * gi.size(), cudaMemcpyHostToDevice));
+    }
     sp.n_seg_bnd = (int64_t)segs.size();
     return NB_OK;
+}
+
+// ---------------------------------------------------------------------------
+// x-runs (the C4 q pass without a per-cell connectivity table).  PAPER.md
+// L248 stores the sparse grid "with their connectivity table" and leaves the
+// format open; the 7-point stencil only needs, per run of consecutive active
+// cells along x, whether the +-x ends continue and where the +-y / +-z
+// neighbour run starts.  A run is cut wherever a neighbour row starts or
+// stops being active, and at every 256-cell dot segment boundary, so each
+// of the four offsets is constant over the run (or the whole run's neighbour
+// is inactive -> outside).  24 B per run instead of 24 B per cell.
+// ---------------------------------------------------------------------------
+struct SpRun {
+    int32_t start;   // own index of the first cell
+    int16_t len;     // cells (<= SEG)
+    int16_t flags;   // bit 0: the first cell's -x neighbour is active (= own cell start - 1), bit 1: the last cell's +x
+    int32_t off[4];  // -y, +y, -z, +z: buffer index of the neighbour minus the cell's own buffer index
+};
+constexpr int32_t SP_NONE = INT32_MIN;
+static_assert(sizeof(SpRun) == 24, "SpRun layout");
+
+static nb_status sp_build_runs(nb_grid *g, int p) {
+    NbSparsePart &sp = g->sp[p];
+    const NbPart &q = g->parts[p];
+    const int nx = g->nx, ny = g->ny;
+    const int64_t plane = (int64_t)nx * ny;
+    struct XRun {
+        int x0, x1;
+        int64_t rank;  // rank of the cell x0 among its plane's active cells
+    };
+    // planes z0 - 1 .. z1 (halo planes only where a neighbour partition exists)
+    const int zlo = q.lo >= 0 ? q.z0 - 1 : q.z0, zhi = q.hi >= 0 ? q.z1 + 1 : q.z1;
+    std::vector<std::vector<XRun>> runs(zhi - zlo);
+    std::vector<std::vector<int32_t>> rowbeg(zhi - zlo);
+    for (int z = zlo; z < zhi; ++z) {
+        auto &R = runs[z - zlo];
+        auto &B = rowbeg[z - zlo];
+        B.assign(ny + 1, 0);
+        const uint8_t *m = g->host_mask.data() + (int64_t)z * plane;
+        int64_t rank = 0;
+        for (int y = 0; y < ny; ++y) {
+            B[y] = (int32_t)R.size();
+            const uint8_t *row = m + (int64_t)y * nx;
+            for (int x = 0; x < nx;) {
+                if (!row[x]) {
+                    ++x;
+                    continue;
+                }
+                int x0 = x;
+                while (x < nx && row[x]) ++x;
+                R.push_back({x0, x, rank});
+                rank += x - x0;
+            }
+        }
+        B[ny] = (int32_t)R.size();
+    }
+    // buffer index of the first cell of plane z ([halo_lo | own | halo_hi])
+    auto base = [&](int z) -> int64_t {
+        if (z < q.z0) return 0;
+        if (z >= q.z1) return sp.hl + sp.n;
+        return sp.hl + sp.pstart[z - q.z0];
+    };
+    std::vector<SpRun> out;
+    std::vector<int32_t> rseg;  // first run of every segment, plane-major
+    std::vector<int> cuts;
+    for (int z = q.z0; z < q.z1; ++z) {
+        const int zl = z - q.z0;
+        const auto &R = runs[z - zlo];
+        const auto &B = rowbeg[z - zlo];
+        const int64_t p0 = sp.pstart[zl];
+        for (int y = 0; y < ny; ++y) {
+            // neighbour rows: -y, +y, -z, +z (plane index into runs, row) or none
+            int nz_[4], ny_[4];
+            nz_[0] = z, ny_[0] = y - 1;
+            nz_[1] = z, ny_[1] = y + 1;
+            nz_[2] = z - 1, ny_[2] = y;
+            nz_[3] = z + 1, ny_[3] = y;
+            bool has[4];
+            for (int d = 0; d < 4; ++d) has[d] = ny_[d] >= 0 && ny_[d] < ny && nz_[d] >= zlo && nz_[d] < zhi;
+            for (int k = B[y]; k < B[y + 1]; ++k) {
+                const XRun &r = R[k];
+                cuts.clear();
+                cuts.push_back(r.x0);
+                cuts.push_back(r.x1);
+                for (int d = 0; d < 4; ++d) {
+                    if (!has[d]) continue;
+                    const auto &NR = runs[nz_[d] - zlo];
+                    const auto &NB = rowbeg[nz_[d] - zlo];
+                    for (int m = NB[ny_[d]]; m < NB[ny_[d] + 1]; ++m) {
+                        if (NR[m].x0 > r.x0 && NR[m].x0 < r.x1) cuts.push_back(NR[m].x0);
+                        if (NR[m].x1 > r.x0 && NR[m].x1 < r.x1) cuts.push_back(NR[m].x1);
+                    }
+                }
+                // 256-cell segment boundaries of the plane's own order
+                for (int64_t sj = (r.rank + SEG - 1) / SEG * SEG; sj < r.rank + (r.x1 - r.x0); sj += SEG)
+                    if (sj > r.rank) cuts.push_back(r.x0 + (int)(sj - r.rank));
+                std::sort(cuts.begin(), cuts.end());
+                cuts.erase(std::unique(cuts.begin(), cuts.end()), cuts.end());
+                for (size_t c = 0; c + 1 < cuts.size(); ++c) {
+                    const int u = cuts[c], v = cuts[c + 1];
+                    SpRun o;
+                    const int64_t j = p0 + r.rank + (u - r.x0);
+                    o.start = (int32_t)j;
+                    o.len = (int16_t)(v - u);
+                    o.flags = (int16_t)((u > r.x0 ? 1 : 0) | (v < r.x1 ? 2 : 0));
+                    const int64_t own = sp.hl + j;
+                    for (int d = 0; d < 4; ++d) {
+                        o.off[d] = SP_NONE;
+                        if (!has[d]) continue;
+                        const auto &NR = runs[nz_[d] - zlo];
+                        const auto &NB = rowbeg[nz_[d] - zlo];
+                        for (int m = NB[ny_[d]]; m < NB[ny_[d] + 1]; ++m)
+                            if (NR[m].x0 <= u && u < NR[m].x1) {
+                                o.off[d] = (int32_t)(base(nz_[d]) + NR[m].rank + (u - NR[m].x0) - own);
+                                break;
+                            }
+                    }
+                    if ((j - p0) % SEG == 0) rseg.push_back((int32_t)out.size());
+                    out.push_back(o);
+                }
+            }
+        }
+    }
+    rseg.push_back((int32_t)out.size());
+    if ((int64_t)rseg.size() != sp.seg_start.back() + 1)
+        NB_FAIL(NB_ESTATE, "sparse x-runs: %zu segment starts, expected %lld", rseg.size() - 1,
+                (long long)sp.seg_start.back());
+    // the device table, segment-indexed so that a thread finds its cell's
+    // entry from (segment, lane) alone: per cell {-z, +z, -y << 2 | x flags,
+    // +y} (16 B; -y offsets fit 30 bits), per segment {first own cell,
+    // cells, plane << 16 | index}
+    const int64_t nseg = (int64_t)rseg.size() - 1;
+    std::vector<int4> nbr((size_t)nseg * SEG, make_int4(SP_NONE, SP_NONE, (SP_NONE >> 2) * 4, SP_NONE));
+    std::vector<int4> info((size_t)std::max<int64_t>(nseg, 1));
+    int64_t sgi = 0;
+    for (int zl = 0; zl < q.nz(); ++zl)
+        for (int64_t k = 0; k < sp.seg_start[zl + 1] - sp.seg_start[zl]; ++k, ++sgi) {
+            const int64_t j0 = sp.pstart[zl] + k * SEG;
+            const int64_t cnt = std::min<int64_t>(SEG, sp.pstart[zl + 1] - j0);
+            info[sgi] = make_int4((int32_t)j0, (int32_t)cnt, (zl << 16) | (int)k, 0);
+            for (int32_t m = rseg[sgi]; m < rseg[sgi + 1]; ++m) {
+                const SpRun &r = out[m];
+                for (int c = 0; c < r.len; ++c) {
+                    const int64_t j = r.start + c;
+                    const int fx = ((c > 0 || (r.flags & 1)) ? 1 : 0) | ((c < r.len - 1 || (r.flags & 2)) ? 2 : 0);
+                    const int32_t ylo = r.off[0] == SP_NONE ? (SP_NONE >> 2) : r.off[0];
+                    if (ylo < -(1 << 29) || ylo >= (1 << 29))
+                        NB_FAIL(NB_EUNSUPPORTED, "sparse neighbour table: -y offset out of range");
+                    nbr[(size_t)sgi * SEG + (j - j0)] = make_int4(r.off[2], r.off[3], (int32_t)((uint32_t)ylo << 2) | fx,
+                                                                  r.off[1]);
+                }
+            }
+        }
+    NB_CUDA(cudaMalloc(&sp.d_nbr, sizeof(int4) * std::max<size_t>(nbr.size(), 1)));
+    NB_CUDA(cudaMalloc(&sp.d_seginfo, sizeof(int4) * info.size()));
+    if (!nbr.empty()) NB_CUDA(cudaMemcpy(sp.d_nbr, nbr.data(), sizeof(int4) * nbr.size(), cudaMemcpyHostToDevice));
+    NB_CUDA(cudaMemcpy(sp.d_seginfo, info.data(), sizeof(int4) * info.size(), cudaMemcpyHostToDevice));
+    sp.n_runs = (int64_t)out.size();
+    return NB_OK;
+}
+
+// 2 segments per block at 6 blocks per SM (40 registers): q pass 0.267 ms
+// at 512^3 on the sphere, against 0.284 (2, 5), 0.299 (1, 6 or 8), 0.287
+// (4, 3), 0.336 (2, 7: spills) and 0.317 for the connectivity-table path
+#ifndef NB_SPR_MINB
+#define NB_SPR_MINB 6
+#endif
+#ifndef NB_SPR_NSB
+#define NB_SPR_NSB 2
+#endif
+constexpr int NSBR = NB_SPR_NSB;  // segments per block of the table-indexed passes
+// The 7-point CG passes on the segment-indexed neighbour table
+// (SPK_CG_Q: q = A p, <p, q>; SPK_CG_INIT: r = b - A x, <r, r>): the same
+// cells per thread, the same canonical neighbour order -x, +x, -y, +y, -z,
+// +z and the same per-segment dot tree as k_sp, so the results are bitwise
+// those of the connectivity-table path.  The table is indexed by (segment,
+// lane): ONE dependent level (segment info + the cell's 16-byte entry, both
+// addressed from blockIdx / threadIdx) before the operand gathers, instead
+// of segment entry -> plane start -> 24-byte connectivity -> gathers.
+template <int K>
+__global__ void __launch_bounds__(SEG, NB_SPR_MINB) k_sp_runs(SpArgs A, const int4 *__restrict__ nbrt,
+                                                             const int4 *__restrict__ seginfo,
+                                                             const int32_t *__restrict__ gidx) {
+    __shared__ double sw[NSBR][SEG / 32];
+    const int t = threadIdx.x;
+    int4 inf[NSBR], nb4[NSBR];
+#pragma unroll
+    for (int k = 0; k < NSBR; ++k) {
+        const int64_t q = (int64_t)blockIdx.x * NSBR + k;
+        const int64_t qc = q < A.nseg ? q : A.nseg - 1;
+        const int64_t gi = gidx ? (int64_t)__ldg(gidx + qc) : A.seg0 + qc;
+        inf[k] = __ldg(seginfo + gi);
+        nb4[k] = __ldg(nbrt + gi * SEG + t);
+        if (q >= A.nseg) inf[k].y = 0;  // no cells
+    }
+    if (K == SPK_CG_Q && A.sc->status != 0) return;
+    const double outv = K == SPK_CG_INIT ? A.outside : 0.0;
+    int64_t i[NSBR];
+    bool valid[NSBR];
+    int32_t nb[NSBR][6];
+#pragma unroll
+    for (int k = 0; k < NSBR; ++k) {
+        valid[k] = t < inf[k].y;
+        const int32_t ii = (int32_t)(A.hl + inf[k].x + t);
+        i[k] = ii;
+        const int fx = nb4[k].z & 3;
+        const int32_t ylo = nb4[k].z >> 2;
+        nb[k][0] = valid[k] && (fx & 1) ? ii - 1 : -1;
+        nb[k][1] = valid[k] && (fx & 2) ? ii + 1 : -1;
+        nb[k][2] = valid[k] && ylo != (SP_NONE >> 2) ? ii + ylo : -1;
+        nb[k][3] = valid[k] && nb4[k].w != SP_NONE ? ii + nb4[k].w : -1;
+        nb[k][4] = valid[k] && nb4[k].x != SP_NONE ? ii + nb4[k].x : -1;
+        nb[k][5] = valid[k] && nb4[k].y != SP_NONE ? ii + nb4[k].y : -1;
+    }
+    double c[NSBR], bb[NSBR], v[NSBR][6];
+#pragma unroll
+    for (int k = 0; k < NSBR; ++k) {
+        c[k] = valid[k] ? __ldg(A.a + i[k]) : 0.0;
+        bb[k] = (K == SPK_CG_INIT && valid[k]) ? __ldg(A.b + i[k]) : 0.0;
+    }
+#pragma unroll
+    for (int k = 0; k < NSBR; ++k)
+#pragma unroll
+        for (int d = 0; d < 6; ++d) v[k][d] = nb[k][d] >= 0 ? __ldg(A.a + nb[k][d]) : outv;
+    double prod[NSBR];
+#pragma unroll
+    for (int k = 0; k < NSBR; ++k) {
+        prod[k] = 0.0;
+        if (!valid[k]) continue;
+        double s = v[k][0];
+#pragma unroll
+        for (int d = 1; d < 6; ++d) s = s + v[k][d];
+        const double ac = fma(6.0, c[k], -s);
+        if (K == SPK_CG_INIT) {
+            const double r = __dsub_rn(bb[k], ac);
+            A.c[i[k]] = r;
+            prod[k] = __dmul_rn(r, r);
+        } else {
+            A.c[i[k]] = ac;
+            prod[k] = __dmul_rn(c[k], ac);
+        }
+    }
+    const int w = t >> 5;
+#pragma unroll
+    for (int k = 0; k < NSBR; ++k) {
+        const double vv = warp_sum_canon(prod[k]);
+        if ((t & 31) == 0) sw[k][w] = vv;
+    }
+    __syncthreads();
+    if (t < NSBR) {
+        int4 it = inf[0];
+#pragma unroll
+        for (int k = 1; k < NSBR; ++k)
+            if (t == k) it = inf[k];
+        if (it.y > 0) {
+            double sum = sw[t][0];
+#pragma unroll
+            for (int ww = 1; ww < SEG / 32; ++ww) sum = __dadd_rn(sum, sw[t][ww]);
+            A.tp[(int64_t)(A.plane0 + (it.z >> 16)) * A.T + (it.z & 0xffff)] = sum;
+        }
+    }
+}
+
+static bool sp_use_runs(const NbSparsePart &sp) { return sp.d_nbr && !getenv("NB_SP_CONN"); }
+
+template <int K>
+static nb_status sp_launch_runs(nb_grid *g, int p, const int32_t *list, const int32_t *gidx, int64_t s0, int64_t n,
+                                SpArgs A, int plane_base, const char *name) {
+    const NbSparsePart &sp = g->sp[p];
+    A.seg = list;
+    A.seg0 = s0;
+    A.nseg = n;
+    A.pstart = sp.d_pstart;
+    A.n = sp.n;
+    A.hl = sp.hl;
+    A.plane0 = plane_base + g->parts[p].z0;
+    A.T = g->T;
+    A.tp = g->tp;
+    LaunchScope ls(g, g->cs, name);
+    k_sp_runs<K><<<(unsigned)((n + NSBR - 1) / NSBR), SEG, 0, g->cs>>>(A, (const int4 *)sp.d_nbr,
+                                                                    (const int4 *)sp.d_seginfo, gidx);
+    return nb_launch_check(name);
 }
 
 nb_status nb_sparse_dot_partials(const nb_field *x, const nb_field *y) {

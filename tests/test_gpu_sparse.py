@@ -191,3 +191,24 @@ def test_sparse_cg_occ_modes_bitwise_equal():
                 assert np.array_equal(x, ref[0]) and r.rr == ref[1], (parts, occ, halo)
     xo, ro, _ = oracle.cg(b, max_iter=11, op=oracle.OP_SPARSE7, mask=m)
     assert np.max(np.abs(ref[0] - xo)) <= 1e-11 * np.max(np.abs(xo))
+
+
+@pytest.mark.parametrize("parts", [1, 3])
+def test_sparse_cg_xruns_bitwise_equal_connectivity_table(parts, monkeypatch):
+    """The q pass / set-up on x-runs (24 B per run) and on the per-cell
+    connectivity table (NB_SP_CONN=1, 24 B per cell) compute the same
+    neighbours in the same order: bitwise equal CG iterates, on the sphere and
+    on a mask with holes, runs split by neighbour rows and segment edges."""
+    n = 40
+    rng = np.random.default_rng(3)
+    masks = [sphere(n), (sphere(n) & (rng.random((n, n, n)) < 0.8)).astype(np.uint8)]
+    for m in masks:
+        b = np.where(m, synth.uniform((n, n, n), seed=6), 0.0)
+        monkeypatch.delenv("NB_SP_CONN", raising=False)
+        xa, ra = run_sparse_cg(m, b, parts, 9)
+        monkeypatch.setenv("NB_SP_CONN", "1")
+        xb, rb = run_sparse_cg(m, b, parts, 9)
+        monkeypatch.delenv("NB_SP_CONN", raising=False)
+        assert np.array_equal(xa, xb) and ra.rr == rb.rr and ra.rr0 == rb.rr0
+        xo, ro, _ = oracle.cg(b, max_iter=9, op=oracle.OP_SPARSE7, mask=m)
+        assert np.max(np.abs(xa - xo)) <= 1e-11 * np.max(np.abs(xo))
