@@ -695,6 +695,42 @@ def bench_skeleton(local, n=512, parts=4, iters=10):
     ms_sk = t(sk.run)
     ms_fused = t(lambda: nb.nb_map_stencil_reduce(x, y, 0.125, iters, nb.OCC_TWO_WAY))
     sk.close()
+    # Listing 3 CG as containers with device scalars,
+    # against the hand-fused 2-phase CG on the same grid (bitwise equal:
+    # tests/test_gpu_skeleton.py)
+    RR, PQ, AL, BE, RR2 = 0, 1, 2, 3, 4
+    b, r, p, q = nb.Field(g), nb.Field(g), nb.Field(g), nb.Field(g)
+    b.fill(nb.FILL_POISSON_RHS)
+    x.fill_const(0.0), p.fill_const(0.0), q.fill_const(0.0)
+    nb.nb_axpby(1.0, b, 0.0, r)
+    with nb.Skeleton(g, nb.OCC_TWO_WAY) as s0:
+        s0.dot(r, r, RR)
+        s0.set_scalar(BE, 0.0)
+        s0.run()
+    cgk = nb.Skeleton(g, nb.OCC_TWO_WAY)
+    cgk.axpby_s(1.0, -1, r, 1.0, BE, p)
+    cgk.poisson(p, q)
+    cgk.dot(p, q, PQ)
+    cgk.scalar(nb.SC_DIV, RR, PQ, AL)
+    cgk.axpby_s(1.0, AL, p, 1.0, -1, x)
+    cgk.axpby_s(-1.0, AL, q, 1.0, -1, r)
+    cgk.dot(r, r, RR2)
+    cgk.scalar(nb.SC_DIV, RR2, RR, BE)
+    cgk.scalar(nb.SC_COPY, RR2, 0, RR)
+    cplan = cgk.describe()
+
+    def run_cg_sk():
+        for _ in range(iters):
+            cgk.run()
+    ms_cg_sk = t(run_cg_sk)
+    cgk.close()
+    x.fill_const(0.0)
+    cg = nb.CG(x, b, occ=nb.OCC_TWO_WAY)
+    cg.prepare(iters)
+    ms_cg_fused = t(lambda: cg.iterate(iters))
+    cg.close()
+    for f in (b, r, p, q):
+        f.close()
     x.close(), y.close()
     g.close()
     cells = n ** 3
@@ -703,7 +739,15 @@ def bench_skeleton(local, n=512, parts=4, iters=10):
             "skeleton_gbs": 56 * cells / ms_sk / 1e6, "fused_gbs": 32 * cells / ms_fused / 1e6,
             "nodes": len(plan["nodes"]), "streams": plan["streams"], "events": plan["events"],
             "note": "skeleton = unfused containers (24 + 16 + 16 = 56 B/cell/iter), as Neon generates them; "
-                    "fused = one kernel per iteration (32 B/cell/iter)"}
+                    "fused = one kernel per iteration (32 B/cell/iter)",
+            "listing3_cg": {"workload": f"Listing 3 CG (UpdateP first, device-scalar alpha / beta), {n}^3 fp64, "
+                                        f"{parts} partitions, Two-way OCC",
+                            "skeleton_ms_per_iter": ms_cg_sk, "fused_ms_per_iter": ms_cg_fused,
+                            "skeleton_mlups": cells / ms_cg_sk / 1e3, "fused_mlups": cells / ms_cg_fused / 1e3,
+                            "skeleton_gbs": 112 * cells / ms_cg_sk / 1e6, "fused_gbs": 64 * cells / ms_cg_fused / 1e6,
+                            "nodes": len(cplan["nodes"]), "streams": cplan["streams"], "events": cplan["events"],
+                            "note": "skeleton = the paper's 6 containers + 3 scalar steps (112 B/cell/iter); fused "
+                                    "= 2 phase kernels (64 B/cell/iter); bitwise equal iterates"}}
 
 
 # ---------------------------------------------------------------------------

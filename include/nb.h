@@ -354,15 +354,44 @@ nb_status nb_fem27_rhs(nb_field *b, double pressure);
  * then a schedule (L333-L396: BFS levels, a stream per concurrent node of
  * the widest level with parent-stream reuse, an event per cross-stream
  * dependency, task order by BFS over data edges + hints).
- * Containers: y = a x + b y (MapOp), y = L(x) (StencilOp, 7-point), and
- * <x, y> -> result slot (ReduceOp, the deterministic dot). */
-typedef enum { NB_SK_AXPBY = 0, NB_SK_LAPLACE7 = 1, NB_SK_DOT = 2 } nb_container_op;
+ * Containers (Listing 3 CG, L154-L163, and the LBM step, L447-L451, are
+ * expressible):
+ *   AXPBY    y = A x + B y (MapOp).  A = a, or a * s[a_slot] when flags has
+ *            NB_SK_A_SLOT (a device scalar: a result slot); B likewise.  Per element:
+ *            b == 1 (immediate): fma(A, x, y); a == 1 (immediate) with a
+ *            device-scalar B: fma(B, y, x) (UpdateP p = r + beta p);
+ *            b == 0 (immediate): A x; otherwise fma(A, x, B y).
+ *   LAPLACE7 y = L(x) (StencilOp, 7-point, L = sum of 6 neighbours - 6 x)
+ *   POISSON  y = A x = -L(x) = fma(6, x_c, -sum) (StencilOp; the CG operator)
+ *   DOT      <x, y> -> slot (ReduceOp, the deterministic dot)
+ *   SCALAR   s[slot] = s[x] / s[y] (NB_SC_DIV), s[x] (NB_SC_COPY) or a
+ *            (NB_SC_SET): a one-thread device step between reductions
+ *            (alpha = rr / pq, beta = rr' / rr, rr = rr'); x, y are slots
+ *   LBM      y = D3Q19 BGK pull step of x (StencilOp on fp32 cardinality-19
+ *            fields; a = omega, b = u_lid, c = rho_w, sop = bc, CAVITY only);
+ *            its halo carries the 5 + 5 z-crossing populations (L256). */
+typedef enum {
+    NB_SK_AXPBY = 0,
+    NB_SK_LAPLACE7 = 1,
+    NB_SK_DOT = 2,
+    NB_SK_POISSON = 3,
+    NB_SK_SCALAR = 4,
+    NB_SK_LBM = 5
+} nb_container_op;
+typedef enum { NB_SC_DIV = 0, NB_SC_COPY = 1, NB_SC_SET = 2 } nb_scalar_op;
 typedef struct {
-    int32_t op;    /* nb_container_op                                         */
-    int32_t x, y;  /* field ids (any non-negative integers naming the data)    */
-    int32_t slot;  /* NB_SK_DOT: result slot in [0, 1024)                      */
-    double a, b;   /* NB_SK_AXPBY coefficients                                 */
+    int32_t op;             /* nb_container_op                                         */
+    int32_t x, y;           /* field ids (any non-negative integers naming the data);
+                               SCALAR: source slots                                    */
+    int32_t slot;           /* DOT / SCALAR: result slot in [0, 1024)                  */
+    double a, b;            /* AXPBY coefficients; SCALAR (SET): a; LBM: omega, u_lid   */
+    int32_t a_slot, b_slot; /* AXPBY with NB_SK_A_SLOT / NB_SK_B_SLOT: device scalar slots */
+    int32_t sop;            /* SCALAR: nb_scalar_op; LBM: nb_lbm_bc                      */
+    int32_t flags;          /* NB_SK_A_SLOT | NB_SK_B_SLOT (0: immediate coefficients)   */
+    double c;               /* LBM: rho_w                                               */
 } nb_container;
+#define NB_SK_A_SLOT 1
+#define NB_SK_B_SLOT 2
 /* Pure host logic (no GPU): plan n containers for an nparts-slab grid and
  * write the plan as JSON into json (cap bytes; json = NULL: only *len) —
  * {"nodes": [{id, name, op, view, container, incoherent, finalize, level,
@@ -375,8 +404,18 @@ typedef struct nb_skeleton nb_skeleton;
  * the grid cannot be destroyed while it lives (NB_ESTATE). */
 nb_status nb_skeleton_create(nb_grid *grid, nb_occ occ, nb_skeleton **out);
 nb_status nb_skeleton_axpby(nb_skeleton *sk, double a, nb_field *x, double b, nb_field *y);
+/* AXPBY with device-scalar coefficients: a_slot / b_slot >= 0 selects a
+ * slot (a, b scale it), -1 keeps the immediate (see above) */
+nb_status nb_skeleton_axpby_s(nb_skeleton *sk, double a, int32_t a_slot, nb_field *x, double b, int32_t b_slot,
+                              nb_field *y);
 nb_status nb_skeleton_laplace7(nb_skeleton *sk, nb_field *x, nb_field *y);
+nb_status nb_skeleton_poisson(nb_skeleton *sk, nb_field *x, nb_field *y);
 nb_status nb_skeleton_dot(nb_skeleton *sk, nb_field *x, nb_field *y, int32_t slot);
+nb_status nb_skeleton_scalar(nb_skeleton *sk, nb_scalar_op sop, int32_t in0, int32_t in1, int32_t out, double a);
+/* fin, fout: fp32 cardinality-19 fields (twoPop: the next step swaps them) */
+nb_status nb_skeleton_lbm(nb_skeleton *sk, nb_field *fin, nb_field *fout, const nb_lbm_params *params);
+/* s[slot] = value, stream-ordered on the grid's compute stream */
+nb_status nb_skeleton_set_scalar(nb_skeleton *sk, int32_t slot, double value);
 /* builds the plan, streams and events (implicit in the first run) */
 nb_status nb_skeleton_compile(nb_skeleton *sk);
 /* enqueue every task in plan order on its stream (asynchronous; ordered

@@ -64,10 +64,13 @@ class LbmParams(C.Structure):
 
 class Container(C.Structure):
     _fields_ = [("op", C.c_int32), ("x", C.c_int32), ("y", C.c_int32), ("slot", C.c_int32),
-                ("a", C.c_double), ("b", C.c_double)]
+                ("a", C.c_double), ("b", C.c_double), ("a_slot", C.c_int32), ("b_slot", C.c_int32),
+                ("sop", C.c_int32), ("flags", C.c_int32), ("c", C.c_double)]
 
 
-SK_AXPBY, SK_LAPLACE7, SK_DOT = 0, 1, 2
+SK_AXPBY, SK_LAPLACE7, SK_DOT, SK_POISSON, SK_SCALAR, SK_LBM = 0, 1, 2, 3, 4, 5
+SC_DIV, SC_COPY, SC_SET = 0, 1, 2
+SK_A_SLOT, SK_B_SLOT = 1, 2
 
 
 # exported symbols and their ctypes signatures (the whole of include/nb.h)
@@ -126,8 +129,13 @@ SIGNATURES = {
     "nb_skeleton_plan": ([I32, I32, P, I32, P, I64, P], I32),
     "nb_skeleton_create": ([P, I32, PP], I32),
     "nb_skeleton_axpby": ([P, D, P, D, P], I32),
+    "nb_skeleton_axpby_s": ([P, D, I32, P, D, I32, P], I32),
     "nb_skeleton_laplace7": ([P, P, P], I32),
+    "nb_skeleton_poisson": ([P, P, P], I32),
     "nb_skeleton_dot": ([P, P, P, I32], I32),
+    "nb_skeleton_scalar": ([P, I32, I32, I32, I32, D], I32),
+    "nb_skeleton_lbm": ([P, P, P, P], I32),
+    "nb_skeleton_set_scalar": ([P, I32, D], I32),
     "nb_skeleton_compile": ([P], I32),
     "nb_skeleton_run": ([P], I32),
     "nb_skeleton_result": ([P, I32, P], I32),
@@ -613,11 +621,16 @@ def _json_out(call):
 
 def nb_skeleton_plan(nparts: int, occ: int, containers) -> dict:
     """Pure host planning (no GPU).  containers: (op, x, y, a, b, slot)
-    tuples with integer field ids; returns the plan (nodes, data edges,
-    hints, task order, streams, events)."""
+    tuples with integer field ids, optionally followed by (a_slot, b_slot,
+    sop): device-scalar coefficient slots (-1: immediate) and the scalar op;
+    returns the plan (nodes, data edges, hints, task order, streams,
+    events)."""
     arr = (Container * max(len(containers), 1))()
-    for i, (op, x, y, a, b, slot) in enumerate(containers):
-        arr[i] = Container(op, x, y, slot, a, b)
+    for i, t in enumerate(containers):
+        op, x, y, a, b, slot = t[:6]
+        a_slot, b_slot, sop = (tuple(t[6:9]) + (-1, -1, 0)[len(t[6:9]):])
+        flags = (SK_A_SLOT if a_slot >= 0 else 0) | (SK_B_SLOT if b_slot >= 0 else 0)
+        arr[i] = Container(op, x, y, slot, a, b, a_slot, b_slot, sop, flags, 0.0)
     return _json_out(lambda buf, cap, n: lib().nb_skeleton_plan(int(nparts), int(occ), arr, len(containers),
                                                                  buf, cap, n))
 
@@ -639,9 +652,30 @@ class Skeleton:
     def axpy(self, a: float, x: Field, y: Field):
         self.axpby(a, x, 1.0, y)
 
+    def axpby_s(self, a: float, a_slot: int, x: Field, b: float, b_slot: int, y: Field):
+        """y = A x + B y with A = a * s[a_slot] (a_slot >= 0) or a, B likewise."""
+        self.fields += [x, y]
+        _check(lib().nb_skeleton_axpby_s(self.handle, float(a), int(a_slot), _h(x), float(b), int(b_slot), _h(y)))
+
     def laplace7(self, x: Field, y: Field):
         self.fields += [x, y]
         _check(lib().nb_skeleton_laplace7(self.handle, _h(x), _h(y)))
+
+    def poisson(self, x: Field, y: Field):
+        """y = A x = -L(x) (the CG operator)."""
+        self.fields += [x, y]
+        _check(lib().nb_skeleton_poisson(self.handle, _h(x), _h(y)))
+
+    def scalar(self, sop: int, in0: int, in1: int, out: int, a: float = 0.0):
+        _check(lib().nb_skeleton_scalar(self.handle, int(sop), int(in0), int(in1), int(out), float(a)))
+
+    def lbm(self, fin: Field, fout: Field, omega: float, u_lid: float = 0.05, rho_w: float = 1.0):
+        self.fields += [fin, fout]
+        prm = LbmParams(omega, u_lid, rho_w, LBM_CAVITY)
+        _check(lib().nb_skeleton_lbm(self.handle, _h(fin), _h(fout), C.byref(prm)))
+
+    def set_scalar(self, slot: int, value: float):
+        _check(lib().nb_skeleton_set_scalar(self.handle, int(slot), float(value)))
 
     def dot(self, x: Field, y: Field, slot: int):
         self.fields += [x, y]

@@ -375,6 +375,11 @@ nb_status nb_nccl_send(nb_grid *g, const void *buf, size_t bytes, int peer, cuda
 nb_status nb_nccl_recv(nb_grid *g, void *buf, size_t bytes, int peer, cudaStream_t s);
 
 int nb_part_owner(const nb_grid *g, int part);
+// y = L(x) or y = -L(x) on a view (nb_stencil.cu); the D3Q19 step of fin
+// into fout on a view without fused halo stores (nb_lbm.cu): Skeleton nodes
+nb_status nb_stencil7(const nb_field *x, nb_field *y, nb_view v, bool neg);
+nb_status nb_lbm_view(nb_field *fin, nb_field *fout, const nb_lbm_params *prm, nb_view v);
+std::vector<std::pair<int, int>> view_ranges(const nb_grid *g, int p, nb_view v);
 // multi-process with the peer-memory transport
 inline bool nb_is_peer(const nb_grid *g) { return g->comm && g->comm->world > 1 && g->comm->peer; }
 // multi-process with the NCCL transport

@@ -411,6 +411,22 @@ static nb_status launch_lbm(nb_grid *g, int p, nb_field *fin, nb_field *fout, co
     return nb_launch_check("k_lbm_d3q19");
 }
 
+// one step of fin into fout on the planes of view v of every local
+// partition, halos as they are (the Skeleton's LBM container: its halo node
+// runs before, explicitly); cavity boundaries
+nb_status nb_lbm_view(nb_field *fin, nb_field *fout, const nb_lbm_params *prm, nb_view v) {
+    NB_TRY(lbm_check(fin));
+    NB_TRY(lbm_check(fout));
+    if (fin->g != fout->g) NB_FAIL(NB_EMISMATCH, "fin and fout belong to different grids");
+    if (fin == fout) NB_FAIL(NB_EINVAL, "twoPop needs two distinct buffers");
+    if (prm->bc != NB_LBM_CAVITY) NB_FAIL(NB_EUNSUPPORTED, "Skeleton LBM containers: cavity boundaries");
+    nb_grid *g = fin->g;
+    if (g->sparse) NB_FAIL(NB_EUNSUPPORTED, "Skeleton LBM containers: dense grids");
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+        for (auto rg : view_ranges(g, p, v)) NB_TRY(launch_lbm(g, p, fin, fout, prm, rg.first, rg.second, false));
+    return NB_OK;
+}
+
 extern "C" nb_status nb_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm_params *prm, int32_t nsteps,
                                  nb_occ occ) {
     if (!pfin || !pfout || !prm) NB_FAIL(NB_EINVAL, "nb_lbm_step: NULL argument");

@@ -47,11 +47,13 @@ namespace {
 enum : int { R_HLO = 1, R_BLO = 2, R_CORE = 4, R_BHI = 8, R_HHI = 16 };
 constexpr int R_OWN = R_BLO | R_CORE | R_BHI, R_ALL = R_OWN | R_HLO | R_HHI;
 
-enum SkOp { SK_MAP = 0, SK_STENCIL = 1, SK_REDUCE = 2, SK_HALO = 3 };
+enum SkOp { SK_MAP = 0, SK_STENCIL = 1, SK_REDUCE = 2, SK_HALO = 3, SK_SCALAR = 4 };
 const char *op_name(int op) {
-    static const char *n[] = {"map", "stencil", "reduce", "halo"};
+    static const char *n[] = {"map", "stencil", "reduce", "halo", "scalar"};
     return n[op];
 }
+// StencilOps read their input's halo (radius 1)
+bool is_stencil(int op) { return op == NB_SK_LAPLACE7 || op == NB_SK_POISSON || op == NB_SK_LBM; }
 const char *view_name(nb_view v) {
     static const char *n[] = {"standard", "internal", "boundary"};
     return n[v];
@@ -78,6 +80,7 @@ struct Node {
     nb_view view = NB_VIEW_STANDARD;
     int container = -1;   // index of the user Container (-1: halo node)
     int halo_field = -1;  // halo nodes
+    bool halo_lbm = false;  // halo of an LBM container: the 5 + 5 z-crossing populations
     bool incoherent = false;
     bool finalize = false;  // reduce part that completes the reduction
     std::vector<Access> acc;
@@ -164,13 +167,22 @@ nb_status build_nodes(const nb_container *c, int n, int nparts, nb_occ occ, Plan
         if (!on && it != coherent_fields.end()) coherent_fields.erase(it);
     };
     for (int i = 0; i < n; ++i) {
-        if (c[i].op < NB_SK_AXPBY || c[i].op > NB_SK_DOT) NB_FAIL(NB_EINVAL, "container %d: bad op %d", i, c[i].op);
+        if (c[i].op < NB_SK_AXPBY || c[i].op > NB_SK_LBM) NB_FAIL(NB_EINVAL, "container %d: bad op %d", i, c[i].op);
+        if (c[i].op == NB_SK_SCALAR) {
+            if (c[i].sop < NB_SC_DIV || c[i].sop > NB_SC_SET) NB_FAIL(NB_EINVAL, "container %d: bad scalar op", i);
+            if (c[i].slot < 0 || c[i].slot >= NB_DOT_SLOTS || c[i].x < 0 || c[i].x >= NB_DOT_SLOTS || c[i].y < 0 ||
+                c[i].y >= NB_DOT_SLOTS)
+                NB_FAIL(NB_EINVAL, "container %d: scalar slot out of range", i);
+            continue;
+        }
         if (c[i].x < 0 || c[i].y < 0 || c[i].x >= TP_FIELD || c[i].y >= TP_FIELD)
             NB_FAIL(NB_EINVAL, "container %d: bad field ids", i);
-        if (c[i].op == NB_SK_LAPLACE7 && c[i].x == c[i].y) NB_FAIL(NB_EINVAL, "container %d: stencil in place", i);
+        if (is_stencil(c[i].op) && c[i].x == c[i].y) NB_FAIL(NB_EINVAL, "container %d: stencil in place", i);
         if (c[i].op == NB_SK_DOT && (c[i].slot < 0 || c[i].slot >= NB_DOT_SLOTS))
             NB_FAIL(NB_EINVAL, "container %d: slot out of range", i);
-        if (c[i].op == NB_SK_LAPLACE7) {
+        if (c[i].op == NB_SK_AXPBY && (c[i].a_slot >= NB_DOT_SLOTS || c[i].b_slot >= NB_DOT_SLOTS))
+            NB_FAIL(NB_EINVAL, "container %d: coefficient slot out of range", i);
+        if (is_stencil(c[i].op)) {
             if (multi && !is_coh(c[i].x)) {
                 incoh[i] = 1;
                 halo_before[i] = c[i].x;
@@ -188,15 +200,17 @@ nb_status build_nodes(const nb_container *c, int n, int nparts, nb_occ occ, Plan
             if (occ == NB_OCC_EXTENDED || occ == NB_OCC_TWO_WAY) {
                 // maps preceding the stencil that produce its input (back to the
                 // previous stencil)
-                for (int j = i - 1; j >= 0 && c[j].op != NB_SK_LAPLACE7; --j)
+                for (int j = i - 1; j >= 0 && !is_stencil(c[j].op); --j)
                     if (c[j].op == NB_SK_AXPBY && c[j].y == c[i].x) split[j] = 1;
             }
             if (occ == NB_OCC_TWO_WAY) {
                 // maps / reduces following the stencil that consume its output
-                for (int j = i + 1; j < n && c[j].op != NB_SK_LAPLACE7; ++j) {
+                for (int j = i + 1; j < n && !is_stencil(c[j].op); ++j) {
+                    if (c[j].op == NB_SK_SCALAR) continue;  // slots, not fields
+                    const bool b_reads = c[j].b != 0.0 || c[j].b_slot >= 0;
                     const bool uses = c[j].x == c[i].y || (c[j].op == NB_SK_DOT && c[j].y == c[i].y) ||
-                                      (c[j].op == NB_SK_AXPBY && c[j].b != 0.0 && c[j].y == c[i].y);
-                    if (uses && c[j].op != NB_SK_LAPLACE7) split[j] = 1;
+                                      (c[j].op == NB_SK_AXPBY && b_reads && c[j].y == c[i].y);
+                    if (uses) split[j] = 1;
                 }
             }
         }
@@ -212,11 +226,17 @@ nb_status build_nodes(const nb_container *c, int n, int nparts, nb_occ occ, Plan
         const int m = view_mask(v);
         if (k.op == NB_SK_AXPBY) {
             a.push_back({k.x, m, false});
-            if (k.b != 0.0) a.push_back({k.y, m, false});
+            if (k.b != 0.0 || k.b_slot >= 0) a.push_back({k.y, m, false});
+            if (k.a_slot >= 0) a.push_back({SCALAR_BASE + k.a_slot, R_ALL, false});
+            if (k.b_slot >= 0) a.push_back({SCALAR_BASE + k.b_slot, R_ALL, false});
             a.push_back({k.y, m, true});
-        } else if (k.op == NB_SK_LAPLACE7) {
+        } else if (is_stencil(k.op)) {
             a.push_back({k.x, stencil_read_mask(v), false});
             a.push_back({k.y, m, true});
+        } else if (k.op == NB_SK_SCALAR) {
+            if (k.sop != NB_SC_SET) a.push_back({SCALAR_BASE + k.x, R_ALL, false});
+            if (k.sop == NB_SC_DIV) a.push_back({SCALAR_BASE + k.y, R_ALL, false});
+            a.push_back({SCALAR_BASE + k.slot, R_ALL, true});
         } else {
             a.push_back({k.x, m, false});
             a.push_back({k.y, m, false});
@@ -225,11 +245,14 @@ nb_status build_nodes(const nb_container *c, int n, int nparts, nb_occ occ, Plan
         }
         return a;
     };
-    static const char *kname[] = {"axpby", "laplace7", "dot"};
+    static const char *kname[] = {"axpby", "laplace7", "dot", "poisson", "scalar", "lbm"};
     for (int i = 0; i < n; ++i) {
         auto mk = [&](nb_view v, bool fin) {
             Node nd;
-            nd.op = c[i].op == NB_SK_AXPBY ? SK_MAP : (c[i].op == NB_SK_LAPLACE7 ? SK_STENCIL : SK_REDUCE);
+            nd.op = c[i].op == NB_SK_AXPBY    ? SK_MAP
+                    : is_stencil(c[i].op)      ? SK_STENCIL
+                    : c[i].op == NB_SK_SCALAR ? SK_SCALAR
+                                              : SK_REDUCE;
             nd.view = v;
             nd.container = i;
             nd.incoherent = incoh[i] != 0;
@@ -248,6 +271,7 @@ nb_status build_nodes(const nb_container *c, int n, int nparts, nb_occ occ, Plan
                 h.op = SK_HALO;
                 h.halo_field = halo_before[i];
                 h.acc = {{halo_before[i], R_BLO | R_BHI, false}, {halo_before[i], R_HLO | R_HHI, true}};
+                h.halo_lbm = c[i].op == NB_SK_LBM;
                 h.name = "halo(f" + std::to_string(halo_before[i]) + ")";
                 add(h);
             }
@@ -265,6 +289,7 @@ nb_status build_nodes(const nb_container *c, int n, int nparts, nb_occ occ, Plan
                 h.op = SK_HALO;
                 h.halo_field = halo_before[i];
                 h.acc = {{halo_before[i], R_BLO | R_BHI, false}, {halo_before[i], R_HLO | R_HHI, true}};
+                h.halo_lbm = c[i].op == NB_SK_LBM;
                 h.name = "halo(f" + std::to_string(halo_before[i]) + ")";
                 add(h);
             }
@@ -275,8 +300,15 @@ nb_status build_nodes(const nb_container *c, int n, int nparts, nb_occ occ, Plan
     return NB_OK;
 }
 
-nb_status plan_graph(const nb_container *c, int n, int nparts, nb_occ occ, Plan &P) {
-    if (n < 0 || (n > 0 && !c)) NB_FAIL(NB_EINVAL, "no containers");
+nb_status plan_graph(const nb_container *cin, int n, int nparts, nb_occ occ, Plan &P) {
+    if (n < 0 || (n > 0 && !cin)) NB_FAIL(NB_EINVAL, "no containers");
+    // normalised copy: a_slot / b_slot = -1 unless flagged
+    std::vector<nb_container> cv(cin, cin + n);
+    for (auto &k : cv) {
+        if (!(k.flags & NB_SK_A_SLOT)) k.a_slot = -1;
+        if (!(k.flags & NB_SK_B_SLOT)) k.b_slot = -1;
+    }
+    const nb_container *c = cv.data();
     if (nparts < 1) NB_FAIL(NB_EINVAL, "nparts < 1");
     if (occ < NB_OCC_NONE || occ > NB_OCC_TWO_WAY) NB_FAIL(NB_EINVAL, "bad OCC mode");
     NB_TRY(build_nodes(c, n, nparts, occ, P));
@@ -459,12 +491,22 @@ extern "C" nb_status nb_skeleton_create(nb_grid *g, nb_occ occ, nb_skeleton **ou
     return NB_OK;
 }
 
-static nb_status sk_add(nb_skeleton *s, int op, nb_field *x, nb_field *y, double a, double b, int slot) {
-    if (!s || !x || !y) NB_FAIL(NB_EINVAL, "NULL argument");
+static nb_status sk_push(nb_skeleton *s, const nb_container &c) {
+    if (!s) NB_FAIL(NB_EINVAL, "NULL skeleton");
     if (s->compiled) NB_FAIL(NB_ESTATE, "skeleton already compiled");
+    s->cont.push_back(c);
+    return NB_OK;
+}
+
+static nb_status sk_add(nb_skeleton *s, int op, nb_field *x, nb_field *y, double a, double b, int slot,
+                        int a_slot = -1, int b_slot = -1) {
+    if (!s || !x || !y) NB_FAIL(NB_EINVAL, "NULL argument");
     if (x->g != s->g || y->g != s->g) NB_FAIL(NB_EMISMATCH, "field of another grid");
     if (x->dt != y->dt || x->card != y->card) NB_FAIL(NB_EMISMATCH, "dtype / cardinality mismatch");
-    if (op == NB_SK_LAPLACE7 && (x->card != 1 || x == y)) NB_FAIL(NB_EINVAL, "laplace7: two distinct scalar fields");
+    if ((op == NB_SK_LAPLACE7 || op == NB_SK_POISSON) && (x->card != 1 || x == y))
+        NB_FAIL(NB_EINVAL, "7-point stencil: two distinct scalar fields");
+    if ((a_slot >= 0 || b_slot >= 0) && x->dt != NB_F64) NB_FAIL(NB_EUNSUPPORTED, "device-scalar maps: fp64 fields");
+    if (a_slot >= NB_DOT_SLOTS || b_slot >= NB_DOT_SLOTS) NB_FAIL(NB_EINVAL, "coefficient slot out of range");
     nb_container c;
     memset(&c, 0, sizeof c);
     c.op = op;
@@ -473,19 +515,124 @@ static nb_status sk_add(nb_skeleton *s, int op, nb_field *x, nb_field *y, double
     c.a = a;
     c.b = b;
     c.slot = slot;
-    s->cont.push_back(c);
-    return NB_OK;
+    c.a_slot = a_slot < 0 ? -1 : a_slot;
+    c.b_slot = b_slot < 0 ? -1 : b_slot;
+    c.flags = (a_slot >= 0 ? NB_SK_A_SLOT : 0) | (b_slot >= 0 ? NB_SK_B_SLOT : 0);
+    return sk_push(s, c);
 }
 
 extern "C" nb_status nb_skeleton_axpby(nb_skeleton *s, double a, nb_field *x, double b, nb_field *y) {
     return sk_add(s, NB_SK_AXPBY, x, y, a, b, 0);
 }
+extern "C" nb_status nb_skeleton_axpby_s(nb_skeleton *s, double a, int32_t a_slot, nb_field *x, double b,
+                                         int32_t b_slot, nb_field *y) {
+    return sk_add(s, NB_SK_AXPBY, x, y, a, b, 0, a_slot, b_slot);
+}
 extern "C" nb_status nb_skeleton_laplace7(nb_skeleton *s, nb_field *x, nb_field *y) {
     return sk_add(s, NB_SK_LAPLACE7, x, y, 0.0, 0.0, 0);
+}
+extern "C" nb_status nb_skeleton_poisson(nb_skeleton *s, nb_field *x, nb_field *y) {
+    return sk_add(s, NB_SK_POISSON, x, y, 0.0, 0.0, 0);
 }
 extern "C" nb_status nb_skeleton_dot(nb_skeleton *s, nb_field *x, nb_field *y, int32_t slot) {
     if (slot < 0 || slot >= NB_DOT_SLOTS) NB_FAIL(NB_EINVAL, "slot out of range [0, %d)", NB_DOT_SLOTS);
     return sk_add(s, NB_SK_DOT, x, y, 0.0, 0.0, slot);
+}
+extern "C" nb_status nb_skeleton_scalar(nb_skeleton *s, nb_scalar_op sop, int32_t in0, int32_t in1, int32_t out,
+                                        double a) {
+    if (sop < NB_SC_DIV || sop > NB_SC_SET) NB_FAIL(NB_EINVAL, "bad scalar op");
+    for (int32_t v : {in0, in1, out})
+        if (v < 0 || v >= NB_DOT_SLOTS) NB_FAIL(NB_EINVAL, "scalar slot out of range [0, %d)", NB_DOT_SLOTS);
+    nb_container c;
+    memset(&c, 0, sizeof c);
+    c.op = NB_SK_SCALAR;
+    c.sop = sop;
+    c.x = in0;
+    c.y = in1;
+    c.slot = out;
+    c.a = a;
+    c.a_slot = c.b_slot = -1;
+    return sk_push(s, c);
+}
+extern "C" nb_status nb_skeleton_lbm(nb_skeleton *s, nb_field *fin, nb_field *fout, const nb_lbm_params *prm) {
+    if (!prm) NB_FAIL(NB_EINVAL, "NULL LBM parameters");
+    if (!fin || !fout || fin->dt != NB_F32 || fin->card != Q19) NB_FAIL(NB_EMISMATCH, "LBM: fp32 fields of 19 components");
+    if (prm->bc != NB_LBM_CAVITY) NB_FAIL(NB_EUNSUPPORTED, "Skeleton LBM containers: cavity boundaries");
+    if (fin == fout) NB_FAIL(NB_EINVAL, "twoPop needs two distinct buffers");
+    NB_TRY(sk_add(s, NB_SK_LBM, fin, fout, prm->omega, prm->u_lid, 0));
+    s->cont.back().c = prm->rho_w;
+    s->cont.back().sop = prm->bc;
+    return NB_OK;
+}
+
+__global__ void k_sk_scalar(double *s, int sop, int x, int y, int out, double a) {
+    if (threadIdx.x != 0) return;
+    if (sop == NB_SC_DIV)
+        s[out] = s[x] / s[y];
+    else if (sop == NB_SC_COPY)
+        s[out] = s[x];
+    else
+        s[out] = a;
+}
+
+extern "C" nb_status nb_skeleton_set_scalar(nb_skeleton *s, int32_t slot, double value) {
+    if (!s) NB_FAIL(NB_EINVAL, "NULL skeleton");
+    if (slot < 0 || slot >= NB_DOT_SLOTS) NB_FAIL(NB_EINVAL, "slot out of range");
+    DeviceGuard dg(s->g->device);
+    LaunchScope ls(s->g, s->g->cs, "k_sk_scalar");
+    k_sk_scalar<<<1, 32, 0, s->g->cs>>>(s->g->dots, NB_SC_SET, 0, 0, slot, value);
+    return nb_launch_check("k_sk_scalar");
+}
+
+// y = A x + B y with device-scalar coefficients (include/nb.h AXPBY rules)
+enum { SKA_B1 = 0, SKA_A1 = 1, SKA_B0 = 2, SKA_GEN = 3 };
+template <int MODE>
+__global__ void __launch_bounds__(256) k_sk_axpby(const double *__restrict__ x, double *__restrict__ y, int64_t n,
+                                                  double a, const double *as, double b, const double *bs) {
+    const double A = as ? a * *as : a, B = bs ? b * *bs : b;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double xv = x[i];
+        if (MODE == SKA_B1)
+            y[i] = fma(A, xv, y[i]);
+        else if (MODE == SKA_A1)
+            y[i] = fma(B, y[i], xv);
+        else if (MODE == SKA_B0)
+            y[i] = A * xv;
+        else
+            y[i] = fma(A, xv, B * y[i]);
+    }
+}
+
+static nb_status sk_axpby_dev(nb_grid *g, const nb_container &c, const nb_field *x, nb_field *y, nb_view v,
+                              cudaStream_t st) {
+    const double *as = c.a_slot >= 0 ? g->dots + c.a_slot : nullptr;
+    const double *bs = c.b_slot >= 0 ? g->dots + c.b_slot : nullptr;
+    const int mode = (c.b_slot < 0 && c.b == 1.0)   ? SKA_B1
+                     : (c.a_slot < 0 && c.a == 1.0) ? SKA_A1
+                     : (c.b_slot < 0 && c.b == 0.0) ? SKA_B0
+                                                    : SKA_GEN;
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const int64_t cs = x->ps * (g->parts[p].nz() + 2);
+        for (auto rg : view_ranges(g, p, v))
+            for (int k = 0; k < x->card; ++k) {
+                const int64_t off = (int64_t)k * cs + (int64_t)(rg.first + 1) * x->ps;
+                const int64_t n = (int64_t)(rg.second - rg.first) * x->ps;
+                const double *xp = (const double *)x->base[p] + off;
+                double *yp = (double *)y->base[p] + off;
+                const int blocks = (int)std::min<int64_t>((n + 255) / 256, 148 * 8);
+                LaunchScope ls(g, st, "k_sk_axpby");
+                if (mode == SKA_B1)
+                    k_sk_axpby<SKA_B1><<<blocks, 256, 0, st>>>(xp, yp, n, c.a, as, c.b, bs);
+                else if (mode == SKA_A1)
+                    k_sk_axpby<SKA_A1><<<blocks, 256, 0, st>>>(xp, yp, n, c.a, as, c.b, bs);
+                else if (mode == SKA_B0)
+                    k_sk_axpby<SKA_B0><<<blocks, 256, 0, st>>>(xp, yp, n, c.a, as, c.b, bs);
+                else
+                    k_sk_axpby<SKA_GEN><<<blocks, 256, 0, st>>>(xp, yp, n, c.a, as, c.b, bs);
+                NB_TRY(nb_launch_check("k_sk_axpby"));
+            }
+    }
+    return NB_OK;
 }
 
 extern "C" nb_status nb_skeleton_compile(nb_skeleton *s) {
@@ -512,14 +659,29 @@ static nb_status run_node(nb_skeleton *s, const Node &n, cudaStream_t st) {
     nb_status r = NB_OK;
     if (n.op == SK_HALO) {
         nb_field *f = s->fields[n.halo_field];
-        r = nb_halo_exchange_planes(f, 0, f->card, true, true, st);
+        r = n.halo_lbm ? nb_halo_run(f, false, 9, 14, 14, 19, st)  // the z-crossing populations
+                       : nb_halo_exchange_planes(f, 0, f->card, true, true, st);
     } else {
         const nb_container &c = s->cont[n.container];
+        if (c.op == NB_SK_SCALAR) {
+            LaunchScope ls(g, st, "k_sk_scalar");
+            k_sk_scalar<<<1, 32, 0, st>>>(g->dots, c.sop, c.x, c.y, c.slot, c.a);
+            r = nb_launch_check("k_sk_scalar");
+            g->cs = saved;
+            return r;
+        }
         nb_field *x = s->fields[c.x], *y = s->fields[c.y];
         if (c.op == NB_SK_AXPBY) {
-            r = nb_axpby(c.a, x, c.b, y, n.view);
-        } else if (c.op == NB_SK_LAPLACE7) {
-            r = nb_laplace7(x, y, n.view);
+            r = (c.a_slot >= 0 || c.b_slot >= 0) ? sk_axpby_dev(g, c, x, y, n.view, st) : nb_axpby(c.a, x, c.b, y, n.view);
+        } else if (c.op == NB_SK_LAPLACE7 || c.op == NB_SK_POISSON) {
+            r = nb_stencil7(x, y, n.view, c.op == NB_SK_POISSON);
+        } else if (c.op == NB_SK_LBM) {
+            nb_lbm_params prm;
+            prm.omega = c.a;
+            prm.u_lid = c.b;
+            prm.rho_w = c.c;
+            prm.bc = (nb_lbm_bc)c.sop;
+            r = nb_lbm_view(x, y, &prm, n.view);
         } else {
             r = nb_dot_partials_view(x, y, n.view);
             if (r == NB_OK && n.finalize) r = nb_reduce_finalize(g, x->card, FIN_STORE, nullptr, c.slot);

@@ -46,7 +46,8 @@ static inline int64_t dcs(const nb_field *f, int p) { return f->ps * (f->g->part
 // 7-point Laplacian y = L(x) (Listing 2).  Algorithmic traffic: read x +
 // write y = 2*sizeof(T) per cell.
 // ===========================================================================
-template <typename TT>
+// NEG: y = -L(x) = fma(6, x_c, -s), the CG operator A (bitwise the CG's A p)
+template <typename TT, bool NEG = false>
 struct Lap7Op {
     using T = TT;
     struct Raw {
@@ -63,7 +64,7 @@ struct Lap7Op {
     __device__ TT val(int, const Raw &r) const { return r.a; }
     __device__ TT nval(int, int64_t i) const { return x[i]; }
     __device__ double cell(int, int64_t i, TT c, TT s, const Raw &) {
-        __stcs(y + i, fma(TT(-6), c, s));
+        __stcs(y + i, NEG ? fma(TT(6), c, -s) : fma(TT(-6), c, s));
         return 0.0;
     }
 };
@@ -81,25 +82,40 @@ static nb_status launch_zmarch(nb_grid *g, const char *name, Op op, PGeo geo, in
 }
 
 extern "C" nb_status nb_laplace7(const nb_field *x, nb_field *y, nb_view v) {
+    return nb_stencil7(x, y, v, false);
+}
+
+// y = L(x) (neg = false) or y = A x = -L(x) (neg = true) on the view
+nb_status nb_stencil7(const nb_field *x, nb_field *y, nb_view v, bool neg) {
     if (!x || !y) NB_FAIL(NB_EINVAL, "nb_laplace7: NULL field");
     if (x->g != y->g) NB_FAIL(NB_EMISMATCH, "fields belong to different grids");
     if (x->dt != y->dt || x->card != 1 || y->card != 1)
         NB_FAIL(NB_EMISMATCH, "nb_laplace7 needs two scalar fields of one dtype");
     nb_grid *g = x->g;
-    if (g->sparse) return nb_sparse_laplace7(x, y, v);
+    if (g->sparse) {
+        if (neg) NB_FAIL(NB_EUNSUPPORTED, "-L on element-sparse grids");
+        return nb_sparse_laplace7(x, y, v);
+    }
     cudaSetDevice(g->device);
     for (int p = 0; p < g->nparts; ++p) {
         if (!g->parts[p].local) continue;
         PGeo geo = pgeo(x, p);
         for (auto rg : view_ranges(g, p, v)) {
-            if (x->dt == NB_F64)
-                NB_TRY(launch_zmarch(g, "k_laplace7",
-                                     Lap7Op<double>{(const double *)x->base[p], (double *)y->base[p], x->outside},
-                                     geo, rg.first, rg.second));
+            const double *xd = (const double *)x->base[p];
+            double *yd = (double *)y->base[p];
+            const float *xf = (const float *)x->base[p];
+            float *yf = (float *)y->base[p];
+            if (x->dt == NB_F64 && !neg)
+                NB_TRY(launch_zmarch(g, "k_laplace7", Lap7Op<double>{xd, yd, x->outside}, geo, rg.first, rg.second));
+            else if (x->dt == NB_F64)
+                NB_TRY(launch_zmarch(g, "k_laplace7", Lap7Op<double, true>{xd, yd, x->outside}, geo, rg.first,
+                                     rg.second));
+            else if (!neg)
+                NB_TRY(launch_zmarch(g, "k_laplace7", Lap7Op<float>{xf, yf, (float)x->outside}, geo, rg.first,
+                                     rg.second));
             else
-                NB_TRY(launch_zmarch(g, "k_laplace7",
-                                     Lap7Op<float>{(const float *)x->base[p], (float *)y->base[p], (float)x->outside},
-                                     geo, rg.first, rg.second));
+                NB_TRY(launch_zmarch(g, "k_laplace7", Lap7Op<float, true>{xf, yf, (float)x->outside}, geo, rg.first,
+                                     rg.second));
         }
     }
     return NB_OK;

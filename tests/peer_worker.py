@@ -214,6 +214,82 @@ def wrapped_cg(g):
 compare("wrapped cg", (20, 20, 20), WORLD, wrapped_cg)
 
 
+# ---- the Skeleton across processes (§V): Listing 3 CG with device
+# scalars, the Fig. 4a loop and the LBM step as generated schedules ----------
+RR, PQ, ALPHA, BETA, RR2 = 0, 1, 2, 3, 4
+
+
+def sk_cg(occ):
+    def fn(g):
+        b, x, r, p, q = (nb.Field(g) for _ in range(5))
+        b.fill_uniform(8)
+        for f in (x, p, q):
+            f.fill_const(0.0)
+        nb.nb_axpby(1.0, b, 0.0, r)
+        with nb.Skeleton(g, occ) as s0:
+            s0.dot(r, r, RR)
+            s0.set_scalar(BETA, 0.0)
+            s0.run()
+        with nb.Skeleton(g, occ) as sk:
+            sk.axpby_s(1.0, -1, r, 1.0, BETA, p)
+            sk.poisson(p, q)
+            sk.dot(p, q, PQ)
+            sk.scalar(nb.SC_DIV, RR, PQ, ALPHA)
+            sk.axpby_s(1.0, ALPHA, p, 1.0, -1, x)
+            sk.axpby_s(-1.0, ALPHA, q, 1.0, -1, r)
+            sk.dot(r, r, RR2)
+            sk.scalar(nb.SC_DIV, RR2, RR, BETA)
+            sk.scalar(nb.SC_COPY, RR2, 0, RR)
+            for _ in range(7):
+                sk.run()
+            rr = sk.result(RR)
+        out = [x.download()]
+        for f in (b, x, r, p, q):
+            f.close()
+        return out, [rr]
+    return fn
+
+
+def sk_c1(occ):
+    def fn(g):
+        x, y = nb.Field(g), nb.Field(g)
+        x.fill_uniform(2)
+        y.fill_const(0.0)
+        with nb.Skeleton(g, occ) as sk:
+            for k in range(4):
+                sk.axpy(0.125, y, x)
+                sk.laplace7(x, y)
+                sk.dot(x, y, k)
+            sk.run()
+            d = [sk.result(k) for k in range(4)]
+        out = [x.download(), y.download()]
+        x.close(), y.close()
+        return out, d
+    return fn
+
+
+def sk_lbm(occ):
+    def fn(g):
+        a, b = nb.Field(g, "f32", 19), nb.Field(g, "f32", 19)
+        nb.nb_lbm_init(a, 1.0, (0.0, 0.0, 0.0))
+        with nb.Skeleton(g, occ) as sk:
+            sk.lbm(a, b, 0.9)
+            sk.lbm(b, a, 0.9)
+            for _ in range(3):
+                sk.run()
+        out = [a.download()]
+        a.close(), b.close()
+        return out, []
+    return fn
+
+
+for occ in (nb.OCC_NONE, nb.OCC_TWO_WAY):
+    compare(f"skeleton listing3 cg occ{occ}", (28, 26, 24), WORLD, sk_cg(occ))
+    compare(f"skeleton c1 occ{occ}", (37, 21, 16), WORLD, sk_c1(occ))
+    compare(f"skeleton lbm occ{occ}", (24, 20, 18), WORLD, sk_lbm(occ))
+compare("skeleton listing3 cg 4 parts", (28, 26, 24), 2 * WORLD, sk_cg(nb.OCC_STANDARD))
+
+
 # ---- the peer path really ran: its kernels were launched ---------------------
 if TRANSPORT != "peer":
     COMM.close()

@@ -161,3 +161,62 @@ def test_invalid_plans_fail():
         plan(2, nb.OCC_NONE, [(nb.SK_DOT, X, Y, 0, 0, 5000)])
     with pytest.raises(nb.NbError):
         plan(0, nb.OCC_NONE)
+
+
+def test_listing3_cg_plan_structure():
+    """Listing 3 CG (L154-L163) with device scalars: the halo of p precedes
+    the stencil; alpha waits for <p, q> and feeds both updates; beta waits
+    for <r, r>; under Two-way OCC the UpdateP map and the stencil split and
+    the internal stencil is hinted before the halo (Fig. 4d pattern)."""
+    P_, Q_, R_, X_ = 0, 1, 2, 3
+    RR, PQ, AL, BE, RR2 = 0, 1, 2, 3, 4
+    C = [(nb.SK_AXPBY, R_, P_, 1.0, 1.0, 0, -1, BE, 0),
+         (nb.SK_POISSON, P_, Q_, 0.0, 0.0, 0),
+         (nb.SK_DOT, P_, Q_, 0.0, 0.0, PQ),
+         (nb.SK_SCALAR, RR, PQ, 0.0, 0.0, AL, -1, -1, nb.SC_DIV),
+         (nb.SK_AXPBY, P_, X_, 1.0, 1.0, 0, AL, -1, 0),
+         (nb.SK_AXPBY, Q_, R_, -1.0, 1.0, 0, AL, -1, 0),
+         (nb.SK_DOT, R_, R_, 0.0, 0.0, RR2),
+         (nb.SK_SCALAR, RR2, RR, 0.0, 0.0, BE, -1, -1, nb.SC_DIV),
+         (nb.SK_SCALAR, RR2, 0, 0.0, 0.0, RR, -1, -1, nb.SC_COPY)]
+    plan = nb.nb_skeleton_plan(4, nb.OCC_TWO_WAY, C)
+    nodes = plan["nodes"]
+    names = [n["name"] for n in nodes]
+    edges = set(map(tuple, plan["data"]))
+    idx = {nm: i for i, nm in enumerate(names)}
+
+    def path(a, b):
+        adj = {}
+        for u, v in edges:
+            adj.setdefault(u, []).append(v)
+        st, seen = [a], set()
+        while st:
+            u = st.pop()
+            if u == b:
+                return True
+            for v in adj.get(u, []):
+                if v not in seen:
+                    seen.add(v)
+                    st.append(v)
+        return False
+    assert "halo(f0)" in names
+    assert "axpby#0[bnd]" in names and "axpby#0[int]" in names       # UpdateP split (Extended)
+    assert "poisson#1[int]" in names and "poisson#1[bnd]" in names
+    assert path(idx["halo(f0)"], idx["poisson#1[bnd]"])
+    assert not path(idx["halo(f0)"], idx["poisson#1[int]"])           # internal stencil overlaps the halo
+    assert (idx["poisson#1[int]"], idx["halo(f0)"]) in set(map(tuple, plan["hints"]))
+    # alpha after <p, q>; both updates after alpha; beta after <r, r>; rr copy after beta (WaR on rr)
+    dot_pq = [i for i, nm in enumerate(names) if nm.startswith("dot#2") and nodes[i]["finalize"]][0]
+    assert path(dot_pq, idx["scalar#3"])
+    def parts_of(prefix):
+        return [i for i, nm in enumerate(names) if nm.split("[")[0] == prefix]
+    for u in parts_of("axpby#4") + parts_of("axpby#5"):  # r <- r - alpha q consumes q: split (Two-way)
+        assert path(idx["scalar#3"], u)
+    assert len(parts_of("axpby#5")) == 2
+    dot_rr = [i for i, nm in enumerate(names) if nm.startswith("dot#6") and nodes[i]["finalize"]][0]
+    assert path(dot_rr, idx["scalar#7"]) and path(idx["scalar#7"], idx["scalar#8"])
+    # the x and r updates touch disjoint data: concurrent
+    for u in parts_of("axpby#4"):
+        for v in parts_of("axpby#5"):
+            assert not path(u, v) and not path(v, u)
+    assert plan["streams"] >= 2
