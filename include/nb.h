@@ -198,15 +198,30 @@ nb_status nb_grid_set_halo_mode(nb_grid *grid, int32_t mode);
 nb_status nb_sync(nb_grid *grid);
 
 /* ---- fields (PAPER.md L58-L63 newField<T>(cardinality, outsideDomainValue),
- * L246 Field, L248 SoA layout, L252 halo regions) --------------------------
- * Device layout per partition (SoA):
- *   [c][zl = -1 .. nz_g][y][x], x-rows padded to a 32-element pitch, one halo
- *   plane below and above the slab.  Halo planes facing the global domain
- *   boundary hold outside_value (the value read for out-of-domain neighbours).
+ * L246 Field, L248 "SoA or AoS organizations without impacting the
+ * application code", L252 halo regions) -----------------------------------
+ * Device layouts per dense partition (x-rows padded to a 32-element pitch,
+ * one halo plane below and above the slab, zl = -1 .. nz_g):
+ *   NB_SOA        [c][zl][y][x]  a component's planes contiguous; a halo
+ *                 exchange is one transfer per component and direction
+ *                 (2 x C per partition, L256)
+ *   NB_SOA_PLANE  [zl][c][y][x]  the components of a plane contiguous: any
+ *                 component range of a plane is ONE transfer (L256 "2")
+ *   NB_AOS        [zl][y][x][c]  the components of a cell contiguous; a
+ *                 halo plane moves whole (all components, one transfer)
+ * Element (c, x, y, zl) sits at c*cstride + ((zl+1)*pstride + y*pitch + x)*estride
+ * (nb_field_partition_ptr; estride = C for AOS, else 1).  Cardinality 1:
+ * the three layouts coincide (reported as NB_SOA).  Halo planes facing the
+ * global domain boundary hold outside_value (the value read for out-of-domain
+ * neighbours).  Maps, dots, halo updates, upload / download / fill, the
+ * 7-point stencil and the D3Q19 twoPop step take every layout; the FEM
+ * operator takes SOA and SOA_PLANE; other operations (AA pattern, D2Q9,
+ * element-sparse grids) take SOA only and return NB_EUNSUPPORTED otherwise.
  * Sparse grids: [c][-halo_lo .. n_g + halo_hi) over the partition's active
  *   cells in (z, y, x) order. */
-nb_status nb_field_create(nb_grid *grid, nb_dtype dtype, int32_t cardinality, double outside_value,
-                          nb_field **out);
+typedef enum { NB_SOA = 0, NB_SOA_PLANE = 1, NB_AOS = 2 } nb_layout;
+nb_status nb_field_create(nb_grid *grid, nb_dtype dtype, int32_t cardinality, nb_layout layout,
+                          double outside_value, nb_field **out);
 nb_status nb_field_destroy(nb_field *field);
 /* Borrowed storage (SURVEY.md §8(b) "field (borrowed)": PyTorch owns the
  * memory).  Pure host logic: the number of elements partition g of a field
@@ -221,8 +236,10 @@ nb_status nb_field_required_elems(const nb_grid *grid, int32_t cardinality, int3
  * library never frees the buffers — the caller keeps them alive until
  * nb_field_destroy.  NB_EINVAL for NULL, misaligned or non-device pointers.
  * With the peer transport the call is collective, like nb_field_create. */
-nb_status nb_field_wrap(nb_grid *grid, nb_dtype dtype, int32_t cardinality, double outside_value,
-                        void *const *dev_ptrs, nb_field **out);
+nb_status nb_field_wrap(nb_grid *grid, nb_dtype dtype, int32_t cardinality, nb_layout layout,
+                        double outside_value, void *const *dev_ptrs, nb_field **out);
+/* the field's layout (cardinality 1: NB_SOA) */
+nb_status nb_field_layout(const nb_field *field, nb_layout *layout);
 /* host: dense logical view, nbytes = Nx*Ny*Nz*card*sizeof(dtype); inactive
  * cells of sparse grids are ignored on upload and read back as outside.
  * Upload is stream-ordered (host buffer must stay valid until nb_sync);
@@ -234,7 +251,8 @@ nb_status nb_field_fill(nb_field *field, nb_fill kind, uint64_t seed, double a, 
  * its neighbours' halo planes (2 transfers per component, L256). */
 nb_status nb_halo_update(nb_field *field);
 /* device pointer of partition g's buffer (element (c, x, y, zl) at
- * ptr + c*cstride + (zl+1)*pstride + y*pitch + x, in elements) */
+ * ptr + c*cstride + ((zl+1)*pstride + y*pitch + x)*estride, in elements;
+ * estride: see the layouts above) */
 nb_status nb_field_partition_ptr(const nb_field *field, int32_t g, void **ptr, int64_t *pitch,
                                  int64_t *pstride, int64_t *cstride);
 

@@ -34,6 +34,7 @@ FILL_CONST, FILL_UNIFORM, FILL_INT_UNIFORM, FILL_POISSON_RHS = 0, 1, 2, 3
 OP_LAPLACE7, OP_FEM27 = 0, 1
 LBM_CAVITY, LBM_PERIODIC = 0, 1
 HALO_FUSED, HALO_STREAM = 0, 1
+SOA, SOA_PLANE, AOS = 0, 1, 2  # field layouts (include/nb.h nb_layout)
 OCC_NAMES = {"none": OCC_NONE, "standard": OCC_STANDARD, "extended": OCC_EXTENDED, "two_way": OCC_TWO_WAY}
 
 
@@ -97,10 +98,11 @@ SIGNATURES = {
     "nb_grid_get_stream": ([P, PP], I32),
     "nb_sync": ([P], I32),
     "nb_grid_set_halo_mode": ([P, I32], I32),
-    "nb_field_create": ([P, I32, I32, D, PP], I32),
+    "nb_field_create": ([P, I32, I32, I32, D, PP], I32),
+    "nb_field_layout": ([P, P], I32),
     "nb_field_destroy": ([P], I32),
     "nb_field_required_elems": ([P, I32, I32, P], I32),
-    "nb_field_wrap": ([P, I32, I32, D, P, PP], I32),
+    "nb_field_wrap": ([P, I32, I32, I32, D, P, PP], I32),
     "nb_field_upload": ([P, P, I64], I32),
     "nb_field_download": ([P, P, I64], I32),
     "nb_field_fill": ([P, I32, U64, D, D], I32),
@@ -381,9 +383,11 @@ class Grid:
 
 class Field:
     """Field of `card` components (PAPER.md L58-L63 newField<T>(cardinality,
-    outsideDomainValue)); SoA layout with z halo planes."""
+    outsideDomainValue)) with z halo planes, in layout SOA (default),
+    SOA_PLANE or AOS (L248; include/nb.h)."""
 
-    def __init__(self, grid: Grid, dtype="f64", card: int = 1, outside: float = 0.0, _buffers=None):
+    def __init__(self, grid: Grid, dtype="f64", card: int = 1, outside: float = 0.0, _buffers=None,
+                 layout: int = 0):
         self.grid = grid
         self.dt = _dtype_code(dtype)
         self.np_dtype = _DT[self.dt]
@@ -392,10 +396,18 @@ class Field:
         self.handle = P()
         self.buffers = _buffers  # borrowed storage (kept alive with the field)
         if _buffers is None:
-            _check(lib().nb_field_create(grid.handle, self.dt, self.card, self.outside, C.byref(self.handle)))
+            _check(lib().nb_field_create(grid.handle, self.dt, self.card, int(layout), self.outside,
+                                         C.byref(self.handle)))
         else:
             ptrs = (C.c_void_p * len(_buffers))(*[b.data_ptr() for b in _buffers])
-            _check(lib().nb_field_wrap(grid.handle, self.dt, self.card, self.outside, ptrs, C.byref(self.handle)))
+            _check(lib().nb_field_wrap(grid.handle, self.dt, self.card, int(layout), self.outside, ptrs,
+                                       C.byref(self.handle)))
+
+    @property
+    def layout(self) -> int:
+        v = C.c_int32()
+        _check(lib().nb_field_layout(self.handle, C.byref(v)))
+        return v.value
 
     @staticmethod
     def required_elems(grid: Grid, card: int, part: int) -> int:
@@ -404,20 +416,20 @@ class Field:
         return n.value
 
     @classmethod
-    def wrap(cls, grid: Grid, buffers, dtype="f64", card: int = 1, outside: float = 0.0):
+    def wrap(cls, grid: Grid, buffers, dtype="f64", card: int = 1, outside: float = 0.0, layout: int = 0):
         """Field over caller-owned torch CUDA tensors, one per local partition
         (each >= required_elems elements; torch keeps ownership)."""
-        return cls(grid, dtype, card, outside, _buffers=list(buffers))
+        return cls(grid, dtype, card, outside, _buffers=list(buffers), layout=layout)
 
     @classmethod
-    def empty_torch(cls, grid: Grid, dtype="f64", card: int = 1, outside: float = 0.0):
+    def empty_torch(cls, grid: Grid, dtype="f64", card: int = 1, outside: float = 0.0, layout: int = 0):
         """Allocate the partitions with torch.empty on the grid's device and wrap them."""
         import torch
         tdt = torch.float64 if _dtype_code(dtype) == 1 else torch.float32
         dev = torch.device("cuda", grid.device)
         bufs = [torch.empty(cls.required_elems(grid, card, p), dtype=tdt, device=dev)
                 for p in range(grid.nparts) if grid.partition_info(p)["local"]]
-        return cls.wrap(grid, bufs, dtype, card, outside)
+        return cls.wrap(grid, bufs, dtype, card, outside, layout)
 
     @property
     def shape(self):

@@ -335,10 +335,20 @@ nb_status nb_halo_run_mode(nb_field *f, bool periodic, int c0u, int c1u, int c0d
     NB_TRY(nb_halo_plan(g->nz, g->nparts, world, rank, periodic, nullptr, 0, &cnt));
     std::vector<nb_halo_msg> msgs(cnt);
     NB_TRY(nb_halo_plan(g->nz, g->nparts, world, rank, periodic, msgs.data(), cnt, &cnt));
-    size_t pb = (size_t)f->ps * f->esz;
-    auto cs_of = [&](int p) { return f->ps * (g->parts[p].nz() + 2); };
-    auto plane_addr = [&](int p, int c, int zl) {
-        return f->base[p] + ((int64_t)c * cs_of(p) + (int64_t)(zl + 1) * f->ps) * f->esz;
+    // the contiguous pieces of components [c0, c1) of plane zl (include/nb.h
+    // layouts): SOA one per component; SOA_PLANE one for the range; AOS the
+    // whole interleaved plane (all components, one transfer)
+    auto pieces = [&](int p, int zl, int c0, int c1) {
+        std::vector<std::pair<int64_t, int64_t>> v;  // (element offset, elements)
+        if (c1 <= c0) return v;
+        const int64_t z = (int64_t)(zl + 1) * f->ps * f->es;
+        if (f->layout == NB_SOA)
+            for (int c = c0; c < c1; ++c) v.push_back({(int64_t)c * nb_cstride(f, p) + z, f->plane});
+        else if (f->layout == NB_SOA_PLANE)
+            v.push_back({(int64_t)c0 * f->plane + z, (int64_t)(c1 - c0) * f->plane});
+        else
+            v.push_back({z, f->plane * f->card});
+        return v;
     };
     if (nb_is_peer(g)) {
         // peer memory: a "ready" round (the neighbours finished reading the
@@ -350,12 +360,14 @@ nb_status nb_halo_run_mode(nb_field *f, bool periodic, int c0u, int c1u, int c0d
         for (auto &m : msgs) {
             if (m.src_rank != rank) continue;  // the sender writes
             int c0 = m.up ? c0u : c0d, c1 = m.up ? c1u : c1d;
-            for (int c = c0; c < c1; ++c) {
+            auto sp = pieces(m.src_part, m.src_plane, c0, c1), dp = pieces(m.dst_part, m.dst_plane, c0, c1);
+            for (size_t k = 0; k < sp.size(); ++k) {
                 if (cb.n == CopyBatch::MAX) {
                     NB_TRY(nb_launch_copy_batch(g, cb, s));
                     cb = CopyBatch();
                 }
-                cb.add(plane_addr(m.dst_part, c, m.dst_plane), plane_addr(m.src_part, c, m.src_plane), pb);
+                cb.add(f->base[m.dst_part] + dp[k].first * f->esz, f->base[m.src_part] + sp[k].first * f->esz,
+                       (size_t)sp[k].second * f->esz);
             }
         }
         if (cb.n) NB_TRY(nb_launch_copy_batch(g, cb, s));
@@ -370,12 +382,14 @@ nb_status nb_halo_run_mode(nb_field *f, bool periodic, int c0u, int c1u, int c0d
     for (auto &m : msgs) {
         int c0 = m.up ? c0u : c0d, c1 = m.up ? c1u : c1d;
         if (m.src_rank == rank && m.dst_rank == rank) {
-            for (int c = c0; c < c1; ++c) {
+            auto sp = pieces(m.src_part, m.src_plane, c0, c1), dp = pieces(m.dst_part, m.dst_plane, c0, c1);
+            for (size_t k = 0; k < sp.size(); ++k) {
                 if (cb.n == CopyBatch::MAX) {
                     NB_TRY(nb_launch_copy_batch(g, cb, s));
                     cb = CopyBatch();
                 }
-                cb.add(plane_addr(m.dst_part, c, m.dst_plane), plane_addr(m.src_part, c, m.src_plane), pb);
+                cb.add(f->base[m.dst_part] + dp[k].first * f->esz, f->base[m.src_part] + sp[k].first * f->esz,
+                       (size_t)sp[k].second * f->esz);
             }
         } else {
             remote = true;
@@ -387,11 +401,14 @@ nb_status nb_halo_run_mode(nb_field *f, bool periodic, int c0u, int c1u, int c0d
     for (auto &m : msgs) {
         if (m.src_rank == rank && m.dst_rank == rank) continue;
         int c0 = m.up ? c0u : c0d, c1 = m.up ? c1u : c1d;
-        for (int c = c0; c < c1; ++c) {
-            if (m.src_rank == rank)
-                NB_TRY(nb_nccl_send(g, plane_addr(m.src_part, c, m.src_plane), pb, m.dst_rank, s));
-            else
-                NB_TRY(nb_nccl_recv(g, plane_addr(m.dst_part, c, m.dst_plane), pb, m.src_rank, s));
+        if (m.src_rank == rank) {
+            for (auto &pc : pieces(m.src_part, m.src_plane, c0, c1))
+                NB_TRY(nb_nccl_send(g, f->base[m.src_part] + pc.first * f->esz, (size_t)pc.second * f->esz,
+                                    m.dst_rank, s));
+        } else {
+            for (auto &pc : pieces(m.dst_part, m.dst_plane, c0, c1))
+                NB_TRY(nb_nccl_recv(g, f->base[m.dst_part] + pc.first * f->esz, (size_t)pc.second * f->esz,
+                                    m.src_rank, s));
         }
     }
     NB_TRY(nb_nccl_group(g, false));
@@ -511,7 +528,7 @@ nb_status nb_grid_scratch(nb_grid *g, nb_dtype dt, int card, int slot, nb_field 
         return NB_OK;
     }
     nb_field *f = nullptr;
-    NB_TRY(nb_field_create(g, dt, card, 0.0, &f));
+    NB_TRY(nb_field_create(g, dt, card, NB_SOA, 0.0, &f));
     g->nfields--;  // owned by the grid
     g->scratch[key] = f;
     *out = f;
@@ -642,12 +659,37 @@ static nb_status fill_const_raw(nb_grid *g, void *p, int64_t n, nb_dtype dt, dou
     return nb_launch_check("k_fill_const");
 }
 
-extern "C" nb_status nb_field_create(nb_grid *g, nb_dtype dt, int32_t card, double outside,
+static int64_t dense_pitch(const nb_grid *g) { return ((int64_t)g->nx + 31) / 32 * 32; }
+
+// layout geometry of a dense field (include/nb.h layouts; nb_field)
+static nb_status set_layout(nb_field *f, nb_layout layout) {
+    if (layout < NB_SOA || layout > NB_AOS) NB_FAIL(NB_EINVAL, "bad layout %d", (int)layout);
+    if (f->g->sparse && layout != NB_SOA && f->card > 1)
+        NB_FAIL(NB_EUNSUPPORTED, "element-sparse grids store fields as SoA");
+    f->layout = f->card == 1 ? NB_SOA : layout;  // one component: the layouts coincide
+    if (f->g->sparse) return NB_OK;
+    f->pitch = dense_pitch(f->g);
+    f->plane = f->pitch * f->g->ny;
+    f->es = f->layout == NB_AOS ? f->card : 1;
+    f->ps = f->layout == NB_SOA_PLANE ? f->card * f->plane : f->plane;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_field_layout(const nb_field *f, nb_layout *layout) {
+    if (!f || !layout) NB_FAIL(NB_EINVAL, "nb_field_layout: NULL argument");
+    *layout = f->layout;
+    return NB_OK;
+}
+
+extern "C" nb_status nb_field_create(nb_grid *g, nb_dtype dt, int32_t card, nb_layout layout, double outside,
                                      nb_field **out) {
     if (!g || !out) NB_FAIL(NB_EINVAL, "nb_field_create: NULL argument");
     *out = nullptr;
     if (dt != NB_F32 && dt != NB_F64) NB_FAIL(NB_EINVAL, "nb_field_create: bad dtype %d", (int)dt);
     if (card < 1 || card > 64) NB_FAIL(NB_EINVAL, "nb_field_create: cardinality %d", card);
+    if (layout < NB_SOA || layout > NB_AOS) NB_FAIL(NB_EINVAL, "nb_field_create: bad layout %d", (int)layout);
+    if (g->sparse && layout != NB_SOA && card > 1)
+        NB_FAIL(NB_EUNSUPPORTED, "nb_field_create: element-sparse grids store fields as SoA");
     DeviceGuard dg(g->device);
     nb_field *f = new nb_field();
     f->g = g;
@@ -657,16 +699,18 @@ extern "C" nb_status nb_field_create(nb_grid *g, nb_dtype dt, int32_t card, doub
     f->esz = dt == NB_F64 ? 8 : 4;
     f->base.assign(g->nparts, nullptr);
     f->bytes.assign(g->nparts, 0);
-    nb_status s = NB_OK;
+    nb_status s = set_layout(f, layout);
+    if (s != NB_OK) {
+        delete f;
+        return s;
+    }
     if (g->sparse) {
         s = nb_sparse_field_alloc(f);
     } else {
-        f->pitch = ((int64_t)g->nx + 31) / 32 * 32;
-        f->ps = f->pitch * g->ny;
         for (int p = 0; p < g->nparts && s == NB_OK; ++p) {
             if (!g->parts[p].local) continue;
-            f->cs = f->ps * (g->parts[p].nz() + 2);
-            size_t bytes = (size_t)f->cs * card * f->esz;
+            f->cs = nb_cstride(f, p);
+            size_t bytes = (size_t)f->plane * (g->parts[p].nz() + 2) * card * f->esz;
             cudaError_t e = cudaMalloc(&f->base[p], bytes);
             if (e != cudaSuccess) {
                 cudaGetLastError();
@@ -702,7 +746,6 @@ extern "C" nb_status nb_field_create(nb_grid *g, nb_dtype dt, int32_t card, doub
 }
 
 // ---- borrowed storage (SURVEY.md §8(b) "field (borrowed)") ---------------
-static int64_t dense_pitch(const nb_grid *g) { return ((int64_t)g->nx + 31) / 32 * 32; }
 
 static nb_status required_elems(const nb_grid *g, int card, int p, int64_t *n) {
     if (p < 0 || p >= g->nparts) NB_FAIL(NB_EINVAL, "partition %d out of range", p);
@@ -718,10 +761,11 @@ extern "C" nb_status nb_field_required_elems(const nb_grid *g, int32_t card, int
     return required_elems(g, card, p, n);
 }
 
-extern "C" nb_status nb_field_wrap(nb_grid *g, nb_dtype dt, int32_t card, double outside, void *const *dev_ptrs,
-                                   nb_field **out) {
+extern "C" nb_status nb_field_wrap(nb_grid *g, nb_dtype dt, int32_t card, nb_layout layout, double outside,
+                                   void *const *dev_ptrs, nb_field **out) {
     if (!g || !out || !dev_ptrs) NB_FAIL(NB_EINVAL, "nb_field_wrap: NULL argument");
     *out = nullptr;
+    if (layout < NB_SOA || layout > NB_AOS) NB_FAIL(NB_EINVAL, "nb_field_wrap: bad layout %d", (int)layout);
     if (dt != NB_F32 && dt != NB_F64) NB_FAIL(NB_EINVAL, "nb_field_wrap: bad dtype %d", (int)dt);
     if (card < 1 || card > 64) NB_FAIL(NB_EINVAL, "nb_field_wrap: cardinality %d", card);
     for (int i = 0; i < g->nlocal; ++i) {
@@ -746,11 +790,7 @@ extern "C" nb_status nb_field_wrap(nb_grid *g, nb_dtype dt, int32_t card, double
     f->bytes.assign(g->nparts, 0);
     f->pcs.assign(g->nparts, 0);
     f->mapped.assign(g->nparts, 0);
-    if (!g->sparse) {
-        f->pitch = dense_pitch(g);
-        f->ps = f->pitch * g->ny;
-    }
-    nb_status s = NB_OK;
+    nb_status s = set_layout(f, layout);
     for (int i = 0; i < g->nlocal && s == NB_OK; ++i) {
         const int p = g->first_local + i;
         int64_t n = 0;
@@ -768,8 +808,8 @@ extern "C" nb_status nb_field_wrap(nb_grid *g, nb_dtype dt, int32_t card, double
                 if (s == NB_OK) s = fill_const_raw(g, b + (size_t)(sp.hl + sp.n) * f->esz, sp.cs - sp.hl - sp.n, dt,
                                                    outside, g->cs);
             }
-        } else {
-            const int64_t cs = f->ps * (g->parts[p].nz() + 2);
+        } else if (f->layout == NB_SOA) {
+            const int64_t cs = nb_cstride(f, p);
             f->pcs[p] = cs;
             for (int c = 0; c < card && s == NB_OK; ++c) {
                 char *b = f->base[p] + (size_t)c * cs * f->esz;
@@ -777,9 +817,14 @@ extern "C" nb_status nb_field_wrap(nb_grid *g, nb_dtype dt, int32_t card, double
                 if (s == NB_OK)
                     s = fill_const_raw(g, b + (size_t)(cs - f->ps) * f->esz, f->ps, dt, outside, g->cs);
             }
+        } else {  // SOA_PLANE / AOS: a halo plane is card * plane contiguous elements
+            f->pcs[p] = nb_cstride(f, p);
+            const int64_t hp = f->plane * card;
+            s = fill_const_raw(g, f->base[p], hp, dt, outside, g->cs);
+            if (s == NB_OK) s = fill_const_raw(g, f->base[p] + (size_t)(n - hp) * f->esz, hp, dt, outside, g->cs);
         }
     }
-    f->cs = f->pcs[g->first_local];
+    if (s == NB_OK) f->cs = f->pcs[g->first_local];
     if (s == NB_OK && nb_is_peer(g)) s = nb_peer_field_map(f);  // collective
     if (s != NB_OK) {
         delete f;
@@ -791,7 +836,7 @@ extern "C" nb_status nb_field_wrap(nb_grid *g, nb_dtype dt, int32_t card, double
 }
 
 // component stride of partition p (dense): ps * (nz_p + 2)
-static inline int64_t dense_cs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
+static inline int64_t dense_cs(const nb_field *f, int p) { return nb_cstride(f, p); }
 
 extern "C" nb_status nb_field_destroy(nb_field *f) {
     if (!f) return NB_OK;
@@ -824,6 +869,67 @@ static size_t logical_bytes(const nb_field *f) {
     return (size_t)f->g->nx * f->g->ny * f->g->nz * f->card * f->esz;
 }
 
+// SOA_PLANE / AOS host transfers: the partition's slab of the dense logical
+// view [c][z][y][x] is staged in a packed device buffer and (un)packed into
+// the layout by one kernel
+template <typename T, bool TO_FIELD>
+__global__ void k_repack(T *field, T *packed, PGeo g, int64_t cstride, int64_t es, int card) {
+    const int x = blockIdx.x * blockDim.x + threadIdx.x, y = blockIdx.y;
+    if (x >= g.nx) return;
+    for (int64_t zc = blockIdx.z; zc < (int64_t)g.nzl * card; zc += gridDim.z) {
+        const int zl = (int)(zc % g.nzl), c = (int)(zc / g.nzl);
+        const int64_t fi = (int64_t)c * cstride + ((int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x) * es;
+        const int64_t pi = (((int64_t)c * g.nzl + zl) * g.ny + y) * g.nx + x;
+        if (TO_FIELD)
+            field[fi] = packed[pi];
+        else
+            packed[pi] = field[fi];
+    }
+}
+
+static nb_status dense_repack(nb_field *f, void *host, bool up) {
+    nb_grid *g = f->g;
+    for (int p = 0; p < g->nparts; ++p) {
+        if (!g->parts[p].local) continue;
+        const NbPart &q = g->parts[p];
+        const size_t slab = (size_t)g->nx * g->ny * q.nz() * f->esz, logical_c = (size_t)g->nx * g->ny * g->nz * f->esz;
+        void *tmp = nullptr;
+        NB_CUDA(cudaMallocAsync(&tmp, slab * f->card, g->cs));
+        char *h = (char *)host + (size_t)q.z0 * g->nx * g->ny * f->esz;
+        PGeo geo = pgeo(f, p);
+        dim3 blk(128), grd((g->nx + 127) / 128, g->ny, (unsigned)std::min<int64_t>((int64_t)geo.nzl * f->card, 65535));
+        if (up)
+            for (int c = 0; c < f->card; ++c)
+                NB_CUDA(cudaMemcpyAsync((char *)tmp + c * slab, h + c * logical_c, slab, cudaMemcpyHostToDevice, g->cs));
+        {
+            LaunchScope ls(g, g->cs, "k_repack");
+            if (f->dt == NB_F64 && up)
+                k_repack<double, true><<<grd, blk, 0, g->cs>>>((double *)f->base[p], (double *)tmp, geo, nb_cstride(f, p),
+                                                               f->es, f->card);
+            else if (f->dt == NB_F64)
+                k_repack<double, false><<<grd, blk, 0, g->cs>>>((double *)f->base[p], (double *)tmp, geo, nb_cstride(f, p),
+                                                                f->es, f->card);
+            else if (up)
+                k_repack<float, true><<<grd, blk, 0, g->cs>>>((float *)f->base[p], (float *)tmp, geo, nb_cstride(f, p),
+                                                              f->es, f->card);
+            else
+                k_repack<float, false><<<grd, blk, 0, g->cs>>>((float *)f->base[p], (float *)tmp, geo, nb_cstride(f, p),
+                                                               f->es, f->card);
+            NB_TRY(nb_launch_check("k_repack"));
+        }
+        if (!up)
+            for (int c = 0; c < f->card; ++c)
+                NB_CUDA(cudaMemcpyAsync(h + c * logical_c, (char *)tmp + c * slab, slab, cudaMemcpyDeviceToHost, g->cs));
+        NB_CUDA(cudaFreeAsync(tmp, g->cs));
+    }
+    if (!up) NB_CUDA(cudaStreamSynchronize(g->cs));
+    return NB_OK;
+}
+static nb_status dense_repack_upload(nb_field *f, const void *host) { return dense_repack(f, (void *)host, true); }
+static nb_status dense_repack_download(const nb_field *f, void *host) {
+    return dense_repack(const_cast<nb_field *>(f), host, false);
+}
+
 extern "C" nb_status nb_field_upload(nb_field *f, const void *host, int64_t nbytes) {
     if (!f || !host) NB_FAIL(NB_EINVAL, "nb_field_upload: NULL argument");
     if ((size_t)nbytes != logical_bytes(f))
@@ -831,6 +937,7 @@ extern "C" nb_status nb_field_upload(nb_field *f, const void *host, int64_t nbyt
     nb_grid *g = f->g;
     DeviceGuard dg(g->device);
     if (g->sparse) return nb_sparse_upload(f, host);
+    if (f->layout != NB_SOA) return dense_repack_upload(f, host);
     const char *h = (const char *)host;
     size_t row = (size_t)g->nx * f->esz, plane = row * g->ny;
     for (int p = 0; p < g->nparts; ++p) {
@@ -853,6 +960,7 @@ extern "C" nb_status nb_field_download(const nb_field *f, void *host, int64_t nb
     nb_grid *g = f->g;
     DeviceGuard dg(g->device);
     if (g->sparse) return nb_sparse_download(f, host);
+    if (f->layout != NB_SOA) return dense_repack_download(f, host);
     char *h = (char *)host;
     size_t row = (size_t)g->nx * f->esz, plane = row * g->ny;
     for (int p = 0; p < g->nparts; ++p) {
@@ -871,7 +979,7 @@ extern "C" nb_status nb_field_download(const nb_field *f, void *host, int64_t nb
 
 // ---- counter-based fill: nb_gen in nb_device.cuh ----------------------------
 template <typename T>
-__global__ void k_fill_gen(T *base, PGeo g, int64_t cstride, int card, int kind, uint64_t seed,
+__global__ void k_fill_gen(T *base, PGeo g, int64_t cstride, int64_t es, int card, int kind, uint64_t seed,
                            double a, double b, double h) {
     int x = blockIdx.x * blockDim.x + threadIdx.x;
     int y = blockIdx.y;
@@ -884,7 +992,7 @@ __global__ void k_fill_gen(T *base, PGeo g, int64_t cstride, int card, int kind,
         uint64_t gidx =
             (uint64_t)x + (uint64_t)g.nx * ((uint64_t)y + (uint64_t)g.ny * ((uint64_t)z + (uint64_t)g.NZ * c));
         double v = nb_gen(kind, seed, gidx, a, b, x, y, z, h);
-        base[(int64_t)c * cstride + (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x] = (T)v;
+        base[(int64_t)c * cstride + ((int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x) * es] = (T)v;
     }
 }
 
@@ -904,10 +1012,10 @@ extern "C" nb_status nb_field_fill(nb_field *f, nb_fill kind, uint64_t seed, dou
         dim3 blk(128), grd((g->nx + 127) / 128, g->ny, (unsigned)std::min<int64_t>((int64_t)geo.nzl * f->card, 65535));
         LaunchScope ls(g, g->cs, "k_fill_gen");
         if (f->dt == NB_F64)
-            k_fill_gen<double><<<grd, blk, 0, g->cs>>>((double *)f->base[p], geo, dense_cs(f, p), f->card,
+            k_fill_gen<double><<<grd, blk, 0, g->cs>>>((double *)f->base[p], geo, dense_cs(f, p), f->es, f->card,
                                                         kind, seed, a, b, h);
         else
-            k_fill_gen<float><<<grd, blk, 0, g->cs>>>((float *)f->base[p], geo, dense_cs(f, p), f->card,
+            k_fill_gen<float><<<grd, blk, 0, g->cs>>>((float *)f->base[p], geo, dense_cs(f, p), f->es, f->card,
                                                        kind, seed, a, b, h);
         NB_TRY(nb_launch_check("k_fill_gen"));
     }
@@ -1014,6 +1122,7 @@ static nb_status check_pair(const nb_field *x, const nb_field *y) {
     if (!x || !y) NB_FAIL(NB_EINVAL, "NULL field");
     if (x->g != y->g) NB_FAIL(NB_EMISMATCH, "fields belong to different grids");
     if (x->dt != y->dt || x->card != y->card) NB_FAIL(NB_EMISMATCH, "dtype / cardinality mismatch");
+    if (x->layout != y->layout) NB_FAIL(NB_EMISMATCH, "layout mismatch");
     return NB_OK;
 }
 
@@ -1045,9 +1154,13 @@ extern "C" nb_status nb_axpby(double a, const nb_field *x, double b, nb_field *y
     for (int p = 0; p < g->nparts; ++p) {
         if (!g->parts[p].local) continue;
         for (auto rg : view_ranges(g, p, v)) {
-            for (int c = 0; c < x->card; ++c) {
-                int64_t off = (int64_t)c * dense_cs(x, p) + (int64_t)(rg.first + 1) * x->ps;
-                int64_t n = (int64_t)(rg.second - rg.first) * x->ps;
+            // SOA: one range per component; SOA_PLANE / AOS: the planes of
+            // all components form one contiguous range
+            const int nr = x->layout == NB_SOA ? x->card : 1;
+            for (int c = 0; c < nr; ++c) {
+                int64_t off = x->layout == NB_SOA ? (int64_t)c * dense_cs(x, p) + (int64_t)(rg.first + 1) * x->ps
+                                                  : (int64_t)(rg.first + 1) * x->plane * x->card;
+                int64_t n = (int64_t)(rg.second - rg.first) * x->plane * (x->layout == NB_SOA ? 1 : x->card);
                 if (x->dt == NB_F64)
                     NB_TRY((launch_axpby<double, double2>(g, (const double *)x->base[p] + off,
                                                           (double *)y->base[p] + off, n, a, b)));
@@ -1071,21 +1184,22 @@ extern "C" nb_status nb_axpy(double a, const nb_field *x, nb_field *y, nb_view v
 // rows sequential, butterfly, then the warps of a 32 x 8 tile in order
 template <typename T>
 __global__ void __launch_bounds__(32 * ZW) k_dot(const T *__restrict__ x, const T *__restrict__ y, PGeo g,
-                                                 int64_t cstride, int nchunk, double *tp, int T_tiles, int tiles_y) {
+                                                 int64_t cstride, int64_t es, int nchunk, double *tp, int T_tiles,
+                                                 int tiles_y) {
     constexpr int ZR = ZR_STO, ZTY = ZW * ZR;
     __shared__ double sw[ZC][ZW];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int xi = blockIdx.x * DOT_TX + lane, yr = blockIdx.y * ZTY + w * ZR;
     const int c = blockIdx.z / nchunk, ch = blockIdx.z % nchunk;
     const int zs = ch * ZC, zend = min(g.nzl, zs + ZC);
-    const int64_t o = (int64_t)c * cstride + (int64_t)yr * g.pitch + xi + g.ps;
+    const int64_t o = (int64_t)yr * g.pitch + xi + g.ps;  // cell index; element = c * cstride + cell * es
     for (int z = zs; z < zend; ++z) {
         double col = 0.0;
 #pragma unroll
         for (int j = 0; j < ZR; ++j) {
             double prod = 0.0;
             if (xi < g.nx && yr + j < g.ny) {
-                const int64_t i = o + (int64_t)z * g.ps + (int64_t)j * g.pitch;
+                const int64_t i = (int64_t)c * cstride + (o + (int64_t)z * g.ps + (int64_t)j * g.pitch) * es;
                 prod = __dmul_rn((double)__ldcs(x + i), (double)__ldcs(y + i));
             }
             col = j == 0 ? prod : __dadd_rn(col, prod);
@@ -1204,7 +1318,7 @@ nb_status nb_dot_partials_view(const nb_field *x, const nb_field *y, nb_view v) 
         if (!g->parts[p].local) continue;
         for (auto rg : view_ranges(g, p, v)) {
             PGeo geo = pgeo(x, p);
-            const int64_t off = (int64_t)rg.first * geo.ps * x->esz;  // planes shift, every component alike
+            const int64_t off = (int64_t)rg.first * geo.ps * x->es * x->esz;  // planes shift, every component alike
             geo.z0 += rg.first;
             geo.nzl = rg.second - rg.first;
             int nchunk = (geo.nzl + ZC - 1) / ZC;
@@ -1212,11 +1326,11 @@ nb_status nb_dot_partials_view(const nb_field *x, const nb_field *y, nb_view v) 
             LaunchScope ls(g, g->cs, "k_dot");
             if (x->dt == NB_F64)
                 k_dot<double><<<grd, blk, 0, g->cs>>>((const double *)(x->base[p] + off),
-                                                       (const double *)(y->base[p] + off), geo, dense_cs(x, p), nchunk,
+                                                       (const double *)(y->base[p] + off), geo, dense_cs(x, p), x->es, nchunk,
                                                        g->tp, g->T, g->tiles_y);
             else
                 k_dot<float><<<grd, blk, 0, g->cs>>>((const float *)(x->base[p] + off),
-                                                      (const float *)(y->base[p] + off), geo, dense_cs(x, p), nchunk,
+                                                      (const float *)(y->base[p] + off), geo, dense_cs(x, p), x->es, nchunk,
                                                       g->tp, g->T, g->tiles_y);
             NB_TRY(nb_launch_check("k_dot"));
         }

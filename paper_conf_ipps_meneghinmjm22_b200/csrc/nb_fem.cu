@@ -1289,7 +1289,7 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_fem_r(double *r, const doubl
     }
 }
 
-static inline int64_t fcs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
+static inline int64_t fcs(const nb_field *f, int p) { return nb_cstride(f, p); }
 
 // what: FEM_SURF = only the surface-node kernels of the TMA path, FEM_BULK =
 // only the streaming kernel, FEM_ALL = both (the OCC schedule runs the
@@ -1385,6 +1385,7 @@ static nb_status fem_check(const nb_field *u) {
     if (!u) NB_FAIL(NB_EINVAL, "NULL field");
     if (u->g->sparse) NB_FAIL(NB_EUNSUPPORTED, "FEM on element-sparse grids is not built (SURVEY f4)");
     if (u->dt != NB_F64 || u->card != 3) NB_FAIL(NB_EMISMATCH, "FEM fields are fp64 with cardinality 3");
+    NB_LAYOUTS(u, (1 << NB_SOA) | (1 << NB_SOA_PLANE), "FEM");
     return NB_OK;
 }
 
@@ -1469,11 +1470,14 @@ nb_status nb_fem_cg_hooks(nb_cg *cg, int parity) {
         int nseg = 0;
         int64_t n = 0;
         if (fused) {
-            n = pn->ps;
+            n = pn->plane;  // one component's plane (SOA and SOA_PLANE)
             for (int c = 0; c < 3; ++c) {
                 if (q.lo >= 0) S.off[nseg++] = (int64_t)c * fcs(pn, p) + pn->ps;
                 if (q.hi >= 0 && q.nz() > 1) S.off[nseg++] = (int64_t)c * fcs(pn, p) + (int64_t)q.nz() * pn->ps;
             }
+        } else if (pn->layout == NB_SOA_PLANE) {  // all own planes of all components: one range
+            n = (int64_t)q.nz() * pn->ps;
+            S.off[nseg++] = pn->ps;
         } else {
             n = (int64_t)q.nz() * pn->ps;
             for (int c = 0; c < 3; ++c) S.off[nseg++] = (int64_t)c * fcs(pn, p) + pn->ps;

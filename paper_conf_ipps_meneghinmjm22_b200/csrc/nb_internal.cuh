@@ -201,7 +201,13 @@ struct nb_field {
     int card = 1;
     double outside = 0.0;
     size_t esz = 8;
-    int64_t pitch = 0, ps = 0, cs = 0;  // elements: row pitch, plane stride, component stride
+    // dense layouts (include/nb.h): element (c, cell) at c*cstride + cell*es,
+    // cell = (zl+1)*ps + y*pitch + x.  plane = pitch*ny cells; ps = plane
+    // (SOA, AOS) or card*plane (SOA_PLANE); es = card (AOS) or 1;
+    // cstride = ps*(nz_p+2) (SOA), plane (SOA_PLANE), 1 (AOS)
+    nb_layout layout = NB_SOA;
+    int64_t es = 1, plane = 0;
+    int64_t pitch = 0, ps = 0, cs = 0;  // cells: row pitch, plane stride; cs: component stride
     std::vector<char *> base;          // per partition (local only)
     std::vector<size_t> bytes;
     std::vector<int64_t> pcs;          // per-partition component stride (elements)
@@ -209,6 +215,19 @@ struct nb_field {
     bool borrowed = false;             // nb_field_wrap: caller-owned buffers (never freed)
     std::vector<uint64_t> map_off;     // per mapped partition: offset inside the peer's allocation
 };
+
+// component stride of partition p of a dense field (elements; see nb_field)
+inline int64_t nb_cstride(const nb_field *f, int p) {
+    if (f->layout == NB_SOA_PLANE) return f->plane;
+    if (f->layout == NB_AOS) return 1;
+    return f->ps * (f->g->parts[p].nz() + 2);
+}
+// fail unless f's layout is one of `mask` (1 << nb_layout)
+#define NB_LAYOUTS(f, mask, what)                                                                       \
+    do {                                                                                                \
+        if (!((mask) & (1 << (f)->layout)))                                                             \
+            NB_FAIL(NB_EUNSUPPORTED, "%s: field layout %d not supported (include/nb.h)", what, (int)(f)->layout); \
+    } while (0)
 
 // partition p's buffer of f is addressable from this process (local or mapped)
 inline bool nb_reachable(const nb_field *f, int p) { return p >= 0 && f->base[p] != nullptr; }
@@ -234,9 +253,10 @@ inline PGeo pgeo(const nb_field *f, int g) {
 }
 
 // pointer to plane zl (may be -1 or nzl: halo) of component c of partition g
+// (SOA / SOA_PLANE: the plane's elements of that component are contiguous)
 template <typename T>
 inline T *plane_ptr(const nb_field *f, int g, int c, int zl) {
-    return reinterpret_cast<T *>(f->base[g]) + (int64_t)c * f->cs + (int64_t)(zl + 1) * f->ps;
+    return reinterpret_cast<T *>(f->base[g]) + (int64_t)c * nb_cstride(f, g) + (int64_t)(zl + 1) * f->ps * f->es;
 }
 
 // ---------------------------------------------------------------------------

@@ -80,25 +80,27 @@ __device__ __forceinline__ void lbm_collide(const float (&f)[Q19], float om, flo
     }
 }
 
+// ES: element stride of a cell index (1: SOA / SOA_PLANE, 19: AOS)
+template <int ES>
 __device__ __forceinline__ void lbm_collide_store(const float (&f)[Q19], const LbmArgs &A, int64_t cell,
                                                   int zl, int64_t row) {
     float o[Q19];
     lbm_collide(f, A.omega, o);
 #pragma unroll
-    for (int i = 0; i < Q19; ++i) __stcs(A.fout[i] + cell, o[i]);
+    for (int i = 0; i < Q19; ++i) __stcs(A.fout[i] + cell * ES, o[i]);
     // halo transfer fused into the producing kernel: outgoing populations of
     // the boundary planes go straight into the neighbours' halo planes
     if (zl == 0 && A.rem_lo[14]) {
 #pragma unroll
-        for (int i = 14; i < 19; ++i) A.rem_lo[i][row] = o[i];
+        for (int i = 14; i < 19; ++i) A.rem_lo[i][row * ES] = o[i];
     }
     if (zl == A.g.nzl - 1 && A.rem_hi[9]) {
 #pragma unroll
-        for (int i = 9; i < 14; ++i) A.rem_hi[i][row] = o[i];
+        for (int i = 9; i < 14; ++i) A.rem_hi[i][row * ES] = o[i];
     }
 }
 
-template <bool PERIODIC>
+template <bool PERIODIC, int ES>
 // x-threads per CTA of the twoPop D3Q19 step (256: 3.18 -> 3.10 ms at
 // 512^3 against 128; 512 is slower, 3.75)
 #ifndef NB_LBM_BX
@@ -121,7 +123,7 @@ __global__ void __launch_bounds__(NB_LBM_BX) k_lbm_d3q19(LbmArgs A, int zb) {
         // loads at uniform offsets
 #pragma unroll
         for (int i = 0; i < Q19; ++i)
-            f[i] = __ldg(A.fin[i] + cell - (int64_t)CZv(i) * g.ps - (int64_t)CYv(i) * g.pitch - CXv(i));
+            f[i] = __ldg(A.fin[i] + (cell - (int64_t)CZv(i) * g.ps - (int64_t)CYv(i) * g.pitch - CXv(i)) * ES);
     } else {
 #pragma unroll
         for (int i = 0; i < Q19; ++i) {
@@ -129,14 +131,14 @@ __global__ void __launch_bounds__(NB_LBM_BX) k_lbm_d3q19(LbmArgs A, int zb) {
             if (PERIODIC) {
                 sx = sx < 0 ? sx + g.nx : (sx >= g.nx ? sx - g.nx : sx);
                 sy = sy < 0 ? sy + g.ny : (sy >= g.ny ? sy - g.ny : sy);
-                f[i] = __ldg(A.fin[i] + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx);
+                f[i] = __ldg(A.fin[i] + ((int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx) * ES);
             } else {
                 // in-domain neighbour, or half-way bounce-back from the
                 // opposite population of this cell (+ moving-lid term)
                 const int sgz = gz - CZv(i);
                 const bool inside = sx >= 0 && sx < g.nx && sy >= 0 && sy < g.ny && sgz >= 0 && sgz < g.NZ;
-                const float *src = inside ? A.fin[i] + (int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx
-                                          : A.fin[OPPv(i)] + cell;
+                const float *src = inside ? A.fin[i] + ((int64_t)(szl + 1) * g.ps + (int64_t)sy * g.pitch + sx) * ES
+                                          : A.fin[OPPv(i)] + cell * ES;
                 float v = __ldg(src);
                 if (CXv(i) != 0 && sy == g.ny && sx >= 0 && sx < g.nx && sgz >= 0 && sgz < g.NZ)
                     v = v + 6.0f * Wv(i) * A.rho_w * ((float)CXv(i) * A.ulid);
@@ -144,11 +146,11 @@ __global__ void __launch_bounds__(NB_LBM_BX) k_lbm_d3q19(LbmArgs A, int zb) {
             }
         }
     }
-    lbm_collide_store(f, A, cell, zl, row);
+    lbm_collide_store<ES>(f, A, cell, zl, row);
 }
 
-__global__ void __launch_bounds__(128) k_lbm_init(float *f, PGeo g, int64_t cs, float rho, float ux, float uy,
-                                                  float uz) {
+__global__ void __launch_bounds__(128) k_lbm_init(float *f, PGeo g, int64_t cs, int64_t es, float rho, float ux,
+                                                  float uy, float uz) {
     const int x = blockIdx.x * blockDim.x + threadIdx.x, y = blockIdx.y, zl = (int)blockIdx.z - 1;
     if (x >= g.nx) return;
     const int64_t cell = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
@@ -156,32 +158,37 @@ __global__ void __launch_bounds__(128) k_lbm_init(float *f, PGeo g, int64_t cs, 
 #pragma unroll
     for (int i = 0; i < Q19; ++i) {
         float cu = (float)CXv(i) * ux + (float)CYv(i) * uy + (float)CZv(i) * uz;
-        f[(int64_t)i * cs + cell] = Wv(i) * rho * (1.0f + 3.0f * cu + 4.5f * cu * cu - 1.5f * usq);
+        f[(int64_t)i * cs + cell * es] = Wv(i) * rho * (1.0f + 3.0f * cu + 4.5f * cu * cu - 1.5f * usq);
     }
 }
 
-__global__ void __launch_bounds__(128) k_lbm_macro(const float *f, float *rho_o, float *u_o, PGeo g, int64_t cs,
-                                                   int64_t cs_rho, int64_t cs_u) {
+// per-field addressing of the macroscopic kernel (the three fields may use
+// different layouts): element (c, zl, y, x) at c*cs + ((zl+1)*ps + y*pitch + x)*es
+struct LbmFa {
+    int64_t ps, cs, es;
+    __device__ __forceinline__ int64_t at(int c, int zl, int64_t row) const { return c * cs + ((zl + 1) * ps + row) * es; }
+};
+__global__ void __launch_bounds__(128) k_lbm_macro(const float *f, float *rho_o, float *u_o, PGeo g, LbmFa af,
+                                                   LbmFa ar, LbmFa au) {
     const int x = blockIdx.x * blockDim.x + threadIdx.x, y = blockIdx.y, zl = blockIdx.z;
     if (x >= g.nx) return;
-    const int64_t cell = (int64_t)(zl + 1) * g.ps + (int64_t)y * g.pitch + x;
+    const int64_t row = (int64_t)y * g.pitch + x;
     float rho = 0.f, jx = 0.f, jy = 0.f, jz = 0.f;
 #pragma unroll
     for (int i = 0; i < Q19; ++i) {
-        float v = f[(int64_t)i * cs + cell];
+        float v = f[af.at(i, zl, row)];
         rho += v;
         jx += (float)CXv(i) * v;
         jy += (float)CYv(i) * v;
         jz += (float)CZv(i) * v;
     }
-    (void)cs_rho;
-    rho_o[cell] = rho;
-    u_o[cell] = jx / rho;
-    u_o[cs_u + cell] = jy / rho;
-    u_o[2 * cs_u + cell] = jz / rho;
+    rho_o[ar.at(0, zl, row)] = rho;
+    u_o[au.at(0, zl, row)] = jx / rho;
+    u_o[au.at(1, zl, row)] = jy / rho;
+    u_o[au.at(2, zl, row)] = jz / rho;
 }
 
-static inline int64_t lcs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
+static inline int64_t lcs(const nb_field *f, int p) { return nb_cstride(f, p); }
 
 static nb_status lbm_check(const nb_field *f) {
     if (!f) NB_FAIL(NB_EINVAL, "NULL field");
@@ -355,7 +362,7 @@ extern "C" nb_status nb_lbm_init(nb_field *f, double rho0, const double u0[3]) {
         PGeo geo = pgeo(f, p);
         dim3 blk(128), grd((g->nx + 127) / 128, g->ny, geo.nzl + 2);  // halo planes too
         LaunchScope ls(g, g->cs, "k_lbm_init");
-        k_lbm_init<<<grd, blk, 0, g->cs>>>((float *)f->base[p], geo, lcs(f, p), (float)rho0, (float)u0[0],
+        k_lbm_init<<<grd, blk, 0, g->cs>>>((float *)f->base[p], geo, lcs(f, p), f->es, (float)rho0, (float)u0[0],
                                            (float)u0[1], (float)u0[2]);
         NB_TRY(nb_launch_check("k_lbm_init"));
     }
@@ -398,16 +405,21 @@ static nb_status launch_lbm(nb_grid *g, int p, nb_field *fin, nb_field *fout, co
         if (zb == 0 && nb_reachable(fout, lo))
             for (int i = 14; i < 19; ++i)
                 A.rem_lo[i] = (float *)fout->base[lo] + (int64_t)i * lcs(fout, lo) +
-                              (int64_t)(g->parts[lo].nz() + 1) * fout->ps;
+                              (int64_t)(g->parts[lo].nz() + 1) * fout->ps * fout->es;
         if (ze == g->parts[p].nz() && nb_reachable(fout, hi))
             for (int i = 9; i < 14; ++i) A.rem_hi[i] = (float *)fout->base[hi] + (int64_t)i * lcs(fout, hi);
     }
     dim3 blk(NB_LBM_BX), grd((g->nx + NB_LBM_BX - 1) / NB_LBM_BX, g->ny, ze - zb);
     LaunchScope ls(g, g->cs, "k_lbm_d3q19");
-    if (per)
-        k_lbm_d3q19<true><<<grd, blk, 0, g->cs>>>(A, zb);
+    const bool aos = fin->layout == NB_AOS;
+    if (per && aos)
+        k_lbm_d3q19<true, Q19><<<grd, blk, 0, g->cs>>>(A, zb);
+    else if (per)
+        k_lbm_d3q19<true, 1><<<grd, blk, 0, g->cs>>>(A, zb);
+    else if (aos)
+        k_lbm_d3q19<false, Q19><<<grd, blk, 0, g->cs>>>(A, zb);
     else
-        k_lbm_d3q19<false><<<grd, blk, 0, g->cs>>>(A, zb);
+        k_lbm_d3q19<false, 1><<<grd, blk, 0, g->cs>>>(A, zb);
     return nb_launch_check("k_lbm_d3q19");
 }
 
@@ -418,6 +430,7 @@ nb_status nb_lbm_view(nb_field *fin, nb_field *fout, const nb_lbm_params *prm, n
     NB_TRY(lbm_check(fin));
     NB_TRY(lbm_check(fout));
     if (fin->g != fout->g) NB_FAIL(NB_EMISMATCH, "fin and fout belong to different grids");
+    if (fin->layout != fout->layout) NB_FAIL(NB_EMISMATCH, "fin and fout have different layouts");
     if (fin == fout) NB_FAIL(NB_EINVAL, "twoPop needs two distinct buffers");
     if (prm->bc != NB_LBM_CAVITY) NB_FAIL(NB_EUNSUPPORTED, "Skeleton LBM containers: cavity boundaries");
     nb_grid *g = fin->g;
@@ -434,6 +447,7 @@ extern "C" nb_status nb_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm
     NB_TRY(lbm_check(fin));
     NB_TRY(lbm_check(fout));
     if (fin->g != fout->g) NB_FAIL(NB_EMISMATCH, "fin and fout belong to different grids");
+    if (fin->layout != fout->layout) NB_FAIL(NB_EMISMATCH, "fin and fout have different layouts");
     if (fin == fout) NB_FAIL(NB_EINVAL, "twoPop needs two distinct buffers");
     if (nsteps < 0) NB_FAIL(NB_EINVAL, "nsteps < 0");
     if (prm->bc != NB_LBM_CAVITY && prm->bc != NB_LBM_PERIODIC) NB_FAIL(NB_EINVAL, "bad bc");
@@ -603,6 +617,7 @@ extern "C" nb_status nb_lbm_step_aa(nb_field *f, const nb_lbm_params *prm, int32
     if (!f || !prm) NB_FAIL(NB_EINVAL, "nb_lbm_step_aa: NULL argument");
     NB_TRY(lbm_check(f));
     if (nsteps < 0 || (nsteps & 1)) NB_FAIL(NB_EINVAL, "nb_lbm_step_aa: nsteps must be even (got %d)", nsteps);
+    NB_LAYOUTS(f, 1 << NB_SOA, "nb_lbm_step_aa");
     if (prm->bc != NB_LBM_CAVITY && prm->bc != NB_LBM_PERIODIC) NB_FAIL(NB_EINVAL, "bad bc");
     nb_grid *g = f->g;
     if (g->sparse) NB_FAIL(NB_EUNSUPPORTED, "AA pattern on element-sparse grids is not built");
@@ -673,7 +688,8 @@ extern "C" nb_status nb_lbm_macroscopic(const nb_field *f, nb_field *rho, nb_fie
         dim3 blk(128), grd((g->nx + 127) / 128, g->ny, geo.nzl);
         LaunchScope ls(g, g->cs, "k_lbm_macro");
         k_lbm_macro<<<grd, blk, 0, g->cs>>>((const float *)f->base[p], (float *)rho->base[p], (float *)u->base[p], geo,
-                                            lcs(f, p), lcs(rho, p), lcs(u, p));
+                                            LbmFa{f->ps, lcs(f, p), f->es}, LbmFa{rho->ps, lcs(rho, p), rho->es},
+                                            LbmFa{u->ps, lcs(u, p), u->es});
         NB_TRY(nb_launch_check("k_lbm_macro"));
     }
     return NB_OK;

@@ -103,6 +103,7 @@ static nb_status d2q9_check(const nb_field *f) {
     if (!f) NB_FAIL(NB_EINVAL, "NULL field");
     const nb_grid *g = f->g;
     if (f->dt != NB_F32 || f->card != 9) NB_FAIL(NB_EMISMATCH, "D2Q9 needs an fp32 field of cardinality 9");
+    NB_LAYOUTS(f, 1 << NB_SOA, "D2Q9");
     if (g->sparse || g->nz != 1 || g->nparts != 1)
         NB_FAIL(NB_EUNSUPPORTED, "D2Q9: a dense grid of one plane (Nz = 1) on one partition");
     return NB_OK;

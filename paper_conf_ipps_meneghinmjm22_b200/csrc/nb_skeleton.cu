@@ -612,7 +612,7 @@ static nb_status sk_axpby_dev(nb_grid *g, const nb_container &c, const nb_field 
                      : (c.b_slot < 0 && c.b == 0.0) ? SKA_B0
                                                     : SKA_GEN;
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
-        const int64_t cs = x->ps * (g->parts[p].nz() + 2);
+        const int64_t cs = nb_cstride(x, p);
         for (auto rg : view_ranges(g, p, v))
             for (int k = 0; k < x->card; ++k) {
                 const int64_t off = (int64_t)k * cs + (int64_t)(rg.first + 1) * x->ps;

@@ -39,7 +39,7 @@ nb_status nb_c1_finalize_all(nb_grid *g, int iters);
 nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x, bool domap,
                      int zb, int ze, const CgScal *sc);
 
-static inline int64_t dcs(const nb_field *f, int p) { return f->ps * (f->g->parts[p].nz() + 2); }
+static inline int64_t dcs(const nb_field *f, int p) { return nb_cstride(f, p); }
 
 
 // ===========================================================================
@@ -764,6 +764,8 @@ static nb_status cg_check(const nb_field *x, const nb_field *b, const nb_cg_para
     if (x->dt != NB_F64 || b->dt != NB_F64) NB_FAIL(NB_EMISMATCH, "CG runs in fp64");
     int card = prm->op == NB_OP_FEM27 ? 3 : 1;
     if (x->card != card || b->card != card) NB_FAIL(NB_EMISMATCH, "CG operator needs cardinality %d", card);
+    if (x->layout != b->layout) NB_FAIL(NB_EMISMATCH, "x and b have different layouts");
+    if (prm->op == NB_OP_FEM27) NB_LAYOUTS(x, (1 << NB_SOA) | (1 << NB_SOA_PLANE), "FEM CG");
     if (prm->op != NB_OP_LAPLACE7 && prm->op != NB_OP_FEM27) NB_FAIL(NB_EINVAL, "bad operator");
     if (prm->occ < NB_OCC_NONE || prm->occ > NB_OCC_TWO_WAY) NB_FAIL(NB_EINVAL, "bad occ");
     if (prm->op == NB_OP_FEM27 && x->g->sparse) NB_FAIL(NB_EUNSUPPORTED, "FEM on sparse grids");
@@ -787,10 +789,10 @@ extern "C" nb_status nb_cg_create(nb_field *x, const nb_field *b, const nb_cg_pa
     cg->b = b;
     cg->prm = *prm;
     int card = x->card;
-    nb_status s = nb_field_create(g, NB_F64, card, 0.0, &cg->r);
-    if (s == NB_OK) s = nb_field_create(g, NB_F64, card, 0.0, &cg->p[0]);
-    if (s == NB_OK) s = nb_field_create(g, NB_F64, card, 0.0, &cg->p[1]);
-    if (s == NB_OK && (prm->op == NB_OP_FEM27 || g->sparse)) s = nb_field_create(g, NB_F64, card, 0.0, &cg->q);
+    nb_status s = nb_field_create(g, NB_F64, card, x->layout, 0.0, &cg->r);
+    if (s == NB_OK) s = nb_field_create(g, NB_F64, card, x->layout, 0.0, &cg->p[0]);
+    if (s == NB_OK) s = nb_field_create(g, NB_F64, card, x->layout, 0.0, &cg->p[1]);
+    if (s == NB_OK && (prm->op == NB_OP_FEM27 || g->sparse)) s = nb_field_create(g, NB_F64, card, x->layout, 0.0, &cg->q);
     if (s == NB_OK && cudaMalloc(&cg->sc, sizeof(CgScal)) != cudaSuccess) {
         nb_set_error("cudaMalloc scalars failed");
         s = NB_ENOMEM;

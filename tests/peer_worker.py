@@ -143,6 +143,24 @@ for bc in (nb.LBM_CAVITY, nb.LBM_PERIODIC):
 compare("lbm periodic 4 parts", (24, 20, 18), 2 * WORLD, lbm(nb.LBM_PERIODIC, nb.OCC_STANDARD, 6))
 
 
+def lbm_layout(layout, bc):
+    """AoS / plane-major SoA populations: the fused boundary stores go into
+    the neighbour's (IPC-mapped) halo with the layout's element stride."""
+    def fn(g):
+        a, b = nb.Field(g, "f32", 19, layout=layout), nb.Field(g, "f32", 19, layout=layout)
+        nb.nb_lbm_init(a, 1.0, (0.01, -0.02, 0.015) if bc == nb.LBM_PERIODIC else (0.0, 0.0, 0.0))
+        a, b = nb.nb_lbm_step(a, b, 0.9, 5, bc=bc, occ=nb.OCC_STANDARD)
+        out = [a.download()]
+        a.close(), b.close()
+        return out, []
+    return fn
+
+
+for layout in (nb.SOA_PLANE, nb.AOS):
+    compare(f"lbm layout{layout} cavity", (24, 20, 18), WORLD, lbm_layout(layout, nb.LBM_CAVITY))
+    compare(f"lbm layout{layout} periodic", (24, 20, 18), WORLD, lbm_layout(layout, nb.LBM_PERIODIC))
+
+
 def lbm_aa(bc):
     def fn(g):
         a = nb.Field(g, "f32", 19)
