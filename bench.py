@@ -302,6 +302,36 @@ def lbm_omega(nx, u_lid=0.05, re=100.0):
     return 1.0 / (3.0 * nu + 0.5)
 
 
+def bench_lbm_layouts(n, steps, local):
+    """SURVEY f3 / PAPER L248: the C3 twoPop step with the populations in
+    each field layout (SoA, plane-major SoA, AoS), 1 GPU, same bits."""
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    hbm, peak_kind = peaks()
+    rows = {}
+    for name, layout in (("soa", nb.SOA), ("soa_plane", nb.SOA_PLANE), ("aos", nb.AOS)):
+        g = nb.Grid((n, n, n), devices=[local])
+        stream = torch.cuda.ExternalStream(g.stream())
+        st = {"a": nb.Field(g, "f32", 19, layout=layout), "b": nb.Field(g, "f32", 19, layout=layout)}
+        nb.nb_lbm_init(st["a"], 1.0, (0.0, 0.0, 0.0))
+        om = lbm_omega(n)
+
+        def run(k):
+            st["a"], st["b"] = nb.nb_lbm_step(st["a"], st["b"], om, k)
+        run(3)
+        g.sync()
+        ms, clocks = timed(1, stream, lambda: run(steps), local)
+        gbs = LBM_BYTES_PER_CELL * n ** 3 * steps / (ms / 1e3) / 1e9
+        rows[name] = {"mlups": n ** 3 * steps / (ms / 1e3) / 1e6, "ms_per_step": ms / steps, "hbm_gbs": gbs,
+                      "hbm_frac": gbs / hbm, "clocks": clocks}
+        st["a"].close(), st["b"].close()
+        g.close()
+    return {"workload": f"C3 D3Q19 cavity {n}^3 fp32 twoPop, populations as SoA [c][z][y][x], plane-major SoA "
+                        "[z][c][y][x] and AoS [z][y][x][c] (PAPER L248; bitwise equal results)",
+            "rows": rows, "peak_kind": peak_kind}
+
+
 def bench_lbm_run(n, steps, warmup, world, local, occ="standard"):
     import torch
 
@@ -911,6 +941,7 @@ def main():
                            "skeleton_f1": bench_skeleton(local),
                            "lbm_sparse_f2": bench_lbm_sparse_run(args.n, 20, 3, local),
                            "lbm_aa_f3": bench_lbm_aa_run(args.n, 20, 4, local),
+                           "lbm_layouts_f3": bench_lbm_layouts(args.n, 10, local),
                            "karman_f4": bench_karman(local)}
             out["cpu_baseline"] = cpu_baseline_cg(args.n)
             out["also"]["lbm_d3q19"]["cpu_baseline"] = cpu_baseline_lbm()
