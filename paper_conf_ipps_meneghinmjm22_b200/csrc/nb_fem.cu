@@ -47,6 +47,10 @@ __host__ __device__ constexpr int fem_cv_class(int o, int i, int j) {
 }
 __host__ __device__ constexpr int fem_cv_sign(int o, int i, int j) { return i == j ? 1 : fem_oc(o, i) * fem_oc(o, j); }
 __constant__ const double *c_cls;       // surface-class stencils [FEM_NCLS][27 * 9] (device memory)
+// element-sparse node classes: (8-bit mask of the node's existing elements,
+// corner a = bit a) * 2 + (gz == 1: Dirichlet columns dropped) [512][27 * 9]
+constexpr int FEM_NSCLS = 512;
+__constant__ const double *c_scls;
 // the surface classes of grids with nx, ny, nz >= 3 (those with all axis
 // states in {0, 1, 2} and a non-Dirichlet z state), copied into constant
 // memory: a warp whose nodes share a class reads each coefficient with one
@@ -198,6 +202,28 @@ static nb_status fem_upload_constants(double E, double nu) {
             }
         }
     }
+    // element-sparse classes: the same accumulation (corner a, then b, in
+    // increasing order) over the node's existing elements, so a node whose
+    // element set is a box surface class gets the very same stencil
+    std::vector<double> scls((size_t)FEM_NSCLS * 243, 0.0);
+    for (int k = 0; k < FEM_NSCLS; ++k) {
+        const int drop = k & 1, em = k >> 1;
+        double *C = scls.data() + (size_t)k * 243;
+        for (int a = 0; a < 8; ++a) {
+            if (!((em >> a) & 1)) continue;
+            for (int b = 0; b < 8; ++b) {
+                const int ox = (b & 1) - (a & 1), oy = ((b >> 1) & 1) - ((a >> 1) & 1), oz = ((b >> 2) & 1) - ((a >> 2) & 1);
+                if (drop && oz == -1) continue;
+                const int o = (oz + 1) * 9 + (oy + 1) * 3 + (ox + 1);
+                for (int i = 0; i < 3; ++i)
+                    for (int j = 0; j < 3; ++j) C[o * 9 + i * 3 + j] += ke[(3 * a + i) * 24 + 3 * b + j];
+            }
+        }
+    }
+    static double *d_scls = nullptr;
+    if (!d_scls) NB_CUDA(cudaMalloc(&d_scls, sizeof(double) * scls.size()));
+    NB_CUDA(cudaMemcpy(d_scls, scls.data(), sizeof(double) * scls.size(), cudaMemcpyHostToDevice));
+    NB_CUDA(cudaMemcpyToSymbol(c_scls, &d_scls, sizeof(d_scls)));
     static double *d_cls = nullptr;
     if (!d_cls) NB_CUDA(cudaMalloc(&d_cls, sizeof(double) * cls.size()));
     NB_CUDA(cudaMemcpy(d_cls, cls.data(), sizeof(double) * cls.size(), cudaMemcpyHostToDevice));
@@ -1381,9 +1407,171 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
     return nb_launch_check(name);
 }
 
+// ===========================================================================
+// K u on element-sparse grids.  One
+// thread per active node of a 256-cell dot segment (the sparse canonical dot
+// order, per component).  The node's 27-neighbourhood comes from the
+// nb_sparse_fem_tables mask and row bases; its existing elements (those with
+// all 8 nodes active) select the stencil: all 8 and gz >= 2 -> the dense
+// interior chain (c_S, structural zeros skipped), otherwise the sparse class
+// stencil over the active positions (fem_node_surf_l's chain), gz = 0 ->
+// identity row.  A full mask therefore reproduces the dense operator bit for
+// bit; general masks are the oracle's element-by-element K (tolerance).
+// ===========================================================================
+struct SpFemArgs {
+    const int32_t *seg;
+    int64_t seg0, nseg;
+    const int64_t *pstart;
+    const uint32_t *fm;
+    const int32_t *fb;
+    int64_t n, hl, cs;
+    int gz0, NZ, T;
+    double *tp;
+    const double *u, *b;
+    double *y;
+    const CgScal *sc;
+};
+
+template <int KIND>  // 0: y = K u; 1: q = K u, <u, q>; 2: y = b - K u, <y, y>
+__global__ void __launch_bounds__(256) k_sp_fem(SpFemArgs A) {
+    __shared__ double sw[3][8];
+    const int t = threadIdx.x;
+    const int e = __ldg(A.seg + A.seg0 + blockIdx.x);
+    const int zl = e >> 16, sg = e & 0xffff;
+    const int64_t j = __ldg(A.pstart + zl) + (int64_t)sg * 256 + t;
+    const bool valid = j < __ldg(A.pstart + zl + 1);
+    if (KIND == 1 && A.sc->status != 0) return;
+    double prod[3] = {0.0, 0.0, 0.0};
+    if (valid) {
+        const int gz = A.gz0 + zl;
+        const int64_t i = A.hl + j;
+        double o[3];
+        if (gz == 0) {  // Dirichlet identity row
+#pragma unroll
+            for (int c = 0; c < 3; ++c) o[c] = A.u[c * A.cs + i];
+        } else {
+            const uint32_t m = __ldg(A.fm + j);
+            int32_t base[9];
+#pragma unroll
+            for (int r = 0; r < 9; ++r) base[r] = __ldg(A.fb + (int64_t)r * A.n + j);
+            int em = 0;  // existing elements: corner a of the element at node - off(a)
+#pragma unroll
+            for (int a = 0; a < 8; ++a) {
+                bool ex = true;
+#pragma unroll
+                for (int b = 0; b < 8; ++b) {
+                    const int ox = (b & 1) - (a & 1), oy = ((b >> 1) & 1) - ((a >> 1) & 1),
+                              oz = ((b >> 2) & 1) - ((a >> 2) & 1);
+                    ex = ex && ((m >> ((ox + 1) + 3 * (oy + 1) + 9 * (oz + 1))) & 1u);
+                }
+                em |= ex ? 1 << a : 0;
+            }
+            const bool drop = gz == 1;
+            const bool interior = em == 0xff && !drop;
+            const double *C = c_scls + (size_t)(em * 2 + (drop ? 1 : 0)) * 243;
+            double acc0 = 0.0, acc1 = 0.0, acc2 = 0.0;
+#pragma unroll
+            for (int q = 0; q < 27; ++q) {
+                if (!((m >> q) & 1u)) continue;
+                const int ox = q % 3 - 1, oy = (q / 3) % 3 - 1, oz = q / 9 - 1, r = q / 3;
+                const uint32_t rb = (m >> (3 * r)) & 7u;
+                const int64_t idx = base[r] + __popc(rb & ((1u << (ox + 1)) - 1u));
+                const double u0 = __ldg(A.u + idx), u1 = __ldg(A.u + A.cs + idx), u2 = __ldg(A.u + 2 * A.cs + idx);
+                if (interior) {
+                    const double *S = c_S + q * 9;
+                    acc0 = fma(S[0], u0, acc0);
+                    if (ox != 0 && oy != 0) acc0 = fma(S[1], u1, acc0);
+                    if (ox != 0 && oz != 0) acc0 = fma(S[2], u2, acc0);
+                    if (oy != 0 && ox != 0) acc1 = fma(S[3], u0, acc1);
+                    acc1 = fma(S[4], u1, acc1);
+                    if (oy != 0 && oz != 0) acc1 = fma(S[5], u2, acc1);
+                    if (oz != 0 && ox != 0) acc2 = fma(S[6], u0, acc2);
+                    if (oz != 0 && oy != 0) acc2 = fma(S[7], u1, acc2);
+                    acc2 = fma(S[8], u2, acc2);
+                } else {
+                    const double *K = C + q * 9;
+                    acc0 = fma(__ldg(K + 0), u0, acc0);
+                    acc0 = fma(__ldg(K + 1), u1, acc0);
+                    acc0 = fma(__ldg(K + 2), u2, acc0);
+                    acc1 = fma(__ldg(K + 3), u0, acc1);
+                    acc1 = fma(__ldg(K + 4), u1, acc1);
+                    acc1 = fma(__ldg(K + 5), u2, acc1);
+                    acc2 = fma(__ldg(K + 6), u0, acc2);
+                    acc2 = fma(__ldg(K + 7), u1, acc2);
+                    acc2 = fma(__ldg(K + 8), u2, acc2);
+                }
+            }
+            o[0] = acc0;
+            o[1] = acc1;
+            o[2] = acc2;
+        }
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+            const int64_t k = c * A.cs + i;
+            if (KIND == 2) {
+                const double r = __dsub_rn(A.b[k], o[c]);
+                A.y[k] = r;
+                prod[c] = __dmul_rn(r, r);
+            } else {
+                A.y[k] = o[c];
+                if (KIND == 1) prod[c] = __dmul_rn(A.u[k], o[c]);
+            }
+        }
+    }
+    if (KIND == 0) return;
+    const int w = t >> 5;
+#pragma unroll
+    for (int c = 0; c < 3; ++c) {
+        const double v = warp_sum_canon(prod[c]);
+        if ((t & 31) == 0) sw[c][w] = v;
+    }
+    __syncthreads();
+    if (t < 3) {
+        double s = sw[t][0];
+#pragma unroll
+        for (int ww = 1; ww < 8; ++ww) s = __dadd_rn(s, sw[t][ww]);
+        A.tp[((int64_t)t * A.NZ + A.gz0 + zl) * A.T + sg] = s;
+    }
+}
+
+nb_status nb_sparse_fem_pass(nb_grid *g, int p, int kind, const int32_t *list, const int32_t *gidx, int64_t s0,
+                             int64_t n, const double *u, const double *b, double *y, const CgScal *sc) {
+    (void)gidx;
+    if (n <= 0) return NB_OK;
+    const NbSparsePart &sp = g->sp[p];
+    SpFemArgs A{};
+    A.seg = list;
+    A.seg0 = s0;
+    A.nseg = n;
+    A.pstart = sp.d_pstart;
+    A.fm = sp.d_fm;
+    A.fb = sp.d_fb;
+    A.n = sp.n;
+    A.hl = sp.hl;
+    A.cs = sp.cs;
+    A.gz0 = g->parts[p].z0;
+    A.NZ = g->nz;
+    A.T = g->T;
+    A.tp = g->tp;
+    A.u = u;
+    A.b = b;
+    A.y = y;
+    A.sc = sc;
+    const char *name = kind == 0 ? "k_fem_apply" : (kind == 1 ? "k_sp_fem_q" : "k_fem_cg_init");
+    LaunchScope ls(g, g->cs, name);
+    if (kind == 0)
+        k_sp_fem<0><<<(unsigned)n, 256, 0, g->cs>>>(A);
+    else if (kind == 1)
+        k_sp_fem<1><<<(unsigned)n, 256, 0, g->cs>>>(A);
+    else
+        k_sp_fem<2><<<(unsigned)n, 256, 0, g->cs>>>(A);
+    return nb_launch_check(name);
+}
+
+nb_status nb_sparse_fem_rhs(nb_field *b, double pr);
+
 static nb_status fem_check(const nb_field *u) {
     if (!u) NB_FAIL(NB_EINVAL, "NULL field");
-    if (u->g->sparse) NB_FAIL(NB_EUNSUPPORTED, "FEM on element-sparse grids is not built (SURVEY f4)");
     if (u->dt != NB_F64 || u->card != 3) NB_FAIL(NB_EMISMATCH, "FEM fields are fp64 with cardinality 3");
     NB_LAYOUTS(u, (1 << NB_SOA) | (1 << NB_SOA_PLANE), "FEM");
     return NB_OK;
@@ -1396,6 +1584,15 @@ extern "C" nb_status nb_fem27_apply(const nb_field *u, nb_field *y, double E, do
     nb_grid *g = u->g;
     cudaSetDevice(g->device);
     NB_TRY(fem_upload_constants(E, nu));
+    if (g->sparse) {
+        NB_TRY(nb_sparse_fem_tables(g));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbSparsePart &sp = g->sp[p];
+            NB_TRY(nb_sparse_fem_pass(g, p, 0, sp.d_seg, nullptr, 0, sp.seg_start.back(),
+                                      (const double *)u->base[p], nullptr, (double *)y->base[p], nullptr));
+        }
+        return NB_OK;
+    }
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         FemArgs A{};
         A.u = (const double *)u->base[p];
@@ -1427,6 +1624,7 @@ extern "C" nb_status nb_fem27_rhs(nb_field *b, double pressure) {
     NB_TRY(fem_check(b));
     nb_grid *g = b->g;
     cudaSetDevice(g->device);
+    if (g->sparse) return nb_sparse_fem_rhs(b, pressure);
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         PGeo geo = pgeo(b, p);
         dim3 blk(128), grd((g->nx + 127) / 128, g->ny, geo.nzl);
@@ -1441,6 +1639,16 @@ extern "C" nb_status nb_fem27_rhs(nb_field *b, double pressure) {
 nb_status nb_fem_cg_init(nb_cg *cg) {
     nb_grid *g = cg->g;
     NB_TRY(fem_upload_constants(cg->prm.fem_E, cg->prm.fem_nu));
+    if (g->sparse) {
+        NB_TRY(nb_sparse_fem_tables(g));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbSparsePart &sp = g->sp[p];
+            NB_TRY(nb_sparse_fem_pass(g, p, 2, sp.d_seg, nullptr, 0, sp.seg_start.back(),
+                                      (const double *)cg->x->base[p], (const double *)cg->b->base[p],
+                                      (double *)cg->r->base[p], nullptr));
+        }
+        return nb_reduce_finalize(g, 3, FIN_CG_INIT, cg->sc, 0);
+    }
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         FemArgs A{};
         A.u = (const double *)cg->x->base[p];
@@ -1458,8 +1666,11 @@ nb_status nb_fem_cg_init(nb_cg *cg) {
 // Both compute the same values in the same order (bitwise).
 static bool fem_fused() { return !getenv("NB_FEM_KERNEL") && !getenv("NB_FEM_3PASS") && nb_tma_enabled(); }
 
+nb_status nb_sparse_fem_cg_hooks(nb_cg *cg);  // nb_sparse.cu
+
 nb_status nb_fem_cg_hooks(nb_cg *cg, int parity) {
     nb_grid *g = cg->g;
+    if (g->sparse) return nb_sparse_fem_cg_hooks(cg);
     nb_field *pn = cg->p[parity], *po = cg->p[parity ^ 1];
     const bool fused = fem_fused();
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {

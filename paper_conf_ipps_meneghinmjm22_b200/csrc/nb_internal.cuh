@@ -147,6 +147,12 @@ struct NbSparsePart {
     void *d_nbr = nullptr;
     void *d_seginfo = nullptr;
     int64_t n_runs = 0;
+    // FEM 27-neighbourhood (lazy, nb_sparse_fem_tables): fm[j] bit
+    // (ox+1) + 3(oy+1) + 9(oz+1) = that neighbour active; fb[r][j] = buffer
+    // index of the first active cell among x-1 .. x+1 of row r = (oy+1) +
+    // 3(oz+1), -1 if none (active cells of a row are consecutive indices)
+    uint32_t *d_fm = nullptr;
+    int32_t *d_fb = nullptr;
 };
 
 struct nb_grid {
@@ -388,6 +394,13 @@ enum { NB_HALO_GENERIC = 0, NB_HALO_SEND = 1 };
 nb_status nb_halo_run_mode(nb_field *f, bool periodic, int c0u, int c1u, int c0d, int c1d, cudaStream_t s,
                            int mode);
 nb_status nb_sparse_halo_run(nb_field *f, int c0u, int c1u, int c0d, int c1d, cudaStream_t s, int mode);
+// element-sparse FEM (nb_sparse.cu tables, nb_fem.cu operator)
+nb_status nb_sparse_fem_tables(nb_grid *g);
+// one pass of the sparse FEM operator over segment list entries [s0, s0+n) of
+// `list` (gidx: their global segment indices, NULL = s0 + q) of partition p.
+// kind: 0 = y = K u, 1 = q = K u with <u, q>, 2 = y = b - K u with <y, y>
+nb_status nb_sparse_fem_pass(nb_grid *g, int p, int kind, const int32_t *list, const int32_t *gidx, int64_t s0,
+                             int64_t n, const double *u, const double *b, double *y, const CgScal *sc);
 nb_status nb_nccl_allreduce_sum(nb_grid *g, const double *send, double *recv, size_t n,
                                 cudaStream_t s);
 nb_status nb_nccl_group(nb_grid *g, bool start);

@@ -47,6 +47,10 @@ void nb_sparse_free(nb_grid *g) {
         cudaFree(s.d_seg_bnd_gi);
         cudaFree(s.d_nbr);
         cudaFree(s.d_seginfo);
+        cudaFree(s.d_fm);
+        cudaFree(s.d_fb);
+        s.d_fm = nullptr;
+        s.d_fb = nullptr;
         s.d_seg_bnd = s.d_seg_bnd_gi = nullptr;
         s.d_nbr = s.d_seginfo = nullptr;
         s.n_runs = 0;
@@ -1229,10 +1233,213 @@ nb_status nb_sparse_cg_flush(nb_cg *cg) {
     nb_grid *g = cg->g;
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         const NbSparsePart &sp = g->sp[p];
-        LaunchScope ls(g, g->cs, "k_sp_cg_flush");
-        k_sp_cg_flush<<<296, 256, 0, g->cs>>>((double *)cg->x->base[p] + sp.hl, (const double *)cg->p[0]->base[p] + sp.hl,
-                                              sp.n, cg->sc);
-        NB_TRY(nb_launch_check("k_sp_cg_flush"));
+        for (int c = 0; c < cg->x->card; ++c) {
+            const int64_t o = (int64_t)c * cg->x->pcs[p] + sp.hl;
+            LaunchScope ls(g, g->cs, "k_sp_cg_flush");
+            k_sp_cg_flush<<<296, 256, 0, g->cs>>>((double *)cg->x->base[p] + o, (const double *)cg->p[0]->base[p] + o,
+                                                  sp.n, cg->sc);
+            NB_TRY(nb_launch_check("k_sp_cg_flush"));
+        }
     }
+    return NB_OK;
+}
+
+// ===========================================================================
+// FEM on element-sparse grids (the
+// linear-elastic FEM on "dense and sparse" domains).  Nodes = active cells;
+// an element exists iff its 8 nodes are active (the oracle's reading,
+// oracle/oracle.c elem_exists).  The operator (nb_fem.cu k_sp_fem) needs each
+// node's 27-neighbourhood: an activity mask and, per (y, z) row, the buffer
+// index of the first active cell among x-1 .. x+1 (a row's active cells are
+// consecutive in the (z, y, x) order), 40 B per node, built here once.
+// ===========================================================================
+__global__ void k_sp_fem_tab(const uint8_t *__restrict__ mask, const int32_t *__restrict__ map, int nx, int ny,
+                             int slab_z0, int nslab, int z0, int hl, int64_t n, uint32_t *fm, int32_t *fb) {
+    const int x = blockIdx.x * blockDim.x + threadIdx.x, y = blockIdx.y, z = z0 + blockIdx.z;
+    if (x >= nx) return;
+    const int64_t plane = (int64_t)nx * ny;
+    const int64_t cell = (int64_t)(z - slab_z0) * plane + (int64_t)y * nx + x;
+    if (!mask[cell]) return;
+    const int64_t j = (int64_t)map[cell] - hl;
+    uint32_t m = 0;
+#pragma unroll
+    for (int r = 0; r < 9; ++r) {
+        const int yy = y + r % 3 - 1, zz = z + r / 3 - 1 - slab_z0;
+        int32_t base = -1;
+        if (yy >= 0 && yy < ny && zz >= 0 && zz < nslab) {
+            const int64_t row = (int64_t)zz * plane + (int64_t)yy * nx;
+#pragma unroll
+            for (int dx = -1; dx <= 1; ++dx) {
+                const int xx = x + dx;
+                if (xx < 0 || xx >= nx || !mask[row + xx]) continue;
+                m |= 1u << (r * 3 + dx + 1);
+                if (base < 0) base = map[row + xx];
+            }
+        }
+        fb[(int64_t)r * n + j] = base;
+    }
+    fm[j] = m;
+}
+
+nb_status nb_sparse_fem_tables(nb_grid *g) {
+    if (!g->sparse) return NB_OK;
+    DeviceGuard dg(g->device);
+    const int nx = g->nx, ny = g->ny;
+    const int64_t plane = (int64_t)nx * ny;
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        NbSparsePart &sp = g->sp[p];
+        if (sp.d_fm) continue;
+        const NbPart &q = g->parts[p];
+        const int slab_z0 = q.z0 - (q.lo >= 0 ? 1 : 0), slab_z1 = q.z1 + (q.hi >= 0 ? 1 : 0);
+        const int nslab = slab_z1 - slab_z0;
+        const int64_t ncell = (int64_t)nslab * plane;
+        uint8_t *d_mask = nullptr;
+        int32_t *d_map = nullptr;
+        void *tmp = nullptr;
+        size_t tmp_bytes = 0;
+        NB_CUDA(cudaMalloc(&sp.d_fm, sizeof(uint32_t) * std::max<int64_t>(sp.n, 1)));
+        NB_CUDA(cudaMalloc(&sp.d_fb, sizeof(int32_t) * 9 * std::max<int64_t>(sp.n, 1)));
+        NB_CUDA(cudaMalloc(&d_mask, ncell));
+        NB_CUDA(cudaMalloc(&d_map, ncell * 4));
+        NB_CUDA(cudaMemcpyAsync(d_mask, g->host_mask.data() + (int64_t)slab_z0 * plane, ncell, cudaMemcpyHostToDevice,
+                                g->cs));
+        cub::TransformInputIterator<int, MaskToInt, const uint8_t *> it(d_mask, MaskToInt());
+        cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, it, d_map, ncell, g->cs);
+        NB_CUDA(cudaMalloc(&tmp, tmp_bytes));
+        NB_CUDA(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, it, d_map, ncell, g->cs));
+        if (q.nz() > 0 && sp.n > 0) {
+            dim3 blk(128), grd((nx + 127) / 128, ny, q.nz());
+            LaunchScope ls(g, g->cs, "k_sp_fem_tab");
+            k_sp_fem_tab<<<grd, blk, 0, g->cs>>>(d_mask, d_map, nx, ny, slab_z0, nslab, q.z0, (int)sp.hl, sp.n, sp.d_fm,
+                                                 sp.d_fb);
+            NB_TRY(nb_launch_check("k_sp_fem_tab"));
+        }
+        NB_CUDA(cudaStreamSynchronize(g->cs));
+        cudaFree(d_mask);
+        cudaFree(d_map);
+        cudaFree(tmp);
+    }
+    return NB_OK;
+}
+
+// consistent nodal load of pressure pr on the exposed top faces (+z) of the
+// existing elements (oracle or_fem_rhs with a mask): a node gets pr/4 from
+// each existing element below it whose top face is exposed (no existing
+// element above), Dirichlet (z = 0) nodes none.  Element tests use the
+// 27-neighbourhood mask: element with lower corner node + (dx, dy, dz)
+__device__ __forceinline__ bool sp_fem_elem(uint32_t m, int dx, int dy, int dz) {
+#pragma unroll
+    for (int b = 0; b < 8; ++b) {
+        const int ox = dx + (b & 1), oy = dy + ((b >> 1) & 1), oz = dz + ((b >> 2) & 1);
+        if (ox < -1 || ox > 1 || oy < -1 || oy > 1 || oz < -1 || oz > 1) return false;
+        if (!((m >> ((ox + 1) + 3 * (oy + 1) + 9 * (oz + 1))) & 1u)) return false;
+    }
+    return true;
+}
+
+__global__ void k_sp_fem_rhs(const int32_t *__restrict__ seg, int64_t nseg, const int64_t *__restrict__ pstart,
+                             const uint32_t *__restrict__ fm, int64_t hl, int64_t cs, int gz0, double pr, double *b) {
+    const int64_t q = blockIdx.x;
+    if (q >= nseg) return;
+    const int e = seg[q], zl = e >> 16;
+    const int64_t j = pstart[zl] + (int64_t)(e & 0xffff) * SEG + threadIdx.x;
+    if (j >= pstart[zl + 1]) return;
+    const int gz = gz0 + zl;
+    const uint32_t m = fm[j];
+    double v = 0.0;
+    if (gz > 0) {
+        // elements below (dz = -1) having this node as a top corner, exposed
+        // when the element above them (dz = 0, same dx, dy) does not exist;
+        // added in the oracle's element order (ey, then ex)
+        for (int dy = -1; dy <= 0; ++dy)
+            for (int dx = -1; dx <= 0; ++dx)
+                if (sp_fem_elem(m, dx, dy, -1) && !sp_fem_elem(m, dx, dy, 0)) v = v + 0.25 * pr;
+    }
+    b[0 * cs + hl + j] = 0.0;
+    b[1 * cs + hl + j] = 0.0;
+    b[2 * cs + hl + j] = v;
+}
+
+nb_status nb_sparse_fem_rhs(nb_field *b, double pr) {
+    nb_grid *g = b->g;
+    NB_TRY(nb_sparse_fem_tables(g));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbSparsePart &sp = g->sp[p];
+        const int64_t nseg = sp.seg_start.back();
+        if (nseg <= 0) continue;
+        LaunchScope ls(g, g->cs, "k_fem_rhs");
+        k_sp_fem_rhs<<<(unsigned)nseg, SEG, 0, g->cs>>>(sp.d_seg, nseg, sp.d_pstart, sp.d_fm, sp.hl, b->pcs[p],
+                                                       g->parts[p].z0, pr, (double *)b->base[p]);
+        NB_TRY(nb_launch_check("k_sp_fem_rhs"));
+    }
+    return NB_OK;
+}
+
+// sparse FEM CG: map (x deferred update, p = r + beta p) per component ->
+// halo(p, 3 components) -> q = K p, <p, q> -> alpha -> r -= alpha q, <r, r>
+// per component -> beta (the Poisson sparse schedule with the FEM operator;
+// OCC as there: boundary map, halo in flight with the interior map / K p,
+// boundary K p after the wait)
+nb_status nb_sparse_fem_cg_hooks(nb_cg *cg) {
+    nb_grid *g = cg->g;
+    nb_field *p_ = cg->p[0];
+    const nb_occ occ = cg->prm.occ;
+    const bool split = occ != NB_OCC_NONE && g->nparts > 1 && (nb_is_peer(g) || nb_halo_on_stream(g));
+    auto map_args = [&](int p, int c) {
+        SpArgs A{};
+        const int64_t o = (int64_t)c * p_->pcs[p];
+        A.a = (const double *)cg->r->base[p] + o;
+        A.c = (double *)p_->base[p] + o;
+        A.d = (double *)cg->x->base[p] + o;
+        A.sc = cg->sc;
+        return A;
+    };
+    auto qpass = [&](int p, const int32_t *list, const int32_t *gi, int64_t s0, int64_t n) {
+        return nb_sparse_fem_pass(g, p, 1, list, gi, s0, n, (const double *)p_->base[p], nullptr,
+                                  (double *)cg->q->base[p], cg->sc);
+    };
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        const NbSparsePart &sp = g->sp[p];
+        for (int c = 0; c < 3; ++c) {
+            if (split)
+                NB_TRY(sp_launch_list<SPK_CG_MAP>(g, p, sp.d_seg_bnd, sp.n_seg_bnd, map_args(p, c), 0, "k_sp_cg_map"));
+            else
+                NB_TRY(sp_launch<SPK_CG_MAP>(g, p, 0, g->parts[p].nz(), map_args(p, c), 0, "k_sp_cg_map"));
+        }
+    }
+    if (!split) {
+        NB_TRY(nb_sparse_halo_update(p_));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbSparsePart &sp = g->sp[p];
+            NB_TRY(qpass(p, sp.d_seg, nullptr, 0, sp.seg_start.back()));
+        }
+    } else {
+        NB_TRY(nb_halo_split_begin(p_, 0, 3, cg->hs));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbPart &q = g->parts[p];
+            const NbSparsePart &sp = g->sp[p];
+            const int ib = q.lo >= 0 ? 1 : 0, ie = std::max(ib, q.nz() - (q.hi >= 0 ? 1 : 0));
+            for (int c = 0; c < 3; ++c)
+                NB_TRY(sp_launch<SPK_CG_MAP>(g, p, ib, ie, map_args(p, c), 0, "k_sp_cg_map"));
+            NB_TRY(qpass(p, sp.d_seg, nullptr, sp.seg_start[ib], sp.seg_start[ie] - sp.seg_start[ib]));
+        }
+        NB_TRY(nb_halo_split_wait(g, cg->hs));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+            const NbSparsePart &sp = g->sp[p];
+            NB_TRY(qpass(p, sp.d_seg_bnd, sp.d_seg_bnd_gi, 0, sp.n_seg_bnd));
+        }
+    }
+    NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+        for (int c = 0; c < 3; ++c) {
+            SpArgs A{};
+            const int64_t o = (int64_t)c * p_->pcs[p];
+            A.a = (const double *)cg->q->base[p] + o;
+            A.c = (double *)cg->r->base[p] + o;
+            A.sc = cg->sc;
+            NB_TRY(sp_launch<SPK_CG_R>(g, p, 0, g->parts[p].nz(), A, c * g->nz, "k_sp_cg_r"));
+        }
+    NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_RR, cg->sc, 0));
+    cg->k += 1;
     return NB_OK;
 }

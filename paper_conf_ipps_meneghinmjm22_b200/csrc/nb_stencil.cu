@@ -768,7 +768,6 @@ static nb_status cg_check(const nb_field *x, const nb_field *b, const nb_cg_para
     if (prm->op == NB_OP_FEM27) NB_LAYOUTS(x, (1 << NB_SOA) | (1 << NB_SOA_PLANE), "FEM CG");
     if (prm->op != NB_OP_LAPLACE7 && prm->op != NB_OP_FEM27) NB_FAIL(NB_EINVAL, "bad operator");
     if (prm->occ < NB_OCC_NONE || prm->occ > NB_OCC_TWO_WAY) NB_FAIL(NB_EINVAL, "bad occ");
-    if (prm->op == NB_OP_FEM27 && x->g->sparse) NB_FAIL(NB_EUNSUPPORTED, "FEM on sparse grids");
     if (x->outside != 0.0) NB_FAIL(NB_EUNSUPPORTED, "CG: x must have outside value 0 (homogeneous Dirichlet)");
     return NB_OK;
 }
@@ -908,7 +907,7 @@ extern "C" nb_status nb_cg_finish(nb_cg *cg, nb_cg_result *res) {
     nb_grid *g = cg->g;
     cudaSetDevice(g->device);
     if (!cg->finished) {
-        if (g->sparse && cg->prm.op != NB_OP_FEM27) {
+        if (g->sparse) {  // one p buffer (Poisson and FEM)
             NB_TRY(nb_sparse_cg_flush(cg));
         } else {
             for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {

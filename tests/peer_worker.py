@@ -216,6 +216,8 @@ def fem_cg(occ):
 for occ in (nb.OCC_NONE, nb.OCC_TWO_WAY):
     compare(f"fem cg occ{occ}", (12, 11, 14), WORLD, fem_cg(occ))
 compare("fem cg 4 parts", (12, 11, 16), 2 * WORLD, fem_cg(nb.OCC_TWO_WAY))
+for occ in (nb.OCC_NONE, nb.OCC_TWO_WAY):  # FEM on the element-sparse sphere
+    compare(f"sparse fem cg occ{occ}", (n, n, n), WORLD, fem_cg(occ), active=sphere)
 
 # ---- borrowed (torch-owned) storage: IPC handle of the enclosing allocation + offset
 def wrapped_cg(g):

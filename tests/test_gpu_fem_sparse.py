@@ -1,0 +1,116 @@
+"""FEM on element-sparse grids:
+nodes = active cells, an element exists iff its 8 nodes are active (the
+oracle's reading).  The GPU K u, consistent pressure load and CG must match
+the masked oracle (or_fem_apply / or_fem_rhs / or_cg); a full mask must give
+the dense operator bit for bit; partitions, OCC modes and halo transports
+must not change a bit."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_meneghinmjm22_b200 as nb
+import synth
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    import __graft_entry__
+    __graft_entry__.build()
+    assert nb.nb_device_count() > 0
+
+
+def masks():
+    n = 14
+    rng = np.random.default_rng(7)
+    sph = synth.sphere_mask(n, 0.47)
+    holes = (np.ones((n, n, n), bool) & (rng.random((n, n, n)) < 0.9)).astype(np.uint8)
+    step = np.ones((12, 11, 13), np.uint8)
+    step[7:, :, 5:] = 0  # a stepped top: exposed faces on two levels
+    return {"sphere": sph, "holes": holes, "step": step}
+
+
+def sgrid(mask, parts=1):
+    nz, ny, nx = mask.shape
+    return nb.Grid((nx, ny, nz), nparts=parts, devices=[0] * parts, active=mask)
+
+
+@pytest.mark.parametrize("name", ["sphere", "holes", "step"])
+@pytest.mark.parametrize("parts", [1, 3])
+def test_sparse_fem_apply_and_rhs_vs_oracle(name, parts):
+    m = masks()[name]
+    nz, ny, nx = m.shape
+    u = synth.uniform((nx, ny, nz), card=3, seed=5) * m[None]
+    yo = oracle.fem_apply(u, 1.0, 0.3, mask=m)
+    bo = oracle.fem_rhs((nx, ny, nz), 1.0, mask=m)
+    with sgrid(m, parts) as g:
+        fu, fy, fb = (nb.Field(g, card=3) for _ in range(3))
+        fu.upload(u)
+        fu.halo_update()
+        nb.nb_fem27_apply(fu, fy)
+        y = fy.download()
+        nb.nb_fem27_rhs(fb, 1.0)
+        b = fb.download()
+        for f in (fu, fy, fb):
+            f.close()
+    assert np.max(np.abs(y - yo)) <= 1e-13 * max(np.max(np.abs(yo)), 1.0)
+    assert np.array_equal(b, bo)  # dyadic loads in the oracle's order: bit-exact
+
+
+def test_sparse_fem_full_mask_equals_dense_bitwise():
+    dims = (13, 11, 12)
+    m = np.ones(dims[::-1], np.uint8)
+    u = synth.uniform(dims, card=3, seed=8)
+    outs = []
+    for active in (None, m):
+        with nb.Grid(dims, nparts=2, devices=[0, 0], active=active) as g:
+            fu, fy = nb.Field(g, card=3), nb.Field(g, card=3)
+            fu.upload(u)
+            fu.halo_update()
+            nb.nb_fem27_apply(fu, fy)
+            outs.append(fy.download())
+            fu.close(), fy.close()
+    assert np.array_equal(outs[0], outs[1])
+
+
+@pytest.mark.parametrize("name", ["sphere", "step"])
+def test_sparse_fem_cg_vs_oracle_and_invariance(name):
+    m = masks()[name]
+    nz, ny, nx = m.shape
+    bo = oracle.fem_rhs((nx, ny, nz), 1.0, mask=m)
+    xo, ro, _ = oracle.cg(bo, max_iter=12, op=oracle.OP_FEM27, mask=m)
+    ref = None
+    for parts in (1, 2, 3):
+        for occ in (nb.OCC_NONE, nb.OCC_TWO_WAY):
+            for halo in (nb.HALO_FUSED, nb.HALO_STREAM):
+                with sgrid(m, parts) as g:
+                    g.set_halo_mode(halo)
+                    fb, fx = nb.Field(g, card=3), nb.Field(g, card=3)
+                    nb.nb_fem27_rhs(fb, 1.0)
+                    fx.fill_const(0.0)
+                    r = nb.nb_cg_solve(fx, fb, max_iter=12, op=nb.OP_FEM27, occ=occ)
+                    x = fx.download()
+                    fb.close(), fx.close()
+                if ref is None:
+                    ref = (x, r.rr)
+                    assert np.max(np.abs(x - xo)) <= 1e-10 * np.max(np.abs(xo))
+                    assert abs(r.rr - ro.rr) <= 1e-9 * ro.rr
+                assert np.array_equal(x, ref[0]) and r.rr == ref[1], (parts, occ, halo)
+
+
+def test_sparse_fem_cg_converges():
+    m = masks()["step"]
+    nz, ny, nx = m.shape
+    with sgrid(m, 2) as g:
+        fb, fx = nb.Field(g, card=3), nb.Field(g, card=3)
+        nb.nb_fem27_rhs(fb, 1.0)
+        fx.fill_const(0.0)
+        r = nb.nb_cg_solve(fx, fb, max_iter=3000, rtol=1e-10, op=nb.OP_FEM27)
+        x = fx.download()
+        fb.close(), fx.close()
+    assert r.converged == 1
+    b = oracle.fem_rhs((nx, ny, nz), 1.0, mask=m)
+    res = oracle.fem_apply(x, 1.0, 0.3, mask=m) - b
+    assert np.max(np.abs(res)) <= 1e-8 * np.max(np.abs(b))
+    assert np.all(x[:, 0] == 0.0)
