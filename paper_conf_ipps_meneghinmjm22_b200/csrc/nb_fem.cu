@@ -1432,8 +1432,11 @@ struct SpFemArgs {
     const CgScal *sc;
 };
 
+#ifndef NB_SPF_MINB
+#define NB_SPF_MINB 8  // 32 registers: 3.04 ms per K p pass at 384^3 (6: 3.19, unbounded: 3.83)
+#endif
 template <int KIND>  // 0: y = K u; 1: q = K u, <u, q>; 2: y = b - K u, <y, y>
-__global__ void __launch_bounds__(256) k_sp_fem(SpFemArgs A) {
+__global__ void __launch_bounds__(256, NB_SPF_MINB) k_sp_fem(SpFemArgs A) {
     __shared__ double sw[3][8];
     const int t = threadIdx.x;
     const int e = __ldg(A.seg + A.seg0 + blockIdx.x);
