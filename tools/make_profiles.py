@@ -17,7 +17,8 @@ GO = os.path.join(ROOT, "gpurun_out")
 os.makedirs(OUT, exist_ok=True)
 
 # kernel label (the name bench.py / nb_profile_read use) from the ncu name
-LABELS = [("k_cgA_tma", "k_msr_cgA"), ("k_cgB_tma", "k_cg_B"), ("k_msr_fast<1, 1>", "k_msr_cgA"),
+LABELS = [("k_sp_runs<4>", "k_sp_cg_q"), ("k_sp_runs<2>", "k_sp_cg_init"), ("k_sp_fem<1>", "k_sp_fem_q"),
+          ("k_sp_fem<0>", "k_sp_fem_apply"), ("k_sp_fem<2>", "k_sp_fem_init"), ("k_cgA_tma", "k_msr_cgA"), ("k_cgB_tma", "k_cg_B"), ("k_msr_fast<1, 1>", "k_msr_cgA"),
           ("k_msr_fast<0", "k_msr_c1"), ("MsrOp<1, 1, 1>", "k_msr_cgA"), ("MsrOp<0,", "k_msr_c1"),
           ("CgBOp", "k_cg_B"), ("CgInitOp", "k_cg_init"), ("Lap7Op", "k_laplace7"), ("k_map_u", "k_map_u"),
           ("k_lbm_d3q19", "k_lbm_d3q19"), ("k_finalize", "k_finalize"), ("k_sp<3>", "k_sp_cg_map"),

@@ -53,4 +53,17 @@ if "fem" in what:
     cg.close()
     b.close(), x.close()
     g.close()
+if "spfem" in what:  # FEM on an element-sparse sphere
+    import synth
+    nf = min(n, 384)
+    g = nb.Grid((nf, nf, nf), active=synth.sphere_mask(nf))
+    b, x = nb.Field(g, card=3), nb.Field(g, card=3)
+    nb.nb_fem27_rhs(b, 1.0)
+    x.fill_const(0.0)
+    cg = nb.CG(x, b, op=nb.OP_FEM27)
+    cg.iterate(2)
+    cg.finish()
+    cg.close()
+    b.close(), x.close()
+    g.close()
 print("prof driver done")

@@ -16,8 +16,8 @@ timeout 900 ncu --set full --clock-control none --import-source on \
     -k regex:"k_lbm_d3q19" -s 1 -c 2 -o gpurun_out/prof_${R}_lbm \
     python tools/prof_driver.py 512 lbm > gpurun_out/prof_${R}_lbm.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on \
-    -k regex:"^k_sp$|k_fem_tma|k_fem_faces|k_fem_surface|k_fem_xface|k_fem_map|k_fem_r$" -c 28 -o gpurun_out/prof_${R}_sparse_fem \
-    python tools/prof_driver.py 512 sparse,fem > gpurun_out/prof_${R}_sparse_fem.log 2>&1
+    -k regex:"^k_sp$|k_sp_runs|k_sp_fem|k_fem_tma|k_fem_faces|k_fem_surface|k_fem_xface|k_fem_map|k_fem_r$" -c 60 -o gpurun_out/prof_${R}_sparse_fem \
+    python tools/prof_driver.py 512 sparse,fem,spfem > gpurun_out/prof_${R}_sparse_fem.log 2>&1
 # raw pages exported here; the reports themselves stay on the box (gpurun
 # copies back at most 64 MiB)
 for rep in gpurun_out/prof_${R}_*.ncu-rep; do
