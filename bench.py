@@ -53,7 +53,11 @@ class ClockSampler:
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
     def __init__(self, gpu: int):
-        self.gpu, self.rows, self.proc = gpu, [], None
+        self.gpu, self.rows, self.proc, self.start = gpu, [], None, 0
+
+    def mark(self):
+        """Samples from here on belong to the timed region."""
+        self.start = len(self.rows)
 
     def __enter__(self):
         try:
@@ -80,11 +84,12 @@ class ClockSampler:
                 self.proc.kill()
 
     def summary(self):
-        sm = [float(r[1]) for r in self.rows if len(r) > 8 and r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in self.rows if len(r) > 8 and r[2].replace(".", "").isdigit()]
+        rows = self.rows[self.start:] or self.rows[-1:]  # the timed region (at least the last sample)
+        sm = [float(r[1]) for r in rows if len(r) > 8 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if len(r) > 8 and r[2].replace(".", "").isdigit()]
         reasons = set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in self.rows:
+        for r in rows:
             if len(r) > 8:
                 for nm, v in zip(names, r[5:9]):
                     if v.strip().lower() == "active":
@@ -138,12 +143,19 @@ def max_over_ranks(world, v):
 
 
 def timed(world, stream, fn, gpu):
-    """Barrier + sync on both sides; CUDA events on the launching stream."""
+    """Barrier + sync on both sides; CUDA events on the launching stream.  The
+    clock sampler (nvidia-smi) is started first and given time to initialise
+    (NVML start-up holds driver locks that would otherwise stall this
+    process's enqueues inside the timed region)."""
     import torch
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    barrier(world)
-    torch.cuda.synchronize()
     with ClockSampler(gpu) as clk:
+        t0 = time.perf_counter()
+        while not clk.rows and time.perf_counter() - t0 < 3.0:
+            time.sleep(0.02)
+        barrier(world)
+        torch.cuda.synchronize()
+        clk.mark()
         ev0.record(stream)
         fn()
         ev1.record(stream)

@@ -34,10 +34,10 @@ nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v);
 bool nb_tma_enabled();
 nb_status nb_cgB_tma(nb_grid *g, const PGeo &geo, const double *p, double *r, int zb, int ze, const CgScal *sc);
 nb_status nb_c1_tma(nb_grid *g, const PGeo &geo, const double *xin, const double *yin, double *xout, double *yout,
-                    double a, bool domap, int zb, int ze);
+                    double a, bool domap, int zb, int ze, int zhi = -1);
 nb_status nb_c1_finalize_all(nb_grid *g, int iters);
 nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x, bool domap,
-                     int zb, int ze, const CgScal *sc);
+                     int zb, int ze, const CgScal *sc, int zhi = -1);
 
 static inline int64_t dcs(const nb_field *f, int p) { return nb_cstride(f, p); }
 
@@ -349,7 +349,9 @@ __global__ void __launch_bounds__(DOT_TX *DOT_TY) k_msr_fast(MsrArgs A, PGeo g, 
 // (rem_lo: lower neighbour's high halo, rem_hi: upper neighbour's low halo)
 // — the halo transfer fused into the producing kernel.
 template <int MODE>
-__global__ void __launch_bounds__(256) k_map_u(MsrArgs A, PGeo g, int zb, int ze, double *rem_lo,
+// planes [zb, ze), or with zhi >= 0 the pair {zb, zhi} (one per blockIdx.z):
+// both boundary planes of a slab in one launch
+__global__ void __launch_bounds__(256) k_map_u(MsrArgs A, PGeo g, int zb, int ze, int zhi, double *rem_lo,
                                                double *rem_hi) {
     if (A.sc && A.sc->status != 0) return;
     double m = A.m, ap = A.ap;
@@ -361,7 +363,11 @@ __global__ void __launch_bounds__(256) k_map_u(MsrArgs A, PGeo g, int zb, int ze
     }
     const int xi = blockIdx.x * blockDim.x + threadIdx.x, yi = blockIdx.y;
     if (xi >= g.nx) return;
-    for (int z = zb + blockIdx.z; z < ze; z += gridDim.z) {
+    if (zhi >= 0) {
+        zb = blockIdx.z ? zhi : zb;
+        ze = zb + 1;
+    }
+    for (int z = zb + (zhi >= 0 ? 0 : (int)blockIdx.z); z < ze; z += gridDim.z) {
         const int64_t row = (int64_t)yi * g.pitch + xi;
         const int64_t ic = row + (int64_t)(z + 1) * g.ps;
         double vc = A.v[ic];
@@ -457,33 +463,47 @@ static double *pl(const nb_field *f, int p, int zl) {
 
 // launch k_map_u on the planes of `planes` (or all when all==true), with
 // fused stores into neighbour halos of `ufield` for local neighbours
-static nb_status launch_map_u(nb_grid *g, int mode, int p, MsrArgs A, const nb_field *ufield, int zb, int ze) {
+static nb_status launch_map_u(nb_grid *g, int mode, int p, MsrArgs A, const nb_field *ufield, int zb, int ze,
+                              int zhi = -1) {
     const NbPart &q = g->parts[p];
     PGeo geo = pgeo(ufield, p);
     double *rem_lo = nullptr, *rem_hi = nullptr;
     if (!nb_halo_on_stream(g)) {  // fused halo: store straight into the neighbour
         if (zb == 0 && nb_reachable(ufield, q.lo)) rem_lo = pl(ufield, q.lo, g->parts[q.lo].nz());
-        if (ze == q.nz() && nb_reachable(ufield, q.hi)) rem_hi = pl(ufield, q.hi, -1);
+        if ((ze == q.nz() || zhi == q.nz() - 1) && nb_reachable(ufield, q.hi)) rem_hi = pl(ufield, q.hi, -1);
     }
-    dim3 blk(128), grd((g->nx + 127) / 128, g->ny, std::min(ze - zb, 64));
+    dim3 blk(128), grd((g->nx + 127) / 128, g->ny, zhi >= 0 ? 2 : std::min(ze - zb, 64));
     LaunchScope ls(g, g->cs, "k_map_u");
     if (mode == MSR_C1)
-        k_map_u<MSR_C1><<<grd, blk, 0, g->cs>>>(A, geo, zb, ze, rem_lo, rem_hi);
+        k_map_u<MSR_C1><<<grd, blk, 0, g->cs>>>(A, geo, zb, ze, zhi, rem_lo, rem_hi);
     else
-        k_map_u<MSR_CG><<<grd, blk, 0, g->cs>>>(A, geo, zb, ze, rem_lo, rem_hi);
+        k_map_u<MSR_CG><<<grd, blk, 0, g->cs>>>(A, geo, zb, ze, zhi, rem_lo, rem_hi);
     return nb_launch_check("k_map_u");
 }
 
+// the boundary planes of partition p as one (zb, zhi) launch pair when there
+// are two (zhi = -1: a single plane zb)
+static std::pair<int, int> bnd_pair(const nb_grid *g, int p) {
+    auto b = bnd_planes(g, p);
+    if (b.empty()) return {-1, -1};
+    if (b.size() == 1) return {b[0], -1};
+    return {b[0], b[1]};
+}
+
 template <int MODE, bool RC, bool DM>
-static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int zb, int ze) {
+static nb_status launch_msr(nb_grid *g, int p, MsrArgs A, const nb_field *f, int zb, int ze, int zhi = -1) {
     if (ze <= zb) return NB_OK;
     const char *name = MODE == MSR_C1 ? "k_msr_c1" : "k_msr_cgA";
     if (MODE == MSR_CG && RC && ZR_MAP == 1 && nb_tma_enabled())  // TMA-staged phase A
-        return nb_cgA_tma(g, pgeo(f, p), A.w, A.v, A.u, A.xs, DM, zb, ze, A.sc);
+        return nb_cgA_tma(g, pgeo(f, p), A.w, A.v, A.u, A.xs, DM, zb, ze, A.sc, zhi);
     // TMA-staged C1 chain: large grids only (the 64^3 C1 config lives in L2,
     // where the register/L1 kernel has lower latency per launch)
     if (MODE == MSR_C1 && RC && ZR_MAP == 1 && nb_tma_enabled() && (int64_t)g->nx * g->ny * g->nz >= (1 << 21))
-        return nb_c1_tma(g, pgeo(f, p), A.w, A.v, A.u, A.out, A.m, DM, zb, ze);
+        return nb_c1_tma(g, pgeo(f, p), A.w, A.v, A.u, A.out, A.m, DM, zb, ze, zhi);
+    if (zhi >= 0) {  // the other kernels take plane ranges: the pair as two launches
+        NB_TRY((launch_msr<MODE, RC, DM>(g, p, A, f, zb, ze)));
+        return launch_msr<MODE, RC, DM>(g, p, A, f, zhi, zhi + 1);
+    }
     if (RC && ZR_MAP == 1 && !getenv("NB_GENERIC_MSR")) {
         // specialised recompute kernel (same arithmetic and dot order); planes
         // per CTA halved while the launch has fewer than two CTAs per SM (the
@@ -566,7 +586,8 @@ static nb_status msr_step_fields(nb_grid *g, nb_occ occ, MsrFields F, double m, 
         if (occ == NB_OCC_NONE || occ == NB_OCC_STANDARD) {
             NB_TRY(launch_map_u(g, MODE, p, args(p), F.u, 0, q.nz()));
         } else {
-            for (int z : bnd_planes(g, p)) NB_TRY(launch_map_u(g, MODE, p, args(p), F.u, z, z + 1));
+            const auto bp = bnd_pair(g, p);  // both boundary planes in one launch
+            if (bp.first >= 0) NB_TRY(launch_map_u(g, MODE, p, args(p), F.u, bp.first, bp.first + 1, bp.second));
         }
     }
     NB_TRY(dist_halo_mark(g, hs));
@@ -587,12 +608,12 @@ static nb_status msr_step_fields(nb_grid *g, nb_occ occ, MsrFields F, double m, 
     NB_TRY(dist_halo_begin(g, F.u, hs));
     NB_TRY(dist_halo_wait(g, hs));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
-        for (int z : bnd_planes(g, p)) {
-            if (occ == NB_OCC_STANDARD)
-                NB_TRY((launch_msr<MODE, false, false>(g, p, args(p), F.u, z, z + 1)));
-            else
-                NB_TRY((launch_msr<MODE, true, false>(g, p, args(p), F.u, z, z + 1)));
-        }
+        const auto bp = bnd_pair(g, p);  // both boundary planes in one launch where the kernel takes pairs
+        if (bp.first < 0) continue;
+        if (occ == NB_OCC_STANDARD)
+            NB_TRY((launch_msr<MODE, false, false>(g, p, args(p), F.u, bp.first, bp.first + 1, bp.second)));
+        else
+            NB_TRY((launch_msr<MODE, true, false>(g, p, args(p), F.u, bp.first, bp.first + 1, bp.second)));
     }
     return NB_OK;
 }

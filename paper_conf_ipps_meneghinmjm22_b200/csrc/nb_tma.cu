@@ -76,8 +76,8 @@ template <bool DOMAP, bool C1, class G>
 __global__ void __launch_bounds__(G::NT, G::MINB_A)
     k_cgA_tma(const __grid_constant__ CUtensorMap m_r, const __grid_constant__ CUtensorMap m_po,
               const __grid_constant__ CUtensorMap m_pn, const __grid_constant__ CUtensorMap m_x, double *pn, double *xs,
-              PGeo g, int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_x, int zc, double c1_a = 0.0,
-              double *c1_out = nullptr) {
+              PGeo g, int zb, int ze, const CgScal *sc, double *tp, int T, int tiles_x, int zc, double c1_a,
+              double *c1_out, int zhi) {
     constexpr int NTX = G::TW / DOT_TX, NTY = G::TH / DOT_TY, NSTAGE = G::NST;
     extern __shared__ __align__(128) double tsm[];
     __shared__ __align__(8) uint64_t bar[NSTAGE];
@@ -91,7 +91,10 @@ __global__ void __launch_bounds__(G::NT, G::MINB_A)
     const int x0 = blockIdx.x * G::TW, y0 = blockIdx.y * G::TH;
     const int xi = x0 + tx * DOT_TX + lane, yi = y0 + w;
     const int cx = tx * DOT_TX + lane + 2;  // box column of the own cell
-    const int zs = zb + blockIdx.z * zc, zend = min(ze, zs + zc);  // zc <= TZC planes per CTA
+    // planes [zb, ze) in chunks of zc, or with zhi >= 0 the pair of single
+    // planes {zb, zhi} (both boundary planes of a slab in one launch)
+    const int zs = zhi >= 0 ? (blockIdx.z ? zhi : zb) : zb + blockIdx.z * zc;
+    const int zend = zhi >= 0 ? zs + 1 : min(ze, zs + zc);  // zc <= TZC planes per CTA
     const int nzl = g.nzl;
     const bool valid = xi < g.nx && yi < g.ny;
     auto halo = [&](int zl) { return zl < 0 || zl >= nzl; };
@@ -415,7 +418,8 @@ static void tma_smem_attr(F *f, int bytes) {
 
 template <bool DOMAP, bool C1, class G>
 static nb_status launch_cgA(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x,
-                            int zb, int ze, const CgScal *sc, double c1_a, double *c1_out, const char *label) {
+                            int zb, int ze, const CgScal *sc, double c1_a, double *c1_out, const char *label,
+                            int zhi = -1) {
     CUtensorMap mr, mpo, mpn, mx;
     NB_TRY(tmap_box(r, geo, G::BXW, G::BYH, &mr));
     NB_TRY(tmap_box(po, geo, G::BXW, G::BYH, &mpo));
@@ -425,28 +429,31 @@ static nb_status launch_cgA(nb_grid *g, const PGeo &geo, const double *r, const 
     const int zc = tma_zc(((g->tiles_x + NTX - 1) / NTX) * ((g->tiles_y + NTY - 1) / NTY), ze - zb, G::MINB_A);
     const int smem = G::NST * G::SA * 8;
     tma_smem_attr(k_cgA_tma<DOMAP, C1, G>, smem);
-    dim3 blk(G::NT), grd((g->tiles_x + NTX - 1) / NTX, (g->tiles_y + NTY - 1) / NTY, (ze - zb + zc - 1) / zc);
+    dim3 blk(G::NT),
+        grd((g->tiles_x + NTX - 1) / NTX, (g->tiles_y + NTY - 1) / NTY, zhi >= 0 ? 2 : (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, label);
     k_cgA_tma<DOMAP, C1, G><<<grd, blk, smem, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T,
-                                                       g->tiles_x, zc, c1_a, c1_out);
+                                                       g->tiles_x, zc, c1_a, c1_out, zhi);
     return nb_launch_check(label);
 }
 
 // CG phase A on planes [zb, ze) of a partition (r, p_old, p_new, x buffers)
 nb_status nb_cgA_tma(nb_grid *g, const PGeo &geo, const double *r, const double *po, double *pn, double *x, bool domap,
-                     int zb, int ze, const CgScal *sc) {
+                     int zb, int ze, const CgScal *sc, int zhi) {
     if (ze <= zb) return NB_OK;
-    return domap ? launch_cgA<true, false, CgGeo>(g, geo, r, po, pn, x, zb, ze, sc, 0.0, nullptr, "k_msr_cgA")
-                 : launch_cgA<false, false, CgGeo>(g, geo, r, po, pn, x, zb, ze, sc, 0.0, nullptr, "k_msr_cgA");
+    return domap ? launch_cgA<true, false, CgGeo>(g, geo, r, po, pn, x, zb, ze, sc, 0.0, nullptr, "k_msr_cgA", zhi)
+                 : launch_cgA<false, false, CgGeo>(g, geo, r, po, pn, x, zb, ze, sc, 0.0, nullptr, "k_msr_cgA", zhi);
 }
 
 // C1 map-stencil-reduce on planes [zb, ze): x_out = x_in + a y_in (stored
 // when domap), y_out = L(x_out), per-plane tile partials of x_out * y_out
 nb_status nb_c1_tma(nb_grid *g, const PGeo &geo, const double *xin, const double *yin, double *xout, double *yout,
-                    double a, bool domap, int zb, int ze) {
+                    double a, bool domap, int zb, int ze, int zhi) {
     if (ze <= zb) return NB_OK;
-    return domap ? launch_cgA<true, true, CgGeo>(g, geo, xin, yin, xout, nullptr, zb, ze, nullptr, a, yout, "k_msr_c1")
-                 : launch_cgA<false, true, CgGeo>(g, geo, xin, yin, xout, nullptr, zb, ze, nullptr, a, yout, "k_msr_c1");
+    return domap ? launch_cgA<true, true, CgGeo>(g, geo, xin, yin, xout, nullptr, zb, ze, nullptr, a, yout, "k_msr_c1",
+                                                 zhi)
+                 : launch_cgA<false, true, CgGeo>(g, geo, xin, yin, xout, nullptr, zb, ze, nullptr, a, yout, "k_msr_c1",
+                                                  zhi);
 }
 
 // CG phase B on planes [zb, ze) of a partition (stored p_new, r)
