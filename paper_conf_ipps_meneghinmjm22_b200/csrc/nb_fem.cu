@@ -1322,6 +1322,9 @@ static inline int64_t fcs(const nb_field *f, int p) { return nb_cstride(f, p); }
 // surface nodes of the interior planes while the halo is in flight)
 enum { FEM_SURF = 1, FEM_BULK = 2, FEM_ALL = 3 };
 
+#ifndef NB_FEM_ZC
+#define NB_FEM_ZC 32  // planes per CTA of the TMA z-march
+#endif
 template <int K>
 static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int zb, int ze, const char *name,
                             int what = FEM_ALL, int zhi = -1) {
@@ -1336,7 +1339,7 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
         k_fem<K><<<grd, blk, 0, g->cs>>>(A, geo, zb, g->tp, g->T);
     } else if (!variant && nb_tma_enabled()) {
         using Cfg = FemTmaCfg<K>;
-        constexpr int ZC = 32, NR = Cfg::NR;
+        constexpr int ZC = NB_FEM_ZC, NR = Cfg::NR;
         FemMaps M;
         if constexpr (K == FEM_CG_A) {
             for (int c = 0; c < 3; ++c) {

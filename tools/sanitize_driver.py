@@ -84,4 +84,74 @@ with nb.Grid((96, 40, 1)) as g:
     nb.nb_d2q9_init(a, 1.0, 0.05, 0.0)
     nb.nb_d2q9_step(a, b, 1.6, 0.05, (24, 20, 5), 3)
     a.close(), b.close()
+# round-2 additions: sparse q pass on the segment-indexed table, sparse FEM
+# (tables, K u, load, CG with OCC on the halo stream), field layouts (AoS /
+# plane-major LBM, dots, halo updates), Skeleton Listing 3 CG + LBM, OCC on
+# sparse CG, CopyBatch with > 32 descriptors
+m = synth.sphere_mask(18, 0.47)
+with nb.Grid((18, 18, 18), nparts=3, devices=[0, 0, 0], active=m) as g:
+    g.set_halo_mode(nb.HALO_STREAM)
+    b, x = nb.Field(g, card=3), nb.Field(g, card=3)
+    nb.nb_fem27_rhs(b, 1.0)
+    x.fill_const(0.0)
+    nb.nb_cg_solve(x, b, max_iter=3, op=nb.OP_FEM27, occ=nb.OCC_TWO_WAY)
+    x.halo_update()
+    nb.nb_fem27_apply(x, b)
+    p, q = nb.Field(g), nb.Field(g)
+    p.fill_uniform(seed=2)
+    q.fill_const(0.0)
+    nb.nb_cg_solve(q, p, max_iter=3, occ=nb.OCC_TWO_WAY)
+    for f in (b, x, p, q):
+        f.close()
+dims = (24, 20, 18)
+for layout in (nb.SOA_PLANE, nb.AOS):
+    with nb.Grid(dims, nparts=3, devices=[0, 0, 0]) as g:
+        a, c = nb.Field(g, "f32", 19, layout=layout), nb.Field(g, "f32", 19, layout=layout)
+        nb.nb_lbm_init(a, 1.0, (0, 0, 0))
+        a, c = nb.nb_lbm_step(a, c, 1.1, 3)
+        rho, u = nb.Field(g, "f32", 1), nb.Field(g, "f32", 3, layout=layout)
+        nb.nb_lbm_macroscopic(a, rho, u)
+        h = synth.uniform(dims, card=3, seed=3)
+        v, w = nb.Field(g, card=3, layout=layout), nb.Field(g, card=3, layout=layout)
+        v.upload(h)
+        w.upload(h)
+        v.halo_update()
+        nb.nb_axpby(0.5, v, 2.0, w)
+        nb.nb_dot(v, w)
+        v.download()
+        for f in (a, c, rho, u, v, w):
+            f.close()
+with nb.Grid((30, 26, 24), nparts=2, devices=[0, 0]) as g:
+    b, x, r, p, q = (nb.Field(g) for _ in range(5))
+    b.fill_uniform(seed=8)
+    for f in (x, p, q):
+        f.fill_const(0.0)
+    nb.nb_axpby(1.0, b, 0.0, r)
+    with nb.Skeleton(g, nb.OCC_TWO_WAY) as s0:
+        s0.dot(r, r, 0)
+        s0.set_scalar(3, 0.0)
+        s0.run()
+    with nb.Skeleton(g, nb.OCC_TWO_WAY) as sk:
+        sk.axpby_s(1.0, -1, r, 1.0, 3, p)
+        sk.poisson(p, q)
+        sk.dot(p, q, 1)
+        sk.scalar(nb.SC_DIV, 0, 1, 2)
+        sk.axpby_s(1.0, 2, p, 1.0, -1, x)
+        sk.axpby_s(-1.0, 2, q, 1.0, -1, r)
+        sk.dot(r, r, 4)
+        sk.scalar(nb.SC_DIV, 4, 0, 3)
+        sk.scalar(nb.SC_COPY, 4, 0, 0)
+        sk.run()
+        sk.run()
+    a, c = nb.Field(g, "f32", 19), nb.Field(g, "f32", 19)
+    nb.nb_lbm_init(a, 1.0, (0, 0, 0))
+    with nb.Skeleton(g, nb.OCC_STANDARD) as sk:
+        sk.lbm(a, c, 1.0)
+        sk.lbm(c, a, 1.0)
+        sk.run()
+    f19 = nb.Field(g, card=19)
+    f19.fill_uniform(seed=1)
+    f19.halo_update()  # 38 plane copies in one batch
+    for f in (b, x, r, p, q, a, c, f19):
+        f.close()
 print("sanitize driver done")
