@@ -586,6 +586,9 @@ def bench_sparse_run(n, steps, warmup, world, local):
                                    f"{nact / n ** 3:.2%}), 7-point CG fp64 (configs[3])",
                        "schedule": f"3 passes, {per_cell} B/active cell/iter incl. the 16 B segment-indexed neighbour table"},
             "hbm_gbs": per_cell * nact * steps / t / 1e9, "hbm_frac": per_cell * nact * steps / t / 1e9 / hbm,
+            # 96 B/active/iter is the minimum of a 24-B
+            # connectivity schedule; the iteration time against it
+            "survey_96B_frac": 96 * nact * steps / t / 1e9 / hbm / world,
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm, "unit": "GB/s",
                          "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": ncu_traffic(dom),
                          "per_rank": world > 1, "local_active_cells": local_act,
