@@ -236,3 +236,68 @@ def test_fem_rhs_virtual_work_on_stepped_mask():
     }
     for name, (v, fn) in tests.items():
         assert abs(float(np.sum(b[2] * v)) - p * integral(fn)) < 1e-12, name
+
+
+# ---- FEM on element-sparse domains (
+# DESIGN reading 10: an element exists iff its 8 nodes are active) ----------
+def _masked_dense_K(mask, ke):
+    """K assembled here (numpy scatter, independent of the oracle's element
+    loop) over the elements whose 8 nodes are all active."""
+    nz, ny, nx = mask.shape
+    N = nx * ny * nz
+    K = np.zeros((3 * N, 3 * N))
+    for ez in range(nz - 1):
+        for ey in range(ny - 1):
+            for ex in range(nx - 1):
+                if not mask[ez:ez + 2, ey:ey + 2, ex:ex + 2].all():
+                    continue
+                dofs = []
+                for a in range(8):
+                    i, j, k = ex + (a & 1), ey + ((a >> 1) & 1), ez + ((a >> 2) & 1)
+                    node = i + nx * (j + ny * k)
+                    dofs += [d * N + node for d in range(3)]
+                K[np.ix_(dofs, dofs)] += ke
+    return K
+
+
+def test_fem_masked_apply_brute_force_and_rigid_modes():
+    """The masked matrix-free K u equals the brute-force assembly over the
+    existing elements (with and without the Dirichlet plane), and on a mask
+    with holes rigid translations / a rotation give K u = 0 without
+    Dirichlet; nodes in no element get y = 0."""
+    rng = np.random.default_rng(11)
+    nz, ny, nx = 5, 4, 6
+    mask = (rng.random((nz, ny, nx)) < 0.8).astype(np.uint8)
+    mask[:, 1:3, 1:4] = 1  # a solid core so that elements exist
+    ke = oracle.fem_ke(E, NU)
+    K = _masked_dense_K(mask, ke)
+    N = nx * ny * nz
+    u = synth.uniform((nx, ny, nz), card=3, seed=4) * mask[None]
+    y = oracle.fem_apply(u, E, NU, mask=mask, dirichlet_z0=False)
+    assert np.max(np.abs(y.ravel() - K @ u.ravel())) < 1e-14
+    # Dirichlet z = 0: identity rows / columns on the ACTIVE z = 0 nodes
+    fixed = np.zeros(3 * N, dtype=bool)
+    act0 = np.zeros((nz, ny, nx), bool)
+    act0[0] = mask[0].astype(bool)
+    for d in range(3):
+        fixed[d * N:(d + 1) * N] = act0.ravel()
+    Kd = K.copy()
+    Kd[fixed, :] = 0
+    Kd[:, fixed] = 0
+    Kd[fixed, fixed] = 1
+    yd = oracle.fem_apply(u, E, NU, mask=mask, dirichlet_z0=True)
+    assert np.max(np.abs(yd.ravel() - Kd @ u.ravel())) < 1e-14
+    # rigid modes on the masked body (no Dirichlet)
+    Z, Y, X = np.meshgrid(np.arange(nz), np.arange(ny), np.arange(nx), indexing="ij")
+    for mode in (np.stack([np.ones_like(X), 0 * X, 0 * X]), np.stack([0 * X, np.ones_like(X), 0 * X]),
+                 np.stack([-Y, X, 0 * X])):
+        assert np.max(np.abs(oracle.fem_apply(mode.astype(float), E, NU, mask=mask, dirichlet_z0=False))) < 1e-13
+    # nodes in no existing element: y = 0
+    in_elem = np.zeros((nz, ny, nx), bool)
+    for ez in range(nz - 1):
+        for ey in range(ny - 1):
+            for ex in range(nx - 1):
+                if mask[ez:ez + 2, ey:ey + 2, ex:ex + 2].all():
+                    in_elem[ez:ez + 2, ey:ey + 2, ex:ex + 2] = True
+    lonely = ~in_elem
+    assert lonely.any() and np.all(y[:, lonely] == 0)
