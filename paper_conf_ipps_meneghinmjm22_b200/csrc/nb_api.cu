@@ -1062,6 +1062,7 @@ nb_status nb_halo_split_wait(nb_grid *g, HaloSync &hs) {
 }
 
 extern "C" nb_status nb_halo_update(nb_field *f) {
+    NB_RANGE("nb_halo_update");
     if (!f) NB_FAIL(NB_EINVAL, "nb_halo_update: NULL field");
     DeviceGuard dg(f->g->device);
     if (f->g->sparse) return nb_sparse_halo_update(f);
@@ -1341,6 +1342,7 @@ nb_status nb_dot_partials_view(const nb_field *x, const nb_field *y, nb_view v) 
 nb_status nb_dot_partials(const nb_field *x, const nb_field *y) { return nb_dot_partials_view(x, y, NB_VIEW_STANDARD); }
 
 extern "C" nb_status nb_dot(const nb_field *x, const nb_field *y, double *host_out) {
+    NB_RANGE("nb_dot");
     NB_TRY(check_pair(x, y));
     if (!host_out) NB_FAIL(NB_EINVAL, "nb_dot: host_out is NULL");
     nb_grid *g = x->g;

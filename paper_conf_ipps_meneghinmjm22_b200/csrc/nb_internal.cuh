@@ -13,6 +13,18 @@
 
 #include "nb.h"
 
+// NVTX ranges (header-only NVTX 3; free when no tool is attached): one per
+// kernel enqueue (LaunchScope) and one per public operation (NB_RANGE), so
+// ncu --nvtx / nsys timelines can attribute launches to library calls
+#include <nvtx3/nvToolsExt.h>
+struct NbRange {
+    explicit NbRange(const char *name) { nvtxRangePushA(name); }
+    ~NbRange() { nvtxRangePop(); }
+};
+#define NB_RANGE_CAT2(a, b) a##b
+#define NB_RANGE_CAT(a, b) NB_RANGE_CAT2(a, b)
+#define NB_RANGE(name) NbRange NB_RANGE_CAT(nb_range_, __LINE__)(name)
+
 // ---------------------------------------------------------------------------
 // error plumbing (no exception crosses the ABI)
 // ---------------------------------------------------------------------------
@@ -274,6 +286,7 @@ struct LaunchScope {
     const char *name;
     cudaEvent_t a = nullptr, b = nullptr;
     LaunchScope(nb_grid *g_, cudaStream_t s_, const char *n) : g(g_), s(s_), name(n) {
+        nvtxRangePushA(n);
         g->launches++;
         if (g->profiling) {
             cudaEventCreate(&a);
@@ -286,6 +299,7 @@ struct LaunchScope {
             cudaEventRecord(b, s);
             g->prof.push_back({name, a, b});
         }
+        nvtxRangePop();
     }
 };
 

@@ -442,6 +442,7 @@ nb_status nb_lbm_view(nb_field *fin, nb_field *fout, const nb_lbm_params *prm, n
 
 extern "C" nb_status nb_lbm_step(nb_field **pfin, nb_field **pfout, const nb_lbm_params *prm, int32_t nsteps,
                                  nb_occ occ) {
+    NB_RANGE("nb_lbm_step");
     if (!pfin || !pfout || !prm) NB_FAIL(NB_EINVAL, "nb_lbm_step: NULL argument");
     nb_field *fin = *pfin, *fout = *pfout;
     NB_TRY(lbm_check(fin));

@@ -692,6 +692,7 @@ static nb_status run_node(nb_skeleton *s, const Node &n, cudaStream_t st) {
 }
 
 extern "C" nb_status nb_skeleton_run(nb_skeleton *s) {
+    NB_RANGE("nb_skeleton_run");
     if (!s) NB_FAIL(NB_EINVAL, "NULL skeleton");
     NB_TRY(nb_skeleton_compile(s));
     nb_grid *g = s->g;

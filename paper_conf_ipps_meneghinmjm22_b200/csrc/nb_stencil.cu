@@ -623,6 +623,7 @@ static nb_status msr_step_fields(nb_grid *g, nb_occ occ, MsrFields F, double m, 
 // ===========================================================================
 extern "C" nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, int32_t iters, nb_occ occ,
                                            double *dots_out) {
+    NB_RANGE("nb_map_stencil_reduce");
     if (!x || !y || !dots_out) NB_FAIL(NB_EINVAL, "nb_map_stencil_reduce: NULL argument");
     if (x->g != y->g) NB_FAIL(NB_EMISMATCH, "fields belong to different grids");
     if (x->dt != NB_F64 || y->dt != NB_F64 || x->card != 1 || y->card != 1)
@@ -798,6 +799,7 @@ nb_status nb_sparse_cg_init(nb_cg *cg);        // nb_sparse.cu
 nb_status nb_sparse_cg_flush(nb_cg *cg);
 
 extern "C" nb_status nb_cg_create(nb_field *x, const nb_field *b, const nb_cg_params *prm, nb_cg **out) {
+    NB_RANGE("nb_cg_create");
     if (!out) NB_FAIL(NB_EINVAL, "nb_cg_create: out is NULL");
     *out = nullptr;
     NB_TRY(cg_check(x, b, prm));
@@ -903,6 +905,7 @@ static nb_status cg_run_chunks(nb_cg *cg, int32_t iters, bool launch) {
 }
 
 extern "C" nb_status nb_cg_iterate(nb_cg *cg, int32_t iters) {
+    NB_RANGE("nb_cg_iterate");
     if (!cg) NB_FAIL(NB_EINVAL, "nb_cg_iterate: NULL solver");
     if (cg->finished) NB_FAIL(NB_ESTATE, "nb_cg_iterate after nb_cg_finish");
     if (iters < 0) NB_FAIL(NB_EINVAL, "iters < 0");
