@@ -22,6 +22,8 @@
 #include <map>
 #include <mutex>
 #include <tuple>
+#include <queue>
+#include <vector>
 
 #include "nb_device.cuh"
 #include "nb_internal.cuh"
@@ -324,15 +326,41 @@ static int tma_zc(int ctas_per_plane, int nplanes, int ctas_per_sm) {
     static int forced = -1;
     if (forced < 0) forced = getenv("NB_CG_ZC") ? std::max(1, std::min(TZC, atoi(getenv("NB_CG_ZC")))) : 0;
     if (forced) return forced;
-    const int64_t cap = (int64_t)sm_count() * ctas_per_sm;
+    static std::mutex mu;
+    static std::map<std::tuple<int, int, int>, int> cache;
+    std::lock_guard<std::mutex> lk(mu);
+    const auto key = std::make_tuple(ctas_per_plane, nplanes, ctas_per_sm);
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
+    // every zc in [2, TZC]: CTAs are dispatched in launch order (the chunks
+    // of a plane range one after another, the last one possibly shorter)
+    // onto cap resident slots; a CTA of p planes costs p + H plane-times
+    // (H: the ring's two z-halo planes and the first load's latency).  The
+    // simulated makespan picks zc (non-powers of two cut the last wave's
+    // idle slots: 62 planes at 512 CTAs per plane take 13, not 16)
+    const int cap = std::max(1, sm_count() * ctas_per_sm);
     constexpr double H = 3.0;
     int best = TZC;
     double best_cost = 1e300;
-    for (int zc = TZC; zc >= 2; zc /= 2) {
-        const int64_t n = (int64_t)ctas_per_plane * ((nplanes + zc - 1) / zc);
-        const double cost = (double)((n + cap - 1) / cap) * (std::min(zc, nplanes) + H);
-        if (cost < best_cost - 1e-9) best_cost = cost, best = zc;
+    std::vector<double> slot;
+    static const bool pow2 = getenv("NB_CG_ZC_POW2") != nullptr;  // the round-1 search (powers of two)
+    for (int zc = TZC; zc >= 2; zc = pow2 ? zc / 2 : zc - 1) {
+        const int nchunk = (nplanes + zc - 1) / zc;
+        slot.assign(cap, 0.0);
+        std::priority_queue<double, std::vector<double>, std::greater<double>> free_at(slot.begin(), slot.end());
+        double end = 0.0;
+        for (int c = 0; c < nchunk; ++c) {
+            const double dur = std::min(zc, nplanes - c * zc) + H;
+            for (int k = 0; k < ctas_per_plane; ++k) {
+                const double t0 = free_at.top();
+                free_at.pop();
+                free_at.push(t0 + dur);
+                end = std::max(end, t0 + dur);
+            }
+        }
+        if (end < best_cost - 1e-9) best_cost = end, best = zc;
     }
+    cache[key] = best;
     return best;
 }
 
