@@ -1224,6 +1224,7 @@ __global__ void __launch_bounds__(RED_THREADS) k_finalize(const double *tp, int 
                                                           int slot) {
     __shared__ double sh[RED_THREADS];
     __shared__ int last;
+    pdl_wait();  // the producing kernel's tile partials (programmatic launch)
     int b = blockIdx.x;
     int c = b / zn, z = z0 + b % zn;
     int plane = c * NZ + z;
@@ -1276,8 +1277,8 @@ nb_status nb_reduce_finalize(nb_grid *g, int card, int mode, void *state, int sl
     bool dist = g->comm && g->comm->world > 1;
     if (!dist) {
         LaunchScope ls(g, s, "k_finalize");
-        k_finalize<<<planes, RED_THREADS, 0, s>>>(g->tp, g->T, g->psum, g->nz, 0, g->nz, card, g->counter,
-                                                  planes, mode, state, g->dots, slot);
+        NB_CUDA(nb_launch_ex(k_finalize, dim3(planes), dim3(RED_THREADS), 0, s, true, (const double *)g->tp, g->T,
+                             g->psum, (int)g->nz, 0, (int)g->nz, card, g->counter, planes, mode, state, g->dots, slot));
         return nb_launch_check("k_finalize");
     }
     if (nb_is_peer(g)) return nb_peer_reduce_finalize(g, card, mode, state, slot);

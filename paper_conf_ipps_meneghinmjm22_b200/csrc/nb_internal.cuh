@@ -7,6 +7,8 @@
 
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
+#include <utility>
 #include <string>
 #include <map>
 #include <vector>
@@ -302,6 +304,32 @@ struct LaunchScope {
         nvtxRangePop();
     }
 };
+
+// Programmatic dependent launch (sm_90+): a kernel launched with
+// nb_launch_ex(..., pdl = true) may start while the previous kernel of its
+// stream drains; it calls pdl_wait() before touching that kernel's results
+// (griddepcontrol.wait: a no-op for a normal launch), and producers call
+// pdl_trigger() once their last stores are issued.  NB_NO_PDL=1 disables.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+inline bool nb_pdl_enabled() {
+    return getenv("NB_NO_PDL") == nullptr;  // read per launch (graphs capture it once)
+}
+template <typename... KArgs, typename... Args>
+inline cudaError_t nb_launch_ex(void (*k)(KArgs...), dim3 grd, dim3 blk, size_t smem, cudaStream_t s, bool pdl,
+                                Args &&...args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grd;
+    cfg.blockDim = blk;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = pdl && nb_pdl_enabled() ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, k, std::forward<Args>(args)...);
+}
 
 // kernels / helpers implemented in the .cu files
 nb_status nb_launch_check(const char *what);

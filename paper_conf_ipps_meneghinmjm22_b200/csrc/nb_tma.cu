@@ -84,6 +84,7 @@ __global__ void __launch_bounds__(G::NT, G::MINB_A)
     extern __shared__ __align__(128) double tsm[];
     __shared__ __align__(8) uint64_t bar[NSTAGE];
     __shared__ double sw[TZC][NTY * NTX][DOT_TY];
+    pdl_wait();  // the previous kernel's scalars and fields (programmatic launch)
     if (!C1 && sc->status != 0) return;
     const double beta = C1 ? c1_a : sc->beta, ap = C1 ? 0.0 : sc->alpha_prev;
     const bool dox = !C1 && DOMAP && sc->pending;
@@ -200,6 +201,7 @@ __global__ void __launch_bounds__(G::NT, G::MINB_A)
         if (tile_x < tiles_x && tile_y * DOT_TY < g.ny)
             tp[((int64_t)g.z0 + zs + zi) * T + (int64_t)tile_y * tiles_x + tile_x] = s;
     }
+    pdl_trigger();  // this CTA's results are stored: the next kernel may launch
 }
 
 // ---------------------------------------------------------------------------
@@ -216,6 +218,7 @@ __global__ void __launch_bounds__(G::NT, G::MINB_B)
     extern __shared__ __align__(128) double tsm[];
     __shared__ __align__(8) uint64_t bar[NSTAGE];
     __shared__ double sw[TZC][NTY * NTX][DOT_TY];
+    pdl_wait();
     if (sc->status != 0) return;
     const double alpha = sc->alpha;
     // warp -> (dot tile t = (ty, tx) of the CTA, row wr of that tile); w = CTA row
@@ -300,6 +303,7 @@ __global__ void __launch_bounds__(G::NT, G::MINB_B)
         if (tile_x < tiles_x && tile_y * DOT_TY < g.ny)
             tp[((int64_t)g.z0 + zs + zi) * T + (int64_t)tile_y * tiles_x + tile_x] = s;
     }
+    pdl_trigger();  // this CTA's results are stored: the next kernel may launch
 }
 
 // ---------------------------------------------------------------------------
@@ -460,8 +464,8 @@ static nb_status launch_cgA(nb_grid *g, const PGeo &geo, const double *r, const 
     dim3 blk(G::NT),
         grd((g->tiles_x + NTX - 1) / NTX, (g->tiles_y + NTY - 1) / NTY, zhi >= 0 ? 2 : (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, label);
-    k_cgA_tma<DOMAP, C1, G><<<grd, blk, smem, g->cs>>>(mr, mpo, mpn, mx, pn, x, geo, zb, ze, sc, g->tp, g->T,
-                                                       g->tiles_x, zc, c1_a, c1_out, zhi);
+    NB_CUDA(nb_launch_ex(k_cgA_tma<DOMAP, C1, G>, grd, blk, (size_t)smem, g->cs, true, mr, mpo, mpn, mx, pn, x, geo,
+                         zb, ze, sc, g->tp, g->T, (int)g->tiles_x, zc, c1_a, c1_out, zhi));
     return nb_launch_check(label);
 }
 
@@ -497,6 +501,7 @@ nb_status nb_cgB_tma(nb_grid *g, const PGeo &geo, const double *p, double *r, in
     tma_smem_attr(k_cgB_tma<G>, smem);
     dim3 blk(G::NT), grd((g->tiles_x + NTX - 1) / NTX, (g->tiles_y + NTY - 1) / NTY, (ze - zb + zc - 1) / zc);
     LaunchScope ls(g, g->cs, "k_cg_B");
-    k_cgB_tma<G><<<grd, blk, smem, g->cs>>>(mp, mr, r, geo, zb, ze, sc, g->tp, g->T, g->tiles_x, zc);
+    NB_CUDA(nb_launch_ex(k_cgB_tma<G>, grd, blk, (size_t)smem, g->cs, true, mp, mr, r, geo, zb, ze, sc, g->tp, g->T,
+                         (int)g->tiles_x, zc));
     return nb_launch_check("k_cgB_tma");
 }
