@@ -937,9 +937,10 @@ struct FemTmaCfg {
     static constexpr int NT = DOT_TX * (DOT_TY / NR);         // threads per CTA
     static constexpr int NST = CGA ? NB_FEM_NST_A : FNST;     // ring stages
     static constexpr int SD = (CGA ? 6 : 3) * (FTPAD / 8);    // doubles per stage
-    // dynamic shared memory bytes: the ring, plus (FEM_CG_A) three p_new
-    // buffers of 3 component tiles
-    static constexpr int SMEM = (NST * SD + (CGA ? 9 * (FTPAD / 8) : 0)) * 8;
+    static constexpr int NPB = CGA ? 3 : 0;                    // p_new buffers
+    // dynamic shared memory bytes: the ring, plus (FEM_CG_A) the p_new
+    // buffers of 3 component tiles each
+    static constexpr int SMEM = (NST * SD + NPB * 3 * (FTPAD / 8)) * 8;
     static constexpr int MINB = CGA ? NB_FEM_MINB_A : NB_FEM_MINB;  // CTAs per SM
 };
 
@@ -959,8 +960,9 @@ struct FemTma {
     double (*sw)[3][DOT_TY];  // [output parity][component][tile row]
     double *tp;
     int T;
-    int tid, lane, x0, y0, x, ya, zs, zend, nplanes, fa, fb, sidx;
-    bool xin, xint, anyfast, dox;
+    int tid, lane, x0, y0, x, ya, zs, zend, nplanes, fa, fb, sidx, bx, by;
+    bool xin, xint, anyfast, dox, ctaint;
+    int64_t cb;  // (ya, x) offset within a plane
     double beta, ap;
     double cv[8];  // canonical stencil values (registers for the whole kernel)
 
@@ -1001,12 +1003,12 @@ struct FemTma {
         double xo[NR][3], pc[NR][3];               // CGA: x and p_old of the own centres
         if constexpr (CGA) {
             if (own && dox) {
+                const double *xp = A.x + (int64_t)(zin + 1) * g.ps + cb;
 #pragma unroll
                 for (int r = 0; r < NR; ++r) {
-                    const int64_t c0 = (int64_t)(zin + 1) * g.ps + (int64_t)(ya + r) * g.pitch + x;
-                    const bool v = xin && ya + r < g.ny;
+                    const bool v = ctaint || (xin && ya + r < g.ny);
 #pragma unroll
-                    for (int c = 0; c < 3; ++c) xo[r][c] = v ? __ldcs(A.x + c * A.cs + c0) : 0.0;
+                    for (int c = 0; c < 3; ++c) xo[r][c] = v ? __ldcs(xp + c * A.cs + r * g.pitch) : 0.0;
                 }
             }
             mbar_wait(&bar[(unsigned)j % NST], ((unsigned)j / NST) & 1u);
@@ -1014,15 +1016,31 @@ struct FemTma {
             // stays readable for this step's epilogue (its centres are the dot's
             // p_new), and is overwritten only at step j+2, past barrier j+1
             double *P = fsm + NST * SD + ((unsigned)j % 3u) * 3 * CP;
+            // the three component boxes are contiguous (r at S, p_old at
+            // S + 3 CP, p_new at P): one flat 16-byte pass over 3 CP doubles
+            // (the 8 padding doubles of a box are never read)
+            constexpr int NP2 = 3 * CP / 2, NIT = (NP2 + NT - 1) / NT;
+            const double2 *S2 = reinterpret_cast<const double2 *>(S);
+            double2 *P2 = reinterpret_cast<double2 *>(P);
             if (!halo(zin)) {  // CTA-uniform
-                for (int c = 0; c < 3; ++c)
-                    for (int e = tid; e < FBX * FBY; e += NT) P[c * CP + e] = fma(beta, S[(3 + c) * CP + e], S[c * CP + e]);
+#pragma unroll
+                for (int k = 0; k < NIT; ++k) {
+                    const int e = tid + k * NT;
+                    if (NP2 % NT == 0 || k + 1 < NIT || e < NP2) {
+                        const double2 rv = S2[e], pv = S2[NP2 + e];
+                        P2[e] = make_double2(fma(beta, pv.x, rv.x), fma(beta, pv.y, rv.y));
+                    }
+                }
 #pragma unroll
                 for (int r = 0; r < NR; ++r)
 #pragma unroll
                     for (int c = 0; c < 3; ++c) pc[r][c] = S[(3 + c) * CP + sidx + r * FBX];
             } else {
-                for (int e = tid; e < 3 * CP; e += NT) P[e] = S[e];
+#pragma unroll
+                for (int k = 0; k < NIT; ++k) {
+                    const int e = tid + k * NT;
+                    if (NP2 % NT == 0 || k + 1 < NIT || e < NP2) P2[e] = S2[e];
+                }
             }
             __syncthreads();  // p_new tiles ready; the raw stage is free; step j-1's dot rows are in sw
             if (tid == 0 && j + NST < nplanes) issue(j + NST);
@@ -1053,15 +1071,15 @@ struct FemTma {
         }
         if constexpr (CGA) {
             if (own) {  // own plane: store p_new and the deferred x += alpha_prev p_old
+                const int64_t c0 = (int64_t)(zin + 1) * g.ps + cb;
 #pragma unroll
                 for (int r = 0; r < NR; ++r) {
-                    const int y = ya + r;
-                    if (xin && y < g.ny) {
-                        const int64_t c0 = (int64_t)(zin + 1) * g.ps + (int64_t)y * g.pitch + x;
+                    if (ctaint || (xin && ya + r < g.ny)) {
+                        const int64_t cr = c0 + r * g.pitch;
 #pragma unroll
                         for (int c = 0; c < 3; ++c) {
-                            __stcs(A.pn + c * A.cs + c0, S[c * CP + sidx + r * FBX]);  // S = this plane's p_new tiles
-                            if (dox) __stcs(A.x + c * A.cs + c0, fma(ap, pc[r][c], xo[r][c]));
+                            __stcs(A.pn + c * A.cs + cr, S[c * CP + sidx + r * FBX]);  // S = this plane's p_new tiles
+                            if (dox) __stcs(A.x + c * A.cs + cr, fma(ap, pc[r][c], xo[r][c]));
                         }
                     }
                 }
@@ -1094,7 +1112,7 @@ struct FemTma {
             double s = w[tid][0];
 #pragma unroll
             for (int k = 1; k < DOT_TY; ++k) s = __dadd_rn(s, w[tid][k]);
-            tp[((int64_t)tid * g.NZ + g.z0 + zl) * T + blockIdx.y * gridDim.x + blockIdx.x] = s;
+            tp[((int64_t)tid * g.NZ + g.z0 + zl) * T + by * gridDim.x + bx] = s;
         }
     }
 
@@ -1102,6 +1120,16 @@ struct FemTma {
     __device__ __forceinline__ void epilogue(int zl, const double (&o3)[NR][3], const double (&cen)[NR][3]) const {
         const bool zfast = zl >= fa && zl < fb;
         double prod[NR * 3];
+        if (K != FEM_CG_INIT && ctaint && zfast) {  // CTA-uniform: every node of the tile is interior
+            const int64_t c0 = (int64_t)(zl + 1) * g.ps + cb;
+#pragma unroll
+            for (int r = 0; r < NR; ++r)
+#pragma unroll
+                for (int c = 0; c < 3; ++c) {
+                    __stcs(A.y + c * A.cs + c0 + r * g.pitch, o3[r][c]);
+                    prod[r * 3 + c] = (K == FEM_CG_Q || CGA) ? __dmul_rn(cen[r][c], o3[r][c]) : 0.0;
+                }
+        } else
 #pragma unroll
         for (int r = 0; r < NR; ++r) {
             const int y = ya + r;
@@ -1150,11 +1178,12 @@ __global__ void __launch_bounds__(FemTmaCfg<K>::NT, FemTmaCfg<K>::MINB)
     FemTma<K, ZC> t{M, A, g, fsm, bar, sw, tp, T};
     t.tid = threadIdx.y * DOT_TX + threadIdx.x;
     t.lane = threadIdx.x;
-    t.x0 = blockIdx.x * DOT_TX;
-    t.y0 = blockIdx.y * DOT_TY;
+    t.bx = blockIdx.x, t.by = blockIdx.y;
+    t.zs = zb0 + blockIdx.z * ZC;
+    t.x0 = t.bx * DOT_TX;
+    t.y0 = t.by * DOT_TY;
     t.x = t.x0 + threadIdx.x;
     t.ya = t.y0 + threadIdx.y * NR;  // rows ya .. ya+NR-1
-    t.zs = zb0 + blockIdx.z * ZC;
     t.zend = min(t.zs + ZC, ze0);
     t.nplanes = t.zend - t.zs + 2;  // planes zs-1 .. zend
     t.xin = t.x < g.nx;
@@ -1164,6 +1193,9 @@ __global__ void __launch_bounds__(FemTmaCfg<K>::NT, FemTmaCfg<K>::MINB)
     t.anyfast = false;
 #pragma unroll
     for (int r = 0; r < NR; ++r) t.anyfast |= t.xint && t.ya + r >= 1 && t.ya + r <= g.ny - 2;
+    // the whole 32 x 8 tile is x/y-interior (no surface node, no row past ny)
+    t.ctaint = t.x0 >= 1 && t.x0 + DOT_TX <= g.nx - 1 && t.y0 >= 1 && t.y0 + DOT_TY <= g.ny - 1;
+    t.cb = (int64_t)t.ya * g.pitch + t.x;
     t.sidx = (threadIdx.y * NR + 1) * FBX + threadIdx.x + 2;
     t.beta = t.ap = 0.0;
     t.dox = false;
