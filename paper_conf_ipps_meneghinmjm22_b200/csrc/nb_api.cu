@@ -564,6 +564,9 @@ extern "C" nb_status nb_grid_destroy(nb_grid *g) {
     cudaFree(g->counter);
     if (g->own_cs && g->cs) cudaStreamDestroy(g->cs);
     if (g->own_hs && g->hs) cudaStreamDestroy(g->hs);
+    if (g->fs) cudaStreamDestroy(g->fs);
+    for (auto &e : g->fev)
+        if (e) cudaEventDestroy(e);
     delete g;
     return NB_OK;
 }

@@ -944,6 +944,41 @@ struct FemTmaCfg {
     static constexpr int MINB = CGA ? NB_FEM_MINB_A : NB_FEM_MINB;  // CTAs per SM
 };
 
+// Which (tile x, tile y, z-chunk) a CTA of the streaming kernel takes.
+// mode 0: the whole grid (blockIdx as is); 1: the surface-free box, tiles
+// [1, tx-2] x [1, ty-2] of chunks [ca, cb] (grid (tx-2, ty-2, cb-ca+1));
+// 2: its complement (1-D grid): every tile of the chunks outside [ca, cb],
+// then the ring of edge tiles of each chunk in [ca, cb].
+struct FemCtaMap {
+    int mode, tx, ty, nc, ca, cb;
+};
+__device__ __forceinline__ void fem_cta(const FemCtaMap &m, int &bx, int &by, int &ck) {
+    if (m.mode == 0) {
+        bx = blockIdx.x, by = blockIdx.y, ck = blockIdx.z;
+    } else if (m.mode == 1) {
+        bx = 1 + blockIdx.x, by = 1 + blockIdx.y, ck = m.ca + blockIdx.z;
+    } else {
+        int L = blockIdx.x;
+        const int tt = m.tx * m.ty, lo = m.ca * tt, hi = (m.nc - 1 - m.cb) * tt;
+        if (L < lo || L - lo < hi) {
+            ck = L < lo ? L / tt : m.cb + 1 + (L - lo) / tt;
+            const int r = (L < lo ? L : L - lo) % tt;
+            bx = r % m.tx, by = r / m.tx;
+        } else {
+            L -= lo + hi;
+            const int R = 2 * m.tx + 2 * (m.ty - 2);
+            ck = m.ca + L / R;
+            int r = L % R;
+            if (r < 2 * m.tx) {
+                by = r < m.tx ? 0 : m.ty - 1, bx = r % m.tx;
+            } else {
+                r -= 2 * m.tx;
+                bx = (r & 1) ? m.tx - 1 : 0, by = 1 + (r >> 1);
+            }
+        }
+    }
+}
+
 // Per-CTA state of the streaming kernel.  A thread owns NR rows of one x
 // column of a 32 x 8 tile and marches ZC output planes; plane j of the
 // chunk (local plane zs - 1 + j) arrives in ring stage j % NST.
@@ -960,7 +995,7 @@ struct FemTma {
     double (*sw)[3][DOT_TY];  // [output parity][component][tile row]
     double *tp;
     int T;
-    int tid, lane, x0, y0, x, ya, zs, zend, nplanes, fa, fb, sidx, bx, by;
+    int tid, lane, x0, y0, x, ya, zs, zend, nplanes, fa, fb, sidx, bx, by, tx;
     bool xin, xint, anyfast, dox, ctaint;
     int64_t cb;  // (ya, x) offset within a plane
     double beta, ap;
@@ -1112,7 +1147,7 @@ struct FemTma {
             double s = w[tid][0];
 #pragma unroll
             for (int k = 1; k < DOT_TY; ++k) s = __dadd_rn(s, w[tid][k]);
-            tp[((int64_t)tid * g.NZ + g.z0 + zl) * T + by * gridDim.x + bx] = s;
+            tp[((int64_t)tid * g.NZ + g.z0 + zl) * T + by * tx + bx] = s;
         }
     }
 
@@ -1168,7 +1203,7 @@ struct FemTma {
 
 template <int K, int ZC, int NR>
 __global__ void __launch_bounds__(FemTmaCfg<K>::NT, FemTmaCfg<K>::MINB)
-    k_fem_tma(const __grid_constant__ FemMaps M, FemArgs A, PGeo g, int zb0, int ze0, double *tp, int T) {
+    k_fem_tma(const __grid_constant__ FemMaps M, FemArgs A, PGeo g, int zb0, int ze0, double *tp, int T, FemCtaMap cm) {
     using Cfg = FemTmaCfg<K>;
     static_assert(Cfg::NR == NR, "rows per thread");
     extern __shared__ __align__(128) double fsm[];
@@ -1178,8 +1213,12 @@ __global__ void __launch_bounds__(FemTmaCfg<K>::NT, FemTmaCfg<K>::MINB)
     FemTma<K, ZC> t{M, A, g, fsm, bar, sw, tp, T};
     t.tid = threadIdx.y * DOT_TX + threadIdx.x;
     t.lane = threadIdx.x;
-    t.bx = blockIdx.x, t.by = blockIdx.y;
-    t.zs = zb0 + blockIdx.z * ZC;
+    {
+        int ck;
+        fem_cta(cm, t.bx, t.by, ck);
+        t.tx = cm.tx;
+        t.zs = zb0 + ck * ZC;
+    }
     t.x0 = t.bx * DOT_TX;
     t.y0 = t.by * DOT_TY;
     t.x = t.x0 + threadIdx.x;
@@ -1382,7 +1421,43 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
         } else {
             for (int c = 0; c < 3; ++c) NB_TRY(tmap_for(A.u + c * A.cs, geo, 0, &M.u[c]));
         }
-        // surface nodes first (converged), then the streaming interior
+        // surface nodes first (converged), then the streaming interior.
+        // NB_FEM_CONC (default on): the surface kernels run on the halo
+        // stream concurrently with the streaming kernel's surface-free box
+        // (interior tiles of the chunks without a z-surface plane: its
+        // epilogue never reads a surface node's output); the rest of the
+        // streaming kernel waits for them on a side stream, and the grid
+        // stream joins both.  Same CTAs, same arithmetic: same bits.
+        const int tx = g->tiles_x, ty = g->tiles_y, nck = (ze - zb + ZC - 1) / ZC;
+        FemCtaMap cm{0, tx, ty, nck, 0, -1};
+        bool conc = false;
+        {
+            const char *cv = getenv("NB_FEM_CONC");
+            if ((!cv || atoi(cv) != 0) && (what == FEM_ALL) && zhi < 0 && tx >= 3 && ty >= 3) {
+                // chunks free of z-surface planes (global z < 2 or z > NZ-2)
+                int ca = 0, cb = nck - 1;
+                while (ca < nck && (geo.z0 + zb + ca * ZC < 2 || geo.z0 + std::min(zb + (ca + 1) * ZC, ze) - 1 > geo.NZ - 2)) ++ca;
+                while (cb >= ca && (geo.z0 + zb + cb * ZC < 2 || geo.z0 + std::min(zb + (cb + 1) * ZC, ze) - 1 > geo.NZ - 2)) --cb;
+                if (cb >= ca) {
+                    cm.ca = ca, cm.cb = cb;
+                    conc = true;
+                }
+            }
+        }
+        cudaStream_t ss = g->cs;  // stream of the surface kernels
+        if (conc) {
+            if (!g->fs) {
+                int lo, hi;
+                NB_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+                NB_CUDA(cudaStreamCreateWithPriority(&g->fs, cudaStreamNonBlocking, hi));
+                for (auto &e : g->fev) NB_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+            }
+            NB_CUDA(cudaEventRecord(g->fev[0], g->cs));  // fork
+            NB_CUDA(cudaStreamWaitEvent(g->hs, g->fev[0], 0));
+            NB_CUDA(cudaStreamWaitEvent(g->fs, g->fev[0], 0));
+            ss = g->hs;
+        }
+        cudaStream_t xs = conc ? g->fs : ss;  // x-face kernel: its own stream (starts with k_fem_surface)
         FemSurf S{};
         const int nx = geo.nx, ny = geo.ny;
         S.ncol_edge = nx * std::min(ny, 2) + std::max(ny - 2, 0) * std::min(nx, 2);
@@ -1408,20 +1483,20 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
             if (xface) {
                 S.ncol_edge = 2 * nx;  // fem_edge_col lists the y = 0 and y = ny-1 rows first
                 dim3 xg((ny - 2 + XF_Y - 1) / XF_Y, zhi >= 0 ? 2 : (ze - zb + XF_Z - 1) / XF_Z, 2);
-                LaunchScope ls(g, g->cs, "k_fem_surface");
-                k_fem_xface<K><<<xg, XF_Y * XF_Z, 0, g->cs>>>(A, geo, zb, ze, zhi);
+                LaunchScope ls(g, xs, "k_fem_surface");
+                k_fem_xface<K><<<xg, XF_Y * XF_Z, 0, xs>>>(A, geo, zb, ze, zhi);
             }
             const int64_t n = (int64_t)S.ncol_edge * nzr + (int64_t)S.nin * S.nzs;
             if (n > 0) {
                 const int blocks = (int)std::min<int64_t>((n + NB_FSURF_BX - 1) / NB_FSURF_BX, 1 << 30);
-                LaunchScope ls(g, g->cs, "k_fem_surface");
-                k_fem_surface<K><<<blocks, NB_FSURF_BX, 0, g->cs>>>(A, geo, zb, ze, S, zhi);
+                LaunchScope ls(g, ss, "k_fem_surface");
+                k_fem_surface<K><<<blocks, NB_FSURF_BX, 0, ss>>>(A, geo, zb, ze, S, zhi);
             }
             if (ncols > 0) {
                 if (zhi >= 0) NB_FAIL(NB_EUNSUPPORTED, "plane pairs with the face-column kernel");
                 dim3 fg((ncols + 63) / 64, (ze - zb + FZC - 1) / FZC);
-                LaunchScope ls(g, g->cs, "k_fem_faces");
-                k_fem_faces<K><<<fg, 64, 0, g->cs>>>(A, geo, zb, ze, ncols);
+                LaunchScope ls(g, ss, "k_fem_faces");
+                k_fem_faces<K><<<fg, 64, 0, ss>>>(A, geo, zb, ze, ncols);
             }
         }
         if (!(what & FEM_BULK)) return NB_OK;
@@ -1430,9 +1505,32 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
             NB_CUDA(cudaFuncSetAttribute(k_fem_tma<K, ZC, NR>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM));
             attr_set |= 1u << g->device;
         }
-        dim3 blk(DOT_TX, DOT_TY / NR), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);
-        LaunchScope ls(g, g->cs, name);
-        k_fem_tma<K, ZC, NR><<<grd, blk, Cfg::SMEM, g->cs>>>(M, A, geo, zb, ze, g->tp, g->T);
+        dim3 blk(DOT_TX, DOT_TY / NR);
+        if (!conc) {
+            LaunchScope ls(g, g->cs, name);
+            k_fem_tma<K, ZC, NR><<<dim3(tx, ty, nck), blk, Cfg::SMEM, g->cs>>>(M, A, geo, zb, ze, g->tp, g->T, cm);
+        } else {
+            NB_CUDA(cudaEventRecord(g->fev[1], ss));  // surface nodes done (x faces: on fs, before the rest)
+            {
+                FemCtaMap c1 = cm;
+                c1.mode = 1;
+                LaunchScope ls(g, g->cs, name);
+                k_fem_tma<K, ZC, NR><<<dim3(tx - 2, ty - 2, cm.cb - cm.ca + 1), blk, Cfg::SMEM, g->cs>>>(
+                    M, A, geo, zb, ze, g->tp, g->T, c1);
+                NB_TRY(nb_launch_check(name));
+            }
+            NB_CUDA(cudaStreamWaitEvent(g->fs, g->fev[1], 0));
+            {
+                FemCtaMap c2 = cm;
+                c2.mode = 2;
+                const int n2 = (nck - (cm.cb - cm.ca + 1)) * tx * ty + (cm.cb - cm.ca + 1) * (2 * tx + 2 * (ty - 2));
+                LaunchScope ls(g, g->fs, name);
+                k_fem_tma<K, ZC, NR><<<n2, blk, Cfg::SMEM, g->fs>>>(M, A, geo, zb, ze, g->tp, g->T, c2);
+                NB_TRY(nb_launch_check(name));
+            }
+            NB_CUDA(cudaEventRecord(g->fev[2], g->fs));
+            NB_CUDA(cudaStreamWaitEvent(g->cs, g->fev[2], 0));  // join
+        }
     } else {
         constexpr int ZC = 16;
         dim3 blk(DOT_TX, DOT_TY), grd(g->tiles_x, g->tiles_y, (ze - zb + ZC - 1) / ZC);

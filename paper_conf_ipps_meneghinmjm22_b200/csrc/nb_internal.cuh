@@ -211,6 +211,10 @@ struct nb_grid {
     std::vector<uint8_t> host_mask;    // [z][y][x] active cells (element-sparse; lazy tables)
     int64_t n_active = 0;
     NbPeer *peer = nullptr;  // peer-memory transport (multi-process)
+    // FEM: surface-node kernels concurrent with the surface-free part of the
+    // streaming kernel (nb_fem.cu fem_launch): a side stream + fork/join events
+    cudaStream_t fs = nullptr;
+    cudaEvent_t fev[3] = {nullptr, nullptr, nullptr};
 };
 
 constexpr int NB_DOT_SLOTS = 1024;
@@ -329,6 +333,14 @@ inline cudaError_t nb_launch_ex(void (*k)(KArgs...), dim3 grd, dim3 blk, size_t 
     cfg.attrs = at;
     cfg.numAttrs = pdl && nb_pdl_enabled() ? 1 : 0;
     return cudaLaunchKernelEx(&cfg, k, std::forward<Args>(args)...);
+}
+
+// graph instantiation flags: kernel nodes keep the priority of the stream
+// they were captured on (the halo / FEM surface streams are high priority);
+// NB_GRAPH_PRIO=0 instantiates without node priorities
+inline unsigned long long nb_graph_flags() {
+    const char *v = getenv("NB_GRAPH_PRIO");
+    return (v && atoi(v) == 0) ? 0ull : (unsigned long long)cudaGraphInstantiateFlagUseNodePriority;
 }
 
 // kernels / helpers implemented in the .cu files

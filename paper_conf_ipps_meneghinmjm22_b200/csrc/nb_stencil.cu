@@ -695,7 +695,7 @@ extern "C" nb_status nb_map_stencil_reduce(nb_field *x, nb_field *y, double a, i
             g->launches = l0;
             if (st == NB_OK && e != cudaSuccess) NB_FAIL(NB_ECUDA, "C1 graph capture: %s", cudaGetErrorString(e));
             if (st == NB_OK) {
-                e = cudaGraphInstantiate(&g->c1_exec, gr, 0);
+                e = cudaGraphInstantiate(&g->c1_exec, gr, nb_graph_flags());
                 cudaGraphDestroy(gr);
                 if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "C1 graph instantiate: %s", cudaGetErrorString(e));
                 g->c1_x = x->base[fl];
@@ -875,7 +875,7 @@ static nb_status cg_graph(nb_cg *cg, int n, int par, std::pair<cudaGraphExec_t, 
         if (s != NB_OK) return s;
         if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "graph capture failed: %s", cudaGetErrorString(e));
         cudaGraphExec_t exec;
-        e = cudaGraphInstantiate(&exec, graph, 0);
+        e = cudaGraphInstantiate(&exec, graph, nb_graph_flags());
         cudaGraphDestroy(graph);
         if (e != cudaSuccess) NB_FAIL(NB_ECUDA, "graph instantiate failed: %s", cudaGetErrorString(e));
         it = cg->graphs.emplace(key, std::make_pair(exec, nl)).first;

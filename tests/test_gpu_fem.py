@@ -109,7 +109,7 @@ def test_fem_cg_converges():
 
 
 @pytest.mark.parametrize("dims,parts", [((17, 13, 40), 1), ((34, 19, 37), 3), ((9, 10, 5), 1), ((20, 70, 13), 2),
-                                        ((2, 9, 6), 1)])
+                                        ((2, 9, 6), 1), ((98, 27, 70), 1), ((70, 20, 100), 2)])
 def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
     """The TMA-staged z-march (default), the register z-march and the
     one-node-per-thread kernel must agree bit for bit: each output receives
@@ -122,13 +122,16 @@ def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
     # (NB_FEM_FACES=col), x-face nodes in the one-thread-per-node surface
     # kernel instead of the shared-memory x-face kernel (NB_FEM_FACES=node)
     # and the 3-pass CG schedule (NB_FEM_3PASS: map -> q = K p -> r), and
-    # the one-CTA-per-plane residual kernel (NB_FEM_R_PLANE) against the
+    # the one-CTA-per-plane residual kernel (NB_FEM_R_PLANE), and the
+    # surface-node kernels serialised before the streaming kernel instead of
+    # concurrent with its surface-free box (NB_FEM_CONC=0; the last two
+    # shapes have >= 3 x 3 tiles and surface-free z-chunks) against the
     # default fused schedule
     envs = {None: {}, "zmarch": {"NB_FEM_KERNEL": "zmarch"}, "plain": {"NB_FEM_KERNEL": "plain"},
             "faces_col": {"NB_FEM_FACES": "col"}, "faces_node": {"NB_FEM_FACES": "node"},
-            "3pass": {"NB_FEM_3PASS": "1"}, "r_plane": {"NB_FEM_R_PLANE": "1"}}
+            "3pass": {"NB_FEM_3PASS": "1"}, "r_plane": {"NB_FEM_R_PLANE": "1"}, "serial": {"NB_FEM_CONC": "0"}}
     for variant, env in envs.items():
-        for k in ("NB_FEM_KERNEL", "NB_FEM_FACES", "NB_FEM_3PASS", "NB_FEM_R_PLANE"):
+        for k in ("NB_FEM_KERNEL", "NB_FEM_FACES", "NB_FEM_3PASS", "NB_FEM_R_PLANE", "NB_FEM_CONC"):
             if k in env:
                 monkeypatch.setenv(k, env[k])
             else:
@@ -146,7 +149,7 @@ def test_fem_kernels_bitwise_equal(dims, parts, monkeypatch):
             out[variant] = (y, fx.download(), r.rr)
             for f in (fu, fy, fb, fx):
                 f.close()
-    for v in ("zmarch", "plain", "faces_col", "faces_node", "3pass", "r_plane"):
+    for v in ("zmarch", "plain", "faces_col", "faces_node", "3pass", "r_plane", "serial"):
         assert np.array_equal(out[None][0], out[v][0]), v
         assert np.array_equal(out[None][1], out[v][1]) and out[None][2] == out[v][2], v
 

@@ -16,6 +16,7 @@ n = int(args[0]) if args else 512
 iters = int(args[1]) if len(args) > 1 else 100
 parts = int(os.environ.get("AB_PARTS", "1"))
 g = nb.Grid((n, n, n), nparts=parts, devices=[0] * parts)
+g.set_halo_mode(int(os.environ.get("AB_HALO", "0")))  # 1: halo copies on the halo stream
 s = torch.cuda.ExternalStream(g.stream())
 b, x = nb.Field(g), nb.Field(g)
 b.fill(nb.FILL_POISSON_RHS)
