@@ -621,6 +621,11 @@ def bench_fem_run(n, steps, warmup, world, local):
     cg.finish()
     cg.close()
     x.fill_const(0.0)
+    # per-kernel times from the serial schedule (NB_FEM_CONC=0: same kernels,
+    # same bits; the timed step runs the surface kernels concurrently with the
+    # surface-free part of phase A, whose stream spans would overlap)
+    conc_env = os.environ.get("NB_FEM_CONC")
+    os.environ["NB_FEM_CONC"] = "0"
     cg = nb.CG(x, b, op=nb.OP_FEM27)
     cg.iterate(1)  # the first iteration has no deferred x update: profile steady-state ones
     pit = 5
@@ -634,6 +639,10 @@ def bench_fem_run(n, steps, warmup, world, local):
     u.halo_update()
     nb.nb_fem27_apply(u, y, 1.0, 0.3)
     aprof = _profiled_kernels(g, lambda: [nb.nb_fem27_apply(u, y, 1.0, 0.3) for _ in range(5)], ["k_fem_apply"])
+    if conc_env is None:
+        os.environ.pop("NB_FEM_CONC", None)
+    else:
+        os.environ["NB_FEM_CONC"] = conc_env
     u.close(), y.close()
     hbm, peak_kind = peaks()
     f64, f64_kind = fp64_peak()
@@ -660,6 +669,8 @@ def bench_fem_run(n, steps, warmup, world, local):
             "roofline": {"bound": "hbm", "kernel": "k_fem_cg_a", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                          "frac": achieved / hbm, "peak_kind": peak_kind, "traffic": ncu_traffic("k_fem_cg_a"),
                          "algorithmic_bytes_per_node": FEM_BYTES["k_fem_cg_a"], "per_rank": world > 1,
+                         "kernel_times": "serial schedule (NB_FEM_CONC=0); the timed step overlaps the "
+                                         "surface kernels with phase A",
                          "kernel_ms_per_iter": {k: v[1] / pit for k, v in prof.items()},
                          "launches_per_iter": {k: v[0] / pit for k, v in prof.items()}},
             "apply_alu": {"bound": "alu", "kernel": "k_fem_apply (interior K u, surface nodes excluded)",
