@@ -538,7 +538,12 @@ template <bool EVEN, bool PERIODIC>
 #ifndef NB_AA_BX
 #define NB_AA_BX 32
 #endif
-__global__ void __launch_bounds__(NB_AA_BX) k_lbm_aa(LbmAAArgs A) {  // 32 wide: 3.44 ms/step at 512^3 (64: 3.62, 128: 3.69, 256: 4.0)
+#ifndef NB_AA_MINB
+// 28 CTAs of one warp per SM (<= 73 registers): 3.49 against 3.95 ms/step
+// with the unconstrained 95 registers (24: 3.66, 32: 3.50; tools/aa_ab.sh)
+#define NB_AA_MINB 28
+#endif
+__global__ void __launch_bounds__(NB_AA_BX, NB_AA_MINB) k_lbm_aa(LbmAAArgs A) {  // 32 wide: 3.44 ms/step at 512^3 (64: 3.62, 128: 3.69, 256: 4.0)
     const int x = blockIdx.x * blockDim.x + threadIdx.x;
     const int y = blockIdx.y;
     const int zl = blockIdx.z;
