@@ -5,6 +5,13 @@
 
 #include "nb_internal.cuh"
 
+// Bulk L2 prefetch of [p, p + bytes) (p 16-byte aligned, bytes a multiple
+// of 16): the copy engine of the SM fetches the lines into L2 without
+// holding a register or a thread; a later load of them is an L2 hit.
+__device__ __forceinline__ void nb_prefetch_l2(const void *p, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
 // xor-butterfly warp sum (offsets 16, 8, 4, 2, 1).  IEEE addition is
 // commutative, so every lane ends with the same bits: the value is a fixed
 // function of the 32 inputs.
@@ -57,6 +64,17 @@ __device__ __forceinline__ int warp_multi_index(int lane) {
     for (int h = M / 2; h >= 1; h >>= 1, o >>= 1)
         if (lane & o) idx += h;
     return idx;
+}
+
+// The N canonical warp sums of v (warp_sum_multi) stored by one lane each:
+// dst[i * stride] = the warp total of value i.  Bitwise equal to N
+// warp_sum_canon calls stored by lane 0.
+template <int N>
+__device__ __forceinline__ void warp_sums_store(const double (&v)[N], int lane, double *dst, int stride) {
+    constexpr int M = WarpMulti<N>::M;
+    const double s = warp_sum_multi<N>(v, lane);
+    const int i = warp_multi_index<N>(lane);
+    if (i < N && (lane & (32 / M - 1)) == 0) dst[i * stride] = s;
 }
 
 // Canonical block tree over n values v[0..n) (stride `stride`) computed by a

@@ -1656,11 +1656,7 @@ __global__ void __launch_bounds__(256, NB_SPF_MINB) k_sp_fem(SpFemArgs A) {
     }
     if (KIND == 0) return;
     const int w = t >> 5;
-#pragma unroll
-    for (int c = 0; c < 3; ++c) {
-        const double v = warp_sum_canon(prod[c]);
-        if ((t & 31) == 0) sw[c][w] = v;
-    }
+    warp_sums_store<3>(prod, t & 31, &sw[0][w], 8);
     __syncthreads();
     if (t < 3) {
         double s = sw[t][0];

@@ -550,6 +550,8 @@ struct SpArgs {
     double *c;
     double *d;
     CgScal *sc;
+    int pf;         // k_sp_runs: L2 prefetch distance in blocks (0: none)
+    float cps;      // k_sp_runs: mean cells per segment of the launch
 };
 
 template <typename T>
@@ -989,6 +991,26 @@ __global__ void __launch_bounds__(SEG, NB_SPR_MINB) k_sp_runs(SpArgs A, const in
                                                              const int32_t *__restrict__ gidx) {
     __shared__ double sw[NSBR][SEG / 32];
     const int t = threadIdx.x;
+    // L2 prefetch of the table entries and operand cells of the block A.pf
+    // blocks ahead (blocks start in index order): when that block runs, its
+    // table loads and its +z gathers hit L2 instead of DRAM, which takes one
+    // DRAM latency off each cell's dependent chain.  The operand window is
+    // estimated from the mean cells per segment (a prefetch only moves data).
+    if (A.pf > 0 && gidx == nullptr && t < 2) {
+        const int64_t qa = ((int64_t)blockIdx.x + A.pf) * NSBR;
+        if (qa < A.nseg) {
+            const int64_t nsa = A.nseg - qa < NSBR ? A.nseg - qa : NSBR;
+            if (t == 0) {
+                nb_prefetch_l2(nbrt + (A.seg0 + qa) * SEG, (uint32_t)(nsa * SEG * sizeof(int4)));
+            } else {
+                const int64_t c0 = A.hl + (int64_t)((float)(A.seg0 + qa) * A.cps);
+                const int64_t a0 = (c0 - 64) & ~(int64_t)15;
+                const int64_t lim = A.hl + A.n;
+                if (a0 >= 0 && a0 + (NSBR * SEG + 128) <= lim)
+                    nb_prefetch_l2(A.a + a0, (uint32_t)((NSBR * SEG + 128) * sizeof(double)));
+            }
+        }
+    }
     int4 inf[NSBR], nb4[NSBR];
 #pragma unroll
     for (int k = 0; k < NSBR; ++k) {
@@ -1047,11 +1069,7 @@ __global__ void __launch_bounds__(SEG, NB_SPR_MINB) k_sp_runs(SpArgs A, const in
         }
     }
     const int w = t >> 5;
-#pragma unroll
-    for (int k = 0; k < NSBR; ++k) {
-        const double vv = warp_sum_canon(prod[k]);
-        if ((t & 31) == 0) sw[k][w] = vv;
-    }
+    warp_sums_store<NSBR>(prod, t & 31, &sw[0][w], SEG / 32);
     __syncthreads();
     if (t < NSBR) {
         int4 it = inf[0];
@@ -1082,6 +1100,13 @@ static nb_status sp_launch_runs(nb_grid *g, int p, const int32_t *list, const in
     A.plane0 = plane_base + g->parts[p].z0;
     A.T = g->T;
     A.tp = g->tp;
+    {
+        // 300-1500 blocks ahead measured equal (0.242 ms vs 0.269 without at
+        // 512^3); 3000 loses the lines before use.  NB_SPR_PF=0 disables.
+        static const int pf = getenv("NB_SPR_PF") ? atoi(getenv("NB_SPR_PF")) : 600;
+        A.pf = gidx ? 0 : pf;
+        A.cps = sp.seg_start.back() > 0 ? (float)((double)sp.n / (double)sp.seg_start.back()) : 256.f;
+    }
     LaunchScope ls(g, g->cs, name);
     k_sp_runs<K><<<(unsigned)((n + NSBR - 1) / NSBR), SEG, 0, g->cs>>>(A, (const int4 *)sp.d_nbr,
                                                                     (const int4 *)sp.d_seginfo, gidx);
