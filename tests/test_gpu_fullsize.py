@@ -110,3 +110,29 @@ def test_c5_fem_384_sampled_nodes_vs_oracle():
         e = exp[:, loc[0], loc[1], loc[2]]
         got = yg[:, z, yy, x]
         assert np.max(np.abs(got - e)) <= 1e-13 * max(1.0, np.max(np.abs(e))), (x, yy, z)
+
+
+def test_c2_poisson_cg_1024_max_size_vs_oracle():
+    """Maximum-size case: 1024^3 fp64 (8 x the C2 bench grid; 8.6 GB per
+    field, the buffer offsets pass 2^33 bytes), 2 CG iterations on the bench
+    path vs the oracle on the whole grid."""
+    n, k = 1024, 2
+    b = synth.poisson_poly_rhs((n, n, n))
+    xo, ro, hist = oracle.cg(b, max_iter=k)
+    del b
+    with nb.Grid((n, n, n)) as g:
+        fb, fx = nb.Field(g), nb.Field(g)
+        fb.fill(nb.FILL_POISSON_RHS)
+        fx.fill_const(0.0)
+        cg = nb.CG(fx, fb)
+        cg.prepare(k)
+        cg.iterate(k)
+        r = cg.finish()
+        cg.close()
+        fb.close()
+        x = fx.download()
+        fx.close()
+    assert r.iters == k
+    assert abs(r.rr0 - hist[0]) <= 1e-12 * hist[0]
+    assert abs(r.rr - ro.rr) <= 1e-10 * ro.rr
+    assert np.max(np.abs(x - xo)) <= 1e-11 * np.max(np.abs(xo))
