@@ -1551,6 +1551,66 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
 // identity row.  A full mask therefore reproduces the dense operator bit for
 // bit; general masks are the oracle's element-by-element K (tolerance).
 // ===========================================================================
+// y_n of an active node off the Dirichlet plane (gz >= 1) from its
+// 27-neighbourhood mask m (bit (ox+1) + 3(oy+1) + 9(oz+1)) and a loader
+// ld(q, u0, u1, u2) of neighbour q's 3 components (called for the active
+// positions in increasing q): the node's existing elements (those with all 8
+// nodes active) select the stencil: all 8 and gz >= 2 -> the dense interior
+// chain (c_S, structural zeros skipped), otherwise the class stencil of the
+// element set (x Dirichlet drop at gz = 1).  Shared by the gather pass and
+// the shared-memory box operator, so the two give the same bits.
+template <class LD>
+__device__ __forceinline__ void sp_fem_node(uint32_t m, int gz, const LD &ld, double (&o)[3]) {
+    int em = 0;  // existing elements: corner a of the element at node - off(a)
+#pragma unroll
+    for (int a = 0; a < 8; ++a) {
+        bool ex = true;
+#pragma unroll
+        for (int b = 0; b < 8; ++b) {
+            const int ox = (b & 1) - (a & 1), oy = ((b >> 1) & 1) - ((a >> 1) & 1), oz = ((b >> 2) & 1) - ((a >> 2) & 1);
+            ex = ex && ((m >> ((ox + 1) + 3 * (oy + 1) + 9 * (oz + 1))) & 1u);
+        }
+        em |= ex ? 1 << a : 0;
+    }
+    const bool drop = gz == 1;
+    const bool interior = em == 0xff && !drop;
+    const double *C = c_scls + (size_t)(em * 2 + (drop ? 1 : 0)) * 243;
+    double acc0 = 0.0, acc1 = 0.0, acc2 = 0.0;
+#pragma unroll
+    for (int q = 0; q < 27; ++q) {
+        if (!((m >> q) & 1u)) continue;
+        const int ox = q % 3 - 1, oy = (q / 3) % 3 - 1, oz = q / 9 - 1;
+        double u0, u1, u2;
+        ld(q, u0, u1, u2);
+        if (interior) {
+            const double *S = c_S + q * 9;
+            acc0 = fma(S[0], u0, acc0);
+            if (ox != 0 && oy != 0) acc0 = fma(S[1], u1, acc0);
+            if (ox != 0 && oz != 0) acc0 = fma(S[2], u2, acc0);
+            if (oy != 0 && ox != 0) acc1 = fma(S[3], u0, acc1);
+            acc1 = fma(S[4], u1, acc1);
+            if (oy != 0 && oz != 0) acc1 = fma(S[5], u2, acc1);
+            if (oz != 0 && ox != 0) acc2 = fma(S[6], u0, acc2);
+            if (oz != 0 && oy != 0) acc2 = fma(S[7], u1, acc2);
+            acc2 = fma(S[8], u2, acc2);
+        } else {
+            const double *K = C + q * 9;
+            acc0 = fma(__ldg(K + 0), u0, acc0);
+            acc0 = fma(__ldg(K + 1), u1, acc0);
+            acc0 = fma(__ldg(K + 2), u2, acc0);
+            acc1 = fma(__ldg(K + 3), u0, acc1);
+            acc1 = fma(__ldg(K + 4), u1, acc1);
+            acc1 = fma(__ldg(K + 5), u2, acc1);
+            acc2 = fma(__ldg(K + 6), u0, acc2);
+            acc2 = fma(__ldg(K + 7), u1, acc2);
+            acc2 = fma(__ldg(K + 8), u2, acc2);
+        }
+    }
+    o[0] = acc0;
+    o[1] = acc1;
+    o[2] = acc2;
+}
+
 struct SpFemArgs {
     const int32_t *seg;
     int64_t seg0, nseg;
@@ -1590,56 +1650,12 @@ __global__ void __launch_bounds__(256, NB_SPF_MINB) k_sp_fem(SpFemArgs A) {
             int32_t base[9];
 #pragma unroll
             for (int r = 0; r < 9; ++r) base[r] = __ldg(A.fb + (int64_t)r * A.n + j);
-            int em = 0;  // existing elements: corner a of the element at node - off(a)
-#pragma unroll
-            for (int a = 0; a < 8; ++a) {
-                bool ex = true;
-#pragma unroll
-                for (int b = 0; b < 8; ++b) {
-                    const int ox = (b & 1) - (a & 1), oy = ((b >> 1) & 1) - ((a >> 1) & 1),
-                              oz = ((b >> 2) & 1) - ((a >> 2) & 1);
-                    ex = ex && ((m >> ((ox + 1) + 3 * (oy + 1) + 9 * (oz + 1))) & 1u);
-                }
-                em |= ex ? 1 << a : 0;
-            }
-            const bool drop = gz == 1;
-            const bool interior = em == 0xff && !drop;
-            const double *C = c_scls + (size_t)(em * 2 + (drop ? 1 : 0)) * 243;
-            double acc0 = 0.0, acc1 = 0.0, acc2 = 0.0;
-#pragma unroll
-            for (int q = 0; q < 27; ++q) {
-                if (!((m >> q) & 1u)) continue;
-                const int ox = q % 3 - 1, oy = (q / 3) % 3 - 1, oz = q / 9 - 1, r = q / 3;
+            sp_fem_node(m, gz, [&](int q, double &u0, double &u1, double &u2) {
+                const int ox = q % 3 - 1, r = q / 3;
                 const uint32_t rb = (m >> (3 * r)) & 7u;
                 const int64_t idx = base[r] + __popc(rb & ((1u << (ox + 1)) - 1u));
-                const double u0 = __ldg(A.u + idx), u1 = __ldg(A.u + A.cs + idx), u2 = __ldg(A.u + 2 * A.cs + idx);
-                if (interior) {
-                    const double *S = c_S + q * 9;
-                    acc0 = fma(S[0], u0, acc0);
-                    if (ox != 0 && oy != 0) acc0 = fma(S[1], u1, acc0);
-                    if (ox != 0 && oz != 0) acc0 = fma(S[2], u2, acc0);
-                    if (oy != 0 && ox != 0) acc1 = fma(S[3], u0, acc1);
-                    acc1 = fma(S[4], u1, acc1);
-                    if (oy != 0 && oz != 0) acc1 = fma(S[5], u2, acc1);
-                    if (oz != 0 && ox != 0) acc2 = fma(S[6], u0, acc2);
-                    if (oz != 0 && oy != 0) acc2 = fma(S[7], u1, acc2);
-                    acc2 = fma(S[8], u2, acc2);
-                } else {
-                    const double *K = C + q * 9;
-                    acc0 = fma(__ldg(K + 0), u0, acc0);
-                    acc0 = fma(__ldg(K + 1), u1, acc0);
-                    acc0 = fma(__ldg(K + 2), u2, acc0);
-                    acc1 = fma(__ldg(K + 3), u0, acc1);
-                    acc1 = fma(__ldg(K + 4), u1, acc1);
-                    acc1 = fma(__ldg(K + 5), u2, acc1);
-                    acc2 = fma(__ldg(K + 6), u0, acc2);
-                    acc2 = fma(__ldg(K + 7), u1, acc2);
-                    acc2 = fma(__ldg(K + 8), u2, acc2);
-                }
-            }
-            o[0] = acc0;
-            o[1] = acc1;
-            o[2] = acc2;
+                u0 = __ldg(A.u + idx), u1 = __ldg(A.u + A.cs + idx), u2 = __ldg(A.u + 2 * A.cs + idx);
+            }, o);
         }
 #pragma unroll
         for (int c = 0; c < 3; ++c) {
@@ -1700,6 +1716,241 @@ nb_status nb_sparse_fem_pass(nb_grid *g, int p, int kind, const int32_t *list, c
     return nb_launch_check(name);
 }
 
+
+// ---- the sparse FEM operator from shared-memory boxes ----------------------
+// The gather pass above issues 81 dependent-address loads per node, nearly
+// all L1 misses (the 9 neighbour rows x 3 components of a warp span ~10 KB),
+// so it streams ~30x its algorithmic bytes through L2.  Here a CTA owns a
+// 32 x 8 tile of a z-chunk (the dense kernels' decomposition of the bounding
+// box; only tiles holding an active node are launched) and stages, per
+// plane, the 34 x 10 box around the tile x 3 components from the compact
+// arrays into a shared-memory ring with 8-byte cp.async (zero-fill for
+// inactive cells), together with the box rows' activity bits.  A box cell's
+// buffer index is its row word's index plus a popcount (nb_sparse_fem_box_
+// tables).  Output plane k is computed when planes k-1 .. k+1 have landed,
+// by sp_fem_node over the staged values: the gather pass's arithmetic, so
+// the same bits.  Each value is read from DRAM once (ring rows from L2).
+#ifndef NB_SFB_NST
+#define NB_SFB_NST 5  // ring stages: planes k-1 .. k+1 in use, k+2, k+3 in flight
+#endif
+#ifndef NB_SFB_ZC
+#define NB_SFB_ZC 16  // output planes per CTA
+#endif
+#ifndef NB_SFB_MINB
+#define NB_SFB_MINB 4
+#endif
+static_assert(NB_SFB_NST >= 4, "the box ring holds planes k-1 .. k+1 and one in flight");
+#define SFB_W 34
+#define SFB_H 10
+#define SFB_C (SFB_W * SFB_H)
+
+struct SpFemBoxArgs {
+    const int4 *items;
+    const uint32_t *rm;
+    const int32_t *ri;
+    int rw, nx, ny, gz0;
+    int64_t cs;
+    const double *u, *b;
+    double *y;
+    const CgScal *sc;
+};
+
+__device__ __forceinline__ void sfb_cp8(double *dst, const double *src, bool on) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(d), "l"(src), "r"(on ? 8 : 0) : "memory");
+}
+
+template <int KIND>  // 0: y = K u; 2: y = b - K u
+__global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A) {
+    __shared__ __align__(16) double S[NB_SFB_NST][3][SFB_C];
+    __shared__ uint64_t RB[NB_SFB_NST][SFB_H];
+    if (A.sc && A.sc->status != 0) return;
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const int4 it = A.items[blockIdx.x];
+    const int x0 = it.x * 32, y0 = it.y * 8, zs = it.z, ze = it.w;
+    const int np = ze - zs + 2;  // staged planes zs-1 .. ze
+    const int wx = it.x;         // the tile's x word
+    // stage plane pl (local plane zs - 1 + pl) into ring slot pl % NST
+    auto issue = [&](int pl) {
+        const int st = pl % NB_SFB_NST;
+        const int64_t row0 = (int64_t)(zs + pl) * A.ny;  // slab row of (zl + 1, y = 0)
+        for (int e = tid; e < SFB_C; e += 256) {
+            const int bx = e % SFB_W, by = e / SFB_W;
+            const int x = x0 - 1 + bx, yy = y0 - 1 + by;
+            int64_t idx = 0;
+            bool act = false;
+            if (x >= 0 && x < A.nx && yy >= 0 && yy < A.ny) {
+                const int64_t k = (row0 + yy) * A.rw + (x >> 5);
+                const uint32_t m = __ldg(A.rm + k);
+                const unsigned b = (unsigned)x & 31u;
+                act = (m >> b) & 1u;
+                idx = __ldg(A.ri + k) + __popc(m & ((1u << b) - 1u));
+            }
+#pragma unroll
+            for (int c = 0; c < 3; ++c) sfb_cp8(&S[st][c][e], A.u + c * A.cs + idx, act);
+        }
+        if (tid < SFB_H) {  // activity bits of box row tid: bit i = x0 - 1 + i
+            const int yy = y0 - 1 + tid;
+            uint64_t bits = 0;
+            if (yy >= 0 && yy < A.ny) {
+                const uint32_t *r = A.rm + (row0 + yy) * A.rw;
+                const uint64_t lo = wx > 0 ? __ldg(r + wx - 1) >> 31 : 0u;
+                const uint64_t hi = wx + 1 < A.rw ? __ldg(r + wx + 1) & 1u : 0u;
+                bits = lo | ((uint64_t)__ldg(r + wx) << 1) | (hi << 33);
+            }
+            RB[st][tid] = bits;
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+#pragma unroll 1
+    for (int pl = 0; pl < NB_SFB_NST - 1; ++pl) {
+        if (pl < np) issue(pl);
+        else asm volatile("cp.async.commit_group;" ::: "memory");
+    }
+    const int x = x0 + lane, y = y0 + w;
+    const bool in = x < A.nx && y < A.ny;
+#pragma unroll 1
+    for (int o = 0; o < ze - zs; ++o) {
+        // planes o .. o+2 are needed; o+3 .. o+NST-2 may stay in flight
+        asm volatile("cp.async.wait_group %0;" ::"n"(NB_SFB_NST - 4) : "memory");
+        __syncthreads();  // every thread's copies landed; plane o-1's slot is free
+        if (o + NB_SFB_NST - 1 < np) issue(o + NB_SFB_NST - 1);
+        else asm volatile("cp.async.commit_group;" ::: "memory");
+        const int zl = zs + o;
+        const int s0 = o % NB_SFB_NST, s1 = (o + 1) % NB_SFB_NST, s2 = (o + 2) % NB_SFB_NST;
+        if (!in || !((RB[s1][w + 1] >> (lane + 1)) & 1u)) continue;
+        const int gz = A.gz0 + zl;
+        double out[3];
+        if (gz == 0) {  // Dirichlet identity row
+#pragma unroll
+            for (int c = 0; c < 3; ++c) out[c] = S[s1][c][(w + 1) * SFB_W + lane + 1];
+        } else {
+            uint32_t m = 0;
+#pragma unroll
+            for (int r = 0; r < 9; ++r) {
+                const int oy = r % 3 - 1, oz = r / 3 - 1;
+                const int st = oz < 0 ? s0 : (oz == 0 ? s1 : s2);
+                m |= (uint32_t)((RB[st][w + 1 + oy] >> lane) & 7u) << (3 * r);
+            }
+            sp_fem_node(m, gz, [&](int q, double &u0, double &u1, double &u2) {
+                const int ox = q % 3 - 1, oy = (q / 3) % 3 - 1, oz = q / 9 - 1;
+                const int st = oz < 0 ? s0 : (oz == 0 ? s1 : s2);
+                const int e = (w + 1 + oy) * SFB_W + lane + 1 + ox;
+                u0 = S[st][0][e], u1 = S[st][1][e], u2 = S[st][2][e];
+            }, out);
+        }
+        const int64_t k = ((int64_t)(zl + 1) * A.ny + y) * A.rw + wx;
+        const int64_t i = __ldg(A.ri + k) + __popc(__ldg(A.rm + k) & ((1u << lane) - 1u));
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+            const int64_t kk = c * A.cs + i;
+            A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], out[c]) : out[c];
+        }
+    }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+}
+
+// per-segment partials of <a, b> (3 components): k_sp_fem's dot, bit for bit
+__global__ void __launch_bounds__(256) k_sp_fem_dot(const int32_t *__restrict__ seg, const int64_t *__restrict__ pstart,
+                                                   int64_t hl, int64_t cs, int gz0, int NZ, int T, double *tp,
+                                                   const double *__restrict__ a, const double *__restrict__ b,
+                                                   const CgScal *sc) {
+    __shared__ double sw[3][8];
+    const int t = threadIdx.x;
+    const int e = __ldg(seg + blockIdx.x);
+    const int zl = e >> 16, sg = e & 0xffff;
+    const int64_t j = __ldg(pstart + zl) + (int64_t)sg * 256 + t;
+    const bool valid = j < __ldg(pstart + zl + 1);
+    if (sc && sc->status != 0) return;
+    double prod[3] = {0.0, 0.0, 0.0};
+    if (valid) {
+        const int64_t i = hl + j;
+#pragma unroll
+        for (int c = 0; c < 3; ++c) prod[c] = __dmul_rn(__ldcs(a + c * cs + i), __ldcs(b + c * cs + i));
+    }
+    const int w = t >> 5;
+    warp_sums_store<3>(prod, t & 31, &sw[0][w], 8);
+    __syncthreads();
+    if (t < 3) {
+        double s = sw[t][0];
+#pragma unroll
+        for (int ww = 1; ww < 8; ++ww) s = __dadd_rn(s, sw[t][ww]);
+        tp[((int64_t)t * NZ + gz0 + zl) * T + sg] = s;
+    }
+}
+
+bool nb_sparse_fem_boxed() { return !getenv("NB_SPF_GATHER"); }
+
+nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> &ranges, const double *u,
+                            const double *b, double *y, const CgScal *sc) {
+    const int4 *items = nullptr;
+    int64_t n = 0;
+    NB_TRY(nb_sparse_fem_box_list(g, p, ranges, NB_SFB_ZC, &items, &n));
+    if (n <= 0) return NB_OK;
+    const NbSparsePart &sp = g->sp[p];
+    SpFemBoxArgs A{};
+    A.items = items;
+    A.rm = sp.d_rm;
+    A.ri = sp.d_ri;
+    A.rw = sp.rw;
+    A.nx = g->nx;
+    A.ny = g->ny;
+    A.gz0 = g->parts[p].z0;
+    A.cs = sp.cs;
+    A.u = u;
+    A.b = b;
+    A.y = y;
+    A.sc = sc;
+    const char *name = kind == 2 ? "k_fem_cg_init" : (sc ? "k_sp_fem_q" : "k_fem_apply");
+    LaunchScope ls(g, g->cs, name);
+    if (kind == 2)
+        k_sp_fem_box<2><<<(unsigned)n, 256, 0, g->cs>>>(A);
+    else
+        k_sp_fem_box<0><<<(unsigned)n, 256, 0, g->cs>>>(A);
+    return nb_launch_check(name);
+}
+
+nb_status nb_sparse_fem_dot(nb_grid *g, int p, const double *a, const double *b, const CgScal *sc) {
+    const NbSparsePart &sp = g->sp[p];
+    const int64_t nseg = sp.seg_start.back();
+    if (nseg <= 0) return NB_OK;
+    LaunchScope ls(g, g->cs, "k_sp_fem_dot");
+    k_sp_fem_dot<<<(unsigned)nseg, 256, 0, g->cs>>>(sp.d_seg, sp.d_pstart, sp.hl, sp.cs, g->parts[p].z0, g->nz, g->T,
+                                                    g->tp, a, b, sc);
+    return nb_launch_check("k_sp_fem_dot");
+}
+
+// local plane ranges of partition p: 0 = all, 1 = the interior (planes whose
+// neighbours are own planes), 2 = the boundary planes facing a neighbour
+static std::vector<int> sp_box_ranges(const nb_grid *g, int p, int which) {
+    const NbPart &q = g->parts[p];
+    const int nz = q.nz();
+    if (which == 0) return {0, nz};
+    const int ib = q.lo >= 0 ? 1 : 0, ie = std::max(ib, nz - (q.hi >= 0 ? 1 : 0));
+    if (which == 1) return {ib, ie};
+    std::vector<int> r;
+    if (q.lo >= 0) r.insert(r.end(), {0, 1});
+    if (q.hi >= 0 && ie < nz) r.insert(r.end(), {nz - 1, nz});
+    return r;
+}
+
+nb_status nb_sparse_fem_box_ranges(nb_grid *g, int p, int which, const double *u, const double *b, double *y,
+                                   const CgScal *sc, int kind) {
+    return nb_sparse_fem_box(g, p, kind, sp_box_ranges(g, p, which), u, b, y, sc);
+}
+
+// build the tables and every list the CG / apply use (outside any capture)
+nb_status nb_sparse_fem_box_prepare(nb_grid *g) {
+    NB_TRY(nb_sparse_fem_box_tables(g));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+        for (int which = 0; which < 3; ++which) {
+            const int4 *it;
+            int64_t n;
+            NB_TRY(nb_sparse_fem_box_list(g, p, sp_box_ranges(g, p, which), NB_SFB_ZC, &it, &n));
+        }
+    return NB_OK;
+}
+
 nb_status nb_sparse_fem_rhs(nb_field *b, double pr);
 
 static nb_status fem_check(const nb_field *u) {
@@ -1717,11 +1968,16 @@ extern "C" nb_status nb_fem27_apply(const nb_field *u, nb_field *y, double E, do
     cudaSetDevice(g->device);
     NB_TRY(fem_upload_constants(E, nu));
     if (g->sparse) {
-        NB_TRY(nb_sparse_fem_tables(g));
+        const bool box = nb_sparse_fem_boxed();
+        NB_TRY(box ? nb_sparse_fem_box_prepare(g) : nb_sparse_fem_tables(g));
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
             const NbSparsePart &sp = g->sp[p];
-            NB_TRY(nb_sparse_fem_pass(g, p, 0, sp.d_seg, nullptr, 0, sp.seg_start.back(),
-                                      (const double *)u->base[p], nullptr, (double *)y->base[p], nullptr));
+            if (box)
+                NB_TRY(nb_sparse_fem_box_ranges(g, p, 0, (const double *)u->base[p], nullptr, (double *)y->base[p],
+                                                nullptr, 0));
+            else
+                NB_TRY(nb_sparse_fem_pass(g, p, 0, sp.d_seg, nullptr, 0, sp.seg_start.back(),
+                                          (const double *)u->base[p], nullptr, (double *)y->base[p], nullptr));
         }
         return NB_OK;
     }
@@ -1773,11 +2029,19 @@ nb_status nb_fem_cg_init(nb_cg *cg) {
     NB_TRY(fem_upload_constants(cg->prm.fem_E, cg->prm.fem_nu));
     if (g->sparse) {
         NB_TRY(nb_sparse_fem_tables(g));
+        const bool box = nb_sparse_fem_boxed();
+        if (box) NB_TRY(nb_sparse_fem_box_prepare(g));  // the q pass's lists, before any capture
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
             const NbSparsePart &sp = g->sp[p];
-            NB_TRY(nb_sparse_fem_pass(g, p, 2, sp.d_seg, nullptr, 0, sp.seg_start.back(),
-                                      (const double *)cg->x->base[p], (const double *)cg->b->base[p],
-                                      (double *)cg->r->base[p], nullptr));
+            double *r = (double *)cg->r->base[p];
+            if (box) {
+                NB_TRY(nb_sparse_fem_box_ranges(g, p, 0, (const double *)cg->x->base[p],
+                                                (const double *)cg->b->base[p], r, nullptr, 2));
+                NB_TRY(nb_sparse_fem_dot(g, p, r, r, nullptr));
+            } else {
+                NB_TRY(nb_sparse_fem_pass(g, p, 2, sp.d_seg, nullptr, 0, sp.seg_start.back(),
+                                          (const double *)cg->x->base[p], (const double *)cg->b->base[p], r, nullptr));
+            }
         }
         return nb_reduce_finalize(g, 3, FIN_CG_INIT, cg->sc, 0);
     }

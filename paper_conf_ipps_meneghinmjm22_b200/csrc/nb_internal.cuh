@@ -167,6 +167,17 @@ struct NbSparsePart {
     // 3(oz+1), -1 if none (active cells of a row are consecutive indices)
     uint32_t *d_fm = nullptr;
     int32_t *d_fb = nullptr;
+    // FEM box tables (lazy, nb_sparse_fem_box_tables): per slab row
+    // (zl + 1, y), zl in [-1, nz], and 32-cell x word w: d_rm = activity
+    // bits, d_ri = buffer index the word's first active cell has (or would
+    // have); rw words per row.  tile_any[zl][ty][tx]: the 32 x 8 tile of
+    // own plane zl holds an active node.  box_lists: (tile, z-chunk) work
+    // items {tx, ty, zs, ze} per set of plane ranges
+    uint32_t *d_rm = nullptr;
+    int32_t *d_ri = nullptr;
+    int rw = 0;
+    std::vector<uint8_t> tile_any;
+    std::map<std::vector<int>, std::pair<int4 *, int64_t>> box_lists;
 };
 
 struct nb_grid {
@@ -455,6 +466,24 @@ nb_status nb_sparse_fem_tables(nb_grid *g);
 // kind: 0 = y = K u, 1 = q = K u with <u, q>, 2 = y = b - K u with <y, y>
 nb_status nb_sparse_fem_pass(nb_grid *g, int p, int kind, const int32_t *list, const int32_t *gidx, int64_t s0,
                              int64_t n, const double *u, const double *b, double *y, const CgScal *sc);
+// the same operator from shared-memory boxes (k_sp_fem_box): the output
+// planes of the local plane ranges {zb0, ze0, zb1, ze1, ...} of partition p.
+// kind: 0 = y = K u, 2 = y = b - K u (no dot: nb_sparse_fem_dot); sc != NULL
+// makes it a no-op once the solver stopped.  Same values as the gather pass.
+bool nb_sparse_fem_boxed();  // the box operator is the default (NB_SPF_GATHER=1: the gather pass)
+nb_status nb_sparse_fem_box_tables(nb_grid *g);
+nb_status nb_sparse_fem_box_list(nb_grid *g, int p, const std::vector<int> &ranges, int zc, const int4 **items,
+                                 int64_t *n);
+nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> &ranges, const double *u,
+                            const double *b, double *y, const CgScal *sc);
+// per-segment partials of <a, b> over the 3 components of partition p (the
+// gather pass's dot, bit for bit), all segments
+nb_status nb_sparse_fem_dot(nb_grid *g, int p, const double *a, const double *b, const CgScal *sc);
+// the box operator over local planes: which = 0 all, 1 the interior (planes
+// whose neighbours are own planes), 2 the boundary planes facing a neighbour
+nb_status nb_sparse_fem_box_ranges(nb_grid *g, int p, int which, const double *u, const double *b, double *y,
+                                   const CgScal *sc, int kind);
+nb_status nb_sparse_fem_box_prepare(nb_grid *g);  // tables + every list (call outside graph capture)
 nb_status nb_nccl_allreduce_sum(nb_grid *g, const double *send, double *recv, size_t n,
                                 cudaStream_t s);
 nb_status nb_nccl_group(nb_grid *g, bool start);

@@ -51,6 +51,13 @@ void nb_sparse_free(nb_grid *g) {
         cudaFree(s.d_fb);
         s.d_fm = nullptr;
         s.d_fb = nullptr;
+        cudaFree(s.d_rm);
+        cudaFree(s.d_ri);
+        s.d_rm = nullptr;
+        s.d_ri = nullptr;
+        s.tile_any.clear();
+        for (auto &kv : s.box_lists) cudaFree(kv.second.first);
+        s.box_lists.clear();
         s.d_seg_bnd = s.d_seg_bnd_gi = nullptr;
         s.d_nbr = s.d_seginfo = nullptr;
         s.n_runs = 0;
@@ -1347,6 +1354,105 @@ nb_status nb_sparse_fem_tables(nb_grid *g) {
     return NB_OK;
 }
 
+// Box tables of the shared-memory FEM operator (nb_fem.cu k_sp_fem_box):
+// a CTA stages the 34 x 10 box of each plane around its 32 x 8 tile from the
+// compact arrays.  A box cell's buffer index is that of its row word's first
+// cell position plus the active cells before it in the word (a popcount), so
+// per (slab row, 32-cell word) the table holds the activity bits and that
+// index: 8 B per 32 cells, built here on the host from the mask.
+nb_status nb_sparse_fem_box_tables(nb_grid *g) {
+    if (!g->sparse) return NB_OK;
+    DeviceGuard dg(g->device);
+    const int nx = g->nx, ny = g->ny;
+    const int64_t plane = (int64_t)nx * ny;
+    const int rw = (nx + 31) / 32, tx = rw, ty = (ny + 7) / 8;
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        NbSparsePart &sp = g->sp[p];
+        if (sp.d_rm) continue;
+        const NbPart &q = g->parts[p];
+        const int nzl = q.nz();
+        if (sp.hl + sp.n + sp.hh >= ((int64_t)1 << 31))
+            NB_FAIL(NB_EUNSUPPORTED, "sparse FEM box tables: more than 2^31 cells in a slab");
+        const int64_t nrow = (int64_t)(nzl + 2) * ny;
+        std::vector<uint32_t> rm((size_t)(nrow * rw), 0u);
+        std::vector<int32_t> ri((size_t)(nrow * rw), 0);
+        sp.tile_any.assign((size_t)nzl * ty * tx, 0);
+        for (int s = 0; s < nzl + 2; ++s) {
+            const int zl = s - 1, gz = q.z0 + zl;
+            int64_t idx;
+            if (zl == -1) {
+                if (q.lo < 0) continue;
+                idx = 0;
+            } else if (zl == nzl) {
+                if (q.hi < 0) continue;
+                idx = sp.hl + sp.n;
+            } else {
+                idx = sp.hl + sp.pstart[zl];
+            }
+            const uint8_t *m = g->host_mask.data() + (int64_t)gz * plane;
+            for (int y = 0; y < ny; ++y) {
+                const uint8_t *row = m + (int64_t)y * nx;
+                const int64_t k0 = ((int64_t)s * ny + y) * rw;
+                for (int w = 0; w < rw; ++w) {
+                    ri[k0 + w] = (int32_t)idx;
+                    uint32_t bits = 0;
+                    const int xe = std::min(nx, 32 * w + 32);
+                    for (int x = 32 * w; x < xe; ++x)
+                        if (row[x]) {
+                            bits |= 1u << (x - 32 * w);
+                            ++idx;
+                        }
+                    rm[k0 + w] = bits;
+                    if (bits && zl >= 0 && zl < nzl) sp.tile_any[((size_t)zl * ty + y / 8) * tx + w] = 1;
+                }
+            }
+        }
+        NB_CUDA(cudaMalloc(&sp.d_rm, sizeof(uint32_t) * rm.size()));
+        NB_CUDA(cudaMalloc(&sp.d_ri, sizeof(int32_t) * ri.size()));
+        NB_CUDA(cudaMemcpy(sp.d_rm, rm.data(), sizeof(uint32_t) * rm.size(), cudaMemcpyHostToDevice));
+        NB_CUDA(cudaMemcpy(sp.d_ri, ri.data(), sizeof(int32_t) * ri.size(), cudaMemcpyHostToDevice));
+        sp.rw = rw;
+    }
+    return NB_OK;
+}
+
+// work items {tile x, tile y, zs, ze}: every (tile, chunk of <= zc planes) of
+// the local plane ranges holding an active node, chunk-major (neighbouring
+// tiles of a chunk run together and share their ring rows in L2); cached
+nb_status nb_sparse_fem_box_list(nb_grid *g, int p, const std::vector<int> &ranges, int zc, const int4 **items,
+                                 int64_t *n) {
+    NB_TRY(nb_sparse_fem_box_tables(g));
+    NbSparsePart &sp = g->sp[p];
+    std::vector<int> key = ranges;
+    key.push_back(zc);
+    auto it = sp.box_lists.find(key);
+    if (it == sp.box_lists.end()) {
+        const int tx = (g->nx + 31) / 32, ty = (g->ny + 7) / 8;
+        std::vector<int4> v;
+        for (size_t r = 0; r + 1 < ranges.size(); r += 2)
+            for (int zs = ranges[r]; zs < ranges[r + 1]; zs += zc) {
+                const int ze = std::min(zs + zc, ranges[r + 1]);
+                for (int by = 0; by < ty; ++by)
+                    for (int bx = 0; bx < tx; ++bx) {
+                        bool any = false;
+                        for (int zl = zs; zl < ze && !any; ++zl)
+                            any = sp.tile_any[((size_t)zl * ty + by) * tx + bx] != 0;
+                        if (any) v.push_back(make_int4(bx, by, zs, ze));
+                    }
+            }
+        int4 *d = nullptr;
+        if (!v.empty()) {
+            DeviceGuard dg(g->device);
+            NB_CUDA(cudaMalloc(&d, sizeof(int4) * v.size()));
+            NB_CUDA(cudaMemcpy(d, v.data(), sizeof(int4) * v.size(), cudaMemcpyHostToDevice));
+        }
+        it = sp.box_lists.emplace(key, std::make_pair(d, (int64_t)v.size())).first;
+    }
+    *items = it->second.first;
+    *n = it->second.second;
+    return NB_OK;
+}
+
 // consistent nodal load of pressure pr on the exposed top faces (+z) of the
 // existing elements (oracle or_fem_rhs with a mask): a node gets pr/4 from
 // each existing element below it whose top face is exposed (no existing
@@ -1423,6 +1529,19 @@ nb_status nb_sparse_fem_cg_hooks(nb_cg *cg) {
         return nb_sparse_fem_pass(g, p, 1, list, gi, s0, n, (const double *)p_->base[p], nullptr,
                                   (double *)cg->q->base[p], cg->sc);
     };
+    // box operator (default): q = K p over plane ranges (which: 0 all, 1
+    // interior, 2 boundary planes), then <p, q> per segment in one pass
+    const bool box = nb_sparse_fem_boxed();
+    auto qbox = [&](int p, int which) {
+        return nb_sparse_fem_box_ranges(g, p, which, (const double *)p_->base[p], nullptr, (double *)cg->q->base[p],
+                                        cg->sc, 0);
+    };
+    auto qdot = [&]() -> nb_status {
+        if (box)
+            for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+                NB_TRY(nb_sparse_fem_dot(g, p, (const double *)p_->base[p], (const double *)cg->q->base[p], cg->sc));
+        return NB_OK;
+    };
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         const NbSparsePart &sp = g->sp[p];
         for (int c = 0; c < 3; ++c) {
@@ -1436,7 +1555,7 @@ nb_status nb_sparse_fem_cg_hooks(nb_cg *cg) {
         NB_TRY(nb_sparse_halo_update(p_));
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
             const NbSparsePart &sp = g->sp[p];
-            NB_TRY(qpass(p, sp.d_seg, nullptr, 0, sp.seg_start.back()));
+            NB_TRY(box ? qbox(p, 0) : qpass(p, sp.d_seg, nullptr, 0, sp.seg_start.back()));
         }
     } else {
         NB_TRY(nb_halo_split_begin(p_, 0, 3, cg->hs));
@@ -1446,14 +1565,15 @@ nb_status nb_sparse_fem_cg_hooks(nb_cg *cg) {
             const int ib = q.lo >= 0 ? 1 : 0, ie = std::max(ib, q.nz() - (q.hi >= 0 ? 1 : 0));
             for (int c = 0; c < 3; ++c)
                 NB_TRY(sp_launch<SPK_CG_MAP>(g, p, ib, ie, map_args(p, c), 0, "k_sp_cg_map"));
-            NB_TRY(qpass(p, sp.d_seg, nullptr, sp.seg_start[ib], sp.seg_start[ie] - sp.seg_start[ib]));
+            NB_TRY(box ? qbox(p, 1) : qpass(p, sp.d_seg, nullptr, sp.seg_start[ib], sp.seg_start[ie] - sp.seg_start[ib]));
         }
         NB_TRY(nb_halo_split_wait(g, cg->hs));
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
             const NbSparsePart &sp = g->sp[p];
-            NB_TRY(qpass(p, sp.d_seg_bnd, sp.d_seg_bnd_gi, 0, sp.n_seg_bnd));
+            NB_TRY(box ? qbox(p, 2) : qpass(p, sp.d_seg_bnd, sp.d_seg_bnd_gi, 0, sp.n_seg_bnd));
         }
     }
+    NB_TRY(qdot());
     NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
         for (int c = 0; c < 3; ++c) {

@@ -114,3 +114,61 @@ def test_sparse_fem_cg_converges():
     res = oracle.fem_apply(x, 1.0, 0.3, mask=m) - b
     assert np.max(np.abs(res)) <= 1e-8 * np.max(np.abs(b))
     assert np.all(x[:, 0] == 0.0)
+
+
+def _run_both(fn):
+    """fn() under the shared-memory box operator (default) and the gather
+    pass (NB_SPF_GATHER=1)."""
+    import os
+    outs = []
+    for gather in (False, True):
+        if gather:
+            os.environ["NB_SPF_GATHER"] = "1"
+        try:
+            outs.append(fn())
+        finally:
+            os.environ.pop("NB_SPF_GATHER", None)
+    return outs
+
+
+@pytest.mark.parametrize("name", ["sphere", "holes", "step", "wide"])
+@pytest.mark.parametrize("parts", [1, 2, 3])
+def test_sparse_fem_box_equals_gather_bitwise(name, parts):
+    """The shared-memory box operator (k_sp_fem_box: 32 x 8 tiles, z-chunks,
+    ragged x / y tiles) and the gather pass compute the same K u and the
+    same CG iterates bit for bit (same per-node arithmetic, same dot)."""
+    if name == "wide":  # several tiles in x and y, a ragged last tile, > 1 z-chunk
+        m = synth.sphere_mask(70, 0.45)[:, :45, :]
+        m = np.ascontiguousarray(m[:40])
+    else:
+        m = masks()[name]
+    nz, ny, nx = m.shape
+    u = synth.uniform((nx, ny, nz), card=3, seed=11) * m[None]
+
+    def apply():
+        with sgrid(m, parts) as g:
+            fu, fy = nb.Field(g, card=3), nb.Field(g, card=3)
+            fu.upload(u)
+            fu.halo_update()
+            nb.nb_fem27_apply(fu, fy)
+            y = fy.download()
+            fu.close(), fy.close()
+        return y
+
+    ya, yb = _run_both(apply)
+    assert np.array_equal(ya, yb)
+    yo = oracle.fem_apply(u, 1.0, 0.3, mask=m)
+    assert np.max(np.abs(ya - yo)) <= 1e-13 * max(np.max(np.abs(yo)), 1.0)
+
+    def cg():
+        with sgrid(m, parts) as g:
+            fb, fx = nb.Field(g, card=3), nb.Field(g, card=3)
+            nb.nb_fem27_rhs(fb, 1.0)
+            fx.fill_const(0.0)
+            r = nb.nb_cg_solve(fx, fb, max_iter=9, op=nb.OP_FEM27, occ=nb.OCC_TWO_WAY)
+            x = fx.download()
+            fb.close(), fx.close()
+        return x, r.rr, r.iters
+
+    (xa, rra, ia), (xb, rrb, ib) = _run_both(cg)
+    assert ia == ib and rra == rrb and np.array_equal(xa, xb)

@@ -1,0 +1,64 @@
+"""A/B of the sparse FEM operator: shared-memory box (default) vs the gather
+pass (NB_SPF_GATHER=1): per-kernel times of one CG iteration (profiled,
+eager) and the CG iteration time (graph), 384^3 full cube and the C4-style
+sphere, plus a bitwise check of the iterates.  Usage: python tools/sparse_fem_box_ab.py [N]"""
+import hashlib
+import json
+import os
+import sys
+
+sys.path.insert(0, os.getcwd())
+import numpy as np
+import torch
+
+import paper_conf_ipps_meneghinmjm22_b200 as nb
+import synth
+
+N = int(sys.argv[1]) if len(sys.argv) > 1 else 384
+KS = ("k_sp_fem_q", "k_sp_fem_dot", "k_sp_cg_map", "k_sp_cg_r", "k_finalize")
+
+
+def run(mask, gather, iters=10):
+    if gather:
+        os.environ["NB_SPF_GATHER"] = "1"
+    else:
+        os.environ.pop("NB_SPF_GATHER", None)
+    g = nb.Grid((N, N, N), active=mask)
+    b, x = nb.Field(g, card=3), nb.Field(g, card=3)
+    nb.nb_fem27_rhs(b, 1.0)
+    x.fill_const(0.0)
+    cg = nb.CG(x, b, op=nb.OP_FEM27)
+    cg.iterate(3)
+    cg.prepare(iters)
+    g.sync()
+    s = torch.cuda.ExternalStream(g.stream())
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    cg.iterate(iters)
+    e1.record(s)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / iters
+    g.profile(True)
+    cg.iterate(2)
+    prof = {k: g.profile_read(k)[1] / 2 for k in KS}
+    g.profile(False)
+    cg.finish()
+    dig = hashlib.sha1(x.download().tobytes()).hexdigest()[:12]
+    cg.close(), b.close(), x.close(), g.close()
+    return {"ms_per_iter": ms, "kernel_ms": prof, "x_digest": dig}
+
+
+out = {"N": N}
+for name, mask in (("full", np.ones((N, N, N), np.uint8)), ("sphere", synth.sphere_mask(N))):
+    act = int(mask.sum())
+    r = {"active": act}
+    for mode in ("box", "gather"):
+        r[mode] = run(mask, mode == "gather")
+    r["same_bits"] = r["box"]["x_digest"] == r["gather"]["x_digest"]
+    q_box = r["box"]["kernel_ms"]["k_sp_fem_q"] + r["box"]["kernel_ms"]["k_sp_fem_dot"]
+    r["q_box_ms"] = q_box
+    r["q_box_frac_hbm_48B"] = 48 * act / (r["box"]["kernel_ms"]["k_sp_fem_q"] / 1e3) / 1e9 / 6451.8
+    out[name] = r
+    print(name, json.dumps(r), flush=True)
+os.makedirs("gpurun_out", exist_ok=True)
+json.dump(out, open("gpurun_out/sparse_fem_box_ab.json", "w"), indent=1)
