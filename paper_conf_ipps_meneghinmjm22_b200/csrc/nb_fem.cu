@@ -1551,6 +1551,33 @@ static nb_status fem_launch(nb_grid *g, int p, FemArgs A, const nb_field *f, int
 // identity row.  A full mask therefore reproduces the dense operator bit for
 // bit; general masks are the oracle's element-by-element K (tolerance).
 // ===========================================================================
+// the interior chain of sp_fem_node: q = 0 .. 26, per q the 9 block
+// entries S[q][i][j] = sign * c_cv[class] in (i, j) order, structural zeros
+// skipped (fem_cv_class < 0) — bitwise the c_S chain, with every coefficient
+// a compile-time constant-bank operand
+template <int I, int J, int Q>
+__device__ __forceinline__ void sp_fem_cfma(double u, double &acc) {
+    constexpr int k = fem_cv_class(Q, I, J);
+    if constexpr (k >= 0) acc = fma(fem_cv_sign(Q, I, J) > 0 ? c_cv[k] : -c_cv[k], u, acc);
+}
+template <int Q, class LD>
+__device__ __forceinline__ void sp_fem_interior(const LD &ld, double &acc0, double &acc1, double &acc2) {
+    if constexpr (Q < 27) {
+        double u0, u1, u2;
+        ld(Q, u0, u1, u2);
+        sp_fem_cfma<0, 0, Q>(u0, acc0);
+        sp_fem_cfma<0, 1, Q>(u1, acc0);
+        sp_fem_cfma<0, 2, Q>(u2, acc0);
+        sp_fem_cfma<1, 0, Q>(u0, acc1);
+        sp_fem_cfma<1, 1, Q>(u1, acc1);
+        sp_fem_cfma<1, 2, Q>(u2, acc1);
+        sp_fem_cfma<2, 0, Q>(u0, acc2);
+        sp_fem_cfma<2, 1, Q>(u1, acc2);
+        sp_fem_cfma<2, 2, Q>(u2, acc2);
+        sp_fem_interior<Q + 1>(ld, acc0, acc1, acc2);
+    }
+}
+
 // y_n of an active node off the Dirichlet plane (gz >= 1) from its
 // 27-neighbourhood mask m (bit (ox+1) + 3(oy+1) + 9(oz+1)) and a loader
 // ld(q, u0, u1, u2) of neighbour q's 3 components (called for the active
@@ -1573,27 +1600,19 @@ __device__ __forceinline__ void sp_fem_node(uint32_t m, int gz, const LD &ld, do
         em |= ex ? 1 << a : 0;
     }
     const bool drop = gz == 1;
-    const bool interior = em == 0xff && !drop;
-    const double *C = c_scls + (size_t)(em * 2 + (drop ? 1 : 0)) * 243;
     double acc0 = 0.0, acc1 = 0.0, acc2 = 0.0;
+    if (em == 0xff && !drop) {
+        // interior: all 27 neighbours active; its own branch keeps the
+        // compiler from if-converting the two chains into one predicated
+        // sequence (measured: both chains' DFMAs and loads issued per node)
+        sp_fem_interior<0>(ld, acc0, acc1, acc2);
+    } else {
+        const double *C = c_scls + (size_t)(em * 2 + (drop ? 1 : 0)) * 243;
 #pragma unroll
-    for (int q = 0; q < 27; ++q) {
-        if (!((m >> q) & 1u)) continue;
-        const int ox = q % 3 - 1, oy = (q / 3) % 3 - 1, oz = q / 9 - 1;
-        double u0, u1, u2;
-        ld(q, u0, u1, u2);
-        if (interior) {
-            const double *S = c_S + q * 9;
-            acc0 = fma(S[0], u0, acc0);
-            if (ox != 0 && oy != 0) acc0 = fma(S[1], u1, acc0);
-            if (ox != 0 && oz != 0) acc0 = fma(S[2], u2, acc0);
-            if (oy != 0 && ox != 0) acc1 = fma(S[3], u0, acc1);
-            acc1 = fma(S[4], u1, acc1);
-            if (oy != 0 && oz != 0) acc1 = fma(S[5], u2, acc1);
-            if (oz != 0 && ox != 0) acc2 = fma(S[6], u0, acc2);
-            if (oz != 0 && oy != 0) acc2 = fma(S[7], u1, acc2);
-            acc2 = fma(S[8], u2, acc2);
-        } else {
+        for (int q = 0; q < 27; ++q) {
+            if (!((m >> q) & 1u)) continue;
+            double u0, u1, u2;
+            ld(q, u0, u1, u2);
             const double *K = C + q * 9;
             acc0 = fma(__ldg(K + 0), u0, acc0);
             acc0 = fma(__ldg(K + 1), u1, acc0);
@@ -1737,9 +1756,9 @@ nb_status nb_sparse_fem_pass(nb_grid *g, int p, int kind, const int32_t *list, c
 #define NB_SFB_ZC 16  // output planes per CTA
 #endif
 #ifndef NB_SFB_MINB
-#define NB_SFB_MINB 4
+#define NB_SFB_MINB 3
 #endif
-static_assert(NB_SFB_NST >= 4, "the box ring holds planes k-1 .. k+1 and one in flight");
+static_assert(NB_SFB_NST >= 5, "the box ring: planes pl-2 .. pl read, pl+1 in flight, pl+2 issued");
 #define SFB_W 34
 #define SFB_H 10
 #define SFB_C (SFB_W * SFB_H)
@@ -1760,6 +1779,33 @@ __device__ __forceinline__ void sfb_cp8(double *dst, const double *src, bool on)
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(d), "l"(src), "r"(on ? 8 : 0) : "memory");
 }
 
+// one staged plane's 9 in-plane positions Q (3 components each, read once
+// at compile-time offsets from the node's centre P) applied to the three
+// outputs it touches: aA (q = 18 + Q), aB (q = 9 + Q), aC (q = Q)
+template <int Q>
+__device__ __forceinline__ void sfb_plane(const double *P, double (&aA)[3], double (&aB)[3], double (&aC)[3]) {
+    if constexpr (Q < 9) {
+        constexpr int e = (Q / 3 - 1) * SFB_W + (Q % 3 - 1);
+        const double u0 = P[e], u1 = P[SFB_C + e], u2 = P[2 * SFB_C + e];
+        auto blk = [&](auto qc, double (&a)[3]) {
+            constexpr int q = decltype(qc)::value;
+            sp_fem_cfma<0, 0, q>(u0, a[0]);
+            sp_fem_cfma<0, 1, q>(u1, a[0]);
+            sp_fem_cfma<0, 2, q>(u2, a[0]);
+            sp_fem_cfma<1, 0, q>(u0, a[1]);
+            sp_fem_cfma<1, 1, q>(u1, a[1]);
+            sp_fem_cfma<1, 2, q>(u2, a[1]);
+            sp_fem_cfma<2, 0, q>(u0, a[2]);
+            sp_fem_cfma<2, 1, q>(u1, a[2]);
+            sp_fem_cfma<2, 2, q>(u2, a[2]);
+        };
+        blk(std::integral_constant<int, 18 + Q>{}, aA);
+        blk(std::integral_constant<int, 9 + Q>{}, aB);
+        blk(std::integral_constant<int, Q>{}, aC);
+        sfb_plane<Q + 1>(P, aA, aB, aC);
+    }
+}
+
 template <int KIND>  // 0: y = K u; 2: y = b - K u
 __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A) {
     __shared__ __align__(16) double S[NB_SFB_NST][3][SFB_C];
@@ -1770,81 +1816,139 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
     const int x0 = it.x * 32, y0 = it.y * 8, zs = it.z, ze = it.w;
     const int np = ze - zs + 2;  // staged planes zs-1 .. ze
     const int wx = it.x;         // the tile's x word
-    // stage plane pl (local plane zs - 1 + pl) into ring slot pl % NST
+    // Staging is split in two so no thread waits on a table load: fetch(pl)
+    // loads plane pl's table words for the thread's (up to 2) box cells and
+    // box row into registers one step ahead; issue(pl) turns them into the
+    // 8-byte cp.async copies into ring slot pl % NST and the row bits.
+    int cx[2], cy[2];
+    bool cv[2];
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const int e = tid + 256 * k;
+        cx[k] = x0 - 1 + e % SFB_W;
+        cy[k] = y0 - 1 + e / SFB_W;
+        cv[k] = e < SFB_C && cx[k] >= 0 && cx[k] < A.nx && cy[k] >= 0 && cy[k] < A.ny;
+    }
+    const int ry = y0 - 1 + tid;  // box row of threads tid < SFB_H
+    const bool rv = tid < SFB_H && ry >= 0 && ry < A.ny;
+    uint32_t tm[2] = {0u, 0u}, rl = 0u, rm = 0u, rh = 0u;
+    int32_t ti[2] = {0, 0};
+    auto fetch = [&](int pl) {
+        const int64_t row0 = (int64_t)(zs + pl) * A.ny;  // slab row of (zl + 1, y = 0), zl = zs - 1 + pl
+#pragma unroll
+        for (int k = 0; k < 2; ++k)
+            if (cv[k]) {
+                const int64_t q = (row0 + cy[k]) * A.rw + (cx[k] >> 5);
+                tm[k] = __ldg(A.rm + q);
+                ti[k] = __ldg(A.ri + q);
+            }
+        if (rv) {
+            const uint32_t *r = A.rm + (row0 + ry) * A.rw;
+            rl = wx > 0 ? __ldg(r + wx - 1) : 0u;
+            rm = __ldg(r + wx);
+            rh = wx + 1 < A.rw ? __ldg(r + wx + 1) : 0u;
+        }
+    };
     auto issue = [&](int pl) {
         const int st = pl % NB_SFB_NST;
-        const int64_t row0 = (int64_t)(zs + pl) * A.ny;  // slab row of (zl + 1, y = 0)
-        for (int e = tid; e < SFB_C; e += 256) {
-            const int bx = e % SFB_W, by = e / SFB_W;
-            const int x = x0 - 1 + bx, yy = y0 - 1 + by;
-            int64_t idx = 0;
-            bool act = false;
-            if (x >= 0 && x < A.nx && yy >= 0 && yy < A.ny) {
-                const int64_t k = (row0 + yy) * A.rw + (x >> 5);
-                const uint32_t m = __ldg(A.rm + k);
-                const unsigned b = (unsigned)x & 31u;
-                act = (m >> b) & 1u;
-                idx = __ldg(A.ri + k) + __popc(m & ((1u << b) - 1u));
-            }
 #pragma unroll
-            for (int c = 0; c < 3; ++c) sfb_cp8(&S[st][c][e], A.u + c * A.cs + idx, act);
-        }
-        if (tid < SFB_H) {  // activity bits of box row tid: bit i = x0 - 1 + i
-            const int yy = y0 - 1 + tid;
-            uint64_t bits = 0;
-            if (yy >= 0 && yy < A.ny) {
-                const uint32_t *r = A.rm + (row0 + yy) * A.rw;
-                const uint64_t lo = wx > 0 ? __ldg(r + wx - 1) >> 31 : 0u;
-                const uint64_t hi = wx + 1 < A.rw ? __ldg(r + wx + 1) & 1u : 0u;
-                bits = lo | ((uint64_t)__ldg(r + wx) << 1) | (hi << 33);
+        for (int k = 0; k < 2; ++k) {
+            const int e = tid + 256 * k;
+            if (e < SFB_C) {
+                const unsigned b = (unsigned)cx[k] & 31u;
+                const bool act = cv[k] && ((tm[k] >> b) & 1u);
+                const int64_t idx = act ? ti[k] + __popc(tm[k] & ((1u << b) - 1u)) : 0;
+#pragma unroll
+                for (int c = 0; c < 3; ++c) sfb_cp8(&S[st][c][e], A.u + c * A.cs + idx, act);
             }
-            RB[st][tid] = bits;
         }
+        if (tid < SFB_H)  // activity bits of box row tid: bit i = x0 - 1 + i
+            RB[st][tid] = rv ? (uint64_t)(rl >> 31) | ((uint64_t)rm << 1) | ((uint64_t)(rh & 1u) << 33) : 0ull;
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
+    // ring: at step pl (plane pl lands) planes pl-2 .. pl are read (the
+    // completed output pl-2 may need all three), pl+1 is in flight and pl+2
+    // is issued into the slot of plane pl-3
+    constexpr int AHEAD = NB_SFB_NST - 3;
 #pragma unroll 1
-    for (int pl = 0; pl < NB_SFB_NST - 1; ++pl) {
-        if (pl < np) issue(pl);
-        else asm volatile("cp.async.commit_group;" ::: "memory");
+    for (int pl = 0; pl < AHEAD; ++pl) {
+        if (pl < np) {
+            fetch(pl);
+            issue(pl);
+        } else {
+            asm volatile("cp.async.commit_group;" ::: "memory");
+        }
     }
+    if (AHEAD < np) fetch(AHEAD);
     const int x = x0 + lane, y = y0 + w;
     const bool in = x < A.nx && y < A.ny;
+    const int ce = (w + 1) * SFB_W + lane + 1;  // the thread's node in a staged box
+    // z-march (the dense kernels' scheme): plane pl's 9 positions x 3
+    // components are read once and applied to output pl-2 (aA, as its oz =
+    // +1 plane), pl-1 (aB, oz = 0) and pl (aC, oz = -1); per output the
+    // blocks arrive in q order, so an interior node gets sp_fem_node's
+    // interior chain bit for bit.  Output pl-2 is then complete: interior
+    // nodes take aA, the others (element set not full, gz = 1) are redone by
+    // sp_fem_node from the three staged planes, gz = 0 is the identity.
+    double aA[3] = {0.0, 0.0, 0.0}, aB[3] = {0.0, 0.0, 0.0};
+    int32_t oi = in ? __ldg(A.ri + ((int64_t)(zs + 1) * A.ny + y) * A.rw + wx) : 0;  // output 0: row zl + 1 = zs + 1
 #pragma unroll 1
-    for (int o = 0; o < ze - zs; ++o) {
-        // planes o .. o+2 are needed; o+3 .. o+NST-2 may stay in flight
-        asm volatile("cp.async.wait_group %0;" ::"n"(NB_SFB_NST - 4) : "memory");
-        __syncthreads();  // every thread's copies landed; plane o-1's slot is free
-        if (o + NB_SFB_NST - 1 < np) issue(o + NB_SFB_NST - 1);
+    for (int pl = 0; pl < np; ++pl) {
+        asm volatile("cp.async.wait_group %0;" ::"n"(AHEAD - 1) : "memory");
+        __syncthreads();  // plane pl landed (all threads' copies); plane pl-3's slot is free
+        if (pl + AHEAD < np) issue(pl + AHEAD);
         else asm volatile("cp.async.commit_group;" ::: "memory");
-        const int zl = zs + o;
-        const int s0 = o % NB_SFB_NST, s1 = (o + 1) % NB_SFB_NST, s2 = (o + 2) % NB_SFB_NST;
-        if (!in || !((RB[s1][w + 1] >> (lane + 1)) & 1u)) continue;
-        const int gz = A.gz0 + zl;
-        double out[3];
-        if (gz == 0) {  // Dirichlet identity row
+        if (pl + AHEAD + 1 < np) fetch(pl + AHEAD + 1);  // lands while this step computes
+        const int sl = pl % NB_SFB_NST;
+        double aC[3] = {0.0, 0.0, 0.0};
+        // warp-uniform: does the row hold an active node of outputs pl-2 .. pl
+        // (centres in planes pl-1 .. pl+1)?  Otherwise the three are never stored
+        const uint64_t rows = (pl >= 1 ? RB[(pl + NB_SFB_NST - 1) % NB_SFB_NST][w + 1] : 0ull) | RB[sl][w + 1] |
+                              (pl + 1 < np ? RB[(pl + 1) % NB_SFB_NST][w + 1] : 0ull);
+        if ((rows >> 1) & 0xffffffffull) sfb_plane<0>(&S[sl][0][ce], aA, aB, aC);
+        if (pl >= 2) {
+            const int o = pl - 2, zl = zs + o;
+            const int s0 = (pl + NB_SFB_NST - 2) % NB_SFB_NST, s1 = (pl + NB_SFB_NST - 1) % NB_SFB_NST;
+            if (in && ((RB[s1][w + 1] >> (lane + 1)) & 1u)) {
+                const int gz = A.gz0 + zl;
+                double out[3] = {aA[0], aA[1], aA[2]};
+                if (gz == 0) {  // Dirichlet identity row
 #pragma unroll
-            for (int c = 0; c < 3; ++c) out[c] = S[s1][c][(w + 1) * SFB_W + lane + 1];
-        } else {
-            uint32_t m = 0;
+                    for (int c = 0; c < 3; ++c) out[c] = S[s1][c][ce];
+                } else {
+                    uint32_t m = 0;
 #pragma unroll
-            for (int r = 0; r < 9; ++r) {
-                const int oy = r % 3 - 1, oz = r / 3 - 1;
-                const int st = oz < 0 ? s0 : (oz == 0 ? s1 : s2);
-                m |= (uint32_t)((RB[st][w + 1 + oy] >> lane) & 7u) << (3 * r);
+                    for (int r = 0; r < 9; ++r) {
+                        const int oy = r % 3 - 1, oz = r / 3 - 1;
+                        const int st = oz < 0 ? s0 : (oz == 0 ? s1 : sl);
+                        m |= (uint32_t)((RB[st][w + 1 + oy] >> lane) & 7u) << (3 * r);
+                    }
+                    if (m != 0x7ffffffu || gz == 1) {
+                        const double *P0 = &S[s0][0][ce], *P1 = &S[s1][0][ce], *P2 = &S[sl][0][ce];
+                        sp_fem_node(m, gz, [&](int q, double &u0, double &u1, double &u2) {
+                            const int ox = q % 3 - 1, oy = (q / 3) % 3 - 1, oz = q / 9 - 1;
+                            const double *P = oz < 0 ? P0 : (oz == 0 ? P1 : P2);
+                            const int e = oy * SFB_W + ox;
+                            u0 = P[e], u1 = P[SFB_C + e], u2 = P[2 * SFB_C + e];
+                        }, out);
+                    }
+                }
+                // buffer index: the row word's index (loaded a step ahead) +
+                // the active cells before x in the word (the staged row bits)
+                const int64_t i = oi + __popc((uint32_t)(RB[s1][w + 1] >> 1) & ((1u << lane) - 1u));
+#pragma unroll
+                for (int c = 0; c < 3; ++c) {
+                    const int64_t kk = c * A.cs + i;
+                    A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], out[c]) : out[c];
+                }
             }
-            sp_fem_node(m, gz, [&](int q, double &u0, double &u1, double &u2) {
-                const int ox = q % 3 - 1, oy = (q / 3) % 3 - 1, oz = q / 9 - 1;
-                const int st = oz < 0 ? s0 : (oz == 0 ? s1 : s2);
-                const int e = (w + 1 + oy) * SFB_W + lane + 1 + ox;
-                u0 = S[st][0][e], u1 = S[st][1][e], u2 = S[st][2][e];
-            }, out);
         }
-        const int64_t k = ((int64_t)(zl + 1) * A.ny + y) * A.rw + wx;
-        const int64_t i = __ldg(A.ri + k) + __popc(__ldg(A.rm + k) & ((1u << lane) - 1u));
+        // the next output's (pl - 1) row word index, consumed next step
+        if (in && pl + 1 < np && pl >= 1) oi = __ldg(A.ri + ((int64_t)(zs + pl) * A.ny + y) * A.rw + wx);
 #pragma unroll
         for (int c = 0; c < 3; ++c) {
-            const int64_t kk = c * A.cs + i;
-            A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], out[c]) : out[c];
+            aA[c] = aB[c];
+            aB[c] = aC[c];
         }
     }
     asm volatile("cp.async.wait_group 0;" ::: "memory");
