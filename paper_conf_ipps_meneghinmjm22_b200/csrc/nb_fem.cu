@@ -1753,7 +1753,7 @@ nb_status nb_sparse_fem_pass(nb_grid *g, int p, int kind, const int32_t *list, c
 #define NB_SFB_NST 5  // ring stages: planes k-1 .. k+1 in use, k+2, k+3 in flight
 #endif
 #ifndef NB_SFB_ZC
-#define NB_SFB_ZC 16  // output planes per CTA
+#define NB_SFB_ZC 32  // output planes per CTA
 #endif
 #ifndef NB_SFB_MINB
 #define NB_SFB_MINB 3
@@ -1888,8 +1888,8 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
     // +1 plane), pl-1 (aB, oz = 0) and pl (aC, oz = -1); per output the
     // blocks arrive in q order, so an interior node gets sp_fem_node's
     // interior chain bit for bit.  Output pl-2 is then complete: interior
-    // nodes take aA, the others (element set not full, gz = 1) are redone by
-    // sp_fem_node from the three staged planes, gz = 0 is the identity.
+    // nodes (27 active neighbours, gz >= 2) store aA; every other node is
+    // k_sp_fem_list's (so no warp here diverges into a class stencil).
     double aA[3] = {0.0, 0.0, 0.0}, aB[3] = {0.0, 0.0, 0.0};
     int32_t oi = in ? __ldg(A.ri + ((int64_t)(zs + 1) * A.ny + y) * A.rw + wx) : 0;  // output 0: row zl + 1 = zs + 1
 #pragma unroll 1
@@ -1909,37 +1909,26 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
         if (pl >= 2) {
             const int o = pl - 2, zl = zs + o;
             const int s0 = (pl + NB_SFB_NST - 2) % NB_SFB_NST, s1 = (pl + NB_SFB_NST - 1) % NB_SFB_NST;
-            if (in && ((RB[s1][w + 1] >> (lane + 1)) & 1u)) {
-                const int gz = A.gz0 + zl;
-                double out[3] = {aA[0], aA[1], aA[2]};
-                if (gz == 0) {  // Dirichlet identity row
+            const int gz = A.gz0 + zl;
+            if (in && gz >= 2 && ((RB[s1][w + 1] >> (lane + 1)) & 1u)) {
+                // interior iff all 27 neighbours are active (then all 8
+                // elements exist); the others are k_sp_fem_list's nodes
+                bool full = true;
 #pragma unroll
-                    for (int c = 0; c < 3; ++c) out[c] = S[s1][c][ce];
-                } else {
-                    uint32_t m = 0;
-#pragma unroll
-                    for (int r = 0; r < 9; ++r) {
-                        const int oy = r % 3 - 1, oz = r / 3 - 1;
-                        const int st = oz < 0 ? s0 : (oz == 0 ? s1 : sl);
-                        m |= (uint32_t)((RB[st][w + 1 + oy] >> lane) & 7u) << (3 * r);
-                    }
-                    if (m != 0x7ffffffu || gz == 1) {
-                        const double *P0 = &S[s0][0][ce], *P1 = &S[s1][0][ce], *P2 = &S[sl][0][ce];
-                        sp_fem_node(m, gz, [&](int q, double &u0, double &u1, double &u2) {
-                            const int ox = q % 3 - 1, oy = (q / 3) % 3 - 1, oz = q / 9 - 1;
-                            const double *P = oz < 0 ? P0 : (oz == 0 ? P1 : P2);
-                            const int e = oy * SFB_W + ox;
-                            u0 = P[e], u1 = P[SFB_C + e], u2 = P[2 * SFB_C + e];
-                        }, out);
-                    }
+                for (int r = 0; r < 9; ++r) {
+                    const int oy = r % 3 - 1, oz = r / 3 - 1;
+                    const int st = oz < 0 ? s0 : (oz == 0 ? s1 : sl);
+                    full = full && ((RB[st][w + 1 + oy] >> lane) & 7u) == 7u;
                 }
-                // buffer index: the row word's index (loaded a step ahead) +
-                // the active cells before x in the word (the staged row bits)
-                const int64_t i = oi + __popc((uint32_t)(RB[s1][w + 1] >> 1) & ((1u << lane) - 1u));
+                if (full) {
+                    // buffer index: the row word's index (loaded a step ahead)
+                    // + the active cells before x in the word (staged row bits)
+                    const int64_t i = oi + __popc((uint32_t)(RB[s1][w + 1] >> 1) & ((1u << lane) - 1u));
 #pragma unroll
-                for (int c = 0; c < 3; ++c) {
-                    const int64_t kk = c * A.cs + i;
-                    A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], out[c]) : out[c];
+                    for (int c = 0; c < 3; ++c) {
+                        const int64_t kk = c * A.cs + i;
+                        A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], aA[c]) : aA[c];
+                    }
                 }
             }
         }
@@ -1952,6 +1941,45 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
         }
     }
     asm volatile("cp.async.wait_group 0;" ::: "memory");
+}
+
+// The non-interior active nodes of the box operator (element set not full,
+// gz <= 1; ~2 % of a cube's nodes): one thread per node of the host-built
+// list {buffer index, gz, 27-neighbourhood mask, 9 row bases} (the gather
+// pass's per-node inputs), same sp_fem_node arithmetic.
+struct SpFemNode {
+    int32_t i, gz;
+    uint32_t m;
+    int32_t base[9];
+};
+static_assert(sizeof(SpFemNode) == 48, "three 16-byte loads per node");
+
+template <int KIND>  // 0: y = K u; 2: y = b - K u
+__global__ void __launch_bounds__(128) k_sp_fem_list(const SpFemNode *__restrict__ L, int64_t n0, int64_t n1,
+                                                    int64_t cs, const double *__restrict__ u,
+                                                    const double *__restrict__ b, double *y, const CgScal *sc) {
+    if (sc && sc->status != 0) return;
+    const int64_t t = n0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= n1) return;
+    const SpFemNode nd = L[t];
+    double o[3];
+    if (nd.gz == 0) {  // Dirichlet identity row
+#pragma unroll
+        for (int c = 0; c < 3; ++c) o[c] = u[c * cs + nd.i];
+    } else {
+        const uint32_t m = nd.m;
+        sp_fem_node(m, nd.gz, [&](int q, double &u0, double &u1, double &u2) {
+            const int ox = q % 3 - 1, r = q / 3;
+            const uint32_t rb = (m >> (3 * r)) & 7u;
+            const int64_t idx = nd.base[r] + __popc(rb & ((1u << (ox + 1)) - 1u));
+            u0 = __ldg(u + idx), u1 = __ldg(u + cs + idx), u2 = __ldg(u + 2 * cs + idx);
+        }, o);
+    }
+#pragma unroll
+    for (int c = 0; c < 3; ++c) {
+        const int64_t k = c * cs + nd.i;
+        y[k] = KIND == 2 ? __dsub_rn(b[k], o[c]) : o[c];
+    }
 }
 
 // per-segment partials of <a, b> (3 components): k_sp_fem's dot, bit for bit
@@ -2006,12 +2034,28 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
     A.y = y;
     A.sc = sc;
     const char *name = kind == 2 ? "k_fem_cg_init" : (sc ? "k_sp_fem_q" : "k_fem_apply");
-    LaunchScope ls(g, g->cs, name);
-    if (kind == 2)
-        k_sp_fem_box<2><<<(unsigned)n, 256, 0, g->cs>>>(A);
-    else
-        k_sp_fem_box<0><<<(unsigned)n, 256, 0, g->cs>>>(A);
-    return nb_launch_check(name);
+    {
+        LaunchScope ls(g, g->cs, name);
+        if (kind == 2)
+            k_sp_fem_box<2><<<(unsigned)n, 256, 0, g->cs>>>(A);
+        else
+            k_sp_fem_box<0><<<(unsigned)n, 256, 0, g->cs>>>(A);
+        NB_TRY(nb_launch_check(name));
+    }
+    // the ranges' non-interior nodes (contiguous per range: the list is in plane order)
+    for (size_t r = 0; r + 1 < ranges.size(); r += 2) {
+        const int64_t a = sp.fnode_start[ranges[r]], e = sp.fnode_start[ranges[r + 1]];
+        if (e <= a) continue;
+        const SpFemNode *L = (const SpFemNode *)sp.d_fnode;
+        const unsigned nb = (unsigned)((e - a + 127) / 128);
+        LaunchScope ls(g, g->cs, name);
+        if (kind == 2)
+            k_sp_fem_list<2><<<nb, 128, 0, g->cs>>>(L, a, e, sp.cs, u, b, y, sc);
+        else
+            k_sp_fem_list<0><<<nb, 128, 0, g->cs>>>(L, a, e, sp.cs, u, b, y, sc);
+        NB_TRY(nb_launch_check(name));
+    }
+    return NB_OK;
 }
 
 nb_status nb_sparse_fem_dot(nb_grid *g, int p, const double *a, const double *b, const CgScal *sc) {

@@ -177,6 +177,11 @@ struct NbSparsePart {
     int32_t *d_ri = nullptr;
     int rw = 0;
     std::vector<uint8_t> tile_any;
+    // the active own nodes the box operator leaves out (element set not full
+    // or gz <= 1), in plane order: 48-B records {buffer index, gz, mask, 9
+    // row bases} (nb_fem.cu SpFemNode); fnode_start[zl] = first of plane zl
+    void *d_fnode = nullptr;
+    std::vector<int64_t> fnode_start;
     std::map<std::vector<int>, std::pair<int4 *, int64_t>> box_lists;
 };
 

@@ -56,6 +56,9 @@ void nb_sparse_free(nb_grid *g) {
         s.d_rm = nullptr;
         s.d_ri = nullptr;
         s.tile_any.clear();
+        cudaFree(s.d_fnode);
+        s.d_fnode = nullptr;
+        s.fnode_start.clear();
         for (auto &kv : s.box_lists) cudaFree(kv.second.first);
         s.box_lists.clear();
         s.d_seg_bnd = s.d_seg_bnd_gi = nullptr;
@@ -1406,6 +1409,68 @@ nb_status nb_sparse_fem_box_tables(nb_grid *g) {
                     if (bits && zl >= 0 && zl < nzl) sp.tile_any[((size_t)zl * ty + y / 8) * tx + w] = 1;
                 }
             }
+        }
+        // non-interior own nodes: interior = all 27 neighbours active (then
+        // all 8 elements exist) and gz >= 2; the 3x3x3 erosion of the slab
+        // mask, separable (x, then y, then z)
+        std::vector<uint8_t> ex((size_t)(nzl + 2) * plane, 0), ey((size_t)(nzl + 2) * plane, 0);
+        auto act = [&](int gz, int y, int x) -> bool {
+            return gz >= 0 && gz < g->nz && y >= 0 && y < ny && x >= 0 && x < nx &&
+                   g->host_mask[(size_t)gz * plane + (size_t)y * nx + x] != 0;
+        };
+        for (int s = 0; s < nzl + 2; ++s) {
+            const int gz = q.z0 + s - 1;
+            if (gz < 0 || gz >= g->nz) continue;
+            for (int y = 0; y < ny; ++y)
+                for (int x = 0; x < nx; ++x)
+                    ex[(size_t)s * plane + (size_t)y * nx + x] = act(gz, y, x - 1) && act(gz, y, x) && act(gz, y, x + 1);
+            for (int y = 0; y < ny; ++y)
+                for (int x = 0; x < nx; ++x) {
+                    const size_t c = (size_t)s * plane + (size_t)y * nx + x;
+                    ey[c] = ex[c] && (y > 0 && ex[c - nx]) && (y + 1 < ny && ex[c + nx]);
+                }
+        }
+        // buffer index of slab row (s, y) cell x (active), from the row tables
+        auto bidx = [&](int s, int y, int x) -> int32_t {
+            const int64_t k = ((int64_t)s * ny + y) * rw + (x >> 5);
+            return ri[k] + __builtin_popcount(rm[k] & ((1u << (x & 31)) - 1u));
+        };
+        struct Node {
+            int32_t i, gz;
+            uint32_t m;
+            int32_t base[9];
+        };
+        std::vector<Node> nodes;
+        sp.fnode_start.assign(nzl + 1, 0);
+        for (int zl = 0; zl < nzl; ++zl) {
+            const int gz = q.z0 + zl;
+            sp.fnode_start[zl] = (int64_t)nodes.size();
+            for (int y = 0; y < ny; ++y)
+                for (int x = 0; x < nx; ++x) {
+                    if (!act(gz, y, x)) continue;
+                    const size_t c = (size_t)y * nx + x;
+                    const bool interior = gz >= 2 && ey[(size_t)zl * plane + c] && ey[(size_t)(zl + 1) * plane + c] &&
+                                          ey[(size_t)(zl + 2) * plane + c];
+                    if (interior) continue;
+                    Node nd{};
+                    nd.i = bidx(zl + 1, y, x);
+                    nd.gz = gz;
+                    for (int r = 0; r < 9; ++r) {
+                        const int oy = r % 3 - 1, oz = r / 3 - 1;
+                        nd.base[r] = -1;
+                        for (int dx = -1; dx <= 1; ++dx)
+                            if (act(gz + oz, y + oy, x + dx)) {
+                                nd.m |= 1u << (3 * r + dx + 1);
+                                if (nd.base[r] < 0) nd.base[r] = bidx(zl + 1 + oz, y + oy, x + dx);
+                            }
+                    }
+                    nodes.push_back(nd);
+                }
+        }
+        sp.fnode_start[nzl] = (int64_t)nodes.size();
+        if (!nodes.empty()) {
+            NB_CUDA(cudaMalloc(&sp.d_fnode, sizeof(Node) * nodes.size()));
+            NB_CUDA(cudaMemcpy(sp.d_fnode, nodes.data(), sizeof(Node) * nodes.size(), cudaMemcpyHostToDevice));
         }
         NB_CUDA(cudaMalloc(&sp.d_rm, sizeof(uint32_t) * rm.size()));
         NB_CUDA(cudaMalloc(&sp.d_ri, sizeof(int32_t) * ri.size()));
