@@ -1767,10 +1767,12 @@ struct SpFemBoxArgs {
     const int4 *items;
     const uint32_t *rm;
     const int32_t *ri;
-    int rw, nx, ny, gz0;
+    int rw, nx, ny, gz0, nzl;
     int64_t cs;
-    const double *u, *b;
+    const double *u, *b;  // KIND 3: u = the p_new buffer (its halo planes are staged as they are)
     double *y;
+    const double *r, *po;  // KIND 3: p_new = r + beta p_old formed while staging own planes
+    double *pn, *x;        // KIND 3: p_new and the deferred x += alpha_prev p_old of own nodes
     const CgScal *sc;
 };
 
@@ -1806,16 +1808,39 @@ __device__ __forceinline__ void sfb_plane(const double *P, double (&aA)[3], doub
     }
 }
 
-template <int KIND>  // 0: y = K u; 2: y = b - K u
+// KIND 0: y = K u; 2: y = b - K u; 3 (sparse FEM CG phase A): own planes
+// stage r and p_old, every thread turns its own box cells into p_new = r +
+// beta p_old (the gather path's map, fma(beta, p_old, r)) right after its
+// copies land, so the one barrier per plane still suffices; halo planes stage
+// the exchanged p_new.  Each active own node stores p_new and, pending, x +=
+// alpha_prev p_old (x loaded a step ahead); interior nodes store q = K p_new.
+template <int KIND>
+struct SfbCfg {
+    static constexpr int NPO = KIND == 3 ? 4 : 0;  // p_old slots: planes pl-1 .. pl+2
+    static constexpr int SMEM = (NB_SFB_NST + NPO) * 3 * SFB_C * 8;
+};
+
+template <int KIND>
 __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A) {
-    __shared__ __align__(16) double S[NB_SFB_NST][3][SFB_C];
+    extern __shared__ __align__(16) double sfb_sm[];
+    double(*S)[3][SFB_C] = reinterpret_cast<double(*)[3][SFB_C]>(sfb_sm);
+    double(*PO)[3][SFB_C] = reinterpret_cast<double(*)[3][SFB_C]>(sfb_sm + NB_SFB_NST * 3 * SFB_C);
+    constexpr int NPO = SfbCfg<KIND>::NPO;
     __shared__ uint64_t RB[NB_SFB_NST][SFB_H];
     if (A.sc && A.sc->status != 0) return;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const int4 it = A.items[blockIdx.x];
     const int x0 = it.x * 32, y0 = it.y * 8, zs = it.z, ze = it.w;
     const int np = ze - zs + 2;  // staged planes zs-1 .. ze
+    const int nout = ze - zs;
     const int wx = it.x;         // the tile's x word
+    double beta = 0.0, ap = 0.0;
+    bool dox = false;
+    if constexpr (KIND == 3) {
+        beta = A.sc->beta;
+        ap = A.sc->alpha_prev;
+        dox = A.sc->pending != 0;
+    }
     // Staging is split in two so no thread waits on a table load: fetch(pl)
     // loads plane pl's table words for the thread's (up to 2) box cells and
     // box row into registers one step ahead; issue(pl) turns them into the
@@ -1833,6 +1858,7 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
     const bool rv = tid < SFB_H && ry >= 0 && ry < A.ny;
     uint32_t tm[2] = {0u, 0u}, rl = 0u, rm = 0u, rh = 0u;
     int32_t ti[2] = {0, 0};
+    auto own = [&](int pl) { const int zl = zs - 1 + pl; return zl >= 0 && zl < A.nzl; };
     auto fetch = [&](int pl) {
         const int64_t row0 = (int64_t)(zs + pl) * A.ny;  // slab row of (zl + 1, y = 0), zl = zs - 1 + pl
 #pragma unroll
@@ -1851,6 +1877,7 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
     };
     auto issue = [&](int pl) {
         const int st = pl % NB_SFB_NST;
+        const bool form = KIND == 3 && own(pl);
 #pragma unroll
         for (int k = 0; k < 2; ++k) {
             const int e = tid + 256 * k;
@@ -1858,8 +1885,16 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
                 const unsigned b = (unsigned)cx[k] & 31u;
                 const bool act = cv[k] && ((tm[k] >> b) & 1u);
                 const int64_t idx = act ? ti[k] + __popc(tm[k] & ((1u << b) - 1u)) : 0;
+                if (form) {
 #pragma unroll
-                for (int c = 0; c < 3; ++c) sfb_cp8(&S[st][c][e], A.u + c * A.cs + idx, act);
+                    for (int c = 0; c < 3; ++c) {
+                        sfb_cp8(&S[st][c][e], A.r + c * A.cs + idx, act);
+                        sfb_cp8(&PO[pl % (NPO ? NPO : 1)][c][e], A.po + c * A.cs + idx, act);
+                    }
+                } else {
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) sfb_cp8(&S[st][c][e], A.u + c * A.cs + idx, act);
+                }
             }
         }
         if (tid < SFB_H)  // activity bits of box row tid: bit i = x0 - 1 + i
@@ -1883,6 +1918,7 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
     const int x = x0 + lane, y = y0 + w;
     const bool in = x < A.nx && y < A.ny;
     const int ce = (w + 1) * SFB_W + lane + 1;  // the thread's node in a staged box
+    const uint32_t lmask = (1u << lane) - 1u;
     // z-march (the dense kernels' scheme): plane pl's 9 positions x 3
     // components are read once and applied to output pl-2 (aA, as its oz =
     // +1 plane), pl-1 (aB, oz = 0) and pl (aC, oz = -1); per output the
@@ -1890,16 +1926,31 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
     // interior chain bit for bit.  Output pl-2 is then complete: interior
     // nodes (27 active neighbours, gz >= 2) store aA; every other node is
     // k_sp_fem_list's (so no warp here diverges into a class stencil).
+    // The output node's buffer index (row word index + active cells before
+    // x) and, for KIND 3, its x are loaded a step ahead.
     double aA[3] = {0.0, 0.0, 0.0}, aB[3] = {0.0, 0.0, 0.0};
-    int32_t oi = in ? __ldg(A.ri + ((int64_t)(zs + 1) * A.ny + y) * A.rw + wx) : 0;  // output 0: row zl + 1 = zs + 1
+    double xo[3] = {0.0, 0.0, 0.0};
+    int32_t oi = 0;   // row word index of the next output to be indexed
+    int64_t ic = 0;   // buffer index of the output completed next step
 #pragma unroll 1
     for (int pl = 0; pl < np; ++pl) {
         asm volatile("cp.async.wait_group %0;" ::"n"(AHEAD - 1) : "memory");
-        __syncthreads();  // plane pl landed (all threads' copies); plane pl-3's slot is free
+        const int sl = pl % NB_SFB_NST;
+        if constexpr (KIND == 3) {
+            if (own(pl)) {  // this thread's box cells of plane pl: p_new = r + beta p_old
+#pragma unroll
+                for (int k = 0; k < 2; ++k) {
+                    const int e = tid + 256 * k;
+                    if (e < SFB_C)
+#pragma unroll
+                        for (int c = 0; c < 3; ++c) S[sl][c][e] = fma(beta, PO[pl % NPO][c][e], S[sl][c][e]);
+                }
+            }
+        }
+        __syncthreads();  // plane pl landed (p_new formed); plane pl-3's slot is free
         if (pl + AHEAD < np) issue(pl + AHEAD);
         else asm volatile("cp.async.commit_group;" ::: "memory");
         if (pl + AHEAD + 1 < np) fetch(pl + AHEAD + 1);  // lands while this step computes
-        const int sl = pl % NB_SFB_NST;
         double aC[3] = {0.0, 0.0, 0.0};
         // warp-uniform: does the row hold an active node of outputs pl-2 .. pl
         // (centres in planes pl-1 .. pl+1)?  Otherwise the three are never stored
@@ -1910,10 +1961,17 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
             const int o = pl - 2, zl = zs + o;
             const int s0 = (pl + NB_SFB_NST - 2) % NB_SFB_NST, s1 = (pl + NB_SFB_NST - 1) % NB_SFB_NST;
             const int gz = A.gz0 + zl;
-            if (in && gz >= 2 && ((RB[s1][w + 1] >> (lane + 1)) & 1u)) {
+            if (in && ((RB[s1][w + 1] >> (lane + 1)) & 1u)) {
+                if constexpr (KIND == 3) {  // every active own node: p_new, deferred x
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) {
+                        __stcs(A.pn + c * A.cs + ic, S[s1][c][ce]);
+                        if (dox) __stcs(A.x + c * A.cs + ic, fma(ap, PO[(pl - 1) % NPO][c][ce], xo[c]));
+                    }
+                }
                 // interior iff all 27 neighbours are active (then all 8
-                // elements exist); the others are k_sp_fem_list's nodes
-                bool full = true;
+                // elements exist) and gz >= 2
+                bool full = gz >= 2;
 #pragma unroll
                 for (int r = 0; r < 9; ++r) {
                     const int oy = r % 3 - 1, oz = r / 3 - 1;
@@ -1921,19 +1979,25 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
                     full = full && ((RB[st][w + 1 + oy] >> lane) & 7u) == 7u;
                 }
                 if (full) {
-                    // buffer index: the row word's index (loaded a step ahead)
-                    // + the active cells before x in the word (staged row bits)
-                    const int64_t i = oi + __popc((uint32_t)(RB[s1][w + 1] >> 1) & ((1u << lane) - 1u));
 #pragma unroll
                     for (int c = 0; c < 3; ++c) {
-                        const int64_t kk = c * A.cs + i;
+                        const int64_t kk = c * A.cs + ic;
                         A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], aA[c]) : aA[c];
                     }
                 }
             }
         }
-        // the next output's (pl - 1) row word index, consumed next step
-        if (in && pl + 1 < np && pl >= 1) oi = __ldg(A.ri + ((int64_t)(zs + pl) * A.ny + y) * A.rw + wx);
+        // the next output (pl - 1, centre plane pl): its buffer index and x
+        if (pl >= 1 && pl - 1 < nout) {
+            const uint64_t cb = RB[sl][w + 1];
+            ic = oi + __popc((uint32_t)(cb >> 1) & lmask);
+            if constexpr (KIND == 3)
+                if (dox && in && ((cb >> (lane + 1)) & 1u))
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) xo[c] = __ldcs(A.x + c * A.cs + ic);
+        }
+        // and the row word index of output pl (centre plane pl + 1)
+        if (in && pl < nout) oi = __ldg(A.ri + ((int64_t)(zs + pl + 1) * A.ny + y) * A.rw + wx);
 #pragma unroll
         for (int c = 0; c < 3; ++c) {
             aA[c] = aB[c];
@@ -2014,7 +2078,7 @@ __global__ void __launch_bounds__(256) k_sp_fem_dot(const int32_t *__restrict__ 
 bool nb_sparse_fem_boxed() { return !getenv("NB_SPF_GATHER"); }
 
 nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> &ranges, const double *u,
-                            const double *b, double *y, const CgScal *sc) {
+                            const double *b, double *y, const CgScal *sc, const SpFemCgA *cga) {
     const int4 *items = nullptr;
     int64_t n = 0;
     NB_TRY(nb_sparse_fem_box_list(g, p, ranges, NB_SFB_ZC, &items, &n));
@@ -2029,18 +2093,39 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
     A.ny = g->ny;
     A.gz0 = g->parts[p].z0;
     A.cs = sp.cs;
+    A.nzl = g->parts[p].nz();
     A.u = u;
     A.b = b;
     A.y = y;
     A.sc = sc;
-    const char *name = kind == 2 ? "k_fem_cg_init" : (sc ? "k_sp_fem_q" : "k_fem_apply");
+    if (kind == 3) {
+        if (!cga || !sc) NB_FAIL(NB_EINVAL, "sparse FEM phase A needs the CG buffers");
+        A.r = cga->r;
+        A.po = cga->po;
+        A.pn = cga->pn;
+        A.x = cga->x;
+        A.u = cga->pn;  // halo planes: the exchanged p_new
+    }
+    const char *name = kind == 2 ? "k_fem_cg_init" : kind == 3 ? "k_sp_fem_cg_a" : (sc ? "k_sp_fem_q" : "k_fem_apply");
     {
+        static bool attr = false;
+        if (!attr) {
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         SfbCfg<3>::SMEM));
+            attr = true;
+        }
         LaunchScope ls(g, g->cs, name);
         if (kind == 2)
-            k_sp_fem_box<2><<<(unsigned)n, 256, 0, g->cs>>>(A);
+            k_sp_fem_box<2><<<(unsigned)n, 256, SfbCfg<2>::SMEM, g->cs>>>(A);
+        else if (kind == 3)
+            k_sp_fem_box<3><<<(unsigned)n, 256, SfbCfg<3>::SMEM, g->cs>>>(A);
         else
-            k_sp_fem_box<0><<<(unsigned)n, 256, 0, g->cs>>>(A);
+            k_sp_fem_box<0><<<(unsigned)n, 256, SfbCfg<0>::SMEM, g->cs>>>(A);
         NB_TRY(nb_launch_check(name));
+    }
+    if (kind == 3) {  // the list nodes' q = K p_new reads the stored p_new
+        kind = 0;
+        u = cga->pn;
     }
     // the ranges' non-interior nodes (contiguous per range: the list is in plane order)
     for (size_t r = 0; r + 1 < ranges.size(); r += 2) {
@@ -2083,8 +2168,37 @@ static std::vector<int> sp_box_ranges(const nb_grid *g, int p, int which) {
 }
 
 nb_status nb_sparse_fem_box_ranges(nb_grid *g, int p, int which, const double *u, const double *b, double *y,
-                                   const CgScal *sc, int kind) {
-    return nb_sparse_fem_box(g, p, kind, sp_box_ranges(g, p, which), u, b, y, sc);
+                                   const CgScal *sc, int kind, const SpFemCgA *cga) {
+    return nb_sparse_fem_box(g, p, kind, sp_box_ranges(g, p, which), u, b, y, sc, cga);
+}
+
+// p_new = r + beta p_old on the boundary planes facing a neighbour (they are
+// the neighbours' halos, sent before phase A): the gather path's map
+// arithmetic, no x update (phase A does it for every own node)
+__global__ void k_sp_pmap(double *pn, const double *po, const double *r, int64_t cs, int64_t a0, int64_t n0,
+                          int64_t a1, int64_t n1, const CgScal *sc) {
+    if (sc->status != 0) return;
+    const double beta = sc->beta;
+    const int64_t n = n0 + n1;
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < 3 * n; t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t c = t / n, k = t % n;
+        const int64_t i = c * cs + (k < n0 ? a0 + k : a1 + (k - n0));
+        pn[i] = fma(beta, po[i], r[i]);
+    }
+}
+
+nb_status nb_sparse_fem_pmap(nb_grid *g, int p, const double *po, const double *r, double *pn, const CgScal *sc) {
+    const NbPart &q = g->parts[p];
+    const NbSparsePart &sp = g->sp[p];
+    const int nz = q.nz();
+    int64_t a0 = 0, n0 = 0, a1 = 0, n1 = 0;
+    if (q.lo >= 0) a0 = sp.hl + sp.pstart[0], n0 = sp.pstart[1] - sp.pstart[0];
+    if (q.hi >= 0 && (q.lo < 0 || nz > 1)) a1 = sp.hl + sp.pstart[nz - 1], n1 = sp.pstart[nz] - sp.pstart[nz - 1];
+    if (n0 + n1 <= 0) return NB_OK;
+    LaunchScope ls(g, g->cs, "k_sp_cg_map");
+    k_sp_pmap<<<(unsigned)std::min<int64_t>((3 * (n0 + n1) + 255) / 256, 148 * 8), 256, 0, g->cs>>>(
+        pn, po, r, sp.cs, a0, n0, a1, n1, sc);
+    return nb_launch_check("k_sp_pmap");
 }
 
 // build the tables and every list the CG / apply use (outside any capture)
@@ -2122,7 +2236,7 @@ extern "C" nb_status nb_fem27_apply(const nb_field *u, nb_field *y, double E, do
             const NbSparsePart &sp = g->sp[p];
             if (box)
                 NB_TRY(nb_sparse_fem_box_ranges(g, p, 0, (const double *)u->base[p], nullptr, (double *)y->base[p],
-                                                nullptr, 0));
+                                                nullptr, 0, nullptr));
             else
                 NB_TRY(nb_sparse_fem_pass(g, p, 0, sp.d_seg, nullptr, 0, sp.seg_start.back(),
                                           (const double *)u->base[p], nullptr, (double *)y->base[p], nullptr));
@@ -2179,12 +2293,18 @@ nb_status nb_fem_cg_init(nb_cg *cg) {
         NB_TRY(nb_sparse_fem_tables(g));
         const bool box = nb_sparse_fem_boxed();
         if (box) NB_TRY(nb_sparse_fem_box_prepare(g));  // the q pass's lists, before any capture
+        // fused phase A (p ping-pong) with NB_SPF_FUSED=1, decided once per
+        // solver: same bits, but 2.70 ms against 1.24 + 1.00 ms for the box
+        // q pass after the separate map at 384^3 — its 8-byte cp.async
+        // staging of six arrays per plane leaves it waiting on data (ncu:
+        // 39 % issue, half the stall samples at the ring wait and barrier)
+        cg->pingpong = box && getenv("NB_SPF_FUSED");
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
             const NbSparsePart &sp = g->sp[p];
             double *r = (double *)cg->r->base[p];
             if (box) {
                 NB_TRY(nb_sparse_fem_box_ranges(g, p, 0, (const double *)cg->x->base[p],
-                                                (const double *)cg->b->base[p], r, nullptr, 2));
+                                                (const double *)cg->b->base[p], r, nullptr, 2, nullptr));
                 NB_TRY(nb_sparse_fem_dot(g, p, r, r, nullptr));
             } else {
                 NB_TRY(nb_sparse_fem_pass(g, p, 2, sp.d_seg, nullptr, 0, sp.seg_start.back(),
@@ -2210,11 +2330,11 @@ nb_status nb_fem_cg_init(nb_cg *cg) {
 // Both compute the same values in the same order (bitwise).
 static bool fem_fused() { return !getenv("NB_FEM_KERNEL") && !getenv("NB_FEM_3PASS") && nb_tma_enabled(); }
 
-nb_status nb_sparse_fem_cg_hooks(nb_cg *cg);  // nb_sparse.cu
+nb_status nb_sparse_fem_cg_hooks(nb_cg *cg, int parity);  // nb_sparse.cu
 
 nb_status nb_fem_cg_hooks(nb_cg *cg, int parity) {
     nb_grid *g = cg->g;
-    if (g->sparse) return nb_sparse_fem_cg_hooks(cg);
+    if (g->sparse) return nb_sparse_fem_cg_hooks(cg, parity);
     nb_field *pn = cg->p[parity], *po = cg->p[parity ^ 1];
     const bool fused = fem_fused();
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {

@@ -479,15 +479,23 @@ bool nb_sparse_fem_boxed();  // the box operator is the default (NB_SPF_GATHER=1
 nb_status nb_sparse_fem_box_tables(nb_grid *g);
 nb_status nb_sparse_fem_box_list(nb_grid *g, int p, const std::vector<int> &ranges, int zc, const int4 **items,
                                  int64_t *n);
+// kind 3 (sparse FEM CG phase A): p_new = r + beta p_old, deferred x, q = K
+// p_new in one pass (the CG's buffers below; p ping-pongs by parity)
+struct SpFemCgA {
+    const double *r, *po;
+    double *pn, *x;
+};
 nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> &ranges, const double *u,
-                            const double *b, double *y, const CgScal *sc);
+                            const double *b, double *y, const CgScal *sc, const SpFemCgA *cga = nullptr);
+// p_new on the boundary planes facing a neighbour (before their halo is sent)
+nb_status nb_sparse_fem_pmap(nb_grid *g, int p, const double *po, const double *r, double *pn, const CgScal *sc);
 // per-segment partials of <a, b> over the 3 components of partition p (the
 // gather pass's dot, bit for bit), all segments
 nb_status nb_sparse_fem_dot(nb_grid *g, int p, const double *a, const double *b, const CgScal *sc);
 // the box operator over local planes: which = 0 all, 1 the interior (planes
 // whose neighbours are own planes), 2 the boundary planes facing a neighbour
 nb_status nb_sparse_fem_box_ranges(nb_grid *g, int p, int which, const double *u, const double *b, double *y,
-                                   const CgScal *sc, int kind);
+                                   const CgScal *sc, int kind, const SpFemCgA *cga);
 nb_status nb_sparse_fem_box_prepare(nb_grid *g);  // tables + every list (call outside graph capture)
 nb_status nb_nccl_allreduce_sum(nb_grid *g, const double *send, double *recv, size_t n,
                                 cudaStream_t s);
@@ -550,5 +558,8 @@ struct nb_cg {
     std::map<std::pair<int, int>, std::pair<cudaGraphExec_t, int64_t>> graphs;  // (count, parity) -> graph, kernels
     HaloSync hs;
     bool finished = false;
+    // sparse FEM CG with the fused phase A: p ping-pongs by iteration parity
+    // (as in the dense CG), so the final flush picks p by sc->iters
+    bool pingpong = false;
 };
 

@@ -1257,8 +1257,9 @@ nb_status nb_sparse_cg_hooks(nb_cg *cg, int parity) {
     return NB_OK;
 }
 
-__global__ void k_sp_cg_flush(double *x, const double *p, int64_t n, const CgScal *sc) {
+__global__ void k_sp_cg_flush(double *x, const double *p0, const double *p1, int64_t n, const CgScal *sc) {
     if (!sc->pending) return;
+    const double *p = (p1 && (sc->iters & 1)) ? p1 : p0;  // ping-pong: the last p_new
     const double a = sc->alpha_prev;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         x[i] = fma(a, p[i], x[i]);
@@ -1272,6 +1273,7 @@ nb_status nb_sparse_cg_flush(nb_cg *cg) {
             const int64_t o = (int64_t)c * cg->x->pcs[p] + sp.hl;
             LaunchScope ls(g, g->cs, "k_sp_cg_flush");
             k_sp_cg_flush<<<296, 256, 0, g->cs>>>((double *)cg->x->base[p] + o, (const double *)cg->p[0]->base[p] + o,
+                                                  cg->pingpong ? (const double *)cg->p[1]->base[p] + o : nullptr,
                                                   sp.n, cg->sc);
             NB_TRY(nb_launch_check("k_sp_cg_flush"));
         }
@@ -1576,11 +1578,54 @@ nb_status nb_sparse_fem_rhs(nb_field *b, double pr) {
 // per component -> beta (the Poisson sparse schedule with the FEM operator;
 // OCC as there: boundary map, halo in flight with the interior map / K p,
 // boundary K p after the wait)
-nb_status nb_sparse_fem_cg_hooks(nb_cg *cg) {
+nb_status nb_sparse_fem_cg_hooks(nb_cg *cg, int parity) {
     nb_grid *g = cg->g;
-    nb_field *p_ = cg->p[0];
     const nb_occ occ = cg->prm.occ;
     const bool split = occ != NB_OCC_NONE && g->nparts > 1 && (nb_is_peer(g) || nb_halo_on_stream(g));
+    if (cg->pingpong) {
+        // fused phase A (the dense FEM CG's schedule on the sparse grid):
+        // p_new of the boundary planes facing a neighbour -> their halo ->
+        // phase A (p_new, deferred x, q = K p_new; interior planes while the
+        // halo flies) -> the list nodes' q -> <p_new, q> -> alpha -> r -> beta.
+        // Same values as the map + q schedule below (bitwise).
+        nb_field *pn = cg->p[parity], *po = cg->p[parity ^ 1];
+        auto cga = [&](int p) {
+            return SpFemCgA{(const double *)cg->r->base[p], (const double *)po->base[p], (double *)pn->base[p],
+                            (double *)cg->x->base[p]};
+        };
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+            NB_TRY(nb_sparse_fem_pmap(g, p, (const double *)po->base[p], (const double *)cg->r->base[p],
+                                      (double *)pn->base[p], cg->sc));
+        auto phase_a = [&](int p, int which) {
+            const SpFemCgA c = cga(p);
+            return nb_sparse_fem_box_ranges(g, p, which, nullptr, nullptr, (double *)cg->q->base[p], cg->sc, 3, &c);
+        };
+        if (!split) {
+            if (g->nparts > 1) NB_TRY(nb_sparse_halo_update(pn));
+            for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) NB_TRY(phase_a(p, 0));
+        } else {
+            NB_TRY(nb_halo_split_begin(pn, 0, 3, cg->hs));
+            for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) NB_TRY(phase_a(p, 1));
+            NB_TRY(nb_halo_split_wait(g, cg->hs));
+            for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) NB_TRY(phase_a(p, 2));
+        }
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+            NB_TRY(nb_sparse_fem_dot(g, p, (const double *)pn->base[p], (const double *)cg->q->base[p], cg->sc));
+        NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+            for (int c = 0; c < 3; ++c) {
+                SpArgs A{};
+                const int64_t o = (int64_t)c * pn->pcs[p];
+                A.a = (const double *)cg->q->base[p] + o;
+                A.c = (double *)cg->r->base[p] + o;
+                A.sc = cg->sc;
+                NB_TRY(sp_launch<SPK_CG_R>(g, p, 0, g->parts[p].nz(), A, c * g->nz, "k_sp_cg_r"));
+            }
+        NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_RR, cg->sc, 0));
+        cg->k += 1;
+        return NB_OK;
+    }
+    nb_field *p_ = cg->p[0];
     auto map_args = [&](int p, int c) {
         SpArgs A{};
         const int64_t o = (int64_t)c * p_->pcs[p];
@@ -1599,7 +1644,7 @@ nb_status nb_sparse_fem_cg_hooks(nb_cg *cg) {
     const bool box = nb_sparse_fem_boxed();
     auto qbox = [&](int p, int which) {
         return nb_sparse_fem_box_ranges(g, p, which, (const double *)p_->base[p], nullptr, (double *)cg->q->base[p],
-                                        cg->sc, 0);
+                                        cg->sc, 0, nullptr);
     };
     auto qdot = [&]() -> nb_status {
         if (box)

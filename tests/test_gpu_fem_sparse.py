@@ -116,18 +116,18 @@ def test_sparse_fem_cg_converges():
     assert np.all(x[:, 0] == 0.0)
 
 
-def _run_both(fn):
-    """fn() under the shared-memory box operator (default) and the gather
-    pass (NB_SPF_GATHER=1)."""
+def _run_both(fn, modes=("NB_SPF_NONE", "NB_SPF_GATHER")):
+    """fn() under each switch in `modes` set to 1 (NB_SPF_NONE: the default,
+    the shared-memory box operator after a separate map; NB_SPF_GATHER: the
+    gather pass; NB_SPF_FUSED: the box operator's fused CG phase A)."""
     import os
     outs = []
-    for gather in (False, True):
-        if gather:
-            os.environ["NB_SPF_GATHER"] = "1"
+    for m in modes:
+        os.environ[m] = "1"
         try:
             outs.append(fn())
         finally:
-            os.environ.pop("NB_SPF_GATHER", None)
+            os.environ.pop(m, None)
     return outs
 
 
@@ -170,5 +170,6 @@ def test_sparse_fem_box_equals_gather_bitwise(name, parts):
             fb.close(), fx.close()
         return x, r.rr, r.iters
 
-    (xa, rra, ia), (xb, rrb, ib) = _run_both(cg)
-    assert ia == ib and rra == rrb and np.array_equal(xa, xb)
+    (xa, rra, ia), (xb, rrb, ib), (xc, rrc, ic) = _run_both(cg, ("NB_SPF_NONE", "NB_SPF_GATHER", "NB_SPF_FUSED"))
+    assert ia == ib == ic and rra == rrb == rrc
+    assert np.array_equal(xa, xb) and np.array_equal(xa, xc)

@@ -15,14 +15,14 @@ import paper_conf_ipps_meneghinmjm22_b200 as nb
 import synth
 
 N = int(sys.argv[1]) if len(sys.argv) > 1 else 384
-KS = ("k_sp_fem_q", "k_sp_fem_dot", "k_sp_cg_map", "k_sp_cg_r", "k_finalize")
+KS = ("k_sp_fem_cg_a", "k_sp_fem_q", "k_sp_fem_dot", "k_sp_cg_map", "k_sp_cg_r", "k_finalize")
+MODES = {"box": {}, "fused": {"NB_SPF_FUSED": "1"}, "gather": {"NB_SPF_GATHER": "1"}}
 
 
-def run(mask, gather, iters=10):
-    if gather:
-        os.environ["NB_SPF_GATHER"] = "1"
-    else:
-        os.environ.pop("NB_SPF_GATHER", None)
+def run(mask, mode, iters=10):
+    for k in ("NB_SPF_FUSED", "NB_SPF_GATHER"):
+        os.environ.pop(k, None)
+    os.environ.update(MODES[mode])
     g = nb.Grid((N, N, N), active=mask)
     b, x = nb.Field(g, card=3), nb.Field(g, card=3)
     nb.nb_fem27_rhs(b, 1.0)
@@ -52,12 +52,9 @@ out = {"N": N}
 for name, mask in (("full", np.ones((N, N, N), np.uint8)), ("sphere", synth.sphere_mask(N))):
     act = int(mask.sum())
     r = {"active": act}
-    for mode in ("box", "gather"):
-        r[mode] = run(mask, mode == "gather")
-    r["same_bits"] = r["box"]["x_digest"] == r["gather"]["x_digest"]
-    q_box = r["box"]["kernel_ms"]["k_sp_fem_q"] + r["box"]["kernel_ms"]["k_sp_fem_dot"]
-    r["q_box_ms"] = q_box
-    r["q_box_frac_hbm_48B"] = 48 * act / (r["box"]["kernel_ms"]["k_sp_fem_q"] / 1e3) / 1e9 / 6451.8
+    for mode in MODES:
+        r[mode] = run(mask, mode)
+    r["same_bits"] = len({r[m]["x_digest"] for m in MODES}) == 1
     out[name] = r
     print(name, json.dumps(r), flush=True)
 os.makedirs("gpurun_out", exist_ok=True)
