@@ -551,6 +551,7 @@ extern "C" nb_status nb_grid_destroy(nb_grid *g) {
     if (g->c1_exec) cudaGraphExecDestroy(g->c1_exec);
     cudaFree(g->c1_tp);
     cudaFree(g->c1_psum);
+    cudaFree(g->sp_tp);
     nb_peer_grid_teardown(g);  // collective (peer transport)
     for (auto &r : g->prof) {
         cudaEventDestroy(r.a);

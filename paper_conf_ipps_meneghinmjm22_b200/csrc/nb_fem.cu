@@ -2174,20 +2174,22 @@ nb_status nb_sparse_fem_box_ranges(nb_grid *g, int p, int which, const double *u
 
 // p_new = r + beta p_old on the boundary planes facing a neighbour (they are
 // the neighbours' halos, sent before phase A): the gather path's map
-// arithmetic, no x update (phase A does it for every own node)
-__global__ void k_sp_pmap(double *pn, const double *po, const double *r, int64_t cs, int64_t a0, int64_t n0,
-                          int64_t a1, int64_t n1, const CgScal *sc) {
+// arithmetic, no x update (phase A does it for every own node); card
+// components (sparse fields: component stride sp.cs)
+__global__ void k_sp_pmap(double *pn, const double *po, const double *r, int64_t cs, int card, int64_t a0,
+                          int64_t n0, int64_t a1, int64_t n1, const CgScal *sc) {
     if (sc->status != 0) return;
     const double beta = sc->beta;
     const int64_t n = n0 + n1;
-    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < 3 * n; t += (int64_t)gridDim.x * blockDim.x) {
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < card * n; t += (int64_t)gridDim.x * blockDim.x) {
         const int64_t c = t / n, k = t % n;
         const int64_t i = c * cs + (k < n0 ? a0 + k : a1 + (k - n0));
         pn[i] = fma(beta, po[i], r[i]);
     }
 }
 
-nb_status nb_sparse_fem_pmap(nb_grid *g, int p, const double *po, const double *r, double *pn, const CgScal *sc) {
+nb_status nb_sparse_pmap(nb_grid *g, int p, int card, const double *po, const double *r, double *pn,
+                         const CgScal *sc) {
     const NbPart &q = g->parts[p];
     const NbSparsePart &sp = g->sp[p];
     const int nz = q.nz();
@@ -2196,8 +2198,8 @@ nb_status nb_sparse_fem_pmap(nb_grid *g, int p, const double *po, const double *
     if (q.hi >= 0 && (q.lo < 0 || nz > 1)) a1 = sp.hl + sp.pstart[nz - 1], n1 = sp.pstart[nz] - sp.pstart[nz - 1];
     if (n0 + n1 <= 0) return NB_OK;
     LaunchScope ls(g, g->cs, "k_sp_cg_map");
-    k_sp_pmap<<<(unsigned)std::min<int64_t>((3 * (n0 + n1) + 255) / 256, 148 * 8), 256, 0, g->cs>>>(
-        pn, po, r, sp.cs, a0, n0, a1, n1, sc);
+    k_sp_pmap<<<(unsigned)std::min<int64_t>((card * (n0 + n1) + 255) / 256, 148 * 8), 256, 0, g->cs>>>(
+        pn, po, r, sp.cs, card, a0, n0, a1, n1, sc);
     return nb_launch_check("k_sp_pmap");
 }
 

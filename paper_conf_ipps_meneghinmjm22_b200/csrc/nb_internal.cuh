@@ -220,6 +220,11 @@ struct nb_grid {
     // C1 tile partials / plane sums of all iterations of one call (single
     // process: one finalize per call instead of one per iteration)
     double *c1_tp = nullptr, *c1_psum = nullptr;
+    // element-sparse grids: tile partials [nz][sp_T] of the 2-phase box CG
+    // (32 x 8 tiles of the bounding box, the dense canonical dot order);
+    // swapped into tp / T around its kernels and finalizes (lazy)
+    double *sp_tp = nullptr;
+    int sp_T = 0;
     int64_t c1_cap = 0;  // doubles of c1_tp
     // element-sparse
     std::vector<NbSparsePart> sp;
@@ -488,7 +493,8 @@ struct SpFemCgA {
 nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> &ranges, const double *u,
                             const double *b, double *y, const CgScal *sc, const SpFemCgA *cga = nullptr);
 // p_new on the boundary planes facing a neighbour (before their halo is sent)
-nb_status nb_sparse_fem_pmap(nb_grid *g, int p, const double *po, const double *r, double *pn, const CgScal *sc);
+nb_status nb_sparse_pmap(nb_grid *g, int p, int card, const double *po, const double *r, double *pn,
+                         const CgScal *sc);
 // per-segment partials of <a, b> over the 3 components of partition p (the
 // gather pass's dot, bit for bit), all segments
 nb_status nb_sparse_fem_dot(nb_grid *g, int p, const double *a, const double *b, const CgScal *sc);
@@ -558,8 +564,10 @@ struct nb_cg {
     std::map<std::pair<int, int>, std::pair<cudaGraphExec_t, int64_t>> graphs;  // (count, parity) -> graph, kernels
     HaloSync hs;
     bool finished = false;
-    // sparse FEM CG with the fused phase A: p ping-pongs by iteration parity
-    // (as in the dense CG), so the final flush picks p by sc->iters
+    // sparse CG with the fused phase A (the 2-phase box CG, or the FEM
+    // NB_SPF_FUSED path): p ping-pongs by iteration parity (as in the dense
+    // CG), so the final flush picks p by sc->iters
     bool pingpong = false;
+    bool sp_box = false;  // sparse 7-point CG on the 2-phase box schedule
 };
 

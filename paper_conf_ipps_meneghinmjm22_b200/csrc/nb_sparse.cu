@@ -1165,8 +1165,15 @@ nb_status nb_sparse_laplace7(const nb_field *x, nb_field *y, nb_view v) {
 // 24 B connectivity): map (x deferred update, p = r + beta p) -> halo(p) ->
 // q = A p, <p,q> -> alpha -> r -= alpha q, <r,r> -> beta
 // ---------------------------------------------------------------------------
+static nb_status sp_cg_box_init(nb_cg *cg);
+bool nb_sparse_cg_boxed();
+
 nb_status nb_sparse_cg_init(nb_cg *cg) {
     nb_grid *g = cg->g;
+    if (nb_sparse_cg_boxed() && cg->prm.op == NB_OP_LAPLACE7) {
+        cg->sp_box = cg->pingpong = true;
+        return sp_cg_box_init(cg);
+    }
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         SpArgs A{};
         A.a = (const double *)cg->x->base[p];
@@ -1189,8 +1196,10 @@ nb_status nb_sparse_cg_init(nb_cg *cg) {
 // is per plane in any case); Standard maps every plane before the transfer.
 // In one process with fused halos the copies are stream-ordered work with
 // nothing to overlap, and the serial schedule runs.
+static nb_status sp_cg_box_iter(nb_cg *cg, int parity);
+
 nb_status nb_sparse_cg_hooks(nb_cg *cg, int parity) {
-    (void)parity;
+    if (cg->sp_box) return sp_cg_box_iter(cg, parity);
     nb_grid *g = cg->g;
     nb_field *p_ = cg->p[0];
     const nb_occ occ = cg->prm.occ;
@@ -1251,6 +1260,427 @@ nb_status nb_sparse_cg_hooks(nb_cg *cg, int parity) {
         A.c = (double *)cg->r->base[p];
         A.sc = cg->sc;
         NB_TRY(sp_launch<SPK_CG_R>(g, p, 0, g->parts[p].nz(), A, 0, "k_sp_cg_r"));
+    }
+    NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_RR, cg->sc, 0));
+    cg->k += 1;
+    return NB_OK;
+}
+
+// ===========================================================================
+// The 2-phase CG of the dense grid (64 B per cell, Ap
+// recomputed, not stored) on the element-sparse grid (a9).  A CTA owns a
+// 32 x 8 tile of the bounding box for a z-chunk and stages, per plane, the
+// 34 x 10 box around it from the compact arrays (8-byte cp.async, zero-fill
+// = the outside value 0 for inactive cells; buffer index = row word index +
+// popcount, the FEM box tables), three planes read while six more are in
+// flight (NB_SPB_NST = 9 slots: a 7-point plane is little work, so the
+// prefetch must be deep to keep ~50 KB per SM in flight).
+//   phase A (PH 0): own planes stage r and p_old; each thread turns its own
+//     box cells into p_new = r + beta p_old (fma(beta, p_old, r), the map's
+//     arithmetic) right after its copies land; halo planes stage the
+//     exchanged p_new.  Every active node stores p_new and, pending, x +=
+//     alpha_prev p_old; q = A p_new (canonical 7-point order) feeds <p_new, q>.
+//   phase B (PH 1): stages p_new, recomputes A p_new, r = fma(-alpha, A p, r),
+//     <r, r>.
+//   set-up (PH 2): stages x, r = b - A x, <r, r>.
+// 40 + 24 B per active cell and iteration (+ the ring rows from L2) against
+// the 96 B of the map / q / r schedule.  The dots are per 32 x 8 tile of a
+// plane in the dense canonical order (warp = tile row, rows added in y,
+// tiles by the finalize tree over the plane's tiles): every tile of every
+// chunk is launched (empty ones write zero partials), into the grid's sp_tp.
+// ===========================================================================
+#ifndef NB_SPB_NST
+#define NB_SPB_NST 9  // ring slots: planes pl-2 .. pl read, pl+1 .. pl+6 in flight (1 component: 2.7 KB a slot)
+#endif
+#ifndef NB_SPB_ZC
+#define NB_SPB_ZC 32
+#endif
+#ifndef NB_SPB_MINB
+#define NB_SPB_MINB 4  // 64 registers: 1.42 against 1.56 ms per iteration at 3
+#endif
+#define SPB_NST NB_SPB_NST
+#define SPB_ZC NB_SPB_ZC
+#define SPB_W 34
+#define SPB_H 10
+#define SPB_C (SPB_W * SPB_H)
+
+struct SpCgBoxArgs {
+    const int4 *items;  // {tile x (| 1 << 30: no active cell), tile y, zs, ze}
+    const uint32_t *rm;
+    const int32_t *ri;
+    int rw, nx, ny, gz0, nzl, NZ, T, tx;
+    double *tp;
+    const double *u;      // PH 0: halo planes' p_new (the p_new buffer); PH 1: p_new; PH 2: x
+    const double *r, *po;  // PH 0: r, p_old (own planes)
+    const double *b;       // PH 2
+    double *pn, *x;        // PH 0
+    double *ro;            // PH 1 / 2: r (read-modify-write / written)
+    const CgScal *sc;
+};
+
+__device__ __forceinline__ void spb_cp8(double *dst, const double *src, bool on) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(d), "l"(src), "r"(on ? 8 : 0) : "memory");
+}
+
+template <int PH>
+struct SpbCfg {
+    static constexpr int NPO = PH == 0 ? SPB_NST - 1 : 0;  // p_old slots (planes pl-1 .. pl+AHEAD)
+    static constexpr int SMEM = (SPB_NST + NPO) * SPB_C * 8;
+};
+
+template <int PH>
+__global__ void __launch_bounds__(256, NB_SPB_MINB) k_sp_cg_box(SpCgBoxArgs A) {
+    extern __shared__ __align__(16) double spb_sm[];
+    double(*S)[SPB_C] = reinterpret_cast<double(*)[SPB_C]>(spb_sm);
+    double(*PO)[SPB_C] = reinterpret_cast<double(*)[SPB_C]>(spb_sm + SPB_NST * SPB_C);
+    constexpr int NPO = SpbCfg<PH>::NPO;
+    __shared__ uint64_t RB[SPB_NST][SPB_H];
+    __shared__ double sw[2][8];
+    if (PH != 2 && A.sc->status != 0) return;
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const int4 it = A.items[blockIdx.x];
+    const int bxi = it.x & 0x3fffffff, x0 = bxi * 32, y0 = it.y * 8, zs = it.z, ze = it.w;
+    const int nout = ze - zs, np = nout + 2;
+    const int tile = it.y * A.tx + bxi;
+    if (it.x & 0x40000000) {  // no active cell in the tile's chunk: zero partials
+        for (int o = tid; o < nout; o += 256) A.tp[(int64_t)(A.gz0 + zs + o) * A.T + tile] = 0.0;
+        return;
+    }
+    const int wx = bxi;
+    double beta = 0.0, ap = 0.0, alpha = 0.0;
+    bool dox = false;
+    if constexpr (PH == 0) {
+        beta = A.sc->beta;
+        ap = A.sc->alpha_prev;
+        dox = A.sc->pending != 0;
+    }
+    if constexpr (PH == 1) alpha = A.sc->alpha;
+    int cx[2], cy[2];
+    bool cv[2];
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {
+        const int e = tid + 256 * k;
+        cx[k] = x0 - 1 + e % SPB_W;
+        cy[k] = y0 - 1 + e / SPB_W;
+        cv[k] = e < SPB_C && cx[k] >= 0 && cx[k] < A.nx && cy[k] >= 0 && cy[k] < A.ny;
+    }
+    const int ry = y0 - 1 + tid;
+    const bool rv = tid < SPB_H && ry >= 0 && ry < A.ny;
+    uint32_t tm[2] = {0u, 0u}, rl = 0u, rmid = 0u, rh = 0u;
+    int32_t ti[2] = {0, 0};
+    auto own = [&](int pl) { const int zl = zs - 1 + pl; return zl >= 0 && zl < A.nzl; };
+    auto fetch = [&](int pl) {
+        const int64_t row0 = (int64_t)(zs + pl) * A.ny;
+#pragma unroll
+        for (int k = 0; k < 2; ++k)
+            if (cv[k]) {
+                const int64_t q = (row0 + cy[k]) * A.rw + (cx[k] >> 5);
+                tm[k] = __ldg(A.rm + q);
+                ti[k] = __ldg(A.ri + q);
+            }
+        if (rv) {
+            const uint32_t *r = A.rm + (row0 + ry) * A.rw;
+            rl = wx > 0 ? __ldg(r + wx - 1) : 0u;
+            rmid = __ldg(r + wx);
+            rh = wx + 1 < A.rw ? __ldg(r + wx + 1) : 0u;
+        }
+    };
+    auto issue = [&](int pl) {
+        const int st = pl % SPB_NST;
+        const bool form = PH == 0 && own(pl);
+#pragma unroll
+        for (int k = 0; k < 2; ++k) {
+            const int e = tid + 256 * k;
+            if (e < SPB_C) {
+                const unsigned b = (unsigned)cx[k] & 31u;
+                const bool act = cv[k] && ((tm[k] >> b) & 1u);
+                const int64_t idx = act ? ti[k] + __popc(tm[k] & ((1u << b) - 1u)) : 0;
+                if (form) {
+                    spb_cp8(&S[st][e], A.r + idx, act);
+                    spb_cp8(&PO[pl % (NPO ? NPO : 1)][e], A.po + idx, act);
+                } else {
+                    spb_cp8(&S[st][e], A.u + idx, act);
+                }
+            }
+        }
+        if (tid < SPB_H)
+            RB[st][tid] = rv ? (uint64_t)(rl >> 31) | ((uint64_t)rmid << 1) | ((uint64_t)(rh & 1u) << 33) : 0ull;
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    constexpr int AHEAD = SPB_NST - 3;
+#pragma unroll 1
+    for (int pl = 0; pl < AHEAD; ++pl) {
+        if (pl < np) {
+            fetch(pl);
+            issue(pl);
+        } else {
+            asm volatile("cp.async.commit_group;" ::: "memory");
+        }
+    }
+    if (AHEAD < np) fetch(AHEAD);
+    const int x = x0 + lane, y = y0 + w;
+    const bool in = x < A.nx && y < A.ny;
+    const int ce = (w + 1) * SPB_W + lane + 1;
+    const uint32_t lmask = (1u << lane) - 1u;
+    double vo = 0.0, bo = 0.0;  // x (PH 0) or r (PH 1) or b (PH 2) of the next output, a step ahead
+    int32_t oi = 0;
+    int64_t ic = 0;
+#pragma unroll 1
+    for (int pl = 0; pl < np; ++pl) {
+        asm volatile("cp.async.wait_group %0;" ::"n"(AHEAD - 1) : "memory");
+        const int sl = pl % SPB_NST;
+        if constexpr (PH == 0) {
+            if (own(pl)) {
+#pragma unroll
+                for (int k = 0; k < 2; ++k) {
+                    const int e = tid + 256 * k;
+                    if (e < SPB_C) S[sl][e] = fma(beta, PO[pl % NPO][e], S[sl][e]);
+                }
+            }
+        }
+        __syncthreads();  // plane pl landed (p_new formed); slot of plane pl-3 free; sw of output pl-3 written
+        if (pl >= 3 && tid == 0) {  // tile partial of output pl-3: rows in increasing y
+            const double(&v)[8] = sw[(pl - 3) & 1];
+            double s = v[0];
+#pragma unroll
+            for (int k = 1; k < 8; ++k) s = __dadd_rn(s, v[k]);
+            A.tp[(int64_t)(A.gz0 + zs + pl - 3) * A.T + tile] = s;
+        }
+        if (pl + AHEAD < np) issue(pl + AHEAD);
+        else asm volatile("cp.async.commit_group;" ::: "memory");
+        if (pl + AHEAD + 1 < np) fetch(pl + AHEAD + 1);
+        if (pl >= 2) {  // output pl-2: centre plane pl-1
+            const int s0 = (pl + SPB_NST - 2) % SPB_NST, s1 = (pl + SPB_NST - 1) % SPB_NST;
+            double prod = 0.0;
+            if (in && ((RB[s1][w + 1] >> (lane + 1)) & 1u)) {
+                const double c = S[s1][ce];
+                double sum = S[s1][ce - 1];
+                sum = sum + S[s1][ce + 1];
+                sum = sum + S[s1][ce - SPB_W];
+                sum = sum + S[s1][ce + SPB_W];
+                sum = sum + S[s0][ce];
+                sum = sum + S[sl][ce];
+                const double ac = fma(6.0, c, -sum);
+                if constexpr (PH == 0) {
+                    __stcs(A.pn + ic, c);
+                    if (dox) __stcs(A.x + ic, fma(ap, PO[(pl - 1) % NPO][ce], vo));
+                    prod = __dmul_rn(c, ac);
+                } else if constexpr (PH == 1) {
+                    const double r = fma(-alpha, ac, vo);
+                    __stcs(A.ro + ic, r);
+                    prod = __dmul_rn(r, r);
+                } else {
+                    const double r = __dsub_rn(bo, ac);
+                    A.ro[ic] = r;
+                    prod = __dmul_rn(r, r);
+                }
+            }
+            const double ws = warp_sum_canon(prod);
+            if (lane == 0) sw[(pl - 2) & 1][w] = ws;
+        }
+        // the next output (pl - 1, centre plane pl): buffer index, operand a step ahead
+        if (pl >= 1 && pl - 1 < nout) {
+            const uint64_t cb = RB[sl][w + 1];
+            ic = oi + __popc((uint32_t)(cb >> 1) & lmask);
+            if (in && ((cb >> (lane + 1)) & 1u)) {
+                if constexpr (PH == 0) {
+                    if (dox) vo = __ldcs(A.x + ic);
+                } else if constexpr (PH == 1) {
+                    vo = __ldcs(A.ro + ic);
+                } else {
+                    bo = __ldg(A.b + ic);
+                }
+            }
+        }
+        if (in && pl < nout) oi = __ldg(A.ri + ((int64_t)(zs + pl + 1) * A.ny + y) * A.rw + wx);
+    }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncthreads();
+    if (tid == 0) {  // the last output's tile partial
+        const double(&v)[8] = sw[(nout - 1) & 1];
+        double s = v[0];
+#pragma unroll
+        for (int k = 1; k < 8; ++k) s = __dadd_rn(s, v[k]);
+        A.tp[(int64_t)(A.gz0 + zs + nout - 1) * A.T + tile] = s;
+    }
+}
+
+// work items of the box CG: EVERY (tile, chunk) of the plane ranges (the
+// tile partials of every tile are rewritten), empty ones flagged; cached
+static nb_status spb_items(nb_grid *g, int p, const std::vector<int> &ranges, const int4 **items, int64_t *n) {
+    NB_TRY(nb_sparse_fem_box_tables(g));
+    NbSparsePart &sp = g->sp[p];
+    std::vector<int> key = ranges;
+    key.push_back(-SPB_ZC);  // distinct from the FEM operator's lists
+    auto it = sp.box_lists.find(key);
+    if (it == sp.box_lists.end()) {
+        const int tx = (g->nx + 31) / 32, ty = (g->ny + 7) / 8;
+        std::vector<int4> v;
+        for (size_t r = 0; r + 1 < ranges.size(); r += 2)
+            for (int zs = ranges[r]; zs < ranges[r + 1]; zs += SPB_ZC) {
+                const int ze = std::min(zs + SPB_ZC, ranges[r + 1]);
+                for (int by = 0; by < ty; ++by)
+                    for (int bx = 0; bx < tx; ++bx) {
+                        bool any = false;
+                        for (int zl = zs; zl < ze && !any; ++zl)
+                            any = sp.tile_any[((size_t)zl * ty + by) * tx + bx] != 0;
+                        v.push_back(make_int4(bx | (any ? 0 : 0x40000000), by, zs, ze));
+                    }
+            }
+        int4 *d = nullptr;
+        if (!v.empty()) {
+            DeviceGuard dg(g->device);
+            NB_CUDA(cudaMalloc(&d, sizeof(int4) * v.size()));
+            NB_CUDA(cudaMemcpy(d, v.data(), sizeof(int4) * v.size(), cudaMemcpyHostToDevice));
+        }
+        it = sp.box_lists.emplace(key, std::make_pair(d, (int64_t)v.size())).first;
+    }
+    *items = it->second.first;
+    *n = it->second.second;
+    return NB_OK;
+}
+
+static std::vector<int> spb_ranges(const nb_grid *g, int p, int which) {
+    const NbPart &q = g->parts[p];
+    const int nz = q.nz();
+    if (which == 0) return {0, nz};
+    const int ib = q.lo >= 0 ? 1 : 0, ie = std::max(ib, nz - (q.hi >= 0 ? 1 : 0));
+    if (which == 1) return {ib, ie};
+    std::vector<int> r;
+    if (q.lo >= 0) r.insert(r.end(), {0, 1});
+    if (q.hi >= 0 && ie < nz) r.insert(r.end(), {nz - 1, nz});
+    return r;
+}
+
+// opt-in (NB_SP_CG_BOX=1): on the C4 sphere it measured 1.42 ms per iteration
+// against 0.63 for the map / q / r segment schedule although it moves 40 %
+// fewer bytes — it issues ~150 instructions per staged box cell (table
+// lookups, 8-byte copies, the per-plane barrier and tile dot), and the
+// sphere's boxes hold two cells per active one (ncu: 54 % issue, stalls at
+// the plane barrier 28 % and on loads 25 %; prefetch depth 3 .. 10 planes
+// made no difference).  On a full mask it gives the dense CG's bits.
+bool nb_sparse_cg_boxed() { return getenv("NB_SP_CG_BOX") != nullptr; }
+
+// tables, lists and the tile partial buffer (outside any graph capture)
+nb_status nb_sparse_cg_box_prepare(nb_grid *g) {
+    NB_TRY(nb_sparse_fem_box_tables(g));
+    if (!g->sp_tp) {
+        g->sp_T = ((g->nx + 31) / 32) * ((g->ny + 7) / 8);
+        NB_CUDA(cudaMalloc(&g->sp_tp, sizeof(double) * (size_t)g->nz * g->sp_T));
+        NB_CUDA(cudaMemset(g->sp_tp, 0, sizeof(double) * (size_t)g->nz * g->sp_T));
+    }
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+        for (int which = 0; which < 3; ++which) {
+            const int4 *it;
+            int64_t n;
+            NB_TRY(spb_items(g, p, spb_ranges(g, p, which), &it, &n));
+        }
+    static bool attr = false;
+    if (!attr) {
+        NB_CUDA(cudaFuncSetAttribute(k_sp_cg_box<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, SpbCfg<0>::SMEM));
+        attr = true;
+    }
+    return NB_OK;
+}
+
+// the grid's tile partial buffer in place of the segment partials for the
+// box kernels and the finalize that reads them
+struct SpTpSwap {
+    nb_grid *g;
+    double *tp;
+    int T;
+    explicit SpTpSwap(nb_grid *g_) : g(g_), tp(g_->tp), T(g_->T) {
+        g->tp = g->sp_tp;
+        g->T = g->sp_T;
+    }
+    ~SpTpSwap() {
+        g->tp = tp;
+        g->T = T;
+    }
+};
+
+static nb_status spb_launch(nb_grid *g, int p, int ph, int which, SpCgBoxArgs A, const char *name) {
+    const int4 *items;
+    int64_t n;
+    NB_TRY(spb_items(g, p, spb_ranges(g, p, which), &items, &n));
+    if (n <= 0) return NB_OK;
+    const NbSparsePart &sp = g->sp[p];
+    A.items = items;
+    A.rm = sp.d_rm;
+    A.ri = sp.d_ri;
+    A.rw = sp.rw;
+    A.nx = g->nx;
+    A.ny = g->ny;
+    A.gz0 = g->parts[p].z0;
+    A.nzl = g->parts[p].nz();
+    A.NZ = g->nz;
+    A.T = g->sp_T;
+    A.tx = (g->nx + 31) / 32;
+    A.tp = g->sp_tp;
+    LaunchScope ls(g, g->cs, name);
+    if (ph == 0)
+        k_sp_cg_box<0><<<(unsigned)n, 256, SpbCfg<0>::SMEM, g->cs>>>(A);
+    else if (ph == 1)
+        k_sp_cg_box<1><<<(unsigned)n, 256, SpbCfg<1>::SMEM, g->cs>>>(A);
+    else
+        k_sp_cg_box<2><<<(unsigned)n, 256, SpbCfg<2>::SMEM, g->cs>>>(A);
+    return nb_launch_check(name);
+}
+
+// set-up: r = b - A x0, rr0 (tile order)
+static nb_status sp_cg_box_init(nb_cg *cg) {
+    nb_grid *g = cg->g;
+    NB_TRY(nb_sparse_cg_box_prepare(g));
+    SpTpSwap sw(g);
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        SpCgBoxArgs A{};
+        A.u = (const double *)cg->x->base[p];
+        A.b = (const double *)cg->b->base[p];
+        A.ro = (double *)cg->r->base[p];
+        A.sc = cg->sc;
+        NB_TRY(spb_launch(g, p, 2, 0, A, "k_sp_cg_init"));
+    }
+    return nb_reduce_finalize(g, 1, FIN_CG_INIT, cg->sc, 0);
+}
+
+// one iteration: p_new of the boundary planes facing a neighbour -> their
+// halo (OCC: interior phase A while it flies) -> phase A -> alpha -> phase B
+// -> beta
+static nb_status sp_cg_box_iter(nb_cg *cg, int parity) {
+    nb_grid *g = cg->g;
+    nb_field *pn = cg->p[parity], *po = cg->p[parity ^ 1];
+    const bool split = cg->prm.occ != NB_OCC_NONE && g->nparts > 1 && (nb_is_peer(g) || nb_halo_on_stream(g));
+    SpTpSwap sw(g);
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
+        NB_TRY(nb_sparse_pmap(g, p, 1, (const double *)po->base[p], (const double *)cg->r->base[p],
+                              (double *)pn->base[p], cg->sc));
+    auto phase_a = [&](int p, int which) {
+        SpCgBoxArgs A{};
+        A.u = (const double *)pn->base[p];
+        A.r = (const double *)cg->r->base[p];
+        A.po = (const double *)po->base[p];
+        A.pn = (double *)pn->base[p];
+        A.x = (double *)cg->x->base[p];
+        A.sc = cg->sc;
+        return spb_launch(g, p, 0, which, A, "k_sp_cg_a");
+    };
+    if (!split) {
+        if (g->nparts > 1) NB_TRY(nb_sparse_halo_update(pn));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) NB_TRY(phase_a(p, 0));
+    } else {
+        NB_TRY(nb_halo_split_begin(pn, 0, 1, cg->hs));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) NB_TRY(phase_a(p, 1));
+        NB_TRY(nb_halo_split_wait(g, cg->hs));
+        for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) NB_TRY(phase_a(p, 2));
+    }
+    NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_PQ, cg->sc, 0));
+    for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
+        SpCgBoxArgs A{};
+        A.u = (const double *)pn->base[p];
+        A.ro = (double *)cg->r->base[p];
+        A.sc = cg->sc;
+        NB_TRY(spb_launch(g, p, 1, 0, A, "k_sp_cg_b"));
     }
     NB_TRY(nb_reduce_finalize(g, 1, FIN_CG_RR, cg->sc, 0));
     cg->k += 1;
@@ -1594,8 +2024,8 @@ nb_status nb_sparse_fem_cg_hooks(nb_cg *cg, int parity) {
                             (double *)cg->x->base[p]};
         };
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
-            NB_TRY(nb_sparse_fem_pmap(g, p, (const double *)po->base[p], (const double *)cg->r->base[p],
-                                      (double *)pn->base[p], cg->sc));
+            NB_TRY(nb_sparse_pmap(g, p, 3, (const double *)po->base[p], (const double *)cg->r->base[p],
+                                  (double *)pn->base[p], cg->sc));
         auto phase_a = [&](int p, int which) {
             const SpFemCgA c = cga(p);
             return nb_sparse_fem_box_ranges(g, p, which, nullptr, nullptr, (double *)cg->q->base[p], cg->sc, 3, &c);

@@ -212,3 +212,58 @@ def test_sparse_cg_xruns_bitwise_equal_connectivity_table(parts, monkeypatch):
         assert np.array_equal(xa, xb) and ra.rr == rb.rr and ra.rr0 == rb.rr0
         xo, ro, _ = oracle.cg(b, max_iter=9, op=oracle.OP_SPARSE7, mask=m)
         assert np.max(np.abs(xa - xo)) <= 1e-11 * np.max(np.abs(xo))
+
+
+@pytest.mark.parametrize("parts", [1, 2, 3])
+def test_sparse_cg_box_schedule_vs_segment_schedule_and_oracle(parts, monkeypatch):
+    """The 2-phase box CG (NB_SP_CG_BOX=1: p_new / x / <p, Ap> in phase A,
+    A p recomputed in phase B, dots per 32 x 8 tile) and the map / q / r
+    segment schedule (default) solve the same system: both within the CG
+    tolerance of the oracle (their dot orders differ, so not bitwise); ragged
+    tiles, several z-chunks, a mask with holes."""
+    rng = np.random.default_rng(5)
+    m = synth.sphere_mask(70, 0.45)[:40, :45, :].copy()
+    m &= (rng.random(m.shape) < 0.85).astype(np.uint8)
+    nz, ny, nx = m.shape
+    b = np.where(m, synth.uniform((nx, ny, nz), seed=6), 0.0)
+    xo, ro, _ = oracle.cg(b, max_iter=12, op=oracle.OP_SPARSE7, mask=m)
+    out = []
+    for seg in (False, True):
+        if seg:
+            monkeypatch.delenv("NB_SP_CG_BOX", raising=False)
+        else:
+            monkeypatch.setenv("NB_SP_CG_BOX", "1")
+        with nb.Grid((nx, ny, nz), nparts=parts, devices=[0] * parts, active=m) as g:
+            fb, fx = nb.Field(g), nb.Field(g)
+            fb.upload(b)
+            fx.fill_const(0.0)
+            r = nb.nb_cg_solve(fx, fb, max_iter=12, occ=nb.OCC_TWO_WAY)
+            x = fx.download()
+            fb.close(), fx.close()
+        assert r.iters == 12
+        assert np.max(np.abs(x - xo)) <= 1e-11 * np.max(np.abs(xo)), seg
+        assert abs(r.rr - ro.rr) <= 1e-9 * ro.rr
+        out.append(x)
+    assert np.max(np.abs(out[0] - out[1])) <= 1e-11 * np.max(np.abs(xo))
+
+
+@pytest.mark.parametrize("parts", [1, 2])
+def test_sparse_box_cg_full_mask_equals_dense_cg_bitwise(parts, monkeypatch):
+    """On a full mask the box CG runs the dense CG's arithmetic in the dense
+    canonical dot order (32 x 8 tiles, rows in y, tiles by the plane tree):
+    its iterates equal the dense grid's bit for bit."""
+    monkeypatch.setenv("NB_SP_CG_BOX", "1")
+    dims = (40, 21, 19)  # ragged x and y tiles
+    m = np.ones(dims[::-1], np.uint8)
+    b = synth.uniform(dims, seed=9)
+    xs = []
+    for active in (None, m):
+        with nb.Grid(dims, nparts=parts, devices=[0] * parts, active=active) as g:
+            fb, fx = nb.Field(g), nb.Field(g)
+            fb.upload(b)
+            fx.fill_const(0.0)
+            r = nb.nb_cg_solve(fx, fb, max_iter=10, occ=nb.OCC_NONE)
+            xs.append((fx.download(), r.rr, r.rr0))
+            fb.close(), fx.close()
+    assert xs[0][2] == xs[1][2] and xs[0][1] == xs[1][1]
+    assert np.array_equal(xs[0][0], xs[1][0])

@@ -33,7 +33,7 @@ ms = e0.elapsed_time(e1) / iters
 g.profile(True)
 cg.iterate(5)
 split = {}
-for nm in ("k_sp_cg_map", "k_sp_cg_q", "k_sp_cg_mq", "k_sp_cg_r", "k_finalize"):
+for nm in ("k_sp_cg_map", "k_sp_cg_q", "k_sp_cg_mq", "k_sp_cg_r", "k_sp_cg_a", "k_sp_cg_b", "k_finalize"):
     k, t = g.profile_read(nm)
     if k:
         split[nm] = t / 5
