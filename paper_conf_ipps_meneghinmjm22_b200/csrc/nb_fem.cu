@@ -2107,9 +2107,33 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
         A.u = cga->pn;  // halo planes: the exchanged p_new
     }
     const char *name = kind == 2 ? "k_fem_cg_init" : kind == 3 ? "k_sp_fem_cg_a" : (sc ? "k_sp_fem_q" : "k_fem_apply");
+    // the list nodes (kinds 0 / 2 read only the input) run on the side
+    // stream concurrently with the box kernel, which leaves the SMs room
+    // (the list kernel is latency-bound: 11-18 % issue alone); kind 3 reads
+    // the box kernel's p_new and runs after it
+    bool conc = false;
+    for (size_t r = 0; r + 1 < ranges.size(); r += 2)
+        conc |= sp.fnode_start[ranges[r + 1]] > sp.fnode_start[ranges[r]];
+    conc = conc && kind != 3 && !getenv("NB_SPF_SERIAL");
+    cudaStream_t ls_stream = g->cs;
+    if (conc) {
+        if (!g->fs) {
+            int lo, hi;
+            NB_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+            NB_CUDA(cudaStreamCreateWithPriority(&g->fs, cudaStreamNonBlocking, hi));
+            for (auto &e : g->fev) NB_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        }
+        NB_CUDA(cudaEventRecord(g->fev[0], g->cs));  // fork
+        NB_CUDA(cudaStreamWaitEvent(g->fs, g->fev[0], 0));
+        ls_stream = g->fs;
+    }
     {
         static bool attr = false;
         if (!attr) {
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         SfbCfg<0>::SMEM));
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         SfbCfg<2>::SMEM));
             NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          SfbCfg<3>::SMEM));
             attr = true;
@@ -2133,12 +2157,16 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
         if (e <= a) continue;
         const SpFemNode *L = (const SpFemNode *)sp.d_fnode;
         const unsigned nb = (unsigned)((e - a + 127) / 128);
-        LaunchScope ls(g, g->cs, name);
+        LaunchScope ls(g, ls_stream, name);
         if (kind == 2)
-            k_sp_fem_list<2><<<nb, 128, 0, g->cs>>>(L, a, e, sp.cs, u, b, y, sc);
+            k_sp_fem_list<2><<<nb, 128, 0, ls_stream>>>(L, a, e, sp.cs, u, b, y, sc);
         else
-            k_sp_fem_list<0><<<nb, 128, 0, g->cs>>>(L, a, e, sp.cs, u, b, y, sc);
+            k_sp_fem_list<0><<<nb, 128, 0, ls_stream>>>(L, a, e, sp.cs, u, b, y, sc);
         NB_TRY(nb_launch_check(name));
+    }
+    if (conc) {
+        NB_CUDA(cudaEventRecord(g->fev[2], g->fs));
+        NB_CUDA(cudaStreamWaitEvent(g->cs, g->fev[2], 0));  // join
     }
     return NB_OK;
 }

@@ -1579,6 +1579,8 @@ nb_status nb_sparse_cg_box_prepare(nb_grid *g) {
     static bool attr = false;
     if (!attr) {
         NB_CUDA(cudaFuncSetAttribute(k_sp_cg_box<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, SpbCfg<0>::SMEM));
+        NB_CUDA(cudaFuncSetAttribute(k_sp_cg_box<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, SpbCfg<1>::SMEM));
+        NB_CUDA(cudaFuncSetAttribute(k_sp_cg_box<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, SpbCfg<2>::SMEM));
         attr = true;
     }
     return NB_OK;
