@@ -680,6 +680,54 @@ def bench_fem_run(n, steps, warmup, world, local):
             **({"note": SHARED_NOTE} if _SHARED_GPU else {})}
 
 
+def bench_fem_sparse_run(n, steps, local):
+    """f4: the C5 FEM CG on element-
+    sparse grids at n^3 — the full cube (every node active: against the dense
+    C5 line) and the C4-recipe sphere (~30 % of the box) — with the K p
+    pass's FP64 roofline (box operator + list nodes, profiled serially)."""
+    import numpy as np
+    import torch
+
+    import paper_conf_ipps_meneghinmjm22_b200 as nb
+    import synth
+    out = {"unit": "MLUPS (active nodes)", "n_gpus": 1, "steps": steps, "dtype": "f64", "scaling": "strong",
+           "config": {"workload": f"f4 FEM Q1 linear elastic CG on element-sparse grids, {n}^3 box, 3 fp64 dof, "
+                                  "E=1 nu=0.3, Dirichlet z=0, pressure on exposed top faces",
+                      "schedule": "map 120 B + K p 48 B (box operator) + <p,q> 48 B + r 72 B per node"}}
+    f64, f64_kind = fp64_peak()
+    for name, mask in (("full_cube", np.ones((n, n, n), np.uint8)), ("sphere", synth.sphere_mask(n))):
+        act = int(mask.sum(dtype="int64"))
+        g = nb.Grid((n, n, n), nparts=1, devices=[local], active=mask)
+        stream = torch.cuda.ExternalStream(g.stream())
+        b, x = nb.Field(g, card=3), nb.Field(g, card=3)
+        nb.nb_fem27_rhs(b, 1.0)
+        x.fill_const(0.0)
+        cg = nb.CG(x, b, op=nb.OP_FEM27)
+        cg.iterate(3)
+        cg.prepare(steps)
+        g.sync()
+        ms, clocks = timed(1, stream, lambda: cg.iterate(steps), local)
+        os.environ["NB_SPF_SERIAL"] = "1"  # list nodes after the box kernel: separable kernel times
+        pit = 3
+        prof = _profiled_kernels(g, lambda: cg.iterate(pit), ["k_sp_fem_q", "k_sp_fem_dot", "k_sp_cg_map",
+                                                                "k_sp_cg_r"])
+        os.environ.pop("NB_SPF_SERIAL", None)
+        cg.finish()
+        cg.close(), b.close(), x.close(), g.close()
+        kp = prof["k_sp_fem_q"][1] / pit
+        out[name] = {"active_nodes": act, "value": act * steps / (ms / 1e3) / 1e6, "ms_per_step": ms / steps,
+                     "kernel_ms_per_iter": {k: v[1] / pit for k, v in prof.items()},
+                     "k_p_roofline": {"bound": "alu", "kernel": "k_sp_fem_box + k_sp_fem_list (q = K p)",
+                                      "achieved": FEM_FLOPS_PER_NODE * act / (kp / 1e3) / 1e12, "peak": f64,
+                                      "unit": "TFLOP/s",
+                                      "frac": FEM_FLOPS_PER_NODE * act / (kp / 1e3) / 1e12 / f64,
+                                      "peak_kind": f64_kind, "hbm_gbs_48B_per_node": 48 * act / (kp / 1e3) / 1e9},
+                     "clocks": clocks}
+    out["value"] = out["sphere"]["value"]
+    out["ms_per_step"] = out["sphere"]["ms_per_step"]
+    return out
+
+
 def bench_c1(local):
     """Config C1 (64^3 fp64, 10 map-stencil-reduce iterations, 1 GPU): a
     launch/latency-bound case.  Timed per synchronous nb_map_stencil_reduce
@@ -968,7 +1016,8 @@ def main():
                            "lbm_sparse_f2": bench_lbm_sparse_run(args.n, 20, 3, local),
                            "lbm_aa_f3": bench_lbm_aa_run(args.n, 20, 4, local),
                            "lbm_layouts_f3": bench_lbm_layouts(args.n, 10, local),
-                           "karman_f4": bench_karman(local)}
+                           "karman_f4": bench_karman(local),
+                           "fem_sparse_f4": bench_fem_sparse_run(384, 20, local)}
             out["cpu_baseline"] = cpu_baseline_cg(args.n)
             out["also"]["lbm_d3q19"]["cpu_baseline"] = cpu_baseline_lbm()
         elif not args.no_extras:
