@@ -3,7 +3,7 @@ sys.path.insert(0, os.getcwd())
 import torch
 import paper_conf_ipps_meneghinmjm22_b200 as nb
 import synth
-n=512; steps=20; cells=n**3
+n=512; steps=int(sys.argv[1]) if len(sys.argv) > 1 else 20; cells=n**3
 g = nb.Grid((n,n,n), devices=[0])
 stream = torch.cuda.ExternalStream(g.stream())
 b, x = nb.Field(g), nb.Field(g)
