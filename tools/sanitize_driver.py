@@ -154,4 +154,29 @@ with nb.Grid((30, 26, 24), nparts=2, devices=[0, 0]) as g:
     f19.halo_update()  # 38 plane copies in one batch
     for f in (b, x, r, p, q, a, c, f19):
         f.close()
+# round-2b additions: the sparse FEM box operator + list nodes (apply, CG
+# q pass, set-up), its fused phase A (NB_SPF_FUSED) and the 7-point 2-phase
+# box CG (NB_SP_CG_BOX) on a ragged mask spanning several tiles and z-chunks
+m = synth.sphere_mask(70, 0.45)[:36, :45, :].copy()
+nz, ny, nx = m.shape
+with nb.Grid((nx, ny, nz), nparts=2, devices=[0, 0], active=m) as g:
+    u, v = nb.Field(g, card=3), nb.Field(g, card=3)
+    u.fill_uniform(seed=7)
+    u.halo_update()
+    nb.nb_fem27_apply(u, v)
+    for env in (None, "NB_SPF_FUSED"):
+        if env:
+            os.environ[env] = "1"
+        nb.nb_fem27_rhs(v, 1.0)
+        u.fill_const(0.0)
+        nb.nb_cg_solve(u, v, max_iter=3, op=nb.OP_FEM27, occ=nb.OCC_TWO_WAY)
+        os.environ.pop("NB_SPF_FUSED", None)
+    x, b = nb.Field(g), nb.Field(g)
+    b.fill_uniform(seed=8)
+    x.fill_const(0.0)
+    os.environ["NB_SP_CG_BOX"] = "1"
+    nb.nb_cg_solve(x, b, max_iter=3, occ=nb.OCC_TWO_WAY)
+    os.environ.pop("NB_SP_CG_BOX", None)
+    for f in (u, v, x, b):
+        f.close()
 print("sanitize driver done")
