@@ -1854,8 +1854,12 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
         cy[k] = y0 - 1 + e / SFB_W;
         cv[k] = e < SFB_C && cx[k] >= 0 && cx[k] < A.nx && cy[k] >= 0 && cy[k] < A.ny;
     }
-    const int ry = y0 - 1 + tid;  // box row of threads tid < SFB_H
-    const bool rv = tid < SFB_H && ry >= 0 && ry < A.ny;
+    // the box rows' bits are built by threads that stage one cell only
+    // (tid >= SFB_C - 256 stage one, the others two): balanced plane steps
+    const int rt = tid - (SFB_C - 256);  // box row of threads 0 <= rt < SFB_H
+    const int ry = y0 - 1 + rt;
+    const bool rown = rt >= 0 && rt < SFB_H;
+    const bool rv = rown && ry >= 0 && ry < A.ny;
     uint32_t tm[2] = {0u, 0u}, rl = 0u, rm = 0u, rh = 0u;
     int32_t ti[2] = {0, 0};
     auto own = [&](int pl) { const int zl = zs - 1 + pl; return zl >= 0 && zl < A.nzl; };
@@ -1897,8 +1901,8 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
                 }
             }
         }
-        if (tid < SFB_H)  // activity bits of box row tid: bit i = x0 - 1 + i
-            RB[st][tid] = rv ? (uint64_t)(rl >> 31) | ((uint64_t)rm << 1) | ((uint64_t)(rh & 1u) << 33) : 0ull;
+        if (rown)  // activity bits of box row rt: bit i = x0 - 1 + i
+            RB[st][rt] = rv ? (uint64_t)(rl >> 31) | ((uint64_t)rm << 1) | ((uint64_t)(rh & 1u) << 33) : 0ull;
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
     // ring: at step pl (plane pl lands) planes pl-2 .. pl are read (the

@@ -1365,8 +1365,10 @@ __global__ void __launch_bounds__(256, NB_SPB_MINB) k_sp_cg_box(SpCgBoxArgs A) {
         cy[k] = y0 - 1 + e / SPB_W;
         cv[k] = e < SPB_C && cx[k] >= 0 && cx[k] < A.nx && cy[k] >= 0 && cy[k] < A.ny;
     }
-    const int ry = y0 - 1 + tid;
-    const bool rv = tid < SPB_H && ry >= 0 && ry < A.ny;
+    const int rt = tid - (SPB_C - 256);  // box row built by a one-cell thread
+    const int ry = y0 - 1 + rt;
+    const bool rown = rt >= 0 && rt < SPB_H;
+    const bool rv = rown && ry >= 0 && ry < A.ny;
     uint32_t tm[2] = {0u, 0u}, rl = 0u, rmid = 0u, rh = 0u;
     int32_t ti[2] = {0, 0};
     auto own = [&](int pl) { const int zl = zs - 1 + pl; return zl >= 0 && zl < A.nzl; };
@@ -1404,8 +1406,8 @@ __global__ void __launch_bounds__(256, NB_SPB_MINB) k_sp_cg_box(SpCgBoxArgs A) {
                 }
             }
         }
-        if (tid < SPB_H)
-            RB[st][tid] = rv ? (uint64_t)(rl >> 31) | ((uint64_t)rmid << 1) | ((uint64_t)(rh & 1u) << 33) : 0ull;
+        if (rown)
+            RB[st][rt] = rv ? (uint64_t)(rl >> 31) | ((uint64_t)rmid << 1) | ((uint64_t)(rh & 1u) << 33) : 0ull;
         asm volatile("cp.async.commit_group;" ::: "memory");
     };
     constexpr int AHEAD = SPB_NST - 3;
