@@ -1774,6 +1774,8 @@ struct SpFemBoxArgs {
     const double *r, *po;  // KIND 3: p_new = r + beta p_old formed while staging own planes
     double *pn, *x;        // KIND 3: p_new and the deferred x += alpha_prev p_old of own nodes
     const CgScal *sc;
+    double *tp;            // KIND 1: <u, q> tile partials [3][NZ][T] (dense canonical order)
+    int NZ, T, tx;
 };
 
 __device__ __forceinline__ void sfb_cp8(double *dst, const double *src, bool on) {
@@ -1827,13 +1829,31 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
     double(*PO)[3][SFB_C] = reinterpret_cast<double(*)[3][SFB_C]>(sfb_sm + NB_SFB_NST * 3 * SFB_C);
     constexpr int NPO = SfbCfg<KIND>::NPO;
     __shared__ uint64_t RB[NB_SFB_NST][SFB_H];
+    __shared__ double sw[2][3][8];  // KIND 1: per output parity, component, tile row
     if (A.sc && A.sc->status != 0) return;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const int4 it = A.items[blockIdx.x];
-    const int x0 = it.x * 32, y0 = it.y * 8, zs = it.z, ze = it.w;
+    const int bxi = it.x & 0x3fffffff;
+    const int x0 = bxi * 32, y0 = it.y * 8, zs = it.z, ze = it.w;
     const int np = ze - zs + 2;  // staged planes zs-1 .. ze
     const int nout = ze - zs;
-    const int wx = it.x;         // the tile's x word
+    const int wx = bxi;          // the tile's x word
+    const int tile = it.y * A.tx + bxi;
+    if (KIND == 1 && (it.x & 0x40000000)) {  // no active node in the tile's chunk: zero partials
+        for (int k = tid; k < 3 * nout; k += 256)
+            A.tp[((int64_t)(k / nout) * A.NZ + A.gz0 + zs + k % nout) * A.T + tile] = 0.0;
+        return;
+    }
+    // KIND 1: the tile partial of output o (3 components): rows in increasing y
+    auto flush = [&](int o) {
+        if (tid < 3) {
+            const double *v = sw[o & 1][tid];
+            double s = v[0];
+#pragma unroll
+            for (int k = 1; k < 8; ++k) s = __dadd_rn(s, v[k]);
+            A.tp[((int64_t)tid * A.NZ + A.gz0 + zs + o) * A.T + tile] = s;
+        }
+    };
     double beta = 0.0, ap = 0.0;
     bool dox = false;
     if constexpr (KIND == 3) {
@@ -1951,7 +1971,8 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
                 }
             }
         }
-        __syncthreads();  // plane pl landed (p_new formed); plane pl-3's slot is free
+        __syncthreads();  // plane pl landed (p_new formed); plane pl-3's slot is free; sw of output pl-3 written
+        if (KIND == 1 && pl >= 3) flush(pl - 3);
         if (pl + AHEAD < np) issue(pl + AHEAD);
         else asm volatile("cp.async.commit_group;" ::: "memory");
         if (pl + AHEAD + 1 < np) fetch(pl + AHEAD + 1);  // lands while this step computes
@@ -1965,6 +1986,7 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
             const int o = pl - 2, zl = zs + o;
             const int s0 = (pl + NB_SFB_NST - 2) % NB_SFB_NST, s1 = (pl + NB_SFB_NST - 1) % NB_SFB_NST;
             const int gz = A.gz0 + zl;
+            double prod[3] = {0.0, 0.0, 0.0};
             if (in && ((RB[s1][w + 1] >> (lane + 1)) & 1u)) {
                 if constexpr (KIND == 3) {  // every active own node: p_new, deferred x
 #pragma unroll
@@ -1989,6 +2011,16 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
                         A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], aA[c]) : aA[c];
                     }
                 }
+                if constexpr (KIND == 1) {  // <u, q>: the list kernel's q for the other nodes (it ran first)
+#pragma unroll
+                    for (int c = 0; c < 3; ++c)
+                        prod[c] = __dmul_rn(S[s1][c][ce], full ? aA[c] : __ldcs(A.y + c * A.cs + ic));
+                }
+            }
+            if constexpr (KIND == 1) {  // the tile row's 3 canonical warp sums
+                const double v = warp_sum_multi<3>(prod, lane);
+                const int i = warp_multi_index<3>(lane);
+                if (i < 3 && (lane & (32 / WarpMulti<3>::M - 1)) == 0) sw[o & 1][i][w] = v;
             }
         }
         // the next output (pl - 1, centre plane pl): its buffer index and x
@@ -2009,6 +2041,10 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
         }
     }
     asm volatile("cp.async.wait_group 0;" ::: "memory");
+    if constexpr (KIND == 1) {  // the last output's partials (the one before was flushed in the loop)
+        __syncthreads();
+        flush(nout - 1);
+    }
 }
 
 // The non-interior active nodes of the box operator (element set not full,
@@ -2085,8 +2121,7 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
                             const double *b, double *y, const CgScal *sc, const SpFemCgA *cga) {
     const int4 *items = nullptr;
     int64_t n = 0;
-    NB_TRY(nb_sparse_fem_box_list(g, p, ranges, NB_SFB_ZC, &items, &n));
-    if (n <= 0) return NB_OK;
+    NB_TRY(nb_sparse_fem_box_list(g, p, ranges, NB_SFB_ZC, &items, &n, kind == 1));
     const NbSparsePart &sp = g->sp[p];
     SpFemBoxArgs A{};
     A.items = items;
@@ -2096,12 +2131,19 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
     A.nx = g->nx;
     A.ny = g->ny;
     A.gz0 = g->parts[p].z0;
-    A.cs = sp.cs;
     A.nzl = g->parts[p].nz();
     A.u = u;
     A.b = b;
     A.y = y;
     A.sc = sc;
+    A.cs = sp.cs;
+    if (kind == 1) {  // <u, q> in tile order: the caller swaps sp_tp in for the finalize
+        NB_TRY(nb_sparse_tile_tp(g));
+        A.tp = g->sp_tp;
+        A.T = g->sp_T;
+        A.NZ = g->nz;
+        A.tx = (g->nx + 31) / 32;
+    }
     if (kind == 3) {
         if (!cga || !sc) NB_FAIL(NB_EINVAL, "sparse FEM phase A needs the CG buffers");
         A.r = cga->r;
@@ -2113,12 +2155,13 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
     const char *name = kind == 2 ? "k_fem_cg_init" : kind == 3 ? "k_sp_fem_cg_a" : (sc ? "k_sp_fem_q" : "k_fem_apply");
     // the list nodes (kinds 0 / 2 read only the input) run on the side
     // stream concurrently with the box kernel, which leaves the SMs room
-    // (the list kernel is latency-bound: 11-18 % issue alone); kind 3 reads
-    // the box kernel's p_new and runs after it
-    bool conc = false;
+    // (the list kernel is latency-bound: 11-18 % issue alone); kind 1 reads
+    // their q for the dot, so they run first; kind 3 reads the box kernel's
+    // p_new and runs after it
+    bool any_list = false;
     for (size_t r = 0; r + 1 < ranges.size(); r += 2)
-        conc |= sp.fnode_start[ranges[r + 1]] > sp.fnode_start[ranges[r]];
-    conc = conc && kind != 3 && !getenv("NB_SPF_SERIAL");
+        any_list |= sp.fnode_start[ranges[r + 1]] > sp.fnode_start[ranges[r]];
+    const bool conc = any_list && (kind == 0 || kind == 2) && !getenv("NB_SPF_SERIAL");
     cudaStream_t ls_stream = g->cs;
     if (conc) {
         if (!g->fs) {
@@ -2131,11 +2174,30 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
         NB_CUDA(cudaStreamWaitEvent(g->fs, g->fev[0], 0));
         ls_stream = g->fs;
     }
-    {
+    auto lists = [&](int lk, const double *lu) -> nb_status {
+        // the ranges' non-interior nodes (contiguous per range: the list is in plane order)
+        for (size_t r = 0; r + 1 < ranges.size(); r += 2) {
+            const int64_t a = sp.fnode_start[ranges[r]], e = sp.fnode_start[ranges[r + 1]];
+            if (e <= a) continue;
+            const SpFemNode *L = (const SpFemNode *)sp.d_fnode;
+            const unsigned nb = (unsigned)((e - a + 127) / 128);
+            LaunchScope ls(g, ls_stream, name);
+            if (lk == 2)
+                k_sp_fem_list<2><<<nb, 128, 0, ls_stream>>>(L, a, e, sp.cs, lu, b, y, sc);
+            else
+                k_sp_fem_list<0><<<nb, 128, 0, ls_stream>>>(L, a, e, sp.cs, lu, b, y, sc);
+            NB_TRY(nb_launch_check(name));
+        }
+        return NB_OK;
+    };
+    if (kind == 1) NB_TRY(lists(0, u));
+    if (n > 0) {
         static bool attr = false;
         if (!attr) {
             NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          SfbCfg<0>::SMEM));
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         SfbCfg<1>::SMEM));
             NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          SfbCfg<2>::SMEM));
             NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -2147,27 +2209,14 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
             k_sp_fem_box<2><<<(unsigned)n, 256, SfbCfg<2>::SMEM, g->cs>>>(A);
         else if (kind == 3)
             k_sp_fem_box<3><<<(unsigned)n, 256, SfbCfg<3>::SMEM, g->cs>>>(A);
+        else if (kind == 1)
+            k_sp_fem_box<1><<<(unsigned)n, 256, SfbCfg<1>::SMEM, g->cs>>>(A);
         else
             k_sp_fem_box<0><<<(unsigned)n, 256, SfbCfg<0>::SMEM, g->cs>>>(A);
         NB_TRY(nb_launch_check(name));
     }
-    if (kind == 3) {  // the list nodes' q = K p_new reads the stored p_new
-        kind = 0;
-        u = cga->pn;
-    }
-    // the ranges' non-interior nodes (contiguous per range: the list is in plane order)
-    for (size_t r = 0; r + 1 < ranges.size(); r += 2) {
-        const int64_t a = sp.fnode_start[ranges[r]], e = sp.fnode_start[ranges[r + 1]];
-        if (e <= a) continue;
-        const SpFemNode *L = (const SpFemNode *)sp.d_fnode;
-        const unsigned nb = (unsigned)((e - a + 127) / 128);
-        LaunchScope ls(g, ls_stream, name);
-        if (kind == 2)
-            k_sp_fem_list<2><<<nb, 128, 0, ls_stream>>>(L, a, e, sp.cs, u, b, y, sc);
-        else
-            k_sp_fem_list<0><<<nb, 128, 0, ls_stream>>>(L, a, e, sp.cs, u, b, y, sc);
-        NB_TRY(nb_launch_check(name));
-    }
+    if (kind == 0 || kind == 2) NB_TRY(lists(kind, u));
+    if (kind == 3) NB_TRY(lists(0, cga->pn));  // the list nodes' q = K p_new reads the stored p_new
     if (conc) {
         NB_CUDA(cudaEventRecord(g->fev[2], g->fs));
         NB_CUDA(cudaStreamWaitEvent(g->cs, g->fev[2], 0));  // join
@@ -2242,9 +2291,10 @@ nb_status nb_sparse_fem_box_prepare(nb_grid *g) {
         for (int which = 0; which < 3; ++which) {
             const int4 *it;
             int64_t n;
-            NB_TRY(nb_sparse_fem_box_list(g, p, sp_box_ranges(g, p, which), NB_SFB_ZC, &it, &n));
+            NB_TRY(nb_sparse_fem_box_list(g, p, sp_box_ranges(g, p, which), NB_SFB_ZC, &it, &n, false));
+            NB_TRY(nb_sparse_fem_box_list(g, p, sp_box_ranges(g, p, which), NB_SFB_ZC, &it, &n, true));
         }
-    return NB_OK;
+    return nb_sparse_tile_tp(g);
 }
 
 nb_status nb_sparse_fem_rhs(nb_field *b, double pr);

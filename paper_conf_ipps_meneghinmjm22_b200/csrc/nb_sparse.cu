@@ -1567,11 +1567,7 @@ bool nb_sparse_cg_boxed() { return getenv("NB_SP_CG_BOX") != nullptr; }
 // tables, lists and the tile partial buffer (outside any graph capture)
 nb_status nb_sparse_cg_box_prepare(nb_grid *g) {
     NB_TRY(nb_sparse_fem_box_tables(g));
-    if (!g->sp_tp) {
-        g->sp_T = ((g->nx + 31) / 32) * ((g->ny + 7) / 8);
-        NB_CUDA(cudaMalloc(&g->sp_tp, sizeof(double) * (size_t)g->nz * g->sp_T));
-        NB_CUDA(cudaMemset(g->sp_tp, 0, sizeof(double) * (size_t)g->nz * g->sp_T));
-    }
+    NB_TRY(nb_sparse_tile_tp(g));
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
         for (int which = 0; which < 3; ++which) {
             const int4 *it;
@@ -1587,22 +1583,6 @@ nb_status nb_sparse_cg_box_prepare(nb_grid *g) {
     }
     return NB_OK;
 }
-
-// the grid's tile partial buffer in place of the segment partials for the
-// box kernels and the finalize that reads them
-struct SpTpSwap {
-    nb_grid *g;
-    double *tp;
-    int T;
-    explicit SpTpSwap(nb_grid *g_) : g(g_), tp(g_->tp), T(g_->T) {
-        g->tp = g->sp_tp;
-        g->T = g->sp_T;
-    }
-    ~SpTpSwap() {
-        g->tp = tp;
-        g->T = T;
-    }
-};
 
 static nb_status spb_launch(nb_grid *g, int p, int ph, int which, SpCgBoxArgs A, const char *name) {
     const int4 *items;
@@ -1921,11 +1901,12 @@ nb_status nb_sparse_fem_box_tables(nb_grid *g) {
 // the local plane ranges holding an active node, chunk-major (neighbouring
 // tiles of a chunk run together and share their ring rows in L2); cached
 nb_status nb_sparse_fem_box_list(nb_grid *g, int p, const std::vector<int> &ranges, int zc, const int4 **items,
-                                 int64_t *n) {
+                                 int64_t *n, bool all) {
     NB_TRY(nb_sparse_fem_box_tables(g));
     NbSparsePart &sp = g->sp[p];
     std::vector<int> key = ranges;
     key.push_back(zc);
+    key.push_back(all ? 1 : 0);
     auto it = sp.box_lists.find(key);
     if (it == sp.box_lists.end()) {
         const int tx = (g->nx + 31) / 32, ty = (g->ny + 7) / 8;
@@ -1938,7 +1919,8 @@ nb_status nb_sparse_fem_box_list(nb_grid *g, int p, const std::vector<int> &rang
                         bool any = false;
                         for (int zl = zs; zl < ze && !any; ++zl)
                             any = sp.tile_any[((size_t)zl * ty + by) * tx + bx] != 0;
-                        if (any) v.push_back(make_int4(bx, by, zs, ze));
+                        // all: every tile (its dot partials are rewritten), empty ones flagged
+                        if (any || all) v.push_back(make_int4(bx | (any ? 0 : 0x40000000), by, zs, ze));
                     }
             }
         int4 *d = nullptr;
@@ -1951,6 +1933,18 @@ nb_status nb_sparse_fem_box_list(nb_grid *g, int p, const std::vector<int> &rang
     }
     *items = it->second.first;
     *n = it->second.second;
+    return NB_OK;
+}
+
+// tile partials of the box kernels' dots: [3 components][nz][sp_T], sp_T =
+// the 32 x 8 tiles of a plane (the dense canonical order); lazy
+nb_status nb_sparse_tile_tp(nb_grid *g) {
+    if (g->sp_tp) return NB_OK;
+    DeviceGuard dg(g->device);
+    g->sp_T = ((g->nx + 31) / 32) * ((g->ny + 7) / 8);
+    const size_t n = (size_t)3 * g->nz * g->sp_T;
+    NB_CUDA(cudaMalloc(&g->sp_tp, sizeof(double) * n));
+    NB_CUDA(cudaMemset(g->sp_tp, 0, sizeof(double) * n));
     return NB_OK;
 }
 
@@ -2076,12 +2070,18 @@ nb_status nb_sparse_fem_cg_hooks(nb_cg *cg, int parity) {
     // box operator (default): q = K p over plane ranges (which: 0 all, 1
     // interior, 2 boundary planes), then <p, q> per segment in one pass
     const bool box = nb_sparse_fem_boxed();
+    // <p, q> in a separate segment-order pass (default: the gather pass's
+    // dot, so the box schedule is bitwise equal to it) or, with
+    // NB_SPF_TILEDOT=1, inside the box kernel in tile order (into sp_tp; the
+    // list nodes then run first, not concurrently): 3.19 against 3.28 ms per
+    // iteration on the full 384^3 cube but 1.24 against 1.22 on the sphere
+    const bool segdot = box && !getenv("NB_SPF_TILEDOT");
     auto qbox = [&](int p, int which) {
         return nb_sparse_fem_box_ranges(g, p, which, (const double *)p_->base[p], nullptr, (double *)cg->q->base[p],
-                                        cg->sc, 0, nullptr);
+                                        cg->sc, segdot ? 0 : 1, nullptr);
     };
     auto qdot = [&]() -> nb_status {
-        if (box)
+        if (segdot)
             for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
                 NB_TRY(nb_sparse_fem_dot(g, p, (const double *)p_->base[p], (const double *)cg->q->base[p], cg->sc));
         return NB_OK;
@@ -2118,7 +2118,12 @@ nb_status nb_sparse_fem_cg_hooks(nb_cg *cg, int parity) {
         }
     }
     NB_TRY(qdot());
-    NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));
+    if (box && !segdot) {
+        SpTpSwap sw(g);
+        NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));
+    } else {
+        NB_TRY(nb_reduce_finalize(g, 3, FIN_CG_PQ, cg->sc, 0));
+    }
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p)
         for (int c = 0; c < 3; ++c) {
             SpArgs A{};

@@ -118,8 +118,10 @@ def test_sparse_fem_cg_converges():
 
 def _run_both(fn, modes=("NB_SPF_NONE", "NB_SPF_GATHER")):
     """fn() under each switch in `modes` set to 1 (NB_SPF_NONE: the default,
-    the shared-memory box operator after a separate map; NB_SPF_GATHER: the
-    gather pass; NB_SPF_FUSED: the box operator's fused CG phase A)."""
+    the shared-memory box operator after a separate map, <p, q> in a
+    separate segment-order pass; NB_SPF_TILEDOT: <p, q> in tile order inside
+    the box kernel; NB_SPF_GATHER: the gather pass; NB_SPF_FUSED: the box
+    operator's fused CG phase A)."""
     import os
     outs = []
     for m in modes:
@@ -170,6 +172,11 @@ def test_sparse_fem_box_equals_gather_bitwise(name, parts):
             fb.close(), fx.close()
         return x, r.rr, r.iters
 
+    # the segment-order dot schedules: bitwise equal (same per-node arithmetic, same dots)
     (xa, rra, ia), (xb, rrb, ib), (xc, rrc, ic) = _run_both(cg, ("NB_SPF_NONE", "NB_SPF_GATHER", "NB_SPF_FUSED"))
     assert ia == ib == ic and rra == rrb == rrc
     assert np.array_equal(xa, xb) and np.array_equal(xa, xc)
+    # <p, q> in tile order (NB_SPF_TILEDOT): the same solve up to the dot's rounding
+    (xd, rrd, idd), = _run_both(cg, ("NB_SPF_TILEDOT",))
+    assert idd == ia and abs(rrd - rra) <= 1e-12 * rra
+    assert np.max(np.abs(xd - xa)) <= 1e-12 * np.max(np.abs(xa))

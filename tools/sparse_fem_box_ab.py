@@ -16,11 +16,12 @@ import synth
 
 N = int(sys.argv[1]) if len(sys.argv) > 1 else 384
 KS = ("k_sp_fem_cg_a", "k_sp_fem_q", "k_sp_fem_dot", "k_sp_cg_map", "k_sp_cg_r", "k_finalize")
-MODES = {"box": {}, "fused": {"NB_SPF_FUSED": "1"}, "gather": {"NB_SPF_GATHER": "1"}}
+MODES = {"box": {}, "tiledot": {"NB_SPF_TILEDOT": "1"}, "fused": {"NB_SPF_FUSED": "1"},
+         "gather": {"NB_SPF_GATHER": "1"}}
 
 
 def run(mask, mode, iters=10):
-    for k in ("NB_SPF_FUSED", "NB_SPF_GATHER"):
+    for k in ("NB_SPF_FUSED", "NB_SPF_GATHER", "NB_SPF_TILEDOT"):
         os.environ.pop(k, None)
     os.environ.update(MODES[mode])
     g = nb.Grid((N, N, N), active=mask)
@@ -54,7 +55,7 @@ for name, mask in (("full", np.ones((N, N, N), np.uint8)), ("sphere", synth.sphe
     r = {"active": act}
     for mode in MODES:
         r[mode] = run(mask, mode)
-    r["same_bits"] = len({r[m]["x_digest"] for m in MODES}) == 1
+    r["same_bits_segment_dot"] = len({r[m]["x_digest"] for m in ("box", "fused", "gather")}) == 1
     out[name] = r
     print(name, json.dumps(r), flush=True)
 os.makedirs("gpurun_out", exist_ok=True)
