@@ -2192,8 +2192,8 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
     };
     if (kind == 1) NB_TRY(lists(0, u));
     if (n > 0) {
-        static bool attr = false;
-        if (!attr) {
+        static unsigned attr_set = 0;  // per device: dynamic shared memory above 48 KB
+        if (g->device >= 32 || !(attr_set & (1u << g->device))) {
             NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          SfbCfg<0>::SMEM));
             NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -2202,7 +2202,7 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
                                          SfbCfg<2>::SMEM));
             NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box<3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          SfbCfg<3>::SMEM));
-            attr = true;
+            if (g->device < 32) attr_set |= 1u << g->device;
         }
         LaunchScope ls(g, g->cs, name);
         if (kind == 2)

@@ -1574,12 +1574,12 @@ nb_status nb_sparse_cg_box_prepare(nb_grid *g) {
             int64_t n;
             NB_TRY(spb_items(g, p, spb_ranges(g, p, which), &it, &n));
         }
-    static bool attr = false;
-    if (!attr) {
+    static unsigned attr_set = 0;  // per device: dynamic shared memory above 48 KB
+    if (g->device >= 32 || !(attr_set & (1u << g->device))) {
         NB_CUDA(cudaFuncSetAttribute(k_sp_cg_box<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, SpbCfg<0>::SMEM));
         NB_CUDA(cudaFuncSetAttribute(k_sp_cg_box<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, SpbCfg<1>::SMEM));
         NB_CUDA(cudaFuncSetAttribute(k_sp_cg_box<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, SpbCfg<2>::SMEM));
-        attr = true;
+        if (g->device < 32) attr_set |= 1u << g->device;
     }
     return NB_OK;
 }
@@ -1851,11 +1851,12 @@ nb_status nb_sparse_fem_box_tables(nb_grid *g) {
             const int64_t k = ((int64_t)s * ny + y) * rw + (x >> 5);
             return ri[k] + __builtin_popcount(rm[k] & ((1u << (x & 31)) - 1u));
         };
-        struct Node {
+        struct Node {  // nb_fem.cu SpFemNode
             int32_t i, gz;
             uint32_t m;
             int32_t base[9];
         };
+        static_assert(sizeof(Node) == 48, "k_sp_fem_list reads 48-byte records");
         std::vector<Node> nodes;
         sp.fnode_start.assign(nzl + 1, 0);
         for (int zl = 0; zl < nzl; ++zl) {
