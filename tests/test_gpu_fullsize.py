@@ -136,3 +136,41 @@ def test_c2_poisson_cg_1024_max_size_vs_oracle():
     assert abs(r.rr0 - hist[0]) <= 1e-12 * hist[0]
     assert abs(r.rr - ro.rr) <= 1e-10 * ro.rr
     assert np.max(np.abs(x - xo)) <= 1e-11 * np.max(np.abs(xo))
+
+
+@pytest.mark.parametrize("shape", ["sphere", "cube"])
+def test_f4_sparse_fem_384_sampled_nodes_vs_oracle(shape):
+    """FEM on element-sparse grids at the C5 size (384^3) through the box
+    operator and its list nodes, in the bench's launch configuration: the
+    C4-recipe sphere (30 % of the box) and the full cube (Dirichlet plane,
+    faces, edges).  Sampled nodes — interior ones (box kernel) and surface /
+    gz <= 1 ones (list kernel) — against the masked oracle on the 3x3x3
+    neighbourhood block (a node's K u row only involves its 8 elements)."""
+    n = 384
+    m = synth.sphere_mask(n) if shape == "sphere" else np.ones((n, n, n), np.uint8)
+    rng = np.random.default_rng(1)
+    act = np.argwhere(m)
+    pts = [tuple(int(v) for v in act[i][::-1]) for i in rng.integers(0, len(act), 12)]
+    # surface nodes: the first and last active x of a few rows
+    for (z, y) in ((n // 2, n // 2), (n // 3, n // 2 + 7), (2 * n // 3, n // 4 + 40)):
+        xs = np.flatnonzero(m[z, y])
+        if xs.size:
+            pts += [(int(xs[0]), y, z), (int(xs[-1]), y, z)]
+    if shape == "cube":
+        pts += [(0, 0, 0), (n - 1, n - 1, n - 1), (5, 7, 1), (n // 2, 0, 2), (n - 1, n // 2, n // 2)]
+    with nb.Grid((n, n, n), active=m) as g:
+        u, y = nb.Field(g, card=3), nb.Field(g, card=3)
+        u.fill_uniform(seed=5)
+        nb.nb_fem27_apply(u, y)
+        ug, yg = u.download(), y.download()
+        u.close(), y.close()
+    for (x, yy, z) in pts:
+        assert m[z, yy, x]
+        sl = [slice(max(c - 1, 0), min(c + 2, n)) for c in (z, yy, x)]
+        mb = np.ascontiguousarray(m[sl[0], sl[1], sl[2]])
+        blk = np.ascontiguousarray(ug[:, sl[0], sl[1], sl[2]])
+        exp = oracle.fem_apply(blk, 1.0, 0.3, dirichlet_z0=(sl[0].start == 0), mask=mb)
+        loc = (z - sl[0].start, yy - sl[1].start, x - sl[2].start)
+        e = exp[:, loc[0], loc[1], loc[2]]
+        got = yg[:, z, yy, x]
+        assert np.max(np.abs(got - e)) <= 1e-13 * max(1.0, np.max(np.abs(e))), (shape, x, yy, z)
