@@ -355,7 +355,11 @@ nb_status nb_d2q9_step(nb_field **fin, nb_field **fout, const nb_d2q9_params *pa
 
 /* ---- FEM: Q1 hex linear elasticity, 27-point ------- */
 /* y = K u (card 3 fp64), Dirichlet u = 0 on the z = 0 plane (identity
- * rows/cols).  Reads u's halo planes: call nb_halo_update(u) first. */
+ * rows/cols).  Reads u's halo planes: call nb_halo_update(u) first.
+ * Element-sparse grids: nodes = active cells, an
+ * element exists iff its 8 nodes are active; y is written at active nodes
+ * only.  NB_EMISMATCH unless u, y are fp64 card-3 fields of one grid;
+ * NB_EUNSUPPORTED for the AoS layout. */
 nb_status nb_fem27_apply(const nb_field *u, nb_field *y, double E, double nu);
 /* b = consistent nodal load of pressure p on the top (z = Nz-1) face */
 nb_status nb_fem27_rhs(nb_field *b, double pressure);
