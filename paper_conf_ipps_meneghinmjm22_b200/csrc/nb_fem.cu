@@ -2047,6 +2047,157 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
     }
 }
 
+// Warp-specialised variant of k_sp_fem_box for kinds 0 / 2 (default;
+// NB_SFB_WS=0 selects the kernel above): two producer warps stage the planes
+// (table words, 8-byte cp.async, row bits) up to NB_SFW_NST planes ahead and
+// signal each slot through an mbarrier (cp.async.mbarrier.arrive.noinc + a
+// release arrive for the row bits); eight consumer warps run the same z-march
+// and epilogue and release a slot (one arrive per warp) after its last read.
+// No CTA-wide barrier in the plane loop: in the single-role kernel the plane
+// barrier and the uneven staging (1.33 cells per thread) held a quarter of
+// the stall samples.  Same arithmetic: same bits.
+#ifndef NB_SFW_NST
+#define NB_SFW_NST 8
+#endif
+#define SFW_PT 64  // producer threads
+#define SFW_SMEM (NB_SFW_NST * 3 * SFB_C * 8)
+
+__device__ __forceinline__ void sfw_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void sfw_cp_arrive(uint64_t *bar) {
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+template <int KIND>  // 0: y = K u; 2: y = b - K u
+__global__ void __launch_bounds__(256 + SFW_PT, 3) k_sp_fem_boxw(SpFemBoxArgs A) {
+    extern __shared__ __align__(16) double sfw_sm[];
+    double(*S)[3][SFB_C] = reinterpret_cast<double(*)[3][SFB_C]>(sfw_sm);
+    __shared__ uint64_t RB[NB_SFW_NST][SFB_H];
+    __shared__ __align__(8) uint64_t full[NB_SFW_NST], empty[NB_SFW_NST];
+    if (A.sc && A.sc->status != 0) return;
+    const int tid = threadIdx.x;
+    const int4 it = A.items[blockIdx.x];
+    const int bxi = it.x & 0x3fffffff;
+    const int x0 = bxi * 32, y0 = it.y * 8, zs = it.z, ze = it.w;
+    const int np = ze - zs + 2;
+    const int nout = ze - zs;
+    const int wx = bxi;
+    if (tid == 0) {
+        for (int k = 0; k < NB_SFW_NST; ++k) {
+            mbar_init(&full[k], SFW_PT + SFB_H);  // producers' copies + the row-bit writers
+            mbar_init(&empty[k], 8);              // one arrive per consumer warp
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (tid >= 256) {  // ---- producers ----
+        const int pt = tid - 256;
+        constexpr int NC = (SFB_C + SFW_PT - 1) / SFW_PT;
+#pragma unroll 1
+        for (int q = 0; q < np; ++q) {
+            const int st = q % NB_SFW_NST;
+            if (q >= NB_SFW_NST) mbar_wait(&empty[st], (uint32_t)((q / NB_SFW_NST) - 1) & 1u);
+            const int64_t row0 = (int64_t)(zs + q) * A.ny;  // slab row of (zl + 1, y = 0), zl = zs - 1 + q
+            uint32_t tm[NC];
+            int32_t ti[NC];
+#pragma unroll
+            for (int k = 0; k < NC; ++k) {
+                const int e = pt + SFW_PT * k;
+                const int x = x0 - 1 + e % SFB_W, yy = y0 - 1 + e / SFB_W;
+                tm[k] = 0u;
+                ti[k] = 0;
+                if (e < SFB_C && x >= 0 && x < A.nx && yy >= 0 && yy < A.ny) {
+                    const int64_t kk = (row0 + yy) * A.rw + (x >> 5);
+                    tm[k] = __ldg(A.rm + kk);
+                    ti[k] = __ldg(A.ri + kk);
+                }
+            }
+#pragma unroll
+            for (int k = 0; k < NC; ++k) {
+                const int e = pt + SFW_PT * k;
+                if (e < SFB_C) {
+                    const unsigned b = (unsigned)(x0 - 1 + e % SFB_W) & 31u;
+                    const bool act = (tm[k] >> b) & 1u;
+                    const int64_t idx = act ? ti[k] + __popc(tm[k] & ((1u << b) - 1u)) : 0;
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) sfb_cp8(&S[st][c][e], A.u + c * A.cs + idx, act);
+                }
+            }
+            sfw_cp_arrive(&full[st]);  // fires when this thread's copies have landed
+            if (pt < SFB_H) {           // activity bits of box row pt: bit i = x0 - 1 + i
+                const int ry = y0 - 1 + pt;
+                uint64_t bits = 0ull;
+                if (ry >= 0 && ry < A.ny) {
+                    const uint32_t *r = A.rm + (row0 + ry) * A.rw;
+                    const uint32_t rl = wx > 0 ? __ldg(r + wx - 1) : 0u, rm = __ldg(r + wx);
+                    const uint32_t rh = wx + 1 < A.rw ? __ldg(r + wx + 1) : 0u;
+                    bits = (uint64_t)(rl >> 31) | ((uint64_t)rm << 1) | ((uint64_t)(rh & 1u) << 33);
+                }
+                RB[st][pt] = bits;
+                sfw_arrive(&full[st]);
+            }
+        }
+        asm volatile("cp.async.wait_all;" ::: "memory");
+        return;
+    }
+    // ---- consumers: k_sp_fem_box's z-march and epilogue ----
+    const int lane = tid & 31, w = tid >> 5;
+    const int x = x0 + lane, y = y0 + w;
+    const bool in = x < A.nx && y < A.ny;
+    const int ce = (w + 1) * SFB_W + lane + 1;
+    const uint32_t lmask = (1u << lane) - 1u;
+    double aA[3] = {0.0, 0.0, 0.0}, aB[3] = {0.0, 0.0, 0.0};
+    int32_t oi = 0;
+    int64_t ic = 0;
+    mbar_wait(&full[0], 0u);
+#pragma unroll 1
+    for (int pl = 0; pl < np; ++pl) {
+        const int sl = pl % NB_SFW_NST;
+        // plane pl+1 too: its row bits take part in the skip test below
+        if (pl + 1 < np) mbar_wait(&full[(pl + 1) % NB_SFW_NST], (uint32_t)((pl + 1) / NB_SFW_NST) & 1u);
+        double aC[3] = {0.0, 0.0, 0.0};
+        const uint64_t rows = (pl >= 1 ? RB[(pl + NB_SFW_NST - 1) % NB_SFW_NST][w + 1] : 0ull) | RB[sl][w + 1] |
+                              (pl + 1 < np ? RB[(pl + 1) % NB_SFW_NST][w + 1] : 0ull);
+        if ((rows >> 1) & 0xffffffffull) sfb_plane<0>(&S[sl][0][ce], aA, aB, aC);
+        if (pl >= 2) {
+            const int o = pl - 2, zl = zs + o;
+            const int s0 = (pl + NB_SFW_NST - 2) % NB_SFW_NST, s1 = (pl + NB_SFW_NST - 1) % NB_SFW_NST;
+            const int gz = A.gz0 + zl;
+            if (in && ((RB[s1][w + 1] >> (lane + 1)) & 1u)) {
+                bool full_nb = gz >= 2;
+#pragma unroll
+                for (int r = 0; r < 9; ++r) {
+                    const int oy = r % 3 - 1, oz = r / 3 - 1;
+                    const int st = oz < 0 ? s0 : (oz == 0 ? s1 : sl);
+                    full_nb = full_nb && ((RB[st][w + 1 + oy] >> lane) & 7u) == 7u;
+                }
+                if (full_nb) {
+#pragma unroll
+                    for (int c = 0; c < 3; ++c) {
+                        const int64_t kk = c * A.cs + ic;
+                        A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], aA[c]) : aA[c];
+                    }
+                }
+            }
+        }
+        if (pl >= 1 && pl - 1 < nout) {  // the next output (pl - 1, centre plane pl): its buffer index
+            const uint64_t cb = RB[sl][w + 1];
+            ic = oi + __popc((uint32_t)(cb >> 1) & lmask);
+        }
+        if (in && pl < nout) oi = __ldg(A.ri + ((int64_t)(zs + pl + 1) * A.ny + y) * A.rw + wx);
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+            aA[c] = aB[c];
+            aB[c] = aC[c];
+        }
+        if (pl >= 2) {  // plane pl-2 is read for the last time in this step
+            __syncwarp();
+            if (lane == 0) sfw_arrive(&empty[(pl - 2) % NB_SFW_NST]);
+        }
+    }
+}
+
 // The non-interior active nodes of the box operator (element set not full,
 // gz <= 1; ~2 % of a cube's nodes): one thread per node of the host-built
 // list {buffer index, gz, 27-neighbourhood mask, 9 row bases} (the gather
@@ -2204,8 +2355,19 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
                                          SfbCfg<3>::SMEM));
             if (g->device < 32) attr_set |= 1u << g->device;
         }
+        static unsigned ws_attr = 0;
+        const bool ws = (kind == 0 || kind == 2) && !(getenv("NB_SFB_WS") && atoi(getenv("NB_SFB_WS")) == 0);
+        if (ws && (g->device >= 32 || !(ws_attr & (1u << g->device)))) {
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_boxw<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, SFW_SMEM));
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_boxw<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, SFW_SMEM));
+            if (g->device < 32) ws_attr |= 1u << g->device;
+        }
         LaunchScope ls(g, g->cs, name);
-        if (kind == 2)
+        if (ws && kind == 2)
+            k_sp_fem_boxw<2><<<(unsigned)n, 256 + SFW_PT, SFW_SMEM, g->cs>>>(A);
+        else if (ws)
+            k_sp_fem_boxw<0><<<(unsigned)n, 256 + SFW_PT, SFW_SMEM, g->cs>>>(A);
+        else if (kind == 2)
             k_sp_fem_box<2><<<(unsigned)n, 256, SfbCfg<2>::SMEM, g->cs>>>(A);
         else if (kind == 3)
             k_sp_fem_box<3><<<(unsigned)n, 256, SfbCfg<3>::SMEM, g->cs>>>(A);
