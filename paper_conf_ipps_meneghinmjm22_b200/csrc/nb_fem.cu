@@ -2047,21 +2047,7 @@ __global__ void __launch_bounds__(256, NB_SFB_MINB) k_sp_fem_box(SpFemBoxArgs A)
     }
 }
 
-// Warp-specialised variant of k_sp_fem_box for kinds 0 / 2 (default;
-// NB_SFB_WS=0 selects the kernel above): two producer warps stage the planes
-// (table words, 8-byte cp.async, row bits) up to NB_SFW_NST planes ahead and
-// signal each slot through an mbarrier (cp.async.mbarrier.arrive.noinc + a
-// release arrive for the row bits); eight consumer warps run the same z-march
-// and epilogue and release a slot (one arrive per warp) after its last read.
-// No CTA-wide barrier in the plane loop: in the single-role kernel the plane
-// barrier and the uneven staging (1.33 cells per thread) held a quarter of
-// the stall samples.  Same arithmetic: same bits.
-#ifndef NB_SFW_NST
-#define NB_SFW_NST 8
-#endif
-#define SFW_PT 64  // producer threads
-#define SFW_SMEM (NB_SFW_NST * 3 * SFB_C * 8)
-
+// mbarrier arrivals of the warp-specialised box kernel below
 __device__ __forceinline__ void sfw_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -2069,54 +2055,147 @@ __device__ __forceinline__ void sfw_cp_arrive(uint64_t *bar) {
     asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
+// Warp-specialised, two-row variant of k_sp_fem_box for kinds 0 / 2
+// (default; NB_SFB_NR1=1 selects the kernel above).  Four producer warps
+// stage the planes (table words loaded one plane ahead, 8-byte cp.async,
+// row bits) up to NB_SF2_NST planes ahead and signal each slot through an
+// mbarrier (cp.async.mbarrier.arrive.noinc, plus a release arrive by the
+// row-bit writers); eight consumer warps run the z-march and release a slot
+// (one arrive per warp) after its last read — no CTA barrier in the plane
+// loop.  A consumer thread owns two rows of a 32 x 16 tile (box 34 x 18):
+// per plane it loads box rows ra-1 .. ra+2 of the three columns once (36
+// values for its 2 nodes instead of 54: the middle rows are kept in
+// registers from one row of positions to the next) and applies each
+// position's blocks in the same q order per node — the same bits.
+// Measured (round 2b, 384^3 full cube, CG iteration): 3.23 ms against 3.26
+// for the single-role kernel; a one-row warp-specialised version: 3.29.
+#ifndef NB_SF2_NST
+#define NB_SF2_NST 6
+#endif
+#define SF2_H 18
+#define SF2_C (SFB_W * SF2_H)
+#define SF2_PT 128
+#define SF2_SMEM (NB_SF2_NST * 3 * SF2_C * 8)
+
+template <int q>
+__device__ __forceinline__ void sf2_blk(double u0, double u1, double u2, double (&a)[3]) {
+    sp_fem_cfma<0, 0, q>(u0, a[0]);
+    sp_fem_cfma<0, 1, q>(u1, a[0]);
+    sp_fem_cfma<0, 2, q>(u2, a[0]);
+    sp_fem_cfma<1, 0, q>(u0, a[1]);
+    sp_fem_cfma<1, 1, q>(u1, a[1]);
+    sp_fem_cfma<1, 2, q>(u2, a[1]);
+    sp_fem_cfma<2, 0, q>(u0, a[2]);
+    sp_fem_cfma<2, 1, q>(u1, a[2]);
+    sp_fem_cfma<2, 2, q>(u2, a[2]);
+}
+// position Q of the plane for both rows: row 0 takes values v0, row 1 v1
+template <int Q>
+__device__ __forceinline__ void sf2_pos(const double (&v0)[3], const double (&v1)[3], double (&aA)[2][3],
+                                        double (&aB)[2][3], double (&aC)[2][3]) {
+    sf2_blk<18 + Q>(v0[0], v0[1], v0[2], aA[0]);
+    sf2_blk<9 + Q>(v0[0], v0[1], v0[2], aB[0]);
+    sf2_blk<Q>(v0[0], v0[1], v0[2], aC[0]);
+    sf2_blk<18 + Q>(v1[0], v1[1], v1[2], aA[1]);
+    sf2_blk<9 + Q>(v1[0], v1[1], v1[2], aB[1]);
+    sf2_blk<Q>(v1[0], v1[1], v1[2], aC[1]);
+}
+// P = the thread's column in box row ra - 1 (component 0) of the plane
+__device__ __forceinline__ void sf2_plane(const double *P, double (&aA)[2][3], double (&aB)[2][3],
+                                          double (&aC)[2][3]) {
+    double keep[3][3], v0[3], v1[3];
+#define SF2_LD(v, j, ox)                                    \
+    {                                                       \
+        const double *pp = P + (j) * SFB_W + (ox);          \
+        v[0] = pp[0], v[1] = pp[SF2_C], v[2] = pp[2 * SF2_C]; \
+    }
+    // oy = -1: rows ra-1 (node 0), ra (node 1, kept)
+    SF2_LD(v0, 0, -1) SF2_LD(v1, 1, -1) keep[0][0] = v1[0], keep[0][1] = v1[1], keep[0][2] = v1[2];
+    sf2_pos<0>(v0, v1, aA, aB, aC);
+    SF2_LD(v0, 0, 0) SF2_LD(v1, 1, 0) keep[1][0] = v1[0], keep[1][1] = v1[1], keep[1][2] = v1[2];
+    sf2_pos<1>(v0, v1, aA, aB, aC);
+    SF2_LD(v0, 0, 1) SF2_LD(v1, 1, 1) keep[2][0] = v1[0], keep[2][1] = v1[1], keep[2][2] = v1[2];
+    sf2_pos<2>(v0, v1, aA, aB, aC);
+    // oy = 0: rows ra (kept), ra+1 (node 1, kept next)
+#pragma unroll
+    for (int ox = 0; ox < 3; ++ox) {
+        SF2_LD(v1, 2, ox - 1)
+        v0[0] = keep[ox][0], v0[1] = keep[ox][1], v0[2] = keep[ox][2];
+        keep[ox][0] = v1[0], keep[ox][1] = v1[1], keep[ox][2] = v1[2];
+        if (ox == 0) sf2_pos<3>(v0, v1, aA, aB, aC);
+        if (ox == 1) sf2_pos<4>(v0, v1, aA, aB, aC);
+        if (ox == 2) sf2_pos<5>(v0, v1, aA, aB, aC);
+    }
+    // oy = +1: rows ra+1 (kept), ra+2
+#pragma unroll
+    for (int ox = 0; ox < 3; ++ox) {
+        SF2_LD(v1, 3, ox - 1)
+        v0[0] = keep[ox][0], v0[1] = keep[ox][1], v0[2] = keep[ox][2];
+        if (ox == 0) sf2_pos<6>(v0, v1, aA, aB, aC);
+        if (ox == 1) sf2_pos<7>(v0, v1, aA, aB, aC);
+        if (ox == 2) sf2_pos<8>(v0, v1, aA, aB, aC);
+    }
+#undef SF2_LD
+}
+
 template <int KIND>  // 0: y = K u; 2: y = b - K u
-__global__ void __launch_bounds__(256 + SFW_PT, 3) k_sp_fem_boxw(SpFemBoxArgs A) {
-    extern __shared__ __align__(16) double sfw_sm[];
-    double(*S)[3][SFB_C] = reinterpret_cast<double(*)[3][SFB_C]>(sfw_sm);
-    __shared__ uint64_t RB[NB_SFW_NST][SFB_H];
-    __shared__ __align__(8) uint64_t full[NB_SFW_NST], empty[NB_SFW_NST];
+__global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A) {
+    extern __shared__ __align__(16) double sf2_sm[];
+    double(*S)[3][SF2_C] = reinterpret_cast<double(*)[3][SF2_C]>(sf2_sm);
+    __shared__ uint64_t RB[NB_SF2_NST][SF2_H];
+    __shared__ __align__(8) uint64_t full[NB_SF2_NST], empty[NB_SF2_NST];
     if (A.sc && A.sc->status != 0) return;
     const int tid = threadIdx.x;
     const int4 it = A.items[blockIdx.x];
     const int bxi = it.x & 0x3fffffff;
-    const int x0 = bxi * 32, y0 = it.y * 8, zs = it.z, ze = it.w;
+    const int x0 = bxi * 32, y0 = it.y * 16, zs = it.z, ze = it.w;
     const int np = ze - zs + 2;
     const int nout = ze - zs;
     const int wx = bxi;
     if (tid == 0) {
-        for (int k = 0; k < NB_SFW_NST; ++k) {
-            mbar_init(&full[k], SFW_PT + SFB_H);  // producers' copies + the row-bit writers
-            mbar_init(&empty[k], 8);              // one arrive per consumer warp
+        for (int k = 0; k < NB_SF2_NST; ++k) {
+            mbar_init(&full[k], SF2_PT + SF2_H);
+            mbar_init(&empty[k], 8);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
     if (tid >= 256) {  // ---- producers ----
+        // a plane's table words are loaded one plane ahead (two register
+        // sets), so the copies of plane q issue while plane q+1's words fly
         const int pt = tid - 256;
-        constexpr int NC = (SFB_C + SFW_PT - 1) / SFW_PT;
-#pragma unroll 1
-        for (int q = 0; q < np; ++q) {
-            const int st = q % NB_SFW_NST;
-            if (q >= NB_SFW_NST) mbar_wait(&empty[st], (uint32_t)((q / NB_SFW_NST) - 1) & 1u);
+        constexpr int NC = (SF2_C + SF2_PT - 1) / SF2_PT;
+        const int ry = y0 - 1 + pt;
+        const bool rown = pt < SF2_H, rv = rown && ry >= 0 && ry < A.ny;
+        auto load_words = [&](int q, uint32_t (&tm)[NC + 3], int32_t (&ti)[NC]) {
             const int64_t row0 = (int64_t)(zs + q) * A.ny;  // slab row of (zl + 1, y = 0), zl = zs - 1 + q
-            uint32_t tm[NC];
-            int32_t ti[NC];
 #pragma unroll
             for (int k = 0; k < NC; ++k) {
-                const int e = pt + SFW_PT * k;
+                const int e = pt + SF2_PT * k;
                 const int x = x0 - 1 + e % SFB_W, yy = y0 - 1 + e / SFB_W;
                 tm[k] = 0u;
                 ti[k] = 0;
-                if (e < SFB_C && x >= 0 && x < A.nx && yy >= 0 && yy < A.ny) {
+                if (e < SF2_C && x >= 0 && x < A.nx && yy >= 0 && yy < A.ny) {
                     const int64_t kk = (row0 + yy) * A.rw + (x >> 5);
                     tm[k] = __ldg(A.rm + kk);
                     ti[k] = __ldg(A.ri + kk);
                 }
             }
+            tm[NC] = tm[NC + 1] = tm[NC + 2] = 0u;
+            if (rv) {  // the row bits' three words
+                const uint32_t *r = A.rm + (row0 + ry) * A.rw;
+                tm[NC] = wx > 0 ? __ldg(r + wx - 1) : 0u;
+                tm[NC + 1] = __ldg(r + wx);
+                tm[NC + 2] = wx + 1 < A.rw ? __ldg(r + wx + 1) : 0u;
+            }
+        };
+        auto issue_plane = [&](int q, const uint32_t (&tm)[NC + 3], const int32_t (&ti)[NC]) {
+            const int st = q % NB_SF2_NST;
+            if (q >= NB_SF2_NST) mbar_wait(&empty[st], (uint32_t)((q / NB_SF2_NST) - 1) & 1u);
 #pragma unroll
             for (int k = 0; k < NC; ++k) {
-                const int e = pt + SFW_PT * k;
-                if (e < SFB_C) {
+                const int e = pt + SF2_PT * k;
+                if (e < SF2_C) {
                     const unsigned b = (unsigned)(x0 - 1 + e % SFB_W) & 31u;
                     const bool act = (tm[k] >> b) & 1u;
                     const int64_t idx = act ? ti[k] + __popc(tm[k] & ((1u << b) - 1u)) : 0;
@@ -2124,76 +2203,90 @@ __global__ void __launch_bounds__(256 + SFW_PT, 3) k_sp_fem_boxw(SpFemBoxArgs A)
                     for (int c = 0; c < 3; ++c) sfb_cp8(&S[st][c][e], A.u + c * A.cs + idx, act);
                 }
             }
-            sfw_cp_arrive(&full[st]);  // fires when this thread's copies have landed
-            if (pt < SFB_H) {           // activity bits of box row pt: bit i = x0 - 1 + i
-                const int ry = y0 - 1 + pt;
-                uint64_t bits = 0ull;
-                if (ry >= 0 && ry < A.ny) {
-                    const uint32_t *r = A.rm + (row0 + ry) * A.rw;
-                    const uint32_t rl = wx > 0 ? __ldg(r + wx - 1) : 0u, rm = __ldg(r + wx);
-                    const uint32_t rh = wx + 1 < A.rw ? __ldg(r + wx + 1) : 0u;
-                    bits = (uint64_t)(rl >> 31) | ((uint64_t)rm << 1) | ((uint64_t)(rh & 1u) << 33);
-                }
-                RB[st][pt] = bits;
+            sfw_cp_arrive(&full[st]);
+            if (rown) {
+                RB[st][pt] = (uint64_t)(tm[NC] >> 31) | ((uint64_t)tm[NC + 1] << 1) |
+                             ((uint64_t)(tm[NC + 2] & 1u) << 33);
                 sfw_arrive(&full[st]);
             }
+        };
+        uint32_t tA[NC + 3], tB[NC + 3];
+        int32_t iA[NC], iB[NC];
+        load_words(0, tA, iA);
+#pragma unroll 1
+        for (int q = 0; q < np; q += 2) {
+            if (q + 1 < np) load_words(q + 1, tB, iB);
+            issue_plane(q, tA, iA);
+            if (q + 1 >= np) break;
+            if (q + 2 < np) load_words(q + 2, tA, iA);
+            issue_plane(q + 1, tB, iB);
         }
         asm volatile("cp.async.wait_all;" ::: "memory");
         return;
     }
-    // ---- consumers: k_sp_fem_box's z-march and epilogue ----
+    // ---- consumers: rows ra = y0 + 2w and ra + 1 ----
     const int lane = tid & 31, w = tid >> 5;
-    const int x = x0 + lane, y = y0 + w;
-    const bool in = x < A.nx && y < A.ny;
-    const int ce = (w + 1) * SFB_W + lane + 1;
+    const int x = x0 + lane, ya = y0 + 2 * w;
+    const bool xin = x < A.nx;
+    const int c0 = 2 * w * SFB_W + lane + 1;  // the thread's column in box row ra - 1
     const uint32_t lmask = (1u << lane) - 1u;
-    double aA[3] = {0.0, 0.0, 0.0}, aB[3] = {0.0, 0.0, 0.0};
-    int32_t oi = 0;
-    int64_t ic = 0;
+    double aA[2][3] = {}, aB[2][3] = {};
+    int32_t oi[2] = {0, 0};
+    int64_t ic[2] = {0, 0};
     mbar_wait(&full[0], 0u);
 #pragma unroll 1
     for (int pl = 0; pl < np; ++pl) {
-        const int sl = pl % NB_SFW_NST;
-        // plane pl+1 too: its row bits take part in the skip test below
-        if (pl + 1 < np) mbar_wait(&full[(pl + 1) % NB_SFW_NST], (uint32_t)((pl + 1) / NB_SFW_NST) & 1u);
-        double aC[3] = {0.0, 0.0, 0.0};
-        const uint64_t rows = (pl >= 1 ? RB[(pl + NB_SFW_NST - 1) % NB_SFW_NST][w + 1] : 0ull) | RB[sl][w + 1] |
-                              (pl + 1 < np ? RB[(pl + 1) % NB_SFW_NST][w + 1] : 0ull);
-        if ((rows >> 1) & 0xffffffffull) sfb_plane<0>(&S[sl][0][ce], aA, aB, aC);
+        const int sl = pl % NB_SF2_NST;
+        if (pl + 1 < np) mbar_wait(&full[(pl + 1) % NB_SF2_NST], (uint32_t)((pl + 1) / NB_SF2_NST) & 1u);
+        double aC[2][3] = {};
+        const int sm1 = (pl + NB_SF2_NST - 1) % NB_SF2_NST, sp1 = (pl + 1) % NB_SF2_NST;
+        const uint64_t rows = (pl >= 1 ? RB[sm1][2 * w + 1] | RB[sm1][2 * w + 2] : 0ull) | RB[sl][2 * w + 1] |
+                              RB[sl][2 * w + 2] | (pl + 1 < np ? RB[sp1][2 * w + 1] | RB[sp1][2 * w + 2] : 0ull);
+        if ((rows >> 1) & 0xffffffffull) sf2_plane(&S[sl][0][c0], aA, aB, aC);
         if (pl >= 2) {
             const int o = pl - 2, zl = zs + o;
-            const int s0 = (pl + NB_SFW_NST - 2) % NB_SFW_NST, s1 = (pl + NB_SFW_NST - 1) % NB_SFW_NST;
+            const int s0 = (pl + NB_SF2_NST - 2) % NB_SF2_NST, s1 = sm1;
             const int gz = A.gz0 + zl;
-            if (in && ((RB[s1][w + 1] >> (lane + 1)) & 1u)) {
-                bool full_nb = gz >= 2;
 #pragma unroll
-                for (int r = 0; r < 9; ++r) {
-                    const int oy = r % 3 - 1, oz = r / 3 - 1;
-                    const int st = oz < 0 ? s0 : (oz == 0 ? s1 : sl);
-                    full_nb = full_nb && ((RB[st][w + 1 + oy] >> lane) & 7u) == 7u;
-                }
-                if (full_nb) {
+            for (int r = 0; r < 2; ++r) {
+                const int br = 2 * w + r + 1;  // the node's box row
+                if (xin && ya + r < A.ny && ((RB[s1][br] >> (lane + 1)) & 1u)) {
+                    bool full_nb = gz >= 2;
 #pragma unroll
-                    for (int c = 0; c < 3; ++c) {
-                        const int64_t kk = c * A.cs + ic;
-                        A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], aA[c]) : aA[c];
+                    for (int k = 0; k < 9; ++k) {
+                        const int oy = k % 3 - 1, oz = k / 3 - 1;
+                        const int st = oz < 0 ? s0 : (oz == 0 ? s1 : sl);
+                        full_nb = full_nb && ((RB[st][br + oy] >> lane) & 7u) == 7u;
+                    }
+                    if (full_nb) {
+#pragma unroll
+                        for (int c = 0; c < 3; ++c) {
+                            const int64_t kk = c * A.cs + ic[r];
+                            A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], aA[r][c]) : aA[r][c];
+                        }
                     }
                 }
             }
         }
-        if (pl >= 1 && pl - 1 < nout) {  // the next output (pl - 1, centre plane pl): its buffer index
-            const uint64_t cb = RB[sl][w + 1];
-            ic = oi + __popc((uint32_t)(cb >> 1) & lmask);
-        }
-        if (in && pl < nout) oi = __ldg(A.ri + ((int64_t)(zs + pl + 1) * A.ny + y) * A.rw + wx);
+        if (pl >= 1 && pl - 1 < nout) {  // the next output's (centre plane pl) buffer indices
 #pragma unroll
-        for (int c = 0; c < 3; ++c) {
-            aA[c] = aB[c];
-            aB[c] = aC[c];
+            for (int r = 0; r < 2; ++r) ic[r] = oi[r] + __popc((uint32_t)(RB[sl][2 * w + r + 1] >> 1) & lmask);
         }
-        if (pl >= 2) {  // plane pl-2 is read for the last time in this step
+        if (xin && pl < nout) {
+#pragma unroll
+            for (int r = 0; r < 2; ++r)
+                if (ya + r < A.ny) oi[r] = __ldg(A.ri + ((int64_t)(zs + pl + 1) * A.ny + ya + r) * A.rw + wx);
+        }
+#pragma unroll
+        for (int r = 0; r < 2; ++r)
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                aA[r][c] = aB[r][c];
+                aB[r][c] = aC[r][c];
+            }
+        if (pl >= 2) {
             __syncwarp();
-            if (lane == 0) sfw_arrive(&empty[(pl - 2) % NB_SFW_NST]);
+            if (lane == 0) sfw_arrive(&empty[(pl - 2) % NB_SF2_NST]);
         }
     }
 }
@@ -2356,17 +2449,24 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
             if (g->device < 32) attr_set |= 1u << g->device;
         }
         static unsigned ws_attr = 0;
-        const bool ws = (kind == 0 || kind == 2) && !(getenv("NB_SFB_WS") && atoi(getenv("NB_SFB_WS")) == 0);
-        if (ws && (g->device >= 32 || !(ws_attr & (1u << g->device)))) {
-            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_boxw<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, SFW_SMEM));
-            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_boxw<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, SFW_SMEM));
+        const bool nr2 = (kind == 0 || kind == 2) && !getenv("NB_SFB_NR1");
+        const int4 *items2 = nullptr;
+        int64_t n2 = 0;
+        SpFemBoxArgs A2 = A;
+        if (nr2) {  // 32 x 16 tiles
+            NB_TRY(nb_sparse_fem_box_list(g, p, ranges, NB_SFB_ZC, &items2, &n2, false, 16));
+            A2.items = items2;
+        }
+        if (nr2 && (g->device >= 32 || !(ws_attr & (1u << g->device)))) {
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box2<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, SF2_SMEM));
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box2<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, SF2_SMEM));
             if (g->device < 32) ws_attr |= 1u << g->device;
         }
         LaunchScope ls(g, g->cs, name);
-        if (ws && kind == 2)
-            k_sp_fem_boxw<2><<<(unsigned)n, 256 + SFW_PT, SFW_SMEM, g->cs>>>(A);
-        else if (ws)
-            k_sp_fem_boxw<0><<<(unsigned)n, 256 + SFW_PT, SFW_SMEM, g->cs>>>(A);
+        if (nr2 && kind == 2)
+            k_sp_fem_box2<2><<<(unsigned)n2, 256 + SF2_PT, SF2_SMEM, g->cs>>>(A2);
+        else if (nr2)
+            k_sp_fem_box2<0><<<(unsigned)n2, 256 + SF2_PT, SF2_SMEM, g->cs>>>(A2);
         else if (kind == 2)
             k_sp_fem_box<2><<<(unsigned)n, 256, SfbCfg<2>::SMEM, g->cs>>>(A);
         else if (kind == 3)
@@ -2455,6 +2555,7 @@ nb_status nb_sparse_fem_box_prepare(nb_grid *g) {
             int64_t n;
             NB_TRY(nb_sparse_fem_box_list(g, p, sp_box_ranges(g, p, which), NB_SFB_ZC, &it, &n, false));
             NB_TRY(nb_sparse_fem_box_list(g, p, sp_box_ranges(g, p, which), NB_SFB_ZC, &it, &n, true));
+            NB_TRY(nb_sparse_fem_box_list(g, p, sp_box_ranges(g, p, which), NB_SFB_ZC, &it, &n, false, 16));
         }
     return nb_sparse_tile_tp(g);
 }

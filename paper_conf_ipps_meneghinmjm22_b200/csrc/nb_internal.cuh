@@ -483,7 +483,7 @@ nb_status nb_sparse_fem_pass(nb_grid *g, int p, int kind, const int32_t *list, c
 bool nb_sparse_fem_boxed();  // the box operator is the default (NB_SPF_GATHER=1: the gather pass)
 nb_status nb_sparse_fem_box_tables(nb_grid *g);
 nb_status nb_sparse_fem_box_list(nb_grid *g, int p, const std::vector<int> &ranges, int zc, const int4 **items,
-                                 int64_t *n, bool all = false);
+                                 int64_t *n, bool all = false, int th = 8);
 nb_status nb_sparse_tile_tp(nb_grid *g);
 // the grid's tile partial buffer (sp_tp, sp_T) in place of the segment
 // partials for the box kernels' dots and the finalize that reads them

@@ -1902,24 +1902,27 @@ nb_status nb_sparse_fem_box_tables(nb_grid *g) {
 // the local plane ranges holding an active node, chunk-major (neighbouring
 // tiles of a chunk run together and share their ring rows in L2); cached
 nb_status nb_sparse_fem_box_list(nb_grid *g, int p, const std::vector<int> &ranges, int zc, const int4 **items,
-                                 int64_t *n, bool all) {
+                                 int64_t *n, bool all, int th) {
     NB_TRY(nb_sparse_fem_box_tables(g));
     NbSparsePart &sp = g->sp[p];
     std::vector<int> key = ranges;
     key.push_back(zc);
     key.push_back(all ? 1 : 0);
+    key.push_back(th);
     auto it = sp.box_lists.find(key);
     if (it == sp.box_lists.end()) {
-        const int tx = (g->nx + 31) / 32, ty = (g->ny + 7) / 8;
+        // tile_any is per 32 x 8 tile; a 32 x th tile spans th / 8 of them
+        const int tx = (g->nx + 31) / 32, ty = (g->ny + 7) / 8, f = th / 8, tyh = (ty + f - 1) / f;
         std::vector<int4> v;
         for (size_t r = 0; r + 1 < ranges.size(); r += 2)
             for (int zs = ranges[r]; zs < ranges[r + 1]; zs += zc) {
                 const int ze = std::min(zs + zc, ranges[r + 1]);
-                for (int by = 0; by < ty; ++by)
+                for (int by = 0; by < tyh; ++by)
                     for (int bx = 0; bx < tx; ++bx) {
                         bool any = false;
                         for (int zl = zs; zl < ze && !any; ++zl)
-                            any = sp.tile_any[((size_t)zl * ty + by) * tx + bx] != 0;
+                            for (int k = 0; k < f && by * f + k < ty && !any; ++k)
+                                any = sp.tile_any[((size_t)zl * ty + by * f + k) * tx + bx] != 0;
                         // all: every tile (its dot partials are rewritten), empty ones flagged
                         if (any || all) v.push_back(make_int4(bx | (any ? 0 : 0x40000000), by, zs, ze));
                     }

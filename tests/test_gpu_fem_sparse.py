@@ -118,10 +118,11 @@ def test_sparse_fem_cg_converges():
 
 def _run_both(fn, modes=("NB_SPF_NONE", "NB_SPF_GATHER")):
     """fn() under each switch in `modes` set to 1 (NB_SPF_NONE: the default,
-    the shared-memory box operator after a separate map, <p, q> in a
-    separate segment-order pass; NB_SPF_TILEDOT: <p, q> in tile order inside
-    the box kernel; NB_SPF_GATHER: the gather pass; NB_SPF_FUSED: the box
-    operator's fused CG phase A)."""
+    the shared-memory box operator (warp-specialised, two rows per thread)
+    after a separate map, <p, q> in a separate segment-order pass;
+    NB_SFB_NR1: the single-role one-row box kernel; NB_SPF_TILEDOT: <p, q> in
+    tile order inside the box kernel; NB_SPF_GATHER: the gather pass;
+    NB_SPF_FUSED: the box operator's fused CG phase A)."""
     import os
     outs = []
     for m in modes:
@@ -157,8 +158,8 @@ def test_sparse_fem_box_equals_gather_bitwise(name, parts):
             fu.close(), fy.close()
         return y
 
-    ya, yb = _run_both(apply)
-    assert np.array_equal(ya, yb)
+    ya, yb, yc = _run_both(apply, ("NB_SPF_NONE", "NB_SPF_GATHER", "NB_SFB_NR1"))
+    assert np.array_equal(ya, yb) and np.array_equal(ya, yc)
     yo = oracle.fem_apply(u, 1.0, 0.3, mask=m)
     assert np.max(np.abs(ya - yo)) <= 1e-13 * max(np.max(np.abs(yo)), 1.0)
 
