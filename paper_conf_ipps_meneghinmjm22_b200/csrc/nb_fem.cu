@@ -2073,9 +2073,13 @@ __device__ __forceinline__ void sfw_cp_arrive(uint64_t *bar) {
 #define NB_SF2_NST 6
 #endif
 #define SF2_H 18
+#ifndef NB_SF2_SLEEP_NS
+#define NB_SF2_SLEEP_NS 256
+#endif
 #define SF2_C (SFB_W * SF2_H)
 #define SF2_PT 128
 #define SF2_SMEM (NB_SF2_NST * 3 * SF2_C * 8)
+#define SF2B_SMEM (NB_SF2_NST * 3 * 36 * SF2_H * 8)
 
 template <int q>
 __device__ __forceinline__ void sf2_blk(double u0, double u1, double u2, double (&a)[3]) {
@@ -2100,26 +2104,28 @@ __device__ __forceinline__ void sf2_pos(const double (&v0)[3], const double (&v1
     sf2_blk<9 + Q>(v1[0], v1[1], v1[2], aB[1]);
     sf2_blk<Q>(v1[0], v1[1], v1[2], aC[1]);
 }
-// P = the thread's column in box row ra - 1 (component 0) of the plane
-__device__ __forceinline__ void sf2_plane(const double *P, double (&aA)[2][3], double (&aB)[2][3],
-                                          double (&aC)[2][3]) {
+// R0 .. R3 = the thread's column (component 0) in box rows ra-1 .. ra+2 of
+// the plane; CS = the component stride of the slot
+template <int CS>
+__device__ __forceinline__ void sf2_plane(const double *R0, const double *R1, const double *R2, const double *R3,
+                                          double (&aA)[2][3], double (&aB)[2][3], double (&aC)[2][3]) {
     double keep[3][3], v0[3], v1[3];
-#define SF2_LD(v, j, ox)                                    \
-    {                                                       \
-        const double *pp = P + (j) * SFB_W + (ox);          \
-        v[0] = pp[0], v[1] = pp[SF2_C], v[2] = pp[2 * SF2_C]; \
+#define SF2_LD(v, R, ox)                                 \
+    {                                                    \
+        const double *pp = (R) + (ox);                   \
+        v[0] = pp[0], v[1] = pp[CS], v[2] = pp[2 * CS];  \
     }
     // oy = -1: rows ra-1 (node 0), ra (node 1, kept)
-    SF2_LD(v0, 0, -1) SF2_LD(v1, 1, -1) keep[0][0] = v1[0], keep[0][1] = v1[1], keep[0][2] = v1[2];
+    SF2_LD(v0, R0, -1) SF2_LD(v1, R1, -1) keep[0][0] = v1[0], keep[0][1] = v1[1], keep[0][2] = v1[2];
     sf2_pos<0>(v0, v1, aA, aB, aC);
-    SF2_LD(v0, 0, 0) SF2_LD(v1, 1, 0) keep[1][0] = v1[0], keep[1][1] = v1[1], keep[1][2] = v1[2];
+    SF2_LD(v0, R0, 0) SF2_LD(v1, R1, 0) keep[1][0] = v1[0], keep[1][1] = v1[1], keep[1][2] = v1[2];
     sf2_pos<1>(v0, v1, aA, aB, aC);
-    SF2_LD(v0, 0, 1) SF2_LD(v1, 1, 1) keep[2][0] = v1[0], keep[2][1] = v1[1], keep[2][2] = v1[2];
+    SF2_LD(v0, R0, 1) SF2_LD(v1, R1, 1) keep[2][0] = v1[0], keep[2][1] = v1[1], keep[2][2] = v1[2];
     sf2_pos<2>(v0, v1, aA, aB, aC);
     // oy = 0: rows ra (kept), ra+1 (node 1, kept next)
 #pragma unroll
     for (int ox = 0; ox < 3; ++ox) {
-        SF2_LD(v1, 2, ox - 1)
+        SF2_LD(v1, R2, ox - 1)
         v0[0] = keep[ox][0], v0[1] = keep[ox][1], v0[2] = keep[ox][2];
         keep[ox][0] = v1[0], keep[ox][1] = v1[1], keep[ox][2] = v1[2];
         if (ox == 0) sf2_pos<3>(v0, v1, aA, aB, aC);
@@ -2129,7 +2135,7 @@ __device__ __forceinline__ void sf2_plane(const double *P, double (&aA)[2][3], d
     // oy = +1: rows ra+1 (kept), ra+2
 #pragma unroll
     for (int ox = 0; ox < 3; ++ox) {
-        SF2_LD(v1, 3, ox - 1)
+        SF2_LD(v1, R3, ox - 1)
         v0[0] = keep[ox][0], v0[1] = keep[ox][1], v0[2] = keep[ox][2];
         if (ox == 0) sf2_pos<6>(v0, v1, aA, aB, aC);
         if (ox == 1) sf2_pos<7>(v0, v1, aA, aB, aC);
@@ -2138,10 +2144,45 @@ __device__ __forceinline__ void sf2_plane(const double *P, double (&aA)[2][3], d
 #undef SF2_LD
 }
 
-template <int KIND>  // 0: y = K u; 2: y = b - K u
+// producers wait for a free slot with a back-off: their spinning took issue
+// slots from the consumers (ncu: ~15 try_wait executions per node)
+__device__ __forceinline__ void sf2_wait_empty(uint64_t *bar, uint32_t parity) {
+    uint32_t done;
+    for (;;) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+        if (done) return;
+        __nanosleep(NB_SF2_SLEEP_NS);
+    }
+}
+
+// one bulk copy (TMA engine) of `bytes` global -> shared, completing on bar
+__device__ __forceinline__ void sf2_bulk(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+
+// BULK: box rows whose 34-cell window is fully active (a contiguous index
+// range) arrive as one bulk copy per component (cp.async.bulk, 272 or 288
+// bytes: an odd first index starts one cell earlier for 16-byte alignment,
+// the row's shift kept in bit 40 of its row bits) into 36-wide rows; the
+// other rows cell by cell as above.  Inactive box cells are not copied at
+// all (an interior node reads active cells only).
+template <int KIND, bool BULK>  // KIND 0: y = K u; 2: y = b - K u
 __global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A) {
+    constexpr int RS = BULK ? 36 : SFB_W;  // box row stride
+    constexpr int C = RS * SF2_H;          // component stride of a slot
     extern __shared__ __align__(16) double sf2_sm[];
-    double(*S)[3][SF2_C] = reinterpret_cast<double(*)[3][SF2_C]>(sf2_sm);
+    double(*S)[3][C] = reinterpret_cast<double(*)[3][C]>(sf2_sm);
     __shared__ uint64_t RB[NB_SF2_NST][SF2_H];
     __shared__ __align__(8) uint64_t full[NB_SF2_NST], empty[NB_SF2_NST];
     if (A.sc && A.sc->status != 0) return;
@@ -2154,13 +2195,78 @@ __global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A)
     const int wx = bxi;
     if (tid == 0) {
         for (int k = 0; k < NB_SF2_NST; ++k) {
-            mbar_init(&full[k], SF2_PT + SF2_H);
+            mbar_init(&full[k], SF2_PT + (BULK ? SF2_PT / 32 : SF2_H));
             mbar_init(&empty[k], 8);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
     if (tid >= 256) {  // ---- producers ----
+      if constexpr (BULK) {
+        // warp pw stages box rows pw, pw + 4, ... (<= 5): lane 6 r + k loads
+        // word k of row r's three rm and three ri words, one plane ahead,
+        // and the warp shares them by shuffles; then one bulk copy per
+        // component (lanes 0-2) if a row's window is fully active, else
+        // cell by cell
+        const int pw = (tid - 256) >> 5, pl_ = tid & 31;
+        constexpr int NRW = (SF2_H + SF2_PT / 32 - 1) / (SF2_PT / 32);  // rows per producer warp
+        auto load_w = [&](int q) -> uint32_t {
+            const int r = pl_ / 6, k = pl_ % 6, j = pw + (SF2_PT / 32) * r, yy = y0 - 1 + j;
+            const int wd = wx - 1 + k % 3;
+            uint32_t v = 0u;
+            if (r < NRW && j < SF2_H && yy >= 0 && yy < A.ny && wd >= 0 && wd < A.rw) {
+                const int64_t kk = ((int64_t)(zs + q) * A.ny + yy) * A.rw + wd;
+                v = k < 3 ? __ldg(A.rm + kk) : (uint32_t)__ldg(A.ri + kk);
+            }
+            return v;
+        };
+        uint32_t wcur = load_w(0);
+#pragma unroll 1
+        for (int q = 0; q < np; ++q) {
+            const int st = q % NB_SF2_NST;
+            const uint32_t wnext = q + 1 < np ? load_w(q + 1) : 0u;
+            if (q >= NB_SF2_NST) sf2_wait_empty(&empty[st], (uint32_t)((q / NB_SF2_NST) - 1) & 1u);
+#pragma unroll
+            for (int r = 0; r < NRW; ++r) {
+                const int j = pw + (SF2_PT / 32) * r;
+                const uint32_t m0 = __shfl_sync(0xffffffffu, wcur, 6 * r), m1 = __shfl_sync(0xffffffffu, wcur, 6 * r + 1),
+                               m2 = __shfl_sync(0xffffffffu, wcur, 6 * r + 2);
+                const int32_t i0 = (int32_t)__shfl_sync(0xffffffffu, wcur, 6 * r + 3),
+                              i1 = (int32_t)__shfl_sync(0xffffffffu, wcur, 6 * r + 4),
+                              i2 = (int32_t)__shfl_sync(0xffffffffu, wcur, 6 * r + 5);
+                if (j >= SF2_H) break;
+                const uint64_t bits = (uint64_t)(m0 >> 31) | ((uint64_t)m1 << 1) | ((uint64_t)(m2 & 1u) << 33);
+                uint64_t sh = 0;
+                if (bits == (1ull << 34) - 1ull) {
+                    const int64_t idx0 = i0 + __popc(m0 & 0x7fffffffu);  // cell x0 - 1
+                    sh = (uint64_t)(idx0 & 1);
+                    if (pl_ < 3)
+                        sf2_bulk(&S[st][pl_][j * RS], A.u + pl_ * A.cs + idx0 - (int64_t)sh, sh ? 288u : 272u,
+                                 &full[st]);
+                } else {
+#pragma unroll
+                    for (int h = 0; h < 2; ++h) {
+                        const int i = pl_ + 32 * h;  // window cell x0 - 1 + i
+                        if (i < SFB_W && ((bits >> i) & 1u)) {
+                            const uint32_t m = i == 0 ? m0 : (i == 33 ? m2 : m1);
+                            const int32_t ib = i == 0 ? i0 : (i == 33 ? i2 : i1);
+                            const unsigned b = i == 0 ? 31u : (i == 33 ? 0u : (unsigned)(i - 1));
+                            const int64_t idx = ib + __popc(m & ((1u << b) - 1u));
+#pragma unroll
+                            for (int c = 0; c < 3; ++c) sfb_cp8(&S[st][c][j * RS + i], A.u + c * A.cs + idx, true);
+                        }
+                    }
+                }
+                if (pl_ == 0) RB[st][j] = bits | (sh << 40);
+            }
+            wcur = wnext;
+            sfw_cp_arrive(&full[st]);  // this thread's cell copies (bulk copies count bytes)
+            __syncwarp();
+            if (pl_ == 0) sfw_arrive(&full[st]);  // after the warp's row bits
+        }
+        asm volatile("cp.async.wait_all;" ::: "memory");
+        return;
+      } else {
         // a plane's table words are loaded one plane ahead (two register
         // sets), so the copies of plane q issue while plane q+1's words fly
         const int pt = tid - 256;
@@ -2191,7 +2297,7 @@ __global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A)
         };
         auto issue_plane = [&](int q, const uint32_t (&tm)[NC + 3], const int32_t (&ti)[NC]) {
             const int st = q % NB_SF2_NST;
-            if (q >= NB_SF2_NST) mbar_wait(&empty[st], (uint32_t)((q / NB_SF2_NST) - 1) & 1u);
+            if (q >= NB_SF2_NST) sf2_wait_empty(&empty[st], (uint32_t)((q / NB_SF2_NST) - 1) & 1u);
 #pragma unroll
             for (int k = 0; k < NC; ++k) {
                 const int e = pt + SF2_PT * k;
@@ -2223,12 +2329,13 @@ __global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A)
         }
         asm volatile("cp.async.wait_all;" ::: "memory");
         return;
+      }
     }
     // ---- consumers: rows ra = y0 + 2w and ra + 1 ----
     const int lane = tid & 31, w = tid >> 5;
     const int x = x0 + lane, ya = y0 + 2 * w;
     const bool xin = x < A.nx;
-    const int c0 = 2 * w * SFB_W + lane + 1;  // the thread's column in box row ra - 1
+    const int c0 = 2 * w * RS + lane + 1;  // the thread's column in box row ra - 1
     const uint32_t lmask = (1u << lane) - 1u;
     double aA[2][3] = {}, aB[2][3] = {};
     int32_t oi[2] = {0, 0};
@@ -2242,7 +2349,17 @@ __global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A)
         const int sm1 = (pl + NB_SF2_NST - 1) % NB_SF2_NST, sp1 = (pl + 1) % NB_SF2_NST;
         const uint64_t rows = (pl >= 1 ? RB[sm1][2 * w + 1] | RB[sm1][2 * w + 2] : 0ull) | RB[sl][2 * w + 1] |
                               RB[sl][2 * w + 2] | (pl + 1 < np ? RB[sp1][2 * w + 1] | RB[sp1][2 * w + 2] : 0ull);
-        if ((rows >> 1) & 0xffffffffull) sf2_plane(&S[sl][0][c0], aA, aB, aC);
+        if ((rows >> 1) & 0xffffffffull) {
+            const double *P = &S[sl][0][c0];
+            if constexpr (BULK) {  // each row at its shift
+                const int b0 = 2 * w;
+                sf2_plane<C>(P + ((RB[sl][b0] >> 40) & 1), P + RS + ((RB[sl][b0 + 1] >> 40) & 1),
+                             P + 2 * RS + ((RB[sl][b0 + 2] >> 40) & 1), P + 3 * RS + ((RB[sl][b0 + 3] >> 40) & 1),
+                             aA, aB, aC);
+            } else {
+                sf2_plane<C>(P, P + RS, P + 2 * RS, P + 3 * RS, aA, aB, aC);
+            }
+        }
         if (pl >= 2) {
             const int o = pl - 2, zl = zs + o;
             const int s0 = (pl + NB_SF2_NST - 2) % NB_SF2_NST, s1 = sm1;
@@ -2450,6 +2567,7 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
         }
         static unsigned ws_attr = 0;
         const bool nr2 = (kind == 0 || kind == 2) && !getenv("NB_SFB_NR1");
+        const bool bulk = !getenv("NB_SFB_NOBULK");
         const int4 *items2 = nullptr;
         int64_t n2 = 0;
         SpFemBoxArgs A2 = A;
@@ -2458,15 +2576,21 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
             A2.items = items2;
         }
         if (nr2 && (g->device >= 32 || !(ws_attr & (1u << g->device)))) {
-            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box2<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, SF2_SMEM));
-            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box2<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, SF2_SMEM));
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box2<0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, SF2_SMEM));
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box2<2, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, SF2_SMEM));
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box2<0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, SF2B_SMEM));
+            NB_CUDA(cudaFuncSetAttribute(k_sp_fem_box2<2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, SF2B_SMEM));
             if (g->device < 32) ws_attr |= 1u << g->device;
         }
         LaunchScope ls(g, g->cs, name);
-        if (nr2 && kind == 2)
-            k_sp_fem_box2<2><<<(unsigned)n2, 256 + SF2_PT, SF2_SMEM, g->cs>>>(A2);
+        if (nr2 && bulk && kind == 2)
+            k_sp_fem_box2<2, true><<<(unsigned)n2, 256 + SF2_PT, SF2B_SMEM, g->cs>>>(A2);
+        else if (nr2 && bulk)
+            k_sp_fem_box2<0, true><<<(unsigned)n2, 256 + SF2_PT, SF2B_SMEM, g->cs>>>(A2);
+        else if (nr2 && kind == 2)
+            k_sp_fem_box2<2, false><<<(unsigned)n2, 256 + SF2_PT, SF2_SMEM, g->cs>>>(A2);
         else if (nr2)
-            k_sp_fem_box2<0><<<(unsigned)n2, 256 + SF2_PT, SF2_SMEM, g->cs>>>(A2);
+            k_sp_fem_box2<0, false><<<(unsigned)n2, 256 + SF2_PT, SF2_SMEM, g->cs>>>(A2);
         else if (kind == 2)
             k_sp_fem_box<2><<<(unsigned)n, 256, SfbCfg<2>::SMEM, g->cs>>>(A);
         else if (kind == 3)
