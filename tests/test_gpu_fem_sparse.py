@@ -181,3 +181,35 @@ def test_sparse_fem_box_equals_gather_bitwise(name, parts):
     (xd, rrd, idd), = _run_both(cg, ("NB_SPF_TILEDOT",))
     assert idd == ia and abs(rrd - rra) <= 1e-12 * rra
     assert np.max(np.abs(xd - xa)) <= 1e-12 * np.max(np.abs(xa))
+
+
+def test_sparse_fem_degenerate_masks():
+    """Degenerate element-sparse FEM domains through the box operator: lone
+    nodes (no element: K u = 0 off the Dirichlet plane, the identity on it),
+    a single element (8 active nodes), and a one-node-thick sheet (no
+    element anywhere) — against the masked oracle."""
+    n = 9
+    cases = {}
+    m = np.zeros((n, n, n), np.uint8)
+    m[4, 3, 5] = 1
+    m[0, 2, 2] = 1
+    cases["lone"] = m
+    m = np.zeros((n, n, n), np.uint8)
+    m[3:5, 4:6, 1:3] = 1
+    cases["one_element"] = m
+    m = np.zeros((n, n, n), np.uint8)
+    m[5, :, :] = 1
+    cases["sheet"] = m
+    for name, m in cases.items():
+        u = synth.uniform((n, n, n), card=3, seed=13) * m[None]
+        yo = oracle.fem_apply(u, 1.0, 0.3, mask=m)
+        with sgrid(m, 1) as g:
+            fu, fy = nb.Field(g, card=3), nb.Field(g, card=3)
+            fu.upload(u)
+            fu.halo_update()
+            nb.nb_fem27_apply(fu, fy)
+            y = fy.download()
+            fu.close(), fy.close()
+        assert np.max(np.abs(y - yo)) <= 1e-13 * max(np.max(np.abs(yo)), 1.0), name
+        if name == "lone":
+            assert np.all(y[:, 4, 3, 5] == 0.0) and np.array_equal(y[:, 0, 2, 2], u[:, 0, 2, 2])
