@@ -205,3 +205,34 @@ def test_f2_sparse_lbm_512_sphere_sampled_planes_vs_oracle():
         act = m[z].astype(bool)
         got = f1[:, z].astype(np.float64)
         assert np.max(np.abs(got[:, act] - exp[:, act]) / np.abs(exp[:, act])) <= 1e-5, z
+
+
+def test_f3_aa_pattern_512_equals_twopop_bitwise():
+    """The AA pattern at the bench size (512^3, one 10.2 GB buffer) against
+    twoPop (two buffers) after 4 steps of the lid-driven cavity from a
+    uniform flow: bit for bit on sampled planes (the lid plane, the walls,
+    the middle), and twoPop's planes against the oracle on a slab."""
+    n = 512
+    omega = oracle.lbm_omega(n)
+    planes = [0, 1, n // 2, n - 2, n - 1]
+    with nb.Grid((n, n, n)) as g:
+        a, b = nb.Field(g, "f32", 19), nb.Field(g, "f32", 19)
+        nb.nb_lbm_init(a, 1.0, (0.02, 0.01, 0.0))
+        a, b = nb.nb_lbm_step(a, b, omega, 3)
+        f3 = np.ascontiguousarray(a.download()[:, n // 2 - 1:n // 2 + 2])
+        a, b = nb.nb_lbm_step(a, b, omega, 1)
+        two = a.download()
+        a.close(), b.close()
+    with nb.Grid((n, n, n)) as g:
+        f = nb.Field(g, "f32", 19)
+        nb.nb_lbm_init(f, 1.0, (0.02, 0.01, 0.0))
+        nb.nb_lbm_step_aa(f, omega, 4)
+        aa = f.download()
+        f.close()
+    for z in planes:
+        assert np.array_equal(aa[:, z], two[:, z]), z
+    # the middle plane of step 4 from step 3's planes (interior slab: no z wall)
+    sub = oracle.lbm_step(f3, omega)
+    exp = sub[:, 1]
+    got = two[:, n // 2].astype(np.float64)
+    assert np.max(np.abs(got - exp) / np.abs(exp)) <= 1e-5
