@@ -236,3 +236,33 @@ def test_f3_aa_pattern_512_equals_twopop_bitwise():
     exp = sub[:, 1]
     got = two[:, n // 2].astype(np.float64)
     assert np.max(np.abs(got - exp) / np.abs(exp)) <= 1e-5
+
+
+def test_f4_karman_32768x8192_sampled_rows_vs_oracle():
+    """The largest PAPER.md Table I domain (32768 x 8192, 268M cells) in the
+    bench's configuration (D2Q9 channel, cylinder r = ny/10 at (nx/5, ny/2),
+    Re 150): after 4 + 1 steps from the uniform inflow, sampled rows (the
+    walls, through the cylinder, between) against the oracle's D2Q9 step on
+    the 3-row slab around each (the cylinder shifted into the slab)."""
+    nx, ny = 32768, 8192
+    u = 0.08
+    cyl = (nx // 5, ny // 2, ny // 10)
+    omega = 1.0 / (3 * u * 2 * cyl[2] / 150.0 + 0.5)
+    rows = [0, 1, cyl[1] - cyl[2] - 1, cyl[1], cyl[1] + cyl[2], ny - 2, ny - 1]
+    with nb.Grid((nx, ny, 1)) as g:
+        a, b = nb.Field(g, "f32", 9), nb.Field(g, "f32", 9)
+        nb.nb_d2q9_init(a, 1.0, u, 0.0)
+        a, b = nb.nb_d2q9_step(a, b, omega, u, cyl, 4)
+        f = a.download()[:, 0]
+        a, b = nb.nb_d2q9_step(a, b, omega, u, cyl, 1)
+        f1 = a.download()[:, 0]
+        a.close(), b.close()
+    assert np.max(np.abs(f1[:, cyl[1]] - f[:, cyl[1]])) > 1e-5  # the cylinder perturbs the flow
+    for y in rows:
+        y0, y1 = max(y - 1, 0), min(y + 2, ny)
+        sub = np.ascontiguousarray(f[:, y0:y1])
+        exp = oracle.d2q9_step(sub, omega, u, (cyl[0], cyl[1] - y0, cyl[2]))[:, y - y0]
+        got = f1[:, y].astype(np.float64)
+        nz = exp != 0
+        assert np.all(got[~nz] == 0), y
+        assert np.max(np.abs(got[nz] - exp[nz]) / np.abs(exp[nz])) <= 1e-5, y
