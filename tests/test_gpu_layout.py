@@ -191,3 +191,25 @@ def test_unsupported_layouts_are_reported():
         with pytest.raises(nb.NbError) as e:
             nb.Field(g, card=3, layout=nb.AOS)
         assert e.value.status == nb.NB_EUNSUPPORTED
+
+
+def test_lbm_layouts_512_bench_config_bitwise():
+    """The bench's layout lines at full size (512^3 cavity, 1 partition):
+    3 steps of the D3Q19 step from a uniform flow on SoA, plane-major SoA
+    and AoS populations give the same bits on sampled planes."""
+    n = 512
+    omega = oracle.lbm_omega(n)
+    planes = [0, 1, n // 2, n - 1]
+    outs = []
+    for layout in LAYOUTS:
+        with nb.Grid((n, n, n)) as g:
+            a, b = nb.Field(g, "f32", 19, layout=layout), nb.Field(g, "f32", 19, layout=layout)
+            nb.nb_lbm_init(a, 1.0, (0.02, 0.01, 0.0))
+            a, b = nb.nb_lbm_step(a, b, omega, 3)
+            f = a.download()
+            outs.append([np.ascontiguousarray(f[:, z]) for z in planes])
+            del f
+            a.close(), b.close()
+    for o in outs[1:]:
+        for x, y in zip(outs[0], o):
+            assert np.array_equal(x, y)

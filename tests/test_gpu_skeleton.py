@@ -222,3 +222,21 @@ def test_skeleton_lbm_bitwise_equals_lbm_step(parts, occ):
         assert ops.count("halo") == 2
         if occ != nb.OCC_NONE:
             assert [n["view"] for n in plan["nodes"] if n["op"] == "stencil"].count("internal") == 2
+
+
+def test_skeleton_listing3_cg_512_bench_config_bitwise():
+    """Listing 3 CG in the bench's skeleton configuration (512^3, 4
+    partitions, Two-way OCC): 2 iterations of the generated schedule equal
+    nb_cg_solve's bit for bit at full size."""
+    dims = (512, 512, 512)
+    bh = synth.uniform(dims, seed=3)
+    xs, rrs, _ = run_listing3(dims, 4, nb.OCC_TWO_WAY, 2, bh)
+    with nb.Grid(dims, nparts=4, devices=[0] * 4) as g:
+        b, x = nb.Field(g), nb.Field(g)
+        b.upload(bh)
+        x.fill_const(0.0)
+        res = nb.nb_cg_solve(x, b, max_iter=2, rtol=0.0, occ=nb.OCC_TWO_WAY)
+        xc = x.download()
+        b.close(), x.close()
+    assert res.iters == 2 and rrs == res.rr
+    assert np.array_equal(xs, xc)
