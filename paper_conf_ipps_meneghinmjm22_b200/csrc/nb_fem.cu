@@ -1776,6 +1776,7 @@ struct SpFemBoxArgs {
     const CgScal *sc;
     double *tp;            // KIND 1: <u, q> tile partials [3][NZ][T] (dense canonical order)
     int NZ, T, tx;
+    int64_t ncell;         // cells of a component's buffer (halo lo + own + halo hi): bulk-copy bound
 };
 
 __device__ __forceinline__ void sfb_cp8(double *dst, const double *src, bool on) {
@@ -2237,8 +2238,10 @@ __global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A)
                 if (j >= SF2_H) break;
                 const uint64_t bits = (uint64_t)(m0 >> 31) | ((uint64_t)m1 << 1) | ((uint64_t)(m2 & 1u) << 33);
                 uint64_t sh = 0;
-                if (bits == (1ull << 34) - 1ull) {
-                    const int64_t idx0 = i0 + __popc(m0 & 0x7fffffffu);  // cell x0 - 1
+                const int64_t idx0 = i0 + __popc(m0 & 0x7fffffffu);  // cell x0 - 1 (if active)
+                // a full window; an odd first index copies one cell more on
+                // each side, which must stay inside the component's cells
+                if (bits == (1ull << 34) - 1ull && (!(idx0 & 1) || idx0 + 34 < A.ncell)) {
                     sh = (uint64_t)(idx0 & 1);
                     if (pl_ < 3)
                         sf2_bulk(&S[st][pl_][j * RS], A.u + pl_ * A.cs + idx0 - (int64_t)sh, sh ? 288u : 272u,
@@ -2498,6 +2501,7 @@ nb_status nb_sparse_fem_box(nb_grid *g, int p, int kind, const std::vector<int> 
     A.y = y;
     A.sc = sc;
     A.cs = sp.cs;
+    A.ncell = sp.hl + sp.n + sp.hh;
     if (kind == 1) {  // <u, q> in tile order: the caller swaps sp_tp in for the finalize
         NB_TRY(nb_sparse_tile_tp(g));
         A.tp = g->sp_tp;
