@@ -548,6 +548,7 @@ extern "C" nb_status nb_grid_destroy(nb_grid *g) {
         nb_field_destroy(kv.second);
     }
     g->scratch.clear();
+    nb_field_cache_clear(g);
     if (g->c1_exec) cudaGraphExecDestroy(g->c1_exec);
     cudaFree(g->c1_tp);
     cudaFree(g->c1_psum);
@@ -685,6 +686,48 @@ extern "C" nb_status nb_field_layout(const nb_field *f, nb_layout *layout) {
     return NB_OK;
 }
 
+// ---- field buffer cache -----------------------------------------------------
+static bool field_cache_on(const nb_grid *g) {
+    // single process only: across processes the buffers are IPC-exported and
+    // mapped by the neighbours per field
+    return !nb_is_peer(g) && !(g->comm && g->comm->world > 1) && !getenv("NB_NO_FIELD_CACHE");
+}
+
+void nb_field_cache_clear(nb_grid *g) {
+    for (auto &kv : g->fcache) cudaFree(kv.second);
+    g->fcache.clear();
+}
+
+nb_status nb_field_buf_alloc(nb_grid *g, size_t bytes, void **out) {
+    *out = nullptr;
+    auto it = g->fcache.find(bytes);
+    if (it != g->fcache.end()) {
+        *out = it->second;
+        g->fcache.erase(it);
+        return NB_OK;
+    }
+    cudaError_t e = cudaMalloc(out, bytes);
+    if (e != cudaSuccess && !g->fcache.empty()) {  // give the cached buffers back and retry
+        cudaGetLastError();
+        nb_field_cache_clear(g);
+        e = cudaMalloc(out, bytes);
+    }
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        *out = nullptr;
+        NB_FAIL(NB_ENOMEM, "nb_field_create: cudaMalloc(%zu) failed: %s", bytes, cudaGetErrorString(e));
+    }
+    return NB_OK;
+}
+
+void nb_field_buf_release(nb_grid *g, void *buf, size_t bytes) {
+    if (!buf) return;
+    if (field_cache_on(g))
+        g->fcache.emplace(bytes, buf);
+    else
+        cudaFree(buf);
+}
+
 extern "C" nb_status nb_field_create(nb_grid *g, nb_dtype dt, int32_t card, nb_layout layout, double outside,
                                      nb_field **out) {
     if (!g || !out) NB_FAIL(NB_EINVAL, "nb_field_create: NULL argument");
@@ -715,13 +758,9 @@ extern "C" nb_status nb_field_create(nb_grid *g, nb_dtype dt, int32_t card, nb_l
             if (!g->parts[p].local) continue;
             f->cs = nb_cstride(f, p);
             size_t bytes = (size_t)f->plane * (g->parts[p].nz() + 2) * card * f->esz;
-            cudaError_t e = cudaMalloc(&f->base[p], bytes);
-            if (e != cudaSuccess) {
-                cudaGetLastError();
-                nb_set_error("nb_field_create: cudaMalloc(%zu) failed: %s", bytes, cudaGetErrorString(e));
-                s = NB_ENOMEM;
-                break;
-            }
+            s = nb_field_buf_alloc(g, bytes, (void **)&f->base[p]);
+            if (s != NB_OK) break;
+            cudaError_t e = cudaSuccess;
             f->bytes[p] = bytes;
             if (outside == 0.0)
                 e = cudaMemsetAsync(f->base[p], 0, bytes, g->cs);
@@ -852,7 +891,8 @@ extern "C" nb_status nb_field_destroy(nb_field *f) {
         if (f->base[p] && p < f->bytes.size()) nb_tma_forget_range(f->base[p], f->base[p] + f->bytes[p]);
     if (!f->borrowed)
         for (size_t p = 0; p < f->base.size(); ++p)
-            if (f->base[p] && !(p < f->mapped.size() && f->mapped[p])) cudaFree(f->base[p]);
+            if (f->base[p] && !(p < f->mapped.size() && f->mapped[p]))
+                nb_field_buf_release(f->g, f->base[p], p < f->bytes.size() ? f->bytes[p] : 0);
     f->g->nfields--;
     delete f;
     return NB_OK;

@@ -220,6 +220,12 @@ struct nb_grid {
     // C1 tile partials / plane sums of all iterations of one call (single
     // process: one finalize per call instead of one per iteration)
     double *c1_tp = nullptr, *c1_psum = nullptr;
+    // field buffer cache (single process): device buffers of destroyed
+    // fields, by exact size, handed to the next field of that size instead
+    // of a cudaFree / cudaMalloc pair (both synchronise and cost tens of ms
+    // at GB sizes: a solver's create / destroy inside a timed region);
+    // released on grid destroy or when a cudaMalloc fails
+    std::multimap<size_t, void *> fcache;
     // element-sparse grids: tile partials [nz][sp_T] of the 2-phase box CG
     // (32 x 8 tiles of the bounding box, the dense canonical dot order);
     // swapped into tp / T around its kernels and finalizes (lazy)
@@ -485,6 +491,10 @@ nb_status nb_sparse_fem_box_tables(nb_grid *g);
 nb_status nb_sparse_fem_box_list(nb_grid *g, int p, const std::vector<int> &ranges, int zc, const int4 **items,
                                  int64_t *n, bool all = false, int th = 8);
 nb_status nb_sparse_tile_tp(nb_grid *g);
+// field buffers through the grid's cache (nb_api.cu)
+nb_status nb_field_buf_alloc(nb_grid *g, size_t bytes, void **out);
+void nb_field_buf_release(nb_grid *g, void *buf, size_t bytes);
+void nb_field_cache_clear(nb_grid *g);
 // the grid's tile partial buffer (sp_tp, sp_T) in place of the segment
 // partials for the box kernels' dots and the finalize that reads them
 struct SpTpSwap {

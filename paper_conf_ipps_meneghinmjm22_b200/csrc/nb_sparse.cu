@@ -247,11 +247,7 @@ nb_status nb_sparse_field_alloc(nb_field *f) {
         const NbSparsePart &sp = g->sp[p];
         f->pcs[p] = sp.cs;
         size_t bytes = (size_t)sp.cs * f->card * f->esz;
-        cudaError_t e = cudaMalloc(&f->base[p], bytes);
-        if (e != cudaSuccess) {
-            cudaGetLastError();
-            NB_FAIL(NB_ENOMEM, "nb_field_create (sparse): cudaMalloc(%zu) failed", bytes);
-        }
+        NB_TRY(nb_field_buf_alloc(g, bytes, (void **)&f->base[p]));
         f->bytes[p] = bytes;
         if (f->outside == 0.0) {
             NB_CUDA(cudaMemsetAsync(f->base[p], 0, bytes, g->cs));
