@@ -222,6 +222,11 @@ nb_status nb_sync(nb_grid *grid);
 typedef enum { NB_SOA = 0, NB_SOA_PLANE = 1, NB_AOS = 2 } nb_layout;
 nb_status nb_field_create(nb_grid *grid, nb_dtype dtype, int32_t cardinality, nb_layout layout,
                           double outside_value, nb_field **out);
+/* Waits for the grid's streams.  In one process the field's device buffers
+ * go to the grid's cache and are handed to the next field of the same size
+ * (no cudaFree / cudaMalloc pair); the cache is freed by nb_grid_destroy and
+ * whenever a later allocation fails (NB_NO_FIELD_CACHE=1 frees at once).
+ * Borrowed buffers (nb_field_wrap) stay the caller's. */
 nb_status nb_field_destroy(nb_field *field);
 /* Borrowed storage (SURVEY.md §8(b) "field (borrowed)": PyTorch owns the
  * memory).  Pure host logic: the number of elements partition g of a field
