@@ -196,6 +196,10 @@ nb_status nb_grid_get_stream(const nb_grid *grid, void **compute_stream);
 nb_status nb_grid_set_halo_mode(nb_grid *grid, int32_t mode);
 /* synchronises: waits for all work of the grid, reports async errors */
 nb_status nb_sync(nb_grid *grid);
+/* Waits for the grid's streams and frees the field buffer cache (the device
+ * buffers of destroyed fields, see nb_field_destroy); *freed_bytes (may be
+ * NULL) receives their total size. */
+nb_status nb_grid_trim(nb_grid *grid, int64_t *freed_bytes);
 
 /* ---- fields (PAPER.md L58-L63 newField<T>(cardinality, outsideDomainValue),
  * L246 Field, L248 "SoA or AoS organizations without impacting the

@@ -97,6 +97,7 @@ SIGNATURES = {
     "nb_grid_set_streams": ([P, P, P], I32),
     "nb_grid_get_stream": ([P, PP], I32),
     "nb_sync": ([P], I32),
+    "nb_grid_trim": ([P, P], I32),
     "nb_grid_set_halo_mode": ([P, I32], I32),
     "nb_field_create": ([P, I32, I32, I32, D, PP], I32),
     "nb_field_layout": ([P, P], I32),
@@ -350,6 +351,12 @@ class Grid:
 
     def sync(self):
         _check(lib().nb_sync(self.handle))
+
+    def trim(self) -> int:
+        """Free the cached device buffers of destroyed fields; returns bytes."""
+        n = C.c_int64()
+        _check(lib().nb_grid_trim(self.handle, C.byref(n)))
+        return n.value
 
     def set_halo_mode(self, mode: int):
         """HALO_FUSED (stores from the boundary kernels) or HALO_STREAM

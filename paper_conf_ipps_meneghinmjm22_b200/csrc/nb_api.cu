@@ -637,6 +637,18 @@ extern "C" nb_status nb_sync(nb_grid *g) {
     return NB_OK;
 }
 
+extern "C" nb_status nb_grid_trim(nb_grid *g, int64_t *freed_bytes) {
+    if (!g) NB_FAIL(NB_EINVAL, "NULL grid");
+    DeviceGuard dg(g->device);
+    NB_CUDA(cudaStreamSynchronize(g->hs));
+    NB_CUDA(cudaStreamSynchronize(g->cs));
+    int64_t n = 0;
+    for (auto &kv : g->fcache) n += (int64_t)kv.first;
+    nb_field_cache_clear(g);
+    if (freed_bytes) *freed_bytes = n;
+    return NB_OK;
+}
+
 // ===========================================================================
 // fields (dense)
 // ===========================================================================
