@@ -2706,7 +2706,7 @@ extern "C" nb_status nb_fem27_apply(const nb_field *u, nb_field *y, double E, do
     NB_TRY(fem_upload_constants(E, nu));
     if (g->sparse) {
         const bool box = nb_sparse_fem_boxed();
-        NB_TRY(box ? nb_sparse_fem_box_prepare(g) : nb_sparse_fem_tables(g));
+        NB_TRY(box ? nb_sparse_fem_box_prepare(g) : nb_sparse_fem_tables(g, true));
         for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
             const NbSparsePart &sp = g->sp[p];
             if (box)
@@ -2765,8 +2765,8 @@ nb_status nb_fem_cg_init(nb_cg *cg) {
     nb_grid *g = cg->g;
     NB_TRY(fem_upload_constants(cg->prm.fem_E, cg->prm.fem_nu));
     if (g->sparse) {
-        NB_TRY(nb_sparse_fem_tables(g));
         const bool box = nb_sparse_fem_boxed();
+        NB_TRY(nb_sparse_fem_tables(g, !box));  // the gather pass needs the row bases
         if (box) NB_TRY(nb_sparse_fem_box_prepare(g));  // the q pass's lists, before any capture
         // fused phase A (p ping-pong) with NB_SPF_FUSED=1, decided once per
         // solver: same bits, but 2.70 ms against 1.24 + 1.00 ms for the box

@@ -476,7 +476,7 @@ nb_status nb_halo_run_mode(nb_field *f, bool periodic, int c0u, int c1u, int c0d
                            int mode);
 nb_status nb_sparse_halo_run(nb_field *f, int c0u, int c1u, int c0d, int c1d, cudaStream_t s, int mode);
 // element-sparse FEM (nb_sparse.cu tables, nb_fem.cu operator)
-nb_status nb_sparse_fem_tables(nb_grid *g);
+nb_status nb_sparse_fem_tables(nb_grid *g, bool with_bases);  // fm; fb (gather pass) if with_bases
 // one pass of the sparse FEM operator over segment list entries [s0, s0+n) of
 // `list` (gidx: their global segment indices, NULL = s0 + q) of partition p.
 // kind: 0 = y = K u, 1 = q = K u with <u, q>, 2 = y = b - K u with <y, y>

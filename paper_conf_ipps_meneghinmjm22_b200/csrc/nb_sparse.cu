@@ -1723,19 +1723,21 @@ __global__ void k_sp_fem_tab(const uint8_t *__restrict__ mask, const int32_t *__
                 if (base < 0) base = map[row + xx];
             }
         }
-        fb[(int64_t)r * n + j] = base;
+        if (fb) fb[(int64_t)r * n + j] = base;
     }
     fm[j] = m;
 }
 
-nb_status nb_sparse_fem_tables(nb_grid *g) {
+nb_status nb_sparse_fem_tables(nb_grid *g, bool with_bases) {
     if (!g->sparse) return NB_OK;
     DeviceGuard dg(g->device);
     const int nx = g->nx, ny = g->ny;
     const int64_t plane = (int64_t)nx * ny;
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         NbSparsePart &sp = g->sp[p];
-        if (sp.d_fm) continue;
+        if (sp.d_fm && (sp.d_fb || !with_bases)) continue;
+        cudaFree(sp.d_fm);  // rebuilt with the row bases
+        sp.d_fm = nullptr;
         const NbPart &q = g->parts[p];
         const int slab_z0 = q.z0 - (q.lo >= 0 ? 1 : 0), slab_z1 = q.z1 + (q.hi >= 0 ? 1 : 0);
         const int nslab = slab_z1 - slab_z0;
@@ -1745,7 +1747,8 @@ nb_status nb_sparse_fem_tables(nb_grid *g) {
         void *tmp = nullptr;
         size_t tmp_bytes = 0;
         NB_CUDA(cudaMalloc(&sp.d_fm, sizeof(uint32_t) * std::max<int64_t>(sp.n, 1)));
-        NB_CUDA(cudaMalloc(&sp.d_fb, sizeof(int32_t) * 9 * std::max<int64_t>(sp.n, 1)));
+        // the 9 row bases (36 B / node) only for the gather pass
+        if (with_bases) NB_CUDA(cudaMalloc(&sp.d_fb, sizeof(int32_t) * 9 * std::max<int64_t>(sp.n, 1)));
         NB_CUDA(cudaMalloc(&d_mask, ncell));
         NB_CUDA(cudaMalloc(&d_map, ncell * 4));
         NB_CUDA(cudaMemcpyAsync(d_mask, g->host_mask.data() + (int64_t)slab_z0 * plane, ncell, cudaMemcpyHostToDevice,
@@ -1988,7 +1991,7 @@ __global__ void k_sp_fem_rhs(const int32_t *__restrict__ seg, int64_t nseg, cons
 
 nb_status nb_sparse_fem_rhs(nb_field *b, double pr) {
     nb_grid *g = b->g;
-    NB_TRY(nb_sparse_fem_tables(g));
+    NB_TRY(nb_sparse_fem_tables(g, false));  // the masks only
     for (int p = g->first_local; p < g->first_local + g->nlocal; ++p) {
         const NbSparsePart &sp = g->sp[p];
         const int64_t nseg = sp.seg_start.back();
