@@ -2343,6 +2343,7 @@ __global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A)
     double aA[2][3] = {}, aB[2][3] = {};
     int32_t oi[2] = {0, 0};
     int64_t ic[2] = {0, 0};
+    double bo[2][3] = {};  // KIND 2: b of the output completed next step
     mbar_wait(&full[0], 0u);
 #pragma unroll 1
     for (int pl = 0; pl < np; ++pl) {
@@ -2382,7 +2383,7 @@ __global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A)
 #pragma unroll
                         for (int c = 0; c < 3; ++c) {
                             const int64_t kk = c * A.cs + ic[r];
-                            A.y[kk] = KIND == 2 ? __dsub_rn(A.b[kk], aA[r][c]) : aA[r][c];
+                            A.y[kk] = KIND == 2 ? __dsub_rn(bo[r][c], aA[r][c]) : aA[r][c];
                         }
                     }
                 }
@@ -2391,6 +2392,13 @@ __global__ void __launch_bounds__(256 + SF2_PT, 2) k_sp_fem_box2(SpFemBoxArgs A)
         if (pl >= 1 && pl - 1 < nout) {  // the next output's (centre plane pl) buffer indices
 #pragma unroll
             for (int r = 0; r < 2; ++r) ic[r] = oi[r] + __popc((uint32_t)(RB[sl][2 * w + r + 1] >> 1) & lmask);
+            if constexpr (KIND == 2) {  // b of the next output, a step ahead (set-up only)
+#pragma unroll
+                for (int r = 0; r < 2; ++r)
+                    if (xin && ya + r < A.ny && ((RB[sl][2 * w + r + 1] >> (lane + 1)) & 1u))
+#pragma unroll
+                        for (int c = 0; c < 3; ++c) bo[r][c] = __ldg(A.b + c * A.cs + ic[r]);
+            }
         }
         if (xin && pl < nout) {
 #pragma unroll
